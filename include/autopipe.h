@@ -1,0 +1,151 @@
+/*
+ * autopipe.h — C-ABI of the B200-native AutoPipe partition cost-model engine.
+ *
+ * The operation is the pipeline cost model of AutoPipe (Hu, Liu, Wang, Wang; ICPP '24) that scores
+ * worker partitions: for a per-layer profile (Table 1 rows L, O, G, P) and a
+ * cluster state (Table 1 rows N, B, FP, BP) it returns, in integer nanoseconds,
+ * the exact steady-state time per mini-batch of a PipeDream-style 1F1B pipeline (PAPER.md:253-278,
+ * Fig. 2 at 463-475): per-stage compute, p2p activations and input gradients at each boundary
+ * (PAPER.md:489-494), ring all-reduce of replicated stages and the
+ * pipeline-fill recurrence (Observation 3). SPEC.md fixes every rounding rule;
+ * results are bit-exact against the CPU oracle in oracle/.
+ *
+ * Conventions (all functions):
+ *  - return AUTOPIPE_OK (0) on success or a negative AUTOPIPE_E_* code; autopipe_last_error(ctx)
+ *    then returns a static, NUL-terminated description (valid until the next call on ctx);
+ *  - "host pointer" = ordinary CPU memory, read during the call and never retained;
+ *    "device pointer" = memory of ctx's CUDA device (e.g. a torch tensor's data_ptr()), which must
+ *    stay valid until the work enqueued on `stream` has completed;
+ *  - `stream` is a cudaStream_t passed as void* (NULL = the legacy default stream);
+ *  - a context is bound to one CUDA device and is not thread-safe; use one per thread/device;
+ *  - there is no CPU fallback: every score is computed by the sm_100a kernels of this library.
+ */
+#ifndef AUTOPIPE_H_
+#define AUTOPIPE_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum {
+  AUTOPIPE_OK = 0,
+  AUTOPIPE_E_INVAL = -1,    /* bad argument (range, NULL pointer, invalid current partition) */
+  AUTOPIPE_E_STATE = -2,    /* called in the wrong order (no profile, or no state since the profile) */
+  AUTOPIPE_E_OVERFLOW = -3, /* inputs whose exact integer arithmetic would not fit (SPEC.md §7) */
+  AUTOPIPE_E_CUDA = -4,     /* a CUDA runtime error (message carries cudaGetErrorString) */
+  AUTOPIPE_E_NOMEM = -5     /* device or host allocation failed */
+};
+
+/* search flags */
+#define AUTOPIPE_USE_ALL_WORKERS 1u /* only partitions with sum r_s = N (reading C-12); default sum r_s <= N */
+
+#define AUTOPIPE_IDLE 0xFFu
+#define AUTOPIPE_MAX_STAGES 8
+#define AUTOPIPE_MAX_WORKERS 8
+#define AUTOPIPE_MAX_LAYERS 255
+
+typedef struct autopipe_ctx autopipe_ctx; /* opaque */
+
+/* One worker partition ("an array of size N, each element the layers assigned to
+ * that worker"), exactly 16 bytes so a kernel reads it with one 128-bit load. */
+typedef struct {
+  uint8_t n_stages;           /* S in [1, min(8, N)] */
+  uint8_t last_layer[7];      /* e_0 < ... < e_{S-2} < L-1 (stage s = layers [e_{s-1}+1, e_s]);
+                                 e_{S-1} = L-1 is implied; entries >= S-1 are ignored (write 0xFF) */
+  uint8_t stage_of_worker[8]; /* per worker w: its stage in [0, S), or 0xFF when idle; w >= N must be 0xFF */
+} autopipe_partition;
+
+/* Result of a search: the lexicographic minimum of (time_ns, index) over the scanned shard. */
+typedef struct {
+  uint64_t time_ns;         /* T_ns of the best candidate (UINT64_MAX if the shard was empty) */
+  uint64_t index;           /* its global index (SPEC.md §5) (UINT64_MAX if empty) */
+  uint64_t evaluated;       /* number of candidates whose score was decided (= shard size) */
+  autopipe_partition part;  /* the best candidate, decoded */
+} autopipe_result;
+
+/* Create a context on CUDA device `cuda_device` (the caller's current device is left unchanged
+ * on return). Returns E_INVAL for a NULL `out`, E_CUDA if the device cannot be used. */
+int autopipe_create(int cuda_device, autopipe_ctx **out);
+
+/* Release every device and host resource of ctx (NULL is a no-op). Synchronises ctx's device. */
+void autopipe_destroy(autopipe_ctx *ctx);
+
+/* Description of the last error on ctx ("" if none). NULL ctx -> description of the last
+ * autopipe_create failure. */
+const char *autopipe_last_error(const autopipe_ctx *ctx);
+
+/* Static metrics (Table 1 rows L, O_i, G_i, P_i, measured once before training,
+ * PAPER.md:819-822). Host pointers, L entries each, copied (the caller keeps ownership):
+ *   act_bytes[l]    O[l]  bytes of layer l's output activation (sent forward at a cut after l);
+ *   grad_bytes[l]   G[l]  bytes of the gradient w.r.t. layer l's input (sent backward at a cut
+ *                         before l; reading C-6);
+ *   weight_bytes[l] P[l]  bytes of layer l's weights (all-reduced when its stage is replicated).
+ * L in [1, 255]; any byte count >= 2^56 -> E_OVERFLOW. Invalidates the state: autopipe_set_state
+ * must be called before any scoring call (else E_STATE). Synchronous. */
+int autopipe_load_profile(autopipe_ctx *ctx, uint32_t L, const uint64_t *act_bytes,
+                          const uint64_t *grad_bytes, const uint64_t *weight_bytes);
+
+/* Dynamic metrics (Table 1 rows N, B_i, FP_ij, BP_ij, refreshed every iteration,
+ * PAPER.md:823-833). Host pointers, copied:
+ *   fp_ns, bp_ns      N x L row-major: forward / backward nanoseconds of layer l on worker w;
+ *   link_fs_per_byte  N x N row-major: inverse bandwidth of the directed link u -> v in
+ *                     femtoseconds per byte (the per-link form of B_i, reading C-5; the diagonal
+ *                     is ignored; 0 = free link).
+ * N in [1, 8]. Rejects (E_OVERFLOW) states whose products bytes*tau reach 2^64 or whose largest
+ * modelled sum reaches 2^59 (SPEC.md §7); picks the 32-bit search path when every r=1 sum fits.
+ * Enqueues the prefix-sum and link-table kernels on `stream` (returns before they finish).
+ * Requires a loaded profile (E_STATE). */
+int autopipe_set_state(autopipe_ctx *ctx, uint32_t N, const uint64_t *fp_ns, const uint64_t *bp_ns,
+                       const uint64_t *link_fs_per_byte, void *stream);
+
+/* Batched scoring of explicit partitions (device pointers; async on `stream`):
+ *   d_parts[count]    input records (any disjoint worker sets, reading C-11);
+ *   d_time_ns[count]  output T_ns per record; an invalid record (SPEC.md §2) gets UINT64_MAX and
+ *                     never fails the batch.
+ * count = 0 is a no-op. Requires a state (E_STATE). */
+int autopipe_eval_partitions(autopipe_ctx *ctx, const autopipe_partition *d_parts, uint64_t count,
+                             uint64_t *d_time_ns, void *stream);
+
+/* Exhaustive search (PAPER.md:896-899 enumerates candidates and scores each with the speed model;
+ * here every candidate is scored exactly). Candidates: S in [s_min, s_max] (1 <= s_min <= s_max <=
+ * min(8, N)), contiguous worker placement (stage s gets workers [R_{s-1}, R_s)), every cut set;
+ * flags: AUTOPIPE_USE_ALL_WORKERS or 0. Scans the global indices [begin, end) of SPEC.md §5
+ * (end = UINT64_MAX means "to the end"; end is clamped to the space size), so a space can be split
+ * across GPUs or resumed. Writes the shard's lexicographic (time_ns, index) minimum to the host
+ * struct *h_out. Synchronous (waits for `stream`). */
+int autopipe_search_optimum(autopipe_ctx *ctx, uint32_t s_min, uint32_t s_max, uint32_t flags,
+                            uint64_t begin, uint64_t end, autopipe_result *h_out, void *stream);
+
+/* RL rollout rewards (the arbiter sees the current and the new partition; the
+ * reward is one-iteration speed with a switching cost). Device pointers, async on `stream`:
+ *   d_parts[count]         proposals; d_time_ns[count] gets T_ns (UINT64_MAX if invalid);
+ *   h_current              HOST pointer to the current partition, or NULL;
+ *   d_switch_bytes[count]  if h_current != NULL: sum over layers l of P[l] * |W_new(l) \ W_old(l)|
+ *                          (SPEC.md §6; UINT64_MAX for an invalid proposal); must be NULL when
+ *                          h_current is NULL.
+ * An invalid *h_current -> E_INVAL. */
+int autopipe_rollout_rewards(autopipe_ctx *ctx, const autopipe_partition *d_parts, uint64_t count,
+                             const autopipe_partition *h_current, uint64_t *d_time_ns,
+                             uint64_t *d_switch_bytes, void *stream);
+
+/* Number of candidates of a search space (requires a state for L and N). */
+int autopipe_count_candidates(const autopipe_ctx *ctx, uint32_t s_min, uint32_t s_max, uint32_t flags,
+                              uint64_t *total);
+
+/* Decode a global index of a search space into its partition record (host utility). */
+int autopipe_decode_index(const autopipe_ctx *ctx, uint32_t s_min, uint32_t s_max, uint32_t flags,
+                          uint64_t index, autopipe_partition *out);
+
+/* Which integer path the last set_state selected: 32 or 64 (0 if no state). */
+int autopipe_int_path(const autopipe_ctx *ctx);
+
+/* Number of kernels this context has launched so far (for launch accounting in benchmarks). */
+uint64_t autopipe_kernel_launches(const autopipe_ctx *ctx);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* AUTOPIPE_H_ */

@@ -1,0 +1,81 @@
+"""ctypes binding of the C-ABI in include/autopipe.h (argument marshalling only).
+
+The shared library ``libautopipe.so`` is built in-tree by ``__graft_entry__.build()`` (nvcc,
+sm_100a). There is no fallback: if the library is missing this module raises on import.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libautopipe.so")
+
+AUTOPIPE_OK = 0
+AUTOPIPE_E_INVAL = -1
+AUTOPIPE_E_STATE = -2
+AUTOPIPE_E_OVERFLOW = -3
+AUTOPIPE_E_CUDA = -4
+AUTOPIPE_E_NOMEM = -5
+USE_ALL_WORKERS = 1
+
+ERROR_NAMES = {AUTOPIPE_E_INVAL: "AUTOPIPE_E_INVAL", AUTOPIPE_E_STATE: "AUTOPIPE_E_STATE",
+               AUTOPIPE_E_OVERFLOW: "AUTOPIPE_E_OVERFLOW", AUTOPIPE_E_CUDA: "AUTOPIPE_E_CUDA",
+               AUTOPIPE_E_NOMEM: "AUTOPIPE_E_NOMEM"}
+
+# every symbol include/autopipe.h declares
+SYMBOLS = ["autopipe_create", "autopipe_destroy", "autopipe_last_error", "autopipe_load_profile",
+           "autopipe_set_state", "autopipe_eval_partitions", "autopipe_search_optimum",
+           "autopipe_rollout_rewards", "autopipe_count_candidates", "autopipe_decode_index",
+           "autopipe_int_path", "autopipe_kernel_launches"]
+
+
+class Partition(ctypes.Structure):
+    _fields_ = [("n_stages", ctypes.c_uint8), ("last_layer", ctypes.c_uint8 * 7),
+                ("stage_of_worker", ctypes.c_uint8 * 8)]
+
+
+class Result(ctypes.Structure):
+    _fields_ = [("time_ns", ctypes.c_uint64), ("index", ctypes.c_uint64),
+                ("evaluated", ctypes.c_uint64), ("part", Partition)]
+
+
+assert ctypes.sizeof(Partition) == 16 and ctypes.sizeof(Result) == 40
+
+
+class AutopipeError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__("%s: %s" % (ERROR_NAMES.get(code, str(code)), msg))
+        self.code = code
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError("libautopipe.so not built (run __graft_entry__.build()); there is no CPU "
+                          "fallback for the cost-model kernels")
+    lib = ctypes.CDLL(LIB_PATH)
+    P = ctypes.c_void_p
+    u32, u64, i32 = ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int
+    pu64 = ctypes.POINTER(ctypes.c_uint64)
+    sig = {
+        "autopipe_create": (i32, [i32, ctypes.POINTER(P)]),
+        "autopipe_destroy": (None, [P]),
+        "autopipe_last_error": (ctypes.c_char_p, [P]),
+        "autopipe_load_profile": (i32, [P, u32, pu64, pu64, pu64]),
+        "autopipe_set_state": (i32, [P, u32, pu64, pu64, pu64, P]),
+        "autopipe_eval_partitions": (i32, [P, P, u64, P, P]),
+        "autopipe_search_optimum": (i32, [P, u32, u32, u32, u64, u64, ctypes.POINTER(Result), P]),
+        "autopipe_rollout_rewards": (i32, [P, P, u64, ctypes.POINTER(Partition), P, P, P]),
+        "autopipe_count_candidates": (i32, [P, u32, u32, u32, pu64]),
+        "autopipe_decode_index": (i32, [P, u32, u32, u32, u64, ctypes.POINTER(Partition)]),
+        "autopipe_int_path": (i32, [P]),
+        "autopipe_kernel_launches": (u64, [P]),
+    }
+    for name, (res, args) in sig.items():
+        fn = getattr(lib, name)
+        fn.restype = res
+        fn.argtypes = args
+    return lib
+
+
+lib = _load()

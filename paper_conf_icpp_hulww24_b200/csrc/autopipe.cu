@@ -1,0 +1,467 @@
+// autopipe.cu — host side of the C-ABI (include/autopipe.h): argument validation, the overflow
+// rules of SPEC.md §7, the integer-path choice, device buffers, shard/index arithmetic of the search
+// space (SPEC.md §5) and kernel launches. No score is ever computed here: every T_ns comes from the
+// sm_100a kernels in k_state.cu / k_eval.cu / k_search.cu / k_search_r1.cu.
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+
+#include "../../include/autopipe.h"
+#include "internal.h"
+
+using namespace ap;
+
+typedef unsigned __int128 u128;
+
+static const u64 LIMIT_BYTES = 1ull << 56;   // any single byte count (and sum P)
+static const u64 LIMIT_TIME = 1ull << 59;    // the largest modelled sum (SPEC.md §7)
+static const u64 LIMIT_TIME32 = 0xFFFFFFF0u; // 32-bit search path
+static const int MAX_BLOCKS = 148 * 32;
+
+struct autopipe_ctx {
+  int device = 0, sms = 148;
+  char err[512] = {0};
+  bool has_profile = false, has_state = false;
+  u32 L = 0, N = 0;
+  int path32 = 0;
+  u64 launches = 0;
+  u64 maxOG = 0, sumP = 0;
+  DevTables tab{};
+  // device buffers
+  u64 *d_raw = nullptr;      // fp [8*255] | bp [8*255] | P [255]
+  u64 *d_tables = nullptr;   // all DevTables arrays
+  BlockOut *d_blocks = nullptr;
+  ResultDev *d_result = nullptr;
+  void *d_work = nullptr;
+  size_t work_bytes = 0;
+  // pinned host staging
+  u64 *h_stage = nullptr;    // fp | bp | tau(64)
+  ResultDev *h_result = nullptr;
+  u64 binom[BINOM_N][BINOM_K];
+};
+
+static char g_create_err[256] = "";
+
+static int fail(autopipe_ctx *c, int code, const char *fmt, ...) {
+  va_list ap_;
+  va_start(ap_, fmt);
+  vsnprintf(c->err, sizeof(c->err), fmt, ap_);
+  va_end(ap_);
+  return code;
+}
+
+static int cuda_fail(autopipe_ctx *c, cudaError_t e, const char *what) {
+  return fail(c, AUTOPIPE_E_CUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+// RAII device switch: the caller's current device is restored on return.
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    cudaGetDevice(&prev);
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+static void host_binomials(u64 (*b)[BINOM_K]) {
+  for (int n = 0; n < BINOM_N; ++n)
+    for (int k = 0; k < BINOM_K; ++k) {
+      if (k == 0) b[n][k] = 1;
+      else if (n == 0) b[n][k] = 0;
+      else b[n][k] = b[n - 1][k - 1] + b[n - 1][k];
+    }
+}
+
+extern "C" int autopipe_create(int cuda_device, autopipe_ctx **out) {
+  if (!out) {
+    snprintf(g_create_err, sizeof(g_create_err), "out is NULL");
+    return AUTOPIPE_E_INVAL;
+  }
+  *out = nullptr;
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess || cuda_device < 0 || cuda_device >= ndev) {
+    snprintf(g_create_err, sizeof(g_create_err), "no CUDA device %d (%s)", cuda_device,
+             e != cudaSuccess ? cudaGetErrorString(e) : "out of range");
+    return AUTOPIPE_E_CUDA;
+  }
+  autopipe_ctx *c = new (std::nothrow) autopipe_ctx();
+  if (!c) return AUTOPIPE_E_NOMEM;
+  c->device = cuda_device;
+  DeviceGuard dg(cuda_device);
+  cudaDeviceGetAttribute(&c->sms, cudaDevAttrMultiProcessorCount, cuda_device);
+  host_binomials(c->binom);
+  upload_binomials(c->binom);
+  // device tables, sized for the limits (L = 255, N = 8): a few hundred KB
+  const size_t Lp1 = MAXL + 1, NL = (size_t)MAXN * Lp1;
+  const size_t words = 3 * NL + Lp1 + 2 * MAXL + 64 + 2 * 7 * MAXL;
+  const size_t words32 = NL + 2 * 7 * MAXL;
+  e = cudaMalloc(&c->d_tables, words * 8 + words32 * 4 + 64);
+  if (e == cudaSuccess) e = cudaMalloc(&c->d_raw, (2 * MAXN * MAXL + MAXL) * 8);
+  if (e == cudaSuccess) e = cudaMalloc(&c->d_blocks, sizeof(BlockOut) * MAX_BLOCKS);
+  if (e == cudaSuccess) e = cudaMalloc(&c->d_result, sizeof(ResultDev));
+  c->work_bytes = 1 << 20;
+  if (e == cudaSuccess) e = cudaMalloc(&c->d_work, c->work_bytes);
+  if (e == cudaSuccess) e = cudaMallocHost(&c->h_stage, (2 * MAXN * MAXL + 64) * 8);
+  if (e == cudaSuccess) e = cudaMallocHost(&c->h_result, sizeof(ResultDev));
+  if (e != cudaSuccess) {
+    snprintf(g_create_err, sizeof(g_create_err), "allocation: %s", cudaGetErrorString(e));
+    autopipe_destroy(c);
+    return AUTOPIPE_E_NOMEM;
+  }
+  u64 *p = c->d_tables;
+  c->tab.PF = p; p += NL;
+  c->tab.PB = p; p += NL;
+  c->tab.PC = p; p += NL;
+  c->tab.PP = p; p += Lp1;
+  c->tab.O = p; p += MAXL;
+  c->tab.G = p; p += MAXL;
+  c->tab.tau = p; p += 64;
+  c->tab.Z = p; p += 7 * MAXL;
+  c->tab.LM = p; p += 7 * MAXL;
+  u32 *q = (u32 *)p;
+  c->tab.PC32 = q; q += NL;
+  c->tab.Z32 = q; q += 7 * MAXL;
+  c->tab.LM32 = q; q += 7 * MAXL;
+  e = cudaMemset(c->d_tables, 0, words * 8 + words32 * 4 + 64);
+  if (e != cudaSuccess) {
+    snprintf(g_create_err, sizeof(g_create_err), "memset: %s", cudaGetErrorString(e));
+    autopipe_destroy(c);
+    return AUTOPIPE_E_CUDA;
+  }
+  *out = c;
+  return AUTOPIPE_OK;
+}
+
+extern "C" void autopipe_destroy(autopipe_ctx *c) {
+  if (!c) return;
+  {
+    DeviceGuard dg(c->device);
+    cudaDeviceSynchronize();
+    if (c->d_tables) cudaFree(c->d_tables);
+    if (c->d_raw) cudaFree(c->d_raw);
+    if (c->d_blocks) cudaFree(c->d_blocks);
+    if (c->d_result) cudaFree(c->d_result);
+    if (c->d_work) cudaFree(c->d_work);
+    if (c->h_stage) cudaFreeHost(c->h_stage);
+    if (c->h_result) cudaFreeHost(c->h_result);
+  }
+  delete c;
+}
+
+extern "C" const char *autopipe_last_error(const autopipe_ctx *c) { return c ? c->err : g_create_err; }
+
+extern "C" int autopipe_load_profile(autopipe_ctx *c, uint32_t L, const uint64_t *O, const uint64_t *G,
+                                     const uint64_t *P) {
+  if (!c) return AUTOPIPE_E_INVAL;
+  c->err[0] = 0;
+  if (L < 1 || L > MAXL) return fail(c, AUTOPIPE_E_INVAL, "L = %u outside [1, 255]", L);
+  if (!O || !G || !P) return fail(c, AUTOPIPE_E_INVAL, "NULL profile array");
+  u64 maxOG = 0;
+  u128 sumP = 0;
+  for (u32 l = 0; l < L; ++l) {
+    if (O[l] >= LIMIT_BYTES || G[l] >= LIMIT_BYTES || P[l] >= LIMIT_BYTES)
+      return fail(c, AUTOPIPE_E_OVERFLOW, "layer %u: a byte count >= 2^56", l);
+    maxOG = umax(maxOG, umax((u64)O[l], (u64)G[l]));
+    sumP += P[l];
+  }
+  if (sumP >= LIMIT_BYTES) return fail(c, AUTOPIPE_E_OVERFLOW, "sum of weight bytes >= 2^56");
+  DeviceGuard dg(c->device);
+  // O, G go straight to their tables; P to the raw area (the state kernel builds its prefix)
+  cudaError_t e = cudaMemcpy(c->tab.O, O, L * 8, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(c->tab.G, G, L * 8, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(c->d_raw + 2 * MAXN * MAXL, P, L * 8, cudaMemcpyHostToDevice);
+  if (e != cudaSuccess) return cuda_fail(c, e, "load_profile copy");
+  c->L = L;
+  c->maxOG = maxOG;
+  c->sumP = (u64)sumP;
+  c->has_profile = true;
+  c->has_state = false;
+  c->path32 = 0;
+  return AUTOPIPE_OK;
+}
+
+extern "C" int autopipe_set_state(autopipe_ctx *c, uint32_t N, const uint64_t *fp, const uint64_t *bp,
+                                  const uint64_t *tau, void *stream) {
+  if (!c) return AUTOPIPE_E_INVAL;
+  c->err[0] = 0;
+  if (!c->has_profile) return fail(c, AUTOPIPE_E_STATE, "set_state before load_profile");
+  if (N < 1 || N > MAXN) return fail(c, AUTOPIPE_E_INVAL, "N = %u outside [1, 8]", N);
+  if (!fp || !bp || !tau) return fail(c, AUTOPIPE_E_INVAL, "NULL state array");
+  const u32 L = c->L;
+  // overflow rules (SPEC.md §7)
+  u64 maxTau = 0;
+  for (u32 u = 0; u < N; ++u)
+    for (u32 v = 0; v < N; ++v)
+      if (u != v) maxTau = umax(maxTau, (u64)tau[u * N + v]);
+  const u64 maxBytes = umax(c->maxOG, c->sumP);
+  if ((u128)maxBytes * maxTau + 999999u >= ((u128)1 << 64))
+    return fail(c, AUTOPIPE_E_OVERFLOW, "bytes * tau reaches 2^64");
+  const u64 maxX = (u64)(((u128)maxBytes * maxTau + 999999u) / 1000000u);
+  const u64 maxXog = (u64)(((u128)c->maxOG * maxTau + 999999u) / 1000000u);
+  u128 sumMax = 0;
+  for (u32 l = 0; l < L; ++l) {
+    u128 m = 0;
+    for (u32 w = 0; w < N; ++w) {
+      const u128 v = (u128)fp[w * L + l] + bp[w * L + l];
+      if (v > m) m = v;
+    }
+    sumMax += m;
+  }
+  const u128 bound = sumMax + 16 + (u128)28 * maxX;
+  if (bound >= LIMIT_TIME) return fail(c, AUTOPIPE_E_OVERFLOW, "modelled times reach 2^59 ns");
+  const u128 bound32 = sumMax + 16 + (u128)14 * maxXog;
+  c->path32 = bound32 < LIMIT_TIME32 ? 1 : 0;
+  DeviceGuard dg(c->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  // stage into pinned memory so the copies are truly asynchronous
+  cudaError_t e = cudaStreamSynchronize(st);  // the staging buffer may still feed a previous copy
+  if (e != cudaSuccess) return cuda_fail(c, e, "set_state sync");
+  u64 *hf = c->h_stage, *hb = hf + MAXN * MAXL, *ht = hb + MAXN * MAXL;
+  memcpy(hf, fp, (size_t)N * L * 8);
+  memcpy(hb, bp, (size_t)N * L * 8);
+  for (int u = 0; u < 8; ++u)
+    for (int v = 0; v < 8; ++v) ht[u * 8 + v] = (u < (int)N && v < (int)N && u != v) ? tau[u * N + v] : 0;
+  e = cudaMemcpyAsync(c->d_raw, hf, (size_t)N * L * 8, cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(c->d_raw + MAXN * MAXL, hb, (size_t)N * L * 8, cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(c->tab.tau, ht, 64 * 8, cudaMemcpyHostToDevice, st);
+  if (e != cudaSuccess) return cuda_fail(c, e, "set_state copy");
+  c->tab.L = L;
+  c->tab.N = N;
+  c->tab.Lp1 = L + 1;
+  c->N = N;
+  c->launches += launch_build_state(c->tab, c->d_raw, c->d_raw + MAXN * MAXL, c->d_raw + 2 * MAXN * MAXL,
+                                    c->path32, st);
+  e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(c, e, "state kernel launch");
+  c->has_state = true;
+  return AUTOPIPE_OK;
+}
+
+extern "C" int autopipe_eval_partitions(autopipe_ctx *c, const autopipe_partition *d_parts, uint64_t count,
+                                        uint64_t *d_time_ns, void *stream) {
+  if (!c) return AUTOPIPE_E_INVAL;
+  c->err[0] = 0;
+  if (!c->has_state) return fail(c, AUTOPIPE_E_STATE, "eval before set_state");
+  if (count == 0) return AUTOPIPE_OK;
+  if (!d_parts || !d_time_ns) return fail(c, AUTOPIPE_E_INVAL, "NULL device pointer");
+  DeviceGuard dg(c->device);
+  c->launches += launch_eval(c->tab, d_parts, count, (u64 *)d_time_ns, nullptr, nullptr, nullptr, nullptr, c->sms,
+                             (cudaStream_t)stream);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(c, e, "eval kernel launch");
+  return AUTOPIPE_OK;
+}
+
+// --- search space arithmetic (SPEC.md §5) ----------------------------------------------------
+static bool build_space(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, SearchSpace &sp) {
+  memset(&sp, 0, sizeof(sp));
+  sp.L = (int)c->L;
+  sp.N = (int)c->N;
+  sp.s_min = (int)s_min;
+  sp.s_max = (int)s_max;
+  sp.flags = (int)(flags & AUTOPIPE_USE_ALL_WORKERS);
+  u128 off = 0;
+  for (int S = (int)s_min; S <= (int)s_max; ++S) {
+    sp.off[S] = (u64)off;
+    const u64 K = (flags & AUTOPIPE_USE_ALL_WORKERS) ? c->binom[c->N - 1][S - 1] : c->binom[c->N][S];
+    const u64 nc = (S - 1 <= (int)c->L - 1) ? c->binom[c->L - 1][S - 1] : 0;
+    sp.ncut[S] = nc;
+    sp.ncomp[S] = K;
+    off += (u128)K * nc;
+    if (off >> 64) return false;
+  }
+  sp.off[s_max + 1] = (u64)off;
+  return true;
+}
+
+static int check_space_args(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags) {
+  if (flags & ~AUTOPIPE_USE_ALL_WORKERS) return fail(c, AUTOPIPE_E_INVAL, "unknown flags 0x%x", flags);
+  const u32 smax_lim = c->N < (u32)MAXS ? c->N : (u32)MAXS;
+  if (s_min < 1 || s_min > s_max || s_max > smax_lim)
+    return fail(c, AUTOPIPE_E_INVAL, "need 1 <= s_min <= s_max <= min(8, N) (got %u, %u, N = %u)", s_min,
+                s_max, c->N);
+  return AUTOPIPE_OK;
+}
+
+extern "C" int autopipe_count_candidates(const autopipe_ctx *cc, uint32_t s_min, uint32_t s_max,
+                                         uint32_t flags, uint64_t *total) {
+  autopipe_ctx *c = const_cast<autopipe_ctx *>(cc);
+  if (!c || !total) return AUTOPIPE_E_INVAL;
+  if (!c->has_state) return fail(c, AUTOPIPE_E_STATE, "count before set_state");
+  int rc = check_space_args(c, s_min, s_max, flags);
+  if (rc) return rc;
+  SearchSpace sp;
+  if (!build_space(c, s_min, s_max, flags, sp)) return fail(c, AUTOPIPE_E_OVERFLOW, "space exceeds 2^64");
+  *total = sp.off[s_max + 1];
+  return AUTOPIPE_OK;
+}
+
+static u64 host_unrank(const autopipe_ctx *c, u64 rank, int k, int n) {
+  u64 out = 0;
+  int x = 0;
+  for (int i = 0; i < k; ++i) {
+    while (c->binom[n - 1 - x][k - 1 - i] <= rank) {
+      rank -= c->binom[n - 1 - x][k - 1 - i];
+      ++x;
+    }
+    out |= (u64)x << (8 * i);
+    ++x;
+  }
+  return out;
+}
+
+extern "C" int autopipe_decode_index(const autopipe_ctx *cc, uint32_t s_min, uint32_t s_max, uint32_t flags,
+                                     uint64_t index, autopipe_partition *out) {
+  autopipe_ctx *c = const_cast<autopipe_ctx *>(cc);
+  if (!c || !out) return AUTOPIPE_E_INVAL;
+  if (!c->has_state) return fail(c, AUTOPIPE_E_STATE, "decode before set_state");
+  int rc = check_space_args(c, s_min, s_max, flags);
+  if (rc) return rc;
+  SearchSpace sp;
+  if (!build_space(c, s_min, s_max, flags, sp)) return fail(c, AUTOPIPE_E_OVERFLOW, "space exceeds 2^64");
+  if (index >= sp.off[s_max + 1]) return fail(c, AUTOPIPE_E_INVAL, "index beyond the space");
+  int S = (int)s_min;
+  while (S < (int)s_max && index >= sp.off[S + 1]) ++S;
+  const u64 rem = index - sp.off[S];
+  const u64 rho = rem / sp.ncut[S], kappa = rem % sp.ncut[S];
+  const bool all = flags & AUTOPIPE_USE_ALL_WORKERS;
+  const u64 Rp = all ? host_unrank(c, rho, S - 1, (int)c->N - 1) : host_unrank(c, rho, S, (int)c->N);
+  const u64 cuts = host_unrank(c, kappa, S - 1, (int)c->L - 1);
+  memset(out, 0xFF, sizeof(*out));
+  out->n_stages = (uint8_t)S;
+  for (int s = 0; s < S - 1; ++s) out->last_layer[s] = (uint8_t)((cuts >> (8 * s)) & 0xFF);
+  int prev = 0;
+  for (int s = 0; s < S; ++s) {
+    const int R = (all && s == S - 1) ? (int)c->N : (int)((Rp >> (8 * s)) & 0xFF) + 1;
+    for (int w = prev; w < R; ++w) out->stage_of_worker[w] = (uint8_t)s;
+    prev = R;
+  }
+  return AUTOPIPE_OK;
+}
+
+extern "C" int autopipe_search_optimum(autopipe_ctx *c, uint32_t s_min, uint32_t s_max, uint32_t flags,
+                                       uint64_t begin, uint64_t end, autopipe_result *h_out, void *stream) {
+  if (!c) return AUTOPIPE_E_INVAL;
+  c->err[0] = 0;
+  if (!c->has_state) return fail(c, AUTOPIPE_E_STATE, "search before set_state");
+  if (!h_out) return fail(c, AUTOPIPE_E_INVAL, "NULL result pointer");
+  int rc = check_space_args(c, s_min, s_max, flags);
+  if (rc) return rc;
+  SearchSpace sp;
+  if (!build_space(c, s_min, s_max, flags, sp)) return fail(c, AUTOPIPE_E_OVERFLOW, "space exceeds 2^64");
+  const u64 total = sp.off[s_max + 1];
+  if (end > total) end = total;
+  memset(h_out, 0, sizeof(*h_out));
+  h_out->time_ns = U64MAX;
+  h_out->index = U64MAX;
+  memset(&h_out->part, 0xFF, sizeof(h_out->part));
+  if (begin >= end) return AUTOPIPE_OK;
+  DeviceGuard dg(c->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  int used = 0;
+  // Split [begin, end) into the r = 1 block of each S (rho = 0: fast kernel) and the rest (generic).
+  u64 cur = begin;
+  for (int S = (int)s_min; S <= (int)s_max && cur < end; ++S) {
+    const u64 blo = sp.off[S], bhi = sp.off[S + 1];
+    if (bhi <= cur) continue;
+    const u64 lo = cur, hi = end < bhi ? end : bhi;
+    // candidates with rho = 0 are [blo, blo + ncut); rho = 0 is all-r=1 iff the first composition
+    // (R = 1..S) has every r_s = 1, which holds for the default flag and for USE_ALL when N = S.
+    const bool r1 = S >= 3 && (!(flags & AUTOPIPE_USE_ALL_WORKERS) || (int)c->N == S);
+    const u64 r1hi = blo + sp.ncut[S];
+    if (r1 && lo < r1hi) {
+      const u64 a = lo, b = hi < r1hi ? hi : r1hi;
+      int nb = 0;
+      c->launches += launch_search_r1(c->tab, sp, S, a - blo, b - blo, c->path32, c->sms, c->d_blocks + used,
+                                      MAX_BLOCKS - used, &nb, c->d_work, c->work_bytes, st);
+      used += nb;
+      if (b < hi) {
+        c->launches += launch_search_generic(c->tab, sp, b, hi, c->sms, c->d_blocks + used, MAX_BLOCKS - used,
+                                             &nb, st);
+        used += nb;
+      }
+    } else {
+      int nb = 0;
+      c->launches += launch_search_generic(c->tab, sp, lo, hi, c->sms, c->d_blocks + used, MAX_BLOCKS - used,
+                                           &nb, st);
+      used += nb;
+    }
+    cur = hi;
+    if (used > MAX_BLOCKS - 4 * c->sms) {  // keep room: fold what we have into one entry
+      c->launches += launch_finalize(c->d_blocks, used, sp, c->d_result, st);
+      cudaMemcpyAsync(c->d_blocks, c->d_result, sizeof(BlockOut), cudaMemcpyDeviceToDevice, st);
+      used = 1;
+    }
+  }
+  c->launches += launch_finalize(c->d_blocks, used, sp, c->d_result, st);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(c, e, "search kernel launch");
+  e = cudaMemcpyAsync(c->h_result, c->d_result, sizeof(ResultDev), cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  if (e != cudaSuccess) return cuda_fail(c, e, "search");
+  h_out->time_ns = c->h_result->time_ns;
+  h_out->index = c->h_result->index;
+  h_out->evaluated = c->h_result->evaluated;
+  memcpy(&h_out->part, c->h_result->part, 16);
+  return AUTOPIPE_OK;
+}
+
+// host-side validation of the current partition of a rollout (same rules as SPEC.md §2)
+static bool host_decode(const autopipe_partition *p, u32 L, u32 N, int &S, u64 &cuts, u64 &masks) {
+  S = p->n_stages;
+  if (S < 1 || S > MAXS || S > (int)N) return false;
+  cuts = 0;
+  int prev = -1;
+  for (int i = 0; i < S - 1; ++i) {
+    const int e = p->last_layer[i];
+    if (e <= prev || e >= (int)L - 1) return false;
+    prev = e;
+    cuts |= (u64)e << (8 * i);
+  }
+  masks = 0;
+  for (int w = 0; w < MAXN; ++w) {
+    const int s = p->stage_of_worker[w];
+    if (s == 0xFF) continue;
+    if (w >= (int)N || s >= S) return false;
+    masks |= 1ull << (8 * s + w);
+  }
+  for (int s = 0; s < S; ++s)
+    if (((masks >> (8 * s)) & 0xFF) == 0) return false;
+  return true;
+}
+
+extern "C" int autopipe_rollout_rewards(autopipe_ctx *c, const autopipe_partition *d_parts, uint64_t count,
+                                        const autopipe_partition *h_current, uint64_t *d_time_ns,
+                                        uint64_t *d_switch_bytes, void *stream) {
+  if (!c) return AUTOPIPE_E_INVAL;
+  c->err[0] = 0;
+  if (!c->has_state) return fail(c, AUTOPIPE_E_STATE, "rollout before set_state");
+  if ((h_current == nullptr) != (d_switch_bytes == nullptr))
+    return fail(c, AUTOPIPE_E_INVAL, "h_current and d_switch_bytes must both be set or both be NULL");
+  int S = 0;
+  u64 cuts = 0, masks = 0;
+  if (h_current && !host_decode(h_current, c->L, c->N, S, cuts, masks))
+    return fail(c, AUTOPIPE_E_INVAL, "invalid current partition");
+  if (count == 0) return AUTOPIPE_OK;
+  if (!d_parts || !d_time_ns) return fail(c, AUTOPIPE_E_INVAL, "NULL device pointer");
+  DeviceGuard dg(c->device);
+  c->launches += launch_eval(c->tab, d_parts, count, (u64 *)d_time_ns, (u64 *)d_switch_bytes, h_current ? &S : nullptr,
+                             &cuts, &masks, c->sms, (cudaStream_t)stream);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(c, e, "rollout kernel launch");
+  return AUTOPIPE_OK;
+}
+
+extern "C" int autopipe_int_path(const autopipe_ctx *c) {
+  return (c && c->has_state) ? (c->path32 ? 32 : 64) : 0;
+}
+
+extern "C" uint64_t autopipe_kernel_launches(const autopipe_ctx *c) { return c ? c->launches : 0; }

@@ -1,0 +1,109 @@
+// common.cuh — device-side data layout and integer helpers of the AutoPipe cost-model engine.
+//
+// Everything is unsigned integer arithmetic (SPEC.md: times in ns, bytes, inverse bandwidth in
+// fs/byte). The host (autopipe.cu) guarantees, through the overflow checks of set_state, that every
+// sum formed here is < 2^59 and every bytes*tau product is < 2^64, so u64 is exact throughout.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace ap {
+
+typedef unsigned long long u64;
+typedef unsigned int u32;
+
+constexpr int MAXS = 8;       // stages (C-15)
+constexpr int MAXN = 8;       // workers
+constexpr int MAXL = 255;     // layers
+constexpr int BINOM_N = 256;  // C(n, k) for n < 256
+constexpr int BINOM_K = 9;    // k <= 8
+constexpr u64 U64MAX = ~0ull;
+
+// Global-memory tables written by the state kernels (k_state.cu) and read by every scoring kernel.
+// All arrays are row-major; "Lp1" = L + 1 (exclusive prefix sums have L + 1 entries).
+struct DevTables {
+  u32 L, N, Lp1, pad;
+  u64 *PF;    // [N][L+1]  exclusive prefix of fp_ns per worker          (row a1)
+  u64 *PB;    // [N][L+1]  exclusive prefix of bp_ns per worker          (row a1)
+  u64 *PC;    // [N][L+1]  exclusive prefix of fp_ns + bp_ns (r = 1 stage cost)
+  u64 *PP;    // [L+1]     exclusive prefix of weight bytes              (row a1)
+  u64 *O;     // [L]       activation bytes
+  u64 *G;     // [L]       input-gradient bytes
+  u64 *tau;   // [8][8]    fs per byte, row u -> column v (padded to 8x8)
+  u64 *Z;     // [7][L]    r = 1 boundary s (worker s -> s+1) cut after layer l: cf + cb   (row a2)
+  u64 *LM;    // [7][L]    ... max(cf, cb)                                                (row a2)
+  u32 *PC32;  // [N][L+1]  32-bit copies for the 32-bit search path (valid iff path32)
+  u32 *Z32;   // [7][L]
+  u32 *LM32;  // [7][L]
+};
+
+__host__ __device__ __forceinline__ u64 umax(u64 a, u64 b) { return a > b ? a : b; }
+__host__ __device__ __forceinline__ u64 umin(u64 a, u64 b) { return a < b ? a : b; }
+
+// ceil(x / 10^6) for the transfer time xfer(x, tau) = ceil(x * tau / 1e6) (SPEC.md §1, C-7).
+__device__ __forceinline__ u64 xfer(u64 bytes, u64 fs_per_byte) {
+  const u64 p = bytes * fs_per_byte;  // < 2^64 (set_state check)
+  return (p + 999999ull) / 1000000ull;
+}
+
+// floor(x / d) for a runtime divisor d in [1, 8] and x < 2^63 (Granlund-Montgomery with N = 63:
+// m = ceil(2^(63+l)/d), l = ceil(log2 d); exact for every x < 2^63).
+__device__ __forceinline__ u64 div_small(u64 x, u32 d) {
+  // branch-free selection of the multiplier and post-shift; d = 1 is the identity
+  const u64 m = (d == 3u || d == 6u) ? 0xaaaaaaaaaaaaaaabull
+              : (d == 5u)            ? 0xcccccccccccccccdull
+              : (d == 7u)            ? 0x924924924924924aull
+                                     : 0x8000000000000000ull;
+  const u32 sh = (d <= 2u) ? 0u : (d <= 4u) ? 1u : 2u;
+  const u64 q = __umul64hi(x, m) >> sh;
+  return d == 1u ? x : q;
+}
+__device__ __forceinline__ u64 ceil_small(u64 x, u32 d) { return div_small(x + d - 1, d); }
+
+__device__ __forceinline__ int byte_at(u64 v, int i) { return (int)((v >> (8 * i)) & 0xFF); }
+
+// Lexicographic (time, index) minimum used by every argmin (reading C-13: smallest index wins ties).
+struct MinLoc {
+  u64 t, idx;
+};
+__device__ __forceinline__ bool better(u64 t1, u64 i1, u64 t2, u64 i2) {
+  return t1 < t2 || (t1 == t2 && i1 < i2);
+}
+__device__ __forceinline__ void warp_minloc(u64 &t, u64 &idx) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const u64 t2 = __shfl_xor_sync(0xffffffffu, t, o);
+    const u64 i2 = __shfl_xor_sync(0xffffffffu, idx, o);
+    if (better(t2, i2, t, idx)) { t = t2; idx = i2; }
+  }
+}
+__device__ __forceinline__ u64 warp_sum(u64 v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+// Block-level (time, index) minimum + evaluated count; thread 0 writes the block's entry.
+// Deterministic: the lexicographic min and the integer sum do not depend on the order.
+struct BlockOut {
+  u64 t, idx, count, pad;
+};
+template <int NT>
+__device__ __forceinline__ void block_minloc_store(u64 t, u64 idx, u64 cnt, BlockOut *dst) {
+  __shared__ u64 st[NT / 32], si[NT / 32], sc[NT / 32];
+  warp_minloc(t, idx);
+  cnt = warp_sum(cnt);
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  if (lane == 0) { st[wid] = t; si[wid] = idx; sc[wid] = cnt; }
+  __syncthreads();
+  if (wid == 0) {
+    t = (lane < NT / 32) ? st[lane] : U64MAX;
+    idx = (lane < NT / 32) ? si[lane] : U64MAX;
+    cnt = (lane < NT / 32) ? sc[lane] : 0;
+    warp_minloc(t, idx);
+    cnt = warp_sum(cnt);
+    if (lane == 0) { dst->t = t; dst->idx = idx; dst->count = cnt; }
+  }
+}
+
+}  // namespace ap

@@ -1,0 +1,212 @@
+// eval.cuh — the closed form of the cost model for one partition (SPEC.md §4), rows a4-a7.
+//
+// T_ns = max( max_s X_s, max_s AR_s, max_s cf_s, max_s cb_s, max_{s<t} ceil(W(s,t)/(t-s+1)) ),
+// W(s,t) = X_s + X_t + sum_{s<u<t}(Fm_u + Bm_u) + sum_{u=s}^{t-1}(cf_u + cb_u).
+// These are the elementary cycles of the timed event graph of the static 1F1B schedule
+// (PAPER.md:253-278, 463-475, 521-580); tests check the equality against the oracle's event
+// simulation bit for bit.
+//
+// A partition is (S, cuts, masks): cuts packed one byte per cut (byte s = e_s, s < S-1), masks
+// packed one byte per stage (byte s = bitmask of the workers of stage s). All loops over stages are
+// fully unrolled so every per-stage value lives in registers.
+#pragma once
+#include "common.cuh"
+
+namespace ap {
+
+// Read-only view of the state tables staged in shared memory.
+struct SmemTab {
+  const u64 *PF, *PB, *PP, *O, *G, *tau;
+  int L, Lp1;
+};
+
+// Number of u64 words the staged tables need: PF, PB (N x (L+1)), PP (L+1), O, G (L), tau (64).
+__host__ __device__ __forceinline__ u32 smem_words(u32 L, u32 N) {
+  return 2u * N * (L + 1) + (L + 1) + 2u * L + 64u;
+}
+
+// Cooperative copy of the global tables into shared memory (every thread of the block calls it).
+__device__ __forceinline__ SmemTab stage_tables(const DevTables &g, u64 *sm) {
+  const u32 L = g.L, N = g.N, Lp1 = g.Lp1;
+  u64 *PF = sm, *PB = PF + N * Lp1, *PP = PB + N * Lp1, *O = PP + Lp1, *G = O + L, *tau = G + L;
+  for (u32 i = threadIdx.x; i < N * Lp1; i += blockDim.x) {
+    PF[i] = g.PF[i];
+    PB[i] = g.PB[i];
+  }
+  for (u32 i = threadIdx.x; i < Lp1; i += blockDim.x) PP[i] = g.PP[i];
+  for (u32 i = threadIdx.x; i < L; i += blockDim.x) {
+    O[i] = g.O[i];
+    G[i] = g.G[i];
+  }
+  for (u32 i = threadIdx.x; i < 64; i += blockDim.x) tau[i] = g.tau[i];
+  __syncthreads();
+  SmemTab t;
+  t.PF = PF; t.PB = PB; t.PP = PP; t.O = O; t.G = G; t.tau = tau;
+  t.L = (int)L; t.Lp1 = (int)Lp1;
+  return t;
+}
+
+// Largest transfer of one stage boundary (row a5): A bytes split into r_send and r_recv equal shards
+// ([floor(iA/r), floor((i+1)A/r))); every overlapping (sender, receiver) pair is one transfer on its
+// directed link, lasting ceil(overlap * tau / 1e6). A merge walk visits the <= r_s + r_r - 1
+// overlapping pairs in order.
+__device__ __forceinline__ u64 boundary_max(u64 A, u32 send, u32 recv, const u64 *tau) {
+  const u32 rs = __popc(send), rr = __popc(recv);
+  if (rs == 1 && rr == 1) {
+    const int u = __ffs(send) - 1, v = __ffs(recv) - 1;
+    return xfer(A, tau[u * 8 + v]);
+  }
+  u64 best = 0;
+  u32 i = 0, j = 0;
+  u64 lo_i = 0, lo_j = 0;
+  u64 hi_i = div_small(A, rs), hi_j = div_small(A, rr);
+  while (i < rs && j < rr) {
+    const u64 lo = umax(lo_i, lo_j), hi = umin(hi_i, hi_j);
+    if (hi > lo) {
+      const int u = __ffs(send) - 1, v = __ffs(recv) - 1;
+      best = umax(best, xfer(hi - lo, tau[u * 8 + v]));
+    }
+    const bool adv_i = hi_i <= hi_j, adv_j = hi_j <= hi_i;
+    if (adv_i) {
+      ++i; send &= send - 1;
+      lo_i = hi_i; hi_i = div_small((u64)(i + 1) * A, rs);
+    }
+    if (adv_j) {
+      ++j; recv &= recv - 1;
+      lo_j = hi_j; hi_j = div_small((u64)(j + 1) * A, rr);
+    }
+  }
+  return best;
+}
+
+// Ring all-reduce of a replicated stage (row a6): 2(r-1) steps of a ceil(P_s/r)-byte chunk over the
+// slowest link of the ring W_s[0] -> W_s[1] -> ... -> W_s[0] (ascending worker order).
+__device__ __forceinline__ u64 allreduce_time(u64 Ps, u32 mask, const u64 *tau) {
+  const u32 r = __popc(mask);
+  const int first = __ffs(mask) - 1;
+  int prev = first;
+  u32 m = mask & (mask - 1);
+  u64 tr = 0;
+  while (m) {
+    const int w = __ffs(m) - 1;
+    m &= m - 1;
+    tr = umax(tr, tau[prev * 8 + w]);
+    prev = w;
+  }
+  tr = umax(tr, tau[prev * 8 + first]);
+  return 2ull * (u64)(r - 1) * xfer(ceil_small(Ps, r), tr);
+}
+
+// The full closed form (rows a4-a7) for one partition; S in [1, 8], the partition already validated.
+__device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, u64 cuts, u64 masks) {
+  u64 X[MAXS], Y[MAXS], Zb[MAXS];
+  u64 T = 0;
+#pragma unroll
+  for (int s = 0; s < MAXS; ++s) {
+    X[s] = 0;
+    Y[s] = 0;
+    if (s < S) {
+      const int a = (s == 0) ? 0 : byte_at(cuts, s - 1) + 1;
+      const int e = (s == S - 1) ? t.L - 1 : byte_at(cuts, s);
+      const u32 mask = (u32)byte_at(masks, s);
+      const u32 r = __popc(mask);
+      u64 fm = 0, bm = 0, xm = 0;
+      u32 m = mask;
+      while (m) {  // row a4: split replicas, ceil(sum / r) per op
+        const int w = __ffs(m) - 1;
+        m &= m - 1;
+        const u64 F = ceil_small(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a], r);
+        const u64 B = ceil_small(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a], r);
+        fm = umax(fm, F);
+        bm = umax(bm, B);
+        xm = umax(xm, F + B);
+      }
+      X[s] = xm;
+      Y[s] = fm + bm;
+      T = umax(T, xm);
+      if (r >= 2) T = umax(T, allreduce_time(t.PP[e + 1] - t.PP[a], mask, t.tau));
+    }
+  }
+#pragma unroll
+  for (int s = 0; s < MAXS - 1; ++s) {  // row a5
+    Zb[s] = 0;
+    if (s < S - 1) {
+      const int e = byte_at(cuts, s);
+      const u32 ms = (u32)byte_at(masks, s), mn = (u32)byte_at(masks, s + 1);
+      const u64 cf = boundary_max(t.O[e], ms, mn, t.tau);
+      const u64 cb = boundary_max(t.G[e + 1], mn, ms, t.tau);
+      Zb[s] = cf + cb;
+      T = umax(T, umax(cf, cb));
+    }
+  }
+  Zb[MAXS - 1] = 0;
+#pragma unroll
+  for (int s = 0; s < MAXS - 1; ++s) {  // row a7: segment cycles, t-s+1 tokens
+    if (s < S - 1) {
+      u64 acc = X[s];
+#pragma unroll
+      for (int u = s + 1; u < MAXS; ++u) {
+        if (u < S) {
+          const u64 W = acc + Zb[u - 1] + X[u];
+          T = umax(T, (W + (u64)(u - s)) / (u64)(u - s + 1));
+          acc += Zb[u - 1] + Y[u];
+        }
+      }
+    }
+  }
+  return T;
+}
+
+// Decode + validate a 16-byte record (SPEC.md §2). Returns false for an invalid record.
+// lo = bytes 0..7 (S, cuts), hi = bytes 8..15 (stage of worker w in byte w).
+__device__ __forceinline__ bool decode_record(u64 lo, u64 hi, int L, int N, int &S, u64 &cuts,
+                                              u64 &masks) {
+  S = (int)(lo & 0xFF);
+  if (S < 1 || S > MAXS || S > N) return false;
+  cuts = lo >> 8;
+  bool ok = true;
+  int prev = -1;
+#pragma unroll
+  for (int i = 0; i < MAXS - 1; ++i) {
+    if (i < S - 1) {
+      const int e = byte_at(cuts, i);
+      ok &= (e > prev) & (e < L - 1);
+      prev = e;
+    }
+  }
+  masks = 0;
+#pragma unroll
+  for (int w = 0; w < MAXN; ++w) {
+    const int s = byte_at(hi, w);
+    if (s != 0xFF) {
+      ok &= (w < N) & (s < S);
+      if (s < S) masks |= 1ull << (8 * s + w);
+    }
+  }
+#pragma unroll
+  for (int s = 0; s < MAXS; ++s)
+    if (s < S) ok &= byte_at(masks, s) != 0;
+  return ok;
+}
+
+// Switch bytes versus the current partition (SPEC.md §6): sum over layers l of
+// P[l] * |W_new(l) \ W_old(l)|, walked over the maximal layer ranges on which both partitions keep
+// the same stage (at most S_new + S_old - 1 ranges), using the weight prefix PP.
+__device__ __forceinline__ u64 switch_bytes(const SmemTab &t, int S, u64 cuts, u64 masks, int So,
+                                            u64 cuts_o, u64 masks_o) {
+  u64 sw = 0;
+  int sn = 0, so = 0, l = 0;
+  while (l < t.L) {
+    const int en = (sn == S - 1) ? t.L - 1 : byte_at(cuts, sn);
+    const int eo = (so == So - 1) ? t.L - 1 : byte_at(cuts_o, so);
+    const int hi = en < eo ? en : eo;
+    const u32 gained = (u32)byte_at(masks, sn) & ~(u32)byte_at(masks_o, so);
+    sw += (u64)__popc(gained) * (t.PP[hi + 1] - t.PP[l]);
+    l = hi + 1;
+    sn += (en == hi);
+    so += (eo == hi);
+  }
+  return sw;
+}
+
+}  // namespace ap

@@ -1,0 +1,173 @@
+"""Python API over the C-ABI (include/autopipe.h): argument marshalling only.
+
+Every score is computed by the sm_100a kernels of ``libautopipe.so``; torch is used for device
+memory and streams. Outputs that the C-ABI defines as ``uint64`` come back as ``torch.int64`` tensors
+holding the same bits (UINT64_MAX reads as -1); ``as_u64`` converts them to numpy uint64.
+"""
+from __future__ import annotations
+
+import ctypes
+from dataclasses import dataclass
+from typing import Optional, Sequence, Tuple
+
+import numpy as np
+import torch
+
+from . import _lib
+from ._lib import AutopipeError, Partition, Result, USE_ALL_WORKERS, lib
+
+U64_MAX = (1 << 64) - 1
+
+
+def _u64_array(x, n: Optional[int] = None) -> np.ndarray:
+    a = np.ascontiguousarray(np.asarray(x, dtype=np.uint64).reshape(-1))
+    if n is not None and a.size != n:
+        raise ValueError("expected %d values, got %d" % (n, a.size))
+    return a
+
+
+def _ptr(a: np.ndarray):
+    return a.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64))
+
+
+def as_u64(t: torch.Tensor) -> np.ndarray:
+    """Reinterpret an int64 tensor written by the kernels as uint64 (host copy)."""
+    return t.detach().cpu().numpy().view(np.uint64)
+
+
+def record_bytes(p: Partition) -> bytes:
+    return bytes(bytearray(p))
+
+
+@dataclass
+class SearchResult:
+    time_ns: int
+    index: int
+    evaluated: int
+    partition: bytes   # the 16-byte record of the best candidate
+
+    @property
+    def empty(self) -> bool:
+        return self.index == U64_MAX
+
+
+class Engine:
+    """One engine per CUDA device (not thread-safe), mirroring ``autopipe_ctx``."""
+
+    def __init__(self, device: int = 0):
+        if not torch.cuda.is_available():
+            raise RuntimeError("the AutoPipe cost-model engine needs a CUDA device (no CPU fallback)")
+        self.device = torch.device("cuda", device)
+        h = ctypes.c_void_p()
+        rc = lib.autopipe_create(int(device), ctypes.byref(h))
+        if rc != 0:
+            raise AutopipeError(rc, lib.autopipe_last_error(None).decode())
+        self._h = h
+        self.L = 0
+        self.N = 0
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib.autopipe_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def _check(self, rc: int):
+        if rc != 0:
+            raise AutopipeError(rc, lib.autopipe_last_error(self._h).decode())
+
+    def _stream(self, stream=None):
+        s = stream if stream is not None else torch.cuda.current_stream(self.device)
+        return ctypes.c_void_p(s.cuda_stream)
+
+    # -- Table 1 inputs --------------------------------------------------------------------
+    def load_profile(self, O: Sequence[int], G: Sequence[int], P: Sequence[int]) -> None:
+        o, g, p = _u64_array(O), _u64_array(G), _u64_array(P)
+        if not (o.size == g.size == p.size):
+            raise ValueError("O, G, P must have the same length L")
+        self._check(lib.autopipe_load_profile(self._h, o.size, _ptr(o), _ptr(g), _ptr(p)))
+        self.L = int(o.size)
+
+    def set_state(self, fp, bp, tau, stream=None) -> None:
+        f = np.asarray(fp, dtype=np.uint64)
+        N = int(f.shape[0]) if f.ndim == 2 else len(fp)
+        fa = _u64_array(fp, N * self.L)
+        ba = _u64_array(bp, N * self.L)
+        ta = _u64_array(tau, N * N)
+        self._check(lib.autopipe_set_state(self._h, N, _ptr(fa), _ptr(ba), _ptr(ta), self._stream(stream)))
+        self.N = N
+
+    def load(self, profile, state, stream=None) -> None:
+        """Convenience: load_profile + set_state from workloads.Profile / workloads.State objects."""
+        self.load_profile(profile.O, profile.G, profile.P)
+        self.set_state(state.f, state.b, state.tau, stream)
+
+    # -- scoring ---------------------------------------------------------------------------
+    def _records(self, parts) -> torch.Tensor:
+        if not isinstance(parts, torch.Tensor):
+            parts = torch.as_tensor(np.asarray(parts, dtype=np.uint8).reshape(-1, 16))
+        if parts.dtype != torch.uint8 or parts.dim() != 2 or parts.shape[1] != 16:
+            raise ValueError("partitions must be a uint8 tensor of shape [n, 16]")
+        if parts.device != self.device:
+            parts = parts.to(self.device)
+        return parts.contiguous()
+
+    def eval_partitions(self, parts, out: Optional[torch.Tensor] = None, stream=None) -> torch.Tensor:
+        recs = self._records(parts)
+        n = recs.shape[0]
+        if out is None:
+            out = torch.empty(n, dtype=torch.int64, device=self.device)
+        self._check(lib.autopipe_eval_partitions(self._h, ctypes.c_void_p(recs.data_ptr()), n,
+                                                 ctypes.c_void_p(out.data_ptr()), self._stream(stream)))
+        return out
+
+    def rollout_rewards(self, parts, current: Optional[bytes] = None, out_t=None, out_sw=None,
+                        stream=None) -> Tuple[torch.Tensor, Optional[torch.Tensor]]:
+        recs = self._records(parts)
+        n = recs.shape[0]
+        if out_t is None:
+            out_t = torch.empty(n, dtype=torch.int64, device=self.device)
+        cur = None
+        if current is not None:
+            cur = Partition.from_buffer_copy(bytes(current))
+            if out_sw is None:
+                out_sw = torch.empty(n, dtype=torch.int64, device=self.device)
+        else:
+            out_sw = None
+        self._check(lib.autopipe_rollout_rewards(
+            self._h, ctypes.c_void_p(recs.data_ptr()), n, ctypes.byref(cur) if cur is not None else None,
+            ctypes.c_void_p(out_t.data_ptr()),
+            ctypes.c_void_p(out_sw.data_ptr()) if out_sw is not None else None, self._stream(stream)))
+        return out_t, out_sw
+
+    def search_optimum(self, s_min: int, s_max: int, flags: int = 0, begin: int = 0,
+                       end: Optional[int] = None, stream=None) -> SearchResult:
+        res = Result()
+        e = U64_MAX if end is None else int(end)
+        self._check(lib.autopipe_search_optimum(self._h, s_min, s_max, flags, int(begin), e,
+                                                ctypes.byref(res), self._stream(stream)))
+        return SearchResult(int(res.time_ns), int(res.index), int(res.evaluated), record_bytes(res.part))
+
+    # -- support ---------------------------------------------------------------------------
+    def count_candidates(self, s_min: int, s_max: int, flags: int = 0) -> int:
+        v = ctypes.c_uint64()
+        self._check(lib.autopipe_count_candidates(self._h, s_min, s_max, flags, ctypes.byref(v)))
+        return int(v.value)
+
+    def decode_index(self, s_min: int, s_max: int, flags: int, index: int) -> bytes:
+        p = Partition()
+        self._check(lib.autopipe_decode_index(self._h, s_min, s_max, flags, int(index), ctypes.byref(p)))
+        return record_bytes(p)
+
+    @property
+    def int_path(self) -> int:
+        return int(lib.autopipe_int_path(self._h))
+
+    @property
+    def kernel_launches(self) -> int:
+        return int(lib.autopipe_kernel_launches(self._h))

@@ -1,0 +1,55 @@
+"""Parallel evaluation of the oracle over many records (test infrastructure)."""
+from __future__ import annotations
+
+import multiprocessing as mp
+import os
+from typing import List, Sequence
+
+_CTX = {}
+
+
+def _init(prof, st):
+    _CTX["prof"] = prof
+    _CTX["st"] = st
+
+
+def _score(rec: bytes) -> int:
+    from oracle.sim import score_record
+    return score_record(_CTX["prof"], _CTX["st"], rec)
+
+
+def _score_pair(args):
+    from oracle.rollout import rollout_rewards
+    rec, cur = args
+    t, sw = rollout_rewards(_CTX["prof"], _CTX["st"], [rec], cur)
+    return t[0], (sw[0] if sw is not None else None)
+
+
+def cores() -> int:
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:
+        return os.cpu_count() or 1
+
+
+def score_many(prof, st, records: Sequence[bytes], procs: int = 0) -> List[int]:
+    records = [bytes(r) for r in records]
+    procs = procs or cores()
+    if procs <= 1 or len(records) < 64:
+        _init(prof, st)
+        return [_score(r) for r in records]
+    with mp.get_context("fork").Pool(procs, initializer=_init, initargs=(prof, st)) as pool:
+        return pool.map(_score, records, chunksize=max(1, len(records) // (procs * 8)))
+
+
+def rollout_many(prof, st, records: Sequence[bytes], current, procs: int = 0):
+    records = [bytes(r) for r in records]
+    procs = procs or cores()
+    args = [(r, current) for r in records]
+    if procs <= 1 or len(records) < 64:
+        _init(prof, st)
+        out = [_score_pair(a) for a in args]
+    else:
+        with mp.get_context("fork").Pool(procs, initializer=_init, initargs=(prof, st)) as pool:
+            out = pool.map(_score_pair, args, chunksize=max(1, len(args) // (procs * 8)))
+    return [o[0] for o in out], [o[1] for o in out]
