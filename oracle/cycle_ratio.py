@@ -77,6 +77,40 @@ def event_graph(prof, st, part: Partition) -> nx.DiGraph:
     return g
 
 
+def ceil_max_cycle_ratio(prof, st, part: Partition) -> int:
+    """ceil(lambda) without enumerating cycles: the smallest integer theta such that no cycle has
+    sum(durations) - theta * sum(tokens) > 0, found by binary search on theta with a Bellman-Ford
+    positive-cycle test (longest paths from a virtual source). Used by ``sim.time_ns`` when the
+    simulation's transient is too long to wait for (two near-equal cycle ratios)."""
+    g = event_graph(prof, st, part)
+    nodes = list(g.nodes)
+    pos = {v: i for i, v in enumerate(nodes)}
+    dur = [g.nodes[v]["dur"] for v in nodes]
+    edges = [(pos[u], pos[v], g.edges[u, v]["tokens"]) for u, v in g.edges]
+
+    def positive_cycle(theta: int) -> bool:
+        d = [0] * len(nodes)
+        for _ in range(len(nodes)):
+            changed = False
+            for (u, v, tok) in edges:
+                nd = d[u] + dur[v] - theta * tok
+                if nd > d[v]:
+                    d[v] = nd
+                    changed = True
+            if not changed:
+                return False
+        return True
+
+    lo, hi = -1, max(1, sum(dur))        # lambda <= sum of all durations (every cycle has >= 1 token)
+    while hi - lo > 1:
+        mid = (lo + hi) // 2
+        if positive_cycle(mid):
+            lo = mid
+        else:
+            hi = mid
+    return hi
+
+
 def max_cycle_ratio(prof, st, part: Partition) -> Fraction:
     g = event_graph(prof, st, part)
     best = None

@@ -24,6 +24,13 @@ from typing import Dict, List, Optional, Tuple
 from .model import U64_MAX, Ingredients, Partition, ceil_div, ingredients, parse_record
 
 MAX_ROUNDS = 10**6
+# time_ns waits this many rounds for the periodic regime before taking ceil(lambda) from the max
+# cycle ratio of the same event graph instead (cycle_ratio.ceil_max_cycle_ratio; reading R-2)
+TIME_NS_ROUNDS = 4000
+
+
+class NoPeriod(RuntimeError):
+    """The schedule did not become periodic within the allowed number of rounds."""
 
 
 class Schedule:
@@ -205,10 +212,11 @@ def compute_period(sched: Schedule, comp=None, max_rounds: int = MAX_ROUNDS) -> 
             return j0, j - j0, m - m0
         seen[key] = (j, m)
         j += 1
-    raise RuntimeError("no periodicity within %d rounds" % max_rounds)
+    raise NoPeriod("no periodicity within %d rounds" % max_rounds)
 
 
-def _allreduce_slope(sched: Schedule, s: int, j0: int, c: int, lam_c: Fraction) -> Fraction:
+def _allreduce_slope(sched: Schedule, s: int, j0: int, c: int, lam_c: Fraction,
+                     max_rounds: int = MAX_ROUNDS) -> Fraction:
     """Asymptotic slope of the all-reduce chain of stage s (SPEC §3).
 
     AR(k) = max(Bmax(k), AR(k-1)) + d. Let o(k) = AR(k) - Bmax(k) - d >= 0 (its backlog). Once the
@@ -231,14 +239,15 @@ def _allreduce_slope(sched: Schedule, s: int, j0: int, c: int, lam_c: Fraction) 
         if all(o(i) > 0 for i in range(k + 1, k + c + 1)) and o(k + c) > o(k):
             return Fraction(d)
         k += c
-        if k > MAX_ROUNDS:
-            raise RuntimeError("all-reduce chain did not settle")
+        if k > max_rounds:
+            raise NoPeriod("all-reduce chain did not settle within %d rounds" % max_rounds)
 
 
-def simulate(prof, st, part: Partition) -> Fraction:
-    """Exact steady-state time per mini-batch lambda (SPEC §3 'Result'), as a Fraction."""
+def simulate(prof, st, part: Partition, max_rounds: int = MAX_ROUNDS) -> Fraction:
+    """Exact steady-state time per mini-batch lambda (SPEC §3 'Result'), as a Fraction.
+    Raises NoPeriod if the periodic regime is not reached within max_rounds rounds."""
     sched = Schedule(ingredients(prof, st, part))
-    periods = [compute_period(sched, comp) for comp in sched.components()]
+    periods = [compute_period(sched, comp, max_rounds) for comp in sched.components()]
     lam = max(Fraction(D, c) for (_, c, D) in periods)
     if len(periods) == 1:
         j0, c, D = periods[0]
@@ -250,7 +259,7 @@ def simulate(prof, st, part: Partition) -> Fraction:
         j0, c, D = 0, 1, max(D for (_, _, D) in periods)
     for s in range(part.S):
         if len(part.W[s]) >= 2:
-            lam = max(lam, _allreduce_slope(sched, s, j0, c, Fraction(D, c)))
+            lam = max(lam, _allreduce_slope(sched, s, j0, c, Fraction(D, c), max_rounds))
     return lam
 
 
@@ -258,7 +267,11 @@ def time_ns(prof, st, part: Optional[Partition]) -> int:
     """T_ns = ceil(lambda) (reading C-7); UINT64_MAX for an invalid record."""
     if part is None:
         return U64_MAX
-    lam = simulate(prof, st, part)
+    try:
+        lam = simulate(prof, st, part, TIME_NS_ROUNDS)
+    except NoPeriod:
+        from .cycle_ratio import ceil_max_cycle_ratio
+        return ceil_max_cycle_ratio(prof, st, part)
     return ceil_div(lam.numerator, lam.denominator)
 
 

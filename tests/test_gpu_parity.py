@@ -30,7 +30,11 @@ def eng():
 
 def gpu_eval(eng, recs):
     from paper_conf_icpp_hulww24_b200 import as_u64
-    t = torch.from_numpy(np.asarray(recs, dtype=np.uint8).reshape(-1, 16))
+    if isinstance(recs, np.ndarray):
+        arr = np.ascontiguousarray(recs, dtype=np.uint8).reshape(-1, 16)
+    else:
+        arr = np.frombuffer(b"".join(bytes(r) for r in recs), dtype=np.uint8).reshape(-1, 16).copy()
+    t = torch.from_numpy(arr)
     out = as_u64(eng.eval_partitions(t))
     torch.cuda.synchronize()
     return [int(x) for x in out]

@@ -124,3 +124,42 @@ def test_toy_all_candidates_cycle_ratio():
     prof, st = W.toy(), W.toy_state()
     for p in candidates(8, 4, 1, 3):
         assert simulate(prof, st, p) == max_cycle_ratio(prof, st, p)
+
+
+def test_ceil_cycle_ratio_equals_simulation():
+    """The long-transient fallback of time_ns (Bellman-Ford on the event graph) equals ceil(lambda)
+    of the simulation wherever the simulation finishes."""
+    from oracle.cycle_ratio import ceil_max_cycle_ratio
+    from oracle.model import parse_record
+    rng = np.random.default_rng(41)
+    n = 0
+    for it in range(30):
+        L = int(rng.integers(1, 12))
+        N = int(rng.integers(1, 9))
+        prof = W.random_profile(L, rng, f_max=int(rng.choice([10, 10**6])), bytes_max=int(rng.choice([10, 10**7])))
+        st = W.random_state_small(prof, N, rng, tau_max=int(rng.choice([10, 10**5])))
+        for r in W.sample_records(L, N, 10, 2000 + it):
+            p = parse_record(bytes(r), L, N)
+            if p is None:
+                continue
+            lam = simulate(prof, st, p)
+            assert ceil_max_cycle_ratio(prof, st, p) == -(-lam.numerator // lam.denominator)
+            n += 1
+    assert n > 200
+
+
+def test_long_transient_uses_cycle_ratio():
+    """A GNMT-16 partition (trace state 11) whose bottleneck worker cycle (207,874,737 ns) beats another
+    stage's (207,821,004 ns) by 0.03%: the faster stage takes thousands of rounds to lock in. time_ns
+    does not wait (cap TIME_NS_ROUNDS) and takes ceil(lambda) from the event graph; the full
+    simulation, given enough rounds, agrees."""
+    from oracle.model import Partition
+    from oracle.sim import NoPeriod, time_ns
+    prof = W.profile("gnmt16")
+    st = W.trace_c3(prof)[-1]
+    part = Partition(5, [6, 8, 11, 15], [[0], [1], [2], [3], [4]])
+    with pytest.raises(NoPeriod):
+        simulate(prof, st, part, max_rounds=2000)
+    lam = simulate(prof, st, part, max_rounds=100_000)
+    assert lam == 207_874_737
+    assert time_ns(prof, st, part) == 207_874_737
