@@ -1,0 +1,405 @@
+#!/usr/bin/env python
+"""Benchmark of the AutoPipe cost-model hot path on B200 (contract: see DESIGN.md §Measurement).
+
+One step = one pass of the whole hot path over the headline workload of BASELINE.json: the
+96-layer, 8-stage exhaustive search (C(95,7) = 11,050,084,695 candidate partitions):
+  a1/a2  state ingest (prefix sums, link tables) from device-resident inputs,
+  a3-a8  unranking + enumeration + exact decision per candidate + argmin,
+  e      the NCCL min-loc across ranks (N > 1; each rank scans 1/N of the index space).
+`value` = candidates decided per second over all ranks (device time, max over ranks);
+`ms_per_step` = time to the exact optimum. `e2e` = the same step through the public API from host
+buffers (load_profile + set_state + search, result back on the host), wall clock, max over ranks.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--state a-nvlink|a-100g|b] [--impl ours|reference]
+Under torchrun, one process per GPU (RANK/LOCAL_RANK/WORLD_SIZE from the environment).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+from math import comb
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+METRIC = "partition evals/sec at 1/2/4/8 B200; time-to-exact-optimum, 96-layer 8-stage"
+UNIT = "evals/s"
+S_STAGES = 8
+TOTAL = comb(95, 7)
+PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
+# integer issue peak: 148 SMs x 4 SMSPs x 32 lanes x 1 instr/clk x sm_max_mhz
+SMS = 148
+LANES_PER_SM_CLK = 128
+
+
+def env_int(name, default):
+    try:
+        return int(os.environ.get(name, default))
+    except ValueError:
+        return default
+
+
+def cores() -> int:
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:
+        return os.cpu_count() or 1
+
+
+def cpu_model() -> str:
+    try:
+        with open("/proc/cpuinfo") as fh:
+            for line in fh:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+# ------------------------------------------------------------------------------------------------
+# clocks during the timed region (pynvml), per the profiling recipe's clocks line
+# ------------------------------------------------------------------------------------------------
+REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+           0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+           0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+
+class ClockSampler:
+    def __init__(self, index: int, period_s: float = 0.02):
+        self.samples, self.reasons, self.max_mhz = [], 0, None
+        self.period = period_s
+        self._stop = threading.Event()
+        self._th = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.nv = None
+
+    def _run(self):
+        nv = self.nv
+        get_r = getattr(nv, "nvmlDeviceGetCurrentClocksEventReasons", None) or \
+            getattr(nv, "nvmlDeviceGetCurrentClocksThrottleReasons")
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                self.reasons |= int(get_r(self.h))
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.nv is not None:
+            self._th = threading.Thread(target=self._run, daemon=True)
+            self._th.start()
+        return self
+
+    def __exit__(self, *a):
+        if self._th is not None:
+            self._stop.set()
+            self._th.join()
+
+    def summary(self):
+        if self.nv is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvml unavailable"]}
+        names = [v for k, v in REASONS.items() if self.reasons & k and k != 0x1]
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": names, "samples": len(self.samples)}
+
+
+# ------------------------------------------------------------------------------------------------
+# CPU baseline: the oracle, as it stands, on the host cores
+# ------------------------------------------------------------------------------------------------
+_PS = {}
+
+
+def _oracle_init(kind):
+    import workloads as W
+    _PS["prof"] = W.gpt96()
+    _PS["st"] = W.gpt_state(kind)
+
+
+def _oracle_score(rec: bytes) -> int:
+    from oracle.sim import score_record
+    return score_record(_PS["prof"], _PS["st"], rec)
+
+
+def oracle_sample(kind: str, n: int, seed: int):
+    import numpy as np
+    from oracle.enumerate import decode
+    from oracle.model import encode_partition
+    rng = np.random.default_rng(seed)
+    return [encode_partition(decode(96, 8, 8, 8, 0, int(i))) for i in rng.integers(0, TOTAL, size=n)]
+
+
+def oracle_throughput(kind: str, target_s: float = 12.0, seed: int = 12345):
+    """Score a bounded random sample of the 96-layer space with the oracle on every host core."""
+    import multiprocessing as mp
+    ncore = cores()
+    _oracle_init(kind)
+    probe = oracle_sample(kind, 16, seed + 1)
+    t0 = time.perf_counter()
+    for r in probe:
+        _oracle_score(r)
+    per = (time.perf_counter() - t0) / len(probe)  # s per candidate per core
+    n = max(ncore * 4, int(target_s / per * ncore))
+    recs = oracle_sample(kind, n, seed)
+    t0 = time.perf_counter()
+    with mp.get_context("fork").Pool(ncore, initializer=_oracle_init, initargs=(kind,)) as pool:
+        pool.map(_oracle_score, recs, chunksize=max(1, n // (ncore * 8)))
+    dt = time.perf_counter() - t0
+    return n / dt, n, dt, ncore
+
+
+def param_dp_time(kind: str):
+    import workloads as W
+    from oracle.param_dp import optimum
+    prof, st = W.gpt96(), W.gpt_state(kind)
+    t0 = time.perf_counter()
+    T, idx, _ = optimum(prof, st, S_STAGES, S_STAGES)
+    return time.perf_counter() - t0, T, idx
+
+
+def run_reference(args, rank: int, world: int):
+    """--impl reference: the oracle timed on the host cores, on this arm's workload and metric."""
+    if rank != 0:
+        return
+    import multiprocessing as mp
+    ncore = cores()
+    per_step = max(ncore * 8, args.ref_sample)
+    _oracle_init(args.state)
+    pool = mp.get_context("fork").Pool(ncore, initializer=_oracle_init, initargs=(args.state,))
+    times = []
+    for step in range(args.warmup + args.steps):
+        recs = oracle_sample(args.state, per_step, 5000 + step)
+        t0 = time.perf_counter()
+        pool.map(_oracle_score, recs, chunksize=max(1, per_step // (ncore * 8)))
+        if step >= args.warmup:
+            times.append(time.perf_counter() - t0)
+    pool.close()
+    total_s = sum(times)
+    value = per_step * args.steps / total_s
+    sample = "%d random candidates of the C(95,7) space per step (seeded), oracle event simulation" % per_step
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * total_s / args.steps,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int (python)",
+        "data": "synthetic", "config": config_block(args, world),
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": ncore, "kind": "oracle",
+                         "sample": sample, "cpu": cpu_model()},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def config_block(args, world):
+    return {"workload": "96-layer transformer profile (GPT-3 shaped, App. B.6), 8 stages, exhaustive "
+                        "C(95,7) cut sets; state %s" % args.state,
+            "layers": 96, "stages": S_STAGES, "candidates": TOTAL, "state": args.state,
+            "parallelism": "index-space shards x%d + NCCL min-loc" % world,
+            "l2": "flushed (256 MiB write) between timed steps"}
+
+
+# ------------------------------------------------------------------------------------------------
+# our arm
+# ------------------------------------------------------------------------------------------------
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--state", default="a-nvlink", choices=["a-nvlink", "a-100g", "b"])
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--ref-sample", type=int, default=0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--secondary", default="b", help="extra state measured in the same run ('' = none)")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    rank, world, local = env_int("RANK", 0), env_int("WORLD_SIZE", 1), env_int("LOCAL_RANK", 0)
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import __graft_entry__
+    __graft_entry__.build()
+    import workloads as W
+    from paper_conf_icpp_hulww24_b200 import Engine
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        dist.init_process_group("nccl", device_id=dev)
+    lo, hi = rank * TOTAL // world, (rank + 1) * TOTAL // world
+
+    def minloc(T, idx):
+        if world == 1:
+            return T, idx
+        t = torch.tensor([T if T < (1 << 63) else (1 << 63) - 1], dtype=torch.int64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MIN)
+        i = torch.tensor([idx if T == t.item() else (1 << 63) - 1], dtype=torch.int64, device=dev)
+        dist.all_reduce(i, op=dist.ReduceOp.MIN)
+        return int(t.item()), int(i.item())
+
+    def barrier():
+        if world > 1:
+            dist.barrier(device_ids=[local])
+
+    def max_over_ranks(x: float) -> float:
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device=dev)
+
+    def measure_state(kind: str):
+        prof, st = W.gpt96(), W.gpt_state(kind)
+        eng = Engine(local)
+        eng.load_profile(prof.O, prof.G, prof.P)
+        d_fp = torch.tensor(np.asarray(st.f, dtype=np.uint64).view(np.int64), device=dev)
+        d_bp = torch.tensor(np.asarray(st.b, dtype=np.uint64).view(np.int64), device=dev)
+        d_tau = torch.tensor(np.asarray(st.tau, dtype=np.uint64).view(np.int64), device=dev)
+        eng.set_timing(True)
+        stream = torch.cuda.current_stream(dev)
+
+        def step():
+            eng.set_state_device(d_fp, d_bp, d_tau)
+            r = eng.search_optimum(S_STAGES, S_STAGES, 0, lo, hi)
+            return r, minloc(r.time_ns, r.index)
+
+        for _ in range(args.warmup):
+            step()
+        torch.cuda.synchronize()
+        barrier()
+        launches0 = eng.kernel_launches
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+        kern_ms, results = [], []
+        with ClockSampler(local) as clk:
+            for k in range(args.steps):
+                flush.fill_(k)                     # L2 flush, outside the timed events
+                torch.cuda.synchronize()
+                ev[k][0].record(stream)
+                r, best = step()
+                ev[k][1].record(stream)
+                kern_ms.append(eng.last_search_ms)
+                results.append(best)
+            torch.cuda.synchronize()
+        barrier()
+        launches = eng.kernel_launches - launches0
+        step_ms = [a.elapsed_time(b) for a, b in ev]
+        rank_total_ms = sum(step_ms)
+        total_ms = max_over_ranks(rank_total_ms)
+        kern_avg = max_over_ranks(sum(kern_ms) / len(kern_ms))
+        assert all(x == results[0] for x in results), "non-deterministic optimum"
+        # e2e: the public API from host buffers (profile + state copied every step, result to host)
+        t_e2e = []
+        for k in range(args.steps):
+            flush.fill_(k)
+            torch.cuda.synchronize()
+            barrier()
+            t0 = time.perf_counter()
+            eng.load_profile(prof.O, prof.G, prof.P)
+            eng.set_state(st.f, st.b, st.tau)
+            r = eng.search_optimum(S_STAGES, S_STAGES, 0, lo, hi)
+            best_e2e = minloc(r.time_ns, r.index)
+            torch.cuda.synchronize()
+            t_e2e.append(time.perf_counter() - t0)
+        assert best_e2e == results[0]
+        e2e_s = max_over_ranks(sum(t_e2e))
+        int_path = eng.int_path
+        eng.close()
+        h2d = 3 * 96 * 8 + 2 * 8 * 96 * 8 + 8 * 8 * 8
+        return {"total_ms": total_ms, "ms_per_step": total_ms / args.steps, "kernel_ms": kern_avg,
+                "value": TOTAL * args.steps / (total_ms / 1000.0), "optimum": results[0],
+                "launches": launches, "clocks": clk.summary(), "int_path": int_path,
+                "e2e": {"value": TOTAL * args.steps / e2e_s, "unit": UNIT, "h2d_bytes_per_step": h2d,
+                        "d2h_bytes_per_step": 40, "ms_per_step": 1000 * e2e_s / args.steps}}
+
+    main_res = measure_state(args.state)
+    extra = {}
+    if args.secondary and args.secondary != args.state:
+        s2 = measure_state(args.secondary)
+        extra[args.secondary] = {"value": s2["value"], "ms_per_step": s2["ms_per_step"],
+                                 "int_path": s2["int_path"], "optimum_T_ns": s2["optimum"][0],
+                                 "optimum_index": s2["optimum"][1], "kernel_ms": s2["kernel_ms"],
+                                 "e2e_value": s2["e2e"]["value"], "clocks": s2["clocks"]}
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    # roofline of the dominant kernel (k_search_r1): integer issue bound
+    peaks = {}
+    try:
+        with open(PEAKS_PATH) as fh:
+            peaks = json.load(fh)
+    except OSError:
+        pass
+    sm_max = float(peaks.get("sm_max_mhz", 1965.0))
+    peak_ops = SMS * LANES_PER_SM_CLK * sm_max * 1e6 / 1e12       # Tops/s of thread-instructions
+    ops_per_cand = OPS_PER_CANDIDATE[main_res["int_path"]]
+    cands_per_rank = hi - lo
+    achieved = ops_per_cand * cands_per_rank / (main_res["kernel_ms"] / 1000.0) / 1e12
+    roofline = {"bound": "alu", "achieved": achieved, "peak": peak_ops, "unit": "Tops/s",
+                "frac": achieved / peak_ops, "traffic": None,
+                "kernel": "k_search_r1<8,%s>" % ("u32" if main_res["int_path"] == 32 else "u64"),
+                "ops_per_candidate": ops_per_cand,
+                "peak_source": "148 SMs x 128 lanes/clk x sm_max_mhz %.0f (MEASURED_PEAKS.json)" % sm_max,
+                "kernel_ms": main_res["kernel_ms"]}
+
+    cpu = None
+    if world == 1 and not args.no_cpu_baseline:
+        v, n, dt, nc = oracle_throughput(args.state)
+        dp_s, dpT, dpI = param_dp_time(args.state)
+        assert (dpT, dpI) == tuple(main_res["optimum"]), "GPU optimum differs from the oracle's parametric DP"
+        cpu = {"value": v, "unit": UNIT, "cores": nc, "kind": "oracle",
+               "sample": "%d seeded random candidates of the C(95,7) space, event simulation, %.1f s" % (n, dt),
+               "cpu": cpu_model(),
+               "extrapolated_exhaustive_s": TOTAL / v,
+               "param_dp_time_to_optimum_s_1core": dp_s}
+
+    line = {
+        "metric": METRIC, "value": main_res["value"], "unit": UNIT, "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": main_res["ms_per_step"],
+        "time_to_optimum_ms": main_res["ms_per_step"],
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+        "dtype": "u32" if main_res["int_path"] == 32 else "u64", "data": "synthetic",
+        "config": config_block(args, world),
+        "optimum": {"T_ns": main_res["optimum"][0], "index": main_res["optimum"][1]},
+        "gpu_launches": main_res["launches"],
+        "clocks": main_res["clocks"],
+        "e2e": main_res["e2e"],
+        "roofline": roofline,
+        "cpu_baseline": cpu,
+        "secondary_states": extra,
+    }
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+# integer thread-instructions per candidate that the exact decision needs at minimum, per path
+# (one broadcast 128-bit column load, three compares, their AND and the loop
+# counter, amortised over a 4-wide unrolled step: 6 for 32-bit values; 64-bit compares take two
+# instructions each: 9)
+OPS_PER_CANDIDATE = {32: 6, 64: 9}
+
+if __name__ == "__main__":
+    main()

@@ -100,6 +100,14 @@ int autopipe_load_profile(autopipe_ctx *ctx, uint32_t L, const uint64_t *act_byt
 int autopipe_set_state(autopipe_ctx *ctx, uint32_t N, const uint64_t *fp_ns, const uint64_t *bp_ns,
                        const uint64_t *link_fs_per_byte, void *stream);
 
+/* Same as autopipe_set_state, with the three arrays in DEVICE memory (e.g. written by an on-GPU
+ * profiler): nothing is copied from the host. The overflow rules are checked by the state kernel on
+ * the device; a violating state makes every later score UINT64_MAX and the next synchronous call
+ * (autopipe_search_optimum, autopipe_int_path) reports AUTOPIPE_E_OVERFLOW. The arrays must stay
+ * valid until the enqueued kernel has run. Async on `stream`. */
+int autopipe_set_state_device(autopipe_ctx *ctx, uint32_t N, const uint64_t *d_fp_ns, const uint64_t *d_bp_ns,
+                              const uint64_t *d_link_fs_per_byte, void *stream);
+
 /* Batched scoring of explicit partitions (device pointers; async on `stream`):
  *   d_parts[count]    input records (any disjoint worker sets, reading C-11);
  *   d_time_ns[count]  output T_ns per record; an invalid record (SPEC.md §2) gets UINT64_MAX and
@@ -143,6 +151,14 @@ int autopipe_int_path(const autopipe_ctx *ctx);
 
 /* Number of kernels this context has launched so far (for launch accounting in benchmarks). */
 uint64_t autopipe_kernel_launches(const autopipe_ctx *ctx);
+
+/* Enable (1) / disable (0) device timing of the search kernels: CUDA events recorded on the launch
+ * stream around the enumeration kernels of each autopipe_search_optimum (excluding the final
+ * reduction and the result copy). */
+int autopipe_set_timing(autopipe_ctx *ctx, int enable);
+
+/* Device milliseconds of the enumeration kernels of the last timed search (-1 if none). */
+double autopipe_last_search_ms(const autopipe_ctx *ctx);
 
 #ifdef __cplusplus
 }

@@ -25,9 +25,10 @@ ERROR_NAMES = {AUTOPIPE_E_INVAL: "AUTOPIPE_E_INVAL", AUTOPIPE_E_STATE: "AUTOPIPE
 
 # every symbol include/autopipe.h declares
 SYMBOLS = ["autopipe_create", "autopipe_destroy", "autopipe_last_error", "autopipe_load_profile",
-           "autopipe_set_state", "autopipe_eval_partitions", "autopipe_search_optimum",
+           "autopipe_set_state", "autopipe_set_state_device", "autopipe_eval_partitions", "autopipe_search_optimum",
            "autopipe_rollout_rewards", "autopipe_count_candidates", "autopipe_decode_index",
-           "autopipe_int_path", "autopipe_kernel_launches"]
+           "autopipe_int_path", "autopipe_kernel_launches", "autopipe_set_timing",
+           "autopipe_last_search_ms"]
 
 
 class Partition(ctypes.Structure):
@@ -63,6 +64,7 @@ def _load():
         "autopipe_last_error": (ctypes.c_char_p, [P]),
         "autopipe_load_profile": (i32, [P, u32, pu64, pu64, pu64]),
         "autopipe_set_state": (i32, [P, u32, pu64, pu64, pu64, P]),
+        "autopipe_set_state_device": (i32, [P, u32, P, P, P, P]),
         "autopipe_eval_partitions": (i32, [P, P, u64, P, P]),
         "autopipe_search_optimum": (i32, [P, u32, u32, u32, u64, u64, ctypes.POINTER(Result), P]),
         "autopipe_rollout_rewards": (i32, [P, P, u64, ctypes.POINTER(Partition), P, P, P]),
@@ -70,6 +72,8 @@ def _load():
         "autopipe_decode_index": (i32, [P, u32, u32, u32, u64, ctypes.POINTER(Partition)]),
         "autopipe_int_path": (i32, [P]),
         "autopipe_kernel_launches": (u64, [P]),
+        "autopipe_set_timing": (i32, [P, i32]),
+        "autopipe_last_search_ms": (ctypes.c_double, [P]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(lib, name)

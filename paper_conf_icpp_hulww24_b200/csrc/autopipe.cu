@@ -23,13 +23,14 @@ struct autopipe_ctx {
   int device = 0, sms = 148;
   char err[512] = {0};
   bool has_profile = false, has_state = false;
+  bool state_on_device = false;  // last state came from device pointers: status not yet read
   u32 L = 0, N = 0;
   int path32 = 0;
   u64 launches = 0;
   u64 maxOG = 0, sumP = 0;
   DevTables tab{};
   // device buffers
-  u64 *d_raw = nullptr;      // fp [8*255] | bp [8*255] | P [255]
+  u64 *d_raw = nullptr;      // fp [8*255] | bp [8*255] | P [255] | tau [64]
   u64 *d_tables = nullptr;   // all DevTables arrays
   BlockOut *d_blocks = nullptr;
   ResultDev *d_result = nullptr;
@@ -38,7 +39,12 @@ struct autopipe_ctx {
   // pinned host staging
   u64 *h_stage = nullptr;    // fp | bp | tau(64)
   ResultDev *h_result = nullptr;
+  u64 *h_status = nullptr;   // pinned copy of the device status word
   u64 binom[BINOM_N][BINOM_K];
+  // optional device timing of the search kernels (autopipe_set_timing)
+  bool timing = false;
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  double last_search_ms = -1.0;
 };
 
 static char g_create_err[256] = "";
@@ -100,16 +106,17 @@ extern "C" int autopipe_create(int cuda_device, autopipe_ctx **out) {
   upload_binomials(c->binom);
   // device tables, sized for the limits (L = 255, N = 8): a few hundred KB
   const size_t Lp1 = MAXL + 1, NL = (size_t)MAXN * Lp1;
-  const size_t words = 3 * NL + Lp1 + 2 * MAXL + 64 + 2 * 7 * MAXL;
+  const size_t words = 3 * NL + Lp1 + 2 * MAXL + 64 + 2 * 7 * MAXL + 2;
   const size_t words32 = NL + 2 * 7 * MAXL;
   e = cudaMalloc(&c->d_tables, words * 8 + words32 * 4 + 64);
-  if (e == cudaSuccess) e = cudaMalloc(&c->d_raw, (2 * MAXN * MAXL + MAXL) * 8);
+  if (e == cudaSuccess) e = cudaMalloc(&c->d_raw, (2 * MAXN * MAXL + MAXL + 64) * 8);
   if (e == cudaSuccess) e = cudaMalloc(&c->d_blocks, sizeof(BlockOut) * MAX_BLOCKS);
   if (e == cudaSuccess) e = cudaMalloc(&c->d_result, sizeof(ResultDev));
   c->work_bytes = 1 << 20;
   if (e == cudaSuccess) e = cudaMalloc(&c->d_work, c->work_bytes);
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_stage, (2 * MAXN * MAXL + 64) * 8);
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_result, sizeof(ResultDev));
+  if (e == cudaSuccess) e = cudaMallocHost(&c->h_status, 2 * sizeof(u64));
   if (e != cudaSuccess) {
     snprintf(g_create_err, sizeof(g_create_err), "allocation: %s", cudaGetErrorString(e));
     autopipe_destroy(c);
@@ -125,6 +132,7 @@ extern "C" int autopipe_create(int cuda_device, autopipe_ctx **out) {
   c->tab.tau = p; p += 64;
   c->tab.Z = p; p += 7 * MAXL;
   c->tab.LM = p; p += 7 * MAXL;
+  c->tab.status = p; p += 2;
   u32 *q = (u32 *)p;
   c->tab.PC32 = q; q += NL;
   c->tab.Z32 = q; q += 7 * MAXL;
@@ -151,6 +159,9 @@ extern "C" void autopipe_destroy(autopipe_ctx *c) {
     if (c->d_work) cudaFree(c->d_work);
     if (c->h_stage) cudaFreeHost(c->h_stage);
     if (c->h_result) cudaFreeHost(c->h_result);
+    if (c->h_status) cudaFreeHost(c->h_status);
+    if (c->ev0) cudaEventDestroy(c->ev0);
+    if (c->ev1) cudaEventDestroy(c->ev1);
   }
   delete c;
 }
@@ -226,22 +237,59 @@ extern "C" int autopipe_set_state(autopipe_ctx *c, uint32_t N, const uint64_t *f
   u64 *hf = c->h_stage, *hb = hf + MAXN * MAXL, *ht = hb + MAXN * MAXL;
   memcpy(hf, fp, (size_t)N * L * 8);
   memcpy(hb, bp, (size_t)N * L * 8);
-  for (int u = 0; u < 8; ++u)
-    for (int v = 0; v < 8; ++v) ht[u * 8 + v] = (u < (int)N && v < (int)N && u != v) ? tau[u * N + v] : 0;
-  e = cudaMemcpyAsync(c->d_raw, hf, (size_t)N * L * 8, cudaMemcpyHostToDevice, st);
-  if (e == cudaSuccess)
-    e = cudaMemcpyAsync(c->d_raw + MAXN * MAXL, hb, (size_t)N * L * 8, cudaMemcpyHostToDevice, st);
-  if (e == cudaSuccess) e = cudaMemcpyAsync(c->tab.tau, ht, 64 * 8, cudaMemcpyHostToDevice, st);
+  memcpy(ht, tau, (size_t)N * N * 8);
+  u64 *rf = c->d_raw, *rb = rf + MAXN * MAXL, *rP = rb + MAXN * MAXL, *rt = rP + MAXL;
+  e = cudaMemcpyAsync(rf, hf, (size_t)N * L * 8, cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(rb, hb, (size_t)N * L * 8, cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(rt, ht, (size_t)N * N * 8, cudaMemcpyHostToDevice, st);
   if (e != cudaSuccess) return cuda_fail(c, e, "set_state copy");
   c->tab.L = L;
   c->tab.N = N;
   c->tab.Lp1 = L + 1;
   c->N = N;
-  c->launches += launch_build_state(c->tab, c->d_raw, c->d_raw + MAXN * MAXL, c->d_raw + 2 * MAXN * MAXL,
-                                    c->path32, st);
+  c->launches += launch_build_state(c->tab, rf, rb, rP, rt, c->sumP, st);
   e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "state kernel launch");
   c->has_state = true;
+  c->state_on_device = false;
+  return AUTOPIPE_OK;
+}
+
+extern "C" int autopipe_set_state_device(autopipe_ctx *c, uint32_t N, const uint64_t *d_fp, const uint64_t *d_bp,
+                                         const uint64_t *d_tau, void *stream) {
+  if (!c) return AUTOPIPE_E_INVAL;
+  c->err[0] = 0;
+  if (!c->has_profile) return fail(c, AUTOPIPE_E_STATE, "set_state before load_profile");
+  if (N < 1 || N > MAXN) return fail(c, AUTOPIPE_E_INVAL, "N = %u outside [1, 8]", N);
+  if (!d_fp || !d_bp || !d_tau) return fail(c, AUTOPIPE_E_INVAL, "NULL state array");
+  DeviceGuard dg(c->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  c->tab.L = c->L;
+  c->tab.N = N;
+  c->tab.Lp1 = c->L + 1;
+  c->N = N;
+  const u64 *rP = c->d_raw + 2 * MAXN * MAXL;
+  c->launches += launch_build_state(c->tab, (const u64 *)d_fp, (const u64 *)d_bp, rP, (const u64 *)d_tau, c->sumP, st);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(c, e, "state kernel launch");
+  c->has_state = true;
+  c->state_on_device = true;  // overflow / path status is read from the device when first needed
+  return AUTOPIPE_OK;
+}
+
+// For a state given in device memory: fetch the status the state kernel computed (synchronises
+// `stream`). Returns AUTOPIPE_E_OVERFLOW if the state violates SPEC.md §7.
+static int sync_status(autopipe_ctx *c, cudaStream_t st) {
+  if (!c->state_on_device) return AUTOPIPE_OK;
+  cudaError_t e = cudaMemcpyAsync(c->h_status, c->tab.status, 2 * sizeof(u64), cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  if (e != cudaSuccess) return cuda_fail(c, e, "state status");
+  c->state_on_device = false;
+  c->path32 = (c->h_status[0] & 2) ? 1 : 0;
+  if (c->h_status[0] & 1) {
+    c->has_state = false;
+    return fail(c, AUTOPIPE_E_OVERFLOW, "device state: bytes * tau reaches 2^64 or modelled times reach 2^59 ns");
+  }
   return AUTOPIPE_OK;
 }
 
@@ -366,6 +414,9 @@ extern "C" int autopipe_search_optimum(autopipe_ctx *c, uint32_t s_min, uint32_t
   if (begin >= end) return AUTOPIPE_OK;
   DeviceGuard dg(c->device);
   cudaStream_t st = (cudaStream_t)stream;
+  rc = sync_status(c, st);
+  if (rc) return rc;
+  if (c->timing) cudaEventRecord(c->ev0, st);
   int used = 0;
   // Split [begin, end) into the r = 1 block of each S (rho = 0: fast kernel) and the rest (generic).
   u64 cur = begin;
@@ -401,12 +452,18 @@ extern "C" int autopipe_search_optimum(autopipe_ctx *c, uint32_t s_min, uint32_t
       used = 1;
     }
   }
+  if (c->timing) cudaEventRecord(c->ev1, st);
   c->launches += launch_finalize(c->d_blocks, used, sp, c->d_result, st);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "search kernel launch");
   e = cudaMemcpyAsync(c->h_result, c->d_result, sizeof(ResultDev), cudaMemcpyDeviceToHost, st);
   if (e == cudaSuccess) e = cudaStreamSynchronize(st);
   if (e != cudaSuccess) return cuda_fail(c, e, "search");
+  if (c->timing) {
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, c->ev0, c->ev1);
+    c->last_search_ms = ms;
+  }
   h_out->time_ns = c->h_result->time_ns;
   h_out->index = c->h_result->index;
   h_out->evaluated = c->h_result->evaluated;
@@ -460,8 +517,27 @@ extern "C" int autopipe_rollout_rewards(autopipe_ctx *c, const autopipe_partitio
   return AUTOPIPE_OK;
 }
 
-extern "C" int autopipe_int_path(const autopipe_ctx *c) {
-  return (c && c->has_state) ? (c->path32 ? 32 : 64) : 0;
+extern "C" int autopipe_int_path(const autopipe_ctx *cc) {
+  autopipe_ctx *c = const_cast<autopipe_ctx *>(cc);
+  if (!c || !c->has_state) return 0;
+  DeviceGuard dg(c->device);
+  cudaDeviceSynchronize();
+  if (sync_status(c, nullptr)) return 0;
+  return c->path32 ? 32 : 64;
 }
 
 extern "C" uint64_t autopipe_kernel_launches(const autopipe_ctx *c) { return c ? c->launches : 0; }
+
+extern "C" int autopipe_set_timing(autopipe_ctx *c, int enable) {
+  if (!c) return AUTOPIPE_E_INVAL;
+  DeviceGuard dg(c->device);
+  if (enable && !c->ev0) {
+    cudaError_t e = cudaEventCreate(&c->ev0);
+    if (e == cudaSuccess) e = cudaEventCreate(&c->ev1);
+    if (e != cudaSuccess) return cuda_fail(c, e, "event create");
+  }
+  c->timing = enable != 0;
+  return AUTOPIPE_OK;
+}
+
+extern "C" double autopipe_last_search_ms(const autopipe_ctx *c) { return c ? c->last_search_ms : -1.0; }

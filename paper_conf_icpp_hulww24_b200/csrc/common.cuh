@@ -35,6 +35,7 @@ struct DevTables {
   u32 *PC32;  // [N][L+1]  32-bit copies for the 32-bit search path (valid iff path32)
   u32 *Z32;   // [7][L]
   u32 *LM32;  // [7][L]
+  u64 *status; // [2] written by the state kernel: [0] bit0 = overflow, bit1 = 32-bit path; [1] = bound
 };
 
 __host__ __device__ __forceinline__ u64 umax(u64 a, u64 b) { return a > b ? a : b; }

@@ -21,7 +21,7 @@ struct ResultDev {
 };
 
 // Each launcher returns the number of kernels it enqueued (for launch accounting).
-int launch_build_state(const DevTables &g, const u64 *fp, const u64 *bp, const u64 *P, int path32,
+int launch_build_state(const DevTables &g, const u64 *fp, const u64 *bp, const u64 *P, const u64 *tau, u64 sumP,
                        cudaStream_t st);
 int launch_eval(const DevTables &g, const void *recs, u64 count, u64 *out_t, u64 *out_sw,
                 const int *cur_S, const u64 *cur_cuts, const u64 *cur_masks, int sms, cudaStream_t st);

@@ -24,6 +24,8 @@ __global__ void __launch_bounds__(256) k_eval(DevTables g, const uint4 *__restri
   extern __shared__ u64 sm[];
   const SmemTab t = stage_tables(g, sm);
   const int L = t.L, N = (int)g.N;
+  // a state that failed the device-side overflow check (set_state_device) scores nothing
+  const bool overflow = (g.status[0] & 1ull) != 0;
   const u64 stride = (u64)gridDim.x * blockDim.x;
   for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < count; i += stride) {
     const uint4 r = __ldg(recs + i);
@@ -31,7 +33,7 @@ __global__ void __launch_bounds__(256) k_eval(DevTables g, const uint4 *__restri
     int S;
     u64 cuts, masks;
     u64 T = U64MAX, sw = U64MAX;
-    if (decode_record(lo, hi, L, N, S, cuts, masks)) {
+    if (!overflow && decode_record(lo, hi, L, N, S, cuts, masks)) {
       T = eval_closed_form(t, S, cuts, masks);
       if (ROLLOUT) sw = switch_bytes(t, S, cuts, masks, cur.S, cur.cuts, cur.masks);
     }

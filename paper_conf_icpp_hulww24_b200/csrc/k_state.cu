@@ -1,16 +1,18 @@
 // k_state.cu — rows a1 and a2: state ingest (per-worker prefix sums of f, b, f+b and of the weight
-// bytes) and the r = 1 link tables, built on the device after every autopipe_set_state.
+// bytes), the r = 1 link tables, and the device-side overflow / integer-path check, built on the
+// device after every autopipe_set_state / autopipe_set_state_device.
 //
 // Table 1 inputs: FP_ij, BP_ij (N x L ns), P_i (L bytes), O_i, G_i (L bytes) and
-// the per-link inverse bandwidth (reading C-5). One launch, two roles:
+// the per-link inverse bandwidth (reading C-5). One launch, four roles by warp:
 //   warps 0 .. 3N   : one row each — warp-shuffle inclusive scan (__shfl_up_sync) over 32-element
 //                     chunks with a running carry, written as an exclusive prefix of L + 1 entries
-//                     (rows: PF[w], PB[w], PC[w] = prefix of f + b, and PP);
+//                     (rows: PF[w], PB[w], PC[w] = prefix of f + b, and PP), plus 32-bit copies of PC;
+//   warp 3N + 1     : copies tau (N x N) into the padded 8 x 8 table and computes the overflow /
+//                     32-bit-path status of SPEC.md §7 (used when the inputs came from device memory);
 //   remaining warps : link tables Z[s][l] = cf + cb and LM[s][l] = max(cf, cb) for the boundary
 //                     between worker s and s + 1 at a cut after layer l, with
 //                     cf = ceil(O[l] * tau[s][s+1] / 1e6) and cb = ceil(G[l+1] * tau[s+1][s] / 1e6)
-//                     (forward activation / backward input gradient, reading C-6).
-// 32-bit copies of PC, Z, LM are written when the host selected the 32-bit search path.
+//                     (forward activation / backward input gradient, reading C-6), and 32-bit copies.
 #include "common.cuh"
 #include "internal.h"
 
@@ -25,9 +27,15 @@ __device__ __forceinline__ u64 warp_incl_scan(u64 v, int lane) {
   return v;
 }
 
-// raw: fp [N][L], bp [N][L], P [L]
+__device__ __forceinline__ u64 warp_max(u64 v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = umax(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+
+// fp, bp: [N][L] ns; P: [L] bytes; tau: [N][N] fs/B (any device memory)
 __global__ void k_build_state(DevTables g, const u64 *__restrict__ fp, const u64 *__restrict__ bp,
-                              const u64 *__restrict__ P, int path32, int scan_warps) {
+                              const u64 *__restrict__ P, const u64 *__restrict__ tau, u64 sumP, int scan_warps) {
   const int lane = threadIdx.x & 31;
   const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;  // global warp id
   const int L = (int)g.L, N = (int)g.N, Lp1 = (int)g.Lp1;
@@ -44,7 +52,7 @@ __global__ void k_build_state(DevTables g, const u64 *__restrict__ fp, const u64
       dst = g.PB + w * Lp1;
     } else {
       dst = g.PC + w * Lp1;
-      if (path32) dst32 = g.PC32 + w * Lp1;
+      dst32 = g.PC32 + w * Lp1;
     }
     u64 carry = 0;
     if (lane == 0) {
@@ -69,29 +77,77 @@ __global__ void k_build_state(DevTables g, const u64 *__restrict__ fp, const u64
     }
     return;
   }
+  if (gw == scan_warps) {
+    // padded tau and the status word (SPEC.md §7 overflow rule, 32-bit search path)
+    for (int i = lane; i < 64; i += 32) {
+      const int u = i >> 3, v = i & 7;
+      g.tau[i] = (u < N && v < N && u != v) ? tau[u * N + v] : 0ull;
+    }
+    u64 mt = 0;
+    for (int i = lane; i < N * N; i += 32)
+      if (i / N != i % N) mt = umax(mt, tau[i]);
+    const u64 maxTau = warp_max(mt);
+    u64 mog = 0;
+    for (int l = lane; l < L; l += 32) mog = umax(mog, umax(g.O[l], g.G[l]));
+    const u64 maxOG = warp_max(mog);
+    // sum over layers of max over workers of (f + b), with overflow detection
+    bool ovf = false;
+    u64 part = 0;
+    for (int l = lane; l < L; l += 32) {
+      u64 m = 0;
+      for (int w = 0; w < N; ++w) {
+        const u64 a = fp[w * L + l], b = bp[w * L + l];
+        if (a >= (1ull << 59) || b >= (1ull << 59)) ovf = true;  // then the bound fails anyway
+        m = umax(m, a + b);
+      }
+      part = (part >= (1ull << 59) || m >= (1ull << 60)) ? (1ull << 59) : part + m;  // saturate
+    }
+    u64 sumMax = part;  // every lane's part <= 2^59 + 2^60, so the 32-lane sum cannot wrap
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) sumMax += __shfl_xor_sync(0xffffffffu, sumMax, o);
+    ovf = __any_sync(0xffffffffu, ovf) || sumMax >= (1ull << 59);
+    if (lane == 0) {
+      const u64 maxBytes = umax(maxOG, sumP);
+      // bytes * tau + 999999 < 2^64
+      const u64 hi = __umul64hi(maxBytes, maxTau), lo = maxBytes * maxTau;
+      if (hi != 0 || lo + 999999ull < lo) ovf = true;
+      const u64 maxX = ovf ? 0 : (lo + 999999ull) / 1000000ull;
+      const u64 maxXog = (maxOG * maxTau + 999999ull) / 1000000ull;  // <= maxX
+      // bound = sumMax + 16 + 28 maxX < 2^59 (sumMax < 2^59 and maxX < 2^55 here: no wrap)
+      u64 bound = ~0ull, bound32 = ~0ull;
+      if (maxX >= (1ull << 55)) ovf = true;
+      if (!ovf) {
+        bound = sumMax + 16 + 28 * maxX;
+        bound32 = sumMax + 16 + 14 * maxXog;
+      }
+      if (bound >= (1ull << 59)) ovf = true;
+      const u64 path32 = (!ovf && bound32 < 0xFFFFFFF0ull) ? 2ull : 0ull;
+      g.status[0] = (ovf ? 1ull : 0ull) | path32;
+      g.status[1] = bound;
+    }
+    return;
+  }
   // link tables: one thread per (s, l), s in [0, N-2], l in [0, L-2]
-  const int t = (blockIdx.x * blockDim.x + threadIdx.x) - scan_warps * 32;
+  const int t = (blockIdx.x * blockDim.x + threadIdx.x) - (scan_warps + 1) * 32;
   const int per = (L > 1) ? L - 1 : 0;
-  if (per == 0 || t >= (N - 1) * per) return;
+  if (t < 0 || per == 0 || t >= (N - 1) * per) return;
   const int s = t / per, l = t % per;
-  const u64 cf = xfer(g.O[l], g.tau[s * 8 + s + 1]);
-  const u64 cb = xfer(g.G[l + 1], g.tau[(s + 1) * 8 + s]);
+  const u64 cf = xfer(g.O[l], tau[s * N + s + 1]);
+  const u64 cb = xfer(g.G[l + 1], tau[(s + 1) * N + s]);
   g.Z[s * L + l] = cf + cb;
   g.LM[s * L + l] = umax(cf, cb);
-  if (path32) {
-    g.Z32[s * L + l] = (u32)(cf + cb);
-    g.LM32[s * L + l] = (u32)umax(cf, cb);
-  }
+  g.Z32[s * L + l] = (u32)(cf + cb);
+  g.LM32[s * L + l] = (u32)umax(cf, cb);
 }
 
-int launch_build_state(const DevTables &g, const u64 *fp, const u64 *bp, const u64 *P, int path32,
+int launch_build_state(const DevTables &g, const u64 *fp, const u64 *bp, const u64 *P, const u64 *tau, u64 sumP,
                        cudaStream_t st) {
   const int scan_warps = 3 * (int)g.N + 1;
   const int links = ((int)g.N - 1) * ((int)g.L > 1 ? (int)g.L - 1 : 0);
-  const int threads = scan_warps * 32 + (links > 0 ? links : 0);
+  const int threads = (scan_warps + 1) * 32 + (links > 0 ? links : 0);
   const int bs = 256;
   const int blocks = (threads + bs - 1) / bs;
-  k_build_state<<<blocks, bs, 0, st>>>(g, fp, bp, P, path32, scan_warps);
+  k_build_state<<<blocks, bs, 0, st>>>(g, fp, bp, P, tau, sumP, scan_warps);
   return 1;
 }
 

@@ -102,6 +102,19 @@ class Engine:
         self._check(lib.autopipe_set_state(self._h, N, _ptr(fa), _ptr(ba), _ptr(ta), self._stream(stream)))
         self.N = N
 
+    def set_state_device(self, fp: torch.Tensor, bp: torch.Tensor, tau: torch.Tensor, stream=None) -> None:
+        """State from device tensors (int64/uint64 bits, shapes [N, L], [N, L], [N, N]); no host copy."""
+        for t in (fp, bp, tau):
+            if t.device != self.device or t.dtype not in (torch.int64, torch.uint64) or not t.is_contiguous():
+                raise ValueError("state tensors must be contiguous 64-bit tensors on the engine's device")
+        N = int(fp.shape[0])
+        if fp.numel() != N * self.L or bp.numel() != N * self.L or tau.numel() != N * N:
+            raise ValueError("expected fp, bp of shape [N, L] and tau of shape [N, N]")
+        self._check(lib.autopipe_set_state_device(self._h, N, ctypes.c_void_p(fp.data_ptr()),
+                                                  ctypes.c_void_p(bp.data_ptr()),
+                                                  ctypes.c_void_p(tau.data_ptr()), self._stream(stream)))
+        self.N = N
+
     def load(self, profile, state, stream=None) -> None:
         """Convenience: load_profile + set_state from workloads.Profile / workloads.State objects."""
         self.load_profile(profile.O, profile.G, profile.P)
@@ -167,6 +180,14 @@ class Engine:
     @property
     def int_path(self) -> int:
         return int(lib.autopipe_int_path(self._h))
+
+    def set_timing(self, enable: bool = True) -> None:
+        self._check(lib.autopipe_set_timing(self._h, 1 if enable else 0))
+
+    @property
+    def last_search_ms(self) -> float:
+        """Device time of the enumeration kernels of the last search (needs set_timing(True))."""
+        return float(lib.autopipe_last_search_ms(self._h))
 
     @property
     def kernel_launches(self) -> int:
