@@ -9,7 +9,8 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libautopipe.so")
+# AUTOPIPE_LIB may name another in-tree build of the same library (kernel-variant experiments)
+LIB_PATH = os.environ.get("AUTOPIPE_LIB") or os.path.join(_HERE, "libautopipe.so")
 
 AUTOPIPE_OK = 0
 AUTOPIPE_E_INVAL = -1

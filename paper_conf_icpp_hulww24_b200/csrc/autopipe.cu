@@ -426,7 +426,7 @@ extern "C" int autopipe_search_optimum(autopipe_ctx *c, uint32_t s_min, uint32_t
     const u64 lo = cur, hi = end < bhi ? end : bhi;
     // candidates with rho = 0 are [blo, blo + ncut); rho = 0 is all-r=1 iff the first composition
     // (R = 1..S) has every r_s = 1, which holds for the default flag and for USE_ALL when N = S.
-    const bool r1 = S >= 3 && (!(flags & AUTOPIPE_USE_ALL_WORKERS) || (int)c->N == S);
+    const bool r1 = S >= 5 && (!(flags & AUTOPIPE_USE_ALL_WORKERS) || (int)c->N == S);
     const u64 r1hi = blo + sp.ncut[S];
     if (r1 && lo < r1hi) {
       const u64 a = lo, b = hi < r1hi ? hi : r1hi;

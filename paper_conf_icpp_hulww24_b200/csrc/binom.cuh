@@ -54,4 +54,37 @@ __device__ __forceinline__ bool lex_next_packed(u64 &packed, int k, int n) {
   return false;
 }
 
+// The same two maps against a binomial table held in shared memory (row n = C(n, 0..8)): the hot
+// kernel unranks once per lane and task, so it avoids the serialised divergent reads of __constant__.
+// Unranking uses the colex dual: r' = C(n,k) - 1 - r = sum_i C(d_i, k-i), d_i = n-1-c_i, each d_i
+// found by a fixed-length binary search (no data-dependent trip count, no divergence).
+__device__ __forceinline__ u64 lex_rank_smem(u64 packed, int k, int n, const u64 *B) {
+  u64 s = 0;
+  for (int i = 0; i < k; ++i) {
+    const int c = (int)((packed >> (8 * i)) & 0xFF);
+    s += B[(n - 1 - c) * BINOM_K + (k - i)];
+  }
+  return B[n * BINOM_K + k] - 1 - s;
+}
+
+__device__ __forceinline__ u64 lex_unrank_smem(u64 rank, int k, int n, const u64 *B) {
+  u64 rp = B[n * BINOM_K + k] - 1 - rank;
+  u64 out = 0;
+  int hi = n - 1;  // d_i < d_{i-1}
+  for (int i = 0; i < k; ++i) {
+    const int m = k - i;
+    // largest d in [0, hi] with C(d, m) <= rp (C(d, m) is non-decreasing in d)
+    int lo = 0, h = hi;
+    while (lo < h) {
+      const int mid = (lo + h + 1) >> 1;
+      if (B[mid * BINOM_K + m] <= rp) lo = mid;
+      else h = mid - 1;
+    }
+    rp -= B[lo * BINOM_K + m];
+    out |= (u64)(n - 1 - lo) << (8 * i);
+    hi = lo - 1;
+  }
+  return out;
+}
+
 }  // namespace ap

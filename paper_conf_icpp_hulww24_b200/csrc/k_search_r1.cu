@@ -1,65 +1,73 @@
 // k_search_r1.cu — the hot kernel: exhaustive search over the block of the space in which every
-// stage runs on one worker (composition R = 1..S, rho = 0 in SPEC.md §5). For the 96-layer, 8-stage
-// workload this block IS the space: C(95,7) = 11,050,084,695 cut sets (rows a3-a8).
+// stage runs on one worker (composition R = 1..S, rho = 0 in SPEC.md §5), S in [5, 8]. For the
+// 96-layer, 8-stage workload this block IS the space: C(95,7) = 11,050,084,695 cut sets
+// (rows a3-a8). Smaller S (tiny spaces) go through the generic kernel.
 //
 // What each candidate costs. With r = 1 the closed form of SPEC.md §4 is
-//   T = max( c_s, lm_s, ceil(W(s,t) / (t-s+1)) ),  W(s,t) = sum_{u=s..t} c_u + sum_{u=s..t-1} z_u,
-// (c_s = stage cost on its worker, z_s = cf_s + cb_s, lm_s = max(cf_s, cb_s)). The search only needs,
-// per candidate, the exact decision "T <= theta" against the running best (theta = best or best-1),
-// and T <= theta iff every term <= theta, i.e. W(s,t) <= theta*(t-s+1) — no division. With the cut
-// sets ordered (outer cuts, x = e_{S-3}, e = e_{S-2}), the terms that involve the last cut e collapse
-// into three comparisons against per-row thresholds:
-//   A[e] <= H1,  K[e] <= H2,  V[e] <= theta,
-// where A[e] = PC_p[e+1], K[e] = PC_p[e+1] + Z_p[e] + (PC_q[L] - PC_q[e+1]), V[e] = max(c_q, lm_p) are
-// per-state column tables (p = S-2, q = S-1), and H1, H2 fold every other term of the candidate.
-// A candidate that passes gets its exact T (with the divisions) and index; it is the rare path.
-// Every candidate of the shard is decided individually; none is skipped.
+//   T = max( c_s, lm_s, ceil(W(s,t) / (t-s+1)) ),  W(s,t) = sum_{u=s..t} c_u + sum_{u=s..t-1} z_u
+// (c_s = stage cost on its worker, z_s = cf_s + cb_s, lm_s = max(cf_s, cb_s) at cut e_s). The search
+// only needs, per candidate, the exact decision "T <= theta" against the running best (theta = best,
+// or best - 1 once the lane is past the best's index), and T <= theta iff every term <= theta, i.e.
+// W(s,t) <= theta * (t-s+1): no division. Scanning the stages left to right with
+//   M_j(k) = min_{s<=j} ( theta * (j-s+1+k) - sum_{u=s..j} (c_u + z_u) ),
+//   M_j(k) = min(theta * (1+k), M_{j-1}(k+1)) - (c_j + z_j),
+// every segment that ends k stages after stage j is "rest <= M_j(k)". For the last two stages
+// p = S-2 (layers x+1..e) and q = S-1 (layers e+1..L-1) all terms collapse into three comparisons
+//   A[e] < H1',  K[e] < H2',  V[e] < TH',
+// with per-state column tables A[e] = PC_p[e+1], K[e] = PC_p[e+1] + Z_p[e] + (PC_q[L] - PC_q[e+1]),
+// V[e] = max(c_q, lm_p), and per-lane thresholds H1 = min(theta, M_{p-1}(1)) + PC_p[x+1],
+// H2 = min(2 theta, M_{p-1}(2)) + PC_p[x+1], TH = theta (the ' versions are +1 for a strict test,
+// and 0 for a lane whose fixed terms already exceed theta). A candidate that passes gets its exact T
+// (with the divisions) and its index: the rare path. Every candidate of the shard is decided.
 //
-// Mapping (the B200 part). Work is grouped by x: all rows (outer cut tuples below x) with the same x
-// have the same number of columns l = L-2-x, so a warp takes 32 rows of one x (one per lane, R
-// consecutive rows per lane) and sweeps the columns in lockstep: the column tables are read with
-// broadcast LDS.128 (one shared-memory wavefront per warp step), per-lane thresholds stay in
-// registers, and there is no divergence in the hot loop. Consecutive rows of a lane differ in one
-// cut (lexicographic successor), so the per-row threshold update touches two stages; a full
-// re-hoist happens only when an earlier cut changes. Warps take tasks from a global atomic counter
-// (persistent grid, a few blocks per SM); the (T, index) argmin is per lane, then warp -> block
-// (shuffles + shared memory) -> grid (k_finalize). The result is the lexicographic (T, index)
-// minimum, independent of the task order, the grid size and the number of GPUs.
+// Mapping (the B200 part). Cut sets are (prefix e_0..e_{S-5}, y = e_{S-4}, x = e_{S-3}, e = e_{S-2}).
+// A warp task fixes y; its 32 lanes take different prefixes (R consecutive ones each). So within a
+// warp, x and e run in lockstep and everything that depends on x or e only is warp-uniform: the
+// x-level update is a broadcast load plus ~20 integer ops per lane, the column sweep is one
+// broadcast 128-bit shared-memory load and three compares per column per lane, and there is no
+// divergence in the hot loop. A lane re-derives its prefix terms (O(S^2)) once per row; a row covers
+// C(L-2-y, 2) candidates. Warps take tasks from a global atomic counter (persistent grid); the
+// (T, index) argmin goes lane -> warp -> block (shuffles + shared memory) -> grid (k_finalize), so the
+// result is the lexicographic (T, index) minimum whatever the task order, grid or GPU count.
 #include "binom.cuh"
 #include "internal.h"
 
 namespace ap {
 
-struct R1XEntry {      // one x value of the schedule (host-built, SPEC.md §5 shard arithmetic)
-  int x;               // e_{S-3}
+struct R1YEntry {      // one y value of the schedule (host-built shard arithmetic, SPEC.md §5)
+  int y;               // e_{S-4}
   u32 rows_per_lane;   // R
-  u64 row_begin;       // first row (lex rank of the outer tuple among NO-subsets of {0..x-1})
-  u64 row_end;         // one past the last row in the shard
-  u64 task_begin;      // global index of this x's first task
+  u64 row_begin;       // first prefix row (lex rank among P-subsets of {0..y-1}) in the shard
+  u64 row_end;         // one past the last
+  u64 task_begin;      // global index of this y's first task
 };
 
 struct R1Header {
-  u64 off;                    // global index of (S, rho = 0, kappa = 0)
+  u64 off;                   // global index of (S, rho = 0, kappa = 0)
   u64 ntasks;
-  u64 lo_outer, hi_outer;     // packed outer cuts of the shard's first / last candidate
-  int lo_x, lo_e, hi_x, hi_e; // their x and e
-  int nx, pad;
-  u32 counter;                // task counter (reset per launch)
-  u32 pad2;
+  u64 lo_pre, hi_pre;        // packed prefix cuts of the shard's first / last candidate
+  int lo_y, lo_x, lo_e;      // and their (y, x, e)
+  int hi_y, hi_x, hi_e;
+  int ny;
+  u32 counter;               // task counter (reset by the header copy before each launch)
 };
 
 template <typename T>
 struct __align__(16) ColT {
   T A, K, V, pad;
 };
-template <typename T>
-struct __align__(16) RowT {
-  T PCa, PCb, Z, LM;  // PC_{p-2}[y+1], PC_{p-1}[y+1], Z_{p-2}[y], LM_{p-2}[y]
+// per-state x table (64-bit): with pcy = PC_{p-1}[y+1] and the lane's row constants
+// N0' = min(theta, M_P(1)) + pcy, N1' = min(2 theta, M_P(2)) + pcy, N2' = min(3 theta, M_P(3)) + pcy:
+//   stage p-1 fits          <=> pc1 <= N0'   and  lm1 <= theta
+//   H1 = min(theta + pcp, N1' + W1),  H2 = min(2 theta + pcp, N2' + W1),  W1 = pcp - pc1 - z1.
+struct __align__(16) XT {
+  unsigned long long pcp, pc1, lm1;  // PC_p[x+1], PC_{p-1}[x+1], LM_{p-1}[x]
+  long long W1;                      // PC_p[x+1] - PC_{p-1}[x+1] - Z_{p-1}[x]
 };
 
 typedef long long i64;
-// theta >= THETA_ALL means "no best yet": every candidate passes (all modelled times are < 2^59,
-// so theta * 8 never overflows i64 for a real theta)
+// theta >= THETA_ALL means "no best yet": every candidate passes. Real thetas are < 2^59 (the state's
+// overflow bound), so theta * 8 and every sum below fit in i64.
 constexpr i64 THETA_ALL = 1ll << 60;
 
 __device__ __forceinline__ i64 smin(i64 a, i64 b) { return a < b ? a : b; }
@@ -94,313 +102,310 @@ __device__ __noinline__ u64 exact_T_r1(const u64 *PC, const u64 *Z, const u64 *L
   return T;
 }
 
-// Per-lane search state for one S.
-template <int S, typename T>
-struct Lane {
-  static constexpr int p = S - 2, q = S - 1, NO = S - 3;
-  // level A (cuts e_0..e_{p-3}, stages 0..p-3)
-  bool aliveA;
-  i64 Ga, Gb, Gc, Gd;
-  u64 baseA;  // PC_{p-2}[a_{p-2}]
-  // task (x) level
-  int x;
-  u64 cx;      // PC_{p-1}[x+1] (S >= 4) or the stage-0 cost (S = 3)
-  u64 zx, lmx; // Z_{p-1}[x], LM_{p-1}[x]
-  u64 base_p;  // PC_p[x+1]
-  // row
-  u64 outer;   // packed e_0..e_{NO-1}
-  bool alive;
-  T H1, H2, TH;
-  // best
-  u64 bestT, bestI;
-  i64 theta;
+// Row terms of one lane, in two parts so that consecutive rows (which usually differ only in the last
+// prefix cut) redo two levels, not all of them. Stages 0..P-2 (the "base", cuts e_0..e_{P-2}) give
+// M_{P-2}(2..5) and their own feasibility; row_finish adds stage P-1 (cut e_{P-1}) and stage P (cut
+// y) and returns whether stages 0..P fit, with N0 = min(theta, M_P(1)), N1 = min(2 theta, M_P(2)),
+// N2 = min(3 theta, M_P(3)). P = S-4.
+struct RowBase {
+  i64 M1, M2, M3, M4, M5;  // M_{P-2}(1..5)
+  int a;               // first layer of stage P-1
+  bool ok;
 };
 
-template <int S, typename T>
-__device__ __forceinline__ void hoist_A(Lane<S, T> &st, const u64 *PC, const u64 *Z, const u64 *LM, int L) {
-  constexpr int p = S - 2;
+template <int S>
+__device__ __noinline__ void row_base(const u64 *PC, const u64 *Z, const u64 *LM, int L, u64 pre, i64 th,
+                                      RowBase &b) {
+  constexpr int P = S - 4;
   const int Lp1 = L + 1;
-  const i64 th = st.theta;
+  i64 M[S + 1];
+#pragma unroll
+  for (int k = 0; k <= S; ++k) M[k] = THETA_ALL * 4;
   bool ok = true;
-  i64 Ga = THETA_ALL * 4, Gb = THETA_ALL * 4, Gc = THETA_ALL * 4, Gd = THETA_ALL * 4;
-  u64 baseA = 0;
-  if constexpr (p >= 3) {
-    const int a2 = byte_at(st.outer, p - 3) + 1;
-    baseA = PC[(p - 2) * Lp1 + a2];
-  }
-  if (th >= THETA_ALL) {
-    st.aliveA = true;
-    st.Ga = Ga; st.Gb = Gb; st.Gc = Gc; st.Gd = Gd;
-    st.baseA = baseA;
-    return;
-  }
-  if constexpr (p >= 3) {
-    // stages 0..p-3 are fixed by the cuts e_0..e_{p-3}
-    i64 c[p - 2 > 0 ? p - 2 : 1], z[p - 2 > 0 ? p - 2 : 1];
+  int a = 0;
+  if (th < THETA_ALL) {
 #pragma unroll
-    for (int u = 0; u <= p - 3; ++u) {
-      const int a = (u == 0) ? 0 : byte_at(st.outer, u - 1) + 1;
-      const int e = byte_at(st.outer, u);
-      c[u] = (i64)(PC[u * Lp1 + e + 1] - PC[u * Lp1 + a]);
-      z[u] = (i64)Z[u * L + e];
-      ok &= (c[u] <= th) & ((i64)LM[u * L + e] <= th);
+    for (int j = 0; j <= P - 2; ++j) {
+      const int e = byte_at(pre, j);
+      const i64 c = (i64)(PC[j * Lp1 + e + 1] - PC[j * Lp1 + a]);
+      const i64 cz = c + (i64)Z[j * L + e];
+      ok &= (c <= th) & ((i64)LM[j * L + e] <= th) & (c <= M[1]);
+#pragma unroll
+      for (int k = 1; k < S - j; ++k) M[k] = smin(th * (1 + k), M[k + 1]) - cz;
+      a = e + 1;
     }
-    // segments inside stages 0..p-3
-#pragma unroll
-    for (int s = 0; s <= p - 3; ++s) {
-      i64 acc = c[s];
-#pragma unroll
-      for (int t = s + 1; t <= p - 3; ++t) {
-        acc += z[t - 1] + c[t];
-        ok &= acc <= th * (t - s + 1);
-      }
-    }
-    // D'_s = sum_{u=s}^{p-3} (c_u + z_u) and the four collapsed thresholds
-    i64 D = 0;
-#pragma unroll
-    for (int s = p - 3; s >= 0; --s) {
-      D += c[s] + z[s];
-      Ga = smin(Ga, th * (p - 1 - s) - D);
-      Gb = smin(Gb, th * (p - s) - D);
-      Gc = smin(Gc, th * (p - s + 1) - D);
-      Gd = smin(Gd, th * (p - s + 2) - D);
-    }
-  }
-  st.aliveA = ok;
-  st.Ga = Ga; st.Gb = Gb; st.Gc = Gc; st.Gd = Gd;
-  st.baseA = baseA;
-}
-
-template <typename T>
-__device__ __forceinline__ T clampT(i64 v) {
-  // threshold for "value <= v" on values of type T (< 2^32 - 16 in the 32-bit path)
-  if (v < 0) return (T)0;  // caller folds the "dead" case separately
-  const u64 m = (sizeof(T) == 4) ? 0xFFFFFFFFull : ~0ull;
-  return (T)((u64)v > m ? m : (u64)v);
-}
-
-// Row thresholds for the current (outer, x) with the current theta.
-template <int S, typename T>
-__device__ __forceinline__ void hoist_row(Lane<S, T> &st, const RowT<T> *rowy) {
-  constexpr int p = S - 2;
-  const i64 th = st.theta;
-  if (th >= THETA_ALL) {
-    st.alive = true;
-    st.H1 = st.H2 = st.TH = (T)~(T)0;
-    return;
-  }
-  i64 h1, h2;
-  bool ok = st.aliveA;
-  if constexpr (S == 3) {
-    const i64 c0 = (i64)st.cx, zx = (i64)st.zx;
-    ok &= (c0 <= th) & ((i64)st.lmx <= th);
-    h1 = smin(th, 2 * th - c0 - zx);
-    h2 = smin(2 * th, 3 * th - c0 - zx);
   } else {
-    const int y = byte_at(st.outer, S - 4);  // e_{p-2}
-    const RowT<T> r = rowy[y];
-    const i64 cpm2 = (i64)((u64)r.PCa - st.baseA);
-    const i64 cpm1 = (i64)(st.cx - (u64)r.PCb);
-    const i64 zpm2 = (i64)(u64)r.Z;
-    const i64 Q = cpm2 + zpm2 + cpm1;
-    const i64 zx = (i64)st.zx;
-    ok &= (cpm2 <= smin(th, st.Ga)) & ((i64)(u64)r.LM <= th) & (cpm1 <= th) & (Q <= smin(2 * th, st.Gb)) &
-          ((i64)st.lmx <= th);
-    h1 = smin(smin(th, 2 * th - cpm1 - zx), smin(3 * th, st.Gc) - Q - zx);
-    h2 = smin(smin(2 * th, 3 * th - cpm1 - zx), smin(4 * th, st.Gd) - Q - zx);
-    (void)p;
+#pragma unroll
+    for (int j = 0; j <= P - 2; ++j) a = byte_at(pre, j) + 1;
   }
-  const i64 H1 = h1 + (i64)st.base_p, H2 = h2 + (i64)st.base_p;
-  ok &= (h1 >= 0) & (h2 >= 0);
-  st.alive = ok;
-  // dead rows: thresholds that no value can meet (values are >= 0, compare with <=): use H < 0 ->
-  // encode by alive flag folded into TH (TH = 0 with alive = false never matters: we test alive).
-  st.H1 = clampT<T>(H1);
-  st.H2 = clampT<T>(H2);
-  st.TH = clampT<T>(th);
+  b.M1 = M[1]; b.M2 = M[2]; b.M3 = M[3]; b.M4 = M[4]; b.M5 = M[5];
+  b.a = a;
+  b.ok = ok;
 }
+
+template <int S>
+__device__ __forceinline__ bool row_finish(const RowBase &b, const u64 *PC, const u64 *Z, const u64 *LM, int L,
+                                           int e1, int y, i64 th, i64 &N0, i64 &N1, i64 &N2) {
+  constexpr int P = S - 4;
+  if (th >= THETA_ALL) {
+    N0 = N1 = N2 = THETA_ALL;
+    return true;
+  }
+  const int Lp1 = L + 1;
+  // stage P-1 = [b.a, e1] on worker P-1:  M_{P-1}(k) = min(theta (1+k), M_{P-2}(k+1)) - cz, k = 1..4
+  const i64 c1 = (i64)(PC[(P - 1) * Lp1 + e1 + 1] - PC[(P - 1) * Lp1 + b.a]);
+  const i64 cz1 = c1 + (i64)Z[(P - 1) * L + e1];
+  const i64 M1_1 = smin(2 * th, b.M2) - cz1, M1_2 = smin(3 * th, b.M3) - cz1, M1_3 = smin(4 * th, b.M4) - cz1,
+            M1_4 = smin(5 * th, b.M5) - cz1;
+  bool ok = b.ok & (c1 <= th) & ((i64)LM[(P - 1) * L + e1] <= th) & (c1 <= b.M1);
+  // stage P = [e1+1, y] on worker P
+  const i64 c0 = (i64)(PC[P * Lp1 + y + 1] - PC[P * Lp1 + e1 + 1]);
+  const i64 cz0 = c0 + (i64)Z[P * L + y];
+  ok &= (c0 <= th) & ((i64)LM[P * L + y] <= th) & (c0 <= M1_1);
+  N0 = smin(th, smin(2 * th, M1_2) - cz0);
+  N1 = smin(2 * th, smin(3 * th, M1_3) - cz0);
+  N2 = smin(3 * th, smin(4 * th, M1_4) - cz0);
+  return ok;
+}
+
+// strict-test threshold for values of type T: "v < thr(h)" == "v <= h"; dead lanes get 0
+template <typename T>
+__device__ __forceinline__ T thr(i64 h, bool alive) {
+  const u64 m = (sizeof(T) == 4) ? 0xFFFFFFFFull : ~0ull;
+  if (!alive || h < 0) return (T)0;
+  const u64 v = (u64)h + 1;
+  return (T)(v > m ? m : v);
+}
+
+// one column of the sweep, read with an explicit 32-bit shared-memory address (one LDS per column
+// for 32-bit tables, two for 64-bit ones)
+__device__ __forceinline__ void lds_col(unsigned a, u32 &A, u32 &K, u32 &V) {
+  u32 pad;
+  asm("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(A), "=r"(K), "=r"(V), "=r"(pad) : "r"(a));
+}
+__device__ __forceinline__ void lds_col(unsigned a, u64 &A, u64 &K, u64 &V) {
+  asm("ld.shared.v2.u64 {%0, %1}, [%2];" : "=l"(A), "=l"(K) : "r"(a));
+  asm("ld.shared.u64 %0, [%1+16];" : "=l"(V) : "r"(a));
+}
+
+__device__ __forceinline__ u32 clamp_u32(i64 v) { return v < 0 ? 0u : (v > 0xFFFFFFFFll ? 0xFFFFFFFFu : (u32)v); }
+
+// Per-row constants and the per-x threshold update. Thresholds are for strict tests (v < H <=> v <= h).
+template <typename T>
+struct XUpd;
+template <>
+struct XUpd<u64> {  // 64-bit path: thresholds straight from the i64 formulas
+  i64 th, N0p, N1p, N2p;
+  __device__ __forceinline__ void row(i64 th_, bool alive, i64 N0, i64 N1, i64 N2, u64 pcy) {
+    th = th_;
+    N0p = alive ? N0 + (i64)pcy : -1;
+    N1p = N1 + (i64)pcy;
+    N2p = N2 + (i64)pcy;
+  }
+  __device__ __forceinline__ u64 TH() const { return thr<u64>(th, true); }
+  __device__ __forceinline__ void x(const XT &v, u64 &H1, u64 &H2) const {
+    const bool alive = ((i64)v.pc1 <= N0p) && ((i64)v.lm1 <= th);
+    H1 = thr<u64>(smin(th + (i64)v.pcp, N1p + v.W1), alive);
+    H2 = thr<u64>(smin(2 * th + (i64)v.pcp, N2p + v.W1), alive);
+  }
+};
+template <>
+struct XUpd<u32> {  // 32-bit path: every table value is < 2^32 - 16, so clamp once per row and stay in 32 bits
+  u32 th1, th2, N0c;
+  i64 N1q, N2q;  // N1' + 1, N2' + 1
+  __device__ __forceinline__ void row(i64 th, bool alive, i64 N0, i64 N1, i64 N2, u64 pcy) {
+    th1 = clamp_u32(th + 1);
+    th2 = clamp_u32(2 * th + 1);
+    N0c = alive ? clamp_u32(N0 + (i64)pcy + 1) : 0u;
+    N1q = N1 + (i64)pcy + 1;
+    N2q = N2 + (i64)pcy + 1;
+  }
+  __device__ __forceinline__ u32 TH() const { return th1; }
+  __device__ __forceinline__ void x(const XT &v, u32 &H1, u32 &H2) const {
+    const u32 pcp = (u32)v.pcp;
+    const bool alive = ((u32)v.pc1 < N0c) & ((u32)v.lm1 < th1);
+    const u32 t1 = min(th1, 0xFFFFFFFFu - pcp) + pcp;  // clamp(theta + 1 + pcp), no overflow
+    const u32 t2 = min(th2, 0xFFFFFFFFu - pcp) + pcp;
+    const u32 s1 = clamp_u32(N1q + v.W1), s2 = clamp_u32(N2q + v.W1);
+    H1 = alive ? min(t1, s1) : 0u;
+    H2 = alive ? min(t2, s2) : 0u;
+  }
+};
 
 template <int S, typename T, int NT>
-__global__ void __launch_bounds__(NT) k_search_r1(DevTables g, const R1Header *__restrict__ hdr_g,
-                                                  const R1XEntry *__restrict__ xt_g, R1Header *counter_hdr,
-                                                  BlockOut *out) {
-  constexpr int p = S - 2, q = S - 1, NO = S - 3;
+__global__ void __launch_bounds__(NT, 2) k_search_r1(DevTables g, const R1Header *__restrict__ hdr_g,
+                                                     const R1YEntry *__restrict__ yt_g, R1Header *counter_hdr,
+                                                     BlockOut *out) {
+  constexpr int p = S - 2, q = S - 1, P = S - 4;
   extern __shared__ __align__(16) unsigned char smraw[];
   const int L = (int)g.L, Lp1 = L + 1, n = L - 1;
   __shared__ R1Header hdr;
   if (threadIdx.x == 0) hdr = *hdr_g;
-  // shared layout: col[n] | rowy[n] | PC[S][Lp1] | Z[S-1][L] | LM[S-1][L] | xt[nx]
+  // shared layout: col[n + 16] | xt[n] | PC[S][Lp1] | Z[S-1][L] | LM[S-1][L] | B[Lp1][9] | yt[ny]
+  // (col carries 16 sentinel columns past e = L-2 that never pass, so the sweep needs no tail code)
   ColT<T> *col = (ColT<T> *)smraw;
-  RowT<T> *rowy = (RowT<T> *)(col + n);
-  u64 *PC = (u64 *)(rowy + n);
+  XT *xt = (XT *)(col + n + 16);
+  u64 *PC = (u64 *)(xt + n);
   u64 *Z = PC + S * Lp1;
   u64 *LM = Z + (S - 1) * L;
-  R1XEntry *xt = (R1XEntry *)(LM + (S - 1) * L);
+  u64 *Bn = LM + (S - 1) * L;
+  R1YEntry *yt = (R1YEntry *)(Bn + Lp1 * BINOM_K);
+  for (int i = threadIdx.x; i < Lp1 * BINOM_K; i += NT) Bn[i] = c_binom[i / BINOM_K][i % BINOM_K];
   for (int i = threadIdx.x; i < S * Lp1; i += NT) PC[i] = g.PC[i];
   for (int i = threadIdx.x; i < (S - 1) * L; i += NT) {
     Z[i] = g.Z[i];
     LM[i] = g.LM[i];
   }
   __syncthreads();
-  const int nx = hdr.nx;
-  for (int i = threadIdx.x; i < nx; i += NT) xt[i] = xt_g[i];
-  for (int e = threadIdx.x; e < n; e += NT) {  // column tables (per state, per S)
-    const u64 A = PC[p * Lp1 + e + 1];
-    const u64 cq = PC[q * Lp1 + L] - PC[q * Lp1 + e + 1];
+  const int ny = hdr.ny;
+  for (int i = threadIdx.x; i < ny; i += NT) yt[i] = yt_g[i];
+  for (int e = threadIdx.x; e < n + 16; e += NT) {  // per-state column and x tables
     ColT<T> cl;
-    cl.A = (T)A;
-    cl.K = (T)(A + Z[p * L + e] + cq);
-    cl.V = (T)umax(cq, LM[p * L + e]);
+    if (e < n) {
+      const u64 A = PC[p * Lp1 + e + 1];
+      const u64 cq = PC[q * Lp1 + L] - PC[q * Lp1 + e + 1];
+      cl.A = (T)A;
+      cl.K = (T)(A + Z[p * L + e] + cq);
+      cl.V = (T)umax(cq, LM[p * L + e]);
+      XT xv;
+      xv.pcp = A;
+      xv.pc1 = PC[(p - 1) * Lp1 + e + 1];
+      xv.lm1 = LM[(p - 1) * L + e];
+      xv.W1 = (i64)A - (i64)xv.pc1 - (i64)Z[(p - 1) * L + e];
+      xt[e] = xv;
+    } else {
+      cl.A = cl.K = cl.V = (T)~(T)0;  // sentinel: "v < threshold" is false for every threshold
+    }
     cl.pad = 0;
     col[e] = cl;
-    RowT<T> rw;
-    if constexpr (S >= 4) {
-      rw.PCa = (T)PC[(p - 2) * Lp1 + e + 1];
-      rw.Z = (T)Z[(p - 2) * L + e];
-      rw.LM = (T)LM[(p - 2) * L + e];
-    } else {
-      rw.PCa = 0; rw.Z = 0; rw.LM = 0;
-    }
-    rw.PCb = (T)PC[(p - 1) * Lp1 + e + 1];
-    rowy[e] = rw;
   }
   __syncthreads();
 
   const int lane = threadIdx.x & 31;
-  Lane<S, T> st;
-  st.bestT = U64MAX;
-  st.bestI = U64MAX;
-  u64 cnt = 0;
+  u64 bestT = U64MAX, bestI = U64MAX, cnt = 0;
   const u64 ntasks = hdr.ntasks;
+  int yi = 0;
   for (;;) {
     u64 task = 0;
     if (lane == 0) task = atomicAdd(&counter_hdr->counter, 1u);
     task = __shfl_sync(0xffffffffu, task, 0);
     if (task >= ntasks) break;
-    // locate the x entry (entries are few; linear scan over shared memory, warp-uniform)
-    int xi = 0;
-    while (xi + 1 < nx && xt[xi + 1].task_begin <= task) ++xi;
-    const R1XEntry xe = xt[xi];
-    const int x = xe.x;
-    const u64 R = xe.rows_per_lane;
-    const u64 r0 = xe.row_begin + (task - xe.task_begin) * 32ull * R + (u64)lane * R;
-    const u64 r1 = umin(r0 + R, xe.row_end);
-    // task-level values
-    st.x = x;
-    if constexpr (S == 3) {
-      st.cx = PC[0 * Lp1 + x + 1];
-      st.zx = Z[0 * L + x];
-      st.lmx = LM[0 * L + x];
-    } else {
-      st.cx = PC[(p - 1) * Lp1 + x + 1];
-      st.zx = Z[(p - 1) * L + x];
-      st.lmx = LM[(p - 1) * L + x];
-    }
-    st.base_p = PC[p * Lp1 + x + 1];
-    const bool has_rows = r0 < r1;
-    const int e_first = x + 1, e_last = L - 2;
-    if (has_rows) {
-      // lex unrank of the lane's first row among NO-subsets of {0..x-1}
-      st.outer = (NO > 0) ? lex_unrank_packed(r0, NO, x) : 0ull;
-    } else {
-      st.outer = 0;
-    }
-    // the theta used for filtering: T <= theta passes. Non-strict (theta = best) while a candidate
-    // of this task may still have a smaller index than the lane's best, strict (best - 1) once the
-    // lane's candidates are past it (indices increase along a lane's rows and columns).
+    // tasks reach a warp in increasing order, so its cursor only moves forward
+    while (yi + 1 < ny && yt[yi + 1].task_begin <= task) ++yi;
+    const R1YEntry ye = yt[yi];
+    const int y = ye.y;
+    const u64 R = ye.rows_per_lane;
+    const u64 r0 = ye.row_begin + (task - ye.task_begin) * 32ull * R + (u64)lane * R;
+    const u64 r1 = umin(r0 + R, ye.row_end);
+    const u64 pcy = PC[(p - 1) * Lp1 + y + 1];  // start of stage p-1 (warp-uniform)
+    u64 pre = (r0 < r1 && P > 0) ? lex_unrank_smem(r0, P, y, Bn) : 0ull;
+    // strictness: theta = best while this lane's task may still hold a smaller index than its best
     bool strict = true;
-    if (has_rows && st.bestT != U64MAX) {
-      int e0 = e_first;
-      if (st.outer == hdr.lo_outer && x == hdr.lo_x) e0 = hdr.lo_e > e0 ? hdr.lo_e : e0;
-      const u64 first_idx =
-          hdr.off + lex_rank_packed(st.outer | ((u64)x << (8 * NO)) | ((u64)e0 << (8 * (NO + 1))), S - 1, n);
-      strict = first_idx > st.bestI;
+    if (r0 < r1 && bestT != U64MAX) {
+      const bool lo_row = (pre == hdr.lo_pre) && (y == hdr.lo_y);
+      const int x0 = lo_row ? hdr.lo_x : y + 1, e0 = lo_row ? hdr.lo_e : y + 2;
+      const u64 first = pre | ((u64)y << (8 * P)) | ((u64)x0 << (8 * (P + 1))) | ((u64)e0 << (8 * (P + 2)));
+      strict = hdr.off + lex_rank_smem(first, S - 1, n, Bn) > bestI;
     }
-    st.theta = (st.bestT == U64MAX) ? THETA_ALL : (i64)st.bestT - (strict ? 1 : 0);
-    u64 row = r0;
-    bool need_A = true;
-    while (true) {
-      const bool active = has_rows && row < r1;
+    RowBase base;
+    bool need_base = true;
+    for (u64 row = r0;; ++row) {
+      const bool active = row < r1;
       if (!__any_sync(0xffffffffu, active)) break;
-      int emin = e_first, emax = e_last;
-      u64 cuts_prefix = 0;  // outer cuts + x, packed (the candidate's cuts without e)
+      // partial rows at the shard boundaries: (x, e) range restricted, checked on the rare path
+      bool lo_part = false, hi_part = false;
+      i64 th = (bestT == U64MAX) ? THETA_ALL : (i64)bestT - (strict ? 1 : 0);
+      bool aliveP = false;
+      i64 N0 = 0, N1 = 0, N2 = 0;
       if (active) {
-        cuts_prefix = st.outer | ((u64)x << (8 * NO));
-        // shard boundaries: the shard's first / last row may be partial
-        if (st.outer == hdr.lo_outer && x == hdr.lo_x) emin = hdr.lo_e > emin ? hdr.lo_e : emin;
-        if (st.outer == hdr.hi_outer && x == hdr.hi_x) emax = hdr.hi_e < emax ? hdr.hi_e : emax;
-        cnt += (emax >= emin) ? (u64)(emax - emin + 1) : 0ull;
-        if (need_A) hoist_A<S, T>(st, PC, Z, LM, L);
-        hoist_row<S, T>(st, rowy);
-        st.alive &= emax >= emin;
-      } else {
-        st.alive = false;
-      }
-      // ---- hot loop: lockstep sweep of the columns e in (x, L-2] -----------------------------
-      bool alive = st.alive;
-      int e = e_first;
-      auto pass = [&](const ColT<T> &c) { return (c.A <= st.H1) & (c.K <= st.H2) & (c.V <= st.TH); };
-      while (e <= e_last) {
-        // 4 columns per step, one broadcast 128-bit shared load each
-        bool hit = false;
-        if (e + 3 <= e_last) {
-          const ColT<T> c0 = col[e], c1 = col[e + 1], c2 = col[e + 2], c3 = col[e + 3];
-          hit = alive & (pass(c0) | pass(c1) | pass(c2) | pass(c3));
-          if (!hit) { e += 4; continue; }
-        } else {
-          hit = alive & pass(col[e]);
-          if (!hit) { e += 1; continue; }
+        lo_part = (pre == hdr.lo_pre) && (y == hdr.lo_y);
+        hi_part = (pre == hdr.hi_pre) && (y == hdr.hi_y);
+        // evaluated candidates of this row: the (x, e) pairs y < x < e <= L-2 within the shard
+        const u64 m = (u64)(L - 2 - y);
+        u64 row_cnt = m * (m - 1) / 2;
+        if (lo_part || hi_part) {
+          auto prank = [&](int x, int e) -> u64 {  // rank of (x, e) among the row's pairs
+            u64 r = 0;
+            for (int xx = y + 1; xx < x; ++xx) r += (u64)(L - 2 - xx);
+            return r + (u64)(e - x - 1);
+          };
+          const u64 rlo = lo_part ? prank(hdr.lo_x, hdr.lo_e) : 0ull;
+          const u64 rhi = hi_part ? prank(hdr.hi_x, hdr.hi_e) + 1 : row_cnt;
+          row_cnt = rhi > rlo ? rhi - rlo : 0ull;
         }
-        // rare path: re-check the (up to 4) columns in order with the current thresholds
-        const int stop = (e + 3 <= e_last) ? e + 3 : e;
-        for (int ee = e; ee <= stop; ++ee) {
-          if (!(alive && pass(col[ee]))) continue;
-          if (ee < emin || ee > emax) continue;  // outside the shard (partial rows only)
-          const u64 cuts = cuts_prefix | ((u64)ee << (8 * (NO + 1)));
-          const u64 Tc = exact_T_r1<S>(PC, Z, LM, L, cuts);
-          const u64 idx = hdr.off + lex_rank_packed(cuts, S - 1, n);
-          if (better(Tc, idx, st.bestT, st.bestI)) {
-            st.bestT = Tc;
-            st.bestI = idx;
+        cnt += row_cnt;
+        if (need_base) row_base<S>(PC, Z, LM, L, pre, th, base);
+        aliveP = row_finish<S>(base, PC, Z, LM, L, byte_at(pre, P - 1), y, th, N0, N1, N2);
+      }
+      XUpd<T> xu;
+      xu.row(th, aliveP && active, N0, N1, N2, pcy);
+      T TH = active ? xu.TH() : (T)0;
+      // ---- x sweep (warp-uniform), then the hot column sweep -------------------------------
+      constexpr unsigned CS = sizeof(ColT<T>);
+      const unsigned cb = (unsigned)__cvta_generic_to_shared(col);
+      const unsigned aend = cb + (unsigned)(L - 1) * CS;  // one past the column e = L-2
+      for (int x = y + 1; x <= L - 3; ++x) {
+        const XT xv = xt[x];
+        T H1, H2;
+        xu.x(xv, H1, H2);
+#ifndef AP_SWEEP
+#define AP_SWEEP 4
+#endif
+        // AP_SWEEP columns per step (sentinel-padded, no tail code), one LDS per column
+        unsigned a = cb + (unsigned)(x + 1) * CS;
+        for (; a < aend; a += AP_SWEEP * CS) {
+          bool hit = false;
+#pragma unroll
+          for (int u = 0; u < AP_SWEEP; ++u) {
+            T A0, K0, V0;
+            lds_col(a + u * CS, A0, K0, V0);
+            hit |= (A0 < H1) & (K0 < H2) & (V0 < TH);
           }
-          // every later candidate of this lane's task has a larger index: strict from here on
-          const i64 th_new = (i64)st.bestT - 1;
-          if (th_new != st.theta) {
-            st.theta = th_new;
-            hoist_A<S, T>(st, PC, Z, LM, L);
-            hoist_row<S, T>(st, rowy);
-            alive = st.alive && (emax >= emin);
+          if (hit) {
+            // rare path: the columns of this step in order, with the current thresholds
+            const int e = (int)((a - cb) / CS);
+            for (int ee = e; ee < e + AP_SWEEP; ++ee) {
+              const ColT<T> c = col[ee];
+              if (!((c.A < H1) & (c.K < H2) & (c.V < TH))) continue;
+              if (lo_part && (x < hdr.lo_x || (x == hdr.lo_x && ee < hdr.lo_e))) continue;
+              if (hi_part && (x > hdr.hi_x || (x == hdr.hi_x && ee > hdr.hi_e))) continue;
+              const u64 cuts = pre | ((u64)y << (8 * P)) | ((u64)x << (8 * (P + 1))) | ((u64)ee << (8 * (P + 2)));
+              const u64 Tc = exact_T_r1<S>(PC, Z, LM, L, cuts);
+              const u64 idx = hdr.off + lex_rank_smem(cuts, S - 1, n, Bn);
+              if (better(Tc, idx, bestT, bestI)) {
+                bestT = Tc;
+                bestI = idx;
+              }
+              // later candidates of this lane have larger indices: strict from here on
+              strict = true;
+              th = (i64)bestT - 1;
+              row_base<S>(PC, Z, LM, L, pre, th, base);
+              aliveP = row_finish<S>(base, PC, Z, LM, L, byte_at(pre, P - 1), y, th, N0, N1, N2);
+              xu.row(th, aliveP, N0, N1, N2, pcy);
+              xu.x(xv, H1, H2);
+              TH = xu.TH();
+            }
           }
         }
-        e = stop + 1;
       }
-      if (!active) {
-        row = r1;  // idle lane: keep sweeping in lockstep until every lane is done
-        continue;
-      }
-      // ---- next row: lexicographic successor of the outer cuts below x --------------------
-      ++row;
-      need_A = false;
-      if (row < r1) {
-        if constexpr (NO == 0) {
-          // one row per x
+      // ---- next row of this lane: lexicographic successor of the prefix below y ------------
+      // usually only the last prefix cut moves (+1): the base (stages 0..P-2) stays valid
+      need_base = false;
+      if (active && row + 1 < r1) {
+        if (byte_at(pre, P - 1) < y - 1) {
+          pre += 1ull << (8 * (P - 1));
         } else {
-          const int ylast = byte_at(st.outer, NO - 1);
-          if (ylast < x - 1) {
-            st.outer += 1ull << (8 * (NO - 1));  // only e_{p-2} moves: level A unchanged
-          } else {
-            lex_next_packed(st.outer, NO, x);
-            need_A = true;
-          }
+          lex_next_packed(pre, P, y);
+          need_base = true;
         }
       }
     }
   }
-  block_minloc_store<NT>(st.bestT, st.bestI, cnt, out + blockIdx.x);
+  block_minloc_store<NT>(bestT, bestI, cnt, out + blockIdx.x);
 }
 
 // ------------------------------------------------------------------------------------------------
-// host side: the task schedule (rows per x restricted to the shard) and the launch
+// host side: the task schedule (rows per y restricted to the shard) and the launch
 // ------------------------------------------------------------------------------------------------
 static u64 hb(int n, int k) {  // host binomial (n < 256, k <= 8); exact in u64
   if (k < 0 || n < 0 || k > n) return 0;
@@ -437,57 +442,59 @@ template <int S, typename T>
 static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u64 k_end, int sms,
                        BlockOut *out, int max_blocks, int *nblocks, void *work, size_t work_bytes,
                        cudaStream_t st) {
-  constexpr int NO = S - 3, NT = 256;
+  constexpr int P = S - 4, NT = 256;
   const int L = (int)g.L, n = L - 1, k = S - 1;
   int lo[8], hi[8];
   host_unrank(k_begin, k, n, lo);
   host_unrank(k_end - 1, k, n, hi);
-  // header + x table in pinned-less host memory, copied into the device work area
-  static thread_local unsigned char hbuf[sizeof(R1Header) + 256 * sizeof(R1XEntry)];
+  static thread_local unsigned char hbuf[sizeof(R1Header) + 256 * sizeof(R1YEntry)];
   R1Header *h = (R1Header *)hbuf;
-  R1XEntry *xt = (R1XEntry *)(hbuf + sizeof(R1Header));
+  R1YEntry *yt = (R1YEntry *)(hbuf + sizeof(R1Header));
   memset(h, 0, sizeof(*h));
   h->off = sp.off[S];
-  for (int i = 0; i < NO; ++i) {
-    h->lo_outer |= (u64)lo[i] << (8 * i);
-    h->hi_outer |= (u64)hi[i] << (8 * i);
+  for (int i = 0; i < P; ++i) {
+    h->lo_pre |= (u64)lo[i] << (8 * i);
+    h->hi_pre |= (u64)hi[i] << (8 * i);
   }
-  h->lo_x = lo[NO]; h->lo_e = lo[NO + 1];
-  h->hi_x = hi[NO]; h->hi_e = hi[NO + 1];
-  int nx = 0;
+  h->lo_y = lo[P]; h->lo_x = lo[P + 1]; h->lo_e = lo[P + 2];
+  h->hi_y = hi[P]; h->hi_x = hi[P + 1]; h->hi_e = hi[P + 2];
+  int ny = 0;
   u64 tasks = 0;
-  const u64 TARGET = 384;  // candidates per lane per task
-  for (int x = NO; x <= L - 3; ++x) {
-    const bool lo_fits = (NO == 0) || lo[NO - 1] < x;
-    const bool hi_fits = (NO == 0) || hi[NO - 1] < x;
-    const u64 rb = count_less(x, NO, lo) + ((lo_fits && x < lo[NO]) ? 1 : 0);
-    const u64 re = count_less(x, NO, hi) + ((hi_fits && x <= hi[NO]) ? 1 : 0);
+  // task size by estimated cost (thread-instructions per lane): a row costs ~150 (prefix terms) +
+  // ~26 per x + ~6 per candidate; ~40k per lane-task keeps ~40 tasks per warp on the 96-layer space,
+  // so the dynamic schedule's tail stays small while the per-task unrank is amortised
+  const u64 TARGET = 40000;
+  for (int y = P; y <= L - 4; ++y) {
+    // rows (prefix, y) whose candidates intersect [lo, hi]: a contiguous range of prefix ranks
+    const bool lo_fits = (P == 0) || lo[P - 1] < y;
+    const bool hi_fits = (P == 0) || hi[P - 1] < y;
+    const u64 rb = count_less(y, P, lo) + ((lo_fits && y < lo[P]) ? 1 : 0);
+    const u64 re = count_less(y, P, hi) + ((hi_fits && y <= hi[P]) ? 1 : 0);
     if (re <= rb) continue;
-    const u64 ell = (u64)(L - 2 - x);
-    u64 R = (TARGET + ell - 1) / ell;
-    const u64 rows = re - rb;
-    // keep at least ~8 tasks per SM overall: do not make R larger than needed
-    const u64 nt = (rows + 32 * R - 1) / (32 * R);
-    R1XEntry &xe = xt[nx++];
-    xe.x = x;
-    xe.rows_per_lane = (u32)R;
-    xe.row_begin = rb;
-    xe.row_end = re;
-    xe.task_begin = tasks;
+    const u64 m = (u64)(L - 2 - y);
+    const u64 row_cost = 150 + 26 * (m - 1) + 6 * (m * (m - 1) / 2);
+    const u64 R = row_cost >= TARGET ? 1 : (TARGET + row_cost - 1) / row_cost;
+    const u64 nt = (re - rb + 32 * R - 1) / (32 * R);
+    R1YEntry &ye = yt[ny++];
+    ye.y = y;
+    ye.rows_per_lane = (u32)R;
+    ye.row_begin = rb;
+    ye.row_end = re;
+    ye.task_begin = tasks;
     tasks += nt;
   }
-  h->nx = nx;
+  h->ny = ny;
   h->ntasks = tasks;
   *nblocks = 0;
   if (tasks == 0) return 0;
-  const size_t hbytes = sizeof(R1Header) + (size_t)nx * sizeof(R1XEntry);
-  // one 16 KB slot per S, so the r = 1 launches of one search never share a schedule buffer
+  const size_t hbytes = sizeof(R1Header) + (size_t)ny * sizeof(R1YEntry);
+  // one 16 KB slot per S, so the launches of one search never share a schedule buffer
   if ((size_t)(S + 1) * 16384 > work_bytes || hbytes > 16384) return 0;
   work = (unsigned char *)work + (size_t)S * 16384;
   // pageable source: the call returns once hbuf has been staged, so hbuf may be reused at once
   cudaMemcpyAsync(work, hbuf, hbytes, cudaMemcpyHostToDevice, st);
-  const size_t smem = (size_t)n * (sizeof(ColT<T>) + sizeof(RowT<T>)) + (size_t)S * (L + 1) * 8 +
-                      2 * (size_t)(S - 1) * L * 8 + (size_t)nx * sizeof(R1XEntry);
+  const size_t smem = (size_t)(n + 16) * sizeof(ColT<T>) + (size_t)n * sizeof(XT) + (size_t)S * (L + 1) * 8 +
+                      2 * (size_t)(S - 1) * L * 8 + (size_t)(L + 1) * BINOM_K * 8 + (size_t)ny * sizeof(R1YEntry);
   cudaFuncSetAttribute(k_search_r1<S, T, NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   int per_sm = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_search_r1<S, T, NT>, NT, smem);
@@ -497,8 +504,8 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
   if (blocks > need) blocks = need;
   if (blocks > (u64)max_blocks) blocks = (u64)max_blocks;
   const R1Header *hd = (const R1Header *)work;
-  const R1XEntry *xd = (const R1XEntry *)((unsigned char *)work + sizeof(R1Header));
-  k_search_r1<S, T, NT><<<(unsigned)blocks, NT, smem, st>>>(g, hd, xd, (R1Header *)work, out);
+  const R1YEntry *yd = (const R1YEntry *)((unsigned char *)work + sizeof(R1Header));
+  k_search_r1<S, T, NT><<<(unsigned)blocks, NT, smem, st>>>(g, hd, yd, (R1Header *)work, out);
   *nblocks = (int)blocks;
   return 1;
 }
@@ -507,13 +514,12 @@ template <typename T>
 static int launch_r1_s(int S, const DevTables &g, const SearchSpace &sp, u64 a, u64 b, int sms, BlockOut *out,
                        int mb, int *nb, void *w, size_t wb, cudaStream_t st) {
   switch (S) {
-    case 3: return launch_r1_t<3, T>(g, sp, a, b, sms, out, mb, nb, w, wb, st);
-    case 4: return launch_r1_t<4, T>(g, sp, a, b, sms, out, mb, nb, w, wb, st);
     case 5: return launch_r1_t<5, T>(g, sp, a, b, sms, out, mb, nb, w, wb, st);
     case 6: return launch_r1_t<6, T>(g, sp, a, b, sms, out, mb, nb, w, wb, st);
     case 7: return launch_r1_t<7, T>(g, sp, a, b, sms, out, mb, nb, w, wb, st);
     case 8: return launch_r1_t<8, T>(g, sp, a, b, sms, out, mb, nb, w, wb, st);
   }
+  *nb = 0;
   return 0;
 }
 
