@@ -177,6 +177,26 @@ __device__ __forceinline__ T thr(i64 h, bool alive) {
   return (T)(v > m ? m : v);
 }
 
+// A warp's folded column table: A'[e] = (V[e] < THw) ? A[e] : MAX and K[e], where THw is the largest
+// strict threshold of the warp's lanes. "A'[e] < H1 and K[e] < H2" then implies "V[e] < THw"; a lane
+// whose own threshold is smaller re-checks V on the rare path. Two compares per column instead of three.
+template <typename T>
+struct __align__(2 * sizeof(T)) FoldT {
+  T A, K;
+};
+__device__ __forceinline__ void lds_fold(unsigned a, u32 &A, u32 &K) {
+  asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(A), "=r"(K) : "r"(a));
+}
+__device__ __forceinline__ void lds_fold(unsigned a, u64 &A, u64 &K) {
+  asm("ld.shared.v2.u64 {%0, %1}, [%2];" : "=l"(A), "=l"(K) : "r"(a));
+}
+__device__ __forceinline__ u32 warp_max_T(u32 v) { return __reduce_max_sync(0xffffffffu, v); }
+__device__ __forceinline__ u64 warp_max_T(u64 v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = umax(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+
 // one column of the sweep, read with an explicit 32-bit shared-memory address (one LDS per column
 // for 32-bit tables, two for 64-bit ones)
 __device__ __forceinline__ void lds_col(unsigned a, u32 &A, u32 &K, u32 &V) {
@@ -250,6 +270,8 @@ __global__ void __launch_bounds__(NT, 2) k_search_r1(DevTables g, const R1Header
   u64 *LM = Z + (S - 1) * L;
   u64 *Bn = LM + (S - 1) * L;
   R1YEntry *yt = (R1YEntry *)(Bn + Lp1 * BINOM_K);
+  // per-warp folded tables follow the schedule (16-byte aligned)
+  FoldT<T> *foldall = (FoldT<T> *)(((uintptr_t)(yt + hdr_g->ny) + 15) & ~(uintptr_t)15);
   for (int i = threadIdx.x; i < Lp1 * BINOM_K; i += NT) Bn[i] = c_binom[i / BINOM_K][i % BINOM_K];
   for (int i = threadIdx.x; i < S * Lp1; i += NT) PC[i] = g.PC[i];
   for (int i = threadIdx.x; i < (S - 1) * L; i += NT) {
@@ -282,6 +304,9 @@ __global__ void __launch_bounds__(NT, 2) k_search_r1(DevTables g, const R1Header
   __syncthreads();
 
   const int lane = threadIdx.x & 31;
+  FoldT<T> *fold = foldall + (threadIdx.x >> 5) * (n + 16);
+  const unsigned fb = (unsigned)__cvta_generic_to_shared(fold);
+  T THw_table = (T)0;  // THw the warp's folded table was built for (0 = not built)
   u64 bestT = U64MAX, bestI = U64MAX, cnt = 0;
   const u64 ntasks = hdr.ntasks;
   int yi = 0;
@@ -340,10 +365,23 @@ __global__ void __launch_bounds__(NT, 2) k_search_r1(DevTables g, const R1Header
       XUpd<T> xu;
       xu.row(th, aliveP && active, N0, N1, N2, pcy);
       T TH = active ? xu.TH() : (T)0;
+      {  // (re)build the warp's folded table when the warp's largest threshold changed
+        const T THw = warp_max_T(TH);
+        if (THw != THw_table) {
+          for (int e = lane; e < n + 16; e += 32) {
+            const ColT<T> c = col[e];
+            FoldT<T> f;
+            f.A = (c.V < THw) ? c.A : (T)~(T)0;
+            f.K = c.K;
+            fold[e] = f;
+          }
+          __syncwarp();
+          THw_table = THw;
+        }
+      }
       // ---- x sweep (warp-uniform), then the hot column sweep -------------------------------
-      constexpr unsigned CS = sizeof(ColT<T>);
-      const unsigned cb = (unsigned)__cvta_generic_to_shared(col);
-      const unsigned aend = cb + (unsigned)(L - 1) * CS;  // one past the column e = L-2
+      constexpr unsigned FS = sizeof(FoldT<T>);
+      const unsigned aend = fb + (unsigned)(L - 1) * FS;  // one past the column e = L-2
       for (int x = y + 1; x <= L - 3; ++x) {
         const XT xv = xt[x];
         T H1, H2;
@@ -352,18 +390,18 @@ __global__ void __launch_bounds__(NT, 2) k_search_r1(DevTables g, const R1Header
 #define AP_SWEEP 4
 #endif
         // AP_SWEEP columns per step (sentinel-padded, no tail code), one LDS per column
-        unsigned a = cb + (unsigned)(x + 1) * CS;
-        for (; a < aend; a += AP_SWEEP * CS) {
+        unsigned a = fb + (unsigned)(x + 1) * FS;
+        for (; a < aend; a += AP_SWEEP * FS) {
           bool hit = false;
 #pragma unroll
           for (int u = 0; u < AP_SWEEP; ++u) {
-            T A0, K0, V0;
-            lds_col(a + u * CS, A0, K0, V0);
-            hit |= (A0 < H1) & (K0 < H2) & (V0 < TH);
+            T A0, K0;
+            lds_fold(a + u * FS, A0, K0);
+            hit |= (A0 < H1) & (K0 < H2);
           }
           if (hit) {
             // rare path: the columns of this step in order, with the current thresholds
-            const int e = (int)((a - cb) / CS);
+            const int e = (int)((a - fb) / FS);
             for (int ee = e; ee < e + AP_SWEEP; ++ee) {
               const ColT<T> c = col[ee];
               if (!((c.A < H1) & (c.K < H2) & (c.V < TH))) continue;
@@ -494,7 +532,8 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
   // pageable source: the call returns once hbuf has been staged, so hbuf may be reused at once
   cudaMemcpyAsync(work, hbuf, hbytes, cudaMemcpyHostToDevice, st);
   const size_t smem = (size_t)(n + 16) * sizeof(ColT<T>) + (size_t)n * sizeof(XT) + (size_t)S * (L + 1) * 8 +
-                      2 * (size_t)(S - 1) * L * 8 + (size_t)(L + 1) * BINOM_K * 8 + (size_t)ny * sizeof(R1YEntry);
+                      2 * (size_t)(S - 1) * L * 8 + (size_t)(L + 1) * BINOM_K * 8 + (size_t)ny * sizeof(R1YEntry) + 16 +
+                      (size_t)(NT / 32) * (n + 16) * sizeof(FoldT<T>);
   cudaFuncSetAttribute(k_search_r1<S, T, NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   int per_sm = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_search_r1<S, T, NT>, NT, smem);
