@@ -33,9 +33,10 @@ UNIT = "evals/s"
 S_STAGES = 8
 TOTAL = comb(95, 7)
 PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
-# integer issue peak: 148 SMs x 4 SMSPs x 32 lanes x 1 instr/clk x sm_max_mhz
+# integer ALU-pipe peak: 148 SMs x 4 SMSPs x 16 lanes/clk (ALU pipe) x sm_max_mhz
 SMS = 148
-LANES_PER_SM_CLK = 128
+ALU_LANES_PER_SM_CLK = 64
+TRAFFIC_PATH = os.path.join(ROOT, "profiles", "round1_traffic.json")
 
 
 def env_int(name, default):
@@ -246,14 +247,13 @@ def main():
         dist.init_process_group("nccl", device_id=dev)
     lo, hi = rank * TOTAL // world, (rank + 1) * TOTAL // world
 
+    from paper_conf_icpp_hulww24_b200.distributed import minloc as dist_minloc
+
     def minloc(T, idx):
         if world == 1:
             return T, idx
-        t = torch.tensor([T if T < (1 << 63) else (1 << 63) - 1], dtype=torch.int64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MIN)
-        i = torch.tensor([idx if T == t.item() else (1 << 63) - 1], dtype=torch.int64, device=dev)
-        dist.all_reduce(i, op=dist.ReduceOp.MIN)
-        return int(t.item()), int(i.item())
+        Tm, Im, _ = dist_minloc(T, idx, 0, device=dev)   # NCCL all_reduce(MIN) x2 (+ SUM)
+        return Tm, Im
 
     def barrier():
         if world > 1:
@@ -345,7 +345,7 @@ def main():
             dist.destroy_process_group()
         return
 
-    # roofline of the dominant kernel (k_search_r1): integer issue bound
+    # roofline of the dominant kernel (k_search_r1): the integer ALU pipe
     peaks = {}
     try:
         with open(PEAKS_PATH) as fh:
@@ -353,15 +353,22 @@ def main():
     except OSError:
         pass
     sm_max = float(peaks.get("sm_max_mhz", 1965.0))
-    peak_ops = SMS * LANES_PER_SM_CLK * sm_max * 1e6 / 1e12       # Tops/s of thread-instructions
+    peak_ops = SMS * ALU_LANES_PER_SM_CLK * sm_max * 1e6 / 1e12       # Tops/s (ALU-pipe int ops)
     ops_per_cand = OPS_PER_CANDIDATE[main_res["int_path"]]
     cands_per_rank = hi - lo
     achieved = ops_per_cand * cands_per_rank / (main_res["kernel_ms"] / 1000.0) / 1e12
+    kname = "k_search_r1<8,%s>" % ("u32" if main_res["int_path"] == 32 else "u64")
+    traffic = None
+    try:
+        with open(TRAFFIC_PATH) as fh:
+            traffic = json.load(fh).get(kname)
+    except (OSError, ValueError):
+        pass
     roofline = {"bound": "alu", "achieved": achieved, "peak": peak_ops, "unit": "Tops/s",
-                "frac": achieved / peak_ops, "traffic": None,
-                "kernel": "k_search_r1<8,%s>" % ("u32" if main_res["int_path"] == 32 else "u64"),
-                "ops_per_candidate": ops_per_cand,
-                "peak_source": "148 SMs x 128 lanes/clk x sm_max_mhz %.0f (MEASURED_PEAKS.json)" % sm_max,
+                "frac": achieved / peak_ops, "traffic": traffic, "traffic_unit": "bytes per launch",
+                "kernel": kname, "ops_per_candidate": ops_per_cand,
+                "peak_source": "derived: 148 SMs x 64 ALU-pipe lanes/clk x sm_max_mhz %.0f "
+                               "(MEASURED_PEAKS.json)" % sm_max,
                 "kernel_ms": main_res["kernel_ms"]}
 
     cpu = None
@@ -395,11 +402,9 @@ def main():
         dist.destroy_process_group()
 
 
-# integer thread-instructions per candidate that the exact decision needs at minimum, per path
-# (one broadcast 128-bit column load, three compares, their AND and the loop
-# counter, amortised over a 4-wide unrolled step: 6 for 32-bit values; 64-bit compares take two
-# instructions each: 9)
-OPS_PER_CANDIDATE = {32: 6, 64: 9}
+# ALU-pipe integer ops the exact per-candidate decision needs: three compares and the
+# two ANDs that combine them; a 64-bit compare is two ALU ops
+OPS_PER_CANDIDATE = {32: 5, 64: 8}
 
 if __name__ == "__main__":
     main()

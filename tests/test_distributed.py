@@ -1,0 +1,109 @@
+"""Multi-process (world size 2, gloo, CPU) tests of the sharded search and the min-loc exchange.
+
+The per-shard search is the oracle's brute force here (CPU); on the GPU it is the CUDA search of the
+shard (tests/test_gpu_parity.py::test_gpt96_shards_match covers 8 shards on one device)."""
+import os
+import socket
+
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    return port
+
+
+class _OracleEngine:
+    """Just the host-side support calls search_distributed needs (count, decode), from the oracle."""
+
+    def __init__(self, L, N):
+        self.L, self.N = L, N
+
+    def count_candidates(self, s_min, s_max, flags):
+        from oracle.enumerate import count
+        return count(self.L, self.N, s_min, s_max, flags)
+
+    def decode_index(self, s_min, s_max, flags, idx):
+        from oracle.enumerate import decode
+        from oracle.model import encode_partition
+        return encode_partition(decode(self.L, self.N, s_min, s_max, flags, idx))
+
+
+def _worker(rank, world, port, q, case):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import workloads as W
+        from oracle.search import brute_force
+        from paper_conf_icpp_hulww24_b200.distributed import minloc, search_distributed
+        from paper_conf_icpp_hulww24_b200.engine import SearchResult
+        if case == "minloc":
+            vals = [(7, 30, 5), (7, 12, 9)] if world == 2 else [(7, 30, 5)]
+            out = [minloc(*vals[rank])]
+            # an empty shard on one rank
+            out.append(minloc(*([(1 << 64) - 1, (1 << 64) - 1, 0], (3, 99, 4))[rank]))
+            q.put((rank, out))
+            return
+        prof, st = W.toy(), W.toy_state()
+        eng = _OracleEngine(prof.L, st.N)
+
+        def shard(b, e):
+            T, idx, part, n = brute_force(prof, st, 1, 4, 0, begin=b, end=e)
+            if n == 0:
+                return SearchResult((1 << 64) - 1, (1 << 64) - 1, 0, bytes([0xFF] * 16))
+            return SearchResult(T, idx, n, b"")
+        r = search_distributed(eng, 1, 4, 0, shard_search=shard)
+        q.put((rank, (r.time_ns, r.index, r.evaluated, r.partition)))
+    finally:
+        dist.destroy_process_group()
+
+
+def _run(world, case):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_worker, args=(r, world, port, q, case)) for r in range(world)]
+    for p in ps:
+        p.start()
+    out = dict(q.get(timeout=240) for _ in range(world))
+    for p in ps:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    return out
+
+
+def test_shard_bounds_cover_exactly():
+    from paper_conf_icpp_hulww24_b200.distributed import shard_bounds
+    for total in (0, 1, 7, 165, 11_050_084_695):
+        for world in (1, 2, 3, 4, 8):
+            prev = 0
+            for r in range(world):
+                lo, hi = shard_bounds(total, r, world)
+                assert lo == prev and hi >= lo
+                prev = hi
+            assert prev == total
+
+
+def test_minloc_gloo_world2():
+    out = _run(2, "minloc")
+    for rank in (0, 1):
+        assert out[rank][0] == (7, 12, 14)          # tie on T: smaller index wins
+        assert out[rank][1] == (3, 99, 4)           # an empty shard never wins
+
+
+def test_search_distributed_gloo_world2_matches_single():
+    from oracle.model import encode_partition
+    from oracle.search import brute_force
+    import workloads as W
+    prof, st = W.toy(), W.toy_state()
+    T, idx, part, n = brute_force(prof, st, 1, 4)
+    out = _run(2, "search")
+    for rank in (0, 1):
+        assert out[rank] == (T, idx, n, encode_partition(part))
