@@ -177,7 +177,7 @@ def run_reference(args, rank: int, world: int):
         return
     import multiprocessing as mp
     ncore = cores()
-    per_step = max(ncore * 8, args.ref_sample)
+    per_step = max(ncore * 150, args.ref_sample)  # ~0.3-0.5 s of oracle work per step
     _oracle_init(args.state)
     pool = mp.get_context("fork").Pool(ncore, initializer=_oracle_init, initargs=(args.state,))
     times = []
