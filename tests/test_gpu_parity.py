@@ -285,3 +285,70 @@ def test_near_overflow_values_exact(eng):
     assert eng.int_path == 64
     recs = [bytes(r) for r in W.sample_records(L, N, 2000, 77)]
     assert gpu_eval(eng, recs) == score_many(prof, st, recs)
+
+
+# ------------------------------------------------------------------------------------------------
+# the hot r = 1 kernel (S >= 5): shards with partial rows and heavy ties, against the eval kernel
+# (itself bit-exact against the oracle) and the parametric DP
+# ------------------------------------------------------------------------------------------------
+
+def _all_records(L, N, smin, smax, flags):
+    from oracle.enumerate import candidates
+    return [encode_partition(p) for p in candidates(L, N, smin, smax, flags)]
+
+
+@pytest.mark.parametrize("S,L,uniform", [(5, 22, False), (6, 24, True), (7, 20, False), (8, 19, True)])
+def test_r1_kernel_shards_and_ties(eng, S, L, uniform):
+    rng = np.random.default_rng(300 + S)
+    if uniform:   # identical layers and workers: huge numbers of exact ties in T
+        prof = W.Profile("u", [1000] * L, [1000] * L, [0] * L, [7] * L, [13] * L)
+        st = W.State([[7] * L] * S, [[13] * L] * S, [[0 if u == v else 5000 for v in range(S)] for u in range(S)])
+    else:
+        prof = W.random_profile(L, rng, f_max=10**6, bytes_max=10**7)
+        st = W.random_state_small(prof, S, rng, tau_max=10**5)
+        st.f = [[x * 1000 for x in row] for row in st.f]
+        st.b = [[x * 1000 for x in row] for row in st.b]
+    eng.load(prof, st)
+    recs = _all_records(L, S, S, S, USE_ALL_WORKERS)       # exactly the r = 1 block
+    times = np.array(gpu_eval(eng, recs), dtype=object)
+    total = len(recs)
+    full = eng.search_optimum(S, S, USE_ALL_WORKERS)
+    T, idx, _ = optimum(prof, st, S, S, USE_ALL_WORKERS)
+    assert (full.time_ns, full.index, full.evaluated) == (T, idx, total)
+    for _ in range(12):
+        b = int(rng.integers(0, total))
+        e = int(rng.integers(b + 1, total + 1))
+        sub = times[b:e]
+        m = min(sub)
+        want = (m, b + list(sub).index(m), e - b)
+        r = eng.search_optimum(S, S, USE_ALL_WORKERS, begin=b, end=e)
+        assert (r.time_ns, r.index, r.evaluated) == want, (b, e)
+
+
+def test_set_state_device_matches_host(eng):
+    prof, st = W.gpt96(), W.gpt_state("b")
+    eng.load(prof, st)
+    host = eng.search_optimum(8, 8, begin=10**9, end=2 * 10**9)
+    dev = torch.device("cuda", 0)
+    as_t = lambda a: torch.tensor(np.asarray(a, dtype=np.uint64).view(np.int64), device=dev)
+    eng.set_state_device(as_t(st.f), as_t(st.b), as_t(st.tau))
+    assert eng.int_path == 64
+    devr = eng.search_optimum(8, 8, begin=10**9, end=2 * 10**9)
+    assert (devr.time_ns, devr.index, devr.evaluated) == (host.time_ns, host.index, host.evaluated)
+    recs = W.sample_records(prof.L, st.N, 500, 5)
+    assert gpu_eval(eng, recs) == score_many(prof, st, [bytes(r) for r in recs])
+
+
+def test_set_state_device_overflow(eng):
+    from paper_conf_icpp_hulww24_b200 import AutopipeError
+    from paper_conf_icpp_hulww24_b200._lib import AUTOPIPE_E_OVERFLOW
+    prof, st = W.toy(), W.toy_state()
+    eng.load(prof, st)
+    dev = torch.device("cuda", 0)
+    big = torch.full((4, 8), 1 << 58, dtype=torch.int64, device=dev)
+    tau = torch.tensor(np.asarray(st.tau, dtype=np.int64), device=dev)
+    eng.set_state_device(big, big, tau)
+    assert gpu_eval(eng, [W.encode(1, [], [0, W.IDLE, W.IDLE, W.IDLE])]) == [U64_MAX]
+    with pytest.raises(AutopipeError) as ex:
+        eng.search_optimum(1, 2)
+    assert ex.value.code == AUTOPIPE_E_OVERFLOW
