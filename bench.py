@@ -223,6 +223,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--ref-sample", type=int, default=0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-configs", action="store_true", help="skip the C1/C2/C3/C5 secondary measurements")
     ap.add_argument("--secondary", default="b", help="extra state measured in the same run ('' = none)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
@@ -371,6 +372,13 @@ def main():
                                "(MEASURED_PEAKS.json)" % sm_max,
                 "kernel_ms": main_res["kernel_ms"]}
 
+    configs = None
+    if world == 1 and not args.no_configs:
+        from tools.bench_configs import measure as measure_configs
+        configs = measure_configs(local)
+        for v in configs.values():
+            v.pop("per_state", None)
+
     cpu = None
     if world == 1 and not args.no_cpu_baseline:
         v, n, dt, nc = oracle_throughput(args.state)
@@ -396,6 +404,7 @@ def main():
         "roofline": roofline,
         "cpu_baseline": cpu,
         "secondary_states": extra,
+        "configs": configs,
     }
     print(json.dumps(line), flush=True)
     if world > 1:

@@ -35,6 +35,7 @@ struct autopipe_ctx {
   BlockOut *d_blocks = nullptr;
   ResultDev *d_result = nullptr;
   void *d_work = nullptr;
+  void *h_work = nullptr;  // pinned mirror of d_work (r = 1 schedules)
   size_t work_bytes = 0;
   // pinned host staging
   u64 *h_stage = nullptr;    // fp | bp | tau(64)
@@ -114,6 +115,7 @@ extern "C" int autopipe_create(int cuda_device, autopipe_ctx **out) {
   if (e == cudaSuccess) e = cudaMalloc(&c->d_result, sizeof(ResultDev));
   c->work_bytes = 1 << 20;
   if (e == cudaSuccess) e = cudaMalloc(&c->d_work, c->work_bytes);
+  if (e == cudaSuccess) e = cudaMallocHost(&c->h_work, c->work_bytes);
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_stage, (2 * MAXN * MAXL + 64) * 8);
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_result, sizeof(ResultDev));
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_status, 2 * sizeof(u64));
@@ -157,6 +159,7 @@ extern "C" void autopipe_destroy(autopipe_ctx *c) {
     if (c->d_blocks) cudaFree(c->d_blocks);
     if (c->d_result) cudaFree(c->d_result);
     if (c->d_work) cudaFree(c->d_work);
+    if (c->h_work) cudaFreeHost(c->h_work);
     if (c->h_stage) cudaFreeHost(c->h_stage);
     if (c->h_result) cudaFreeHost(c->h_result);
     if (c->h_status) cudaFreeHost(c->h_status);
@@ -301,8 +304,10 @@ extern "C" int autopipe_eval_partitions(autopipe_ctx *c, const autopipe_partitio
   if (count == 0) return AUTOPIPE_OK;
   if (!d_parts || !d_time_ns) return fail(c, AUTOPIPE_E_INVAL, "NULL device pointer");
   DeviceGuard dg(c->device);
-  c->launches += launch_eval(c->tab, d_parts, count, (u64 *)d_time_ns, nullptr, nullptr, nullptr, nullptr, c->sms,
-                             (cudaStream_t)stream);
+  // a state given in device memory has not been classified on the host yet: use the 64-bit path
+  const int p32 = c->state_on_device ? 0 : c->path32;
+  c->launches += launch_eval(c->tab, d_parts, count, (u64 *)d_time_ns, nullptr, nullptr, nullptr, nullptr, p32,
+                             c->sms, (cudaStream_t)stream);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "eval kernel launch");
   return AUTOPIPE_OK;
@@ -432,16 +437,16 @@ extern "C" int autopipe_search_optimum(autopipe_ctx *c, uint32_t s_min, uint32_t
       const u64 a = lo, b = hi < r1hi ? hi : r1hi;
       int nb = 0;
       c->launches += launch_search_r1(c->tab, sp, S, a - blo, b - blo, c->path32, c->sms, c->d_blocks + used,
-                                      MAX_BLOCKS - used, &nb, c->d_work, c->work_bytes, st);
+                                      MAX_BLOCKS - used, &nb, c->d_work, c->h_work, c->work_bytes, st);
       used += nb;
       if (b < hi) {
-        c->launches += launch_search_generic(c->tab, sp, b, hi, c->sms, c->d_blocks + used, MAX_BLOCKS - used,
+        c->launches += launch_search_generic(c->tab, sp, b, hi, c->path32, c->sms, c->d_blocks + used, MAX_BLOCKS - used,
                                              &nb, st);
         used += nb;
       }
     } else {
       int nb = 0;
-      c->launches += launch_search_generic(c->tab, sp, lo, hi, c->sms, c->d_blocks + used, MAX_BLOCKS - used,
+      c->launches += launch_search_generic(c->tab, sp, lo, hi, c->path32, c->sms, c->d_blocks + used, MAX_BLOCKS - used,
                                            &nb, st);
       used += nb;
     }
@@ -510,8 +515,9 @@ extern "C" int autopipe_rollout_rewards(autopipe_ctx *c, const autopipe_partitio
   if (count == 0) return AUTOPIPE_OK;
   if (!d_parts || !d_time_ns) return fail(c, AUTOPIPE_E_INVAL, "NULL device pointer");
   DeviceGuard dg(c->device);
+  const int p32 = c->state_on_device ? 0 : c->path32;
   c->launches += launch_eval(c->tab, d_parts, count, (u64 *)d_time_ns, (u64 *)d_switch_bytes, h_current ? &S : nullptr,
-                             &cuts, &masks, c->sms, (cudaStream_t)stream);
+                             &cuts, &masks, p32, c->sms, (cudaStream_t)stream);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "rollout kernel launch");
   return AUTOPIPE_OK;

@@ -10,6 +10,8 @@
 // packed one byte per stage (byte s = bitmask of the workers of stage s). All loops over stages are
 // fully unrolled so every per-stage value lives in registers.
 #pragma once
+#include <type_traits>
+
 #include "common.cuh"
 
 namespace ap {
@@ -98,9 +100,15 @@ __device__ __forceinline__ u64 allreduce_time(u64 Ps, u32 mask, const u64 *tau) 
 }
 
 // The full closed form (rows a4-a7) for one partition; S in [1, 8], the partition already validated.
+// P32: the state's r = 1 bound fits 32 bits (autopipe_set_state), so every stage value X, Y, every
+// boundary sum Z and every segment sum W(s,t) is < 2^32 - 16 and the 28 segment terms use 32-bit
+// adds and divisions by constants; the all-reduce terms (weight bytes) stay 64-bit.
+template <bool P32>
 __device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, u64 cuts, u64 masks) {
-  u64 X[MAXS], Y[MAXS], Zb[MAXS];
-  u64 T = 0;
+  typedef typename std::conditional<P32, u32, u64>::type V;
+  V X[MAXS], Y[MAXS], Zb[MAXS];
+  V T = 0;
+  u64 TAR = 0;
 #pragma unroll
   for (int s = 0; s < MAXS; ++s) {
     X[s] = 0;
@@ -110,21 +118,26 @@ __device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, u64 cut
       const int e = (s == S - 1) ? t.L - 1 : byte_at(cuts, s);
       const u32 mask = (u32)byte_at(masks, s);
       const u32 r = __popc(mask);
-      u64 fm = 0, bm = 0, xm = 0;
       u32 m = mask;
+      // first replica unconditionally; the loop only runs for replicated stages
+      int w = __ffs(m) - 1;
+      m &= m - 1;
+      u64 F = ceil_small(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a], r);
+      u64 B = ceil_small(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a], r);
+      u64 fm = F, bm = B, xm = F + B;
       while (m) {  // row a4: split replicas, ceil(sum / r) per op
-        const int w = __ffs(m) - 1;
+        w = __ffs(m) - 1;
         m &= m - 1;
-        const u64 F = ceil_small(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a], r);
-        const u64 B = ceil_small(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a], r);
+        F = ceil_small(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a], r);
+        B = ceil_small(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a], r);
         fm = umax(fm, F);
         bm = umax(bm, B);
         xm = umax(xm, F + B);
       }
-      X[s] = xm;
-      Y[s] = fm + bm;
-      T = umax(T, xm);
-      if (r >= 2) T = umax(T, allreduce_time(t.PP[e + 1] - t.PP[a], mask, t.tau));
+      X[s] = (V)xm;
+      Y[s] = (V)(fm + bm);
+      T = T > (V)xm ? T : (V)xm;
+      if (r >= 2) TAR = umax(TAR, allreduce_time(t.PP[e + 1] - t.PP[a], mask, t.tau));
     }
   }
 #pragma unroll
@@ -135,26 +148,28 @@ __device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, u64 cut
       const u32 ms = (u32)byte_at(masks, s), mn = (u32)byte_at(masks, s + 1);
       const u64 cf = boundary_max(t.O[e], ms, mn, t.tau);
       const u64 cb = boundary_max(t.G[e + 1], mn, ms, t.tau);
-      Zb[s] = cf + cb;
-      T = umax(T, umax(cf, cb));
+      Zb[s] = (V)(cf + cb);
+      const V lm = (V)umax(cf, cb);
+      T = T > lm ? T : lm;
     }
   }
   Zb[MAXS - 1] = 0;
 #pragma unroll
   for (int s = 0; s < MAXS - 1; ++s) {  // row a7: segment cycles, t-s+1 tokens
     if (s < S - 1) {
-      u64 acc = X[s];
+      V acc = X[s];
 #pragma unroll
       for (int u = s + 1; u < MAXS; ++u) {
         if (u < S) {
-          const u64 W = acc + Zb[u - 1] + X[u];
-          T = umax(T, (W + (u64)(u - s)) / (u64)(u - s + 1));
+          const V W = acc + Zb[u - 1] + X[u];
+          const V c = (W + (V)(u - s)) / (V)(u - s + 1);
+          T = T > c ? T : c;
           acc += Zb[u - 1] + Y[u];
         }
       }
     }
   }
-  return T;
+  return umax((u64)T, TAR);
 }
 
 // Decode + validate a 16-byte record (SPEC.md §2). Returns false for an invalid record.

@@ -24,16 +24,16 @@ struct ResultDev {
 int launch_build_state(const DevTables &g, const u64 *fp, const u64 *bp, const u64 *P, const u64 *tau, u64 sumP,
                        cudaStream_t st);
 int launch_eval(const DevTables &g, const void *recs, u64 count, u64 *out_t, u64 *out_sw,
-                const int *cur_S, const u64 *cur_cuts, const u64 *cur_masks, int sms, cudaStream_t st);
+                const int *cur_S, const u64 *cur_cuts, const u64 *cur_masks, int path32, int sms, cudaStream_t st);
 // Generic exhaustive search over [begin, end) (any S, any composition); writes one BlockOut per block
 // into out[out_offset ...] and returns the number of blocks used via *nblocks.
-int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, u64 end, int sms,
+int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, u64 end, int path32, int sms,
                           BlockOut *out, int max_blocks, int *nblocks, cudaStream_t st);
 // Fast search over the r = 1 block of one S (all stages on one worker; SPEC.md §5, rho = 0),
 // restricted to the cut ranks [k_begin, k_end). path32 selects the 32-bit tables.
 int launch_search_r1(const DevTables &g, const SearchSpace &sp, int S, u64 k_begin, u64 k_end,
                      int path32, int sms, BlockOut *out, int max_blocks, int *nblocks, void *work,
-                     size_t work_bytes, cudaStream_t st);
+                     void *pinned, size_t work_bytes, cudaStream_t st);
 int launch_finalize(const BlockOut *in, int n, const SearchSpace &sp, ResultDev *out, cudaStream_t st);
 
 void upload_binomials(const u64 (*tab)[BINOM_K]);

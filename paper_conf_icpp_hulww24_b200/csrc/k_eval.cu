@@ -17,7 +17,7 @@ struct CurPart {
   int S, valid;
 };
 
-template <bool ROLLOUT>
+template <bool ROLLOUT, bool P32>
 __global__ void __launch_bounds__(256) k_eval(DevTables g, const uint4 *__restrict__ recs, u64 count,
                                               u64 *__restrict__ out_t, u64 *__restrict__ out_sw,
                                               CurPart cur) {
@@ -34,7 +34,7 @@ __global__ void __launch_bounds__(256) k_eval(DevTables g, const uint4 *__restri
     u64 cuts, masks;
     u64 T = U64MAX, sw = U64MAX;
     if (!overflow && decode_record(lo, hi, L, N, S, cuts, masks)) {
-      T = eval_closed_form(t, S, cuts, masks);
+      T = eval_closed_form<P32>(t, S, cuts, masks);
       if (ROLLOUT) sw = switch_bytes(t, S, cuts, masks, cur.S, cur.cuts, cur.masks);
     }
     out_t[i] = T;
@@ -49,7 +49,7 @@ static int grid_for(u64 count, int sms) {
 }
 
 int launch_eval(const DevTables &g, const void *recs, u64 count, u64 *out_t, u64 *out_sw,
-                const int *cur_S, const u64 *cur_cuts, const u64 *cur_masks, int sms, cudaStream_t st) {
+                const int *cur_S, const u64 *cur_cuts, const u64 *cur_masks, int path32, int sms, cudaStream_t st) {
   if (count == 0) return 0;
   const size_t smem = (size_t)smem_words(g.L, g.N) * sizeof(u64);
   CurPart cur{0, 0, 0, 0};
@@ -60,10 +60,13 @@ int launch_eval(const DevTables &g, const void *recs, u64 count, u64 *out_t, u64
     cur.valid = 1;
   }
   const int grid = grid_for(count, sms);
-  if (out_sw)
-    k_eval<true><<<grid, 256, smem, st>>>(g, (const uint4 *)recs, count, out_t, out_sw, cur);
-  else
-    k_eval<false><<<grid, 256, smem, st>>>(g, (const uint4 *)recs, count, out_t, nullptr, cur);
+  if (out_sw) {
+    if (path32) k_eval<true, true><<<grid, 256, smem, st>>>(g, (const uint4 *)recs, count, out_t, out_sw, cur);
+    else k_eval<true, false><<<grid, 256, smem, st>>>(g, (const uint4 *)recs, count, out_t, out_sw, cur);
+  } else {
+    if (path32) k_eval<false, true><<<grid, 256, smem, st>>>(g, (const uint4 *)recs, count, out_t, nullptr, cur);
+    else k_eval<false, false><<<grid, 256, smem, st>>>(g, (const uint4 *)recs, count, out_t, nullptr, cur);
+  }
   return 1;
 }
 

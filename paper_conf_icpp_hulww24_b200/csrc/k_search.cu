@@ -50,11 +50,26 @@ __device__ __forceinline__ void unrank_global(const SearchSpace &sp, u64 idx, in
   cuts = lex_unrank_packed(kappa, S - 1, sp.L - 1);
 }
 
-template <int NT>
+// same, against a binomial table in shared memory (fixed-length binary searches, no divergence)
+__device__ __forceinline__ void unrank_global_smem(const SearchSpace &sp, u64 idx, int &S, u64 &Rp, u64 &cuts,
+                                                   const u64 *Bn) {
+  S = sp.s_min;
+  while (S < sp.s_max && idx >= sp.off[S + 1]) ++S;
+  const u64 rem = idx - sp.off[S];
+  const u64 rho = rem / sp.ncut[S], kappa = rem % sp.ncut[S];
+  Rp = lex_unrank_smem(rho, comp_k(sp, S), comp_n(sp), Bn);
+  cuts = lex_unrank_smem(kappa, S - 1, sp.L - 1, Bn);
+}
+
+template <int NT, bool P32>
 __global__ void __launch_bounds__(NT) k_search_generic(DevTables g, SearchSpace sp, u64 begin, u64 end,
                                                        u64 per_thread, BlockOut *out) {
   extern __shared__ u64 sm[];
-  const SmemTab t = stage_tables(g, sm);
+  // binomial rows n <= L (n = N <= 8 <= L + 1 for the compositions too) after the state tables
+  u64 *Bn = sm + smem_words(g.L, g.N);
+  const int nb = ((int)g.L + 1 > 9 ? (int)g.L + 1 : 9) * BINOM_K;
+  for (int i = threadIdx.x; i < nb; i += NT) Bn[i] = c_binom[i / BINOM_K][i % BINOM_K];
+  const SmemTab t = stage_tables(g, sm);  // ends with __syncthreads()
   const u64 gtid = (u64)blockIdx.x * NT + threadIdx.x;
   u64 bestT = U64MAX, bestI = U64MAX, cnt = 0;
   const u64 span = end - begin;
@@ -63,10 +78,10 @@ __global__ void __launch_bounds__(NT) k_search_generic(DevTables g, SearchSpace 
     const u64 i1 = (end - i0 < per_thread) ? end : i0 + per_thread;
     int S;
     u64 Rp, cuts;
-    unrank_global(sp, i0, S, Rp, cuts);
+    unrank_global_smem(sp, i0, S, Rp, cuts, Bn);
     u64 masks = masks_from(sp, S, Rp);
     for (u64 i = i0; i < i1; ++i) {
-      const u64 T = eval_closed_form(t, S, cuts, masks);
+      const u64 T = eval_closed_form<P32>(t, S, cuts, masks);
       if (T < bestT) {  // indices increase along the thread's range: strict < keeps the first
         bestT = T;
         bestI = i;
@@ -88,19 +103,22 @@ __global__ void __launch_bounds__(NT) k_search_generic(DevTables g, SearchSpace 
   block_minloc_store<NT>(bestT, bestI, cnt, out + blockIdx.x);
 }
 
-int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, u64 end, int sms,
+int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, u64 end, int path32, int sms,
                           BlockOut *out, int max_blocks, int *nblocks, cudaStream_t st) {
   constexpr int NT = 256;
   const u64 span = end - begin;
-  // at least 8 candidates per thread; at most 4 blocks per SM (persistent)
-  u64 threads = (span + 7) / 8;
+  // at least 4 candidates per thread (the unrank is a few binary searches); up to 8 blocks per SM
+  u64 threads = (span + 3) / 4;
   u64 blocks = (threads + NT - 1) / NT;
-  const u64 cap = (u64)sms * 4 < (u64)max_blocks ? (u64)sms * 4 : (u64)max_blocks;
+  const u64 cap = (u64)sms * 8 < (u64)max_blocks ? (u64)sms * 8 : (u64)max_blocks;
   if (blocks > cap) blocks = cap;
   if (blocks == 0) blocks = 1;
   const u64 per = (span + blocks * NT - 1) / (blocks * NT);
-  const size_t smem = (size_t)smem_words(g.L, g.N) * sizeof(u64);
-  k_search_generic<NT><<<(unsigned)blocks, NT, smem, st>>>(g, sp, begin, end, per ? per : 1, out);
+  const size_t smem = ((size_t)smem_words(g.L, g.N) + (size_t)((g.L + 1 > 9 ? g.L + 1 : 9) * BINOM_K)) * sizeof(u64);
+  if (path32)
+    k_search_generic<NT, true><<<(unsigned)blocks, NT, smem, st>>>(g, sp, begin, end, per ? per : 1, out);
+  else
+    k_search_generic<NT, false><<<(unsigned)blocks, NT, smem, st>>>(g, sp, begin, end, per ? per : 1, out);
   *nblocks = (int)blocks;
   return 1;
 }

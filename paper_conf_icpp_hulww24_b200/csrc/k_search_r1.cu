@@ -478,14 +478,16 @@ static u64 count_less(int x, int k, const int *t) {
 
 template <int S, typename T>
 static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u64 k_end, int sms,
-                       BlockOut *out, int max_blocks, int *nblocks, void *work, size_t work_bytes,
+                       BlockOut *out, int max_blocks, int *nblocks, void *work, void *pinned, size_t work_bytes,
                        cudaStream_t st) {
   constexpr int P = S - 4, NT = 256;
   const int L = (int)g.L, n = L - 1, k = S - 1;
   int lo[8], hi[8];
   host_unrank(k_begin, k, n, lo);
   host_unrank(k_end - 1, k, n, hi);
-  static thread_local unsigned char hbuf[sizeof(R1Header) + 256 * sizeof(R1YEntry)];
+  // schedule staged in the context's pinned buffer (one 16 KB slot per S, like the device work area),
+  // so the copy below is a true async DMA and never waits for earlier work on the stream
+  unsigned char *hbuf = (unsigned char *)pinned + (size_t)S * 16384;
   R1Header *h = (R1Header *)hbuf;
   R1YEntry *yt = (R1YEntry *)(hbuf + sizeof(R1Header));
   memset(h, 0, sizeof(*h));
@@ -529,7 +531,6 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
   // one 16 KB slot per S, so the launches of one search never share a schedule buffer
   if ((size_t)(S + 1) * 16384 > work_bytes || hbytes > 16384) return 0;
   work = (unsigned char *)work + (size_t)S * 16384;
-  // pageable source: the call returns once hbuf has been staged, so hbuf may be reused at once
   cudaMemcpyAsync(work, hbuf, hbytes, cudaMemcpyHostToDevice, st);
   const size_t smem = (size_t)(n + 16) * sizeof(ColT<T>) + (size_t)n * sizeof(XT) + (size_t)S * (L + 1) * 8 +
                       2 * (size_t)(S - 1) * L * 8 + (size_t)(L + 1) * BINOM_K * 8 + (size_t)ny * sizeof(R1YEntry) + 16 +
@@ -551,23 +552,23 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
 
 template <typename T>
 static int launch_r1_s(int S, const DevTables &g, const SearchSpace &sp, u64 a, u64 b, int sms, BlockOut *out,
-                       int mb, int *nb, void *w, size_t wb, cudaStream_t st) {
+                       int mb, int *nb, void *w, void *pin, size_t wb, cudaStream_t st) {
   switch (S) {
-    case 5: return launch_r1_t<5, T>(g, sp, a, b, sms, out, mb, nb, w, wb, st);
-    case 6: return launch_r1_t<6, T>(g, sp, a, b, sms, out, mb, nb, w, wb, st);
-    case 7: return launch_r1_t<7, T>(g, sp, a, b, sms, out, mb, nb, w, wb, st);
-    case 8: return launch_r1_t<8, T>(g, sp, a, b, sms, out, mb, nb, w, wb, st);
+    case 5: return launch_r1_t<5, T>(g, sp, a, b, sms, out, mb, nb, w, pin, wb, st);
+    case 6: return launch_r1_t<6, T>(g, sp, a, b, sms, out, mb, nb, w, pin, wb, st);
+    case 7: return launch_r1_t<7, T>(g, sp, a, b, sms, out, mb, nb, w, pin, wb, st);
+    case 8: return launch_r1_t<8, T>(g, sp, a, b, sms, out, mb, nb, w, pin, wb, st);
   }
   *nb = 0;
   return 0;
 }
 
 int launch_search_r1(const DevTables &g, const SearchSpace &sp, int S, u64 k_begin, u64 k_end, int path32,
-                     int sms, BlockOut *out, int max_blocks, int *nblocks, void *work, size_t work_bytes,
-                     cudaStream_t st) {
+                     int sms, BlockOut *out, int max_blocks, int *nblocks, void *work, void *pinned,
+                     size_t work_bytes, cudaStream_t st) {
   if (path32)
-    return launch_r1_s<u32>(S, g, sp, k_begin, k_end, sms, out, max_blocks, nblocks, work, work_bytes, st);
-  return launch_r1_s<u64>(S, g, sp, k_begin, k_end, sms, out, max_blocks, nblocks, work, work_bytes, st);
+    return launch_r1_s<u32>(S, g, sp, k_begin, k_end, sms, out, max_blocks, nblocks, work, pinned, work_bytes, st);
+  return launch_r1_s<u64>(S, g, sp, k_begin, k_end, sms, out, max_blocks, nblocks, work, pinned, work_bytes, st);
 }
 
 }  // namespace ap

@@ -1,0 +1,88 @@
+#!/usr/bin/env python
+"""Secondary measurements on the other BASELINE.json configs (1 GPU, device-timed with CUDA events):
+
+  C1 toy       exhaustive search of the 165-candidate space
+  C2 VGG-16    exhaustive search (1,184,040 candidates, replicas, heterogeneous links)
+  C3 GNMT-16 / BERT-24 state trace: per state switch, set_state + full search (re-score latency)
+  C5 ResNet-50 rollouts: 1M random records per step, eval and rollout (T + switch bytes)
+
+Used by bench.py (key "configs") and runnable on its own.
+"""
+import json
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+
+def _timed(fn, reps=5, warm=2):
+    import torch
+    for _ in range(warm):
+        fn()
+    torch.cuda.synchronize()
+    out = []
+    for _ in range(reps):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        r = fn()
+        b.record()
+        torch.cuda.synchronize()
+        out.append(a.elapsed_time(b))
+    return sum(out) / len(out), r
+
+
+def measure(device: int = 0, rollout_records: int = 1 << 20):
+    import torch
+    import workloads as W
+    from paper_conf_icpp_hulww24_b200 import Engine
+    eng = Engine(device)
+    res = {}
+    # C1 / C2: exhaustive searches
+    for name, prof, st, smax in (("C1_toy", W.toy(), W.toy_state(), 4), ("C2_vgg16", W.vgg16(), W.vgg_state(), 8)):
+        eng.load(prof, st)
+        n = eng.count_candidates(1, smax)
+        ms, r = _timed(lambda: eng.search_optimum(1, smax))
+        res[name] = {"candidates": n, "ms_to_optimum": ms, "evals_per_s": n / (ms / 1e3),
+                     "optimum_T_ns": r.time_ns, "optimum_index": r.index, "int_path": eng.int_path}
+    # C3: state traces, re-score latency per switch (state copy + state kernel + search)
+    for name in ("gnmt16", "bert24"):
+        prof = W.profile(name)
+        eng.load_profile(prof.O, prof.G, prof.P)
+        per = []
+        for st in W.trace_c3(prof):
+            smax = min(8, st.N)
+
+            def step(st=st, smax=smax):
+                eng.set_state(st.f, st.b, st.tau)
+                return eng.search_optimum(1, smax)
+            ms, r = _timed(step, reps=3, warm=1)
+            n = eng.count_candidates(1, smax)
+            per.append({"state": st.label, "N": st.N, "candidates": n, "ms": ms, "T_ns": r.time_ns,
+                        "index": r.index})
+        res["C3_" + name] = {"states": len(per), "mean_rescore_ms": sum(p["ms"] for p in per) / len(per),
+                             "max_rescore_ms": max(p["ms"] for p in per), "per_state": per}
+    # C5: rollouts
+    prof = W.resnet50()
+    st = W.rollout_state(prof, 0)
+    eng.load(prof, st)
+    recs = torch.from_numpy(W.sample_records(prof.L, st.N, rollout_records, 1000)).cuda()
+    cur = bytes(recs[0].cpu().numpy())
+    out_t = torch.empty(rollout_records, dtype=torch.int64, device="cuda")
+    out_s = torch.empty_like(out_t)
+    ms_e, _ = _timed(lambda: eng.eval_partitions(recs, out=out_t))
+    ms_r, _ = _timed(lambda: eng.rollout_rewards(recs, cur, out_t=out_t, out_sw=out_s))
+    res["C5_resnet50_rollout"] = {"records": rollout_records, "eval_ms": ms_e,
+                                  "eval_records_per_s": rollout_records / (ms_e / 1e3),
+                                  "rollout_ms": ms_r, "rollout_records_per_s": rollout_records / (ms_r / 1e3),
+                                  "eval_GBps_algorithmic": rollout_records * 24 / (ms_e / 1e3) / 1e9,
+                                  "int_path": eng.int_path}
+    eng.close()
+    return res
+
+
+if __name__ == "__main__":
+    import __graft_entry__
+    __graft_entry__.build()
+    print(json.dumps(measure()))
