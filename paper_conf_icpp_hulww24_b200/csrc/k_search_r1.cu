@@ -382,49 +382,92 @@ __global__ void __launch_bounds__(NT, 2) k_search_r1(DevTables g, const R1Header
       // ---- x sweep (warp-uniform), then the hot column sweep -------------------------------
       constexpr unsigned FS = sizeof(FoldT<T>);
       const unsigned aend = fb + (unsigned)(L - 1) * FS;  // one past the column e = L-2
-      for (int x = y + 1; x <= L - 3; ++x) {
-        const XT xv = xt[x];
-        T H1, H2;
-        xu.x(xv, H1, H2);
-#ifndef AP_SWEEP
-#define AP_SWEEP 4
-#endif
-        // AP_SWEEP columns per step (sentinel-padded, no tail code), one LDS per column
-        unsigned a = fb + (unsigned)(x + 1) * FS;
-        for (; a < aend; a += AP_SWEEP * FS) {
+      // Rare path: candidate (xk, ee) passed the filter; decide it exactly. Afterwards every later
+      // candidate of this lane in index order is larger, so theta becomes strict (best - 1) and the
+      // row terms are recomputed (the caller refreshes its slots' thresholds).
+      auto rare = [&](int xk, int ee, const ColT<T> &c, const T h1, const T h2) -> bool {
+        if (!((c.A < h1) & (c.K < h2) & (c.V < TH))) return false;
+        if (lo_part && (xk < hdr.lo_x || (xk == hdr.lo_x && ee < hdr.lo_e))) return false;
+        if (hi_part && (xk > hdr.hi_x || (xk == hdr.hi_x && ee > hdr.hi_e))) return false;
+        const u64 cuts = pre | ((u64)y << (8 * P)) | ((u64)xk << (8 * (P + 1))) | ((u64)ee << (8 * (P + 2)));
+        const u64 Tc = exact_T_r1<S>(PC, Z, LM, L, cuts);
+        const u64 idx = hdr.off + lex_rank_smem(cuts, S - 1, n, Bn);
+        if (better(Tc, idx, bestT, bestI)) {
+          bestT = Tc;
+          bestI = idx;
+        }
+        strict = true;
+        th = (i64)bestT - 1;
+        row_base<S>(PC, Z, LM, L, pre, th, base);
+        aliveP = row_finish<S>(base, PC, Z, LM, L, byte_at(pre, P - 1), y, th, N0, N1, N2);
+        xu.row(th, aliveP, N0, N1, N2, pcy);
+        TH = xu.TH();
+        return true;
+      };
+      // single-x sweep from column address a0 (used for the second x of a pair after it hit)
+      auto sweep1 = [&](int xk, const XT &xv, T &H1, T &H2, unsigned a0) {
+        for (unsigned a = a0; a < aend; a += 4 * FS) {
           bool hit = false;
 #pragma unroll
-          for (int u = 0; u < AP_SWEEP; ++u) {
+          for (int u = 0; u < 4; ++u) {
             T A0, K0;
             lds_fold(a + u * FS, A0, K0);
             hit |= (A0 < H1) & (K0 < H2);
           }
           if (hit) {
-            // rare path: the columns of this step in order, with the current thresholds
             const int e = (int)((a - fb) / FS);
-            for (int ee = e; ee < e + AP_SWEEP; ++ee) {
-              const ColT<T> c = col[ee];
-              if (!((c.A < H1) & (c.K < H2) & (c.V < TH))) continue;
-              if (lo_part && (x < hdr.lo_x || (x == hdr.lo_x && ee < hdr.lo_e))) continue;
-              if (hi_part && (x > hdr.hi_x || (x == hdr.hi_x && ee > hdr.hi_e))) continue;
-              const u64 cuts = pre | ((u64)y << (8 * P)) | ((u64)x << (8 * (P + 1))) | ((u64)ee << (8 * (P + 2)));
-              const u64 Tc = exact_T_r1<S>(PC, Z, LM, L, cuts);
-              const u64 idx = hdr.off + lex_rank_smem(cuts, S - 1, n, Bn);
-              if (better(Tc, idx, bestT, bestI)) {
-                bestT = Tc;
-                bestI = idx;
-              }
-              // later candidates of this lane have larger indices: strict from here on
-              strict = true;
-              th = (i64)bestT - 1;
-              row_base<S>(PC, Z, LM, L, pre, th, base);
-              aliveP = row_finish<S>(base, PC, Z, LM, L, byte_at(pre, P - 1), y, th, N0, N1, N2);
-              xu.row(th, aliveP, N0, N1, N2, pcy);
-              xu.x(xv, H1, H2);
-              TH = xu.TH();
+            for (int ee = e; ee < e + 4; ++ee)
+              if (rare(xk, ee, col[ee], H1, H2)) xu.x(xv, H1, H2);
+          }
+        }
+      };
+      // Two x values per pass: x and x+1 test the same columns e > x+1, so one broadcast load serves
+      // two candidates and the two compare chains are independent. Hits of x are decided at once; a
+      // hit of x+1 only records where its rescan starts, and x+1 is rescanned after x is finished,
+      // so candidates are always decided in increasing index order (tie-break, reading C-13).
+      for (int x = y + 1; x <= L - 3; x += 2) {
+        const bool two = x + 1 <= L - 3;
+        const XT xva = xt[x];
+        const XT xvb = xt[two ? x + 1 : x];
+        T H1a, H2a, H1b, H2b;
+        xu.x(xva, H1a, H2a);
+        xu.x(xvb, H1b, H2b);
+        if (!two) H1b = H2b = (T)0;
+        {  // column x+1 belongs to x only
+          const unsigned a1 = fb + (unsigned)(x + 1) * FS;
+          T A0, K0;
+          lds_fold(a1, A0, K0);
+          if ((A0 < H1a) & (K0 < H2a)) {
+            if (rare(x, x + 1, col[x + 1], H1a, H2a)) {
+              xu.x(xva, H1a, H2a);
+              if (two) xu.x(xvb, H1b, H2b);
             }
           }
         }
+        unsigned firstb = 0xFFFFFFFFu;
+        for (unsigned a = fb + (unsigned)(x + 2) * FS; a < aend; a += 4 * FS) {
+          bool ha = false, hb = false;
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            T A0, K0;
+            lds_fold(a + u * FS, A0, K0);
+            ha |= (A0 < H1a) & (K0 < H2a);
+            hb |= (A0 < H1b) & (K0 < H2b);
+          }
+          if (ha | hb) {
+            if (ha) {
+              const int e = (int)((a - fb) / FS);
+              for (int ee = e; ee < e + 4; ++ee) {
+                if (rare(x, ee, col[ee], H1a, H2a)) {
+                  xu.x(xva, H1a, H2a);
+                  if (two) xu.x(xvb, H1b, H2b);
+                }
+              }
+            }
+            if (hb && firstb == 0xFFFFFFFFu) firstb = a;
+          }
+        }
+        if (firstb != 0xFFFFFFFFu) sweep1(x + 1, xvb, H1b, H2b, firstb);
       }
       // ---- next row of this lane: lexicographic successor of the prefix below y ------------
       // usually only the last prefix cut moves (+1): the base (stages 0..P-2) stays valid
