@@ -61,6 +61,28 @@ __device__ __forceinline__ u64 div_small(u64 x, u32 d) {
 }
 __device__ __forceinline__ u64 ceil_small(u64 x, u32 d) { return div_small(x + d - 1, d); }
 
+// The same division with the multiplier chosen once per divisor (hoisted out of loops over replicas
+// and shards). d in [1, 8]; x < 2^63.
+struct Div8 {
+  u64 m;
+  u32 sh, d;
+  __device__ __forceinline__ explicit Div8(u32 d_) : d(d_) {
+    m = (d == 3u || d == 6u) ? 0xaaaaaaaaaaaaaaabull
+      : (d == 5u)            ? 0xcccccccccccccccdull
+      : (d == 7u)            ? 0x924924924924924aull
+                             : 0x8000000000000000ull;
+    sh = (d <= 2u) ? 0u : (d <= 4u) ? 1u : 2u;
+  }
+  __device__ __forceinline__ u64 div(u64 x) const { return d == 1u ? x : (__umul64hi(x, m) >> sh); }
+  __device__ __forceinline__ u64 ceil(u64 x) const { return div(x + d - 1); }
+  // floor(k / d) for 0 <= k < 64: (k * ceil(2^16 / d)) >> 16 is exact on that range
+  __device__ __forceinline__ u32 small(u32 k) const {
+    const u32 M = (d == 1u) ? 65536u : (d == 2u) ? 32768u : (d == 3u) ? 21846u : (d == 4u) ? 16384u
+                : (d == 5u) ? 13108u : (d == 6u) ? 10923u : (d == 7u) ? 9363u : 8192u;
+    return (k * M) >> 16;
+  }
+};
+
 __device__ __forceinline__ int byte_at(u64 v, int i) { return (int)((v >> (8 * i)) & 0xFF); }
 
 // Lexicographic (time, index) minimum used by every argmin (reading C-13: smallest index wins ties).

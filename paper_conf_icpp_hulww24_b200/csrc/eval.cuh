@@ -58,10 +58,14 @@ __device__ __forceinline__ u64 boundary_max(u64 A, u32 send, u32 recv, const u64
     const int u = __ffs(send) - 1, v = __ffs(recv) - 1;
     return xfer(A, tau[u * 8 + v]);
   }
+  // shard boundaries floor(i A / r) = i q + floor(i rem / r) with A = q r + rem (rem < r <= 8, i <= 8)
+  const Div8 ds(rs), dr(rr);
+  const u64 qs = ds.div(A), qr = dr.div(A);
+  const u32 rems = (u32)(A - qs * rs), remr = (u32)(A - qr * rr);
   u64 best = 0;
   u32 i = 0, j = 0;
   u64 lo_i = 0, lo_j = 0;
-  u64 hi_i = div_small(A, rs), hi_j = div_small(A, rr);
+  u64 hi_i = qs + ds.small(rems), hi_j = qr + dr.small(remr);
   while (i < rs && j < rr) {
     const u64 lo = umax(lo_i, lo_j), hi = umin(hi_i, hi_j);
     if (hi > lo) {
@@ -71,11 +75,11 @@ __device__ __forceinline__ u64 boundary_max(u64 A, u32 send, u32 recv, const u64
     const bool adv_i = hi_i <= hi_j, adv_j = hi_j <= hi_i;
     if (adv_i) {
       ++i; send &= send - 1;
-      lo_i = hi_i; hi_i = div_small((u64)(i + 1) * A, rs);
+      lo_i = hi_i; hi_i = (u64)(i + 1) * qs + ds.small((i + 1) * rems);
     }
     if (adv_j) {
       ++j; recv &= recv - 1;
-      lo_j = hi_j; hi_j = div_small((u64)(j + 1) * A, rr);
+      lo_j = hi_j; hi_j = (u64)(j + 1) * qr + dr.small((j + 1) * remr);
     }
   }
   return best;
@@ -96,7 +100,7 @@ __device__ __forceinline__ u64 allreduce_time(u64 Ps, u32 mask, const u64 *tau) 
     prev = w;
   }
   tr = umax(tr, tau[prev * 8 + first]);
-  return 2ull * (u64)(r - 1) * xfer(ceil_small(Ps, r), tr);
+  return 2ull * (u64)(r - 1) * xfer(Div8(r).ceil(Ps), tr);
 }
 
 // The full closed form (rows a4-a7) for one partition; S in [1, 8], the partition already validated.
@@ -118,18 +122,19 @@ __device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, u64 cut
       const int e = (s == S - 1) ? t.L - 1 : byte_at(cuts, s);
       const u32 mask = (u32)byte_at(masks, s);
       const u32 r = __popc(mask);
+      const Div8 dv(r);
       u32 m = mask;
       // first replica unconditionally; the loop only runs for replicated stages
       int w = __ffs(m) - 1;
       m &= m - 1;
-      u64 F = ceil_small(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a], r);
-      u64 B = ceil_small(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a], r);
+      u64 F = dv.ceil(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a]);
+      u64 B = dv.ceil(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a]);
       u64 fm = F, bm = B, xm = F + B;
       while (m) {  // row a4: split replicas, ceil(sum / r) per op
         w = __ffs(m) - 1;
         m &= m - 1;
-        F = ceil_small(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a], r);
-        B = ceil_small(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a], r);
+        F = dv.ceil(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a]);
+        B = dv.ceil(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a]);
         fm = umax(fm, F);
         bm = umax(bm, B);
         xm = umax(xm, F + B);
