@@ -163,3 +163,48 @@ def test_long_transient_uses_cycle_ratio():
     lam = simulate(prof, st, part, max_rounds=100_000)
     assert lam == 207_874_737
     assert time_ns(prof, st, part) == 207_874_737
+
+
+# --------------------------------------------------------------------------------------------
+# the two-worker neighbourhood, by definition
+# --------------------------------------------------------------------------------------------
+
+def test_neighbourhood_by_hand():
+    """L = 3 layers, N = 2 workers, p = stage [0] on w0, stage [1,2] on w1. With two workers every
+    other valid partition differs in at most two entries of the per-worker layer array, so the
+    neighbourhood is all six others (derived by hand in oracle/neighbourhood.py's docstring terms)."""
+    from oracle.model import Partition, encode_partition
+    from oracle.neighbourhood import all_partitions, neighbourhood
+    p = Partition(2, [0], [[0], [1]])
+    want = sorted([
+        W.encode(1, [], [0, 0]), W.encode(1, [], [0, W.IDLE]), W.encode(1, [], [W.IDLE, 0]),
+        W.encode(2, [0], [1, 0]), W.encode(2, [1], [0, 1]), W.encode(2, [1], [1, 0]),
+    ])
+    assert neighbourhood(3, 2, p) == want
+    assert len(list(all_partitions(3, 2))) == 7
+
+
+def test_neighbourhood_distance_one_moves():
+    """L = 2, N = 3, p = one stage on w0 (w1, w2 idle). Single-worker changes: w1 or w2 joins the
+    stage (w0 cannot change alone: the layers would be uncovered)."""
+    from oracle.model import Partition, encode_partition
+    from oracle.neighbourhood import layer_sets, neighbourhood
+    p = Partition(1, [], [[0]])
+    nb = neighbourhood(2, 3, p)
+    from oracle.model import parse_record
+    d1 = [r for r in nb if sum(a != b for a, b in zip(layer_sets(parse_record(r, 2, 3), 2, 3),
+                                                       layer_sets(p, 2, 3))) == 1]
+    assert sorted(d1) == sorted([W.encode(1, [], [0, 0, W.IDLE]), W.encode(1, [], [0, W.IDLE, 0])])
+
+
+def test_neighbourhood_symmetric():
+    from oracle.model import parse_record
+    from oracle.neighbourhood import all_partitions, neighbourhood
+    from oracle.model import encode_partition
+    L, N = 4, 3
+    parts = list(all_partitions(L, N))
+    nbs = {encode_partition(p): set(neighbourhood(L, N, p)) for p in parts[::3]}
+    for a, na in nbs.items():
+        for b in na:
+            if b in nbs:
+                assert a in nbs[b]
