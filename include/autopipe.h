@@ -138,6 +138,24 @@ int autopipe_rollout_rewards(autopipe_ctx *ctx, const autopipe_partition *d_part
                              const autopipe_partition *h_current, uint64_t *d_time_ns,
                              uint64_t *d_switch_bytes, void *stream);
 
+/* NEXT row f1 — the two-worker neighbourhood ("we limit the new partition solution
+ * to only change the two workers' tasks in comparison to the old one"; the partition is the
+ * per-worker array of assigned layers). Reading F-1: the neighbourhood
+ * of *h_current is every valid partition whose per-worker layer-set array differs from the current
+ * one in one or two entries (a worker joining/leaving a stage, a boundary moved between two workers'
+ * stages, a stage split between two workers, two workers exchanging stages, ...).
+ *   autopipe_neighbourhood: writes the neighbours (canonical records, deterministic order) to the
+ *     device array d_out[capacity] and their number to *h_count (which may exceed capacity: only the
+ *     first `capacity` are written). Synchronous.
+ *   autopipe_neighbourhood_best: scores every neighbour with the cost model and returns the minimum
+ *     of (time_ns, record bytes) in *h_out (index = UINT64_MAX, evaluated = neighbourhood size;
+ *     time_ns = UINT64_MAX if the neighbourhood is empty). Synchronous.
+ * An invalid *h_current -> E_INVAL; requires a state (E_STATE). */
+int autopipe_neighbourhood(autopipe_ctx *ctx, const autopipe_partition *h_current, autopipe_partition *d_out,
+                           uint64_t capacity, uint64_t *h_count, void *stream);
+int autopipe_neighbourhood_best(autopipe_ctx *ctx, const autopipe_partition *h_current, autopipe_result *h_out,
+                                void *stream);
+
 /* Number of candidates of a search space (requires a state for L and N). */
 int autopipe_count_candidates(const autopipe_ctx *ctx, uint32_t s_min, uint32_t s_max, uint32_t flags,
                               uint64_t *total);

@@ -59,10 +59,10 @@ def best_neighbour(prof, st, current_rec: bytes) -> Tuple[int, bytes, int]:
     cur = parse_record(current_rec, L, N)
     if cur is None:
         raise ValueError("invalid current partition")
-    best = None
+    best = ((1 << 64) - 1, bytes([0xFF] * 16))  # an empty neighbourhood (one worker, one stage)
     recs = neighbourhood(L, N, cur)
     for rec in recs:
         T = time_ns(prof, st, parse_record(rec, L, N))
-        if best is None or (T, rec) < best:
+        if (T, rec) < best:
             best = (T, rec)
     return best[0], best[1], len(recs)

@@ -35,6 +35,8 @@ struct autopipe_ctx {
   BlockOut *d_blocks = nullptr;
   ResultDev *d_result = nullptr;
   void *d_work = nullptr;
+  void *d_nslots = nullptr;  // neighbourhood slots (records), times, count
+  u64 *d_ntimes = nullptr, *d_ncount = nullptr, *h_ncount = nullptr;
   void *h_work = nullptr;  // pinned mirror of d_work (r = 1 schedules)
   size_t work_bytes = 0;
   // pinned host staging
@@ -116,6 +118,10 @@ extern "C" int autopipe_create(int cuda_device, autopipe_ctx **out) {
   c->work_bytes = 1 << 20;
   if (e == cudaSuccess) e = cudaMalloc(&c->d_work, c->work_bytes);
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_work, c->work_bytes);
+  if (e == cudaSuccess) e = cudaMalloc(&c->d_nslots, (size_t)NEIGH_ITEMS * NEIGH_MAXOPT * 16);
+  if (e == cudaSuccess) e = cudaMalloc(&c->d_ntimes, (size_t)NEIGH_ITEMS * NEIGH_MAXOPT * 8);
+  if (e == cudaSuccess) e = cudaMalloc(&c->d_ncount, 8);
+  if (e == cudaSuccess) e = cudaMallocHost(&c->h_ncount, 8);
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_stage, (2 * MAXN * MAXL + 64) * 8);
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_result, sizeof(ResultDev));
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_status, 2 * sizeof(u64));
@@ -160,6 +166,10 @@ extern "C" void autopipe_destroy(autopipe_ctx *c) {
     if (c->d_result) cudaFree(c->d_result);
     if (c->d_work) cudaFree(c->d_work);
     if (c->h_work) cudaFreeHost(c->h_work);
+    if (c->d_nslots) cudaFree(c->d_nslots);
+    if (c->d_ntimes) cudaFree(c->d_ntimes);
+    if (c->d_ncount) cudaFree(c->d_ncount);
+    if (c->h_ncount) cudaFreeHost(c->h_ncount);
     if (c->h_stage) cudaFreeHost(c->h_stage);
     if (c->h_result) cudaFreeHost(c->h_result);
     if (c->h_status) cudaFreeHost(c->h_status);
@@ -547,3 +557,61 @@ extern "C" int autopipe_set_timing(autopipe_ctx *c, int enable) {
 }
 
 extern "C" double autopipe_last_search_ms(const autopipe_ctx *c) { return c ? c->last_search_ms : -1.0; }
+
+// --- NEXT row f1: the two-worker neighbourhood (reading F-1) ----------------
+static int neigh_prepare(autopipe_ctx *c, const autopipe_partition *h_current, u64 &nslots, cudaStream_t st) {
+  if (!c->has_state) return fail(c, AUTOPIPE_E_STATE, "neighbourhood before set_state");
+  if (!h_current) return fail(c, AUTOPIPE_E_INVAL, "NULL current partition");
+  int S = 0;
+  u64 cuts = 0, masks = 0;
+  if (!host_decode(h_current, c->L, c->N, S, cuts, masks))
+    return fail(c, AUTOPIPE_E_INVAL, "invalid current partition");
+  u64 sow = 0;
+  for (int w = 0; w < MAXN; ++w) sow |= (u64)h_current->stage_of_worker[w] << (8 * w);
+  nslots = (u64)((int)c->N + (int)c->N * ((int)c->N - 1) / 2) * NEIGH_MAXOPT;
+  c->launches += launch_neigh_gen(S, cuts, sow, (int)c->L, (int)c->N, c->d_nslots, st);
+  return AUTOPIPE_OK;
+}
+
+extern "C" int autopipe_neighbourhood(autopipe_ctx *c, const autopipe_partition *h_current, autopipe_partition *d_out,
+                                      uint64_t capacity, uint64_t *h_count, void *stream) {
+  if (!c) return AUTOPIPE_E_INVAL;
+  c->err[0] = 0;
+  if (!h_count || (capacity && !d_out)) return fail(c, AUTOPIPE_E_INVAL, "NULL output");
+  DeviceGuard dg(c->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  u64 nslots = 0;
+  int rc = neigh_prepare(c, h_current, nslots, st);
+  if (rc) return rc;
+  c->launches += launch_neigh_compact(c->d_nslots, nslots, d_out, capacity, c->d_ncount, st);
+  cudaError_t e = cudaMemcpyAsync(c->h_ncount, c->d_ncount, 8, cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  if (e != cudaSuccess) return cuda_fail(c, e, "neighbourhood");
+  *h_count = *c->h_ncount;
+  return AUTOPIPE_OK;
+}
+
+extern "C" int autopipe_neighbourhood_best(autopipe_ctx *c, const autopipe_partition *h_current,
+                                           autopipe_result *h_out, void *stream) {
+  if (!c) return AUTOPIPE_E_INVAL;
+  c->err[0] = 0;
+  if (!h_out) return fail(c, AUTOPIPE_E_INVAL, "NULL result pointer");
+  DeviceGuard dg(c->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  int rc = sync_status(c, st);
+  if (rc) return rc;
+  u64 nslots = 0;
+  rc = neigh_prepare(c, h_current, nslots, st);
+  if (rc) return rc;
+  c->launches += launch_eval(c->tab, c->d_nslots, nslots, c->d_ntimes, nullptr, nullptr, nullptr, nullptr, c->path32,
+                             c->sms, st);
+  c->launches += launch_neigh_best(c->d_nslots, c->d_ntimes, nslots, c->d_result, st);
+  cudaError_t e = cudaMemcpyAsync(c->h_result, c->d_result, sizeof(ResultDev), cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  if (e != cudaSuccess) return cuda_fail(c, e, "neighbourhood_best");
+  h_out->time_ns = c->h_result->time_ns;
+  h_out->index = c->h_result->index;
+  h_out->evaluated = c->h_result->evaluated;
+  memcpy(&h_out->part, c->h_result->part, 16);
+  return AUTOPIPE_OK;
+}

@@ -38,4 +38,11 @@ int launch_finalize(const BlockOut *in, int n, const SearchSpace &sp, ResultDev 
 
 void upload_binomials(const u64 (*tab)[BINOM_K]);
 
+// NEXT row f1: the two-worker neighbourhood (k_neigh.cu). Slots: (N + C(N,2)) * NEIGH_MAXOPT records.
+constexpr int NEIGH_MAXOPT = 544;  // >= (8+2) + (8+1) + 2*(255-1) options per changed-worker set
+constexpr int NEIGH_ITEMS = 8 + 28;
+int launch_neigh_gen(int S, u64 cuts, u64 sow, int L, int N, void *slots, cudaStream_t st);
+int launch_neigh_compact(const void *slots, u64 nslots, void *out, u64 cap, u64 *count, cudaStream_t st);
+int launch_neigh_best(const void *slots, const u64 *times, u64 nslots, ResultDev *res, cudaStream_t st);
+
 }  // namespace ap

@@ -4,3 +4,4 @@
 #include "k_eval.cu"
 #include "k_search.cu"
 #include "k_search_r1.cu"
+#include "k_neigh.cu"

@@ -166,6 +166,38 @@ class Engine:
                                                 ctypes.byref(res), self._stream(stream)))
         return SearchResult(int(res.time_ns), int(res.index), int(res.evaluated), record_bytes(res.part))
 
+    # -- NEXT row f1: the two-worker neighbourhood ------------------------
+    def neighbourhood(self, current: bytes, capacity: int = 1 << 15, stream=None) -> torch.Tensor:
+        """All partitions differing from `current` in one or two workers' layer sets (uint8 [n, 16])."""
+        cur = Partition.from_buffer_copy(bytes(current))
+        out = torch.empty((capacity, 16), dtype=torch.uint8, device=self.device)
+        n = ctypes.c_uint64()
+        self._check(lib.autopipe_neighbourhood(self._h, ctypes.byref(cur), ctypes.c_void_p(out.data_ptr()),
+                                               capacity, ctypes.byref(n), self._stream(stream)))
+        if n.value > capacity:
+            return self.neighbourhood(current, int(n.value), stream)
+        return out[: n.value]
+
+    def best_neighbour(self, current: bytes, stream=None) -> SearchResult:
+        """The neighbour with the smallest (T_ns, record bytes); evaluated = neighbourhood size."""
+        cur = Partition.from_buffer_copy(bytes(current))
+        res = Result()
+        self._check(lib.autopipe_neighbourhood_best(self._h, ctypes.byref(cur), ctypes.byref(res),
+                                                    self._stream(stream)))
+        return SearchResult(int(res.time_ns), int(res.index), int(res.evaluated), record_bytes(res.part))
+
+    def local_search(self, start: bytes, max_steps: int = 100):
+        """The paper's gradual migration: move to the best two-worker neighbour while
+        it is strictly faster. Returns the path [(T_ns, record), ...] starting at `start`."""
+        t0 = self.eval_partitions(torch.frombuffer(bytearray(start), dtype=torch.uint8).view(1, 16))
+        path = [(int(t0.cpu().numpy().view(np.uint64)[0]), bytes(start))]
+        for _ in range(max_steps):
+            r = self.best_neighbour(path[-1][1])
+            if r.time_ns >= path[-1][0]:
+                break
+            path.append((r.time_ns, r.partition))
+        return path
+
     # -- support ---------------------------------------------------------------------------
     def count_candidates(self, s_min: int, s_max: int, flags: int = 0) -> int:
         v = ctypes.c_uint64()

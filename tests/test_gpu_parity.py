@@ -352,3 +352,54 @@ def test_set_state_device_overflow(eng):
     with pytest.raises(AutopipeError) as ex:
         eng.search_optimum(1, 2)
     assert ex.value.code == AUTOPIPE_E_OVERFLOW
+
+
+# ------------------------------------------------------------------------------------------------
+# NEXT row f1: the two-worker neighbourhood against the oracle's definition
+# ------------------------------------------------------------------------------------------------
+
+@pytest.mark.parametrize("seed", range(4))
+def test_neighbourhood_matches_oracle(eng, seed):
+    from oracle.neighbourhood import all_partitions, best_neighbour, neighbourhood
+    rng = np.random.default_rng(500 + seed)
+    for it in range(4):
+        L = int(rng.integers(2, 8))
+        N = int(rng.integers(1, 5))
+        prof = W.random_profile(L, rng, f_max=1000, bytes_max=10**6)
+        st = W.random_state_small(prof, N, rng, tau_max=10**4)
+        eng.load(prof, st)
+        parts = list(all_partitions(L, N))
+        for k in rng.choice(len(parts), size=min(4, len(parts)), replace=False):
+            cur = encode_partition(parts[int(k)])
+            got = eng.neighbourhood(cur).cpu().numpy()
+            got = sorted(bytes(r) for r in got)
+            assert got == neighbourhood(L, N, parts[int(k)])
+            T, rec, n = best_neighbour(prof, st, cur)
+            r = eng.best_neighbour(cur)
+            assert (r.time_ns, r.partition, r.evaluated) == (T, rec, n)
+
+
+def test_neighbourhood_gpt96_and_local_search(eng):
+    """On the 96-layer space: the neighbourhood's best equals the minimum over the eval kernel of the
+    listed neighbours, and the paper's gradual migration from the even split strictly descends and
+    never beats the exhaustive optimum."""
+    prof, st = W.gpt96(), W.gpt_state("b")
+    eng.load(prof, st)
+    even = W.contiguous_record(96, [11, 23, 35, 47, 59, 71, 83], [1] * 8)
+    nb = eng.neighbourhood(even)
+    t = [int(x) for x in as_u64_list(eng.eval_partitions(nb))]
+    recs = [bytes(r) for r in nb.cpu().numpy()]
+    best = min(zip(t, recs))
+    r = eng.best_neighbour(even)
+    assert (r.time_ns, r.partition, r.evaluated) == (best[0], best[1], len(recs))
+    path = eng.local_search(even, max_steps=200)
+    assert all(a[0] > b[0] for a, b in zip(path, path[1:]))
+    opt = eng.search_optimum(8, 8)
+    assert path[-1][0] >= opt.time_ns
+    assert score_many(prof, st, [path[-1][1]])[0] == path[-1][0]
+
+
+def as_u64_list(t):
+    from paper_conf_icpp_hulww24_b200 import as_u64
+    torch.cuda.synchronize()
+    return as_u64(t)
