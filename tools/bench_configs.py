@@ -78,6 +78,22 @@ def measure(device: int = 0, rollout_records: int = 1 << 20):
                                   "rollout_ms": ms_r, "rollout_records_per_s": rollout_records / (ms_r / 1e3),
                                   "eval_GBps_algorithmic": rollout_records * 24 / (ms_e / 1e3) / 1e9,
                                   "int_path": eng.int_path}
+    # f1: the paper's two-worker neighbourhood step and its gradual migration on
+    # the 96-layer profile, heterogeneous state C4b, starting from the even split
+    prof, st = W.gpt96(), W.gpt_state("b")
+    eng.load(prof, st)
+    even = W.contiguous_record(96, [11, 23, 35, 47, 59, 71, 83], [1] * 8)
+    ms_n, r = _timed(lambda: eng.best_neighbour(even))
+    import time as _t
+    t0 = _t.perf_counter()
+    path = eng.local_search(even, max_steps=500)
+    ls_s = _t.perf_counter() - t0
+    opt = eng.search_optimum(8, 8)
+    res["F1_neighbourhood_gpt96_C4b"] = {"neighbours": r.evaluated, "ms_per_step": ms_n,
+                                         "local_search_steps": len(path) - 1, "local_search_wall_ms": 1e3 * ls_s,
+                                         "start_T_ns": path[0][0], "local_opt_T_ns": path[-1][0],
+                                         "exhaustive_opt_T_ns": opt.time_ns,
+                                         "local_over_exhaustive": path[-1][0] / opt.time_ns}
     eng.close()
     return res
 
