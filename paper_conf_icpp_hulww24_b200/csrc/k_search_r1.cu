@@ -324,6 +324,30 @@ __global__ void __launch_bounds__(NT, 2) k_search_r1(DevTables g, const R1Header
     const u64 r1 = umin(r0 + R, ye.row_end);
     const u64 pcy = PC[(p - 1) * Lp1 + y + 1];  // start of stage p-1 (warp-uniform)
     u64 pre = (r0 < r1 && P > 0) ? lex_unrank_smem(r0, P, y, Bn) : 0ull;
+    // Seed: the lane's first row with the remaining layers split evenly over the last three stages.
+    // Its exact T (and index) tightens theta before the sweep, so far fewer candidates reach the rare
+    // path while a lane's best is still poor (most visible when a GPU scans a small shard).
+    if (r0 < r1) {
+      const int rem = L - 1 - y;  // layers y+1 .. L-1 for stages p-1, p, q
+      int xs = y + rem / 3, es = y + (2 * rem) / 3;
+      if (xs <= y) xs = y + 1;
+      if (es <= xs) es = xs + 1;
+      if (es > L - 2) es = L - 2;
+      if (xs >= es) xs = es - 1;
+      const u64 cuts = pre | ((u64)y << (8 * P)) | ((u64)xs << (8 * (P + 1))) | ((u64)es << (8 * (P + 2)));
+      // inside the shard? (only the shard's first and last rows can be partial)
+      bool in = true;
+      if (pre == hdr.lo_pre && y == hdr.lo_y) in &= (xs > hdr.lo_x) || (xs == hdr.lo_x && es >= hdr.lo_e);
+      if (pre == hdr.hi_pre && y == hdr.hi_y) in &= (xs < hdr.hi_x) || (xs == hdr.hi_x && es <= hdr.hi_e);
+      if (in) {
+        const u64 Ts = exact_T_r1<S>(PC, Z, LM, L, cuts);
+        const u64 is = hdr.off + lex_rank_smem(cuts, S - 1, n, Bn);
+        if (better(Ts, is, bestT, bestI)) {
+          bestT = Ts;
+          bestI = is;
+        }
+      }
+    }
     // strictness: theta = best while this lane's task may still hold a smaller index than its best
     bool strict = true;
     if (r0 < r1 && bestT != U64MAX) {
@@ -543,19 +567,29 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
   h->hi_y = hi[P]; h->hi_x = hi[P + 1]; h->hi_e = hi[P + 2];
   int ny = 0;
   u64 tasks = 0;
-  // task size by estimated cost (thread-instructions per lane): a row costs ~150 (prefix terms) +
-  // ~26 per x + ~6 per candidate; ~40k per lane-task keeps ~40 tasks per warp on the 96-layer space,
-  // so the dynamic schedule's tail stays small while the per-task unrank is amortised
-  const u64 TARGET = 40000;
+  // Task size by estimated cost (thread-instructions per lane): a row costs ~150 (prefix terms) +
+  // ~26 per x + ~6 per candidate. The target per lane-task is set so the shard splits into ~40 tasks
+  // per resident warp (2 x 8 warps per SM): the dynamic schedule's tail stays small at any shard size
+  // (a full 96-layer space on one GPU, or 1/8 of it per GPU), and the per-task unrank is amortised.
+  u64 rb_[256], re_[256], cost_[256];
+  u64 total_cost = 0;
   for (int y = P; y <= L - 4; ++y) {
     // rows (prefix, y) whose candidates intersect [lo, hi]: a contiguous range of prefix ranks
     const bool lo_fits = (P == 0) || lo[P - 1] < y;
     const bool hi_fits = (P == 0) || hi[P - 1] < y;
-    const u64 rb = count_less(y, P, lo) + ((lo_fits && y < lo[P]) ? 1 : 0);
-    const u64 re = count_less(y, P, hi) + ((hi_fits && y <= hi[P]) ? 1 : 0);
-    if (re <= rb) continue;
+    rb_[y] = count_less(y, P, lo) + ((lo_fits && y < lo[P]) ? 1 : 0);
+    re_[y] = count_less(y, P, hi) + ((hi_fits && y <= hi[P]) ? 1 : 0);
     const u64 m = (u64)(L - 2 - y);
-    const u64 row_cost = 150 + 26 * (m - 1) + 6 * (m * (m - 1) / 2);
+    cost_[y] = 150 + 26 * (m - 1) + 6 * (m * (m - 1) / 2);
+    if (re_[y] > rb_[y]) total_cost += (re_[y] - rb_[y]) * cost_[y];
+  }
+  const u64 lane_tasks = (u64)sms * 16 * 32 * 40;
+  u64 TARGET = total_cost / (lane_tasks ? lane_tasks : 1);
+  if (TARGET < 4000) TARGET = 4000;
+  for (int y = P; y <= L - 4; ++y) {
+    const u64 rb = rb_[y], re = re_[y];
+    if (re <= rb) continue;
+    const u64 row_cost = cost_[y];
     const u64 R = row_cost >= TARGET ? 1 : (TARGET + row_cost - 1) / row_cost;
     const u64 nt = (re - rb + 32 * R - 1) / (32 * R);
     R1YEntry &ye = yt[ny++];
