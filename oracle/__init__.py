@@ -18,6 +18,8 @@ Modules
   param_dp    parametric DP: exact search optimum + lexicographically-first argmin
   cycle_ratio max cycle ratio of the explicit timed event graph (cross-check of sim)
   rollout     rollout reward = T_ns + switch bytes (SPEC §6)
+  neighbourhood  the two-worker neighbourhood by definition (NEXT f1)
+  switching   switching cost as time: startup refill + weight migration, amortised reward (NEXT f2)
 
 Parity status: every function here is pinned by tests/test_oracle_*.py (worked examples of the
 paper, closed forms, invariants, textbook reductions, brute force). None is "parity unpinned".
