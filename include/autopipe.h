@@ -156,6 +156,27 @@ int autopipe_neighbourhood(autopipe_ctx *ctx, const autopipe_partition *h_curren
 int autopipe_neighbourhood_best(autopipe_ctx *ctx, const autopipe_partition *h_current, autopipe_result *h_out,
                                 void *stream);
 
+/* NEXT row f2 — switching cost as time (a switch pauses training and the
+ * pipeline "requires a restart phase, i.e., startup starts in Figure 2, which brings bubbles";
+ * layer weights move to the workers that newly hold them; the
+ * reward is one-iteration speed with the normalised switching cost). Reading F-2:
+ *   refill_ns   = max(0, C_{S-1} - S * T_ns): C_k is when stage 0 finishes the backward pass of
+ *                 mini-batch k in the 1F1B schedule of the proposal started empty at time 0;
+ *   migrate_ns  = max over workers w of the sum of w's weight messages: for every stage of the
+ *                 current partition that covers some of w's new layers and does not contain w, one
+ *                 message of those layers' weight bytes from the holder with the smallest tau[u][w];
+ *   reward_ns   = T_ns + ceil((refill_ns + migrate_ns) / horizon);
+ *   both costs are 0 when every worker keeps its layer set (then reward_ns = T_ns).
+ * Device pointers, async on `stream`: d_parts[count] proposals; d_reward_ns[count] required;
+ * d_time_ns, d_refill_ns, d_migrate_ns may each be NULL. An invalid proposal gets UINT64_MAX in
+ * every output. h_current: HOST pointer, required (invalid -> E_INVAL); horizon >= 1 (else E_INVAL).
+ * E_OVERFLOW if the state's bound on modelled sums (SPEC.md §7) reaches 2^52 ns (startup event times
+ * stay below 2^62). For a state set with autopipe_set_state_device this call synchronises `stream`
+ * once to read the state's status. */
+int autopipe_switch_rewards(autopipe_ctx *ctx, const autopipe_partition *d_parts, uint64_t count,
+                            const autopipe_partition *h_current, uint64_t horizon, uint64_t *d_time_ns,
+                            uint64_t *d_refill_ns, uint64_t *d_migrate_ns, uint64_t *d_reward_ns, void *stream);
+
 /* Number of candidates of a search space (requires a state for L and N). */
 int autopipe_count_candidates(const autopipe_ctx *ctx, uint32_t s_min, uint32_t s_max, uint32_t flags,
                               uint64_t *total);

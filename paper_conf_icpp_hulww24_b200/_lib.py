@@ -29,7 +29,8 @@ SYMBOLS = ["autopipe_create", "autopipe_destroy", "autopipe_last_error", "autopi
            "autopipe_set_state", "autopipe_set_state_device", "autopipe_eval_partitions", "autopipe_search_optimum",
            "autopipe_rollout_rewards", "autopipe_count_candidates", "autopipe_decode_index",
            "autopipe_int_path", "autopipe_kernel_launches", "autopipe_set_timing",
-           "autopipe_last_search_ms", "autopipe_neighbourhood", "autopipe_neighbourhood_best"]
+           "autopipe_last_search_ms", "autopipe_neighbourhood", "autopipe_neighbourhood_best",
+           "autopipe_switch_rewards"]
 
 
 class Partition(ctypes.Structure):
@@ -77,6 +78,7 @@ def _load():
         "autopipe_last_search_ms": (ctypes.c_double, [P]),
         "autopipe_neighbourhood": (i32, [P, ctypes.POINTER(Partition), P, u64, pu64, P]),
         "autopipe_neighbourhood_best": (i32, [P, ctypes.POINTER(Partition), ctypes.POINTER(Result), P]),
+        "autopipe_switch_rewards": (i32, [P, P, u64, ctypes.POINTER(Partition), u64, P, P, P, P, P]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(lib, name)

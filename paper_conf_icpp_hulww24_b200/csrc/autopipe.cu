@@ -28,6 +28,7 @@ struct autopipe_ctx {
   int path32 = 0;
   u64 launches = 0;
   u64 maxOG = 0, sumP = 0;
+  u64 bound = 0;  // the state's bound on modelled sums (SPEC.md §7)
   DevTables tab{};
   // device buffers
   u64 *d_raw = nullptr;      // fp [8*255] | bp [8*255] | P [255] | tau [64]
@@ -242,6 +243,7 @@ extern "C" int autopipe_set_state(autopipe_ctx *c, uint32_t N, const uint64_t *f
   if (bound >= LIMIT_TIME) return fail(c, AUTOPIPE_E_OVERFLOW, "modelled times reach 2^59 ns");
   const u128 bound32 = sumMax + 16 + (u128)14 * maxXog;
   c->path32 = bound32 < LIMIT_TIME32 ? 1 : 0;
+  c->bound = (u64)bound;
   DeviceGuard dg(c->device);
   cudaStream_t st = (cudaStream_t)stream;
   // stage into pinned memory so the copies are truly asynchronous
@@ -299,6 +301,7 @@ static int sync_status(autopipe_ctx *c, cudaStream_t st) {
   if (e != cudaSuccess) return cuda_fail(c, e, "state status");
   c->state_on_device = false;
   c->path32 = (c->h_status[0] & 2) ? 1 : 0;
+  c->bound = c->h_status[1];
   if (c->h_status[0] & 1) {
     c->has_state = false;
     return fail(c, AUTOPIPE_E_OVERFLOW, "device state: bytes * tau reaches 2^64 or modelled times reach 2^59 ns");
@@ -613,5 +616,38 @@ extern "C" int autopipe_neighbourhood_best(autopipe_ctx *c, const autopipe_parti
   h_out->index = c->h_result->index;
   h_out->evaluated = c->h_result->evaluated;
   memcpy(&h_out->part, c->h_result->part, 16);
+  return AUTOPIPE_OK;
+}
+
+// --- NEXT row f2: switching cost as time (reading F-2) ----
+static const u64 LIMIT_SWITCH = 1ull << 52;  // startup event times < 2^10 * bound (DESIGN.md §3 F-2)
+
+extern "C" int autopipe_switch_rewards(autopipe_ctx *c, const autopipe_partition *d_parts, uint64_t count,
+                                       const autopipe_partition *h_current, uint64_t horizon, uint64_t *d_time_ns,
+                                       uint64_t *d_refill_ns, uint64_t *d_migrate_ns, uint64_t *d_reward_ns,
+                                       void *stream) {
+  if (!c) return AUTOPIPE_E_INVAL;
+  c->err[0] = 0;
+  if (!c->has_state) return fail(c, AUTOPIPE_E_STATE, "switch rewards before set_state");
+  if (!h_current) return fail(c, AUTOPIPE_E_INVAL, "NULL current partition");
+  if (horizon == 0) return fail(c, AUTOPIPE_E_INVAL, "horizon must be >= 1");
+  int S = 0;
+  u64 cuts = 0, masks = 0;
+  if (!host_decode(h_current, c->L, c->N, S, cuts, masks))
+    return fail(c, AUTOPIPE_E_INVAL, "invalid current partition");
+  if (count == 0) return AUTOPIPE_OK;
+  if (!d_parts || !d_reward_ns) return fail(c, AUTOPIPE_E_INVAL, "NULL device pointer");
+  DeviceGuard dg(c->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  int rc = sync_status(c, st);
+  if (rc) return rc;
+  if (c->bound >= LIMIT_SWITCH)
+    return fail(c, AUTOPIPE_E_OVERFLOW, "switch rewards need modelled times below 2^52 ns");
+  u64 sow = 0;
+  for (int w = 0; w < MAXN; ++w) sow |= (u64)h_current->stage_of_worker[w] << (8 * w);
+  c->launches += launch_switch(c->tab, d_parts, count, S, cuts, masks, sow, horizon, (u64 *)d_time_ns,
+                               (u64 *)d_refill_ns, (u64 *)d_migrate_ns, (u64 *)d_reward_ns, c->path32, c->sms, st);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(c, e, "switch kernel launch");
   return AUTOPIPE_OK;
 }

@@ -45,4 +45,9 @@ int launch_neigh_gen(int S, u64 cuts, u64 sow, int L, int N, void *slots, cudaSt
 int launch_neigh_compact(const void *slots, u64 nslots, void *out, u64 cap, u64 *count, cudaStream_t st);
 int launch_neigh_best(const void *slots, const u64 *times, u64 nslots, ResultDev *res, cudaStream_t st);
 
+// NEXT row f2: switching cost as time (k_switch.cu).
+int launch_switch(const DevTables &g, const void *recs, u64 count, const int cur_S, const u64 cur_cuts,
+                  const u64 cur_masks, const u64 cur_sow, u64 horizon, u64 *out_t, u64 *out_refill,
+                  u64 *out_mig, u64 *out_reward, int path32, int sms, cudaStream_t st);
+
 }  // namespace ap

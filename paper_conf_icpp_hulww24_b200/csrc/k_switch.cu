@@ -1,0 +1,292 @@
+// k_switch.cu — NEXT row f2: the switching cost of a proposal as time (autopipe_switch_rewards).
+//
+// The paper's switch pauses training and restarts the pipeline, whose "startup state" (Fig. 2)
+// brings bubbles, and moves layer weights to the workers that newly hold them
+// (PAPER.md:973-981); the arbiter's reward is the one-iteration time with the normalised switching
+// cost. Reading F-2 makes that an integer:
+//
+//   refill  = max(0, C_{S-1} - S * T)   C_k: stage 0 finishes mini-batch k's backward pass in the
+//                                        static 1F1B schedule started empty at time 0
+//   migrate = max over workers of the sum of their weight messages (one per old stage that covers
+//             some of their new layers without holding them; cheapest holder's link)
+//   reward  = T + ceil((refill + migrate) / H)
+//
+// One thread per proposal. C_{S-1} comes from the schedule's own max-plus recurrence, run round by
+// round in dependency order (no event queue):
+//   round -1, k = 0..S-1, stages ascending   F_s(k) for k < n_s = S - s
+//   round  j = 0..S-1, stages descending      B_s(j), then F_s(j + n_s)
+// B_s(j) needs backward boundary s of j, produced just before in the same round by stage s+1;
+// F_s(j + n_s) needs forward boundary s-1 of j + n_s, produced one round earlier by stage s-1, so
+// one "latest" value per boundary suffices. Every worker keeps its own free time (its op list is
+// the 1F1B order), every boundary is a barrier over the sending replicas followed by FIFO transfers
+// on its directed links (one per overlapping shard pair; the links of different boundaries are
+// distinct, so one free time per pair). Worker state lives in registers (loops over the 8 worker
+// slots are unrolled and predicated on the worker's stage); per-pair durations and link free times
+// in two small per-thread arrays.
+#include "eval.cuh"
+#include "internal.h"
+
+namespace ap {
+
+// The current partition, pre-digested on the host: old stage ranges and per-worker layer sets.
+struct SwitchCur {
+  u64 wkey;          // byte w: 0xFF idle, else old stage of w
+  u32 range[MAXS];   // old stage s: a | e << 8
+  u32 wrange[MAXN];  // worker w: a | e << 8, 0xFFFF if idle (its layer set)
+  u32 masks[MAXS];   // old stage s: worker bitmask
+  int S;
+};
+
+constexpr int MAXPAIRS = 2 * MAXN;  // sum over boundaries of (r_s + r_{s+1} - 1) <= 2 sum r - (S-1)
+
+// Durations of every transfer of one boundary, in merge order (see boundary_max in eval.cuh).
+__device__ __forceinline__ int boundary_pairs(u64 A, u32 send, u32 recv, const u64 *tau, u64 *d, int n) {
+  const u32 rs = __popc(send), rr = __popc(recv);
+  if (rs == 1 && rr == 1) {
+    d[n] = xfer(A, tau[(__ffs(send) - 1) * 8 + __ffs(recv) - 1]);
+    return n + 1;
+  }
+  const Div8 ds(rs), dr(rr);
+  const u64 qs = ds.div(A), qr = dr.div(A);
+  const u32 rems = (u32)(A - qs * rs), remr = (u32)(A - qr * rr);
+  u32 i = 0, j = 0;
+  u64 lo_i = 0, lo_j = 0;
+  u64 hi_i = qs + ds.small(rems), hi_j = qr + dr.small(remr);
+  while (i < rs && j < rr) {
+    const u64 lo = umax(lo_i, lo_j), hi = umin(hi_i, hi_j);
+    if (hi > lo) d[n++] = xfer(hi - lo, tau[(__ffs(send) - 1) * 8 + __ffs(recv) - 1]);
+    const bool adv_i = hi_i <= hi_j, adv_j = hi_j <= hi_i;
+    if (adv_i) {
+      ++i; send &= send - 1;
+      lo_i = hi_i; hi_i = (u64)(i + 1) * qs + ds.small((i + 1) * rems);
+    }
+    if (adv_j) {
+      ++j; recv &= recv - 1;
+      lo_j = hi_j; hi_j = (u64)(j + 1) * qr + dr.small((j + 1) * remr);
+    }
+  }
+  return n;
+}
+
+// Barrier at `bar`, then the FIFO transfers [lo, hi) of one boundary; returns its completion.
+__device__ __forceinline__ u64 run_boundary(u64 bar, const u64 *d, u64 *lf, int lo, int hi) {
+  u64 done = bar;
+  for (int p = lo; p < hi; ++p) {
+    const u64 e = umax(bar, lf[p]) + d[p];
+    lf[p] = e;
+    done = umax(done, e);
+  }
+  return done;
+}
+
+// C_{S-1} of the startup (see the file comment). sw: byte w = stage of worker w (0xFF idle).
+__device__ __forceinline__ u64 startup_completion(const SmemTab &t, int S, u64 cuts, u64 masks, u64 sw) {
+  u64 Fd[MAXN], Bd[MAXN], wf[MAXN];
+  int stg[MAXN];
+#pragma unroll
+  for (int w = 0; w < MAXN; ++w) {
+    const int s = byte_at(sw, w);
+    stg[w] = s;  // 0xFF never matches a stage
+    wf[w] = 0;
+    Fd[w] = 0;
+    Bd[w] = 0;
+    if (s != 0xFF) {
+      const int a = (s == 0) ? 0 : byte_at(cuts, s - 1) + 1;
+      const int e = (s == S - 1) ? t.L - 1 : byte_at(cuts, s);
+      const Div8 dv((u32)__popc((u32)byte_at(masks, s)));
+      Fd[w] = dv.ceil(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a]);
+      Bd[w] = dv.ceil(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a]);
+    }
+  }
+  // transfers: forward boundary s = pairs [offF[s], offF[s+1]), backward boundary s likewise
+  u64 dF[MAXPAIRS], dB[MAXPAIRS], lfF[MAXPAIRS], lfB[MAXPAIRS];
+  int offF[MAXS], offB[MAXS];
+  int nf = 0, nb = 0;
+#pragma unroll
+  for (int s = 0; s < MAXS - 1; ++s) {
+    offF[s] = nf;
+    offB[s] = nb;
+    if (s < S - 1) {
+      const int e = byte_at(cuts, s);
+      const u32 ms = (u32)byte_at(masks, s), mn = (u32)byte_at(masks, s + 1);
+      nf = boundary_pairs(t.O[e], ms, mn, t.tau, dF, nf);
+      nb = boundary_pairs(t.G[e + 1], mn, ms, t.tau, dB, nb);
+    }
+  }
+  offF[MAXS - 1] = nf;
+  offB[MAXS - 1] = nb;
+  for (int p = 0; p < nf; ++p) lfF[p] = 0;
+  for (int p = 0; p < nb; ++p) lfB[p] = 0;
+
+  u64 fdl[MAXS];  // latest completion of forward boundary s
+#pragma unroll
+  for (int s = 0; s < MAXS; ++s) fdl[s] = 0;
+  // round -1: F_s(k) for k < n_s, k-major so boundary s-1 of k is ready when stage s needs it
+  for (int k = 0; k < S; ++k) {
+#pragma unroll
+    for (int s = 0; s < MAXS; ++s) {
+      if (s < S - k) {
+        const u64 ready = (s == 0) ? 0 : fdl[s > 0 ? s - 1 : 0];
+        u64 bar = 0;
+#pragma unroll
+        for (int w = 0; w < MAXN; ++w)
+          if (stg[w] == s) {
+            wf[w] = umax(wf[w], ready) + Fd[w];
+            bar = umax(bar, wf[w]);
+          }
+        if (s < S - 1) fdl[s] = run_boundary(bar, dF, lfF, offF[s], offF[s + 1]);
+      }
+    }
+  }
+  // rounds j = 0..S-1: stages from the last to the first, B_s(j) then F_s(j + n_s)
+  u64 C = 0;
+  for (int j = 0; j < S; ++j) {
+    u64 bd = 0;  // completion of backward boundary s of mini-batch j, flowing towards stage 0
+#pragma unroll
+    for (int s = MAXS - 1; s >= 0; --s) {
+      if (s < S) {
+        const u64 readyB = (s == S - 1) ? 0 : bd;
+        u64 bar = 0;
+#pragma unroll
+        for (int w = 0; w < MAXN; ++w)
+          if (stg[w] == s) {
+            wf[w] = umax(wf[w], readyB) + Bd[w];
+            bar = umax(bar, wf[w]);
+          }
+        if (s > 0) bd = run_boundary(bar, dB, lfB, offB[s > 0 ? s - 1 : 0], offB[s]);
+        else C = bar;
+        const u64 readyF = (s == 0) ? 0 : fdl[s > 0 ? s - 1 : 0];
+        u64 barF = 0;
+#pragma unroll
+        for (int w = 0; w < MAXN; ++w)
+          if (stg[w] == s) {
+            wf[w] = umax(wf[w], readyF) + Fd[w];
+            barF = umax(barF, wf[w]);
+          }
+        if (s < S - 1) fdl[s] = run_boundary(barF, dF, lfF, offF[s], offF[s + 1]);
+      }
+    }
+  }
+  return C;
+}
+
+// Weight migration (reading F-2): per receiving worker, the sum of its messages; the max over workers.
+// tmin[so * 8 + w] = min over the holders u of old stage so of tau[u][w].
+__device__ __forceinline__ u64 migrate_time(const SmemTab &t, int S, u64 cuts, u64 sw, const SwitchCur &cur,
+                                            const u64 *tmin) {
+  u64 best = 0;
+#pragma unroll
+  for (int w = 0; w < MAXN; ++w) {
+    const int s = byte_at(sw, w);
+    if (s != 0xFF) {
+      const int a = (s == 0) ? 0 : byte_at(cuts, s - 1) + 1;
+      const int e = (s == S - 1) ? t.L - 1 : byte_at(cuts, s);
+      const int own = byte_at(cur.wkey, w);
+      u64 sum = 0;
+#pragma unroll
+      for (int so = 0; so < MAXS; ++so) {
+        if (so < cur.S && so != own) {
+          const int lo = max(a, (int)(cur.range[so] & 0xFF)), hi = min(e, (int)(cur.range[so] >> 8));
+          if (lo <= hi) sum += xfer(t.PP[hi + 1] - t.PP[lo], tmin[so * 8 + w]);
+        }
+      }
+      best = umax(best, sum);
+    }
+  }
+  return best;
+}
+
+template <bool P32>
+__global__ void __launch_bounds__(256) k_switch(DevTables g, const uint4 *__restrict__ recs, u64 count,
+                                                SwitchCur cur, u64 horizon, u64 *__restrict__ out_t,
+                                                u64 *__restrict__ out_refill, u64 *__restrict__ out_mig,
+                                                u64 *__restrict__ out_reward) {
+  extern __shared__ u64 sm[];
+  const SmemTab t = stage_tables(g, sm);
+  __shared__ u64 tmin[MAXS * 8];
+  if (threadIdx.x < MAXS * 8) {
+    const int so = threadIdx.x >> 3, w = threadIdx.x & 7;
+    u64 m = U64MAX;
+    if (so < cur.S)
+      for (int u = 0; u < MAXN; ++u)
+        if ((cur.masks[so] >> u) & 1u) m = umin(m, t.tau[u * 8 + w]);
+    tmin[threadIdx.x] = m;
+  }
+  __syncthreads();
+  const int L = t.L, N = (int)g.N;
+  const bool overflow = (g.status[0] & 1ull) != 0;
+  const u64 stride = (u64)gridDim.x * blockDim.x;
+  for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < count; i += stride) {
+    const uint4 r = __ldg(recs + i);
+    const u64 lo = (u64)r.x | ((u64)r.y << 32), hi = (u64)r.z | ((u64)r.w << 32);
+    int S;
+    u64 cuts, masks;
+    u64 T = U64MAX, R = U64MAX, M = U64MAX, RW = U64MAX;
+    if (!overflow && decode_record(lo, hi, L, N, S, cuts, masks)) {
+      T = eval_closed_form<P32>(t, S, cuts, masks);
+      // per-worker layer sets, compared with the current partition's
+      bool same = true;
+#pragma unroll
+      for (int w = 0; w < MAXN; ++w) {
+        const int s = byte_at(hi, w);
+        u32 key = 0xFFFFu;
+        if (s != 0xFF) {
+          const int a = (s == 0) ? 0 : byte_at(cuts, s - 1) + 1;
+          const int e = (s == S - 1) ? L - 1 : byte_at(cuts, s);
+          key = (u32)a | ((u32)e << 8);
+        }
+        same &= key == cur.wrange[w];
+      }
+      if (same) {
+        R = 0;
+        M = 0;
+        RW = T;
+      } else {
+        const u64 C = startup_completion(t, S, cuts, masks, hi);
+        const u64 ST = (u64)S * T;
+        R = C > ST ? C - ST : 0;
+        M = migrate_time(t, S, cuts, hi, cur, tmin);
+        const u64 x = R + M;
+        RW = T + (x / horizon + (x % horizon != 0));
+      }
+    }
+    if (out_t) out_t[i] = T;
+    if (out_refill) out_refill[i] = R;
+    if (out_mig) out_mig[i] = M;
+    out_reward[i] = RW;
+  }
+}
+
+int launch_switch(const DevTables &g, const void *recs, u64 count, const int cur_S, const u64 cur_cuts,
+                  const u64 cur_masks, const u64 cur_sow, u64 horizon, u64 *out_t, u64 *out_refill,
+                  u64 *out_mig, u64 *out_reward, int path32, int sms, cudaStream_t st) {
+  if (count == 0) return 0;
+  SwitchCur cur;
+  cur.S = cur_S;
+  cur.wkey = cur_sow;
+  for (int s = 0; s < MAXS; ++s) {
+    cur.masks[s] = (u32)((cur_masks >> (8 * s)) & 0xFF);
+    cur.range[s] = 0;
+    if (s < cur_S) {
+      const u32 a = (s == 0) ? 0 : (u32)((cur_cuts >> (8 * (s - 1))) & 0xFF) + 1;
+      const u32 e = (s == cur_S - 1) ? g.L - 1 : (u32)((cur_cuts >> (8 * s)) & 0xFF);
+      cur.range[s] = a | (e << 8);
+    }
+  }
+  for (int w = 0; w < MAXN; ++w) {
+    const int s = (int)((cur_sow >> (8 * w)) & 0xFF);
+    cur.wrange[w] = (s == 0xFF) ? 0xFFFFu : cur.range[s];
+  }
+  const size_t smem = (size_t)smem_words(g.L, g.N) * sizeof(u64);
+  const u64 need = (count + 255) / 256, cap = (u64)sms * 8;
+  const int grid = (int)(need < cap ? need : cap);
+  if (path32)
+    k_switch<true><<<grid, 256, smem, st>>>(g, (const uint4 *)recs, count, cur, horizon, out_t, out_refill, out_mig,
+                                            out_reward);
+  else
+    k_switch<false><<<grid, 256, smem, st>>>(g, (const uint4 *)recs, count, cur, horizon, out_t, out_refill, out_mig,
+                                             out_reward);
+  return 1;
+}
+
+}  // namespace ap

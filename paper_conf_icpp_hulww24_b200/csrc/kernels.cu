@@ -5,3 +5,4 @@
 #include "k_search.cu"
 #include "k_search_r1.cu"
 #include "k_neigh.cu"
+#include "k_switch.cu"

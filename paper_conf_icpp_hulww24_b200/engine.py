@@ -158,6 +158,24 @@ class Engine:
             ctypes.c_void_p(out_sw.data_ptr()) if out_sw is not None else None, self._stream(stream)))
         return out_t, out_sw
 
+    def switch_rewards(self, parts, current: bytes, horizon: int, outputs=("time", "refill", "migrate"),
+                       stream=None) -> dict:
+        """NEXT row f2 (reading F-2): per proposal, the reward
+        T_ns + ceil((refill_ns + migrate_ns) / horizon) versus the current partition. Returns a dict
+        of int64 tensors: "reward" always, plus each name in `outputs`."""
+        recs = self._records(parts)
+        n = recs.shape[0]
+        cur = Partition.from_buffer_copy(bytes(current))
+        out = {k: torch.empty(n, dtype=torch.int64, device=self.device)
+               for k in ("reward",) + tuple(outputs)}
+
+        def ptr(k):
+            return ctypes.c_void_p(out[k].data_ptr()) if k in out else None
+        self._check(lib.autopipe_switch_rewards(
+            self._h, ctypes.c_void_p(recs.data_ptr()), n, ctypes.byref(cur), int(horizon), ptr("time"),
+            ptr("refill"), ptr("migrate"), ptr("reward"), self._stream(stream)))
+        return out
+
     def search_optimum(self, s_min: int, s_max: int, flags: int = 0, begin: int = 0,
                        end: Optional[int] = None, stream=None) -> SearchResult:
         res = Result()

@@ -53,3 +53,22 @@ def rollout_many(prof, st, records: Sequence[bytes], current, procs: int = 0):
         with mp.get_context("fork").Pool(procs, initializer=_init, initargs=(prof, st)) as pool:
             out = pool.map(_score_pair, args, chunksize=max(1, len(args) // (procs * 8)))
     return [o[0] for o in out], [o[1] for o in out]
+
+
+def _switch_one(args):
+    from oracle.model import parse_record
+    from oracle.switching import switch_reward
+    rec, cur, horizon = args
+    p = parse_record(cur, len(_CTX["prof"].O), len(_CTX["st"].f))
+    return switch_reward(_CTX["prof"], _CTX["st"], rec, p, horizon)
+
+
+def switch_many(prof, st, records: Sequence[bytes], current: bytes, horizon: int, procs: int = 0):
+    """oracle.switching.switch_reward over many proposals: list of (T, refill, migrate, reward)."""
+    args = [(bytes(r), bytes(current), horizon) for r in records]
+    procs = procs or cores()
+    if procs <= 1 or len(args) < 64:
+        _init(prof, st)
+        return [_switch_one(a) for a in args]
+    with mp.get_context("fork").Pool(procs, initializer=_init, initargs=(prof, st)) as pool:
+        return pool.map(_switch_one, args, chunksize=max(1, len(args) // (procs * 8)))

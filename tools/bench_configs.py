@@ -73,6 +73,9 @@ def measure(device: int = 0, rollout_records: int = 1 << 20):
     out_s = torch.empty_like(out_t)
     ms_e, _ = _timed(lambda: eng.eval_partitions(recs, out=out_t))
     ms_r, _ = _timed(lambda: eng.rollout_rewards(recs, cur, out_t=out_t, out_sw=out_s))
+    ms_s, _ = _timed(lambda: eng.switch_rewards(recs, cur, 100, outputs=(), stream=None))
+    res["F2_resnet50_switch_rewards"] = {"records": rollout_records, "ms": ms_s,
+                                         "records_per_s": rollout_records / (ms_s / 1e3), "horizon": 100}
     res["C5_resnet50_rollout"] = {"records": rollout_records, "eval_ms": ms_e,
                                   "eval_records_per_s": rollout_records / (ms_e / 1e3),
                                   "rollout_ms": ms_r, "rollout_records_per_s": rollout_records / (ms_r / 1e3),
