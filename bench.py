@@ -246,7 +246,10 @@ def main():
     if world > 1:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
         dist.init_process_group("nccl", device_id=dev)
-    lo, hi = rank * TOTAL // world, (rank + 1) * TOTAL // world
+    # contiguous shards of about equal device cost (host-only estimate; any split gives the same optimum)
+    from paper_conf_icpp_hulww24_b200.distributed import balanced_bounds
+    bounds = balanced_bounds(96, 8, S_STAGES, S_STAGES, 0, world)
+    lo, hi = bounds[rank], bounds[rank + 1]
 
     from paper_conf_icpp_hulww24_b200.distributed import minloc as dist_minloc
 

@@ -177,6 +177,15 @@ int autopipe_switch_rewards(autopipe_ctx *ctx, const autopipe_partition *d_parts
                             const autopipe_partition *h_current, uint64_t horizon, uint64_t *d_time_ns,
                             uint64_t *d_refill_ns, uint64_t *d_migrate_ns, uint64_t *d_reward_ns, void *stream);
 
+/* Multi-GPU split: G + 1 global indices bounds[0] = 0 < ... <= bounds[G] = space size
+ * such that the contiguous shards [bounds[g], bounds[g+1]) of the space (S in [s_min, s_max], flags as
+ * in autopipe_search_optimum; L layers, N workers) cost about the same device time: the estimate
+ * counts rows and columns of the fast kernel (short rows cost more per candidate), so shards are not
+ * equal in candidates. Host-only (no context, no GPU); any split gives the same global optimum.
+ * E_INVAL on bad arguments, E_OVERFLOW if the space exceeds 2^64. */
+int autopipe_balanced_shards(uint32_t L, uint32_t N, uint32_t s_min, uint32_t s_max, uint32_t flags, uint32_t G,
+                             uint64_t *bounds);
+
 /* Number of candidates of a search space (requires a state for L and N). */
 int autopipe_count_candidates(const autopipe_ctx *ctx, uint32_t s_min, uint32_t s_max, uint32_t flags,
                               uint64_t *total);

@@ -30,7 +30,7 @@ SYMBOLS = ["autopipe_create", "autopipe_destroy", "autopipe_last_error", "autopi
            "autopipe_rollout_rewards", "autopipe_count_candidates", "autopipe_decode_index",
            "autopipe_int_path", "autopipe_kernel_launches", "autopipe_set_timing",
            "autopipe_last_search_ms", "autopipe_neighbourhood", "autopipe_neighbourhood_best",
-           "autopipe_switch_rewards"]
+           "autopipe_switch_rewards", "autopipe_balanced_shards"]
 
 
 class Partition(ctypes.Structure):
@@ -79,6 +79,7 @@ def _load():
         "autopipe_neighbourhood": (i32, [P, ctypes.POINTER(Partition), P, u64, pu64, P]),
         "autopipe_neighbourhood_best": (i32, [P, ctypes.POINTER(Partition), ctypes.POINTER(Result), P]),
         "autopipe_switch_rewards": (i32, [P, P, u64, ctypes.POINTER(Partition), u64, P, P, P, P, P]),
+        "autopipe_balanced_shards": (i32, [u32, u32, u32, u32, u32, u32, pu64]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(lib, name)

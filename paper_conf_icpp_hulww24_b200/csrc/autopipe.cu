@@ -3,6 +3,7 @@
 // space (SPEC.md §5) and kernel launches. No score is ever computed here: every T_ns comes from the
 // sm_100a kernels in k_state.cu / k_eval.cu / k_search.cu / k_search_r1.cu.
 #include <cstdarg>
+#include <cstdlib>
 #include <cstdio>
 #include <cstring>
 #include <new>
@@ -471,6 +472,15 @@ extern "C" int autopipe_search_optimum(autopipe_ctx *c, uint32_t s_min, uint32_t
     }
   }
   if (c->timing) cudaEventRecord(c->ev1, st);
+  if (getenv("AUTOPIPE_R1_STATS") && used > 0) {  // diagnostics: rare-path decisions per search
+    BlockOut *hb = new BlockOut[used];
+    cudaMemcpyAsync(hb, c->d_blocks, sizeof(BlockOut) * used, cudaMemcpyDeviceToHost, st);
+    cudaStreamSynchronize(st);
+    u64 rare = 0, cnt = 0;
+    for (int i = 0; i < used; ++i) { rare += hb[i].pad; cnt += hb[i].count; }
+    fprintf(stderr, "[autopipe] blocks %d candidates %llu rare %llu\n", used, cnt, rare);
+    delete[] hb;
+  }
   c->launches += launch_finalize(c->d_blocks, used, sp, c->d_result, st);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "search kernel launch");
@@ -649,5 +659,130 @@ extern "C" int autopipe_switch_rewards(autopipe_ctx *c, const autopipe_partition
                                (u64 *)d_refill_ns, (u64 *)d_migrate_ns, (u64 *)d_reward_ns, c->path32, c->sms, st);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "switch kernel launch");
+  return AUTOPIPE_OK;
+}
+
+// --- cost-balanced contiguous shards of a search space ---------------
+// Estimated device cost (thread-instructions per lane) of the r = 1 kernel: a row (prefix, y) costs
+// ROW + X * (m - 1) + CAND * m (m - 1) / 2 with m = L - 2 - y (calibrated on B200: the per-row term
+// is what makes the high-index shards, whose rows are short, slower per candidate); the generic
+// kernel costs GEN * S per candidate.
+namespace {
+const u64 COST_ROW = 400, COST_X = 26, COST_CAND = 6, COST_GEN = 40;
+u64 hbin[256][9];
+void hbin_init() {
+  static bool done = false;
+  if (done) return;
+  for (int n = 0; n < 256; ++n)
+    for (int k = 0; k < 9; ++k) hbin[n][k] = (k == 0) ? 1 : (n == 0 ? 0 : hbin[n - 1][k - 1] + hbin[n - 1][k]);
+  done = true;
+}
+inline u64 hbn(int n, int k) { return (k < 0 || n < 0 || k > n) ? 0 : hbin[n][k]; }
+void unrank_cuts(u64 rank, int k, int n, int *out) {
+  int x = 0;
+  for (int i = 0; i < k; ++i) {
+    while (hbn(n - 1 - x, k - 1 - i) <= rank) {
+      rank -= hbn(n - 1 - x, k - 1 - i);
+      ++x;
+    }
+    out[i] = x++;
+  }
+}
+// k-subsets of {0..x-1} lexicographically smaller than the increasing tuple t
+u64 count_less_t(int x, int k, const int *t) {
+  u64 cnt = 0;
+  int prev = -1;
+  for (int i = 0; i < k; ++i) {
+    const int lim = t[i] < x ? t[i] : x;
+    for (int v = prev + 1; v < lim; ++v) cnt += hbn(x - 1 - v, k - 1 - i);
+    if (t[i] >= x) return cnt;
+    prev = t[i];
+  }
+  return cnt;
+}
+inline double row_cost(int L, int y) {
+  const double m = (double)(L - 2 - y);
+  return (double)COST_ROW + COST_X * (m - 1) + COST_CAND * m * (m - 1) / 2;
+}
+// cost of the first `kappa` cut sets (lexicographic) of an r = 1 block with S stages
+double r1_prefix_cost(int L, int S, u64 kappa, u64 ncut) {
+  if (kappa == 0) return 0.0;
+  const int P = S - 4, n = L - 1, k = S - 1;
+  int lo[8];
+  const bool end = kappa >= ncut;
+  unrank_cuts(end ? ncut - 1 : kappa, k, n, lo);
+  double c = 0.0;
+  for (int y = P; y <= L - 4; ++y) {
+    const bool fits = (P == 0) || lo[P - 1] < y;
+    u64 rows = count_less_t(y, P, lo) + ((fits && y < lo[P]) ? 1 : 0);
+    if (end && fits && y == lo[P]) rows += 1;  // the last row itself
+    c += (double)rows * row_cost(L, y);
+  }
+  return c;
+}
+}  // namespace
+
+extern "C" int autopipe_balanced_shards(uint32_t L, uint32_t N, uint32_t s_min, uint32_t s_max, uint32_t flags,
+                                        uint32_t G, uint64_t *bounds) {
+  if (!bounds || G < 1 || L < 1 || L > MAXL || N < 1 || N > MAXN) return AUTOPIPE_E_INVAL;
+  if (flags & ~AUTOPIPE_USE_ALL_WORKERS) return AUTOPIPE_E_INVAL;
+  const u32 smax_lim = N < (u32)MAXS ? N : (u32)MAXS;
+  if (s_min < 1 || s_min > s_max || s_max > smax_lim) return AUTOPIPE_E_INVAL;
+  hbin_init();
+  const bool all = flags & AUTOPIPE_USE_ALL_WORKERS;
+  // blocks of the index space in order: per S, the r = 1 block (if the fast kernel takes it) and the rest
+  struct Blk { u64 lo, hi; int S; bool r1; double c0, c1; };
+  Blk blk[2 * MAXS];
+  int nb = 0;
+  u128 off = 0;
+  double acc = 0.0;
+  for (int S = (int)s_min; S <= (int)s_max; ++S) {
+    const u64 K = all ? hbn((int)N - 1, S - 1) : hbn((int)N, S);
+    const u64 nc = (S - 1 <= (int)L - 1) ? hbn((int)L - 1, S - 1) : 0;
+    const u128 sz = (u128)K * nc;
+    if ((off + sz) >> 64) return AUTOPIPE_E_OVERFLOW;
+    const bool r1 = S >= 5 && (!all || (int)N == S) && nc > 0;
+    u64 start = (u64)off;
+    if (r1) {
+      const double c = r1_prefix_cost((int)L, S, nc, nc);
+      blk[nb++] = {start, start + nc, S, true, acc, acc + c};
+      acc += c;
+      start += nc;
+    }
+    const u64 rest = (u64)(off + sz) - start;
+    if (rest) {
+      const double c = (double)rest * COST_GEN * S;
+      blk[nb++] = {start, start + rest, S, false, acc, acc + c};
+      acc += c;
+    }
+    off += sz;
+  }
+  const u64 total = (u64)off;
+  bounds[0] = 0;
+  bounds[G] = total;
+  for (u32 g = 1; g < G; ++g) {
+    const double target = acc * (double)g / (double)G;
+    u64 b = total;
+    for (int i = 0; i < nb; ++i) {
+      if (target > blk[i].c1) continue;
+      const Blk &B = blk[i];
+      if (!B.r1) {
+        const double f = (B.c1 > B.c0) ? (target - B.c0) / (B.c1 - B.c0) : 0.0;
+        b = B.lo + (u64)(f * (double)(B.hi - B.lo));
+      } else {  // bisection on the cut rank: the prefix cost is monotone
+        u64 a = 0, z = B.hi - B.lo;
+        while (a < z) {
+          const u64 mid = a + (z - a) / 2;
+          if (B.c0 + r1_prefix_cost((int)L, B.S, mid, B.hi - B.lo) < target) a = mid + 1;
+          else z = mid;
+        }
+        b = B.lo + a;
+      }
+      break;
+    }
+    if (b < bounds[g - 1]) b = bounds[g - 1];
+    if (b > total) b = total;
+    bounds[g] = b;
+  }
   return AUTOPIPE_OK;
 }

@@ -29,17 +29,23 @@
 // C(L-2-y, 2) candidates. Warps take tasks from a global atomic counter (persistent grid); the
 // (T, index) argmin goes lane -> warp -> block (shuffles + shared memory) -> grid (k_finalize), so the
 // result is the lexicographic (T, index) minimum whatever the task order, grid or GPU count.
+#include <cstdlib>
+
 #include "binom.cuh"
 #include "internal.h"
 
 namespace ap {
 
+constexpr int R1_MAXCHUNK = 16;
 struct R1YEntry {      // one y value of the schedule (host-built shard arithmetic, SPEC.md §5)
   int y;               // e_{S-4}
   u32 rows_per_lane;   // R
   u64 row_begin;       // first prefix row (lex rank among P-subsets of {0..y-1}) in the shard
   u64 row_end;         // one past the last
   u64 task_begin;      // global index of this y's first task
+  u32 nchunks;         // a row's x range [y+1, L-3] is split into nchunks tasks (long rows only)
+  unsigned char xcut[R1_MAXCHUNK + 1];  // chunk c covers x in [xcut[c], xcut[c+1])
+  unsigned char pad[7];
 };
 
 struct R1Header {
@@ -50,6 +56,8 @@ struct R1Header {
   int hi_y, hi_x, hi_e;
   int ny;
   u32 counter;               // task counter (reset by the header copy before each launch)
+  u32 share;                 // 1: lanes share the grid's best T (theta below)
+  u64 theta;                 // smallest T found so far by any lane (UINT64_MAX at launch; atomicMin)
 };
 
 template <typename T>
@@ -307,7 +315,7 @@ __global__ void __launch_bounds__(NT, 2) k_search_r1(DevTables g, const R1Header
   FoldT<T> *fold = foldall + (threadIdx.x >> 5) * (n + 16);
   const unsigned fb = (unsigned)__cvta_generic_to_shared(fold);
   T THw_table = (T)0;  // THw the warp's folded table was built for (0 = not built)
-  u64 bestT = U64MAX, bestI = U64MAX, cnt = 0;
+  u64 bestT = U64MAX, bestI = U64MAX, cnt = 0, nrare = 0;
   const u64 ntasks = hdr.ntasks;
   int yi = 0;
   for (;;) {
@@ -315,12 +323,21 @@ __global__ void __launch_bounds__(NT, 2) k_search_r1(DevTables g, const R1Header
     if (lane == 0) task = atomicAdd(&counter_hdr->counter, 1u);
     task = __shfl_sync(0xffffffffu, task, 0);
     if (task >= ntasks) break;
+    // the grid's best T so far (any lane, any block): a candidate with a larger T cannot be the
+    // shard's minimum, so every lane may filter against it (non-strict: ties are decided exactly)
+    u64 tg = U64MAX;
+    if (lane == 0 && (hdr.share & 1)) tg = __ldcg(&counter_hdr->theta);
+    tg = __shfl_sync(0xffffffffu, tg, 0);
+    const i64 thg = tg < (u64)THETA_ALL ? (i64)tg : THETA_ALL;
     // tasks reach a warp in increasing order, so its cursor only moves forward
     while (yi + 1 < ny && yt[yi + 1].task_begin <= task) ++yi;
-    const R1YEntry ye = yt[yi];
+    const R1YEntry &ye = yt[yi];
     const int y = ye.y;
     const u64 R = ye.rows_per_lane;
-    const u64 r0 = ye.row_begin + (task - ye.task_begin) * 32ull * R + (u64)lane * R;
+    const u64 local = task - ye.task_begin, grp = local / ye.nchunks;
+    const int ch = (int)(local - grp * ye.nchunks);
+    const int xa = ye.xcut[ch], xb = ye.xcut[ch + 1];  // this task's x range [xa, xb)
+    const u64 r0 = ye.row_begin + grp * 32ull * R + (u64)lane * R;
     const u64 r1 = umin(r0 + R, ye.row_end);
     const u64 pcy = PC[(p - 1) * Lp1 + y + 1];  // start of stage p-1 (warp-uniform)
     u64 pre = (r0 < r1 && P > 0) ? lex_unrank_smem(r0, P, y, Bn) : 0ull;
@@ -348,12 +365,17 @@ __global__ void __launch_bounds__(NT, 2) k_search_r1(DevTables g, const R1Header
         }
       }
     }
+    {  // publish the warp's best seed (one atomic per warp, only if it improves the grid's bound)
+      u64 wm = bestT;
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) wm = umin(wm, __shfl_xor_sync(0xffffffffu, wm, o));
+      if (lane == 0 && wm < tg && (hdr.share & 2)) atomicMin(&counter_hdr->theta, wm);
+    }
     // strictness: theta = best while this lane's task may still hold a smaller index than its best
     bool strict = true;
     if (r0 < r1 && bestT != U64MAX) {
-      const bool lo_row = (pre == hdr.lo_pre) && (y == hdr.lo_y);
-      const int x0 = lo_row ? hdr.lo_x : y + 1, e0 = lo_row ? hdr.lo_e : y + 2;
-      const u64 first = pre | ((u64)y << (8 * P)) | ((u64)x0 << (8 * (P + 1))) | ((u64)e0 << (8 * (P + 2)));
+      // a lower bound of the lane's first candidate in this task (non-strict is always safe)
+      const u64 first = pre | ((u64)y << (8 * P)) | ((u64)xa << (8 * (P + 1))) | ((u64)(xa + 1) << (8 * (P + 2)));
       strict = hdr.off + lex_rank_smem(first, S - 1, n, Bn) > bestI;
     }
     RowBase base;
@@ -364,25 +386,22 @@ __global__ void __launch_bounds__(NT, 2) k_search_r1(DevTables g, const R1Header
       // partial rows at the shard boundaries: (x, e) range restricted, checked on the rare path
       bool lo_part = false, hi_part = false;
       i64 th = (bestT == U64MAX) ? THETA_ALL : (i64)bestT - (strict ? 1 : 0);
+      if (thg < th) th = thg;
       bool aliveP = false;
       i64 N0 = 0, N1 = 0, N2 = 0;
       if (active) {
         lo_part = (pre == hdr.lo_pre) && (y == hdr.lo_y);
         hi_part = (pre == hdr.hi_pre) && (y == hdr.hi_y);
         // evaluated candidates of this row: the (x, e) pairs y < x < e <= L-2 within the shard
-        const u64 m = (u64)(L - 2 - y);
-        u64 row_cnt = m * (m - 1) / 2;
-        if (lo_part || hi_part) {
-          auto prank = [&](int x, int e) -> u64 {  // rank of (x, e) among the row's pairs
-            u64 r = 0;
-            for (int xx = y + 1; xx < x; ++xx) r += (u64)(L - 2 - xx);
-            return r + (u64)(e - x - 1);
-          };
-          const u64 rlo = lo_part ? prank(hdr.lo_x, hdr.lo_e) : 0ull;
-          const u64 rhi = hi_part ? prank(hdr.hi_x, hdr.hi_e) + 1 : row_cnt;
-          row_cnt = rhi > rlo ? rhi - rlo : 0ull;
-        }
-        cnt += row_cnt;
+        // rank of the pair (x, e) among the row's pairs y < x < e <= L-2 (closed form)
+        auto prank = [&](int x, int e) -> u64 {
+          const u64 a = (u64)(x - y - 1), m1 = (u64)(L - 3 - y);  // m1 = pairs with x = y + 1
+          return a * m1 - a * (a - 1) / 2 + (u64)(e - x - 1);
+        };
+        u64 rlo = prank(xa, xa + 1), rhi = prank(xb, xb + 1);  // this task's x chunk
+        if (lo_part) rlo = umax(rlo, prank(hdr.lo_x, hdr.lo_e));
+        if (hi_part) rhi = umin(rhi, prank(hdr.hi_x, hdr.hi_e) + 1);
+        cnt += rhi > rlo ? rhi - rlo : 0ull;
         if (need_base) row_base<S>(PC, Z, LM, L, pre, th, base);
         aliveP = row_finish<S>(base, PC, Z, LM, L, byte_at(pre, P - 1), y, th, N0, N1, N2);
       }
@@ -416,12 +435,14 @@ __global__ void __launch_bounds__(NT, 2) k_search_r1(DevTables g, const R1Header
         const u64 cuts = pre | ((u64)y << (8 * P)) | ((u64)xk << (8 * (P + 1))) | ((u64)ee << (8 * (P + 2)));
         const u64 Tc = exact_T_r1<S>(PC, Z, LM, L, cuts);
         const u64 idx = hdr.off + lex_rank_smem(cuts, S - 1, n, Bn);
+        ++nrare;
         if (better(Tc, idx, bestT, bestI)) {
           bestT = Tc;
           bestI = idx;
         }
         strict = true;
         th = (i64)bestT - 1;
+        if (thg < th) th = thg;
         row_base<S>(PC, Z, LM, L, pre, th, base);
         aliveP = row_finish<S>(base, PC, Z, LM, L, byte_at(pre, P - 1), y, th, N0, N1, N2);
         xu.row(th, aliveP, N0, N1, N2, pcy);
@@ -449,8 +470,8 @@ __global__ void __launch_bounds__(NT, 2) k_search_r1(DevTables g, const R1Header
       // two candidates and the two compare chains are independent. Hits of x are decided at once; a
       // hit of x+1 only records where its rescan starts, and x+1 is rescanned after x is finished,
       // so candidates are always decided in increasing index order (tie-break, reading C-13).
-      for (int x = y + 1; x <= L - 3; x += 2) {
-        const bool two = x + 1 <= L - 3;
+      for (int x = xa; x < xb; x += 2) {
+        const bool two = x + 1 < xb;
         const XT xva = xt[x];
         const XT xvb = xt[two ? x + 1 : x];
         T H1a, H2a, H1b, H2b;
@@ -505,19 +526,45 @@ __global__ void __launch_bounds__(NT, 2) k_search_r1(DevTables g, const R1Header
         }
       }
     }
+    {  // publish the warp's best after the task (one reduction-atomic per warp and task: a
+       // per-improvement atomic on one address serialises at L2 and costs more than it saves)
+      u64 wm = bestT;
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) wm = umin(wm, __shfl_xor_sync(0xffffffffu, wm, o));
+      if (lane == 0 && wm < tg && (hdr.share & 2)) atomicMin(&counter_hdr->theta, wm);
+    }
   }
   block_minloc_store<NT>(bestT, bestI, cnt, out + blockIdx.x);
+  // diagnostics: rare-path decisions of the block (BlockOut.pad; read by AUTOPIPE_R1_STATS)
+  nrare = warp_sum(nrare);
+  __shared__ u64 rs[NT / 32];
+  if ((threadIdx.x & 31) == 0) rs[threadIdx.x >> 5] = nrare;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    u64 t = 0;
+    for (int i = 0; i < NT / 32; ++i) t += rs[i];
+    out[blockIdx.x].pad = t;
+  }
 }
 
 // ------------------------------------------------------------------------------------------------
 // host side: the task schedule (rows per y restricted to the shard) and the launch
 // ------------------------------------------------------------------------------------------------
-static u64 hb(int n, int k) {  // host binomial (n < 256, k <= 8); exact in u64
-  if (k < 0 || n < 0 || k > n) return 0;
-  u64 r = 1;
-  for (int i = 1; i <= k; ++i) r = r * (u64)(n - k + i) / (u64)i;
-  return r;
+static u64 env_u64(const char *name, u64 dflt) {  // tuning knobs for experiments (unset: defaults)
+  const char *v = getenv(name);
+  return (v && *v) ? strtoull(v, nullptr, 10) : dflt;
 }
+
+// host binomials C(n, k), n < 256, k <= 8 (exact in u64), built once
+static u64 g_hb[256][9];
+static void init_hb() {
+  static bool done = false;
+  if (done) return;
+  for (int n = 0; n < 256; ++n)
+    for (int k = 0; k < 9; ++k) g_hb[n][k] = (k == 0) ? 1 : (n == 0 ? 0 : g_hb[n - 1][k - 1] + g_hb[n - 1][k]);
+  done = true;
+}
+static inline u64 hb(int n, int k) { return (k < 0 || n < 0 || k > n) ? 0 : g_hb[n][k]; }
 
 static void host_unrank(u64 rank, int k, int n, int *out) {
   int x = 0;
@@ -549,6 +596,7 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
                        cudaStream_t st) {
   constexpr int P = S - 4, NT = 256;
   const int L = (int)g.L, n = L - 1, k = S - 1;
+  init_hb();
   int lo[8], hi[8];
   host_unrank(k_begin, k, n, lo);
   host_unrank(k_end - 1, k, n, hi);
@@ -558,6 +606,9 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
   R1Header *h = (R1Header *)hbuf;
   R1YEntry *yt = (R1YEntry *)(hbuf + sizeof(R1Header));
   memset(h, 0, sizeof(*h));
+  h->theta = U64MAX;
+  static const u64 share = env_u64("AUTOPIPE_R1_SHARE", 3);
+  h->share = (u32)share;
   h->off = sp.off[S];
   for (int i = 0; i < P; ++i) {
     h->lo_pre |= (u64)lo[i] << (8 * i);
@@ -583,22 +634,43 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
     cost_[y] = 150 + 26 * (m - 1) + 6 * (m * (m - 1) / 2);
     if (re_[y] > rb_[y]) total_cost += (re_[y] - rb_[y]) * cost_[y];
   }
-  const u64 lane_tasks = (u64)sms * 16 * 32 * 40;
+  static const u64 tpw = env_u64("AUTOPIPE_R1_TPW", 30), min_target = env_u64("AUTOPIPE_R1_MINTARGET", 12000);
+  const u64 lane_tasks = (u64)sms * 16 * 32 * tpw;
   u64 TARGET = total_cost / (lane_tasks ? lane_tasks : 1);
-  if (TARGET < 4000) TARGET = 4000;
+  if (TARGET < min_target) TARGET = min_target;
   for (int y = P; y <= L - 4; ++y) {
     const u64 rb = rb_[y], re = re_[y];
     if (re <= rb) continue;
     const u64 row_cost = cost_[y];
     const u64 R = row_cost >= TARGET ? 1 : (TARGET + row_cost - 1) / row_cost;
-    const u64 nt = (re - rb + 32 * R - 1) / (32 * R);
     R1YEntry &ye = yt[ny++];
+    memset(&ye, 0, sizeof(ye));
+    // a row longer than the target is split into x chunks of about equal candidate counts, so a
+    // small shard still gives every warp many tasks (a whole row can hold ~4000 candidates)
+    const int x_first = y + 1, x_end = L - 2;  // x in [y+1, L-3]
+    static const u64 max_chunks = env_u64("AUTOPIPE_R1_CHUNKS", 16);
+    u64 nch = row_cost > TARGET ? (row_cost + TARGET - 1) / TARGET : 1;
+    if (nch > max_chunks) nch = max_chunks;
+    if (nch > (u64)R1_MAXCHUNK) nch = R1_MAXCHUNK;
+    if (nch > (u64)(x_end - x_first)) nch = (u64)(x_end - x_first);
+    if (nch < 1) nch = 1;
+    const u64 m = (u64)(L - 2 - y), pairs = m * (m - 1) / 2;
+    int nc = 0;
+    ye.xcut[nc++] = (unsigned char)x_first;
+    u64 acc = 0;
+    for (int x = x_first; x < x_end && nc < (int)nch; ++x) {
+      acc += (u64)(L - 2 - x);  // pairs with this x
+      if (acc * nch >= pairs * (u64)nc && x + 1 < x_end) ye.xcut[nc++] = (unsigned char)(x + 1);
+    }
+    ye.xcut[nc] = (unsigned char)x_end;
+    const u64 nt = (re - rb + 32 * R - 1) / (32 * R);
     ye.y = y;
     ye.rows_per_lane = (u32)R;
     ye.row_begin = rb;
     ye.row_end = re;
     ye.task_begin = tasks;
-    tasks += nt;
+    ye.nchunks = (u32)nc;
+    tasks += nt * (u64)nc;
   }
   h->ny = ny;
   h->ntasks = tasks;
@@ -612,10 +684,21 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
   const size_t smem = (size_t)(n + 16) * sizeof(ColT<T>) + (size_t)n * sizeof(XT) + (size_t)S * (L + 1) * 8 +
                       2 * (size_t)(S - 1) * L * 8 + (size_t)(L + 1) * BINOM_K * 8 + (size_t)ny * sizeof(R1YEntry) + 16 +
                       (size_t)(NT / 32) * (n + 16) * sizeof(FoldT<T>);
-  cudaFuncSetAttribute(k_search_r1<S, T, NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  int per_sm = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_search_r1<S, T, NT>, NT, smem);
-  if (per_sm < 1) per_sm = 1;
+  // the attribute and the occupancy query cost microseconds each: redo them only when smem changes
+  // (per device: a process may drive several GPUs, one context each)
+  static size_t smem_set[64] = {0};
+  static int per_sm_dev[64] = {0};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 0 || dev >= 64) dev = 0;
+  if (smem != smem_set[dev]) {
+    cudaFuncSetAttribute(k_search_r1<S, T, NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    int q = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&q, k_search_r1<S, T, NT>, NT, smem);
+    per_sm_dev[dev] = q < 1 ? 1 : q;
+    smem_set[dev] = smem;
+  }
+  const int per_sm = per_sm_dev[dev];
   u64 blocks = (u64)sms * per_sm;
   const u64 need = (tasks + (NT / 32) - 1) / (NT / 32);
   if (blocks > need) blocks = need;

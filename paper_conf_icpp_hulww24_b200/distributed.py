@@ -8,7 +8,7 @@ world size.
 """
 from __future__ import annotations
 
-from typing import Callable, Optional, Tuple
+from typing import Callable, List, Optional, Tuple
 
 import torch
 import torch.distributed as dist
@@ -23,6 +23,19 @@ def shard_bounds(total: int, rank: int, world: int) -> Tuple[int, int]:
     if world < 1 or not (0 <= rank < world):
         raise ValueError("bad rank/world")
     return rank * total // world, (rank + 1) * total // world
+
+
+def balanced_bounds(L: int, N: int, s_min: int, s_max: int, flags: int, world: int) -> List[int]:
+    """world + 1 global indices splitting the space into contiguous shards of about equal device cost
+    (autopipe_balanced_shards: host-only, no GPU). Equal-candidate shards leave the last rank, whose
+    rows are short, up to ~1.3x slower than the first on the 96-layer space."""
+    import ctypes
+    from ._lib import lib
+    out = (ctypes.c_uint64 * (world + 1))()
+    rc = lib.autopipe_balanced_shards(L, N, s_min, s_max, flags, world, out)
+    if rc != 0:
+        raise ValueError("autopipe_balanced_shards failed (%d)" % rc)
+    return [int(x) for x in out]
 
 
 def minloc(T: int, idx: int, evaluated: int, group=None, device=None) -> Tuple[int, int, int]:
@@ -47,15 +60,20 @@ def minloc(T: int, idx: int, evaluated: int, group=None, device=None) -> Tuple[i
 
 def search_distributed(engine, s_min: int, s_max: int, flags: int = 0, group=None,
                        shard_search: Optional[Callable[[int, int], SearchResult]] = None,
-                       device=None) -> SearchResult:
+                       device=None, balanced: bool = True) -> SearchResult:
     """Exhaustive search of the whole space across the ranks of `group`.
 
     `shard_search(begin, end)` defaults to the engine's CUDA search of that shard; tests pass a
-    stand-in to exercise the distributed logic on CPU. The winner's record is decoded from its
+    stand-in to exercise the distributed logic on CPU. `balanced` splits by estimated device cost
+    (balanced_bounds) instead of equal candidate counts; the result is the same either way. The winner's record is decoded from its
     global index on every rank (no record broadcast needed)."""
     rank, world = dist.get_rank(group), dist.get_world_size(group)
-    total = engine.count_candidates(s_min, s_max, flags)
-    lo, hi = shard_bounds(total, rank, world)
+    if balanced:
+        b = balanced_bounds(engine.L, engine.N, s_min, s_max, flags, world)
+        lo, hi = b[rank], b[rank + 1]
+    else:
+        total = engine.count_candidates(s_min, s_max, flags)
+        lo, hi = shard_bounds(total, rank, world)
     if shard_search is None:
         def shard_search(b, e):
             return engine.search_optimum(s_min, s_max, flags, begin=b, end=e)

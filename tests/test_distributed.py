@@ -107,3 +107,31 @@ def test_search_distributed_gloo_world2_matches_single():
     out = _run(2, "search")
     for rank in (0, 1):
         assert out[rank] == (T, idx, n, encode_partition(part))
+
+
+def test_balanced_bounds_partition_the_space():
+    """autopipe_balanced_shards (host-only): contiguous, ordered, covering exactly [0, total), for
+    spaces with and without the fast kernel's blocks; G = 1 is the whole space."""
+    from math import comb
+    from oracle.enumerate import count
+    from paper_conf_icpp_hulww24_b200.distributed import balanced_bounds
+    for (L, N, smin, smax, flags) in ((96, 8, 8, 8, 0), (96, 8, 1, 8, 0), (21, 8, 1, 8, 0), (8, 4, 1, 4, 0),
+                                      (26, 8, 5, 8, 1), (18, 5, 1, 5, 1)):
+        total = count(L, N, smin, smax, flags) if L < 60 else (
+            comb(95, 7) if smin == 8 else sum(comb(N, S) * comb(L - 1, S - 1) for S in range(smin, smax + 1)))
+        for G in (1, 2, 3, 8):
+            b = balanced_bounds(L, N, smin, smax, flags, G)
+            assert len(b) == G + 1 and b[0] == 0 and b[-1] == total
+            assert all(x <= y for x, y in zip(b, b[1:]))
+    # the 96-layer space: later shards (short rows) get fewer candidates than earlier ones
+    b = balanced_bounds(96, 8, 8, 8, 0, 8)
+    sizes = [y - x for x, y in zip(b, b[1:])]
+    assert sizes[-1] < sizes[0] and abs(sum(sizes) - comb(95, 7)) == 0
+
+
+def test_balanced_bounds_rejects_bad_arguments():
+    from paper_conf_icpp_hulww24_b200.distributed import balanced_bounds
+    for args in ((96, 8, 0, 8, 0, 2), (96, 8, 3, 2, 0, 2), (96, 4, 1, 5, 0, 2), (96, 8, 1, 8, 2, 2),
+                 (96, 8, 1, 8, 0, 0), (0, 8, 1, 1, 0, 1), (256, 8, 1, 8, 0, 1)):
+        with pytest.raises(ValueError):
+            balanced_bounds(*args)
