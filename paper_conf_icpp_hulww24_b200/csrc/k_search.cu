@@ -128,6 +128,11 @@ int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, 
 // the winning index into its 16-byte partition record.
 // ---------------------------------------------------------------------------------------------
 __global__ void __launch_bounds__(256) k_finalize(const BlockOut *in, int n, SearchSpace sp, ResultDev *res) {
+  // binomial rows 0..L (all the unranking needs) in shared memory: the winner is decoded with
+  // fixed-length binary searches instead of a serial walk over __constant__ (which misses its cache)
+  __shared__ u64 Bn[(MAXL + 1) * BINOM_K];
+  const int rows = (sp.L > sp.N ? sp.L : sp.N) + 1;  // cut sets of {0..L-2}, compositions of {1..N}
+  for (int i = threadIdx.x; i < rows * BINOM_K; i += 256) Bn[i] = c_binom[i / BINOM_K][i % BINOM_K];
   u64 t = U64MAX, idx = U64MAX, cnt = 0;
   for (int i = threadIdx.x; i < n; i += 256) {
     const BlockOut b = in[i];
@@ -146,7 +151,7 @@ __global__ void __launch_bounds__(256) k_finalize(const BlockOut *in, int n, Sea
     if (slot.idx != U64MAX) {
       int S;
       u64 Rp, cuts;
-      unrank_global(sp, slot.idx, S, Rp, cuts);
+      unrank_global_smem(sp, slot.idx, S, Rp, cuts, Bn);
       const u64 masks = masks_from(sp, S, Rp);
       rec[0] = (unsigned char)S;
       for (int s = 0; s < S - 1; ++s) rec[1 + s] = (unsigned char)byte_at(cuts, s);

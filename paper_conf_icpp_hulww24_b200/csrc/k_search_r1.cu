@@ -344,7 +344,7 @@ __global__ void __launch_bounds__(NT, 2) k_search_r1(DevTables g, const R1Header
     // Seed: the lane's first row with the remaining layers split evenly over the last three stages.
     // Its exact T (and index) tightens theta before the sweep, so far fewer candidates reach the rare
     // path while a lane's best is still poor (most visible when a GPU scans a small shard).
-    if (r0 < r1) {
+    if (r0 < r1 && ((hdr.share & 4) || tg == U64MAX)) {
       const int rem = L - 1 - y;  // layers y+1 .. L-1 for stages p-1, p, q
       int xs = y + rem / 3, es = y + (2 * rem) / 3;
       if (xs <= y) xs = y + 1;
@@ -606,8 +606,8 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
   R1Header *h = (R1Header *)hbuf;
   R1YEntry *yt = (R1YEntry *)(hbuf + sizeof(R1Header));
   memset(h, 0, sizeof(*h));
-  h->theta = U64MAX;
-  static const u64 share = env_u64("AUTOPIPE_R1_SHARE", 3);
+  h->theta = env_u64("AUTOPIPE_R1_THETA0", U64MAX);  // experiment knob: a known bound (unset: none)
+  static const u64 share = env_u64("AUTOPIPE_R1_SHARE", 7);
   h->share = (u32)share;
   h->off = sp.off[S];
   for (int i = 0; i < P; ++i) {
@@ -638,18 +638,34 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
   const u64 lane_tasks = (u64)sms * 16 * 32 * tpw;
   u64 TARGET = total_cost / (lane_tasks ? lane_tasks : 1);
   if (TARGET < min_target) TARGET = min_target;
+  // Guided sizes: warps take tasks in schedule order, so the kernel ends about one task length after
+  // the last task starts. Tasks in the final 15 % of the cost shrink linearly to 1/4 of the target
+  // (smaller ones pay more per-task overhead than they save in tail; measured on B200).
+  static const u64 guided = env_u64("AUTOPIPE_R1_GUIDED", 2);
+  u64 cum = 0;
   for (int y = P; y <= L - 4; ++y) {
     const u64 rb = rb_[y], re = re_[y];
     if (re <= rb) continue;
     const u64 row_cost = cost_[y];
-    const u64 R = row_cost >= TARGET ? 1 : (TARGET + row_cost - 1) / row_cost;
+    u64 tgt = TARGET;
+    if (guided && total_cost) {
+      const double frac = (double)cum / (double)total_cost, left = 1.0 - frac;
+      const double zone = guided == 1 ? 0.25 : 0.15, floor_ = guided == 1 ? 1.0 / 16 : 0.25;
+      if (left < zone) {
+        const double g = left / zone > floor_ ? left / zone : floor_;
+        tgt = (u64)((double)TARGET * g);
+        if (tgt < 1) tgt = 1;
+      }
+    }
+    cum += (re - rb) * row_cost;
+    const u64 R = row_cost >= tgt ? 1 : (tgt + row_cost - 1) / row_cost;
     R1YEntry &ye = yt[ny++];
     memset(&ye, 0, sizeof(ye));
     // a row longer than the target is split into x chunks of about equal candidate counts, so a
     // small shard still gives every warp many tasks (a whole row can hold ~4000 candidates)
     const int x_first = y + 1, x_end = L - 2;  // x in [y+1, L-3]
     static const u64 max_chunks = env_u64("AUTOPIPE_R1_CHUNKS", 16);
-    u64 nch = row_cost > TARGET ? (row_cost + TARGET - 1) / TARGET : 1;
+    u64 nch = row_cost > tgt ? (row_cost + tgt - 1) / tgt : 1;
     if (nch > max_chunks) nch = max_chunks;
     if (nch > (u64)R1_MAXCHUNK) nch = R1_MAXCHUNK;
     if (nch > (u64)(x_end - x_first)) nch = (u64)(x_end - x_first);
