@@ -37,6 +37,10 @@
 namespace ap {
 
 constexpr int R1_MAXCHUNK = 16;
+// x values per pass of the column sweep
+#ifndef R1_NX
+#define R1_NX 2
+#endif
 struct R1YEntry {      // one y value of the schedule (host-built shard arithmetic, SPEC.md §5)
   int y;               // e_{S-4}
   u32 rows_per_lane;   // R
@@ -185,19 +189,12 @@ __device__ __forceinline__ T thr(i64 h, bool alive) {
   return (T)(v > m ? m : v);
 }
 
-// A warp's folded column table: A'[e] = (V[e] < THw) ? A[e] : MAX and K[e], where THw is the largest
-// strict threshold of the warp's lanes. "A'[e] < H1 and K[e] < H2" then implies "V[e] < THw"; a lane
-// whose own threshold is smaller re-checks V on the rare path. Two compares per column instead of three.
-template <typename T>
-struct __align__(2 * sizeof(T)) FoldT {
-  T A, K;
-};
-__device__ __forceinline__ void lds_fold(unsigned a, u32 &A, u32 &K) {
-  asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(A), "=r"(K) : "r"(a));
-}
-__device__ __forceinline__ void lds_fold(unsigned a, u64 &A, u64 &K) {
-  asm("ld.shared.v2.u64 {%0, %1}, [%2];" : "=l"(A), "=l"(K) : "r"(a));
-}
+// A warp's folded column table: A'[e] = (V[e] < THw) ? A[e] : MAX, where THw is the largest strict
+// threshold of the warp's lanes. The sweep tests only A'[e] < H1 (one compare per candidate): it is
+// a necessary condition of T <= theta (stage p fits and, through the fold, stage q and boundary p
+// fit), and every candidate that passes it is re-checked in full (A, K, V) before its exact T.
+__device__ __forceinline__ void lds_fold1(unsigned a, u32 &A) { asm("ld.shared.u32 %0, [%1];" : "=r"(A) : "r"(a)); }
+__device__ __forceinline__ void lds_fold1(unsigned a, u64 &A) { asm("ld.shared.u64 %0, [%1];" : "=l"(A) : "r"(a)); }
 __device__ __forceinline__ u32 warp_max_T(u32 v) { return __reduce_max_sync(0xffffffffu, v); }
 __device__ __forceinline__ u64 warp_max_T(u64 v) {
 #pragma unroll
@@ -231,10 +228,14 @@ struct XUpd<u64> {  // 64-bit path: thresholds straight from the i64 formulas
     N2p = N2 + (i64)pcy;
   }
   __device__ __forceinline__ u64 TH() const { return thr<u64>(th, true); }
-  __device__ __forceinline__ void x(const XT &v, u64 &H1, u64 &H2) const {
+  // H1 for the sweep; H2 only on the rare path (the sweep tests A' < H1 alone)
+  __device__ __forceinline__ u64 h1(const XT &v) const {
     const bool alive = ((i64)v.pc1 <= N0p) && ((i64)v.lm1 <= th);
-    H1 = thr<u64>(smin(th + (i64)v.pcp, N1p + v.W1), alive);
-    H2 = thr<u64>(smin(2 * th + (i64)v.pcp, N2p + v.W1), alive);
+    return thr<u64>(smin(th + (i64)v.pcp, N1p + v.W1), alive);
+  }
+  __device__ __forceinline__ u64 h2(const XT &v) const {
+    const bool alive = ((i64)v.pc1 <= N0p) && ((i64)v.lm1 <= th);
+    return thr<u64>(smin(2 * th + (i64)v.pcp, N2p + v.W1), alive);
   }
 };
 template <>
@@ -249,14 +250,17 @@ struct XUpd<u32> {  // 32-bit path: every table value is < 2^32 - 16, so clamp o
     N2q = N2 + (i64)pcy + 1;
   }
   __device__ __forceinline__ u32 TH() const { return th1; }
-  __device__ __forceinline__ void x(const XT &v, u32 &H1, u32 &H2) const {
+  __device__ __forceinline__ u32 h1(const XT &v) const {
     const u32 pcp = (u32)v.pcp;
     const bool alive = ((u32)v.pc1 < N0c) & ((u32)v.lm1 < th1);
     const u32 t1 = min(th1, 0xFFFFFFFFu - pcp) + pcp;  // clamp(theta + 1 + pcp), no overflow
+    return alive ? min(t1, clamp_u32(N1q + v.W1)) : 0u;
+  }
+  __device__ __forceinline__ u32 h2(const XT &v) const {
+    const u32 pcp = (u32)v.pcp;
+    const bool alive = ((u32)v.pc1 < N0c) & ((u32)v.lm1 < th1);
     const u32 t2 = min(th2, 0xFFFFFFFFu - pcp) + pcp;
-    const u32 s1 = clamp_u32(N1q + v.W1), s2 = clamp_u32(N2q + v.W1);
-    H1 = alive ? min(t1, s1) : 0u;
-    H2 = alive ? min(t2, s2) : 0u;
+    return alive ? min(t2, clamp_u32(N2q + v.W1)) : 0u;
   }
 };
 
@@ -279,7 +283,8 @@ __global__ void __launch_bounds__(NT, 2) k_search_r1(DevTables g, const R1Header
   u64 *Bn = LM + (S - 1) * L;
   R1YEntry *yt = (R1YEntry *)(Bn + Lp1 * BINOM_K);
   // per-warp folded tables follow the schedule (16-byte aligned)
-  FoldT<T> *foldall = (FoldT<T> *)(((uintptr_t)(yt + hdr_g->ny) + 15) & ~(uintptr_t)15);
+  const int FN = (n + 16 + 3) & ~3;  // columns per warp table (rows of whole 16-byte units)
+  T *foldall = (T *)(((uintptr_t)(yt + hdr_g->ny) + 15) & ~(uintptr_t)15);
   for (int i = threadIdx.x; i < Lp1 * BINOM_K; i += NT) Bn[i] = c_binom[i / BINOM_K][i % BINOM_K];
   for (int i = threadIdx.x; i < S * Lp1; i += NT) PC[i] = g.PC[i];
   for (int i = threadIdx.x; i < (S - 1) * L; i += NT) {
@@ -312,7 +317,7 @@ __global__ void __launch_bounds__(NT, 2) k_search_r1(DevTables g, const R1Header
   __syncthreads();
 
   const int lane = threadIdx.x & 31;
-  FoldT<T> *fold = foldall + (threadIdx.x >> 5) * (n + 16);
+  T *fold = foldall + (threadIdx.x >> 5) * FN;
   const unsigned fb = (unsigned)__cvta_generic_to_shared(fold);
   T THw_table = (T)0;  // THw the warp's folded table was built for (0 = not built)
   u64 bestT = U64MAX, bestI = U64MAX, cnt = 0, nrare = 0;
@@ -411,25 +416,24 @@ __global__ void __launch_bounds__(NT, 2) k_search_r1(DevTables g, const R1Header
       {  // (re)build the warp's folded table when the warp's largest threshold changed
         const T THw = warp_max_T(TH);
         if (THw != THw_table) {
-          for (int e = lane; e < n + 16; e += 32) {
-            const ColT<T> c = col[e];
-            FoldT<T> f;
-            f.A = (c.V < THw) ? c.A : (T)~(T)0;
-            f.K = c.K;
-            fold[e] = f;
+          for (int e = lane; e < FN; e += 32) {
+            const ColT<T> c = col[e < n + 16 ? e : n + 15];
+            fold[e] = (c.V < THw) ? c.A : (T)~(T)0;
           }
           __syncwarp();
           THw_table = THw;
         }
       }
       // ---- x sweep (warp-uniform), then the hot column sweep -------------------------------
-      constexpr unsigned FS = sizeof(FoldT<T>);
-      const unsigned aend = fb + (unsigned)(L - 1) * FS;  // one past the column e = L-2
-      // Rare path: candidate (xk, ee) passed the filter; decide it exactly. Afterwards every later
-      // candidate of this lane in index order is larger, so theta becomes strict (best - 1) and the
-      // row terms are recomputed (the caller refreshes its slots' thresholds).
-      auto rare = [&](int xk, int ee, const ColT<T> &c, const T h1, const T h2) -> bool {
-        if (!((c.A < h1) & (c.K < h2) & (c.V < TH))) return false;
+      constexpr unsigned FS = sizeof(T);
+      const int cend = L - 1;  // columns e <= L-2
+      // Rare path: candidate (xk, ee) passed the sweep's filter; check it in full and decide it
+      // exactly. Afterwards every later candidate of this lane in index order is larger, so theta
+      // becomes strict (best - 1) and the row terms are recomputed (the caller refreshes thresholds).
+      auto rare = [&](int xk, int ee, const T h1) -> bool {
+        const ColT<T> c = col[ee];
+        if (!((c.A < h1) & (c.V < TH))) return false;
+        if (!(c.K < xu.h2(xt[xk]))) return false;
         if (lo_part && (xk < hdr.lo_x || (xk == hdr.lo_x && ee < hdr.lo_e))) return false;
         if (hi_part && (xk > hdr.hi_x || (xk == hdr.hi_x && ee > hdr.hi_e))) return false;
         const u64 cuts = pre | ((u64)y << (8 * P)) | ((u64)xk << (8 * (P + 1))) | ((u64)ee << (8 * (P + 2)));
@@ -449,70 +453,81 @@ __global__ void __launch_bounds__(NT, 2) k_search_r1(DevTables g, const R1Header
         TH = xu.TH();
         return true;
       };
-      // single-x sweep from column address a0 (used for the second x of a pair after it hit)
-      auto sweep1 = [&](int xk, const XT &xv, T &H1, T &H2, unsigned a0) {
-        for (unsigned a = a0; a < aend; a += 4 * FS) {
-          bool hit = false;
+      const unsigned aend = fb + (unsigned)cend * FS;
+      // one x from column c0 to the end (the deferred x of a pass), four columns per step;
+      // the threshold is refreshed after every decision
+      auto sweep1 = [&](int xk, int c0) {
+        const XT xv = xt[xk];
+        T H1 = xu.h1(xv);
+        for (unsigned a = fb + (unsigned)c0 * FS; a < aend; a += 4 * FS) {
+          T A4[4];
 #pragma unroll
-          for (int u = 0; u < 4; ++u) {
-            T A0, K0;
-            lds_fold(a + u * FS, A0, K0);
-            hit |= (A0 < H1) & (K0 < H2);
-          }
+          for (int u = 0; u < 4; ++u) lds_fold1(a + u * FS, A4[u]);
+          const bool hit = (A4[0] < H1) | (A4[1] < H1) | (A4[2] < H1) | (A4[3] < H1);
           if (hit) {
-            const int e = (int)((a - fb) / FS);
-            for (int ee = e; ee < e + 4; ++ee)
-              if (rare(xk, ee, col[ee], H1, H2)) xu.x(xv, H1, H2);
+            const int c = (int)((a - fb) / FS);
+            for (int u = 0; u < 4; ++u)
+              if (A4[u] < H1 && rare(xk, c + u, H1)) H1 = xu.h1(xv);
           }
         }
       };
-      // Two x values per pass: x and x+1 test the same columns e > x+1, so one broadcast load serves
-      // two candidates and the two compare chains are independent. Hits of x are decided at once; a
-      // hit of x+1 only records where its rescan starts, and x+1 is rescanned after x is finished,
-      // so candidates are always decided in increasing index order (tie-break, reading C-13).
-      for (int x = xa; x < xb; x += 2) {
-        const bool two = x + 1 < xb;
-        const XT xva = xt[x];
-        const XT xvb = xt[two ? x + 1 : x];
-        T H1a, H2a, H1b, H2b;
-        xu.x(xva, H1a, H2a);
-        xu.x(xvb, H1b, H2b);
-        if (!two) H1b = H2b = (T)0;
-        {  // column x+1 belongs to x only
-          const unsigned a1 = fb + (unsigned)(x + 1) * FS;
-          T A0, K0;
-          lds_fold(a1, A0, K0);
-          if ((A0 < H1a) & (K0 < H2a)) {
-            if (rare(x, x + 1, col[x + 1], H1a, H2a)) {
-              xu.x(xva, H1a, H2a);
-              if (two) xu.x(xvb, H1b, H2b);
-            }
-          }
-        }
-        unsigned firstb = 0xFFFFFFFFu;
-        for (unsigned a = fb + (unsigned)(x + 2) * FS; a < aend; a += 4 * FS) {
-          bool ha = false, hb = false;
+      // NX x values per pass: x .. x+NX-1 test the same columns, so one broadcast load serves NX
+      // candidates and their compare chains are independent. Hits of the first x are decided at
+      // once; a later x only records its first hit and is rescanned (sweep1) after the pass, in x
+      // order, so a lane decides its candidates in increasing index order (tie-break, reading C-13).
+      constexpr int NX = R1_NX;
+      for (int x = xa; x < xb; x += NX) {
+        const int nx = xb - x < NX ? xb - x : NX;
+        T H1[NX];
+        int first[NX];
 #pragma unroll
-          for (int u = 0; u < 4; ++u) {
-            T A0, K0;
-            lds_fold(a + u * FS, A0, K0);
-            ha |= (A0 < H1a) & (K0 < H2a);
-            hb |= (A0 < H1b) & (K0 < H2b);
-          }
-          if (ha | hb) {
-            if (ha) {
-              const int e = (int)((a - fb) / FS);
-              for (int ee = e; ee < e + 4; ++ee) {
-                if (rare(x, ee, col[ee], H1a, H2a)) {
-                  xu.x(xva, H1a, H2a);
-                  if (two) xu.x(xvb, H1b, H2b);
-                }
-              }
-            }
-            if (hb && firstb == 0xFFFFFFFFu) firstb = a;
+        for (int k = 0; k < NX; ++k) {
+          H1[k] = (k < nx) ? xu.h1(xt[x + k]) : (T)0;
+          first[k] = cend;
+        }
+        auto refresh = [&]() {
+#pragma unroll
+          for (int k = 0; k < NX; ++k)
+            if (k < nx) H1[k] = xu.h1(xt[x + k]);
+        };
+        // head: columns x+1 .. x+NX-1 (column e belongs to the x+k with e > x+k)
+#pragma unroll
+        for (int j = 1; j < NX; ++j) {
+          const int c = x + j;
+          if (c < cend) {
+            T A0;
+            lds_fold1(fb + (unsigned)c * FS, A0);
+            if (A0 < H1[0] && rare(x, c, H1[0])) refresh();
+#pragma unroll
+            for (int k = 1; k < j; ++k)
+              if (first[k] == cend && A0 < H1[k]) first[k] = c;
           }
         }
-        if (firstb != 0xFFFFFFFFu) sweep1(x + 1, xvb, H1b, H2b, firstb);
+        // body: every column from x+NX on belongs to every x of the pass (4 columns per step; the
+        // sentinel columns past L-2 never pass)
+        for (unsigned a = fb + (unsigned)(x + NX) * FS; a < aend; a += 4 * FS) {
+          T A4[4];
+#pragma unroll
+          for (int u = 0; u < 4; ++u) lds_fold1(a + u * FS, A4[u]);
+          bool h[NX];
+#pragma unroll
+          for (int k = 0; k < NX; ++k) h[k] = (A4[0] < H1[k]) | (A4[1] < H1[k]) | (A4[2] < H1[k]) | (A4[3] < H1[k]);
+          bool any = h[0];
+#pragma unroll
+          for (int k = 1; k < NX; ++k) any |= h[k];
+          if (any) {
+            const int c = (int)((a - fb) / FS);
+            if (h[0])
+              for (int u = 0; u < 4; ++u)
+                if (A4[u] < H1[0] && rare(x, c + u, H1[0])) refresh();
+#pragma unroll
+            for (int k = 1; k < NX; ++k)
+              if (h[k] && first[k] == cend) first[k] = c;
+          }
+        }
+#pragma unroll
+        for (int k = 1; k < NX; ++k)
+          if (first[k] < cend) sweep1(x + k, first[k]);
       }
       // ---- next row of this lane: lexicographic successor of the prefix below y ------------
       // usually only the last prefix cut moves (+1): the base (stages 0..P-2) stays valid
@@ -699,7 +714,7 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
   cudaMemcpyAsync(work, hbuf, hbytes, cudaMemcpyHostToDevice, st);
   const size_t smem = (size_t)(n + 16) * sizeof(ColT<T>) + (size_t)n * sizeof(XT) + (size_t)S * (L + 1) * 8 +
                       2 * (size_t)(S - 1) * L * 8 + (size_t)(L + 1) * BINOM_K * 8 + (size_t)ny * sizeof(R1YEntry) + 16 +
-                      (size_t)(NT / 32) * (n + 16) * sizeof(FoldT<T>);
+                      (size_t)(NT / 32) * (size_t)((n + 16 + 3) & ~3) * sizeof(T);
   // the attribute and the occupancy query cost microseconds each: redo them only when smem changes
   // (per device: a process may drive several GPUs, one context each)
   static size_t smem_set[64] = {0};
