@@ -414,9 +414,10 @@ def main():
         dist.destroy_process_group()
 
 
-# ALU-pipe integer ops the exact per-candidate decision needs: three compares and the
-# two ANDs that combine them; a 64-bit compare is two ALU ops
-OPS_PER_CANDIDATE = {32: 5, 64: 8}
+# Algorithmic ALU-pipe integer ops per candidate: the sweep decides a candidate with
+# one compare of its folded column value A'[e] against the lane's threshold H1 (the full A, K, V
+# check runs only for the rare candidates that pass); a 64-bit compare is two ALU ops
+OPS_PER_CANDIDATE = {32: 1, 64: 2}
 
 if __name__ == "__main__":
     main()

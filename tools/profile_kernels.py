@@ -1,6 +1,7 @@
 #!/usr/bin/env python
 """One launch of each hot kernel, for ncu captures (not a benchmark):
-C4a search (u32 path), C4b search (u64 path), one 1M-record rollout batch (ResNet-50, App. B C5)."""
+C4a search (u32 path), C4b search (u64 path), one 1M-record rollout batch (ResNet-50, App. B C5),
+and one 1M-record switch-reward batch (NEXT row f2)."""
 import os
 import sys
 
@@ -30,3 +31,6 @@ t, sw = eng.rollout_rewards(recs, bytes(recs[0].cpu().numpy()))
 t2 = eng.eval_partitions(recs)
 torch.cuda.synchronize()
 print("rollout", int((t == t2).all()))
+out = eng.switch_rewards(recs, bytes(recs[0].cpu().numpy()), 100)
+torch.cuda.synchronize()
+print("switch", int(out["reward"].shape[0]))
