@@ -20,6 +20,7 @@ Modules
   rollout     rollout reward = T_ns + switch bytes (SPEC §6)
   neighbourhood  the two-worker neighbourhood by definition (NEXT f1)
   switching   switching cost as time: startup refill + weight migration, amortised reward (NEXT f2)
+  schedules   schedule variants (2BW, GPipe, DAPPLE) and the sharded parameter server (NEXT f3)
 
 Parity status: every function here is pinned by tests/test_oracle_*.py (worked examples of the
 paper, closed forms, invariants, textbook reductions, brute force). None is "parity unpinned".

@@ -16,11 +16,13 @@ from fractions import Fraction
 
 import networkx as nx
 
-from .model import Partition, ingredients
+from typing import Optional
+
+from .model import Ingredients, Partition, ingredients
 
 
-def event_graph(prof, st, part: Partition) -> nx.DiGraph:
-    ing = ingredients(prof, st, part)
+def event_graph(prof, st, part: Partition, ing: Optional[Ingredients] = None) -> nx.DiGraph:
+    ing = ing if ing is not None else ingredients(prof, st, part)
     S = part.S
     g = nx.DiGraph()
 
@@ -77,12 +79,12 @@ def event_graph(prof, st, part: Partition) -> nx.DiGraph:
     return g
 
 
-def ceil_max_cycle_ratio(prof, st, part: Partition) -> int:
+def ceil_max_cycle_ratio(prof, st, part: Partition, ing: Optional[Ingredients] = None) -> int:
     """ceil(lambda) without enumerating cycles: the smallest integer theta such that no cycle has
     sum(durations) - theta * sum(tokens) > 0, found by binary search on theta with a Bellman-Ford
     positive-cycle test (longest paths from a virtual source). Used by ``sim.time_ns`` when the
     simulation's transient is too long to wait for (two near-equal cycle ratios)."""
-    g = event_graph(prof, st, part)
+    g = event_graph(prof, st, part, ing)
     nodes = list(g.nodes)
     pos = {v: i for i, v in enumerate(nodes)}
     dur = [g.nodes[v]["dur"] for v in nodes]

@@ -243,35 +243,42 @@ def _allreduce_slope(sched: Schedule, s: int, j0: int, c: int, lam_c: Fraction,
             raise NoPeriod("all-reduce chain did not settle within %d rounds" % max_rounds)
 
 
-def simulate(prof, st, part: Partition, max_rounds: int = MAX_ROUNDS) -> Fraction:
-    """Exact steady-state time per mini-batch lambda (SPEC §3 'Result'), as a Fraction.
-    Raises NoPeriod if the periodic regime is not reached within max_rounds rounds."""
-    sched = Schedule(ingredients(prof, st, part))
+def steady_state(sched: Schedule, max_rounds: int = MAX_ROUNDS) -> Tuple[int, int, int]:
+    """(j0, c, D): the compute events of ``sched`` are periodic from round j0 with period c and shift D
+    (lambda_compute = D / c), combining the independent groups of ``Schedule.components``."""
     periods = [compute_period(sched, comp, max_rounds) for comp in sched.components()]
-    lam = max(Fraction(D, c) for (_, c, D) in periods)
     if len(periods) == 1:
-        j0, c, D = periods[0]
-    else:
-        # S = 1 with replicas: each replica runs back to back from t = 0, so B_w(k) = (k+1) X_w exactly
-        # (its round vector repeats from round 0 with period 1); the slowest replica is the max at
-        # every k, hence max_w B_w(k) is periodic from 0 with period 1 and shift max_w X_w.
-        assert all(j0 == 0 and c == 1 for (j0, c, _) in periods)
-        j0, c, D = 0, 1, max(D for (_, _, D) in periods)
+        return periods[0]
+    # S = 1 with replicas: each replica runs back to back from t = 0, so B_w(k) = (k+1) X_w exactly
+    # (its round vector repeats from round 0 with period 1); the slowest replica is the max at
+    # every k, hence max_w B_w(k) is periodic from 0 with period 1 and shift max_w X_w.
+    assert all(j0 == 0 and c == 1 for (j0, c, _) in periods)
+    return 0, 1, max(D for (_, _, D) in periods)
+
+
+def simulate(prof, st, part: Partition, max_rounds: int = MAX_ROUNDS, ing: Optional[Ingredients] = None
+             ) -> Fraction:
+    """Exact steady-state time per mini-batch lambda (SPEC §3 'Result'), as a Fraction.
+    Raises NoPeriod if the periodic regime is not reached within max_rounds rounds. ``ing`` replaces
+    the ingredients of SPEC §2-3 (used by the PS synchronisation of oracle/schedules.py)."""
+    sched = Schedule(ing if ing is not None else ingredients(prof, st, part))
+    j0, c, D = steady_state(sched, max_rounds)
+    lam = Fraction(D, c)
     for s in range(part.S):
         if len(part.W[s]) >= 2:
             lam = max(lam, _allreduce_slope(sched, s, j0, c, Fraction(D, c), max_rounds))
     return lam
 
 
-def time_ns(prof, st, part: Optional[Partition]) -> int:
+def time_ns(prof, st, part: Optional[Partition], ing: Optional[Ingredients] = None) -> int:
     """T_ns = ceil(lambda) (reading C-7); UINT64_MAX for an invalid record."""
     if part is None:
         return U64_MAX
     try:
-        lam = simulate(prof, st, part, TIME_NS_ROUNDS)
+        lam = simulate(prof, st, part, TIME_NS_ROUNDS, ing)
     except NoPeriod:
         from .cycle_ratio import ceil_max_cycle_ratio
-        return ceil_max_cycle_ratio(prof, st, part)
+        return ceil_max_cycle_ratio(prof, st, part, ing)
     return ceil_div(lam.numerator, lam.denominator)
 
 
