@@ -177,6 +177,41 @@ int autopipe_switch_rewards(autopipe_ctx *ctx, const autopipe_partition *d_parts
                             const autopipe_partition *h_current, uint64_t horizon, uint64_t *d_time_ns,
                             uint64_t *d_refill_ns, uint64_t *d_migrate_ns, uint64_t *d_reward_ns, void *stream);
 
+/* NEXT row f3 — schedule variants and the PS synchronisation scheme. The paper contrasts PipeDream's
+ * asynchronous 1F1B with the flushing pipelines GPipe (micro-batches, forward recomputation,
+ * PAPER.md:279-292) and DAPPLE and with PipeDream-2BW (double-buffered weights,
+ * coalesced weight gradients), applies AutoPipe to DAPPLE and 2BW
+ * (PAPER.md:1341-1350), and synchronises data parallelism by PS or ring all-reduce
+ * (PAPER.md:1081-1082, 1114-1117). Reading F-3 fixes the timing of each:
+ *   schedule      AUTOPIPE_SCHED_PIPEDREAM  static 1F1B steady state, sync every mini-batch (default);
+ *                 AUTOPIPE_SCHED_2BW        the same steady state, one sync per M micro-batches;
+ *                 AUTOPIPE_SCHED_GPIPE      one flushed iteration: F(0..M-1) then B(0..M-1) per worker;
+ *                 AUTOPIPE_SCHED_DAPPLE     one flushed iteration in 1F1B order (min(S-s, M) warm-up);
+ *   sync          AUTOPIPE_SYNC_RING (default) or AUTOPIPE_SYNC_PS (a parameter server sharded over
+ *                 the stage's replicas, each server taking its pushes and pulls one at a time);
+ *   micro_batches M >= 1 micro-batches per iteration (must be 1 for PIPEDREAM; <= 65536);
+ *   flags         AUTOPIPE_RECOMPUTE (GPipe only: every backward op re-runs the forward).
+ * The profile's FP/BP/O/G then describe one micro-batch, and every T_ns returned by
+ * autopipe_eval_partitions, autopipe_rollout_rewards, autopipe_search_optimum and
+ * autopipe_neighbourhood_best is the time of one iteration (M micro-batches). The setting belongs to
+ * the context and survives load_profile / set_state. Scoring calls under a schedule other than
+ * PIPEDREAM return E_OVERFLOW when 16 (M + 1) times the state's bound on modelled sums reaches 2^63
+ * (for a device state they synchronise `stream` once to read that bound); autopipe_switch_rewards
+ * needs the PIPEDREAM schedule (E_STATE otherwise; either sync). Bad values -> E_INVAL. Host-only. */
+#define AUTOPIPE_SCHED_PIPEDREAM 0u
+#define AUTOPIPE_SCHED_2BW 1u
+#define AUTOPIPE_SCHED_GPIPE 2u
+#define AUTOPIPE_SCHED_DAPPLE 3u
+#define AUTOPIPE_SYNC_RING 0u
+#define AUTOPIPE_SYNC_PS 1u
+#define AUTOPIPE_RECOMPUTE 1u
+#define AUTOPIPE_MAX_MICRO_BATCHES 65536u
+int autopipe_set_schedule(autopipe_ctx *ctx, uint32_t schedule, uint32_t sync, uint32_t micro_batches,
+                          uint32_t flags);
+/* The context's current schedule setting (any output pointer may be NULL). */
+int autopipe_get_schedule(const autopipe_ctx *ctx, uint32_t *schedule, uint32_t *sync, uint32_t *micro_batches,
+                          uint32_t *flags);
+
 /* Multi-GPU split: G + 1 global indices bounds[0] = 0 < ... <= bounds[G] = space size
  * such that the contiguous shards [bounds[g], bounds[g+1]) of the space (S in [s_min, s_max], flags as
  * in autopipe_search_optimum; L layers, N workers) cost about the same device time: the estimate

@@ -79,15 +79,16 @@ def event_graph(prof, st, part: Partition, ing: Optional[Ingredients] = None) ->
     return g
 
 
-def ceil_max_cycle_ratio(prof, st, part: Partition, ing: Optional[Ingredients] = None) -> int:
+def ceil_max_cycle_ratio(prof, st, part: Partition, ing: Optional[Ingredients] = None, scale: int = 1) -> int:
     """ceil(lambda) without enumerating cycles: the smallest integer theta such that no cycle has
     sum(durations) - theta * sum(tokens) > 0, found by binary search on theta with a Bellman-Ford
     positive-cycle test (longest paths from a virtual source). Used by ``sim.time_ns`` when the
-    simulation's transient is too long to wait for (two near-equal cycle ratios)."""
+    simulation's transient is too long to wait for (two near-equal cycle ratios). ``scale`` = k
+    returns ceil(k * lambda) instead (durations scaled by k; 2BW's iteration of k micro-batches)."""
     g = event_graph(prof, st, part, ing)
     nodes = list(g.nodes)
     pos = {v: i for i, v in enumerate(nodes)}
-    dur = [g.nodes[v]["dur"] for v in nodes]
+    dur = [g.nodes[v]["dur"] * scale for v in nodes]
     edges = [(pos[u], pos[v], g.edges[u, v]["tokens"]) for u, v in g.edges]
 
     def positive_cycle(theta: int) -> bool:

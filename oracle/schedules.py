@@ -44,7 +44,7 @@ from math import gcd
 from typing import Dict, List, Optional, Sequence, Tuple
 
 from .model import U64_MAX, Ingredients, Partition, ceil_div, ingredients, parse_record, shards, xfer
-from .sim import MAX_ROUNDS, NoPeriod, Schedule, steady_state, time_ns
+from .sim import MAX_ROUNDS, TIME_NS_ROUNDS, NoPeriod, Schedule, steady_state, time_ns
 
 PIPEDREAM, TWO_BW, GPIPE, DAPPLE = 0, 1, 2, 3
 RING, PS = 0, 1
@@ -73,7 +73,8 @@ def model_ingredients(prof, st, part: Partition, sync: int) -> Ingredients:
 
 
 # --- TWO_BW: the 1F1B steady state with one synchronisation per M micro-batches ----------------
-def _coalesced_chain_slope(sched: Schedule, s: int, M: int, d: int, j0: int, c: int, D: int) -> Fraction:
+def _coalesced_chain_slope(sched: Schedule, s: int, M: int, d: int, j0: int, c: int, D: int,
+                           max_rounds: int = MAX_ROUNDS) -> Fraction:
     """Asymptotic time per iteration of the synchronisation chain of stage s when it runs once per
     M micro-batches: SY(k) = max(Bmax(kM + M - 1), SY(k-1)) + d. With o(k) = SY(k) - Bmax(kM+M-1) - d
     >= 0 and the compute events periodic from round j0 (period c rounds, shift D), k -> k + c'
@@ -104,20 +105,32 @@ def _coalesced_chain_slope(sched: Schedule, s: int, M: int, d: int, j0: int, c: 
         if all(o(i) > 0 for i in range(k + 1, k + cp + 1)) and o(k + cp) > o(k):
             return Fraction(d)
         k += cp
-        if k * M > MAX_ROUNDS:
+        if k * M > max_rounds:
             raise NoPeriod("coalesced synchronisation did not settle")
 
 
-def two_bw_lambda(prof, st, part: Partition, M: int, sync: int) -> Fraction:
+def two_bw_lambda(prof, st, part: Partition, M: int, sync: int, max_rounds: int = MAX_ROUNDS) -> Fraction:
     """Exact steady-state time per iteration (M micro-batches) of the 2BW pipeline."""
     ing = model_ingredients(prof, st, part, sync)
     sched = Schedule(ing)
-    j0, c, D = steady_state(sched)
+    j0, c, D = steady_state(sched, max_rounds)
     lam = Fraction(M * D, c)
     for s in range(part.S):
         if len(part.W[s]) >= 2:
-            lam = max(lam, _coalesced_chain_slope(sched, s, M, ing.ar[s], j0, c, D))
+            lam = max(lam, _coalesced_chain_slope(sched, s, M, ing.ar[s], j0, c, D, max_rounds))
     return lam
+
+
+def two_bw_time_ns_cycles(prof, st, part: Partition, M: int, sync: int) -> int:
+    """ceil of the 2BW time per iteration without waiting for the periodic regime (R-2):
+    ceil(M * lambda_compute) from the max cycle ratio of the 1F1B event graph with the per-mini-batch
+    synchronisation removed (durations scaled by M), and the coalesced chain's own rate d (nothing
+    waits for it, so its slope is max(M lambda_compute, d) by the backlog argument above)."""
+    from .cycle_ratio import ceil_max_cycle_ratio
+    ing = model_ingredients(prof, st, part, sync)
+    sync_d = [ing.ar[s] for s in range(part.S) if len(part.W[s]) >= 2]
+    ing.ar = [0] * part.S
+    return max([ceil_max_cycle_ratio(prof, st, part, ing, scale=M)] + sync_d)
 
 
 # --- GPIPE / DAPPLE: one flushed iteration -------------------------------------------------------
@@ -271,7 +284,10 @@ def model_time_ns(prof, st, part: Optional[Partition], schedule: int = PIPEDREAM
     if schedule == PIPEDREAM:
         return time_ns(prof, st, part, model_ingredients(prof, st, part, sync))
     if schedule == TWO_BW:
-        lam = two_bw_lambda(prof, st, part, M, sync)
+        try:
+            lam = two_bw_lambda(prof, st, part, M, sync, TIME_NS_ROUNDS)
+        except NoPeriod:
+            return two_bw_time_ns_cycles(prof, st, part, M, sync)
         return ceil_div(lam.numerator, lam.denominator)
     if schedule in (GPIPE, DAPPLE):
         return flush_makespan(prof, st, part, schedule, M, recompute and schedule == GPIPE, sync)

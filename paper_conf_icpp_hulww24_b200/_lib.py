@@ -19,6 +19,11 @@ AUTOPIPE_E_OVERFLOW = -3
 AUTOPIPE_E_CUDA = -4
 AUTOPIPE_E_NOMEM = -5
 USE_ALL_WORKERS = 1
+# row f3 (schedule variants, reading F-3)
+SCHED_PIPEDREAM, SCHED_2BW, SCHED_GPIPE, SCHED_DAPPLE = 0, 1, 2, 3
+SYNC_RING, SYNC_PS = 0, 1
+RECOMPUTE = 1
+MAX_MICRO_BATCHES = 65536
 
 ERROR_NAMES = {AUTOPIPE_E_INVAL: "AUTOPIPE_E_INVAL", AUTOPIPE_E_STATE: "AUTOPIPE_E_STATE",
                AUTOPIPE_E_OVERFLOW: "AUTOPIPE_E_OVERFLOW", AUTOPIPE_E_CUDA: "AUTOPIPE_E_CUDA",
@@ -30,7 +35,8 @@ SYMBOLS = ["autopipe_create", "autopipe_destroy", "autopipe_last_error", "autopi
            "autopipe_rollout_rewards", "autopipe_count_candidates", "autopipe_decode_index",
            "autopipe_int_path", "autopipe_kernel_launches", "autopipe_set_timing",
            "autopipe_last_search_ms", "autopipe_neighbourhood", "autopipe_neighbourhood_best",
-           "autopipe_switch_rewards", "autopipe_balanced_shards"]
+           "autopipe_switch_rewards", "autopipe_balanced_shards", "autopipe_set_schedule",
+           "autopipe_get_schedule"]
 
 
 class Partition(ctypes.Structure):
@@ -80,6 +86,8 @@ def _load():
         "autopipe_neighbourhood_best": (i32, [P, ctypes.POINTER(Partition), ctypes.POINTER(Result), P]),
         "autopipe_switch_rewards": (i32, [P, P, u64, ctypes.POINTER(Partition), u64, P, P, P, P, P]),
         "autopipe_balanced_shards": (i32, [u32, u32, u32, u32, u32, u32, pu64]),
+        "autopipe_set_schedule": (i32, [P, u32, u32, u32, u32]),
+        "autopipe_get_schedule": (i32, [P] + [ctypes.POINTER(ctypes.c_uint32)] * 4),
     }
     for name, (res, args) in sig.items():
         fn = getattr(lib, name)

@@ -30,6 +30,7 @@ struct autopipe_ctx {
   u64 launches = 0;
   u64 maxOG = 0, sumP = 0;
   u64 bound = 0;  // the state's bound on modelled sums (SPEC.md §7)
+  ModelP model{SCHED_PIPEDREAM, SYNC_RING, 1, 0};  // row f3: schedule variant + sync scheme
   DevTables tab{};
   // device buffers
   u64 *d_raw = nullptr;      // fp [8*255] | bp [8*255] | P [255] | tau [64]
@@ -310,6 +311,48 @@ static int sync_status(autopipe_ctx *c, cudaStream_t st) {
   return AUTOPIPE_OK;
 }
 
+// Row f3: a schedule other than PipeDream scales sums by up to 16 (M + 1) (an iteration of M
+// micro-batches, recomputation, every op and transfer on a critical path); refuse states for which
+// that could reach 2^63. Reads the device status first for a state set from device memory.
+static int check_model(autopipe_ctx *c, cudaStream_t st) {
+  if (c->model.sched == SCHED_PIPEDREAM) return AUTOPIPE_OK;
+  int rc = sync_status(c, st);
+  if (rc) return rc;
+  if ((u128)c->bound * 16u * ((u128)c->model.M + 1) >= ((u128)1 << 63))
+    return fail(c, AUTOPIPE_E_OVERFLOW, "16 (M + 1) x the state's bound reaches 2^63 ns");
+  return AUTOPIPE_OK;
+}
+
+extern "C" int autopipe_set_schedule(autopipe_ctx *c, uint32_t schedule, uint32_t sync, uint32_t micro_batches,
+                                     uint32_t flags) {
+  if (!c) return AUTOPIPE_E_INVAL;
+  c->err[0] = 0;
+  if (schedule > AUTOPIPE_SCHED_DAPPLE) return fail(c, AUTOPIPE_E_INVAL, "unknown schedule %u", schedule);
+  if (sync > AUTOPIPE_SYNC_PS) return fail(c, AUTOPIPE_E_INVAL, "unknown sync scheme %u", sync);
+  if (micro_batches < 1 || micro_batches > AUTOPIPE_MAX_MICRO_BATCHES)
+    return fail(c, AUTOPIPE_E_INVAL, "micro_batches = %u outside [1, %u]", micro_batches, AUTOPIPE_MAX_MICRO_BATCHES);
+  if (schedule == AUTOPIPE_SCHED_PIPEDREAM && micro_batches != 1)
+    return fail(c, AUTOPIPE_E_INVAL, "the PipeDream schedule has one mini-batch per iteration (M = 1)");
+  if (flags & ~AUTOPIPE_RECOMPUTE) return fail(c, AUTOPIPE_E_INVAL, "unknown flags 0x%x", flags);
+  if ((flags & AUTOPIPE_RECOMPUTE) && schedule != AUTOPIPE_SCHED_GPIPE)
+    return fail(c, AUTOPIPE_E_INVAL, "AUTOPIPE_RECOMPUTE applies to the GPipe schedule only");
+  c->model.sched = schedule;
+  c->model.sync = sync;
+  c->model.M = micro_batches;
+  c->model.recompute = (flags & AUTOPIPE_RECOMPUTE) ? 1u : 0u;
+  return AUTOPIPE_OK;
+}
+
+extern "C" int autopipe_get_schedule(const autopipe_ctx *c, uint32_t *schedule, uint32_t *sync,
+                                     uint32_t *micro_batches, uint32_t *flags) {
+  if (!c) return AUTOPIPE_E_INVAL;
+  if (schedule) *schedule = c->model.sched;
+  if (sync) *sync = c->model.sync;
+  if (micro_batches) *micro_batches = c->model.M;
+  if (flags) *flags = c->model.recompute ? AUTOPIPE_RECOMPUTE : 0u;
+  return AUTOPIPE_OK;
+}
+
 extern "C" int autopipe_eval_partitions(autopipe_ctx *c, const autopipe_partition *d_parts, uint64_t count,
                                         uint64_t *d_time_ns, void *stream) {
   if (!c) return AUTOPIPE_E_INVAL;
@@ -318,10 +361,12 @@ extern "C" int autopipe_eval_partitions(autopipe_ctx *c, const autopipe_partitio
   if (count == 0) return AUTOPIPE_OK;
   if (!d_parts || !d_time_ns) return fail(c, AUTOPIPE_E_INVAL, "NULL device pointer");
   DeviceGuard dg(c->device);
+  int rc = check_model(c, (cudaStream_t)stream);
+  if (rc) return rc;
   // a state given in device memory has not been classified on the host yet: use the 64-bit path
   const int p32 = c->state_on_device ? 0 : c->path32;
   c->launches += launch_eval(c->tab, d_parts, count, (u64 *)d_time_ns, nullptr, nullptr, nullptr, nullptr, p32,
-                             c->sms, (cudaStream_t)stream);
+                             c->model, c->sms, (cudaStream_t)stream);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "eval kernel launch");
   return AUTOPIPE_OK;
@@ -435,6 +480,8 @@ extern "C" int autopipe_search_optimum(autopipe_ctx *c, uint32_t s_min, uint32_t
   cudaStream_t st = (cudaStream_t)stream;
   rc = sync_status(c, st);
   if (rc) return rc;
+  rc = check_model(c, st);
+  if (rc) return rc;
   if (c->timing) cudaEventRecord(c->ev0, st);
   int used = 0;
   // Split [begin, end) into the r = 1 block of each S (rho = 0: fast kernel) and the rest (generic).
@@ -445,7 +492,9 @@ extern "C" int autopipe_search_optimum(autopipe_ctx *c, uint32_t s_min, uint32_t
     const u64 lo = cur, hi = end < bhi ? end : bhi;
     // candidates with rho = 0 are [blo, blo + ncut); rho = 0 is all-r=1 iff the first composition
     // (R = 1..S) has every r_s = 1, which holds for the default flag and for USE_ALL when N = S.
-    const bool r1 = S >= 5 && (!(flags & AUTOPIPE_USE_ALL_WORKERS) || (int)c->N == S);
+    // The fast kernel decides the PipeDream closed form; other schedules (row f3) go to the generic one.
+    const bool r1 = S >= 5 && (!(flags & AUTOPIPE_USE_ALL_WORKERS) || (int)c->N == S) &&
+                    c->model.sched == SCHED_PIPEDREAM;
     const u64 r1hi = blo + sp.ncut[S];
     if (r1 && lo < r1hi) {
       const u64 a = lo, b = hi < r1hi ? hi : r1hi;
@@ -454,13 +503,13 @@ extern "C" int autopipe_search_optimum(autopipe_ctx *c, uint32_t s_min, uint32_t
                                       MAX_BLOCKS - used, &nb, c->d_work, c->h_work, c->work_bytes, st);
       used += nb;
       if (b < hi) {
-        c->launches += launch_search_generic(c->tab, sp, b, hi, c->path32, c->sms, c->d_blocks + used, MAX_BLOCKS - used,
+        c->launches += launch_search_generic(c->tab, sp, b, hi, c->path32, c->model, c->sms, c->d_blocks + used, MAX_BLOCKS - used,
                                              &nb, st);
         used += nb;
       }
     } else {
       int nb = 0;
-      c->launches += launch_search_generic(c->tab, sp, lo, hi, c->path32, c->sms, c->d_blocks + used, MAX_BLOCKS - used,
+      c->launches += launch_search_generic(c->tab, sp, lo, hi, c->path32, c->model, c->sms, c->d_blocks + used, MAX_BLOCKS - used,
                                            &nb, st);
       used += nb;
     }
@@ -538,9 +587,11 @@ extern "C" int autopipe_rollout_rewards(autopipe_ctx *c, const autopipe_partitio
   if (count == 0) return AUTOPIPE_OK;
   if (!d_parts || !d_time_ns) return fail(c, AUTOPIPE_E_INVAL, "NULL device pointer");
   DeviceGuard dg(c->device);
+  int rc = check_model(c, (cudaStream_t)stream);
+  if (rc) return rc;
   const int p32 = c->state_on_device ? 0 : c->path32;
   c->launches += launch_eval(c->tab, d_parts, count, (u64 *)d_time_ns, (u64 *)d_switch_bytes, h_current ? &S : nullptr,
-                             &cuts, &masks, p32, c->sms, (cudaStream_t)stream);
+                             &cuts, &masks, p32, c->model, c->sms, (cudaStream_t)stream);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "rollout kernel launch");
   return AUTOPIPE_OK;
@@ -613,11 +664,13 @@ extern "C" int autopipe_neighbourhood_best(autopipe_ctx *c, const autopipe_parti
   cudaStream_t st = (cudaStream_t)stream;
   int rc = sync_status(c, st);
   if (rc) return rc;
+  rc = check_model(c, st);
+  if (rc) return rc;
   u64 nslots = 0;
   rc = neigh_prepare(c, h_current, nslots, st);
   if (rc) return rc;
   c->launches += launch_eval(c->tab, c->d_nslots, nslots, c->d_ntimes, nullptr, nullptr, nullptr, nullptr, c->path32,
-                             c->sms, st);
+                             c->model, c->sms, st);
   c->launches += launch_neigh_best(c->d_nslots, c->d_ntimes, nslots, c->d_result, st);
   cudaError_t e = cudaMemcpyAsync(c->h_result, c->d_result, sizeof(ResultDev), cudaMemcpyDeviceToHost, st);
   if (e == cudaSuccess) e = cudaStreamSynchronize(st);
@@ -641,6 +694,8 @@ extern "C" int autopipe_switch_rewards(autopipe_ctx *c, const autopipe_partition
   if (!c->has_state) return fail(c, AUTOPIPE_E_STATE, "switch rewards before set_state");
   if (!h_current) return fail(c, AUTOPIPE_E_INVAL, "NULL current partition");
   if (horizon == 0) return fail(c, AUTOPIPE_E_INVAL, "horizon must be >= 1");
+  if (c->model.sched != SCHED_PIPEDREAM)
+    return fail(c, AUTOPIPE_E_STATE, "switch rewards are defined for the PipeDream schedule (reading F-2)");
   int S = 0;
   u64 cuts = 0, masks = 0;
   if (!host_decode(h_current, c->L, c->N, S, cuts, masks))
@@ -656,7 +711,8 @@ extern "C" int autopipe_switch_rewards(autopipe_ctx *c, const autopipe_partition
   u64 sow = 0;
   for (int w = 0; w < MAXN; ++w) sow |= (u64)h_current->stage_of_worker[w] << (8 * w);
   c->launches += launch_switch(c->tab, d_parts, count, S, cuts, masks, sow, horizon, (u64 *)d_time_ns,
-                               (u64 *)d_refill_ns, (u64 *)d_migrate_ns, (u64 *)d_reward_ns, c->path32, c->sms, st);
+                               (u64 *)d_refill_ns, (u64 *)d_migrate_ns, (u64 *)d_reward_ns, c->path32, (int)c->model.sync,
+                               c->sms, st);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "switch kernel launch");
   return AUTOPIPE_OK;

@@ -38,6 +38,16 @@ struct DevTables {
   u64 *status; // [2] written by the state kernel: [0] bit0 = overflow, bit1 = 32-bit path; [1] = bound
 };
 
+// The model a scoring call evaluates (NEXT row f3, reading F-3; autopipe_set_schedule).
+enum { SCHED_PIPEDREAM = 0, SCHED_2BW = 1, SCHED_GPIPE = 2, SCHED_DAPPLE = 3 };
+enum { SYNC_RING = 0, SYNC_PS = 1 };
+struct ModelP {
+  u32 sched;      // SCHED_*
+  u32 sync;       // SYNC_*: how a replicated stage synchronises its gradients
+  u32 M;          // micro-batches per iteration (1 for PipeDream)
+  u32 recompute;  // GPipe: the backward op re-runs the forward
+};
+
 __host__ __device__ __forceinline__ u64 umax(u64 a, u64 b) { return a > b ? a : b; }
 __host__ __device__ __forceinline__ u64 umin(u64 a, u64 b) { return a < b ? a : b; }
 

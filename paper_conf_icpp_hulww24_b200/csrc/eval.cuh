@@ -103,12 +103,55 @@ __device__ __forceinline__ u64 allreduce_time(u64 Ps, u32 mask, const u64 *tau) 
   return 2ull * (u64)(r - 1) * xfer(Div8(r).ceil(Ps), tr);
 }
 
+// Sharded parameter server of a replicated stage (row f3, reading F-3; PS scheme):
+// replica i serves bytes [floor(iP/r), floor((i+1)P/r)) of the stage's weights; every other replica
+// pushes that gradient shard to it and pulls the updated shard back. A server takes its pushes one
+// after another (and sends its pulls one after another); servers work in parallel:
+//   PS = max_v sum_{u != v} xfer(|shard_v|, tau[u][v]) + max_v sum_{u != v} xfer(|shard_v|, tau[v][u]).
+__device__ __forceinline__ u64 ps_time(u64 Ps, u32 mask, const u64 *tau) {
+  const u32 r = __popc(mask);
+  const Div8 dv(r);
+  const u64 q = dv.div(Ps);
+  const u32 rem = (u32)(Ps - q * r);
+  u64 push = 0, pull = 0, lo = 0;
+  u32 mv = mask;
+  for (u32 i = 0; i < r; ++i) {
+    const int v = __ffs(mv) - 1;
+    mv &= mv - 1;
+    const u64 hi = (u64)(i + 1) * q + dv.small((i + 1) * rem);
+    const u64 sz = hi - lo;
+    lo = hi;
+    u64 in = 0, out = 0;
+    u32 mu = mask & ~(1u << v);
+    while (mu) {
+      const int u = __ffs(mu) - 1;
+      mu &= mu - 1;
+      in += xfer(sz, tau[u * 8 + v]);
+      out += xfer(sz, tau[v * 8 + u]);
+    }
+    push = umax(push, in);
+    pull = umax(pull, out);
+  }
+  return push + pull;
+}
+
+// Gradient synchronisation of a replicated stage (r >= 2) under the model's scheme.
+__device__ __forceinline__ u64 sync_time(int sync, u64 Ps, u32 mask, const u64 *tau) {
+  return sync == SYNC_PS ? ps_time(Ps, mask, tau) : allreduce_time(Ps, mask, tau);
+}
+
 // The full closed form (rows a4-a7) for one partition; S in [1, 8], the partition already validated.
 // P32: the state's r = 1 bound fits 32 bits (autopipe_set_state), so every stage value X, Y, every
 // boundary sum Z and every segment sum W(s,t) is < 2^32 - 16 and the 28 segment terms use 32-bit
-// adds and divisions by constants; the all-reduce terms (weight bytes) stay 64-bit.
-template <bool P32>
-__device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, u64 cuts, u64 masks) {
+// adds and divisions by constants; the synchronisation terms (weight bytes) stay 64-bit.
+// BW (PipeDream-2BW, row f3, reading F-3): the time of an iteration of M micro-batches of the same
+// steady state, with one synchronisation per iteration: every compute term is scaled by M before its
+// ceiling (ceil(M W / k)), the synchronisation terms are not (64-bit only; M * bound < 2^59 is
+// checked on the host).
+template <bool P32, bool BW = false>
+__device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, u64 cuts, u64 masks, int sync = SYNC_RING,
+                                                u32 M = 1) {
+  static_assert(!(P32 && BW), "the 2BW form is 64-bit");
   typedef typename std::conditional<P32, u32, u64>::type V;
   V X[MAXS], Y[MAXS], Zb[MAXS];
   V T = 0;
@@ -141,8 +184,9 @@ __device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, u64 cut
       }
       X[s] = (V)xm;
       Y[s] = (V)(fm + bm);
-      T = T > (V)xm ? T : (V)xm;
-      if (r >= 2) TAR = umax(TAR, allreduce_time(t.PP[e + 1] - t.PP[a], mask, t.tau));
+      const V xs = BW ? (V)(xm * M) : (V)xm;
+      T = T > xs ? T : xs;
+      if (r >= 2) TAR = umax(TAR, sync_time(sync, t.PP[e + 1] - t.PP[a], mask, t.tau));
     }
   }
 #pragma unroll
@@ -154,7 +198,7 @@ __device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, u64 cut
       const u64 cf = boundary_max(t.O[e], ms, mn, t.tau);
       const u64 cb = boundary_max(t.G[e + 1], mn, ms, t.tau);
       Zb[s] = (V)(cf + cb);
-      const V lm = (V)umax(cf, cb);
+      const V lm = BW ? (V)(umax(cf, cb) * M) : (V)umax(cf, cb);
       T = T > lm ? T : lm;
     }
   }
@@ -166,7 +210,7 @@ __device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, u64 cut
 #pragma unroll
       for (int u = s + 1; u < MAXS; ++u) {
         if (u < S) {
-          const V W = acc + Zb[u - 1] + X[u];
+          const V W = BW ? (acc + Zb[u - 1] + X[u]) * M : acc + Zb[u - 1] + X[u];
           const V c = (W + (V)(u - s)) / (V)(u - s + 1);
           T = T > c ? T : c;
           acc += Zb[u - 1] + Y[u];

@@ -24,11 +24,12 @@ struct ResultDev {
 int launch_build_state(const DevTables &g, const u64 *fp, const u64 *bp, const u64 *P, const u64 *tau, u64 sumP,
                        cudaStream_t st);
 int launch_eval(const DevTables &g, const void *recs, u64 count, u64 *out_t, u64 *out_sw,
-                const int *cur_S, const u64 *cur_cuts, const u64 *cur_masks, int path32, int sms, cudaStream_t st);
+                const int *cur_S, const u64 *cur_cuts, const u64 *cur_masks, int path32, const ModelP &m, int sms,
+                cudaStream_t st);
 // Generic exhaustive search over [begin, end) (any S, any composition); writes one BlockOut per block
 // into out[out_offset ...] and returns the number of blocks used via *nblocks.
-int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, u64 end, int path32, int sms,
-                          BlockOut *out, int max_blocks, int *nblocks, cudaStream_t st);
+int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, u64 end, int path32, const ModelP &m,
+                          int sms, BlockOut *out, int max_blocks, int *nblocks, cudaStream_t st);
 // Fast search over the r = 1 block of one S (all stages on one worker; SPEC.md §5, rho = 0),
 // restricted to the cut ranks [k_begin, k_end). path32 selects the 32-bit tables.
 int launch_search_r1(const DevTables &g, const SearchSpace &sp, int S, u64 k_begin, u64 k_end,
@@ -48,6 +49,6 @@ int launch_neigh_best(const void *slots, const u64 *times, u64 nslots, ResultDev
 // NEXT row f2: switching cost as time (k_switch.cu).
 int launch_switch(const DevTables &g, const void *recs, u64 count, const int cur_S, const u64 cur_cuts,
                   const u64 cur_masks, const u64 cur_sow, u64 horizon, u64 *out_t, u64 *out_refill,
-                  u64 *out_mig, u64 *out_reward, int path32, int sms, cudaStream_t st);
+                  u64 *out_mig, u64 *out_reward, int path32, int sync, int sms, cudaStream_t st);
 
 }  // namespace ap

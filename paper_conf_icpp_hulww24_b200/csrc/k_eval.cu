@@ -9,6 +9,7 @@
 // Invalid records (SPEC.md §2) score UINT64_MAX and never fail the batch.
 #include "eval.cuh"
 #include "internal.h"
+#include "sched.cuh"
 
 namespace ap {
 
@@ -17,10 +18,11 @@ struct CurPart {
   int S, valid;
 };
 
-template <bool ROLLOUT, bool P32>
+// MODE: the schedule of the model (row f3; SCHED_PIPEDREAM is the 1F1B closed form of rows a4-a7).
+template <bool ROLLOUT, bool P32, int MODE>
 __global__ void __launch_bounds__(256) k_eval(DevTables g, const uint4 *__restrict__ recs, u64 count,
                                               u64 *__restrict__ out_t, u64 *__restrict__ out_sw,
-                                              CurPart cur) {
+                                              CurPart cur, ModelP m) {
   extern __shared__ u64 sm[];
   const SmemTab t = stage_tables(g, sm);
   const int L = t.L, N = (int)g.N;
@@ -34,7 +36,7 @@ __global__ void __launch_bounds__(256) k_eval(DevTables g, const uint4 *__restri
     u64 cuts, masks;
     u64 T = U64MAX, sw = U64MAX;
     if (!overflow && decode_record(lo, hi, L, N, S, cuts, masks)) {
-      T = eval_closed_form<P32>(t, S, cuts, masks);
+      T = model_time<MODE, P32>(t, S, cuts, masks, m);
       if (ROLLOUT) sw = switch_bytes(t, S, cuts, masks, cur.S, cur.cuts, cur.masks);
     }
     out_t[i] = T;
@@ -48,8 +50,28 @@ static int grid_for(u64 count, int sms) {
   return (int)(need < cap ? (need ? need : 1) : cap);
 }
 
+template <bool ROLLOUT, bool P32, int MODE>
+static void run_eval(int grid, size_t smem, cudaStream_t st, const DevTables &g, const void *recs, u64 count,
+                     u64 *out_t, u64 *out_sw, const CurPart &cur, const ModelP &m) {
+  k_eval<ROLLOUT, P32, MODE><<<grid, 256, smem, st>>>(g, (const uint4 *)recs, count, out_t, out_sw, cur, m);
+}
+
+template <bool ROLLOUT>
+static void dispatch_eval(int grid, size_t smem, cudaStream_t st, const DevTables &g, const void *recs, u64 count,
+                          u64 *out_t, u64 *out_sw, const CurPart &cur, const ModelP &m, int path32) {
+  switch (m.sched) {
+    case SCHED_2BW: run_eval<ROLLOUT, false, SCHED_2BW>(grid, smem, st, g, recs, count, out_t, out_sw, cur, m); break;
+    case SCHED_GPIPE: run_eval<ROLLOUT, false, SCHED_GPIPE>(grid, smem, st, g, recs, count, out_t, out_sw, cur, m); break;
+    case SCHED_DAPPLE: run_eval<ROLLOUT, false, SCHED_DAPPLE>(grid, smem, st, g, recs, count, out_t, out_sw, cur, m); break;
+    default:
+      if (path32) run_eval<ROLLOUT, true, SCHED_PIPEDREAM>(grid, smem, st, g, recs, count, out_t, out_sw, cur, m);
+      else run_eval<ROLLOUT, false, SCHED_PIPEDREAM>(grid, smem, st, g, recs, count, out_t, out_sw, cur, m);
+  }
+}
+
 int launch_eval(const DevTables &g, const void *recs, u64 count, u64 *out_t, u64 *out_sw,
-                const int *cur_S, const u64 *cur_cuts, const u64 *cur_masks, int path32, int sms, cudaStream_t st) {
+                const int *cur_S, const u64 *cur_cuts, const u64 *cur_masks, int path32, const ModelP &m, int sms,
+                cudaStream_t st) {
   if (count == 0) return 0;
   const size_t smem = (size_t)smem_words(g.L, g.N) * sizeof(u64);
   CurPart cur{0, 0, 0, 0};
@@ -60,13 +82,8 @@ int launch_eval(const DevTables &g, const void *recs, u64 count, u64 *out_t, u64
     cur.valid = 1;
   }
   const int grid = grid_for(count, sms);
-  if (out_sw) {
-    if (path32) k_eval<true, true><<<grid, 256, smem, st>>>(g, (const uint4 *)recs, count, out_t, out_sw, cur);
-    else k_eval<true, false><<<grid, 256, smem, st>>>(g, (const uint4 *)recs, count, out_t, out_sw, cur);
-  } else {
-    if (path32) k_eval<false, true><<<grid, 256, smem, st>>>(g, (const uint4 *)recs, count, out_t, nullptr, cur);
-    else k_eval<false, false><<<grid, 256, smem, st>>>(g, (const uint4 *)recs, count, out_t, nullptr, cur);
-  }
+  if (out_sw) dispatch_eval<true>(grid, smem, st, g, recs, count, out_t, out_sw, cur, m, path32);
+  else dispatch_eval<false>(grid, smem, st, g, recs, count, out_t, nullptr, cur, m, path32);
   return 1;
 }
 

@@ -12,6 +12,7 @@
 #include "binom.cuh"
 #include "eval.cuh"
 #include "internal.h"
+#include "sched.cuh"
 
 namespace ap {
 
@@ -61,9 +62,9 @@ __device__ __forceinline__ void unrank_global_smem(const SearchSpace &sp, u64 id
   cuts = lex_unrank_smem(kappa, S - 1, sp.L - 1, Bn);
 }
 
-template <int NT, bool P32>
+template <int NT, bool P32, int MODE>
 __global__ void __launch_bounds__(NT) k_search_generic(DevTables g, SearchSpace sp, u64 begin, u64 end,
-                                                       u64 per_thread, BlockOut *out) {
+                                                       u64 per_thread, BlockOut *out, ModelP m) {
   extern __shared__ u64 sm[];
   // binomial rows n <= L (n = N <= 8 <= L + 1 for the compositions too) after the state tables
   u64 *Bn = sm + smem_words(g.L, g.N);
@@ -81,7 +82,7 @@ __global__ void __launch_bounds__(NT) k_search_generic(DevTables g, SearchSpace 
     unrank_global_smem(sp, i0, S, Rp, cuts, Bn);
     u64 masks = masks_from(sp, S, Rp);
     for (u64 i = i0; i < i1; ++i) {
-      const u64 T = eval_closed_form<P32>(t, S, cuts, masks);
+      const u64 T = model_time<MODE, P32>(t, S, cuts, masks, m);
       if (T < bestT) {  // indices increase along the thread's range: strict < keeps the first
         bestT = T;
         bestI = i;
@@ -103,22 +104,30 @@ __global__ void __launch_bounds__(NT) k_search_generic(DevTables g, SearchSpace 
   block_minloc_store<NT>(bestT, bestI, cnt, out + blockIdx.x);
 }
 
-int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, u64 end, int path32, int sms,
-                          BlockOut *out, int max_blocks, int *nblocks, cudaStream_t st) {
+int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, u64 end, int path32, const ModelP &m,
+                          int sms, BlockOut *out, int max_blocks, int *nblocks, cudaStream_t st) {
   constexpr int NT = 256;
   const u64 span = end - begin;
-  // at least 4 candidates per thread (the unrank is a few binary searches); up to 8 blocks per SM
-  u64 threads = (span + 3) / 4;
+  // at least 4 candidates per thread (the unrank is a few binary searches); up to 8 blocks per SM.
+  // A flushed schedule costs ~M S stage steps per candidate: one candidate per thread is enough.
+  const u64 min_per = (m.sched == SCHED_GPIPE || m.sched == SCHED_DAPPLE) ? 1 : 4;
+  u64 threads = (span + min_per - 1) / min_per;
   u64 blocks = (threads + NT - 1) / NT;
   const u64 cap = (u64)sms * 8 < (u64)max_blocks ? (u64)sms * 8 : (u64)max_blocks;
   if (blocks > cap) blocks = cap;
   if (blocks == 0) blocks = 1;
   const u64 per = (span + blocks * NT - 1) / (blocks * NT);
   const size_t smem = ((size_t)smem_words(g.L, g.N) + (size_t)((g.L + 1 > 9 ? g.L + 1 : 9) * BINOM_K)) * sizeof(u64);
-  if (path32)
-    k_search_generic<NT, true><<<(unsigned)blocks, NT, smem, st>>>(g, sp, begin, end, per ? per : 1, out);
-  else
-    k_search_generic<NT, false><<<(unsigned)blocks, NT, smem, st>>>(g, sp, begin, end, per ? per : 1, out);
+  const unsigned nbk = (unsigned)blocks;
+  const u64 pt = per ? per : 1;
+  switch (m.sched) {
+    case SCHED_2BW: k_search_generic<NT, false, SCHED_2BW><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m); break;
+    case SCHED_GPIPE: k_search_generic<NT, false, SCHED_GPIPE><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m); break;
+    case SCHED_DAPPLE: k_search_generic<NT, false, SCHED_DAPPLE><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m); break;
+    default:
+      if (path32) k_search_generic<NT, true, SCHED_PIPEDREAM><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m);
+      else k_search_generic<NT, false, SCHED_PIPEDREAM><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m);
+  }
   *nblocks = (int)blocks;
   return 1;
 }

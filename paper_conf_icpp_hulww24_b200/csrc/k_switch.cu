@@ -25,6 +25,7 @@
 // in two small per-thread arrays.
 #include "eval.cuh"
 #include "internal.h"
+#include "sched.cuh"
 
 namespace ap {
 
@@ -36,48 +37,6 @@ struct SwitchCur {
   u32 masks[MAXS];   // old stage s: worker bitmask
   int S;
 };
-
-constexpr int MAXPAIRS = 2 * MAXN;  // sum over boundaries of (r_s + r_{s+1} - 1) <= 2 sum r - (S-1)
-
-// Durations of every transfer of one boundary, in merge order (see boundary_max in eval.cuh).
-__device__ __forceinline__ int boundary_pairs(u64 A, u32 send, u32 recv, const u64 *tau, u64 *d, int n) {
-  const u32 rs = __popc(send), rr = __popc(recv);
-  if (rs == 1 && rr == 1) {
-    d[n] = xfer(A, tau[(__ffs(send) - 1) * 8 + __ffs(recv) - 1]);
-    return n + 1;
-  }
-  const Div8 ds(rs), dr(rr);
-  const u64 qs = ds.div(A), qr = dr.div(A);
-  const u32 rems = (u32)(A - qs * rs), remr = (u32)(A - qr * rr);
-  u32 i = 0, j = 0;
-  u64 lo_i = 0, lo_j = 0;
-  u64 hi_i = qs + ds.small(rems), hi_j = qr + dr.small(remr);
-  while (i < rs && j < rr) {
-    const u64 lo = umax(lo_i, lo_j), hi = umin(hi_i, hi_j);
-    if (hi > lo) d[n++] = xfer(hi - lo, tau[(__ffs(send) - 1) * 8 + __ffs(recv) - 1]);
-    const bool adv_i = hi_i <= hi_j, adv_j = hi_j <= hi_i;
-    if (adv_i) {
-      ++i; send &= send - 1;
-      lo_i = hi_i; hi_i = (u64)(i + 1) * qs + ds.small((i + 1) * rems);
-    }
-    if (adv_j) {
-      ++j; recv &= recv - 1;
-      lo_j = hi_j; hi_j = (u64)(j + 1) * qr + dr.small((j + 1) * remr);
-    }
-  }
-  return n;
-}
-
-// Barrier at `bar`, then the FIFO transfers [lo, hi) of one boundary; returns its completion.
-__device__ __forceinline__ u64 run_boundary(u64 bar, const u64 *d, u64 *lf, int lo, int hi) {
-  u64 done = bar;
-  for (int p = lo; p < hi; ++p) {
-    const u64 e = umax(bar, lf[p]) + d[p];
-    lf[p] = e;
-    done = umax(done, e);
-  }
-  return done;
-}
 
 // C_{S-1} of the startup (see the file comment). sw: byte w = stage of worker w (0xFF idle).
 __device__ __forceinline__ u64 startup_completion(const SmemTab &t, int S, u64 cuts, u64 masks, u64 sw) {
@@ -198,7 +157,7 @@ __device__ __forceinline__ u64 migrate_time(const SmemTab &t, int S, u64 cuts, u
 
 template <bool P32>
 __global__ void __launch_bounds__(256) k_switch(DevTables g, const uint4 *__restrict__ recs, u64 count,
-                                                SwitchCur cur, u64 horizon, u64 *__restrict__ out_t,
+                                                SwitchCur cur, u64 horizon, u32 sync, u64 *__restrict__ out_t,
                                                 u64 *__restrict__ out_refill, u64 *__restrict__ out_mig,
                                                 u64 *__restrict__ out_reward) {
   extern __shared__ u64 sm[];
@@ -223,7 +182,7 @@ __global__ void __launch_bounds__(256) k_switch(DevTables g, const uint4 *__rest
     u64 cuts, masks;
     u64 T = U64MAX, R = U64MAX, M = U64MAX, RW = U64MAX;
     if (!overflow && decode_record(lo, hi, L, N, S, cuts, masks)) {
-      T = eval_closed_form<P32>(t, S, cuts, masks);
+      T = eval_closed_form<P32>(t, S, cuts, masks, (int)sync);
       // per-worker layer sets, compared with the current partition's
       bool same = true;
 #pragma unroll
@@ -259,7 +218,7 @@ __global__ void __launch_bounds__(256) k_switch(DevTables g, const uint4 *__rest
 
 int launch_switch(const DevTables &g, const void *recs, u64 count, const int cur_S, const u64 cur_cuts,
                   const u64 cur_masks, const u64 cur_sow, u64 horizon, u64 *out_t, u64 *out_refill,
-                  u64 *out_mig, u64 *out_reward, int path32, int sms, cudaStream_t st) {
+                  u64 *out_mig, u64 *out_reward, int path32, int sync, int sms, cudaStream_t st) {
   if (count == 0) return 0;
   SwitchCur cur;
   cur.S = cur_S;
@@ -281,10 +240,10 @@ int launch_switch(const DevTables &g, const void *recs, u64 count, const int cur
   const u64 need = (count + 255) / 256, cap = (u64)sms * 8;
   const int grid = (int)(need < cap ? need : cap);
   if (path32)
-    k_switch<true><<<grid, 256, smem, st>>>(g, (const uint4 *)recs, count, cur, horizon, out_t, out_refill, out_mig,
+    k_switch<true><<<grid, 256, smem, st>>>(g, (const uint4 *)recs, count, cur, horizon, (u32)sync, out_t, out_refill, out_mig,
                                             out_reward);
   else
-    k_switch<false><<<grid, 256, smem, st>>>(g, (const uint4 *)recs, count, cur, horizon, out_t, out_refill, out_mig,
+    k_switch<false><<<grid, 256, smem, st>>>(g, (const uint4 *)recs, count, cur, horizon, (u32)sync, out_t, out_refill, out_mig,
                                              out_reward);
   return 1;
 }

@@ -1,0 +1,197 @@
+// sched.cuh — the flushed schedule variants of NEXT row f3 (reading F-3) and the
+// max-plus helpers they share with the startup recurrence of row f2 (k_switch.cu).
+//
+// GPipe and DAPPLE's 1F1B with flush run one iteration of M
+// micro-batches from an empty pipeline; T_ns = the time the last stage finishes its last backward
+// (plus its gradient synchronisation if replicated). One thread evaluates one partition by running
+// the schedule's own max-plus recurrence in a dependency order (no event queue):
+//   GPipe   forward phase k = 0..M-1, stages ascending: F_s(k) on every replica, forward boundary s;
+//           backward phase k = 0..M-1, stages descending: B_s(k), backward boundary s-1
+//   DAPPLE  warm-up k = 0..n_0-1, stages ascending: F_s(k) for k < n_s = min(S - s, M);
+//           rounds j = 0..M-1, stages descending: B_s(j), then F_s(j + n_s) if j + n_s < M
+// In both orders every op's inputs are produced before it (B_s(j) reads backward boundary s of j,
+// produced just before by stage s+1; F_s(k) reads forward boundary s-1 of k, produced earlier by
+// stage s-1), each worker's ops are visited in its own list order, and each boundary's transfers in
+// micro-batch order, so one "latest" value per boundary, one free time per worker (registers) and one
+// free time per directed link (the links of different boundaries are distinct) reproduce the
+// ready-driven execution exactly.
+#pragma once
+#include "eval.cuh"
+
+namespace ap {
+
+constexpr int MAXPAIRS = 2 * MAXN;  // sum over boundaries of (r_s + r_{s+1} - 1) <= 2 sum r - (S-1)
+
+// Durations of every transfer of one boundary, in merge order (see boundary_max in eval.cuh).
+__device__ __forceinline__ int boundary_pairs(u64 A, u32 send, u32 recv, const u64 *tau, u64 *d, int n) {
+  const u32 rs = __popc(send), rr = __popc(recv);
+  if (rs == 1 && rr == 1) {
+    d[n] = xfer(A, tau[(__ffs(send) - 1) * 8 + __ffs(recv) - 1]);
+    return n + 1;
+  }
+  const Div8 ds(rs), dr(rr);
+  const u64 qs = ds.div(A), qr = dr.div(A);
+  const u32 rems = (u32)(A - qs * rs), remr = (u32)(A - qr * rr);
+  u32 i = 0, j = 0;
+  u64 lo_i = 0, lo_j = 0;
+  u64 hi_i = qs + ds.small(rems), hi_j = qr + dr.small(remr);
+  while (i < rs && j < rr) {
+    const u64 lo = umax(lo_i, lo_j), hi = umin(hi_i, hi_j);
+    if (hi > lo) d[n++] = xfer(hi - lo, tau[(__ffs(send) - 1) * 8 + __ffs(recv) - 1]);
+    const bool adv_i = hi_i <= hi_j, adv_j = hi_j <= hi_i;
+    if (adv_i) {
+      ++i; send &= send - 1;
+      lo_i = hi_i; hi_i = (u64)(i + 1) * qs + ds.small((i + 1) * rems);
+    }
+    if (adv_j) {
+      ++j; recv &= recv - 1;
+      lo_j = hi_j; hi_j = (u64)(j + 1) * qr + dr.small((j + 1) * remr);
+    }
+  }
+  return n;
+}
+
+// Barrier at `bar`, then the FIFO transfers [lo, hi) of one boundary; returns its completion.
+__device__ __forceinline__ u64 run_boundary(u64 bar, const u64 *d, u64 *lf, int lo, int hi) {
+  u64 done = bar;
+  for (int p = lo; p < hi; ++p) {
+    const u64 e = umax(bar, lf[p]) + d[p];
+    lf[p] = e;
+    done = umax(done, e);
+  }
+  return done;
+}
+
+
+// T_ns of one flushed iteration (GPipe or DAPPLE) of a validated partition.
+template <int SCHED>
+__device__ __forceinline__ u64 flush_makespan(const SmemTab &t, int S, u64 cuts, u64 masks, const ModelP &m) {
+  static_assert(SCHED == SCHED_GPIPE || SCHED == SCHED_DAPPLE, "flushed schedules only");
+  const int M = (int)m.M;
+  u64 Fd[MAXN], Bd[MAXN], wf[MAXN];
+  int stg[MAXN];
+#pragma unroll
+  for (int w = 0; w < MAXN; ++w) {
+    stg[w] = 0xFF;  // idle: never matches a stage
+#pragma unroll
+    for (int s = 0; s < MAXS; ++s)
+      if (s < S && ((masks >> (8 * s + w)) & 1ull)) stg[w] = s;
+    wf[w] = 0;
+    Fd[w] = 0;
+    Bd[w] = 0;
+    const int s = stg[w];
+    if (s != 0xFF) {
+      const int a = (s == 0) ? 0 : byte_at(cuts, s - 1) + 1;
+      const int e = (s == S - 1) ? t.L - 1 : byte_at(cuts, s);
+      const Div8 dv((u32)__popc((u32)byte_at(masks, s)));
+      Fd[w] = dv.ceil(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a]);
+      Bd[w] = dv.ceil(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a]);
+      if (SCHED == SCHED_GPIPE && m.recompute) Bd[w] += Fd[w];  // the backward op re-runs the forward
+    }
+  }
+  u64 dF[MAXPAIRS], dB[MAXPAIRS], lfF[MAXPAIRS], lfB[MAXPAIRS];
+  int offF[MAXS], offB[MAXS];
+  int nf = 0, nb = 0;
+#pragma unroll
+  for (int s = 0; s < MAXS - 1; ++s) {
+    offF[s] = nf;
+    offB[s] = nb;
+    if (s < S - 1) {
+      const int e = byte_at(cuts, s);
+      const u32 ms = (u32)byte_at(masks, s), mn = (u32)byte_at(masks, s + 1);
+      nf = boundary_pairs(t.O[e], ms, mn, t.tau, dF, nf);
+      nb = boundary_pairs(t.G[e + 1], mn, ms, t.tau, dB, nb);
+    }
+  }
+  offF[MAXS - 1] = nf;
+  offB[MAXS - 1] = nb;
+  for (int p = 0; p < nf; ++p) lfF[p] = 0;
+  for (int p = 0; p < nb; ++p) lfB[p] = 0;
+
+  u64 fdl[MAXS], last[MAXS];
+#pragma unroll
+  for (int s = 0; s < MAXS; ++s) {
+    fdl[s] = 0;
+    last[s] = 0;
+  }
+  // F_s(k) on every replica of stage s, then forward boundary s
+#define AP_FWD(s_)                                                                  \
+  {                                                                                 \
+    const u64 ready = ((s_) == 0) ? 0 : fdl[(s_) > 0 ? (s_) - 1 : 0];               \
+    u64 bar = 0;                                                                    \
+    _Pragma("unroll") for (int w = 0; w < MAXN; ++w) if (stg[w] == (s_)) {          \
+      wf[w] = umax(wf[w], ready) + Fd[w];                                           \
+      bar = umax(bar, wf[w]);                                                       \
+    }                                                                               \
+    if ((s_) < S - 1) fdl[s_] = run_boundary(bar, dF, lfF, offF[s_], offF[(s_) + 1]); \
+  }
+  // B_s(k) on every replica of stage s (input: bd), then backward boundary s-1 (into bd)
+#define AP_BWD(s_, k_)                                                              \
+  {                                                                                 \
+    const u64 ready = ((s_) == S - 1) ? 0 : bd;                                     \
+    u64 bar = 0;                                                                    \
+    _Pragma("unroll") for (int w = 0; w < MAXN; ++w) if (stg[w] == (s_)) {          \
+      wf[w] = umax(wf[w], ready) + Bd[w];                                           \
+      bar = umax(bar, wf[w]);                                                       \
+    }                                                                               \
+    if ((s_) > 0) bd = run_boundary(bar, dB, lfB, offB[(s_) > 0 ? (s_) - 1 : 0], offB[s_]); \
+    if ((k_) == M - 1) last[s_] = bar;                                              \
+  }
+  if (SCHED == SCHED_GPIPE) {
+    for (int k = 0; k < M; ++k) {
+#pragma unroll
+      for (int s = 0; s < MAXS; ++s)
+        if (s < S) AP_FWD(s)
+    }
+    for (int k = 0; k < M; ++k) {
+      u64 bd = 0;
+#pragma unroll
+      for (int s = MAXS - 1; s >= 0; --s)
+        if (s < S) AP_BWD(s, k)
+    }
+  } else {
+    const int nw = S < M ? S : M;  // n_0 = min(S, M) warm-up rounds
+    for (int k = 0; k < nw; ++k) {
+#pragma unroll
+      for (int s = 0; s < MAXS; ++s)
+        if (s < S && k < S - s) AP_FWD(s)  // k < n_s = min(S - s, M) (k < M already)
+    }
+    for (int j = 0; j < M; ++j) {
+      u64 bd = 0;
+#pragma unroll
+      for (int s = MAXS - 1; s >= 0; --s) {
+        if (s < S) {
+          AP_BWD(s, j)
+          if (j + (S - s) < M) AP_FWD(s)  // F_s(j + n_s), n_s = S - s when j + n_s < M
+        }
+      }
+    }
+  }
+#undef AP_FWD
+#undef AP_BWD
+  u64 T = 0;
+#pragma unroll
+  for (int s = 0; s < MAXS; ++s) {
+    if (s < S) {
+      const u32 mask = (u32)byte_at(masks, s);
+      u64 x = last[s];
+      if (__popc(mask) >= 2) {
+        const int a = (s == 0) ? 0 : byte_at(cuts, s - 1) + 1;
+        const int e = (s == S - 1) ? t.L - 1 : byte_at(cuts, s);
+        x += sync_time((int)m.sync, t.PP[e + 1] - t.PP[a], mask, t.tau);
+      }
+      T = umax(T, x);
+    }
+  }
+  return T;
+}
+
+// T_ns of a validated partition under the model (row f3): MODE = the schedule, fixed per kernel.
+template <int MODE, bool P32>
+__device__ __forceinline__ u64 model_time(const SmemTab &t, int S, u64 cuts, u64 masks, const ModelP &m) {
+  if (MODE == SCHED_PIPEDREAM) return eval_closed_form<P32>(t, S, cuts, masks, (int)m.sync);
+  if (MODE == SCHED_2BW) return eval_closed_form<false, true>(t, S, cuts, masks, (int)m.sync, m.M);
+  return flush_makespan<MODE == SCHED_PIPEDREAM || MODE == SCHED_2BW ? SCHED_GPIPE : MODE>(t, S, cuts, masks, m);
+}
+
+}  // namespace ap

@@ -216,6 +216,20 @@ class Engine:
             path.append((r.time_ns, r.partition))
         return path
 
+    # -- NEXT row f3: schedule variants (reading F-3) -----
+    def set_schedule(self, schedule: int = _lib.SCHED_PIPEDREAM, sync: int = _lib.SYNC_RING,
+                     micro_batches: int = 1, recompute: bool = False) -> None:
+        """Select the model every later scoring call evaluates: the schedule (SCHED_PIPEDREAM, _2BW,
+        _GPIPE, _DAPPLE), the data-parallel sync (SYNC_RING, SYNC_PS), M micro-batches per
+        iteration and GPipe's forward recomputation. Times are then per iteration of M micro-batches."""
+        self._check(lib.autopipe_set_schedule(self._h, int(schedule), int(sync), int(micro_batches),
+                                              _lib.RECOMPUTE if recompute else 0))
+
+    def get_schedule(self) -> Tuple[int, int, int, bool]:
+        v = [ctypes.c_uint32() for _ in range(4)]
+        self._check(lib.autopipe_get_schedule(self._h, *[ctypes.byref(x) for x in v]))
+        return v[0].value, v[1].value, v[2].value, bool(v[3].value & _lib.RECOMPUTE)
+
     # -- support ---------------------------------------------------------------------------
     def count_candidates(self, s_min: int, s_max: int, flags: int = 0) -> int:
         v = ctypes.c_uint64()

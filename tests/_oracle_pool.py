@@ -72,3 +72,22 @@ def switch_many(prof, st, records: Sequence[bytes], current: bytes, horizon: int
         return [_switch_one(a) for a in args]
     with mp.get_context("fork").Pool(procs, initializer=_init, initargs=(prof, st)) as pool:
         return pool.map(_switch_one, args, chunksize=max(1, len(args) // (procs * 8)))
+
+
+def _sched_one(args):
+    from oracle.schedules import score_record
+    rec, model = args
+    return score_record(_CTX["prof"], _CTX["st"], rec, *model)
+
+
+def sched_many(prof, st, records: Sequence[bytes], schedule: int, sync: int, M: int, recompute: bool,
+               procs: int = 0) -> List[int]:
+    """oracle.schedules.score_record (row f3) over many records."""
+    model = (schedule, sync, M, recompute)
+    args = [(bytes(r), model) for r in records]
+    procs = procs or cores()
+    if procs <= 1 or len(args) < 64:
+        _init(prof, st)
+        return [_sched_one(a) for a in args]
+    with mp.get_context("fork").Pool(procs, initializer=_init, initargs=(prof, st)) as pool:
+        return pool.map(_sched_one, args, chunksize=max(1, len(args) // (procs * 8)))

@@ -299,6 +299,42 @@ def test_two_bw_pipeline_with_replicas():
                 expect.numerator, expect.denominator)
 
 
+def test_two_bw_cycle_route_equals_simulation():
+    """The fallback for long transients (max cycle ratio with durations scaled by M, then the sync
+    rate) equals the simulation wherever the simulation settles, with and without replicas."""
+    rng = np.random.default_rng(16)
+    for _ in range(25):
+        L, N = int(rng.integers(2, 9)), int(rng.integers(1, 6))
+        prof = W.random_profile(L, rng, f_max=300, bytes_max=10**5)
+        st = W.random_state_small(prof, N, rng, tau_max=3000)
+        p = random_part(rng, L, N)
+        for M in (1, 2, 5):
+            for sync in (SC.RING, SC.PS):
+                lam = SC.two_bw_lambda(prof, st, p, M, sync)
+                assert SC.two_bw_time_ns_cycles(prof, st, p, M, sync) == ceil_div(lam.numerator, lam.denominator)
+
+
+def test_two_bw_long_transient_state():
+    """GNMT-16 states whose 1F1B transients outlast the simulation budget (R-2) still get
+    T = max(ceil(M lambda_c), d): between M (ceil(lambda_c) - 1) and M ceil(lambda_c), or the sync d."""
+    from oracle.model import parse_record
+    prof = W.gnmt16()
+    st = W.random_state(prof, 8, np.random.default_rng(17), free_link_p=0.1)
+    recs = W.sample_records(prof.L, 8, 150, 41, random_placement_p=0.6)
+    for rec in recs:
+        p = parse_record(bytes(rec), prof.L, 8)
+        if p is None:
+            continue
+        assert SC.model_time_ns(prof, st, p, SC.TWO_BW, SC.PS, 1) == SC.model_time_ns(prof, st, p, SC.PIPEDREAM, SC.PS)
+        ing = SC.model_ingredients(prof, st, p, SC.PS)
+        d = max([ing.ar[s] for s in range(p.S) if len(p.W[s]) >= 2] + [0])
+        ing.ar = [0] * p.S
+        c1 = time_ns(prof, st, p, ing)               # ceil(lambda_compute)
+        T8 = SC.model_time_ns(prof, st, p, SC.TWO_BW, SC.PS, 8)
+        assert d <= T8 <= max(8 * c1, d)
+        assert T8 == d or T8 > 8 * (c1 - 1)
+
+
 # --------------------------------------------------------------------------------------------
 # invariants
 # --------------------------------------------------------------------------------------------

@@ -5,6 +5,7 @@
   C2 VGG-16    exhaustive search (1,184,040 candidates, replicas, heterogeneous links)
   C3 GNMT-16 / BERT-24 state trace: per state switch, set_state + full search (re-score latency)
   C5 ResNet-50 rollouts: 1M random records per step, eval and rollout (T + switch bytes)
+  f1 / f2 / f3 NEXT rows: neighbourhood step, switch rewards, schedule variants (BERT-24 search, rollouts)
 
 Used by bench.py (key "configs") and runnable on its own.
 """
@@ -97,6 +98,38 @@ def measure(device: int = 0, rollout_records: int = 1 << 20):
                                          "start_T_ns": path[0][0], "local_opt_T_ns": path[-1][0],
                                          "exhaustive_opt_T_ns": opt.time_ns,
                                          "local_over_exhaustive": path[-1][0] / opt.time_ns}
+    # f3: schedule variants on the BERT profile the paper uses for its DAPPLE / 2BW comparison
+    # (BERT-24 here), all-100 Gb/s state, M = 8 micro-batches: exhaustive search
+    # of S in [1, 8], sum r <= 8 under each model; ResNet-50 rollout records scored per schedule.
+    from paper_conf_icpp_hulww24_b200 import _lib as L_
+    prof = W.bert24()
+    st = W.trace_c3(prof)[0]
+    eng.load(prof, st)
+    n = eng.count_candidates(1, 8)
+    f3 = {}
+    for label, model in (("pipedream_ring", (L_.SCHED_PIPEDREAM, L_.SYNC_RING, 1, False)),
+                         ("pipedream_ps", (L_.SCHED_PIPEDREAM, L_.SYNC_PS, 1, False)),
+                         ("2bw_M8", (L_.SCHED_2BW, L_.SYNC_RING, 8, False)),
+                         ("gpipe_M8_recompute", (L_.SCHED_GPIPE, L_.SYNC_RING, 8, True)),
+                         ("dapple_M8", (L_.SCHED_DAPPLE, L_.SYNC_RING, 8, False))):
+        eng.set_schedule(*model)
+        ms, r = _timed(lambda: eng.search_optimum(1, 8), reps=3, warm=1)
+        rec = r.partition
+        f3[label] = {"ms_to_optimum": ms, "evals_per_s": n / (ms / 1e3), "optimum_T_ns": r.time_ns,
+                     "optimum_index": r.index, "stages": rec[0],
+                     "replicas": [sum(1 for w in range(8) if rec[8 + w] == s) for s in range(rec[0])]}
+    eng.set_schedule()
+    prof = W.resnet50()
+    st = W.rollout_state(prof, 0)
+    eng.load(prof, st)
+    for label, model in (("rollout_2bw_M8", (L_.SCHED_2BW, L_.SYNC_PS, 8, False)),
+                         ("rollout_gpipe_M8", (L_.SCHED_GPIPE, L_.SYNC_RING, 8, False)),
+                         ("rollout_dapple_M8", (L_.SCHED_DAPPLE, L_.SYNC_PS, 8, False))):
+        eng.set_schedule(*model)
+        ms, _ = _timed(lambda: eng.eval_partitions(recs, out=out_t))
+        f3[label] = {"records": rollout_records, "ms": ms, "records_per_s": rollout_records / (ms / 1e3)}
+    eng.set_schedule()
+    res["F3_schedules_bert24_M8"] = dict(candidates=n, **f3)
     eng.close()
     return res
 
