@@ -52,9 +52,9 @@ __host__ __device__ __forceinline__ u64 umax(u64 a, u64 b) { return a > b ? a : 
 __host__ __device__ __forceinline__ u64 umin(u64 a, u64 b) { return a < b ? a : b; }
 
 // ceil(x / 10^6) for the transfer time xfer(x, tau) = ceil(x * tau / 1e6) (SPEC.md §1, C-7).
+__device__ __forceinline__ u64 xfer_fs(u64 p) { return (p + 999999ull) / 1000000ull; }
 __device__ __forceinline__ u64 xfer(u64 bytes, u64 fs_per_byte) {
-  const u64 p = bytes * fs_per_byte;  // < 2^64 (set_state check)
-  return (p + 999999ull) / 1000000ull;
+  return xfer_fs(bytes * fs_per_byte);  // the product is < 2^64 (set_state check)
 }
 
 // floor(x / d) for a runtime divisor d in [1, 8] and x < 2^63 (Granlund-Montgomery with N = 63:
@@ -75,22 +75,20 @@ __device__ __forceinline__ u64 ceil_small(u64 x, u32 d) { return div_small(x + d
 // and shards). d in [1, 8]; x < 2^63.
 struct Div8 {
   u64 m;
-  u32 sh, d;
+  u32 sh, d, Ms;
   __device__ __forceinline__ explicit Div8(u32 d_) : d(d_) {
     m = (d == 3u || d == 6u) ? 0xaaaaaaaaaaaaaaabull
       : (d == 5u)            ? 0xcccccccccccccccdull
       : (d == 7u)            ? 0x924924924924924aull
                              : 0x8000000000000000ull;
     sh = (d <= 2u) ? 0u : (d <= 4u) ? 1u : 2u;
+    // floor(k / d) for 0 <= k < 64: (k * ceil(2^16 / d)) >> 16 is exact on that range
+    Ms = (d == 1u) ? 65536u : (d == 2u) ? 32768u : (d == 3u) ? 21846u : (d == 4u) ? 16384u
+       : (d == 5u) ? 13108u : (d == 6u) ? 10923u : (d == 7u) ? 9363u : 8192u;
   }
   __device__ __forceinline__ u64 div(u64 x) const { return d == 1u ? x : (__umul64hi(x, m) >> sh); }
   __device__ __forceinline__ u64 ceil(u64 x) const { return div(x + d - 1); }
-  // floor(k / d) for 0 <= k < 64: (k * ceil(2^16 / d)) >> 16 is exact on that range
-  __device__ __forceinline__ u32 small(u32 k) const {
-    const u32 M = (d == 1u) ? 65536u : (d == 2u) ? 32768u : (d == 3u) ? 21846u : (d == 4u) ? 16384u
-                : (d == 5u) ? 13108u : (d == 6u) ? 10923u : (d == 7u) ? 9363u : 8192u;
-    return (k * M) >> 16;
-  }
+  __device__ __forceinline__ u32 small(u32 k) const { return (k * Ms) >> 16; }
 };
 
 __device__ __forceinline__ int byte_at(u64 v, int i) { return (int)((v >> (8 * i)) & 0xFF); }

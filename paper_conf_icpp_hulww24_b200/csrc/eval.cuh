@@ -51,7 +51,8 @@ __device__ __forceinline__ SmemTab stage_tables(const DevTables &g, u64 *sm) {
 // Largest transfer of one stage boundary (row a5): A bytes split into r_send and r_recv equal shards
 // ([floor(iA/r), floor((i+1)A/r))); every overlapping (sender, receiver) pair is one transfer on its
 // directed link, lasting ceil(overlap * tau / 1e6). A merge walk visits the <= r_s + r_r - 1
-// overlapping pairs in order.
+// overlapping pairs in order; since the duration is monotone in overlap * tau, the walk keeps the
+// largest product and rounds once.
 __device__ __forceinline__ u64 boundary_max(u64 A, u32 send, u32 recv, const u64 *tau) {
   const u32 rs = __popc(send), rr = __popc(recv);
   if (rs == 1 && rr == 1) {
@@ -70,7 +71,7 @@ __device__ __forceinline__ u64 boundary_max(u64 A, u32 send, u32 recv, const u64
     const u64 lo = umax(lo_i, lo_j), hi = umin(hi_i, hi_j);
     if (hi > lo) {
       const int u = __ffs(send) - 1, v = __ffs(recv) - 1;
-      best = umax(best, xfer(hi - lo, tau[u * 8 + v]));
+      best = umax(best, (hi - lo) * tau[u * 8 + v]);
     }
     const bool adv_i = hi_i <= hi_j, adv_j = hi_j <= hi_i;
     if (adv_i) {
@@ -82,7 +83,7 @@ __device__ __forceinline__ u64 boundary_max(u64 A, u32 send, u32 recv, const u64
       lo_j = hi_j; hi_j = (u64)(j + 1) * qr + dr.small((j + 1) * remr);
     }
   }
-  return best;
+  return xfer_fs(best);
 }
 
 // Ring all-reduce of a replicated stage (row a6): 2(r-1) steps of a ceil(P_s/r)-byte chunk over the

@@ -18,9 +18,12 @@ struct CurPart {
   int S, valid;
 };
 
+#ifndef EVAL_MINB
+#define EVAL_MINB 4
+#endif
 // MODE: the schedule of the model (row f3; SCHED_PIPEDREAM is the 1F1B closed form of rows a4-a7).
 template <bool ROLLOUT, bool P32, int MODE>
-__global__ void __launch_bounds__(256) k_eval(DevTables g, const uint4 *__restrict__ recs, u64 count,
+__global__ void __launch_bounds__(256, MODE == SCHED_PIPEDREAM ? EVAL_MINB : 2) k_eval(DevTables g, const uint4 *__restrict__ recs, u64 count,
                                               u64 *__restrict__ out_t, u64 *__restrict__ out_sw,
                                               CurPart cur, ModelP m) {
   extern __shared__ u64 sm[];

@@ -41,6 +41,15 @@ constexpr int R1_MAXCHUNK = 16;
 #ifndef R1_NX
 #define R1_NX 2
 #endif
+// resident blocks per SM the register budget is sized for (__launch_bounds__ min blocks), per path:
+// 3 x 256 threads for the 32-bit tables (85 registers, no spills; 3.47 -> 3.30 ms for C(95,7) on
+// B200), 2 for the 64-bit ones (3 spills and runs slower)
+#ifndef R1_MINB32
+#define R1_MINB32 3
+#endif
+#ifndef R1_MINB64
+#define R1_MINB64 2
+#endif
 struct R1YEntry {      // one y value of the schedule (host-built shard arithmetic, SPEC.md §5)
   int y;               // e_{S-4}
   u32 rows_per_lane;   // R
@@ -265,7 +274,7 @@ struct XUpd<u32> {  // 32-bit path: every table value is < 2^32 - 16, so clamp o
 };
 
 template <int S, typename T, int NT>
-__global__ void __launch_bounds__(NT, 2) k_search_r1(DevTables g, const R1Header *__restrict__ hdr_g,
+__global__ void __launch_bounds__(NT, sizeof(T) == 4 ? R1_MINB32 : R1_MINB64) k_search_r1(DevTables g, const R1Header *__restrict__ hdr_g,
                                                      const R1YEntry *__restrict__ yt_g, R1Header *counter_hdr,
                                                      BlockOut *out) {
   constexpr int p = S - 2, q = S - 1, P = S - 4;
