@@ -10,6 +10,7 @@
 #include "eval.cuh"
 #include "internal.h"
 #include "sched.cuh"
+#include "sortchunk.cuh"
 
 namespace ap {
 
@@ -21,22 +22,10 @@ struct CurPart {
 #ifndef EVAL_MINB
 #define EVAL_MINB 4
 #endif
-// 1: each block scores its records in chunks sorted by shape (see k_eval)
+// 1: each block scores its records in chunks sorted by shape (sortchunk.cuh)
 #ifndef EVAL_SORT
 #define EVAL_SORT 1
 #endif
-constexpr int EV_PER = 4;              // records per thread and chunk
-constexpr int EV_CH = 256 * EV_PER;    // records per chunk
-constexpr int EV_NB = 64;              // shape buckets
-
-// Shape of a record: S and the number of extra replicas (sum r - S), 64 buckets. Records of one
-// shape run the same stage, replica and boundary loops, so a warp of them does not diverge.
-__device__ __forceinline__ u32 shape_key(const uint4 &r) {
-  const u32 S = r.x & 0xFFu;
-  const u32 n = (u32)(__popc(__vcmpne4(r.z, 0xFFFFFFFFu)) + __popc(__vcmpne4(r.w, 0xFFFFFFFFu))) >> 3;
-  return ((S & 7u) << 3) | ((n - S) & 7u);
-}
-
 template <bool ROLLOUT, bool P32, int MODE>
 __device__ __forceinline__ void score_one(const SmemTab &t, int L, int N, bool overflow, const uint4 &r, u64 i,
                                           u64 *__restrict__ out_t, u64 *__restrict__ out_sw, const CurPart &cur,
@@ -69,61 +58,9 @@ __global__ void __launch_bounds__(256, MODE == SCHED_PIPEDREAM ? EVAL_MINB : 2)
   // a state that failed the device-side overflow check (set_state_device) scores nothing
   const bool overflow = (g.status[0] & 1ull) != 0;
 #if EVAL_SORT
-  __shared__ uint4 srec[EV_CH];
-  __shared__ u32 sidx[EV_CH];
-  __shared__ u32 hist[EV_NB];
-  const int tid = threadIdx.x;
-  const u64 nch = (count + EV_CH - 1) / EV_CH;
-  for (u64 ch = blockIdx.x; ch < nch; ch += gridDim.x) {
-    const u64 base = ch * EV_CH;
-    if (tid < EV_NB) hist[tid] = 0;
-    __syncthreads();
-    uint4 rr[EV_PER];
-    u32 key[EV_PER], rank[EV_PER];
-#pragma unroll
-    for (int j = 0; j < EV_PER; ++j) {
-      const u64 i = base + (u64)(j * 256 + tid);
-      key[j] = EV_NB;
-      rank[j] = 0;
-      if (i < count) {
-        rr[j] = __ldg(recs + i);
-        key[j] = shape_key(rr[j]);
-        rank[j] = atomicAdd(&hist[key[j]], 1u);
-      }
-    }
-    __syncthreads();
-    if (tid < 32) {  // exclusive scan of the 64 bucket counts, two per lane
-      const u32 a = hist[2 * tid], b = hist[2 * tid + 1];
-      u32 v = a + b;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const u32 y = __shfl_up_sync(0xffffffffu, v, o);
-        if (tid >= o) v += y;
-      }
-      const u32 ex = v - (a + b);
-      hist[2 * tid] = ex;
-      hist[2 * tid + 1] = ex + a;
-    }
-    __syncthreads();
-#pragma unroll
-    for (int j = 0; j < EV_PER; ++j) {
-      if (key[j] < EV_NB) {
-        const u32 slot = hist[key[j]] + rank[j];
-        srec[slot] = rr[j];
-        sidx[slot] = (u32)(j * 256 + tid);
-      }
-    }
-    __syncthreads();
-    const u64 left = count - base;
-    const u32 nvalid = left < (u64)EV_CH ? (u32)left : (u32)EV_CH;
-#pragma unroll 1
-    for (int j = 0; j < EV_PER; ++j) {
-      const u32 slot = (u32)(j * 256 + tid);
-      if (slot < nvalid)
-        score_one<ROLLOUT, P32, MODE>(t, L, N, overflow, srec[slot], base + sidx[slot], out_t, out_sw, cur, m);
-    }
-    __syncthreads();  // the next chunk reuses srec / sidx / hist
-  }
+  for_each_sorted(recs, count, [&](const uint4 &r, u64 i) {
+    score_one<ROLLOUT, P32, MODE>(t, L, N, overflow, r, i, out_t, out_sw, cur, m);
+  });
 #else
   const u64 stride = (u64)gridDim.x * blockDim.x;
   for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < count; i += stride)
