@@ -34,3 +34,13 @@ print("rollout", int((t == t2).all()))
 out = eng.switch_rewards(recs, bytes(recs[0].cpu().numpy()), 100)
 torch.cuda.synchronize()
 print("switch", int(out["reward"].shape[0]))
+# NEXT row f3: the same records under the DAPPLE schedule (flushed iteration, M = 8)
+eng.set_schedule(3, 0, 8)
+t3 = eng.eval_partitions(recs)
+torch.cuda.synchronize()
+eng.set_schedule()
+print("dapple", int(t3.shape[0]))
+# C2 VGG-16: the generic search kernel (replicas, heterogeneous links)
+eng.load(W.vgg16(), W.vgg_state())
+r = eng.search_optimum(1, 8)
+print("vgg", r.time_ns, r.index)
