@@ -33,14 +33,22 @@ class Partition:
 
 
 def parse_record(rec: bytes, L: int, N: int) -> Optional[Partition]:
-    """Decode a 16-byte record (SPEC §2). Returns None for an invalid record.
+    """Decode a 16-byte record (SPEC §2) or a 32-byte wide record (NEXT row f4: S <= 16 stages,
+    N <= 16 workers, for the paper's 10-GPU testbed). Returns None if invalid.
 
-    Invalid iff: S not in [1, min(8,N)]; first S-1 cuts not strictly increasing or not < L-1;
-    a stage without a worker; a worker >= N with a stage; a stage id not in [0,S) or 0xFF.
+    16 bytes: S, last_layer[7], stage_of_worker[8]; 32 bytes: S, last_layer[15], stage_of_worker[16].
+    Invalid iff: S not in [1, min(MS, N)] (MS = 8 or 16); first S-1 cuts not strictly increasing or
+    not < L-1; a stage without a worker; a worker >= N with a stage; a stage id not in [0,S) or 0xFF.
     """
     rec = bytes(rec)
+    if len(rec) == 16:
+        MS, off = 8, 8
+    elif len(rec) == 32:
+        MS, off = 16, 16
+    else:
+        raise ValueError("a partition record has 16 or 32 bytes")
     S = rec[0]
-    if not (1 <= S <= min(8, N)):
+    if not (1 <= S <= min(MS, N)):
         return None
     cuts = list(rec[1:S])
     prev = -1
@@ -49,8 +57,8 @@ def parse_record(rec: bytes, L: int, N: int) -> Optional[Partition]:
             return None
         prev = e
     W: List[List[int]] = [[] for _ in range(S)]
-    for w in range(8):
-        s = rec[8 + w]
+    for w in range(MS):
+        s = rec[off + w]
         if s == IDLE:
             continue
         if w >= N or s >= S:
@@ -61,14 +69,16 @@ def parse_record(rec: bytes, L: int, N: int) -> Optional[Partition]:
     return Partition(S, cuts, W)
 
 
-def encode_partition(p: Partition) -> bytes:
-    rec = bytearray([IDLE] * 16)
+def encode_partition(p: Partition, wide: bool = False) -> bytes:
+    """The 16-byte record of p, or its 32-byte wide record (needed when S > 8 or a worker >= 8)."""
+    n, off = (32, 16) if wide else (16, 8)
+    rec = bytearray([IDLE] * n)
     rec[0] = p.S
     for i, e in enumerate(p.cuts):
         rec[1 + i] = e
     for s, ws in enumerate(p.W):
         for w in ws:
-            rec[8 + w] = s
+            rec[off + w] = s
     return bytes(rec)
 
 

@@ -300,6 +300,15 @@ def rollout_state(prof: Profile, step: int) -> State:
     return make_state(prof, k, nic_gbps=nic, label=f"rollout-step{step}")
 
 
+def testbed_state(prof: Profile, seed: int = 10, N: int = 10) -> State:
+    """NEXT f4: the paper's testbed size, 10 GPUs with per-GPU NIC speeds from
+    {10, 25, 40, 100} Gb/s (its network settings) and slowdowns in {1, 2} (co-located jobs), seeded."""
+    rng = np.random.default_rng(seed)
+    k = rng.integers(1, 3, size=N).tolist()
+    nic = rng.choice([10, 25, 40, 100], size=N).tolist()
+    return make_state(prof, k, nic_gbps=nic, label=f"testbed{N}-seed{seed}")
+
+
 def random_state(prof: Profile, N: int, rng: np.random.Generator, max_slow: int = 3,
                  free_link_p: float = 0.0) -> State:
     """A random heterogeneous state: per-worker slowdown, per-directed-link speed (asymmetric)."""
@@ -337,33 +346,39 @@ def random_state_small(prof: Profile, N: int, rng: np.random.Generator, tau_max:
 # Partition records (SPEC.md §2): 16 bytes = S, last_layer[7], stage_of_worker[8]
 # --------------------------------------------------------------------------------------------
 
-def encode(S: int, cuts: Sequence[int], stage_of_worker: Sequence[int]) -> bytes:
-    rec = bytearray([IDLE] * 16)
+def encode(S: int, cuts: Sequence[int], stage_of_worker: Sequence[int], wide: bool = False) -> bytes:
+    """16-byte record, or the 32-byte wide record (S, last_layer[15], stage_of_worker[16]; NEXT f4)."""
+    n, off = (32, 16) if wide else (16, 8)
+    rec = bytearray([IDLE] * n)
     rec[0] = S
     for i, e in enumerate(cuts):
         rec[1 + i] = e
     for w, s in enumerate(stage_of_worker):
-        rec[8 + w] = s
+        rec[off + w] = s
     return bytes(rec)
 
 
-def contiguous_record(L: int, cuts: Sequence[int], sizes: Sequence[int]) -> bytes:
+def contiguous_record(L: int, cuts: Sequence[int], sizes: Sequence[int], wide: bool = False) -> bytes:
     """Stage s gets the next sizes[s] workers in state order."""
     sow, w = [], 0
     for s, r in enumerate(sizes):
         sow += [s] * r
-    return encode(len(sizes), cuts, sow)
+    return encode(len(sizes), cuts, sow, wide)
 
 
 def sample_records(L: int, N: int, count: int, seed: int, random_placement_p: float = 0.5,
-                   s_max: int = 8) -> np.ndarray:
-    """C5 record sampler (App. B): S ~ U{1..min(8,N)}, uniform cut set, uniform composition with
+                   s_max: int = 8, wide: bool = False) -> np.ndarray:
+    """C5 record sampler (App. B): S ~ U{1..min(s_max,N)}, uniform cut set, uniform composition with
     sum r <= N, contiguous placement in (1-p) of the records and a random worker permutation in p.
 
-    Returns a (count, 16) uint8 array. Vectorised per S; seeded with ``numpy.random.default_rng``.
+    Returns a (count, 16) uint8 array, or (count, 32) wide records (S <= 16, N <= 16; NEXT f4).
+    Vectorised per S; seeded with ``numpy.random.default_rng``.
     """
     rng = np.random.default_rng(seed)
-    out = np.full((count, 16), IDLE, dtype=np.uint8)
+    width, off = (32, 16) if wide else (16, 8)
+    if not wide and (s_max > 8 or N > 8):
+        raise ValueError("16-byte records hold S <= 8 and N <= 8; use wide=True")
+    out = np.full((count, width), IDLE, dtype=np.uint8)
     smax = min(s_max, N, L)
     S = rng.integers(1, smax + 1, size=count)
     out[:, 0] = S
@@ -387,7 +402,7 @@ def sample_records(L: int, N: int, count: int, seed: int, random_placement_p: fl
         perms = np.argsort(rng.random((n, N)), axis=1)
         shuffled = np.take_along_axis(stage, perms, axis=1)
         stage = np.where(perm_rows[:, None], shuffled, stage)
-        out[idx, 8:8 + N] = stage.astype(np.uint8)
+        out[idx, off:off + N] = stage.astype(np.uint8)
     return out
 
 
@@ -395,19 +410,20 @@ def corrupt_records(recs: np.ndarray, L: int, N: int, seed: int, frac: float = 0
     """Mutate a fraction of records with random field edits (some stay valid, most become invalid)."""
     rng = np.random.default_rng(seed)
     out = recs.copy()
+    MS = 16 if out.shape[1] == 32 else 8
     rows = np.nonzero(rng.random(len(out)) < frac)[0]
     for r in rows:
         kind = int(rng.integers(0, 6))
         if kind == 0:
-            out[r, 0] = int(rng.choice([0, 9, 255, min(8, N) + 1]))
+            out[r, 0] = int(rng.choice([0, MS + 1, 255, min(MS, N) + 1]))
         elif kind == 1:
-            out[r, 1 + int(rng.integers(0, 7))] = int(rng.integers(0, 256))
+            out[r, 1 + int(rng.integers(0, MS - 1))] = int(rng.integers(0, 256))
         elif kind == 2:
-            out[r, 8 + int(rng.integers(0, 8))] = int(rng.integers(0, 256))
+            out[r, MS + int(rng.integers(0, MS))] = int(rng.integers(0, 256))
         elif kind == 3:
-            out[r, 8 + int(rng.integers(0, 8))] = IDLE
+            out[r, MS + int(rng.integers(0, MS))] = IDLE
         elif kind == 4:
             out[r, 1] = L - 1
         else:
-            out[r, 8 + int(rng.integers(0, 8))] = int(rng.integers(0, 8))
+            out[r, MS + int(rng.integers(0, MS))] = int(rng.integers(0, MS))
     return out
