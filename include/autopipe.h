@@ -65,6 +65,21 @@ typedef struct {
   autopipe_partition part;  /* the best candidate, decoded */
 } autopipe_result;
 
+/* NEXT row f4 — the wide record: up to 16 stages and 16 workers, for clusters beyond 8 GPUs such as
+ * the paper's 10-GPU testbed. Same meaning and validity rules as
+ * autopipe_partition with S in [1, min(16, N)]; exactly 32 bytes (two 128-bit loads). */
+#define AUTOPIPE_MAX_STAGES_W 16
+#define AUTOPIPE_MAX_WORKERS_W 16
+typedef struct {
+  uint8_t n_stages;            /* S in [1, min(16, N)] */
+  uint8_t last_layer[15];      /* e_0 < ... < e_{S-2} < L-1; entries >= S-1 ignored (write 0xFF) */
+  uint8_t stage_of_worker[16]; /* per worker w: its stage in [0, S), or 0xFF; w >= N must be 0xFF */
+} autopipe_partition_w;
+typedef struct {
+  uint64_t time_ns, index, evaluated;
+  autopipe_partition_w part;
+} autopipe_result_w;
+
 /* Create a context on CUDA device `cuda_device` (the caller's current device is left unchanged
  * on return). Returns E_INVAL for a NULL `out`, E_CUDA if the device cannot be used. */
 int autopipe_create(int cuda_device, autopipe_ctx **out);
@@ -93,8 +108,11 @@ int autopipe_load_profile(autopipe_ctx *ctx, uint32_t L, const uint64_t *act_byt
  *   link_fs_per_byte  N x N row-major: inverse bandwidth of the directed link u -> v in
  *                     femtoseconds per byte (the per-link form of B_i, reading C-5; the diagonal
  *                     is ignored; 0 = free link).
- * N in [1, 8]. Rejects (E_OVERFLOW) states whose products bytes*tau reach 2^64 or whose largest
- * modelled sum reaches 2^59 (SPEC.md §7); picks the 32-bit search path when every r=1 sum fits.
+ * N in [1, 16] (N > 8 is the wide range of row f4: the 16-byte calls then score records naming
+ * workers < 8 only, and the 16-byte search / decode / neighbourhood / switch calls return E_INVAL; use
+ * the _w calls). Rejects (E_OVERFLOW) states whose products bytes*tau reach 2^64 or whose largest
+ * modelled sum reaches 2^59 (SPEC.md §7; the bound counts 7 stage boundaries for N <= 8, 15 for
+ * N > 8); picks the 32-bit search path when every r=1 sum fits.
  * Enqueues the prefix-sum and link-table kernels on `stream` (returns before they finish).
  * Requires a loaded profile (E_STATE). */
 int autopipe_set_state(autopipe_ctx *ctx, uint32_t N, const uint64_t *fp_ns, const uint64_t *bp_ns,
@@ -177,6 +195,21 @@ int autopipe_switch_rewards(autopipe_ctx *ctx, const autopipe_partition *d_parts
                             const autopipe_partition *h_current, uint64_t horizon, uint64_t *d_time_ns,
                             uint64_t *d_refill_ns, uint64_t *d_migrate_ns, uint64_t *d_reward_ns, void *stream);
 
+/* NEXT row f4 — the wide calls: the same operations as autopipe_eval_partitions,
+ * autopipe_rollout_rewards, autopipe_search_optimum and autopipe_decode_index over 32-byte records
+ * (S <= 16 stages, N <= 16 workers), with the same arguments, ownership, ordering (SPEC.md §5 with S up
+ * to min(16, N)), error behaviour and schedule setting (row f3). The search's fast r = 1 kernel serves
+ * S in [5, 8]; every other S runs the generic kernel. A space larger than 2^64 -> E_OVERFLOW. */
+int autopipe_eval_partitions_w(autopipe_ctx *ctx, const autopipe_partition_w *d_parts, uint64_t count,
+                               uint64_t *d_time_ns, void *stream);
+int autopipe_rollout_rewards_w(autopipe_ctx *ctx, const autopipe_partition_w *d_parts, uint64_t count,
+                               const autopipe_partition_w *h_current, uint64_t *d_time_ns,
+                               uint64_t *d_switch_bytes, void *stream);
+int autopipe_search_optimum_w(autopipe_ctx *ctx, uint32_t s_min, uint32_t s_max, uint32_t flags, uint64_t begin,
+                              uint64_t end, autopipe_result_w *h_out, void *stream);
+int autopipe_decode_index_w(const autopipe_ctx *ctx, uint32_t s_min, uint32_t s_max, uint32_t flags,
+                            uint64_t index, autopipe_partition_w *out);
+
 /* NEXT row f3 — schedule variants and the PS synchronisation scheme. The paper contrasts PipeDream's
  * asynchronous 1F1B with the flushing pipelines GPipe (micro-batches, forward recomputation,
  * PAPER.md:279-292) and DAPPLE and with PipeDream-2BW (double-buffered weights,
@@ -221,7 +254,7 @@ int autopipe_get_schedule(const autopipe_ctx *ctx, uint32_t *schedule, uint32_t 
 int autopipe_balanced_shards(uint32_t L, uint32_t N, uint32_t s_min, uint32_t s_max, uint32_t flags, uint32_t G,
                              uint64_t *bounds);
 
-/* Number of candidates of a search space (requires a state for L and N). */
+/* Number of candidates of a search space (requires a state for L and N); S up to min(16, N). */
 int autopipe_count_candidates(const autopipe_ctx *ctx, uint32_t s_min, uint32_t s_max, uint32_t flags,
                               uint64_t *total);
 

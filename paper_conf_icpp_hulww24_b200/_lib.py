@@ -36,7 +36,8 @@ SYMBOLS = ["autopipe_create", "autopipe_destroy", "autopipe_last_error", "autopi
            "autopipe_int_path", "autopipe_kernel_launches", "autopipe_set_timing",
            "autopipe_last_search_ms", "autopipe_neighbourhood", "autopipe_neighbourhood_best",
            "autopipe_switch_rewards", "autopipe_balanced_shards", "autopipe_set_schedule",
-           "autopipe_get_schedule"]
+           "autopipe_get_schedule", "autopipe_eval_partitions_w", "autopipe_rollout_rewards_w",
+           "autopipe_search_optimum_w", "autopipe_decode_index_w"]
 
 
 class Partition(ctypes.Structure):
@@ -49,7 +50,18 @@ class Result(ctypes.Structure):
                 ("evaluated", ctypes.c_uint64), ("part", Partition)]
 
 
+class PartitionW(ctypes.Structure):  # row f4: S <= 16 stages, N <= 16 workers
+    _fields_ = [("n_stages", ctypes.c_uint8), ("last_layer", ctypes.c_uint8 * 15),
+                ("stage_of_worker", ctypes.c_uint8 * 16)]
+
+
+class ResultW(ctypes.Structure):
+    _fields_ = [("time_ns", ctypes.c_uint64), ("index", ctypes.c_uint64),
+                ("evaluated", ctypes.c_uint64), ("part", PartitionW)]
+
+
 assert ctypes.sizeof(Partition) == 16 and ctypes.sizeof(Result) == 40
+assert ctypes.sizeof(PartitionW) == 32 and ctypes.sizeof(ResultW) == 56
 
 
 class AutopipeError(RuntimeError):
@@ -87,6 +99,10 @@ def _load():
         "autopipe_switch_rewards": (i32, [P, P, u64, ctypes.POINTER(Partition), u64, P, P, P, P, P]),
         "autopipe_balanced_shards": (i32, [u32, u32, u32, u32, u32, u32, pu64]),
         "autopipe_set_schedule": (i32, [P, u32, u32, u32, u32]),
+        "autopipe_eval_partitions_w": (i32, [P, P, u64, P, P]),
+        "autopipe_rollout_rewards_w": (i32, [P, P, u64, ctypes.POINTER(PartitionW), P, P, P]),
+        "autopipe_search_optimum_w": (i32, [P, u32, u32, u32, u64, u64, ctypes.POINTER(ResultW), P]),
+        "autopipe_decode_index_w": (i32, [P, u32, u32, u32, u64, ctypes.POINTER(PartitionW)]),
         "autopipe_get_schedule": (i32, [P] + [ctypes.POINTER(ctypes.c_uint32)] * 4),
     }
     for name, (res, args) in sig.items():

@@ -81,12 +81,16 @@ struct DeviceGuard {
   }
 };
 
+// C(n, k), n < 256, k <= 16, saturated at UINT64_MAX (only spaces below 2^64 are ever indexed)
 static void host_binomials(u64 (*b)[BINOM_K]) {
   for (int n = 0; n < BINOM_N; ++n)
     for (int k = 0; k < BINOM_K; ++k) {
       if (k == 0) b[n][k] = 1;
       else if (n == 0) b[n][k] = 0;
-      else b[n][k] = b[n - 1][k - 1] + b[n - 1][k];
+      else {
+        const u64 x = b[n - 1][k - 1], y = b[n - 1][k];
+        b[n][k] = (x > U64MAX - y) ? U64MAX : x + y;
+      }
     }
 }
 
@@ -111,11 +115,11 @@ extern "C" int autopipe_create(int cuda_device, autopipe_ctx **out) {
   host_binomials(c->binom);
   upload_binomials(c->binom);
   // device tables, sized for the limits (L = 255, N = 8): a few hundred KB
-  const size_t Lp1 = MAXL + 1, NL = (size_t)MAXN * Lp1;
-  const size_t words = 3 * NL + Lp1 + 2 * MAXL + 64 + 2 * 7 * MAXL + 2;
+  const size_t Lp1 = MAXL + 1, NL = (size_t)MAXNW * Lp1, TT = (size_t)TAUW * TAUW;
+  const size_t words = 3 * NL + Lp1 + 2 * MAXL + TT + 2 * 7 * MAXL + 2;
   const size_t words32 = NL + 2 * 7 * MAXL;
   e = cudaMalloc(&c->d_tables, words * 8 + words32 * 4 + 64);
-  if (e == cudaSuccess) e = cudaMalloc(&c->d_raw, (2 * MAXN * MAXL + MAXL + 64) * 8);
+  if (e == cudaSuccess) e = cudaMalloc(&c->d_raw, (2 * MAXNW * MAXL + MAXL + TT) * 8);
   if (e == cudaSuccess) e = cudaMalloc(&c->d_blocks, sizeof(BlockOut) * MAX_BLOCKS);
   if (e == cudaSuccess) e = cudaMalloc(&c->d_result, sizeof(ResultDev));
   c->work_bytes = 1 << 20;
@@ -125,7 +129,7 @@ extern "C" int autopipe_create(int cuda_device, autopipe_ctx **out) {
   if (e == cudaSuccess) e = cudaMalloc(&c->d_ntimes, (size_t)NEIGH_ITEMS * NEIGH_MAXOPT * 8);
   if (e == cudaSuccess) e = cudaMalloc(&c->d_ncount, 8);
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_ncount, 8);
-  if (e == cudaSuccess) e = cudaMallocHost(&c->h_stage, (2 * MAXN * MAXL + 64) * 8);
+  if (e == cudaSuccess) e = cudaMallocHost(&c->h_stage, (2 * MAXNW * MAXL + TT) * 8);
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_result, sizeof(ResultDev));
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_status, 2 * sizeof(u64));
   if (e != cudaSuccess) {
@@ -140,7 +144,7 @@ extern "C" int autopipe_create(int cuda_device, autopipe_ctx **out) {
   c->tab.PP = p; p += Lp1;
   c->tab.O = p; p += MAXL;
   c->tab.G = p; p += MAXL;
-  c->tab.tau = p; p += 64;
+  c->tab.tau = p; p += TT;
   c->tab.Z = p; p += 7 * MAXL;
   c->tab.LM = p; p += 7 * MAXL;
   c->tab.status = p; p += 2;
@@ -203,7 +207,7 @@ extern "C" int autopipe_load_profile(autopipe_ctx *c, uint32_t L, const uint64_t
   // O, G go straight to their tables; P to the raw area (the state kernel builds its prefix)
   cudaError_t e = cudaMemcpy(c->tab.O, O, L * 8, cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemcpy(c->tab.G, G, L * 8, cudaMemcpyHostToDevice);
-  if (e == cudaSuccess) e = cudaMemcpy(c->d_raw + 2 * MAXN * MAXL, P, L * 8, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(c->d_raw + 2 * MAXNW * MAXL, P, L * 8, cudaMemcpyHostToDevice);
   if (e != cudaSuccess) return cuda_fail(c, e, "load_profile copy");
   c->L = L;
   c->maxOG = maxOG;
@@ -219,7 +223,7 @@ extern "C" int autopipe_set_state(autopipe_ctx *c, uint32_t N, const uint64_t *f
   if (!c) return AUTOPIPE_E_INVAL;
   c->err[0] = 0;
   if (!c->has_profile) return fail(c, AUTOPIPE_E_STATE, "set_state before load_profile");
-  if (N < 1 || N > MAXN) return fail(c, AUTOPIPE_E_INVAL, "N = %u outside [1, 8]", N);
+  if (N < 1 || N > MAXNW) return fail(c, AUTOPIPE_E_INVAL, "N = %u outside [1, 16]", N);
   if (!fp || !bp || !tau) return fail(c, AUTOPIPE_E_INVAL, "NULL state array");
   const u32 L = c->L;
   // overflow rules (SPEC.md §7)
@@ -241,9 +245,12 @@ extern "C" int autopipe_set_state(autopipe_ctx *c, uint32_t N, const uint64_t *f
     }
     sumMax += m;
   }
-  const u128 bound = sumMax + 16 + (u128)28 * maxX;
+  // up to 7 boundaries (N <= 8) or 15 (N <= 16, wide records): 4 transfer bounds per boundary, one
+  // rounding per stage (SPEC.md §7)
+  const bool wideN = N > (u32)MAXN;
+  const u128 bound = sumMax + (wideN ? 32 : 16) + (u128)(wideN ? 60 : 28) * maxX;
   if (bound >= LIMIT_TIME) return fail(c, AUTOPIPE_E_OVERFLOW, "modelled times reach 2^59 ns");
-  const u128 bound32 = sumMax + 16 + (u128)14 * maxXog;
+  const u128 bound32 = sumMax + (wideN ? 32 : 16) + (u128)(wideN ? 30 : 14) * maxXog;
   c->path32 = bound32 < LIMIT_TIME32 ? 1 : 0;
   c->bound = (u64)bound;
   DeviceGuard dg(c->device);
@@ -251,11 +258,11 @@ extern "C" int autopipe_set_state(autopipe_ctx *c, uint32_t N, const uint64_t *f
   // stage into pinned memory so the copies are truly asynchronous
   cudaError_t e = cudaStreamSynchronize(st);  // the staging buffer may still feed a previous copy
   if (e != cudaSuccess) return cuda_fail(c, e, "set_state sync");
-  u64 *hf = c->h_stage, *hb = hf + MAXN * MAXL, *ht = hb + MAXN * MAXL;
+  u64 *hf = c->h_stage, *hb = hf + MAXNW * MAXL, *ht = hb + MAXNW * MAXL;
   memcpy(hf, fp, (size_t)N * L * 8);
   memcpy(hb, bp, (size_t)N * L * 8);
   memcpy(ht, tau, (size_t)N * N * 8);
-  u64 *rf = c->d_raw, *rb = rf + MAXN * MAXL, *rP = rb + MAXN * MAXL, *rt = rP + MAXL;
+  u64 *rf = c->d_raw, *rb = rf + MAXNW * MAXL, *rP = rb + MAXNW * MAXL, *rt = rP + MAXL;
   e = cudaMemcpyAsync(rf, hf, (size_t)N * L * 8, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess) e = cudaMemcpyAsync(rb, hb, (size_t)N * L * 8, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess) e = cudaMemcpyAsync(rt, ht, (size_t)N * N * 8, cudaMemcpyHostToDevice, st);
@@ -277,7 +284,7 @@ extern "C" int autopipe_set_state_device(autopipe_ctx *c, uint32_t N, const uint
   if (!c) return AUTOPIPE_E_INVAL;
   c->err[0] = 0;
   if (!c->has_profile) return fail(c, AUTOPIPE_E_STATE, "set_state before load_profile");
-  if (N < 1 || N > MAXN) return fail(c, AUTOPIPE_E_INVAL, "N = %u outside [1, 8]", N);
+  if (N < 1 || N > MAXNW) return fail(c, AUTOPIPE_E_INVAL, "N = %u outside [1, 16]", N);
   if (!d_fp || !d_bp || !d_tau) return fail(c, AUTOPIPE_E_INVAL, "NULL state array");
   DeviceGuard dg(c->device);
   cudaStream_t st = (cudaStream_t)stream;
@@ -285,7 +292,7 @@ extern "C" int autopipe_set_state_device(autopipe_ctx *c, uint32_t N, const uint
   c->tab.N = N;
   c->tab.Lp1 = c->L + 1;
   c->N = N;
-  const u64 *rP = c->d_raw + 2 * MAXN * MAXL;
+  const u64 *rP = c->d_raw + 2 * MAXNW * MAXL;
   c->launches += launch_build_state(c->tab, (const u64 *)d_fp, (const u64 *)d_bp, rP, (const u64 *)d_tau, c->sumP, st);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "state kernel launch");
@@ -353,8 +360,8 @@ extern "C" int autopipe_get_schedule(const autopipe_ctx *c, uint32_t *schedule, 
   return AUTOPIPE_OK;
 }
 
-extern "C" int autopipe_eval_partitions(autopipe_ctx *c, const autopipe_partition *d_parts, uint64_t count,
-                                        uint64_t *d_time_ns, void *stream) {
+static int eval_impl(autopipe_ctx *c, const void *d_parts, uint64_t count, bool wide, uint64_t *d_time_ns,
+                     void *stream) {
   if (!c) return AUTOPIPE_E_INVAL;
   c->err[0] = 0;
   if (!c->has_state) return fail(c, AUTOPIPE_E_STATE, "eval before set_state");
@@ -365,11 +372,21 @@ extern "C" int autopipe_eval_partitions(autopipe_ctx *c, const autopipe_partitio
   if (rc) return rc;
   // a state given in device memory has not been classified on the host yet: use the 64-bit path
   const int p32 = c->state_on_device ? 0 : c->path32;
-  c->launches += launch_eval(c->tab, d_parts, count, (u64 *)d_time_ns, nullptr, nullptr, nullptr, nullptr, p32,
+  c->launches += launch_eval(c->tab, d_parts, count, wide, (u64 *)d_time_ns, nullptr, nullptr, nullptr, nullptr, p32,
                              c->model, c->sms, (cudaStream_t)stream);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "eval kernel launch");
   return AUTOPIPE_OK;
+}
+
+extern "C" int autopipe_eval_partitions(autopipe_ctx *c, const autopipe_partition *d_parts, uint64_t count,
+                                        uint64_t *d_time_ns, void *stream) {
+  return eval_impl(c, d_parts, count, false, d_time_ns, stream);
+}
+
+extern "C" int autopipe_eval_partitions_w(autopipe_ctx *c, const autopipe_partition_w *d_parts, uint64_t count,
+                                          uint64_t *d_time_ns, void *stream) {
+  return eval_impl(c, d_parts, count, true, d_time_ns, stream);
 }
 
 // --- search space arithmetic (SPEC.md §5) ----------------------------------------------------
@@ -385,6 +402,7 @@ static bool build_space(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, Search
     sp.off[S] = (u64)off;
     const u64 K = (flags & AUTOPIPE_USE_ALL_WORKERS) ? c->binom[c->N - 1][S - 1] : c->binom[c->N][S];
     const u64 nc = (S - 1 <= (int)c->L - 1) ? c->binom[c->L - 1][S - 1] : 0;
+    if (nc == U64MAX) return false;  // saturated binomial: the space exceeds 2^64
     sp.ncut[S] = nc;
     sp.ncomp[S] = K;
     off += (u128)K * nc;
@@ -394,11 +412,16 @@ static bool build_space(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, Search
   return true;
 }
 
-static int check_space_args(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags) {
+// wide: the space is read through 32-byte records (S <= 16, any N <= 16); otherwise 16-byte records
+// (S <= 8 and N <= 8: a contiguous placement may use any of the N workers).
+static int check_space_args(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, bool wide) {
   if (flags & ~AUTOPIPE_USE_ALL_WORKERS) return fail(c, AUTOPIPE_E_INVAL, "unknown flags 0x%x", flags);
-  const u32 smax_lim = c->N < (u32)MAXS ? c->N : (u32)MAXS;
+  if (!wide && c->N > (u32)MAXN)
+    return fail(c, AUTOPIPE_E_INVAL, "N = %u > 8 workers: 16-byte records cannot name them (use the _w calls)", c->N);
+  const u32 lim = wide ? (u32)MAXSW : (u32)MAXS;
+  const u32 smax_lim = c->N < lim ? c->N : lim;
   if (s_min < 1 || s_min > s_max || s_max > smax_lim)
-    return fail(c, AUTOPIPE_E_INVAL, "need 1 <= s_min <= s_max <= min(8, N) (got %u, %u, N = %u)", s_min,
+    return fail(c, AUTOPIPE_E_INVAL, "need 1 <= s_min <= s_max <= min(%u, N) (got %u, %u, N = %u)", lim, s_min,
                 s_max, c->N);
   return AUTOPIPE_OK;
 }
@@ -408,7 +431,7 @@ extern "C" int autopipe_count_candidates(const autopipe_ctx *cc, uint32_t s_min,
   autopipe_ctx *c = const_cast<autopipe_ctx *>(cc);
   if (!c || !total) return AUTOPIPE_E_INVAL;
   if (!c->has_state) return fail(c, AUTOPIPE_E_STATE, "count before set_state");
-  int rc = check_space_args(c, s_min, s_max, flags);
+  int rc = check_space_args(c, s_min, s_max, flags, true);
   if (rc) return rc;
   SearchSpace sp;
   if (!build_space(c, s_min, s_max, flags, sp)) return fail(c, AUTOPIPE_E_OVERFLOW, "space exceeds 2^64");
@@ -416,26 +439,22 @@ extern "C" int autopipe_count_candidates(const autopipe_ctx *cc, uint32_t s_min,
   return AUTOPIPE_OK;
 }
 
-static u64 host_unrank(const autopipe_ctx *c, u64 rank, int k, int n) {
-  u64 out = 0;
+// sorted k-subset (k <= 16) of {0..n-1} of a given lex rank, one element per entry
+static void host_unrank(const autopipe_ctx *c, u64 rank, int k, int n, int *out) {
   int x = 0;
   for (int i = 0; i < k; ++i) {
     while (c->binom[n - 1 - x][k - 1 - i] <= rank) {
       rank -= c->binom[n - 1 - x][k - 1 - i];
       ++x;
     }
-    out |= (u64)x << (8 * i);
-    ++x;
+    out[i] = x++;
   }
-  return out;
 }
 
-extern "C" int autopipe_decode_index(const autopipe_ctx *cc, uint32_t s_min, uint32_t s_max, uint32_t flags,
-                                     uint64_t index, autopipe_partition *out) {
-  autopipe_ctx *c = const_cast<autopipe_ctx *>(cc);
-  if (!c || !out) return AUTOPIPE_E_INVAL;
+// Global index -> record bytes (16 or 32 as wide): S, the cuts, the stage of every worker.
+static int decode_impl(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, u64 index, bool wide, uint8_t *rec) {
   if (!c->has_state) return fail(c, AUTOPIPE_E_STATE, "decode before set_state");
-  int rc = check_space_args(c, s_min, s_max, flags);
+  int rc = check_space_args(c, s_min, s_max, flags, wide);
   if (rc) return rc;
   SearchSpace sp;
   if (!build_space(c, s_min, s_max, flags, sp)) return fail(c, AUTOPIPE_E_OVERFLOW, "space exceeds 2^64");
@@ -445,36 +464,55 @@ extern "C" int autopipe_decode_index(const autopipe_ctx *cc, uint32_t s_min, uin
   const u64 rem = index - sp.off[S];
   const u64 rho = rem / sp.ncut[S], kappa = rem % sp.ncut[S];
   const bool all = flags & AUTOPIPE_USE_ALL_WORKERS;
-  const u64 Rp = all ? host_unrank(c, rho, S - 1, (int)c->N - 1) : host_unrank(c, rho, S, (int)c->N);
-  const u64 cuts = host_unrank(c, kappa, S - 1, (int)c->L - 1);
-  memset(out, 0xFF, sizeof(*out));
-  out->n_stages = (uint8_t)S;
-  for (int s = 0; s < S - 1; ++s) out->last_layer[s] = (uint8_t)((cuts >> (8 * s)) & 0xFF);
+  int Rp[MAXSW], cuts[MAXSW];
+  if (all) host_unrank(c, rho, S - 1, (int)c->N - 1, Rp);
+  else host_unrank(c, rho, S, (int)c->N, Rp);
+  host_unrank(c, kappa, S - 1, (int)c->L - 1, cuts);
+  const int n = wide ? 32 : 16, off = wide ? 16 : 8;
+  memset(rec, 0xFF, n);
+  rec[0] = (uint8_t)S;
+  for (int s = 0; s < S - 1; ++s) rec[1 + s] = (uint8_t)cuts[s];
   int prev = 0;
   for (int s = 0; s < S; ++s) {
-    const int R = (all && s == S - 1) ? (int)c->N : (int)((Rp >> (8 * s)) & 0xFF) + 1;
-    for (int w = prev; w < R; ++w) out->stage_of_worker[w] = (uint8_t)s;
+    const int R = (all && s == S - 1) ? (int)c->N : Rp[s] + 1;
+    for (int w = prev; w < R; ++w) rec[off + w] = (uint8_t)s;
     prev = R;
   }
   return AUTOPIPE_OK;
 }
 
-extern "C" int autopipe_search_optimum(autopipe_ctx *c, uint32_t s_min, uint32_t s_max, uint32_t flags,
-                                       uint64_t begin, uint64_t end, autopipe_result *h_out, void *stream) {
+extern "C" int autopipe_decode_index(const autopipe_ctx *cc, uint32_t s_min, uint32_t s_max, uint32_t flags,
+                                     uint64_t index, autopipe_partition *out) {
+  autopipe_ctx *c = const_cast<autopipe_ctx *>(cc);
+  if (!c || !out) return AUTOPIPE_E_INVAL;
+  return decode_impl(c, s_min, s_max, flags, index, false, (uint8_t *)out);
+}
+
+extern "C" int autopipe_decode_index_w(const autopipe_ctx *cc, uint32_t s_min, uint32_t s_max, uint32_t flags,
+                                       uint64_t index, autopipe_partition_w *out) {
+  autopipe_ctx *c = const_cast<autopipe_ctx *>(cc);
+  if (!c || !out) return AUTOPIPE_E_INVAL;
+  return decode_impl(c, s_min, s_max, flags, index, true, (uint8_t *)out);
+}
+
+// The search of a 16-byte space (wide = false) or a wide one (row f4). Writes time, index, evaluated
+// and the best record (16 or 32 bytes) to the host.
+static int search_impl(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, u64 begin, u64 end, bool wide,
+                       u64 *h_tie, uint8_t *h_rec, void *stream) {
   if (!c) return AUTOPIPE_E_INVAL;
   c->err[0] = 0;
   if (!c->has_state) return fail(c, AUTOPIPE_E_STATE, "search before set_state");
-  if (!h_out) return fail(c, AUTOPIPE_E_INVAL, "NULL result pointer");
-  int rc = check_space_args(c, s_min, s_max, flags);
+  if (!h_tie || !h_rec) return fail(c, AUTOPIPE_E_INVAL, "NULL result pointer");
+  int rc = check_space_args(c, s_min, s_max, flags, wide);
   if (rc) return rc;
   SearchSpace sp;
   if (!build_space(c, s_min, s_max, flags, sp)) return fail(c, AUTOPIPE_E_OVERFLOW, "space exceeds 2^64");
   const u64 total = sp.off[s_max + 1];
   if (end > total) end = total;
-  memset(h_out, 0, sizeof(*h_out));
-  h_out->time_ns = U64MAX;
-  h_out->index = U64MAX;
-  memset(&h_out->part, 0xFF, sizeof(h_out->part));
+  h_tie[0] = U64MAX;
+  h_tie[1] = U64MAX;
+  h_tie[2] = 0;
+  memset(h_rec, 0xFF, wide ? 32 : 16);
   if (begin >= end) return AUTOPIPE_OK;
   DeviceGuard dg(c->device);
   cudaStream_t st = (cudaStream_t)stream;
@@ -493,7 +531,7 @@ extern "C" int autopipe_search_optimum(autopipe_ctx *c, uint32_t s_min, uint32_t
     // candidates with rho = 0 are [blo, blo + ncut); rho = 0 is all-r=1 iff the first composition
     // (R = 1..S) has every r_s = 1, which holds for the default flag and for USE_ALL when N = S.
     // The fast kernel decides the PipeDream closed form; other schedules (row f3) go to the generic one.
-    const bool r1 = S >= 5 && (!(flags & AUTOPIPE_USE_ALL_WORKERS) || (int)c->N == S) &&
+    const bool r1 = S >= 5 && S <= MAXS && (!(flags & AUTOPIPE_USE_ALL_WORKERS) || (int)c->N == S) &&
                     c->model.sched == SCHED_PIPEDREAM;
     const u64 r1hi = blo + sp.ncut[S];
     if (r1 && lo < r1hi) {
@@ -503,19 +541,19 @@ extern "C" int autopipe_search_optimum(autopipe_ctx *c, uint32_t s_min, uint32_t
                                       MAX_BLOCKS - used, &nb, c->d_work, c->h_work, c->work_bytes, st);
       used += nb;
       if (b < hi) {
-        c->launches += launch_search_generic(c->tab, sp, b, hi, c->path32, c->model, c->sms, c->d_blocks + used, MAX_BLOCKS - used,
+        c->launches += launch_search_generic(c->tab, sp, b, hi, c->path32, c->model, wide, c->sms, c->d_blocks + used, MAX_BLOCKS - used,
                                              &nb, st);
         used += nb;
       }
     } else {
       int nb = 0;
-      c->launches += launch_search_generic(c->tab, sp, lo, hi, c->path32, c->model, c->sms, c->d_blocks + used, MAX_BLOCKS - used,
+      c->launches += launch_search_generic(c->tab, sp, lo, hi, c->path32, c->model, wide, c->sms, c->d_blocks + used, MAX_BLOCKS - used,
                                            &nb, st);
       used += nb;
     }
     cur = hi;
     if (used > MAX_BLOCKS - 4 * c->sms) {  // keep room: fold what we have into one entry
-      c->launches += launch_finalize(c->d_blocks, used, sp, c->d_result, st);
+      c->launches += launch_finalize(c->d_blocks, used, sp, c->d_result, wide, st);
       cudaMemcpyAsync(c->d_blocks, c->d_result, sizeof(BlockOut), cudaMemcpyDeviceToDevice, st);
       used = 1;
     }
@@ -530,7 +568,7 @@ extern "C" int autopipe_search_optimum(autopipe_ctx *c, uint32_t s_min, uint32_t
     fprintf(stderr, "[autopipe] blocks %d candidates %llu rare %llu\n", used, cnt, rare);
     delete[] hb;
   }
-  c->launches += launch_finalize(c->d_blocks, used, sp, c->d_result, st);
+  c->launches += launch_finalize(c->d_blocks, used, sp, c->d_result, wide, st);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "search kernel launch");
   e = cudaMemcpyAsync(c->h_result, c->d_result, sizeof(ResultDev), cudaMemcpyDeviceToHost, st);
@@ -541,48 +579,85 @@ extern "C" int autopipe_search_optimum(autopipe_ctx *c, uint32_t s_min, uint32_t
     cudaEventElapsedTime(&ms, c->ev0, c->ev1);
     c->last_search_ms = ms;
   }
-  h_out->time_ns = c->h_result->time_ns;
-  h_out->index = c->h_result->index;
-  h_out->evaluated = c->h_result->evaluated;
-  memcpy(&h_out->part, c->h_result->part, 16);
+  h_tie[0] = c->h_result->time_ns;
+  h_tie[1] = c->h_result->index;
+  h_tie[2] = c->h_result->evaluated;
+  memcpy(h_rec, c->h_result->part, wide ? 32 : 16);
   return AUTOPIPE_OK;
 }
 
-// host-side validation of the current partition of a rollout (same rules as SPEC.md §2)
-static bool host_decode(const autopipe_partition *p, u32 L, u32 N, int &S, u64 &cuts, u64 &masks) {
-  S = p->n_stages;
-  if (S < 1 || S > MAXS || S > (int)N) return false;
-  cuts = 0;
+extern "C" int autopipe_search_optimum(autopipe_ctx *c, uint32_t s_min, uint32_t s_max, uint32_t flags,
+                                       uint64_t begin, uint64_t end, autopipe_result *h_out, void *stream) {
+  if (!c) return AUTOPIPE_E_INVAL;
+  if (!h_out) return fail(c, AUTOPIPE_E_INVAL, "NULL result pointer");
+  u64 tie[3];
+  const int rc = search_impl(c, s_min, s_max, flags, begin, end, false, tie, (uint8_t *)&h_out->part, stream);
+  h_out->time_ns = tie[0];
+  h_out->index = tie[1];
+  h_out->evaluated = tie[2];
+  return rc;
+}
+
+extern "C" int autopipe_search_optimum_w(autopipe_ctx *c, uint32_t s_min, uint32_t s_max, uint32_t flags,
+                                         uint64_t begin, uint64_t end, autopipe_result_w *h_out, void *stream) {
+  if (!c) return AUTOPIPE_E_INVAL;
+  if (!h_out) return fail(c, AUTOPIPE_E_INVAL, "NULL result pointer");
+  u64 tie[3];
+  const int rc = search_impl(c, s_min, s_max, flags, begin, end, true, tie, (uint8_t *)&h_out->part, stream);
+  h_out->time_ns = tie[0];
+  h_out->index = tie[1];
+  h_out->evaluated = tie[2];
+  return rc;
+}
+
+// host-side validation of a current partition (same rules as SPEC.md §2), 16-byte (MS = 8) or wide
+// (MS = 16) record bytes; its packed parts as the kernels read them (P8: cuts[0], masks[0]; P16:
+// cut bytes in cuts[0..1], 16-bit stage masks in masks[0..3]).
+static bool host_decode_rec(const uint8_t *rec, bool wide, u32 L, u32 N, int &S, u64 *cuts, u64 *masks) {
+  const int MS = wide ? MAXSW : MAXS, off = wide ? 16 : 8, mb = wide ? 16 : 8;
+  S = rec[0];
+  if (S < 1 || S > MS || S > (int)N) return false;
+  cuts[0] = cuts[1] = 0;
+  for (int i = 0; i < 4; ++i) masks[i] = 0;
   int prev = -1;
   for (int i = 0; i < S - 1; ++i) {
-    const int e = p->last_layer[i];
+    const int e = rec[1 + i];
     if (e <= prev || e >= (int)L - 1) return false;
     prev = e;
-    cuts |= (u64)e << (8 * i);
+    cuts[i >> 3] |= (u64)e << (8 * (i & 7));
   }
-  masks = 0;
-  for (int w = 0; w < MAXN; ++w) {
-    const int s = p->stage_of_worker[w];
+  u32 sm[MAXSW] = {0};
+  for (int w = 0; w < MS; ++w) {
+    const int s = rec[off + w];
     if (s == 0xFF) continue;
     if (w >= (int)N || s >= S) return false;
-    masks |= 1ull << (8 * s + w);
+    sm[s] |= 1u << w;
   }
-  for (int s = 0; s < S; ++s)
-    if (((masks >> (8 * s)) & 0xFF) == 0) return false;
+  for (int s = 0; s < S; ++s) {
+    if (sm[s] == 0) return false;
+    if (wide) masks[s >> 2] |= (u64)sm[s] << (16 * (s & 3));
+    else masks[0] |= (u64)sm[s] << (mb * s);
+  }
+  return true;
+}
+static bool host_decode(const autopipe_partition *p, u32 L, u32 N, int &S, u64 &cuts, u64 &masks) {
+  u64 c2[2], m4[4];
+  if (!host_decode_rec((const uint8_t *)p, false, L, N, S, c2, m4)) return false;
+  cuts = c2[0];
+  masks = m4[0];
   return true;
 }
 
-extern "C" int autopipe_rollout_rewards(autopipe_ctx *c, const autopipe_partition *d_parts, uint64_t count,
-                                        const autopipe_partition *h_current, uint64_t *d_time_ns,
-                                        uint64_t *d_switch_bytes, void *stream) {
+static int rollout_impl(autopipe_ctx *c, const void *d_parts, uint64_t count, const uint8_t *h_current, bool wide,
+                        uint64_t *d_time_ns, uint64_t *d_switch_bytes, void *stream) {
   if (!c) return AUTOPIPE_E_INVAL;
   c->err[0] = 0;
   if (!c->has_state) return fail(c, AUTOPIPE_E_STATE, "rollout before set_state");
   if ((h_current == nullptr) != (d_switch_bytes == nullptr))
     return fail(c, AUTOPIPE_E_INVAL, "h_current and d_switch_bytes must both be set or both be NULL");
   int S = 0;
-  u64 cuts = 0, masks = 0;
-  if (h_current && !host_decode(h_current, c->L, c->N, S, cuts, masks))
+  u64 cuts[2], masks[4];
+  if (h_current && !host_decode_rec(h_current, wide, c->L, c->N, S, cuts, masks))
     return fail(c, AUTOPIPE_E_INVAL, "invalid current partition");
   if (count == 0) return AUTOPIPE_OK;
   if (!d_parts || !d_time_ns) return fail(c, AUTOPIPE_E_INVAL, "NULL device pointer");
@@ -590,11 +665,23 @@ extern "C" int autopipe_rollout_rewards(autopipe_ctx *c, const autopipe_partitio
   int rc = check_model(c, (cudaStream_t)stream);
   if (rc) return rc;
   const int p32 = c->state_on_device ? 0 : c->path32;
-  c->launches += launch_eval(c->tab, d_parts, count, (u64 *)d_time_ns, (u64 *)d_switch_bytes, h_current ? &S : nullptr,
-                             &cuts, &masks, p32, c->model, c->sms, (cudaStream_t)stream);
+  c->launches += launch_eval(c->tab, d_parts, count, wide, (u64 *)d_time_ns, (u64 *)d_switch_bytes,
+                             h_current ? &S : nullptr, cuts, masks, p32, c->model, c->sms, (cudaStream_t)stream);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "rollout kernel launch");
   return AUTOPIPE_OK;
+}
+
+extern "C" int autopipe_rollout_rewards(autopipe_ctx *c, const autopipe_partition *d_parts, uint64_t count,
+                                        const autopipe_partition *h_current, uint64_t *d_time_ns,
+                                        uint64_t *d_switch_bytes, void *stream) {
+  return rollout_impl(c, d_parts, count, (const uint8_t *)h_current, false, d_time_ns, d_switch_bytes, stream);
+}
+
+extern "C" int autopipe_rollout_rewards_w(autopipe_ctx *c, const autopipe_partition_w *d_parts, uint64_t count,
+                                          const autopipe_partition_w *h_current, uint64_t *d_time_ns,
+                                          uint64_t *d_switch_bytes, void *stream) {
+  return rollout_impl(c, d_parts, count, (const uint8_t *)h_current, true, d_time_ns, d_switch_bytes, stream);
 }
 
 extern "C" int autopipe_int_path(const autopipe_ctx *cc) {
@@ -626,6 +713,7 @@ extern "C" double autopipe_last_search_ms(const autopipe_ctx *c) { return c ? c-
 static int neigh_prepare(autopipe_ctx *c, const autopipe_partition *h_current, u64 &nslots, cudaStream_t st) {
   if (!c->has_state) return fail(c, AUTOPIPE_E_STATE, "neighbourhood before set_state");
   if (!h_current) return fail(c, AUTOPIPE_E_INVAL, "NULL current partition");
+  if (c->N > (u32)MAXN) return fail(c, AUTOPIPE_E_INVAL, "the neighbourhood uses 16-byte records: N <= 8");
   int S = 0;
   u64 cuts = 0, masks = 0;
   if (!host_decode(h_current, c->L, c->N, S, cuts, masks))
@@ -669,8 +757,8 @@ extern "C" int autopipe_neighbourhood_best(autopipe_ctx *c, const autopipe_parti
   u64 nslots = 0;
   rc = neigh_prepare(c, h_current, nslots, st);
   if (rc) return rc;
-  c->launches += launch_eval(c->tab, c->d_nslots, nslots, c->d_ntimes, nullptr, nullptr, nullptr, nullptr, c->path32,
-                             c->model, c->sms, st);
+  c->launches += launch_eval(c->tab, c->d_nslots, nslots, false, c->d_ntimes, nullptr, nullptr, nullptr, nullptr,
+                             c->path32, c->model, c->sms, st);
   c->launches += launch_neigh_best(c->d_nslots, c->d_ntimes, nslots, c->d_result, st);
   cudaError_t e = cudaMemcpyAsync(c->h_result, c->d_result, sizeof(ResultDev), cudaMemcpyDeviceToHost, st);
   if (e == cudaSuccess) e = cudaStreamSynchronize(st);
@@ -694,6 +782,7 @@ extern "C" int autopipe_switch_rewards(autopipe_ctx *c, const autopipe_partition
   if (!c->has_state) return fail(c, AUTOPIPE_E_STATE, "switch rewards before set_state");
   if (!h_current) return fail(c, AUTOPIPE_E_INVAL, "NULL current partition");
   if (horizon == 0) return fail(c, AUTOPIPE_E_INVAL, "horizon must be >= 1");
+  if (c->N > (u32)MAXN) return fail(c, AUTOPIPE_E_INVAL, "switch rewards use 16-byte records: N <= 8");
   if (c->model.sched != SCHED_PIPEDREAM)
     return fail(c, AUTOPIPE_E_STATE, "switch rewards are defined for the PipeDream schedule (reading F-2)");
   int S = 0;

@@ -5,7 +5,8 @@
 
 namespace ap {
 
-// Binomial coefficients C(n, k), n < 256, k <= 8, uploaded once per context by autopipe_create.
+// Binomial coefficients C(n, k), n < 256, k <= 16 (saturated at UINT64_MAX: a space whose size
+// fits 64 bits only ever reads entries below its size), uploaded once per context by autopipe_create.
 __constant__ u64 c_binom[BINOM_N][BINOM_K];
 
 void upload_binomials(const u64 (*tab)[BINOM_K]) {
@@ -58,18 +59,37 @@ __device__ __forceinline__ bool lex_next_packed(u64 &packed, int k, int n) {
 // kernel unranks once per lane and task, so it avoids the serialised divergent reads of __constant__.
 // Unranking uses the colex dual: r' = C(n,k) - 1 - r = sum_i C(d_i, k-i), d_i = n-1-c_i, each d_i
 // found by a fixed-length binary search (no data-dependent trip count, no divergence).
+// B: rows n of C(n, 0..BK-1) (BK = BK8 = 9 for 16-byte spaces, BINOM_K = 17 for wide ones).
+template <int BK = BK8>
 __device__ __forceinline__ u64 lex_rank_smem(u64 packed, int k, int n, const u64 *B) {
   u64 s = 0;
   for (int i = 0; i < k; ++i) {
     const int c = (int)((packed >> (8 * i)) & 0xFF);
-    s += B[(n - 1 - c) * BINOM_K + (k - i)];
+    s += B[(n - 1 - c) * BK + (k - i)];
   }
-  return B[n * BINOM_K + k] - 1 - s;
+  return B[n * BK + k] - 1 - s;
 }
 
-__device__ __forceinline__ u64 lex_unrank_smem(u64 rank, int k, int n, const u64 *B) {
-  u64 rp = B[n * BINOM_K + k] - 1 - rank;
-  u64 out = 0;
+// Byte i of a packed subset: one u64 (k <= 8) or a pair (k <= 16, wide spaces of row f4).
+struct Pk2 {
+  u64 lo, hi;
+};
+__device__ __forceinline__ int pk_get(u64 v, int i) { return byte_at(v, i); }
+__device__ __forceinline__ int pk_get(const Pk2 &v, int i) { return byte_at(i < 8 ? v.lo : v.hi, i & 7); }
+__device__ __forceinline__ void pk_or(u64 &v, int i, int x) { v |= (u64)x << (8 * i); }
+__device__ __forceinline__ void pk_or(Pk2 &v, int i, int x) {
+  const u64 b = (u64)x << (8 * (i & 7));
+  if (i < 8) v.lo |= b;
+  else v.hi |= b;
+}
+__device__ __forceinline__ void pk_zero(u64 &v) { v = 0; }
+__device__ __forceinline__ void pk_zero(Pk2 &v) { v.lo = v.hi = 0; }
+
+template <int BK = BK8, typename PK = u64>
+__device__ __forceinline__ PK lex_unrank_smem(u64 rank, int k, int n, const u64 *B) {
+  u64 rp = B[n * BK + k] - 1 - rank;
+  PK out;
+  pk_zero(out);
   int hi = n - 1;  // d_i < d_{i-1}
   for (int i = 0; i < k; ++i) {
     const int m = k - i;
@@ -77,14 +97,31 @@ __device__ __forceinline__ u64 lex_unrank_smem(u64 rank, int k, int n, const u64
     int lo = 0, h = hi;
     while (lo < h) {
       const int mid = (lo + h + 1) >> 1;
-      if (B[mid * BINOM_K + m] <= rp) lo = mid;
+      if (B[mid * BK + m] <= rp) lo = mid;
       else h = mid - 1;
     }
-    rp -= B[lo * BINOM_K + m];
-    out |= (u64)(n - 1 - lo) << (8 * i);
+    rp -= B[lo * BK + m];
+    pk_or(out, i, n - 1 - lo);
     hi = lo - 1;
   }
   return out;
+}
+
+// Lexicographic successor of a packed sorted k-subset (k <= 16) of {0..n-1}; false when it was the last.
+__device__ __forceinline__ bool lex_next_pk2(Pk2 &p, int k, int n) {
+  for (int i = k - 1; i >= 0; --i) {
+    const int c = pk_get(p, i);
+    if (c < n - k + i) {
+      Pk2 q;
+      // keep bytes 0..i-1, then c+1, c+2, ...
+      q.lo = (i >= 8) ? p.lo : (i == 0 ? 0ull : (p.lo & ((1ull << (8 * i)) - 1)));
+      q.hi = (i > 8) ? (p.hi & ((1ull << (8 * (i - 8))) - 1)) : 0ull;
+      for (int j = i; j < k; ++j) pk_or(q, j, c + 1 + (j - i));
+      p = q;
+      return true;
+    }
+  }
+  return false;
 }
 
 }  // namespace ap

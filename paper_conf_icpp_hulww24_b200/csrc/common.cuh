@@ -12,11 +12,15 @@ namespace ap {
 typedef unsigned long long u64;
 typedef unsigned int u32;
 
-constexpr int MAXS = 8;       // stages (C-15)
-constexpr int MAXN = 8;       // workers
+constexpr int MAXS = 8;       // stages of a 16-byte record (C-15)
+constexpr int MAXN = 8;       // workers of a 16-byte record
+constexpr int MAXSW = 16;     // stages of a 32-byte wide record (row f4)
+constexpr int MAXNW = 16;     // workers of a state and of a wide record (row f4)
+constexpr int TAUW = 16;      // row stride of the padded tau table
 constexpr int MAXL = 255;     // layers
 constexpr int BINOM_N = 256;  // C(n, k) for n < 256
-constexpr int BINOM_K = 9;    // k <= 8
+constexpr int BINOM_K = 17;   // k <= 16 (wide spaces, row f4; saturated at UINT64_MAX)
+constexpr int BK8 = 9;        // columns k <= 8 staged in shared memory for 16-byte spaces
 constexpr u64 U64MAX = ~0ull;
 
 // Global-memory tables written by the state kernels (k_state.cu) and read by every scoring kernel.
@@ -29,7 +33,7 @@ struct DevTables {
   u64 *PP;    // [L+1]     exclusive prefix of weight bytes              (row a1)
   u64 *O;     // [L]       activation bytes
   u64 *G;     // [L]       input-gradient bytes
-  u64 *tau;   // [8][8]    fs per byte, row u -> column v (padded to 8x8)
+  u64 *tau;   // [16][16]  fs per byte, row u -> column v (padded to 16 x 16)
   u64 *Z;     // [7][L]    r = 1 boundary s (worker s -> s+1) cut after layer l: cf + cb   (row a2)
   u64 *LM;    // [7][L]    ... max(cf, cb)                                                (row a2)
   u32 *PC32;  // [N][L+1]  32-bit copies for the 32-bit search path (valid iff path32)
@@ -57,39 +61,45 @@ __device__ __forceinline__ u64 xfer(u64 bytes, u64 fs_per_byte) {
   return xfer_fs(bytes * fs_per_byte);  // the product is < 2^64 (set_state check)
 }
 
-// floor(x / d) for a runtime divisor d in [1, 8] and x < 2^63 (Granlund-Montgomery with N = 63:
-// m = ceil(2^(63+l)/d), l = ceil(log2 d); exact for every x < 2^63).
-__device__ __forceinline__ u64 div_small(u64 x, u32 d) {
-  // branch-free selection of the multiplier and post-shift; d = 1 is the identity
-  const u64 m = (d == 3u || d == 6u) ? 0xaaaaaaaaaaaaaaabull
-              : (d == 5u)            ? 0xcccccccccccccccdull
-              : (d == 7u)            ? 0x924924924924924aull
-                                     : 0x8000000000000000ull;
-  const u32 sh = (d <= 2u) ? 0u : (d <= 4u) ? 1u : 2u;
-  const u64 q = __umul64hi(x, m) >> sh;
-  return d == 1u ? x : q;
-}
-__device__ __forceinline__ u64 ceil_small(u64 x, u32 d) { return div_small(x + d - 1, d); }
-
-// The same division with the multiplier chosen once per divisor (hoisted out of loops over replicas
-// and shards). d in [1, 8]; x < 2^63.
-struct Div8 {
+// floor(x / d) for a runtime divisor d in [1, MAXD] (a replica count; MAXD = 8 for the 16-byte
+// records, 16 for the wide ones) and x < 2^63, by Granlund-Montgomery with N = 63:
+// m = ceil(2^(63+l) / d), l = ceil(log2 d), q = mulhi(x, m) >> (l - 1); exact for every x < 2^63
+// (d = 1 is the identity). The multiplier is chosen once per divisor, hoisted out of the loops over
+// replicas and shards.
+template <int MAXD = 8>
+struct DivR {
   u64 m;
   u32 sh, d, Ms;
-  __device__ __forceinline__ explicit Div8(u32 d_) : d(d_) {
-    m = (d == 3u || d == 6u) ? 0xaaaaaaaaaaaaaaabull
-      : (d == 5u)            ? 0xcccccccccccccccdull
-      : (d == 7u)            ? 0x924924924924924aull
-                             : 0x8000000000000000ull;
-    sh = (d <= 2u) ? 0u : (d <= 4u) ? 1u : 2u;
-    // floor(k / d) for 0 <= k < 64: (k * ceil(2^16 / d)) >> 16 is exact on that range
+  __device__ __forceinline__ explicit DivR(u32 d_) : d(d_) {
+    if (MAXD <= 8) {
+      m = (d == 3u || d == 6u) ? 0xaaaaaaaaaaaaaaabull
+        : (d == 5u)            ? 0xcccccccccccccccdull
+        : (d == 7u)            ? 0x924924924924924aull
+                               : 0x8000000000000000ull;
+      sh = (d <= 2u) ? 0u : (d <= 4u) ? 1u : 2u;
+    } else {
+      m = (d == 3u || d == 6u || d == 12u) ? 0xaaaaaaaaaaaaaaabull
+        : (d == 5u || d == 10u)            ? 0xcccccccccccccccdull
+        : (d == 7u || d == 14u)            ? 0x924924924924924aull
+        : (d == 9u)                        ? 0xe38e38e38e38e38full
+        : (d == 11u)                       ? 0xba2e8ba2e8ba2e8cull
+        : (d == 13u)                       ? 0x9d89d89d89d89d8aull
+        : (d == 15u)                       ? 0x8888888888888889ull
+                                           : 0x8000000000000000ull;
+      sh = (d <= 2u) ? 0u : (d <= 4u) ? 1u : (d <= 8u) ? 2u : 3u;
+    }
+    // floor(k / d) for 0 <= k < 256: (k * ceil(2^16 / d)) >> 16 is exact on that range
     Ms = (d == 1u) ? 65536u : (d == 2u) ? 32768u : (d == 3u) ? 21846u : (d == 4u) ? 16384u
        : (d == 5u) ? 13108u : (d == 6u) ? 10923u : (d == 7u) ? 9363u : 8192u;
+    if (MAXD > 8 && d > 8u)
+      Ms = (d == 9u) ? 7282u : (d == 10u) ? 6554u : (d == 11u) ? 5958u : (d == 12u) ? 5462u
+         : (d == 13u) ? 5042u : (d == 14u) ? 4682u : (d == 15u) ? 4370u : 4096u;
   }
   __device__ __forceinline__ u64 div(u64 x) const { return d == 1u ? x : (__umul64hi(x, m) >> sh); }
   __device__ __forceinline__ u64 ceil(u64 x) const { return div(x + d - 1); }
   __device__ __forceinline__ u32 small(u32 k) const { return (k * Ms) >> 16; }
 };
+typedef DivR<8> Div8;
 
 __device__ __forceinline__ int byte_at(u64 v, int i) { return (int)((v >> (8 * i)) & 0xFF); }
 

@@ -6,9 +6,10 @@
 // (PAPER.md:253-278, 463-475, 521-580); tests check the equality against the oracle's event
 // simulation bit for bit.
 //
-// A partition is (S, cuts, masks): cuts packed one byte per cut (byte s = e_s, s < S-1), masks
-// packed one byte per stage (byte s = bitmask of the workers of stage s). All loops over stages are
-// fully unrolled so every per-stage value lives in registers.
+// A partition is S plus a part type P giving cut e_i (i < S-1) and the worker bitmask of stage s:
+// P8 for the 16-byte record (S, N <= 8: cuts and masks one byte each, packed in a u64) and P16 for
+// the 32-byte wide record of NEXT row f4 (S, N <= 16: 15 cut bytes, 16-bit masks). All loops over
+// stages are fully unrolled to P::MS so every per-stage value lives in registers.
 #pragma once
 #include <type_traits>
 
@@ -16,15 +17,33 @@
 
 namespace ap {
 
+struct P8 {  // 16-byte records: byte i of cuts = e_i, byte s of masks = workers of stage s
+  static constexpr int MS = 8, MN = 8;
+  u64 cuts, masks;
+  __device__ __forceinline__ int cut(int i) const { return byte_at(cuts, i); }
+  __device__ __forceinline__ u32 mask(int s) const { return (u32)byte_at(masks, s); }
+};
+struct P16 {  // 32-byte wide records (row f4): cut bytes in c[0..1], 16-bit stage masks in m[0..3]
+  static constexpr int MS = 16, MN = 16;
+  u64 c[2], m[4];
+  // selects, not array indexing: a runtime index must not push the part into local memory
+  __device__ __forceinline__ int cut(int i) const { return (int)(((i < 8 ? c[0] : c[1]) >> (8 * (i & 7))) & 0xFF); }
+  __device__ __forceinline__ u32 mask(int s) const {
+    const int q = s >> 2;
+    const u64 v = q == 0 ? m[0] : q == 1 ? m[1] : q == 2 ? m[2] : m[3];
+    return (u32)((v >> (16 * (s & 3))) & 0xFFFF);
+  }
+};
+
 // Read-only view of the state tables staged in shared memory.
 struct SmemTab {
   const u64 *PF, *PB, *PP, *O, *G, *tau;
   int L, Lp1;
 };
 
-// Number of u64 words the staged tables need: PF, PB (N x (L+1)), PP (L+1), O, G (L), tau (64).
+// Number of u64 words the staged tables need: PF, PB (N x (L+1)), PP (L+1), O, G (L), tau (16 x 16).
 __host__ __device__ __forceinline__ u32 smem_words(u32 L, u32 N) {
-  return 2u * N * (L + 1) + (L + 1) + 2u * L + 64u;
+  return 2u * N * (L + 1) + (L + 1) + 2u * L + (u32)(TAUW * TAUW);
 }
 
 // Cooperative copy of the global tables into shared memory (every thread of the block calls it).
@@ -40,7 +59,7 @@ __device__ __forceinline__ SmemTab stage_tables(const DevTables &g, u64 *sm) {
     O[i] = g.O[i];
     G[i] = g.G[i];
   }
-  for (u32 i = threadIdx.x; i < 64; i += blockDim.x) tau[i] = g.tau[i];
+  for (u32 i = threadIdx.x; i < (u32)(TAUW * TAUW); i += blockDim.x) tau[i] = g.tau[i];
   __syncthreads();
   SmemTab t;
   t.PF = PF; t.PB = PB; t.PP = PP; t.O = O; t.G = G; t.tau = tau;
@@ -52,15 +71,16 @@ __device__ __forceinline__ SmemTab stage_tables(const DevTables &g, u64 *sm) {
 // ([floor(iA/r), floor((i+1)A/r))); every overlapping (sender, receiver) pair is one transfer on its
 // directed link, lasting ceil(overlap * tau / 1e6). A merge walk visits the <= r_s + r_r - 1
 // overlapping pairs in order; since the duration is monotone in overlap * tau, the walk keeps the
-// largest product and rounds once.
+// largest product and rounds once. MAXD = the largest replica count (8 or 16).
+template <int MAXD = 8>
 __device__ __forceinline__ u64 boundary_max(u64 A, u32 send, u32 recv, const u64 *tau) {
   const u32 rs = __popc(send), rr = __popc(recv);
   if (rs == 1 && rr == 1) {
     const int u = __ffs(send) - 1, v = __ffs(recv) - 1;
-    return xfer(A, tau[u * 8 + v]);
+    return xfer(A, tau[u * TAUW + v]);
   }
-  // shard boundaries floor(i A / r) = i q + floor(i rem / r) with A = q r + rem (rem < r <= 8, i <= 8)
-  const Div8 ds(rs), dr(rr);
+  // shard boundaries floor(i A / r) = i q + floor(i rem / r) with A = q r + rem (rem < r <= 16, i <= 16)
+  const DivR<MAXD> ds(rs), dr(rr);
   const u64 qs = ds.div(A), qr = dr.div(A);
   const u32 rems = (u32)(A - qs * rs), remr = (u32)(A - qr * rr);
   u64 best = 0;
@@ -71,7 +91,7 @@ __device__ __forceinline__ u64 boundary_max(u64 A, u32 send, u32 recv, const u64
     const u64 lo = umax(lo_i, lo_j), hi = umin(hi_i, hi_j);
     if (hi > lo) {
       const int u = __ffs(send) - 1, v = __ffs(recv) - 1;
-      best = umax(best, (hi - lo) * tau[u * 8 + v]);
+      best = umax(best, (hi - lo) * tau[u * TAUW + v]);
     }
     const bool adv_i = hi_i <= hi_j, adv_j = hi_j <= hi_i;
     if (adv_i) {
@@ -88,6 +108,7 @@ __device__ __forceinline__ u64 boundary_max(u64 A, u32 send, u32 recv, const u64
 
 // Ring all-reduce of a replicated stage (row a6): 2(r-1) steps of a ceil(P_s/r)-byte chunk over the
 // slowest link of the ring W_s[0] -> W_s[1] -> ... -> W_s[0] (ascending worker order).
+template <int MAXD = 8>
 __device__ __forceinline__ u64 allreduce_time(u64 Ps, u32 mask, const u64 *tau) {
   const u32 r = __popc(mask);
   const int first = __ffs(mask) - 1;
@@ -97,11 +118,11 @@ __device__ __forceinline__ u64 allreduce_time(u64 Ps, u32 mask, const u64 *tau) 
   while (m) {
     const int w = __ffs(m) - 1;
     m &= m - 1;
-    tr = umax(tr, tau[prev * 8 + w]);
+    tr = umax(tr, tau[prev * TAUW + w]);
     prev = w;
   }
-  tr = umax(tr, tau[prev * 8 + first]);
-  return 2ull * (u64)(r - 1) * xfer(Div8(r).ceil(Ps), tr);
+  tr = umax(tr, tau[prev * TAUW + first]);
+  return 2ull * (u64)(r - 1) * xfer(DivR<MAXD>(r).ceil(Ps), tr);
 }
 
 // Sharded parameter server of a replicated stage (row f3, reading F-3; PS scheme):
@@ -109,9 +130,10 @@ __device__ __forceinline__ u64 allreduce_time(u64 Ps, u32 mask, const u64 *tau) 
 // pushes that gradient shard to it and pulls the updated shard back. A server takes its pushes one
 // after another (and sends its pulls one after another); servers work in parallel:
 //   PS = max_v sum_{u != v} xfer(|shard_v|, tau[u][v]) + max_v sum_{u != v} xfer(|shard_v|, tau[v][u]).
+template <int MAXD = 8>
 __device__ __forceinline__ u64 ps_time(u64 Ps, u32 mask, const u64 *tau) {
   const u32 r = __popc(mask);
-  const Div8 dv(r);
+  const DivR<MAXD> dv(r);
   const u64 q = dv.div(Ps);
   const u32 rem = (u32)(Ps - q * r);
   u64 push = 0, pull = 0, lo = 0;
@@ -127,8 +149,8 @@ __device__ __forceinline__ u64 ps_time(u64 Ps, u32 mask, const u64 *tau) {
     while (mu) {
       const int u = __ffs(mu) - 1;
       mu &= mu - 1;
-      in += xfer(sz, tau[u * 8 + v]);
-      out += xfer(sz, tau[v * 8 + u]);
+      in += xfer(sz, tau[u * TAUW + v]);
+      out += xfer(sz, tau[v * TAUW + u]);
     }
     push = umax(push, in);
     pull = umax(pull, out);
@@ -137,36 +159,38 @@ __device__ __forceinline__ u64 ps_time(u64 Ps, u32 mask, const u64 *tau) {
 }
 
 // Gradient synchronisation of a replicated stage (r >= 2) under the model's scheme.
+template <int MAXD = 8>
 __device__ __forceinline__ u64 sync_time(int sync, u64 Ps, u32 mask, const u64 *tau) {
-  return sync == SYNC_PS ? ps_time(Ps, mask, tau) : allreduce_time(Ps, mask, tau);
+  return sync == SYNC_PS ? ps_time<MAXD>(Ps, mask, tau) : allreduce_time<MAXD>(Ps, mask, tau);
 }
 
-// The full closed form (rows a4-a7) for one partition; S in [1, 8], the partition already validated.
+// The full closed form (rows a4-a7) for one partition; S in [1, P::MS], the partition already validated.
 // P32: the state's r = 1 bound fits 32 bits (autopipe_set_state), so every stage value X, Y, every
-// boundary sum Z and every segment sum W(s,t) is < 2^32 - 16 and the 28 segment terms use 32-bit
+// boundary sum Z and every segment sum W(s,t) is < 2^32 - 16 and the segment terms use 32-bit
 // adds and divisions by constants; the synchronisation terms (weight bytes) stay 64-bit.
 // BW (PipeDream-2BW, row f3, reading F-3): the time of an iteration of M micro-batches of the same
 // steady state, with one synchronisation per iteration: every compute term is scaled by M before its
 // ceiling (ceil(M W / k)), the synchronisation terms are not (64-bit only; M * bound < 2^59 is
 // checked on the host).
-template <bool P32, bool BW = false>
-__device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, u64 cuts, u64 masks, int sync = SYNC_RING,
+template <bool P32, bool BW = false, typename P = P8>
+__device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, const P &p, int sync = SYNC_RING,
                                                 u32 M = 1) {
   static_assert(!(P32 && BW), "the 2BW form is 64-bit");
+  constexpr int MS = P::MS;
   typedef typename std::conditional<P32, u32, u64>::type V;
-  V X[MAXS], Y[MAXS], Zb[MAXS];
+  V X[MS], Y[MS], Zb[MS];
   V T = 0;
   u64 TAR = 0;
 #pragma unroll
-  for (int s = 0; s < MAXS; ++s) {
+  for (int s = 0; s < MS; ++s) {
     X[s] = 0;
     Y[s] = 0;
     if (s < S) {
-      const int a = (s == 0) ? 0 : byte_at(cuts, s - 1) + 1;
-      const int e = (s == S - 1) ? t.L - 1 : byte_at(cuts, s);
-      const u32 mask = (u32)byte_at(masks, s);
+      const int a = (s == 0) ? 0 : p.cut(s - 1) + 1;
+      const int e = (s == S - 1) ? t.L - 1 : p.cut(s);
+      const u32 mask = p.mask(s);
       const u32 r = __popc(mask);
-      const Div8 dv(r);
+      const DivR<P::MN> dv(r);
       u32 m = mask;
       // first replica unconditionally; the loop only runs for replicated stages
       int w = __ffs(m) - 1;
@@ -187,29 +211,29 @@ __device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, u64 cut
       Y[s] = (V)(fm + bm);
       const V xs = BW ? (V)(xm * M) : (V)xm;
       T = T > xs ? T : xs;
-      if (r >= 2) TAR = umax(TAR, sync_time(sync, t.PP[e + 1] - t.PP[a], mask, t.tau));
+      if (r >= 2) TAR = umax(TAR, sync_time<P::MN>(sync, t.PP[e + 1] - t.PP[a], mask, t.tau));
     }
   }
 #pragma unroll
-  for (int s = 0; s < MAXS - 1; ++s) {  // row a5
+  for (int s = 0; s < MS - 1; ++s) {  // row a5
     Zb[s] = 0;
     if (s < S - 1) {
-      const int e = byte_at(cuts, s);
-      const u32 ms = (u32)byte_at(masks, s), mn = (u32)byte_at(masks, s + 1);
-      const u64 cf = boundary_max(t.O[e], ms, mn, t.tau);
-      const u64 cb = boundary_max(t.G[e + 1], mn, ms, t.tau);
+      const int e = p.cut(s);
+      const u32 ms = p.mask(s), mn = p.mask(s + 1);
+      const u64 cf = boundary_max<P::MN>(t.O[e], ms, mn, t.tau);
+      const u64 cb = boundary_max<P::MN>(t.G[e + 1], mn, ms, t.tau);
       Zb[s] = (V)(cf + cb);
       const V lm = BW ? (V)(umax(cf, cb) * M) : (V)umax(cf, cb);
       T = T > lm ? T : lm;
     }
   }
-  Zb[MAXS - 1] = 0;
+  Zb[MS - 1] = 0;
 #pragma unroll
-  for (int s = 0; s < MAXS - 1; ++s) {  // row a7: segment cycles, t-s+1 tokens
+  for (int s = 0; s < MS - 1; ++s) {  // row a7: segment cycles, t-s+1 tokens
     if (s < S - 1) {
       V acc = X[s];
 #pragma unroll
-      for (int u = s + 1; u < MAXS; ++u) {
+      for (int u = s + 1; u < MS; ++u) {
         if (u < S) {
           const V W = BW ? (acc + Zb[u - 1] + X[u]) * M : acc + Zb[u - 1] + X[u];
           const V c = (W + (V)(u - s)) / (V)(u - s + 1);
@@ -224,22 +248,21 @@ __device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, u64 cut
 
 // Decode + validate a 16-byte record (SPEC.md §2). Returns false for an invalid record.
 // lo = bytes 0..7 (S, cuts), hi = bytes 8..15 (stage of worker w in byte w).
-__device__ __forceinline__ bool decode_record(u64 lo, u64 hi, int L, int N, int &S, u64 &cuts,
-                                              u64 &masks) {
+__device__ __forceinline__ bool decode_record(u64 lo, u64 hi, int L, int N, int &S, P8 &p) {
   S = (int)(lo & 0xFF);
   if (S < 1 || S > MAXS || S > N) return false;
-  cuts = lo >> 8;
+  p.cuts = lo >> 8;
   bool ok = true;
   int prev = -1;
 #pragma unroll
   for (int i = 0; i < MAXS - 1; ++i) {
     if (i < S - 1) {
-      const int e = byte_at(cuts, i);
+      const int e = byte_at(p.cuts, i);
       ok &= (e > prev) & (e < L - 1);
       prev = e;
     }
   }
-  masks = 0;
+  u64 masks = 0;
 #pragma unroll
   for (int w = 0; w < MAXN; ++w) {
     const int s = byte_at(hi, w);
@@ -248,24 +271,63 @@ __device__ __forceinline__ bool decode_record(u64 lo, u64 hi, int L, int N, int 
       if (s < S) masks |= 1ull << (8 * s + w);
     }
   }
+  p.masks = masks;
 #pragma unroll
   for (int s = 0; s < MAXS; ++s)
     if (s < S) ok &= byte_at(masks, s) != 0;
   return ok;
 }
 
+// Decode + validate a 32-byte wide record (row f4; same rules with S <= 16 and 16 workers).
+// r0 = bytes 0..15 (S, cuts e_0..e_14), r1 = bytes 16..31 (stage of worker w in byte w).
+__device__ __forceinline__ bool decode_record_w(const uint4 &r0, const uint4 &r1, int L, int N, int &S, P16 &p) {
+  const u64 a = (u64)r0.x | ((u64)r0.y << 32), b = (u64)r0.z | ((u64)r0.w << 32);
+  S = (int)(a & 0xFF);
+  if (S < 1 || S > MAXSW || S > N) return false;
+  p.c[0] = (a >> 8) | (b << 56);  // cut bytes 0..7 (record bytes 1..8)
+  p.c[1] = b >> 8;                // cut bytes 8..14
+  bool ok = true;
+  int prev = -1;
+#pragma unroll
+  for (int i = 0; i < MAXSW - 1; ++i) {
+    if (i < S - 1) {
+      const int e = p.cut(i);
+      ok &= (e > prev) & (e < L - 1);
+      prev = e;
+    }
+  }
+  const u64 w0 = (u64)r1.x | ((u64)r1.y << 32), w1 = (u64)r1.z | ((u64)r1.w << 32);
+  p.m[0] = p.m[1] = p.m[2] = p.m[3] = 0;
+#pragma unroll
+  for (int w = 0; w < MAXNW; ++w) {
+    const int s = byte_at(w < 8 ? w0 : w1, w & 7);
+    if (s != 0xFF) {
+      ok &= (w < N) & (s < S);
+      const u64 bit = (s < S) ? 1ull << (16 * (s & 3) + w) : 0ull;  // registers only: no dynamic index
+      p.m[0] |= (s >> 2) == 0 ? bit : 0ull;
+      p.m[1] |= (s >> 2) == 1 ? bit : 0ull;
+      p.m[2] |= (s >> 2) == 2 ? bit : 0ull;
+      p.m[3] |= (s >> 2) == 3 ? bit : 0ull;
+    }
+  }
+#pragma unroll
+  for (int s = 0; s < MAXSW; ++s)
+    if (s < S) ok &= p.mask(s) != 0;
+  return ok;
+}
+
 // Switch bytes versus the current partition (SPEC.md §6): sum over layers l of
 // P[l] * |W_new(l) \ W_old(l)|, walked over the maximal layer ranges on which both partitions keep
 // the same stage (at most S_new + S_old - 1 ranges), using the weight prefix PP.
-__device__ __forceinline__ u64 switch_bytes(const SmemTab &t, int S, u64 cuts, u64 masks, int So,
-                                            u64 cuts_o, u64 masks_o) {
+template <typename P>
+__device__ __forceinline__ u64 switch_bytes(const SmemTab &t, int S, const P &p, int So, const P &po) {
   u64 sw = 0;
   int sn = 0, so = 0, l = 0;
   while (l < t.L) {
-    const int en = (sn == S - 1) ? t.L - 1 : byte_at(cuts, sn);
-    const int eo = (so == So - 1) ? t.L - 1 : byte_at(cuts_o, so);
+    const int en = (sn == S - 1) ? t.L - 1 : p.cut(sn);
+    const int eo = (so == So - 1) ? t.L - 1 : po.cut(so);
     const int hi = en < eo ? en : eo;
-    const u32 gained = (u32)byte_at(masks, sn) & ~(u32)byte_at(masks_o, so);
+    const u32 gained = p.mask(sn) & ~po.mask(so);
     sw += (u64)__popc(gained) * (t.PP[hi + 1] - t.PP[l]);
     l = hi + 1;
     sn += (en == hi);

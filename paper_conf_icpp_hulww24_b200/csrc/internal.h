@@ -9,33 +9,35 @@ namespace ap {
 // S stages (off[s_max + 1] = total), ncut[S] = C(L-1, S-1) candidates per composition.
 struct SearchSpace {
   int L, N, s_min, s_max, flags, pad0, pad1, pad2;
-  u64 off[MAXS + 2];
-  u64 ncut[MAXS + 2];
-  u64 ncomp[MAXS + 2];
+  u64 off[MAXSW + 2];
+  u64 ncut[MAXSW + 2];
+  u64 ncomp[MAXSW + 2];
 };
 
 // Device-side result of a search (mirrors autopipe_result).
 struct ResultDev {
   u64 time_ns, index, evaluated;
-  unsigned char part[16];
+  unsigned char part[32];  // the 16-byte record, or the 32-byte wide record (row f4)
 };
 
 // Each launcher returns the number of kernels it enqueued (for launch accounting).
 int launch_build_state(const DevTables &g, const u64 *fp, const u64 *bp, const u64 *P, const u64 *tau, u64 sumP,
                        cudaStream_t st);
-int launch_eval(const DevTables &g, const void *recs, u64 count, u64 *out_t, u64 *out_sw,
+// Explicit records, 16-byte (wide = false) or 32-byte (row f4). cur_cuts / cur_masks: the current
+// partition's packed parts (1 and 1 words, or 2 and 4 words for wide), or cur_S = nullptr.
+int launch_eval(const DevTables &g, const void *recs, u64 count, bool wide, u64 *out_t, u64 *out_sw,
                 const int *cur_S, const u64 *cur_cuts, const u64 *cur_masks, int path32, const ModelP &m, int sms,
                 cudaStream_t st);
 // Generic exhaustive search over [begin, end) (any S, any composition); writes one BlockOut per block
 // into out[out_offset ...] and returns the number of blocks used via *nblocks.
 int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, u64 end, int path32, const ModelP &m,
-                          int sms, BlockOut *out, int max_blocks, int *nblocks, cudaStream_t st);
+                          bool wide, int sms, BlockOut *out, int max_blocks, int *nblocks, cudaStream_t st);
 // Fast search over the r = 1 block of one S (all stages on one worker; SPEC.md §5, rho = 0),
 // restricted to the cut ranks [k_begin, k_end). path32 selects the 32-bit tables.
 int launch_search_r1(const DevTables &g, const SearchSpace &sp, int S, u64 k_begin, u64 k_end,
                      int path32, int sms, BlockOut *out, int max_blocks, int *nblocks, void *work,
                      void *pinned, size_t work_bytes, cudaStream_t st);
-int launch_finalize(const BlockOut *in, int n, const SearchSpace &sp, ResultDev *out, cudaStream_t st);
+int launch_finalize(const BlockOut *in, int n, const SearchSpace &sp, ResultDev *out, bool wide, cudaStream_t st);
 
 void upload_binomials(const u64 (*tab)[BINOM_K]);
 

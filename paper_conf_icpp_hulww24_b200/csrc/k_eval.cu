@@ -7,6 +7,8 @@
 // counting sort over 64 buckets), and every thread scores records of one shape: the closed form of
 // SPEC.md §4 in registers, one 8-byte store per output at the record's position.
 // Invalid records (SPEC.md §2) score UINT64_MAX and never fail the batch.
+#include <cstring>
+
 #include "eval.cuh"
 #include "internal.h"
 #include "sched.cuh"
@@ -14,8 +16,9 @@
 
 namespace ap {
 
-struct CurPart {
-  u64 cuts, masks;
+struct CurPart {  // the current partition of a rollout (16-byte or wide)
+  P8 p8;
+  P16 p16;
   int S, valid;
 };
 
@@ -26,31 +29,36 @@ struct CurPart {
 #ifndef EVAL_SORT
 #define EVAL_SORT 1
 #endif
-template <bool ROLLOUT, bool P32, int MODE>
-__device__ __forceinline__ void score_one(const SmemTab &t, int L, int N, bool overflow, const uint4 &r, u64 i,
+// Decode + validate + score one record; Rec16 -> P8 (16-byte records), Rec32 -> P16 (wide, row f4).
+__device__ __forceinline__ bool decode_any(const Rec16 &r, int L, int N, int &S, P8 &p) {
+  return decode_record((u64)r.a.x | ((u64)r.a.y << 32), (u64)r.a.z | ((u64)r.a.w << 32), L, N, S, p);
+}
+__device__ __forceinline__ bool decode_any(const Rec32 &r, int L, int N, int &S, P16 &p) {
+  return decode_record_w(r.a, r.b, L, N, S, p);
+}
+__device__ __forceinline__ const P8 &cur_part(const CurPart &c, const P8 *) { return c.p8; }
+__device__ __forceinline__ const P16 &cur_part(const CurPart &c, const P16 *) { return c.p16; }
+
+template <bool ROLLOUT, bool P32, int MODE, typename P, typename Rec>
+__device__ __forceinline__ void score_one(const SmemTab &t, int L, int N, bool overflow, const Rec &r, u64 i,
                                           u64 *__restrict__ out_t, u64 *__restrict__ out_sw, const CurPart &cur,
                                           const ModelP &m) {
-  const u64 lo = (u64)r.x | ((u64)r.y << 32), hi = (u64)r.z | ((u64)r.w << 32);
   int S;
-  u64 cuts, masks;
+  P p;
   u64 T = U64MAX, sw = U64MAX;
-  if (!overflow && decode_record(lo, hi, L, N, S, cuts, masks)) {
-    T = model_time<MODE, P32>(t, S, cuts, masks, m);
-    if (ROLLOUT) sw = switch_bytes(t, S, cuts, masks, cur.S, cur.cuts, cur.masks);
+  if (!overflow && decode_any(r, L, N, S, p)) {
+    T = model_time<MODE, P32>(t, S, p, m);
+    if (ROLLOUT) sw = switch_bytes(t, S, p, cur.S, cur_part(cur, (const P *)nullptr));
   }
   out_t[i] = T;
   if (ROLLOUT) out_sw[i] = sw;
 }
 
 // MODE: the schedule of the model (row f3; SCHED_PIPEDREAM is the 1F1B closed form of rows a4-a7).
-// With EVAL_SORT a block takes chunks of EV_CH consecutive records (coalesced 128-bit loads), counts
-// them into shape buckets in shared memory, and scores them in bucket order: random rollout records
-// mix S = 1..8 and replica counts, and scoring them in input order left ~9 of 32 lanes active
-// (ncu); in bucket order the warps run uniform loop trip counts. Each time goes back to the
-// record's own position (8-byte scattered stores within the chunk).
-template <bool ROLLOUT, bool P32, int MODE>
-__global__ void __launch_bounds__(256, MODE == SCHED_PIPEDREAM ? EVAL_MINB : 2)
-    k_eval(DevTables g, const uint4 *__restrict__ recs, u64 count, u64 *__restrict__ out_t, u64 *__restrict__ out_sw,
+// Rec / P: 16-byte records (P8) or 32-byte wide records (P16, row f4).
+template <bool ROLLOUT, bool P32, int MODE, typename Rec, typename P>
+__global__ void __launch_bounds__(256, (MODE == SCHED_PIPEDREAM && P::MS == 8) ? EVAL_MINB : 2)
+    k_eval(DevTables g, const Rec *__restrict__ recs, u64 count, u64 *__restrict__ out_t, u64 *__restrict__ out_sw,
            CurPart cur, ModelP m) {
   extern __shared__ u64 sm[];
   const SmemTab t = stage_tables(g, sm);
@@ -58,57 +66,72 @@ __global__ void __launch_bounds__(256, MODE == SCHED_PIPEDREAM ? EVAL_MINB : 2)
   // a state that failed the device-side overflow check (set_state_device) scores nothing
   const bool overflow = (g.status[0] & 1ull) != 0;
 #if EVAL_SORT
-  for_each_sorted(recs, count, [&](const uint4 &r, u64 i) {
-    score_one<ROLLOUT, P32, MODE>(t, L, N, overflow, r, i, out_t, out_sw, cur, m);
+  for_each_sorted(recs, count, [&](const Rec &r, u64 i) {
+    score_one<ROLLOUT, P32, MODE, P>(t, L, N, overflow, r, i, out_t, out_sw, cur, m);
   });
 #else
   const u64 stride = (u64)gridDim.x * blockDim.x;
   for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < count; i += stride)
-    score_one<ROLLOUT, P32, MODE>(t, L, N, overflow, __ldg(recs + i), i, out_t, out_sw, cur, m);
+    score_one<ROLLOUT, P32, MODE, P>(t, L, N, overflow, load_rec(recs + i), i, out_t, out_sw, cur, m);
 #endif
 }
 
-static int grid_for(u64 count, int sms) {
+static int grid_for(u64 count, int sms, int per_sm) {
   const u64 per = EVAL_SORT ? (u64)EV_CH : 256;  // records per block and step
   const u64 need = (count + per - 1) / per;
-  const u64 cap = (u64)sms * (EVAL_SORT ? EVAL_MINB : 8);  // one wave of resident blocks
+  const u64 cap = (u64)sms * (EVAL_SORT ? per_sm : 8);  // one wave of resident blocks
   return (int)(need < cap ? (need ? need : 1) : cap);
 }
 
-template <bool ROLLOUT, bool P32, int MODE>
-static void run_eval(int grid, size_t smem, cudaStream_t st, const DevTables &g, const void *recs, u64 count,
+template <bool ROLLOUT, bool P32, int MODE, typename Rec, typename P>
+static void run_eval(int sms, size_t smem, cudaStream_t st, const DevTables &g, const void *recs, u64 count,
                      u64 *out_t, u64 *out_sw, const CurPart &cur, const ModelP &m) {
-  k_eval<ROLLOUT, P32, MODE><<<grid, 256, smem, st>>>(g, (const uint4 *)recs, count, out_t, out_sw, cur, m);
+  const int per_sm = (MODE == SCHED_PIPEDREAM && P::MS == 8) ? EVAL_MINB : 2;
+  k_eval<ROLLOUT, P32, MODE, Rec, P><<<grid_for(count, sms, per_sm), 256, smem, st>>>(g, (const Rec *)recs, count,
+                                                                                     out_t, out_sw, cur, m);
 }
 
-template <bool ROLLOUT>
-static void dispatch_eval(int grid, size_t smem, cudaStream_t st, const DevTables &g, const void *recs, u64 count,
+template <bool ROLLOUT, typename Rec, typename P>
+static void dispatch_eval(int sms, size_t smem, cudaStream_t st, const DevTables &g, const void *recs, u64 count,
                           u64 *out_t, u64 *out_sw, const CurPart &cur, const ModelP &m, int path32) {
   switch (m.sched) {
-    case SCHED_2BW: run_eval<ROLLOUT, false, SCHED_2BW>(grid, smem, st, g, recs, count, out_t, out_sw, cur, m); break;
-    case SCHED_GPIPE: run_eval<ROLLOUT, false, SCHED_GPIPE>(grid, smem, st, g, recs, count, out_t, out_sw, cur, m); break;
-    case SCHED_DAPPLE: run_eval<ROLLOUT, false, SCHED_DAPPLE>(grid, smem, st, g, recs, count, out_t, out_sw, cur, m); break;
+    case SCHED_2BW: run_eval<ROLLOUT, false, SCHED_2BW, Rec, P>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m); break;
+    case SCHED_GPIPE: run_eval<ROLLOUT, false, SCHED_GPIPE, Rec, P>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m); break;
+    case SCHED_DAPPLE: run_eval<ROLLOUT, false, SCHED_DAPPLE, Rec, P>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m); break;
     default:
-      if (path32) run_eval<ROLLOUT, true, SCHED_PIPEDREAM>(grid, smem, st, g, recs, count, out_t, out_sw, cur, m);
-      else run_eval<ROLLOUT, false, SCHED_PIPEDREAM>(grid, smem, st, g, recs, count, out_t, out_sw, cur, m);
+      if (path32) run_eval<ROLLOUT, true, SCHED_PIPEDREAM, Rec, P>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m);
+      else run_eval<ROLLOUT, false, SCHED_PIPEDREAM, Rec, P>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m);
   }
 }
 
-int launch_eval(const DevTables &g, const void *recs, u64 count, u64 *out_t, u64 *out_sw,
+// cur_rec: the current partition's record (16 or 32 bytes as `wide`), already validated by the host,
+// or nullptr. Its S and parts are decoded here.
+int launch_eval(const DevTables &g, const void *recs, u64 count, bool wide, u64 *out_t, u64 *out_sw,
                 const int *cur_S, const u64 *cur_cuts, const u64 *cur_masks, int path32, const ModelP &m, int sms,
                 cudaStream_t st) {
   if (count == 0) return 0;
   const size_t smem = (size_t)smem_words(g.L, g.N) * sizeof(u64);
-  CurPart cur{0, 0, 0, 0};
+  CurPart cur;
+  memset(&cur, 0, sizeof(cur));
   if (cur_S) {
     cur.S = *cur_S;
-    cur.cuts = *cur_cuts;
-    cur.masks = *cur_masks;
+    if (wide) {
+      cur.p16.c[0] = cur_cuts[0];
+      cur.p16.c[1] = cur_cuts[1];
+      for (int i = 0; i < 4; ++i) cur.p16.m[i] = cur_masks[i];
+    } else {
+      cur.p8.cuts = cur_cuts[0];
+      cur.p8.masks = cur_masks[0];
+    }
     cur.valid = 1;
   }
-  const int grid = grid_for(count, sms);
-  if (out_sw) dispatch_eval<true>(grid, smem, st, g, recs, count, out_t, out_sw, cur, m, path32);
-  else dispatch_eval<false>(grid, smem, st, g, recs, count, out_t, nullptr, cur, m, path32);
+  if (wide) {
+    if (out_sw) dispatch_eval<true, Rec32, P16>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m, path32);
+    else dispatch_eval<false, Rec32, P16>(sms, smem, st, g, recs, count, out_t, nullptr, cur, m, path32);
+  } else {
+    if (out_sw) dispatch_eval<true, Rec16, P8>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m, path32);
+    else dispatch_eval<false, Rec16, P8>(sms, smem, st, g, recs, count, out_t, nullptr, cur, m, path32);
+  }
   return 1;
 }
 

@@ -16,60 +16,87 @@
 
 namespace ap {
 
-__device__ __forceinline__ u64 first_subset(int k) {
-  u64 p = 0;
-  for (int j = 0; j < k; ++j) p |= (u64)j << (8 * j);
-  return p;
-}
+// Space-generic pieces: a 16-byte space (S, N <= 8: P8, subsets packed in one u64, binomial rows of 9
+// columns in shared memory) or a wide one (row f4; S, N <= 16: P16, Pk2 subsets, 17 columns).
+template <typename P>
+struct SpaceT;
+template <>
+struct SpaceT<P8> {
+  typedef u64 PK;
+  static constexpr int BK = BK8;
+  __device__ static bool next(PK &p, int k, int n) { return lex_next_packed(p, k, n); }
+  __device__ static P8 part(u64 cuts, u64 masks) { return P8{cuts, masks}; }
+};
+template <>
+struct SpaceT<P16> {
+  typedef Pk2 PK;
+  static constexpr int BK = BINOM_K;
+  __device__ static bool next(PK &p, int k, int n) { return lex_next_pk2(p, k, n); }
+};
 
-// masks of a contiguous placement: stage s gets workers [R_{s-1}, R_s)
-__device__ __forceinline__ u64 masks_from(const SearchSpace &sp, int S, u64 Rp) {
-  const bool all = sp.flags & 1;
-  u64 masks = 0;
-  int prev = 0;
-#pragma unroll
-  for (int s = 0; s < MAXS; ++s) {
-    if (s < S) {
-      const int R = (all && s == S - 1) ? sp.N : byte_at(Rp, s) + 1;
-      const u32 m = ((1u << R) - 1u) & ~((1u << prev) - 1u);
-      masks |= (u64)m << (8 * s);
-      prev = R;
-    }
-  }
-  return masks;
+template <typename PK>
+__device__ __forceinline__ PK first_subset(int k) {
+  PK p;
+  pk_zero(p);
+  for (int j = 0; j < k; ++j) pk_or(p, j, j);
+  return p;
 }
 
 __device__ __forceinline__ int comp_k(const SearchSpace &sp, int S) { return (sp.flags & 1) ? S - 1 : S; }
 __device__ __forceinline__ int comp_n(const SearchSpace &sp) { return (sp.flags & 1) ? sp.N - 1 : sp.N; }
 
-__device__ __forceinline__ void unrank_global(const SearchSpace &sp, u64 idx, int &S, u64 &Rp, u64 &cuts) {
-  S = sp.s_min;
-  while (S < sp.s_max && idx >= sp.off[S + 1]) ++S;
-  const u64 rem = idx - sp.off[S];
-  const u64 rho = rem / sp.ncut[S], kappa = rem % sp.ncut[S];
-  Rp = lex_unrank_packed(rho, comp_k(sp, S), comp_n(sp));
-  cuts = lex_unrank_packed(kappa, S - 1, sp.L - 1);
+// The partition of (S, composition Rp, cut set): contiguous placement, stage s gets workers
+// [R_{s-1}, R_s) (reading C-11).
+template <typename P, typename PK>
+__device__ __forceinline__ P part_from(const SearchSpace &sp, int S, const PK &Rp, const PK &cuts) {
+  const bool all = sp.flags & 1;
+  P p;
+  int prev = 0;
+  if constexpr (P::MS == 8) {
+    p.cuts = cuts;
+    p.masks = 0;
+  } else {
+    p.c[0] = cuts.lo;
+    p.c[1] = cuts.hi;
+    p.m[0] = p.m[1] = p.m[2] = p.m[3] = 0;
+  }
+#pragma unroll
+  for (int s = 0; s < P::MS; ++s) {
+    if (s < S) {
+      const int R = (all && s == S - 1) ? sp.N : pk_get(Rp, s) + 1;
+      const u32 m = ((1u << R) - 1u) & ~((1u << prev) - 1u);
+      if constexpr (P::MS == 8) p.masks |= (u64)m << (8 * s);
+      else p.m[s >> 2] |= (u64)m << (16 * (s & 3));
+      prev = R;
+    }
+  }
+  return p;
 }
 
-// same, against a binomial table in shared memory (fixed-length binary searches, no divergence)
-__device__ __forceinline__ void unrank_global_smem(const SearchSpace &sp, u64 idx, int &S, u64 &Rp, u64 &cuts,
+// global index -> (S, composition, cut set), against a binomial table in shared memory
+// (fixed-length binary searches, no divergence)
+template <int BK, typename PK>
+__device__ __forceinline__ void unrank_global_smem(const SearchSpace &sp, u64 idx, int &S, PK &Rp, PK &cuts,
                                                    const u64 *Bn) {
   S = sp.s_min;
   while (S < sp.s_max && idx >= sp.off[S + 1]) ++S;
   const u64 rem = idx - sp.off[S];
   const u64 rho = rem / sp.ncut[S], kappa = rem % sp.ncut[S];
-  Rp = lex_unrank_smem(rho, comp_k(sp, S), comp_n(sp), Bn);
-  cuts = lex_unrank_smem(kappa, S - 1, sp.L - 1, Bn);
+  Rp = lex_unrank_smem<BK, PK>(rho, comp_k(sp, S), comp_n(sp), Bn);
+  cuts = lex_unrank_smem<BK, PK>(kappa, S - 1, sp.L - 1, Bn);
 }
 
-template <int NT, bool P32, int MODE>
+template <int NT, bool P32, int MODE, typename P>
 __global__ void __launch_bounds__(NT) k_search_generic(DevTables g, SearchSpace sp, u64 begin, u64 end,
                                                        u64 per_thread, BlockOut *out, ModelP m) {
+  typedef SpaceT<P> SP;
+  typedef typename SP::PK PK;
+  constexpr int BK = SP::BK;
   extern __shared__ u64 sm[];
-  // binomial rows n <= L (n = N <= 8 <= L + 1 for the compositions too) after the state tables
+  // binomial rows n <= L (n = N <= 16 <= L + 1 for the compositions too) after the state tables
   u64 *Bn = sm + smem_words(g.L, g.N);
-  const int nb = ((int)g.L + 1 > 9 ? (int)g.L + 1 : 9) * BINOM_K;
-  for (int i = threadIdx.x; i < nb; i += NT) Bn[i] = c_binom[i / BINOM_K][i % BINOM_K];
+  const int nb = ((int)g.L + 1 > MAXNW + 1 ? (int)g.L + 1 : MAXNW + 1) * BK;
+  for (int i = threadIdx.x; i < nb; i += NT) Bn[i] = c_binom[i / BK][i % BK];
   const SmemTab t = stage_tables(g, sm);  // ends with __syncthreads()
   const u64 gtid = (u64)blockIdx.x * NT + threadIdx.x;
   u64 bestT = U64MAX, bestI = U64MAX, cnt = 0;
@@ -78,34 +105,47 @@ __global__ void __launch_bounds__(NT) k_search_generic(DevTables g, SearchSpace 
     const u64 i0 = begin + gtid * per_thread;
     const u64 i1 = (end - i0 < per_thread) ? end : i0 + per_thread;
     int S;
-    u64 Rp, cuts;
-    unrank_global_smem(sp, i0, S, Rp, cuts, Bn);
-    u64 masks = masks_from(sp, S, Rp);
+    PK Rp, cuts;
+    unrank_global_smem<BK>(sp, i0, S, Rp, cuts, Bn);
+    P p = part_from<P>(sp, S, Rp, cuts);
     for (u64 i = i0; i < i1; ++i) {
-      const u64 T = model_time<MODE, P32>(t, S, cuts, masks, m);
+      const u64 T = model_time<MODE, P32>(t, S, p, m);
       if (T < bestT) {  // indices increase along the thread's range: strict < keeps the first
         bestT = T;
         bestI = i;
       }
       ++cnt;
       if (i + 1 == i1) break;
-      if (!lex_next_packed(cuts, S - 1, sp.L - 1)) {  // cut set exhausted: next composition
-        cuts = first_subset(S - 1);
-        if (!lex_next_packed(Rp, comp_k(sp, S), comp_n(sp))) {  // compositions exhausted: next S
+      if (!SP::next(cuts, S - 1, sp.L - 1)) {  // cut set exhausted: next composition
+        cuts = first_subset<PK>(S - 1);
+        if (!SP::next(Rp, comp_k(sp, S), comp_n(sp))) {  // compositions exhausted: next S
           ++S;
           if (S > sp.s_max) break;
-          Rp = first_subset(comp_k(sp, S));
-          cuts = first_subset(S - 1);
+          Rp = first_subset<PK>(comp_k(sp, S));
+          cuts = first_subset<PK>(S - 1);
         }
-        masks = masks_from(sp, S, Rp);
       }
+      p = part_from<P>(sp, S, Rp, cuts);
     }
   }
   block_minloc_store<NT>(bestT, bestI, cnt, out + blockIdx.x);
 }
 
+template <int NT, typename P>
+static void run_search_generic(unsigned nbk, size_t smem, cudaStream_t st, const DevTables &g, const SearchSpace &sp,
+                               u64 begin, u64 end, u64 pt, BlockOut *out, const ModelP &m, int path32) {
+  switch (m.sched) {
+    case SCHED_2BW: k_search_generic<NT, false, SCHED_2BW, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m); break;
+    case SCHED_GPIPE: k_search_generic<NT, false, SCHED_GPIPE, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m); break;
+    case SCHED_DAPPLE: k_search_generic<NT, false, SCHED_DAPPLE, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m); break;
+    default:
+      if (path32) k_search_generic<NT, true, SCHED_PIPEDREAM, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m);
+      else k_search_generic<NT, false, SCHED_PIPEDREAM, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m);
+  }
+}
+
 int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, u64 end, int path32, const ModelP &m,
-                          int sms, BlockOut *out, int max_blocks, int *nblocks, cudaStream_t st) {
+                          bool wide, int sms, BlockOut *out, int max_blocks, int *nblocks, cudaStream_t st) {
   constexpr int NT = 256;
   const u64 span = end - begin;
   // at least 4 candidates per thread (the unrank is a few binary searches); up to 8 blocks per SM.
@@ -117,31 +157,28 @@ int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, 
   if (blocks > cap) blocks = cap;
   if (blocks == 0) blocks = 1;
   const u64 per = (span + blocks * NT - 1) / (blocks * NT);
-  const size_t smem = ((size_t)smem_words(g.L, g.N) + (size_t)((g.L + 1 > 9 ? g.L + 1 : 9) * BINOM_K)) * sizeof(u64);
+  const int BK = wide ? BINOM_K : BK8;
+  const size_t smem = ((size_t)smem_words(g.L, g.N) +
+                       (size_t)(((int)g.L + 1 > MAXNW + 1 ? (int)g.L + 1 : MAXNW + 1) * BK)) * sizeof(u64);
   const unsigned nbk = (unsigned)blocks;
   const u64 pt = per ? per : 1;
-  switch (m.sched) {
-    case SCHED_2BW: k_search_generic<NT, false, SCHED_2BW><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m); break;
-    case SCHED_GPIPE: k_search_generic<NT, false, SCHED_GPIPE><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m); break;
-    case SCHED_DAPPLE: k_search_generic<NT, false, SCHED_DAPPLE><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m); break;
-    default:
-      if (path32) k_search_generic<NT, true, SCHED_PIPEDREAM><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m);
-      else k_search_generic<NT, false, SCHED_PIPEDREAM><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m);
-  }
+  if (wide) run_search_generic<NT, P16>(nbk, smem, st, g, sp, begin, end, pt, out, m, path32);
+  else run_search_generic<NT, P8>(nbk, smem, st, g, sp, begin, end, pt, out, m, path32);
   *nblocks = (int)blocks;
   return 1;
 }
 
 // ---------------------------------------------------------------------------------------------
 // grid-level finalisation: one block reduces the per-block (T, index, count) entries, then decodes
-// the winning index into its 16-byte partition record.
+// the winning index into its partition record (16 bytes, or 32 for a wide space).
 // ---------------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(256) k_finalize(const BlockOut *in, int n, SearchSpace sp, ResultDev *res) {
+__global__ void __launch_bounds__(256) k_finalize(const BlockOut *in, int n, SearchSpace sp, ResultDev *res, int wide) {
   // binomial rows 0..L (all the unranking needs) in shared memory: the winner is decoded with
   // fixed-length binary searches instead of a serial walk over __constant__ (which misses its cache)
   __shared__ u64 Bn[(MAXL + 1) * BINOM_K];
+  const int BK = wide ? BINOM_K : BK8;
   const int rows = (sp.L > sp.N ? sp.L : sp.N) + 1;  // cut sets of {0..L-2}, compositions of {1..N}
-  for (int i = threadIdx.x; i < rows * BINOM_K; i += 256) Bn[i] = c_binom[i / BINOM_K][i % BINOM_K];
+  for (int i = threadIdx.x; i < rows * BK; i += 256) Bn[i] = c_binom[i / BK][i % BK];
   u64 t = U64MAX, idx = U64MAX, cnt = 0;
   for (int i = threadIdx.x; i < n; i += 256) {
     const BlockOut b = in[i];
@@ -155,25 +192,37 @@ __global__ void __launch_bounds__(256) k_finalize(const BlockOut *in, int n, Sea
     res->time_ns = slot.t;
     res->index = slot.idx;
     res->evaluated = slot.count;
-    unsigned char rec[16];
-    for (int i = 0; i < 16; ++i) rec[i] = 0xFF;
+    unsigned char rec[32];
+    for (int i = 0; i < 32; ++i) rec[i] = 0xFF;
+    const int off = wide ? 16 : 8;
     if (slot.idx != U64MAX) {
       int S;
-      u64 Rp, cuts;
-      unrank_global_smem(sp, slot.idx, S, Rp, cuts, Bn);
-      const u64 masks = masks_from(sp, S, Rp);
-      rec[0] = (unsigned char)S;
-      for (int s = 0; s < S - 1; ++s) rec[1 + s] = (unsigned char)byte_at(cuts, s);
-      for (int s = 0; s < S; ++s)
-        for (int w = 0; w < MAXN; ++w)
-          if ((byte_at(masks, s) >> w) & 1) rec[8 + w] = (unsigned char)s;
+      if (wide) {
+        Pk2 Rp, cuts;
+        unrank_global_smem<BINOM_K>(sp, slot.idx, S, Rp, cuts, Bn);
+        const P16 p = part_from<P16>(sp, S, Rp, cuts);
+        rec[0] = (unsigned char)S;
+        for (int s = 0; s < S - 1; ++s) rec[1 + s] = (unsigned char)p.cut(s);
+        for (int s = 0; s < S; ++s)
+          for (int w = 0; w < MAXNW; ++w)
+            if ((p.mask(s) >> w) & 1) rec[off + w] = (unsigned char)s;
+      } else {
+        u64 Rp, cuts;
+        unrank_global_smem<BK8>(sp, slot.idx, S, Rp, cuts, Bn);
+        const P8 p = part_from<P8>(sp, S, Rp, cuts);
+        rec[0] = (unsigned char)S;
+        for (int s = 0; s < S - 1; ++s) rec[1 + s] = (unsigned char)p.cut(s);
+        for (int s = 0; s < S; ++s)
+          for (int w = 0; w < MAXN; ++w)
+            if ((p.mask(s) >> w) & 1) rec[off + w] = (unsigned char)s;
+      }
     }
-    for (int i = 0; i < 16; ++i) res->part[i] = rec[i];
+    for (int i = 0; i < 32; ++i) res->part[i] = rec[i];
   }
 }
 
-int launch_finalize(const BlockOut *in, int n, const SearchSpace &sp, ResultDev *out, cudaStream_t st) {
-  k_finalize<<<1, 256, 0, st>>>(in, n, sp, out);
+int launch_finalize(const BlockOut *in, int n, const SearchSpace &sp, ResultDev *out, bool wide, cudaStream_t st) {
+  k_finalize<<<1, 256, 0, st>>>(in, n, sp, out, wide ? 1 : 0);
   return 1;
 }
 

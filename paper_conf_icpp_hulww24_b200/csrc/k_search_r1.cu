@@ -290,11 +290,11 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? R1_MINB32 : R1_MINB64) k_
   u64 *Z = PC + S * Lp1;
   u64 *LM = Z + (S - 1) * L;
   u64 *Bn = LM + (S - 1) * L;
-  R1YEntry *yt = (R1YEntry *)(Bn + Lp1 * BINOM_K);
+  R1YEntry *yt = (R1YEntry *)(Bn + Lp1 * BK8);
   // per-warp folded tables follow the schedule (16-byte aligned)
   const int FN = (n + 16 + 3) & ~3;  // columns per warp table (rows of whole 16-byte units)
   T *foldall = (T *)(((uintptr_t)(yt + hdr_g->ny) + 15) & ~(uintptr_t)15);
-  for (int i = threadIdx.x; i < Lp1 * BINOM_K; i += NT) Bn[i] = c_binom[i / BINOM_K][i % BINOM_K];
+  for (int i = threadIdx.x; i < Lp1 * BK8; i += NT) Bn[i] = c_binom[i / BK8][i % BK8];
   for (int i = threadIdx.x; i < S * Lp1; i += NT) PC[i] = g.PC[i];
   for (int i = threadIdx.x; i < (S - 1) * L; i += NT) {
     Z[i] = g.Z[i];
@@ -722,7 +722,7 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
   work = (unsigned char *)work + (size_t)S * 16384;
   cudaMemcpyAsync(work, hbuf, hbytes, cudaMemcpyHostToDevice, st);
   const size_t smem = (size_t)(n + 16) * sizeof(ColT<T>) + (size_t)n * sizeof(XT) + (size_t)S * (L + 1) * 8 +
-                      2 * (size_t)(S - 1) * L * 8 + (size_t)(L + 1) * BINOM_K * 8 + (size_t)ny * sizeof(R1YEntry) + 16 +
+                      2 * (size_t)(S - 1) * L * 8 + (size_t)(L + 1) * BK8 * 8 + (size_t)ny * sizeof(R1YEntry) + 16 +
                       (size_t)(NT / 32) * (size_t)((n + 16 + 3) & ~3) * sizeof(T);
   // the attribute and the occupancy query cost microseconds each: redo them only when smem changes
   // (per device: a process may drive several GPUs, one context each)

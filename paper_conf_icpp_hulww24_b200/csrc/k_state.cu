@@ -7,7 +7,7 @@
 //   warps 0 .. 3N   : one row each — warp-shuffle inclusive scan (__shfl_up_sync) over 32-element
 //                     chunks with a running carry, written as an exclusive prefix of L + 1 entries
 //                     (rows: PF[w], PB[w], PC[w] = prefix of f + b, and PP), plus 32-bit copies of PC;
-//   warp 3N + 1     : copies tau (N x N) into the padded 8 x 8 table and computes the overflow /
+//   warp 3N + 1     : copies tau (N x N) into the padded 16 x 16 table and computes the overflow /
 //                     32-bit-path status of SPEC.md §7 (used when the inputs came from device memory);
 //   remaining warps : link tables Z[s][l] = cf + cb and LM[s][l] = max(cf, cb) for the boundary
 //                     between worker s and s + 1 at a cut after layer l, with
@@ -79,8 +79,8 @@ __global__ void k_build_state(DevTables g, const u64 *__restrict__ fp, const u64
   }
   if (gw == scan_warps) {
     // padded tau and the status word (SPEC.md §7 overflow rule, 32-bit search path)
-    for (int i = lane; i < 64; i += 32) {
-      const int u = i >> 3, v = i & 7;
+    for (int i = lane; i < TAUW * TAUW; i += 32) {
+      const int u = i / TAUW, v = i % TAUW;
       g.tau[i] = (u < N && v < N && u != v) ? tau[u * N + v] : 0ull;
     }
     u64 mt = 0;
@@ -113,12 +113,14 @@ __global__ void k_build_state(DevTables g, const u64 *__restrict__ fp, const u64
       if (hi != 0 || lo + 999999ull < lo) ovf = true;
       const u64 maxX = ovf ? 0 : (lo + 999999ull) / 1000000ull;
       const u64 maxXog = (maxOG * maxTau + 999999ull) / 1000000ull;  // <= maxX
-      // bound = sumMax + 16 + 28 maxX < 2^59 (sumMax < 2^59 and maxX < 2^55 here: no wrap)
+      // bound = sumMax + 16 + 28 maxX < 2^59 (N <= 8; 32 + 60 maxX for N <= 16, wide records; sumMax <
+      // 2^59 and maxX < 2^55 here: no wrap). The host path (autopipe_set_state) uses the same rule.
       u64 bound = ~0ull, bound32 = ~0ull;
       if (maxX >= (1ull << 55)) ovf = true;
+      const bool wideN = N > MAXN;
       if (!ovf) {
-        bound = sumMax + 16 + 28 * maxX;
-        bound32 = sumMax + 16 + 14 * maxXog;
+        bound = sumMax + (wideN ? 32 : 16) + (wideN ? 60 : 28) * maxX;
+        bound32 = sumMax + (wideN ? 32 : 16) + (wideN ? 30 : 14) * maxXog;
       }
       if (bound >= (1ull << 59)) ovf = true;
       const u64 path32 = (!ovf && bound32 < 0xFFFFFFF0ull) ? 2ull : 0ull;

@@ -168,7 +168,7 @@ __global__ void __launch_bounds__(256) k_switch(DevTables g, const uint4 *__rest
     u64 m = U64MAX;
     if (so < cur.S)
       for (int u = 0; u < MAXN; ++u)
-        if ((cur.masks[so] >> u) & 1u) m = umin(m, t.tau[u * 8 + w]);
+        if ((cur.masks[so] >> u) & 1u) m = umin(m, t.tau[u * TAUW + w]);
     tmin[threadIdx.x] = m;
   }
   __syncthreads();
@@ -179,10 +179,11 @@ __global__ void __launch_bounds__(256) k_switch(DevTables g, const uint4 *__rest
     const uint4 r = __ldg(recs + i);
     const u64 lo = (u64)r.x | ((u64)r.y << 32), hi = (u64)r.z | ((u64)r.w << 32);
     int S;
-    u64 cuts, masks;
+    P8 pp;
     u64 T = U64MAX, R = U64MAX, M = U64MAX, RW = U64MAX;
-    if (!overflow && decode_record(lo, hi, L, N, S, cuts, masks)) {
-      T = eval_closed_form<P32>(t, S, cuts, masks, (int)sync);
+    if (!overflow && decode_record(lo, hi, L, N, S, pp)) {
+      const u64 cuts = pp.cuts, masks = pp.masks;
+      T = eval_closed_form<P32>(t, S, pp, (int)sync);
       // per-worker layer sets, compared with the current partition's
       bool same = true;
 #pragma unroll

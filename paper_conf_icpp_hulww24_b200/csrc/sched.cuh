@@ -23,13 +23,14 @@ namespace ap {
 constexpr int MAXPAIRS = 2 * MAXN;  // sum over boundaries of (r_s + r_{s+1} - 1) <= 2 sum r - (S-1)
 
 // Durations of every transfer of one boundary, in merge order (see boundary_max in eval.cuh).
+template <int MAXD = 8>
 __device__ __forceinline__ int boundary_pairs(u64 A, u32 send, u32 recv, const u64 *tau, u64 *d, int n) {
   const u32 rs = __popc(send), rr = __popc(recv);
   if (rs == 1 && rr == 1) {
-    d[n] = xfer(A, tau[(__ffs(send) - 1) * 8 + __ffs(recv) - 1]);
+    d[n] = xfer(A, tau[(__ffs(send) - 1) * TAUW + __ffs(recv) - 1]);
     return n + 1;
   }
-  const Div8 ds(rs), dr(rr);
+  const DivR<MAXD> ds(rs), dr(rr);
   const u64 qs = ds.div(A), qr = dr.div(A);
   const u32 rems = (u32)(A - qs * rs), remr = (u32)(A - qr * rr);
   u32 i = 0, j = 0;
@@ -37,7 +38,7 @@ __device__ __forceinline__ int boundary_pairs(u64 A, u32 send, u32 recv, const u
   u64 hi_i = qs + ds.small(rems), hi_j = qr + dr.small(remr);
   while (i < rs && j < rr) {
     const u64 lo = umax(lo_i, lo_j), hi = umin(hi_i, hi_j);
-    if (hi > lo) d[n++] = xfer(hi - lo, tau[(__ffs(send) - 1) * 8 + __ffs(recv) - 1]);
+    if (hi > lo) d[n++] = xfer(hi - lo, tau[(__ffs(send) - 1) * TAUW + __ffs(recv) - 1]);
     const bool adv_i = hi_i <= hi_j, adv_j = hi_j <= hi_i;
     if (adv_i) {
       ++i; send &= send - 1;
@@ -63,54 +64,55 @@ __device__ __forceinline__ u64 run_boundary(u64 bar, const u64 *d, u64 *lf, int 
 }
 
 
-// T_ns of one flushed iteration (GPipe or DAPPLE) of a validated partition.
-template <int SCHED>
-__device__ __forceinline__ u64 flush_makespan(const SmemTab &t, int S, u64 cuts, u64 masks, const ModelP &m) {
+// T_ns of one flushed iteration (GPipe or DAPPLE) of a validated partition (P8 or the wide P16).
+template <int SCHED, typename P>
+__device__ __forceinline__ u64 flush_makespan(const SmemTab &t, int S, const P &p, const ModelP &m) {
   static_assert(SCHED == SCHED_GPIPE || SCHED == SCHED_DAPPLE, "flushed schedules only");
+  constexpr int MS = P::MS, MN = P::MN, NP = 2 * P::MN;
   const int M = (int)m.M;
-  u64 Fd[MAXN], Bd[MAXN], wf[MAXN];
-  int stg[MAXN];
+  u64 Fd[MN], Bd[MN], wf[MN];
+  int stg[MN];
 #pragma unroll
-  for (int w = 0; w < MAXN; ++w) {
+  for (int w = 0; w < MN; ++w) {
     stg[w] = 0xFF;  // idle: never matches a stage
 #pragma unroll
-    for (int s = 0; s < MAXS; ++s)
-      if (s < S && ((masks >> (8 * s + w)) & 1ull)) stg[w] = s;
+    for (int s = 0; s < MS; ++s)
+      if (s < S && ((p.mask(s) >> w) & 1u)) stg[w] = s;
     wf[w] = 0;
     Fd[w] = 0;
     Bd[w] = 0;
     const int s = stg[w];
     if (s != 0xFF) {
-      const int a = (s == 0) ? 0 : byte_at(cuts, s - 1) + 1;
-      const int e = (s == S - 1) ? t.L - 1 : byte_at(cuts, s);
-      const Div8 dv((u32)__popc((u32)byte_at(masks, s)));
+      const int a = (s == 0) ? 0 : p.cut(s - 1) + 1;
+      const int e = (s == S - 1) ? t.L - 1 : p.cut(s);
+      const DivR<MN> dv((u32)__popc(p.mask(s)));
       Fd[w] = dv.ceil(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a]);
       Bd[w] = dv.ceil(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a]);
       if (SCHED == SCHED_GPIPE && m.recompute) Bd[w] += Fd[w];  // the backward op re-runs the forward
     }
   }
-  u64 dF[MAXPAIRS], dB[MAXPAIRS], lfF[MAXPAIRS], lfB[MAXPAIRS];
-  int offF[MAXS], offB[MAXS];
+  u64 dF[NP], dB[NP], lfF[NP], lfB[NP];
+  int offF[MS], offB[MS];
   int nf = 0, nb = 0;
 #pragma unroll
-  for (int s = 0; s < MAXS - 1; ++s) {
+  for (int s = 0; s < MS - 1; ++s) {
     offF[s] = nf;
     offB[s] = nb;
     if (s < S - 1) {
-      const int e = byte_at(cuts, s);
-      const u32 ms = (u32)byte_at(masks, s), mn = (u32)byte_at(masks, s + 1);
-      nf = boundary_pairs(t.O[e], ms, mn, t.tau, dF, nf);
-      nb = boundary_pairs(t.G[e + 1], mn, ms, t.tau, dB, nb);
+      const int e = p.cut(s);
+      const u32 ms = p.mask(s), mn = p.mask(s + 1);
+      nf = boundary_pairs<MN>(t.O[e], ms, mn, t.tau, dF, nf);
+      nb = boundary_pairs<MN>(t.G[e + 1], mn, ms, t.tau, dB, nb);
     }
   }
-  offF[MAXS - 1] = nf;
-  offB[MAXS - 1] = nb;
-  for (int p = 0; p < nf; ++p) lfF[p] = 0;
-  for (int p = 0; p < nb; ++p) lfB[p] = 0;
+  offF[MS - 1] = nf;
+  offB[MS - 1] = nb;
+  for (int q = 0; q < nf; ++q) lfF[q] = 0;
+  for (int q = 0; q < nb; ++q) lfB[q] = 0;
 
-  u64 fdl[MAXS], last[MAXS];
+  u64 fdl[MS], last[MS];
 #pragma unroll
-  for (int s = 0; s < MAXS; ++s) {
+  for (int s = 0; s < MS; ++s) {
     fdl[s] = 0;
     last[s] = 0;
   }
@@ -119,7 +121,7 @@ __device__ __forceinline__ u64 flush_makespan(const SmemTab &t, int S, u64 cuts,
   {                                                                                 \
     const u64 ready = ((s_) == 0) ? 0 : fdl[(s_) > 0 ? (s_) - 1 : 0];               \
     u64 bar = 0;                                                                    \
-    _Pragma("unroll") for (int w = 0; w < MAXN; ++w) if (stg[w] == (s_)) {          \
+    _Pragma("unroll") for (int w = 0; w < MN; ++w) if (stg[w] == (s_)) {          \
       wf[w] = umax(wf[w], ready) + Fd[w];                                           \
       bar = umax(bar, wf[w]);                                                       \
     }                                                                               \
@@ -130,7 +132,7 @@ __device__ __forceinline__ u64 flush_makespan(const SmemTab &t, int S, u64 cuts,
   {                                                                                 \
     const u64 ready = ((s_) == S - 1) ? 0 : bd;                                     \
     u64 bar = 0;                                                                    \
-    _Pragma("unroll") for (int w = 0; w < MAXN; ++w) if (stg[w] == (s_)) {          \
+    _Pragma("unroll") for (int w = 0; w < MN; ++w) if (stg[w] == (s_)) {          \
       wf[w] = umax(wf[w], ready) + Bd[w];                                           \
       bar = umax(bar, wf[w]);                                                       \
     }                                                                               \
@@ -140,26 +142,26 @@ __device__ __forceinline__ u64 flush_makespan(const SmemTab &t, int S, u64 cuts,
   if (SCHED == SCHED_GPIPE) {
     for (int k = 0; k < M; ++k) {
 #pragma unroll
-      for (int s = 0; s < MAXS; ++s)
+      for (int s = 0; s < MS; ++s)
         if (s < S) AP_FWD(s)
     }
     for (int k = 0; k < M; ++k) {
       u64 bd = 0;
 #pragma unroll
-      for (int s = MAXS - 1; s >= 0; --s)
+      for (int s = MS - 1; s >= 0; --s)
         if (s < S) AP_BWD(s, k)
     }
   } else {
     const int nw = S < M ? S : M;  // n_0 = min(S, M) warm-up rounds
     for (int k = 0; k < nw; ++k) {
 #pragma unroll
-      for (int s = 0; s < MAXS; ++s)
+      for (int s = 0; s < MS; ++s)
         if (s < S && k < S - s) AP_FWD(s)  // k < n_s = min(S - s, M) (k < M already)
     }
     for (int j = 0; j < M; ++j) {
       u64 bd = 0;
 #pragma unroll
-      for (int s = MAXS - 1; s >= 0; --s) {
+      for (int s = MS - 1; s >= 0; --s) {
         if (s < S) {
           AP_BWD(s, j)
           if (j + (S - s) < M) AP_FWD(s)  // F_s(j + n_s), n_s = S - s when j + n_s < M
@@ -171,14 +173,14 @@ __device__ __forceinline__ u64 flush_makespan(const SmemTab &t, int S, u64 cuts,
 #undef AP_BWD
   u64 T = 0;
 #pragma unroll
-  for (int s = 0; s < MAXS; ++s) {
+  for (int s = 0; s < MS; ++s) {
     if (s < S) {
-      const u32 mask = (u32)byte_at(masks, s);
+      const u32 mask = p.mask(s);
       u64 x = last[s];
       if (__popc(mask) >= 2) {
-        const int a = (s == 0) ? 0 : byte_at(cuts, s - 1) + 1;
-        const int e = (s == S - 1) ? t.L - 1 : byte_at(cuts, s);
-        x += sync_time((int)m.sync, t.PP[e + 1] - t.PP[a], mask, t.tau);
+        const int a = (s == 0) ? 0 : p.cut(s - 1) + 1;
+        const int e = (s == S - 1) ? t.L - 1 : p.cut(s);
+        x += sync_time<MN>((int)m.sync, t.PP[e + 1] - t.PP[a], mask, t.tau);
       }
       T = umax(T, x);
     }
@@ -187,11 +189,11 @@ __device__ __forceinline__ u64 flush_makespan(const SmemTab &t, int S, u64 cuts,
 }
 
 // T_ns of a validated partition under the model (row f3): MODE = the schedule, fixed per kernel.
-template <int MODE, bool P32>
-__device__ __forceinline__ u64 model_time(const SmemTab &t, int S, u64 cuts, u64 masks, const ModelP &m) {
-  if (MODE == SCHED_PIPEDREAM) return eval_closed_form<P32>(t, S, cuts, masks, (int)m.sync);
-  if (MODE == SCHED_2BW) return eval_closed_form<false, true>(t, S, cuts, masks, (int)m.sync, m.M);
-  return flush_makespan<MODE == SCHED_PIPEDREAM || MODE == SCHED_2BW ? SCHED_GPIPE : MODE>(t, S, cuts, masks, m);
+template <int MODE, bool P32, typename P>
+__device__ __forceinline__ u64 model_time(const SmemTab &t, int S, const P &p, const ModelP &m) {
+  if (MODE == SCHED_PIPEDREAM) return eval_closed_form<P32, false, P>(t, S, p, (int)m.sync);
+  if (MODE == SCHED_2BW) return eval_closed_form<false, true, P>(t, S, p, (int)m.sync, m.M);
+  return flush_makespan<MODE == SCHED_PIPEDREAM || MODE == SCHED_2BW ? SCHED_GPIPE : MODE, P>(t, S, p, m);
 }
 
 }  // namespace ap

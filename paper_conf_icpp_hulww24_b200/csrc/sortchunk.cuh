@@ -15,19 +15,37 @@ constexpr int EV_PER = 4;              // records per thread and chunk
 constexpr int EV_CH = 256 * EV_PER;    // records per chunk
 constexpr int EV_NB = 64;              // shape buckets
 
+struct Rec16 {  // a 16-byte partition record
+  uint4 a;
+};
+struct Rec32 {  // a 32-byte wide partition record (row f4)
+  uint4 a, b;
+};
+__device__ __forceinline__ Rec16 load_rec(const Rec16 *p) { return Rec16{__ldg(&p->a)}; }
+__device__ __forceinline__ Rec32 load_rec(const Rec32 *p) { return Rec32{__ldg(&p->a), __ldg(&p->b)}; }
+
+__device__ __forceinline__ u32 workers_named(u32 v) { return (u32)__popc(__vcmpne4(v, 0xFFFFFFFFu)) >> 3; }
+
 // Shape of a record: S and the number of extra replicas (sum r - S), 64 buckets. Records of one
 // shape run the same stage, replica and boundary loops, so a warp of them does not diverge.
-__device__ __forceinline__ u32 shape_key(const uint4 &r) {
-  const u32 S = r.x & 0xFFu;
-  const u32 n = (u32)(__popc(__vcmpne4(r.z, 0xFFFFFFFFu)) + __popc(__vcmpne4(r.w, 0xFFFFFFFFu))) >> 3;
+__device__ __forceinline__ u32 shape_key(const Rec16 &r) {
+  const u32 S = r.a.x & 0xFFu;
+  const u32 n = workers_named(r.a.z) + workers_named(r.a.w);
   return ((S & 7u) << 3) | ((n - S) & 7u);
+}
+// wide records: S in 1..16 (4 bits) and extra replicas 0, 1, 2, >= 3 (2 bits)
+__device__ __forceinline__ u32 shape_key(const Rec32 &r) {
+  const u32 S = r.a.x & 0xFFu;
+  const u32 n = workers_named(r.b.x) + workers_named(r.b.y) + workers_named(r.b.z) + workers_named(r.b.w);
+  const u32 extra = n - S;  // wraps for an invalid record: any bucket is fine
+  return (((S - 1u) & 15u) << 2) | (extra < 3u ? extra : 3u);
 }
 
 // f(record, global index) for every record of recs[0, count), block-strided over chunks; every thread
 // of the block must call it (it synchronises the block).
-template <typename F>
-__device__ __forceinline__ void for_each_sorted(const uint4 *__restrict__ recs, u64 count, F &&f) {
-  __shared__ uint4 srec[EV_CH];
+template <typename Rec, typename F>
+__device__ __forceinline__ void for_each_sorted(const Rec *__restrict__ recs, u64 count, F &&f) {
+  __shared__ Rec srec[EV_CH];
   __shared__ u32 sidx[EV_CH];
   __shared__ u32 hist[EV_NB];
   const int tid = threadIdx.x;
@@ -36,7 +54,7 @@ __device__ __forceinline__ void for_each_sorted(const uint4 *__restrict__ recs, 
     const u64 base = ch * EV_CH;
     if (tid < EV_NB) hist[tid] = 0;
     __syncthreads();
-    uint4 rr[EV_PER];
+    Rec rr[EV_PER];
     u32 key[EV_PER], rank[EV_PER];
 #pragma unroll
     for (int j = 0; j < EV_PER; ++j) {
@@ -44,7 +62,7 @@ __device__ __forceinline__ void for_each_sorted(const uint4 *__restrict__ recs, 
       key[j] = EV_NB;
       rank[j] = 0;
       if (i < count) {
-        rr[j] = __ldg(recs + i);
+        rr[j] = load_rec(recs + i);
         key[j] = shape_key(rr[j]);
         rank[j] = atomicAdd(&hist[key[j]], 1u);
       }

@@ -14,7 +14,7 @@ import numpy as np
 import torch
 
 from . import _lib
-from ._lib import AutopipeError, Partition, Result, USE_ALL_WORKERS, lib
+from ._lib import AutopipeError, Partition, PartitionW, Result, ResultW, USE_ALL_WORKERS, lib
 
 U64_MAX = (1 << 64) - 1
 
@@ -122,10 +122,13 @@ class Engine:
 
     # -- scoring ---------------------------------------------------------------------------
     def _records(self, parts) -> torch.Tensor:
+        """Records as a contiguous uint8 device tensor [n, 16] (or [n, 32]: wide records, row f4)."""
         if not isinstance(parts, torch.Tensor):
-            parts = torch.as_tensor(np.asarray(parts, dtype=np.uint8).reshape(-1, 16))
-        if parts.dtype != torch.uint8 or parts.dim() != 2 or parts.shape[1] != 16:
-            raise ValueError("partitions must be a uint8 tensor of shape [n, 16]")
+            a = np.asarray(parts, dtype=np.uint8)
+            width = a.shape[-1] if a.ndim == 2 else 16
+            parts = torch.as_tensor(a.reshape(-1, width))
+        if parts.dtype != torch.uint8 or parts.dim() != 2 or parts.shape[1] not in (16, 32):
+            raise ValueError("partitions must be a uint8 tensor of shape [n, 16] or [n, 32]")
         if parts.device != self.device:
             parts = parts.to(self.device)
         return parts.contiguous()
@@ -135,24 +138,26 @@ class Engine:
         n = recs.shape[0]
         if out is None:
             out = torch.empty(n, dtype=torch.int64, device=self.device)
-        self._check(lib.autopipe_eval_partitions(self._h, ctypes.c_void_p(recs.data_ptr()), n,
-                                                 ctypes.c_void_p(out.data_ptr()), self._stream(stream)))
+        fn = lib.autopipe_eval_partitions_w if recs.shape[1] == 32 else lib.autopipe_eval_partitions
+        self._check(fn(self._h, ctypes.c_void_p(recs.data_ptr()), n, ctypes.c_void_p(out.data_ptr()),
+                       self._stream(stream)))
         return out
 
     def rollout_rewards(self, parts, current: Optional[bytes] = None, out_t=None, out_sw=None,
                         stream=None) -> Tuple[torch.Tensor, Optional[torch.Tensor]]:
         recs = self._records(parts)
         n = recs.shape[0]
+        wide = recs.shape[1] == 32
         if out_t is None:
             out_t = torch.empty(n, dtype=torch.int64, device=self.device)
         cur = None
         if current is not None:
-            cur = Partition.from_buffer_copy(bytes(current))
+            cur = (PartitionW if wide else Partition).from_buffer_copy(bytes(current))
             if out_sw is None:
                 out_sw = torch.empty(n, dtype=torch.int64, device=self.device)
         else:
             out_sw = None
-        self._check(lib.autopipe_rollout_rewards(
+        self._check((lib.autopipe_rollout_rewards_w if wide else lib.autopipe_rollout_rewards)(
             self._h, ctypes.c_void_p(recs.data_ptr()), n, ctypes.byref(cur) if cur is not None else None,
             ctypes.c_void_p(out_t.data_ptr()),
             ctypes.c_void_p(out_sw.data_ptr()) if out_sw is not None else None, self._stream(stream)))
@@ -176,12 +181,19 @@ class Engine:
             ptr("refill"), ptr("migrate"), ptr("reward"), self._stream(stream)))
         return out
 
+    def _wide(self, s_max: int, wide: Optional[bool]) -> bool:
+        """Spaces with S > 8 or N > 8 workers need 32-byte records (row f4)."""
+        return (s_max > 8 or self.N > 8) if wide is None else bool(wide)
+
     def search_optimum(self, s_min: int, s_max: int, flags: int = 0, begin: int = 0,
-                       end: Optional[int] = None, stream=None) -> SearchResult:
-        res = Result()
+                       end: Optional[int] = None, stream=None, wide: Optional[bool] = None) -> SearchResult:
+        """Exhaustive search of [begin, end) of the space; the result's partition is a 16-byte record,
+        or a 32-byte one for a wide space (S > 8 or N > 8, or wide=True)."""
+        w = self._wide(s_max, wide)
+        res = ResultW() if w else Result()
         e = U64_MAX if end is None else int(end)
-        self._check(lib.autopipe_search_optimum(self._h, s_min, s_max, flags, int(begin), e,
-                                                ctypes.byref(res), self._stream(stream)))
+        fn = lib.autopipe_search_optimum_w if w else lib.autopipe_search_optimum
+        self._check(fn(self._h, s_min, s_max, flags, int(begin), e, ctypes.byref(res), self._stream(stream)))
         return SearchResult(int(res.time_ns), int(res.index), int(res.evaluated), record_bytes(res.part))
 
     # -- NEXT row f1: the two-worker neighbourhood (PAPER.md:896-906) ------------------------
@@ -236,9 +248,11 @@ class Engine:
         self._check(lib.autopipe_count_candidates(self._h, s_min, s_max, flags, ctypes.byref(v)))
         return int(v.value)
 
-    def decode_index(self, s_min: int, s_max: int, flags: int, index: int) -> bytes:
-        p = Partition()
-        self._check(lib.autopipe_decode_index(self._h, s_min, s_max, flags, int(index), ctypes.byref(p)))
+    def decode_index(self, s_min: int, s_max: int, flags: int, index: int, wide: Optional[bool] = None) -> bytes:
+        w = self._wide(s_max, wide)
+        p = PartitionW() if w else Partition()
+        fn = lib.autopipe_decode_index_w if w else lib.autopipe_decode_index
+        self._check(fn(self._h, s_min, s_max, flags, int(index), ctypes.byref(p)))
         return record_bytes(p)
 
     @property
