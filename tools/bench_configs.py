@@ -130,6 +130,24 @@ def measure(device: int = 0, rollout_records: int = 1 << 20):
         f3[label] = {"records": rollout_records, "ms": ms, "records_per_s": rollout_records / (ms / 1e3)}
     eng.set_schedule()
     res["F3_schedules_bert24_M8"] = dict(candidates=n, **f3)
+    # f4: the paper's 10-GPU testbed (wide records): exhaustive S <= 10 search of VGG-16 and
+    # ResNet-50 on 10 heterogeneous workers, and 1M wide rollout records (S <= 10)
+    f4 = {}
+    for name in ("vgg16", "resnet50"):
+        prof = W.profile(name)
+        st = W.testbed_state(prof, seed=10)
+        eng.load(prof, st)
+        n = eng.count_candidates(1, 10)
+        ms, r = _timed(lambda: eng.search_optimum(1, 10), reps=3, warm=1)
+        f4["search_" + name] = {"candidates": n, "ms_to_optimum": ms, "evals_per_s": n / (ms / 1e3),
+                                "optimum_T_ns": r.time_ns, "stages": r.partition[0]}
+    prof = W.resnet50()
+    st = W.testbed_state(prof, seed=10)
+    eng.load(prof, st)
+    wrecs = torch.from_numpy(W.sample_records(prof.L, 10, rollout_records, 1010, s_max=10, wide=True)).cuda()
+    ms, _ = _timed(lambda: eng.eval_partitions(wrecs, out=out_t))
+    f4["eval_wide_resnet50"] = {"records": rollout_records, "ms": ms, "records_per_s": rollout_records / (ms / 1e3)}
+    res["F4_testbed10"] = f4
     eng.close()
     return res
 
