@@ -47,6 +47,11 @@ struct autopipe_ctx {
   ResultDev *h_result = nullptr;
   u64 *h_status = nullptr;   // pinned copy of the device status word
   u64 binom[BINOM_N][BINOM_K];
+  // the search's kernels (one or two per S) run on NAUX internal streams, forked from and joined back
+  // into the caller's stream: a short model's space is a dozen small launches, latency-bound in series
+  static const int NAUX = 4;
+  cudaStream_t aux[NAUX] = {nullptr, nullptr, nullptr, nullptr};
+  cudaEvent_t ev_fork = nullptr, ev_join[NAUX] = {nullptr, nullptr, nullptr, nullptr};
   // optional device timing of the search kernels (autopipe_set_timing)
   bool timing = false;
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
@@ -182,6 +187,11 @@ extern "C" void autopipe_destroy(autopipe_ctx *c) {
     if (c->h_status) cudaFreeHost(c->h_status);
     if (c->ev0) cudaEventDestroy(c->ev0);
     if (c->ev1) cudaEventDestroy(c->ev1);
+    for (int i = 0; i < autopipe_ctx::NAUX; ++i) {
+      if (c->aux[i]) cudaStreamDestroy(c->aux[i]);
+      if (c->ev_join[i]) cudaEventDestroy(c->ev_join[i]);
+    }
+    if (c->ev_fork) cudaEventDestroy(c->ev_fork);
   }
   delete c;
 }
@@ -520,9 +530,35 @@ static int search_impl(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, u64 beg
   if (rc) return rc;
   rc = check_model(c, st);
   if (rc) return rc;
+  if (!c->ev_fork) {  // internal streams and events, created once
+    cudaError_t e = cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming);
+    for (int i = 0; i < autopipe_ctx::NAUX && e == cudaSuccess; ++i) {
+      e = cudaStreamCreateWithFlags(&c->aux[i], cudaStreamNonBlocking);
+      if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_join[i], cudaEventDisableTiming);
+    }
+    if (e != cudaSuccess) return cuda_fail(c, e, "search streams");
+  }
   if (c->timing) cudaEventRecord(c->ev0, st);
-  int used = 0;
-  // Split [begin, end) into the r = 1 block of each S (rho = 0: fast kernel) and the rest (generic).
+  int used = 0, nlaunch = 0;
+  bool forked = false;
+  auto next_stream = [&]() -> cudaStream_t {  // fork on first use, then round-robin
+    if (!forked) {
+      cudaEventRecord(c->ev_fork, st);
+      for (int i = 0; i < autopipe_ctx::NAUX; ++i) cudaStreamWaitEvent(c->aux[i], c->ev_fork, 0);
+      forked = true;
+    }
+    return c->aux[(nlaunch++) % autopipe_ctx::NAUX];
+  };
+  auto join = [&]() {
+    if (!forked) return;
+    for (int i = 0; i < autopipe_ctx::NAUX; ++i) {
+      cudaEventRecord(c->ev_join[i], c->aux[i]);
+      cudaStreamWaitEvent(st, c->ev_join[i], 0);
+    }
+    forked = false;
+  };
+  // Split [begin, end) into the r = 1 block of each S (rho = 0: fast kernel) and the rest (generic);
+  // the pieces write disjoint block-result ranges and run concurrently.
   u64 cur = begin;
   for (int S = (int)s_min; S <= (int)s_max && cur < end; ++S) {
     const u64 blo = sp.off[S], bhi = sp.off[S + 1];
@@ -538,26 +574,28 @@ static int search_impl(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, u64 beg
       const u64 a = lo, b = hi < r1hi ? hi : r1hi;
       int nb = 0;
       c->launches += launch_search_r1(c->tab, sp, S, a - blo, b - blo, c->path32, c->sms, c->d_blocks + used,
-                                      MAX_BLOCKS - used, &nb, c->d_work, c->h_work, c->work_bytes, st);
+                                      MAX_BLOCKS - used, &nb, c->d_work, c->h_work, c->work_bytes, next_stream());
       used += nb;
       if (b < hi) {
-        c->launches += launch_search_generic(c->tab, sp, b, hi, c->path32, c->model, wide, c->sms, c->d_blocks + used, MAX_BLOCKS - used,
-                                             &nb, st);
+        c->launches += launch_search_generic(c->tab, sp, b, hi, c->path32, c->model, wide, c->sms, c->d_blocks + used,
+                                             MAX_BLOCKS - used, &nb, next_stream());
         used += nb;
       }
     } else {
       int nb = 0;
-      c->launches += launch_search_generic(c->tab, sp, lo, hi, c->path32, c->model, wide, c->sms, c->d_blocks + used, MAX_BLOCKS - used,
-                                           &nb, st);
+      c->launches += launch_search_generic(c->tab, sp, lo, hi, c->path32, c->model, wide, c->sms, c->d_blocks + used,
+                                           MAX_BLOCKS - used, &nb, next_stream());
       used += nb;
     }
     cur = hi;
     if (used > MAX_BLOCKS - 4 * c->sms) {  // keep room: fold what we have into one entry
+      join();
       c->launches += launch_finalize(c->d_blocks, used, sp, c->d_result, wide, st);
       cudaMemcpyAsync(c->d_blocks, c->d_result, sizeof(BlockOut), cudaMemcpyDeviceToDevice, st);
       used = 1;
     }
   }
+  join();
   if (c->timing) cudaEventRecord(c->ev1, st);
   if (getenv("AUTOPIPE_R1_STATS") && used > 0) {  // diagnostics: rare-path decisions per search
     BlockOut *hb = new BlockOut[used];

@@ -150,7 +150,8 @@ int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, 
   const u64 span = end - begin;
   // at least 4 candidates per thread (the unrank is a few binary searches); up to 8 blocks per SM.
   // A flushed schedule costs ~M S stage steps per candidate: one candidate per thread is enough.
-  const u64 min_per = (m.sched == SCHED_GPIPE || m.sched == SCHED_DAPPLE) ? 1 : 4;
+  // A small span (a launch of a short model's space) is latency-bound: one candidate per thread.
+  const u64 min_per = (m.sched == SCHED_GPIPE || m.sched == SCHED_DAPPLE || span <= (u64)sms * 8 * NT * 4) ? 1 : 4;
   u64 threads = (span + min_per - 1) / min_per;
   u64 blocks = (threads + NT - 1) / NT;
   const u64 cap = (u64)sms * 8 < (u64)max_blocks ? (u64)sms * 8 : (u64)max_blocks;

@@ -661,7 +661,13 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
   static const u64 tpw = env_u64("AUTOPIPE_R1_TPW", 30), min_target = env_u64("AUTOPIPE_R1_MINTARGET", 12000);
   const u64 lane_tasks = (u64)sms * 16 * 32 * tpw;
   u64 TARGET = total_cost / (lane_tasks ? lane_tasks : 1);
-  if (TARGET < min_target) TARGET = min_target;
+  // Floor on the task size: 12,000 amortises the per-task unrank and seed, but a small space (a
+  // 21-26-layer model) would then be a handful of tasks on 2-6 blocks, latency-bound for 100-300 us.
+  // Small spaces get tasks sized to give every resident warp slot about two (floor 300).
+  u64 floor_t = min_target;
+  const u64 fill = total_cost / ((u64)sms * 16 * 32 * 2);
+  if (fill < floor_t) floor_t = fill > 300 ? fill : 300;
+  if (TARGET < floor_t) TARGET = floor_t;
   // Guided sizes: warps take tasks in schedule order, so the kernel ends about one task length after
   // the last task starts. Tasks in the final 15 % of the cost shrink linearly to 1/4 of the target
   // (smaller ones pay more per-task overhead than they save in tail; measured on B200).
