@@ -241,11 +241,20 @@ def main():
     import workloads as W
     from paper_conf_icpp_hulww24_b200 import Engine
 
+    # AUTOPIPE_BENCH_BACKEND=gloo (test only): ranks may share a GPU (rank -> cuda:rank % count) so the
+    # multi-rank path (shards, min-loc, max-over-ranks timing, one JSON line) runs on a 1-GPU box.
+    # Its numbers are not scaling numbers; the driver's runs use NCCL, one GPU per rank.
+    backend = os.environ.get("AUTOPIPE_BENCH_BACKEND", "nccl")
+    if backend == "gloo":
+        local = local % max(torch.cuda.device_count(), 1)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "gloo":
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
     # contiguous shards of about equal device cost (host-only estimate; any split gives the same optimum)
     from paper_conf_icpp_hulww24_b200.distributed import balanced_bounds
     bounds = balanced_bounds(96, 8, S_STAGES, S_STAGES, 0, world)
@@ -261,7 +270,10 @@ def main():
 
     def barrier():
         if world > 1:
-            dist.barrier(device_ids=[local])
+            if backend == "gloo":
+                dist.barrier()
+            else:
+                dist.barrier(device_ids=[local])
 
     def max_over_ranks(x: float) -> float:
         if world == 1:
