@@ -178,17 +178,20 @@ __device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, const P
   static_assert(!(P32 && BW), "the 2BW form is 64-bit");
   constexpr int MS = P::MS;
   typedef typename std::conditional<P32, u32, u64>::type V;
-  V X[MS], Y[MS], Zb[MS];
+  // One pass over the stages u = 0..S-1. After stage u, acc[s] (s <= u) = X_s + sum_{s<v<=u} Y_v +
+  // sum_{s<=v<u} Z_v, so the segment (s, u) is W(s,u) = acc[s] (before adding stage u's Y) + Z_{u-1}
+  // + X_u: one running sum per open segment start instead of the three per-stage arrays (the wide
+  // 16-stage form keeps its registers).
+  V acc[MS];
   V T = 0;
   u64 TAR = 0;
 #pragma unroll
-  for (int s = 0; s < MS; ++s) {
-    X[s] = 0;
-    Y[s] = 0;
-    if (s < S) {
-      const int a = (s == 0) ? 0 : p.cut(s - 1) + 1;
-      const int e = (s == S - 1) ? t.L - 1 : p.cut(s);
-      const u32 mask = p.mask(s);
+  for (int u = 0; u < MS; ++u) {
+    acc[u] = 0;
+    if (u < S) {
+      const int a = (u == 0) ? 0 : p.cut(u - 1) + 1;
+      const int e = (u == S - 1) ? t.L - 1 : p.cut(u);
+      const u32 mask = p.mask(u);
       const u32 r = __popc(mask);
       const DivR<P::MN> dv(r);
       u32 m = mask;
@@ -207,40 +210,29 @@ __device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, const P
         bm = umax(bm, B);
         xm = umax(xm, F + B);
       }
-      X[s] = (V)xm;
-      Y[s] = (V)(fm + bm);
+      const V X = (V)xm, Y = (V)(fm + bm);
       const V xs = BW ? (V)(xm * M) : (V)xm;
       T = T > xs ? T : xs;
       if (r >= 2) TAR = umax(TAR, sync_time<P::MN>(sync, t.PP[e + 1] - t.PP[a], mask, t.tau));
-    }
-  }
+      if (u > 0) {
+        // row a5: boundary u-1 (activation O[e_{u-1}] forward, gradient G[e_{u-1}+1] backward)
+        const int eb = p.cut(u - 1);
+        const u32 mp = p.mask(u - 1);
+        const u64 cf = boundary_max<P::MN>(t.O[eb], mp, mask, t.tau);
+        const u64 cb = boundary_max<P::MN>(t.G[eb + 1], mask, mp, t.tau);
+        const V Z = (V)(cf + cb);
+        const V lm = BW ? (V)(umax(cf, cb) * M) : (V)umax(cf, cb);
+        T = T > lm ? T : lm;
+        // row a7: the segment cycles ending at stage u, u-s+1 tokens
 #pragma unroll
-  for (int s = 0; s < MS - 1; ++s) {  // row a5
-    Zb[s] = 0;
-    if (s < S - 1) {
-      const int e = p.cut(s);
-      const u32 ms = p.mask(s), mn = p.mask(s + 1);
-      const u64 cf = boundary_max<P::MN>(t.O[e], ms, mn, t.tau);
-      const u64 cb = boundary_max<P::MN>(t.G[e + 1], mn, ms, t.tau);
-      Zb[s] = (V)(cf + cb);
-      const V lm = BW ? (V)(umax(cf, cb) * M) : (V)umax(cf, cb);
-      T = T > lm ? T : lm;
-    }
-  }
-  Zb[MS - 1] = 0;
-#pragma unroll
-  for (int s = 0; s < MS - 1; ++s) {  // row a7: segment cycles, t-s+1 tokens
-    if (s < S - 1) {
-      V acc = X[s];
-#pragma unroll
-      for (int u = s + 1; u < MS; ++u) {
-        if (u < S) {
-          const V W = BW ? (acc + Zb[u - 1] + X[u]) * M : acc + Zb[u - 1] + X[u];
+        for (int s = 0; s < u; ++s) {
+          const V W = BW ? (acc[s] + Z + X) * M : acc[s] + Z + X;
           const V c = (W + (V)(u - s)) / (V)(u - s + 1);
           T = T > c ? T : c;
-          acc += Zb[u - 1] + Y[u];
+          acc[s] += Z + Y;
         }
       }
+      acc[u] = X;
     }
   }
   return umax((u64)T, TAR);
