@@ -41,6 +41,14 @@ constexpr int R1_MAXCHUNK = 16;
 #ifndef R1_NX
 #define R1_NX 2
 #endif
+// aligned 4-column groups in the sweep body (128-bit shared loads)
+#ifndef R1_V4
+#define R1_V4 1
+#endif
+// two groups (8 columns) per step of the scan loop
+#ifndef R1_G8
+#define R1_G8 1
+#endif
 // resident blocks per SM the register budget is sized for (__launch_bounds__ min blocks), per path:
 // 3 x 256 threads for the 32-bit tables (85 registers, no spills; 3.47 -> 3.30 ms for C(95,7) on
 // B200), 2 for the 64-bit ones (3 spills and runs slower)
@@ -204,6 +212,14 @@ __device__ __forceinline__ T thr(i64 h, bool alive) {
 // fit), and every candidate that passes it is re-checked in full (A, K, V) before its exact T.
 __device__ __forceinline__ void lds_fold1(unsigned a, u32 &A) { asm("ld.shared.u32 %0, [%1];" : "=r"(A) : "r"(a)); }
 __device__ __forceinline__ void lds_fold1(unsigned a, u64 &A) { asm("ld.shared.u64 %0, [%1];" : "=l"(A) : "r"(a)); }
+// four consecutive folded columns from a 16-byte-aligned address (32 bytes for 64-bit tables)
+__device__ __forceinline__ void lds_group4(unsigned a, u32 (&A)[4]) {
+  asm("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(A[0]), "=r"(A[1]), "=r"(A[2]), "=r"(A[3]) : "r"(a));
+}
+__device__ __forceinline__ void lds_group4(unsigned a, u64 (&A)[4]) {
+  asm("ld.shared.v2.u64 {%0, %1}, [%2];" : "=l"(A[0]), "=l"(A[1]) : "r"(a));
+  asm("ld.shared.v2.u64 {%0, %1}, [%2+16];" : "=l"(A[2]), "=l"(A[3]) : "r"(a));
+}
 __device__ __forceinline__ u32 warp_max_T(u32 v) { return __reduce_max_sync(0xffffffffu, v); }
 __device__ __forceinline__ u64 warp_max_T(u64 v) {
 #pragma unroll
@@ -392,30 +408,39 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? R1_MINB32 : R1_MINB64) k_
       const u64 first = pre | ((u64)y << (8 * P)) | ((u64)xa << (8 * (P + 1))) | ((u64)(xa + 1) << (8 * (P + 2)));
       strict = hdr.off + lex_rank_smem(first, S - 1, n, Bn) > bestI;
     }
+    // evaluated candidates of this task: the (x, e) pairs y < x < e <= L-2 of the x chunk in each of
+    // the lane's rows, restricted on the shard's first / last row (at most one of each per shard:
+    // the lo row is row_begin of y = lo_y, the hi row is row_end - 1 of y = hi_y)
+    const bool task_lo = r0 < r1 && y == hdr.lo_y && r0 == ye.row_begin;
+    const bool task_hi = r0 < r1 && y == hdr.hi_y && r1 == ye.row_end;
+    if (r0 < r1) {
+      // rank of the pair (x, e) among the row's pairs (closed form)
+      auto prank = [&](int x, int e) -> u64 {
+        const u64 a = (u64)(x - y - 1), m1 = (u64)(L - 3 - y);  // m1 = pairs with x = y + 1
+        return a * m1 - a * (a - 1) / 2 + (u64)(e - x - 1);
+      };
+      const u64 flo = prank(xa, xa + 1), fhi = prank(xb, xb + 1);  // this task's x chunk
+      const u64 lo1 = task_lo ? umax(flo, prank(hdr.lo_x, hdr.lo_e)) : flo;
+      const u64 hi1 = task_hi ? umin(fhi, prank(hdr.hi_x, hdr.hi_e) + 1) : fhi;
+      const u64 full = fhi - flo, nrows = r1 - r0;
+      if (nrows == 1) {
+        cnt += hi1 > lo1 ? hi1 - lo1 : 0ull;
+      } else {
+        cnt += (nrows - 2) * full + (fhi > lo1 ? fhi - lo1 : 0ull) + (hi1 > flo ? hi1 - flo : 0ull);
+      }
+    }
     RowBase base;
     bool need_base = true;
     for (u64 row = r0;; ++row) {
       const bool active = row < r1;
       if (!__any_sync(0xffffffffu, active)) break;
       // partial rows at the shard boundaries: (x, e) range restricted, checked on the rare path
-      bool lo_part = false, hi_part = false;
+      const bool lo_part = task_lo && row == r0, hi_part = task_hi && row + 1 == r1;
       i64 th = (bestT == U64MAX) ? THETA_ALL : (i64)bestT - (strict ? 1 : 0);
       if (thg < th) th = thg;
       bool aliveP = false;
       i64 N0 = 0, N1 = 0, N2 = 0;
       if (active) {
-        lo_part = (pre == hdr.lo_pre) && (y == hdr.lo_y);
-        hi_part = (pre == hdr.hi_pre) && (y == hdr.hi_y);
-        // evaluated candidates of this row: the (x, e) pairs y < x < e <= L-2 within the shard
-        // rank of the pair (x, e) among the row's pairs y < x < e <= L-2 (closed form)
-        auto prank = [&](int x, int e) -> u64 {
-          const u64 a = (u64)(x - y - 1), m1 = (u64)(L - 3 - y);  // m1 = pairs with x = y + 1
-          return a * m1 - a * (a - 1) / 2 + (u64)(e - x - 1);
-        };
-        u64 rlo = prank(xa, xa + 1), rhi = prank(xb, xb + 1);  // this task's x chunk
-        if (lo_part) rlo = umax(rlo, prank(hdr.lo_x, hdr.lo_e));
-        if (hi_part) rhi = umin(rhi, prank(hdr.hi_x, hdr.hi_e) + 1);
-        cnt += rhi > rlo ? rhi - rlo : 0ull;
         if (need_base) row_base<S>(PC, Z, LM, L, pre, th, base);
         aliveP = row_finish<S>(base, PC, Z, LM, L, byte_at(pre, P - 1), y, th, N0, N1, N2);
       }
@@ -512,28 +537,109 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? R1_MINB32 : R1_MINB64) k_
               if (first[k] == cend && A0 < H1[k]) first[k] = c;
           }
         }
-        // body: every column from x+NX on belongs to every x of the pass (4 columns per step; the
-        // sentinel columns past L-2 never pass)
-        for (unsigned a = fb + (unsigned)(x + NX) * FS; a < aend; a += 4 * FS) {
-          T A4[4];
+        // 64-bit tables: every column from x+NX on belongs to every x of the pass (4 columns per step,
+        // four 64-bit loads; the sentinel columns past L-2 never pass)
+        auto body64 = [&]() {
+          for (unsigned a = fb + (unsigned)(x + NX) * FS; a < aend; a += 4 * FS) {
+            T A4[4];
 #pragma unroll
-          for (int u = 0; u < 4; ++u) lds_fold1(a + u * FS, A4[u]);
-          bool h[NX];
+            for (int u = 0; u < 4; ++u) lds_fold1(a + u * FS, A4[u]);
+            bool h[NX];
 #pragma unroll
-          for (int k = 0; k < NX; ++k) h[k] = (A4[0] < H1[k]) | (A4[1] < H1[k]) | (A4[2] < H1[k]) | (A4[3] < H1[k]);
-          bool any = h[0];
+            for (int k = 0; k < NX; ++k) h[k] = (A4[0] < H1[k]) | (A4[1] < H1[k]) | (A4[2] < H1[k]) | (A4[3] < H1[k]);
+            bool any = h[0];
 #pragma unroll
-          for (int k = 1; k < NX; ++k) any |= h[k];
-          if (any) {
-            const int c = (int)((a - fb) / FS);
-            if (h[0])
+            for (int k = 1; k < NX; ++k) any |= h[k];
+            if (any) {
+              const int c = (int)((a - fb) / FS);
+              if (h[0])
+                for (int u = 0; u < 4; ++u)
+                  if (A4[u] < H1[0] && rare(x, c + u, H1[0])) refresh();
+#pragma unroll
+              for (int k = 1; k < NX; ++k)
+                if (h[k] && first[k] == cend) first[k] = c;
+            }
+          }
+        };
+#if R1_V4
+        // body: every column from cs = x+NX on belongs to every x of the pass. Columns go in aligned
+        // groups of 4 (one 128-bit shared load on the 32-bit path); the first group starts at cs
+        // rounded down, its columns below cs masked to MAX; the sentinel columns past L-2 never pass.
+        // The scan loop only tests the group's minimum against Hm, the largest threshold still
+        // live (H1[0], and H1[k] of a later x until its first hit is recorded): one compare per group
+        // and no branch into the hit code until something passes.
+        const int cs = x + NX;
+        if constexpr (sizeof(T) != 4) {
+          body64();
+        } else if (cs < cend) {
+          T Hm;
+          auto set_hm = [&]() {
+            Hm = H1[0];
+#pragma unroll
+            for (int k = 1; k < NX; ++k)
+              if (first[k] == cend && H1[k] > Hm) Hm = H1[k];
+          };
+          set_hm();
+          auto group = [&](unsigned o, const T (&A4)[4]) {
+            const int c = (int)(o / FS);
+            if ((A4[0] < H1[0]) | (A4[1] < H1[0]) | (A4[2] < H1[0]) | (A4[3] < H1[0]))
               for (int u = 0; u < 4; ++u)
                 if (A4[u] < H1[0] && rare(x, c + u, H1[0])) refresh();
 #pragma unroll
             for (int k = 1; k < NX; ++k)
-              if (h[k] && first[k] == cend) first[k] = c;
+              if (first[k] == cend && ((A4[0] < H1[k]) | (A4[1] < H1[k]) | (A4[2] < H1[k]) | (A4[3] < H1[k])))
+                first[k] = c > cs ? c : cs;
+            set_hm();
+          };
+          const unsigned oend = (unsigned)cend * FS;
+          unsigned o = (unsigned)(cs & ~3) * FS;
+          T A4[4];
+          lds_group4(fb + o, A4);
+          {
+            const int d = cs & 3;
+            if (d > 0) A4[0] = (T)~(T)0;
+            if (d > 1) A4[1] = (T)~(T)0;
+            if (d > 2) A4[2] = (T)~(T)0;
+          }
+          for (;;) {
+            if (min(min(A4[0], A4[1]), min(A4[2], A4[3])) < Hm) group(o, A4);
+            o += 4 * FS;
+            if (o >= oend) break;
+            // tight scan to the next group with a column below Hm
+#if R1_G8
+            // (two groups per step: one compare per 8 columns; the sentinels cover the overrun)
+            T B4[4];
+            bool hitb = false;
+            for (;;) {
+              lds_group4(fb + o, A4);
+              lds_group4(fb + o + 4 * FS, B4);
+              if (min(min(min(A4[0], A4[1]), min(A4[2], A4[3])), min(min(B4[0], B4[1]), min(B4[2], B4[3]))) < Hm) {
+                hitb = true;
+                break;
+              }
+              o += 8 * FS;
+              if (o >= oend) break;
+            }
+            if (!hitb) break;
+            if (min(min(A4[0], A4[1]), min(A4[2], A4[3])) < Hm) group(o, A4);
+            o += 4 * FS;
+            if (o >= oend) break;
+#pragma unroll
+            for (int u = 0; u < 4; ++u) A4[u] = B4[u];
+#else
+            for (;;) {
+              lds_group4(fb + o, A4);
+              if (min(min(A4[0], A4[1]), min(A4[2], A4[3])) < Hm) break;
+              o += 4 * FS;
+              if (o >= oend) break;
+            }
+            if (o >= oend) break;
+#endif
           }
         }
+#else
+        body64();
+#endif
 #pragma unroll
         for (int k = 1; k < NX; ++k)
           if (first[k] < cend) sweep1(x + k, first[k]);
