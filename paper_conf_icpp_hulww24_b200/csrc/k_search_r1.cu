@@ -23,9 +23,10 @@
 // Mapping (the B200 part). Cut sets are (prefix e_0..e_{S-5}, y = e_{S-4}, x = e_{S-3}, e = e_{S-2}).
 // A warp task fixes y; its 32 lanes take different prefixes (R consecutive ones each). So within a
 // warp, x and e run in lockstep and everything that depends on x or e only is warp-uniform: the
-// x-level update is a broadcast load plus ~20 integer ops per lane, the column sweep is one
-// broadcast 128-bit shared-memory load and three compares per column per lane, and there is no
-// divergence in the hot loop. A lane re-derives its prefix terms (O(S^2)) once per row; a row covers
+// x-level update is a broadcast load plus ~20 integer ops per lane, the column sweep reads a
+// warp-private folded table with broadcast 128-bit shared-memory loads (8 columns, two x values,
+// one compare of their minimum per step on the 32-bit path), and there is no divergence in the hot
+// loop. A lane re-derives its prefix terms (O(S^2)) once per row; a row covers
 // C(L-2-y, 2) candidates. Warps take tasks from a global atomic counter (persistent grid); the
 // (T, index) argmin goes lane -> warp -> block (shuffles + shared memory) -> grid (k_finalize), so the
 // result is the lexicographic (T, index) minimum whatever the task order, grid or GPU count.
@@ -52,6 +53,13 @@ constexpr int R1_MAXCHUNK = 16;
 // resident blocks per SM the register budget is sized for (__launch_bounds__ min blocks), per path:
 // 3 x 256 threads for the 32-bit tables (85 registers, no spills; 3.47 -> 3.30 ms for C(95,7) on
 // B200), 2 for the 64-bit ones (3 spills and runs slower)
+// threads per block, per path
+#ifndef R1_NT32
+#define R1_NT32 256
+#endif
+#ifndef R1_NT64
+#define R1_NT64 256
+#endif
 #ifndef R1_MINB32
 #define R1_MINB32 3
 #endif
@@ -724,7 +732,7 @@ template <int S, typename T>
 static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u64 k_end, int sms,
                        BlockOut *out, int max_blocks, int *nblocks, void *work, void *pinned, size_t work_bytes,
                        cudaStream_t st) {
-  constexpr int P = S - 4, NT = 256;
+  constexpr int P = S - 4, NT = sizeof(T) == 4 ? R1_NT32 : R1_NT64;
   const int L = (int)g.L, n = L - 1, k = S - 1;
   init_hb();
   int lo[8], hi[8];
