@@ -260,13 +260,8 @@ def main():
     bounds = balanced_bounds(96, 8, S_STAGES, S_STAGES, 0, world)
     lo, hi = bounds[rank], bounds[rank + 1]
 
-    from paper_conf_icpp_hulww24_b200.distributed import minloc as dist_minloc
-
-    def minloc(T, idx):
-        if world == 1:
-            return T, idx
-        Tm, Im, _ = dist_minloc(T, idx, 0, device=dev)   # NCCL all_reduce(MIN) x2 (+ SUM)
-        return Tm, Im
+    from paper_conf_icpp_hulww24_b200 import result_from_bytes
+    from paper_conf_icpp_hulww24_b200.distributed import minloc_device
 
     def barrier():
         if world > 1:
@@ -295,35 +290,43 @@ def main():
         stream = torch.cuda.current_stream(dev)
 
         def step():
+            # a1-a8 + e, all enqueued on the stream with no host wait: state kernel, the shard's
+            # asynchronous search (result stays in device memory), and for N > 1 the device min-loc
+            # (one NCCL all-gather of 40 B per rank + one reduction kernel)
             eng.set_state_device(d_fp, d_bp, d_tau)
-            r = eng.search_optimum(S_STAGES, S_STAGES, 0, lo, hi)
-            return r, minloc(r.time_ns, r.index)
+            r = eng.search_optimum_async(S_STAGES, S_STAGES, 0, lo, hi)
+            return minloc_device(r) if world > 1 else r
 
         for _ in range(args.warmup):
             step()
         torch.cuda.synchronize()
         barrier()
+        eng.search_times()                         # drain the warm-up searches' kernel times
         launches0 = eng.kernel_launches
         ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-        kern_ms, results = [], []
+        outs = []
         with ClockSampler(local) as clk:
             for k in range(args.steps):
-                flush.fill_(k)                     # L2 flush, outside the timed events
-                torch.cuda.synchronize()
+                flush.fill_(k)                     # L2 flush: enqueued before the step's start event
                 ev[k][0].record(stream)
-                r, best = step()
+                outs.append(step())
                 ev[k][1].record(stream)
-                kern_ms.append(eng.last_search_ms)
-                results.append(best)
             torch.cuda.synchronize()
         barrier()
-        launches = eng.kernel_launches - launches0
+        # this library's kernels in the timed region: the context's (state, both gated search paths,
+        # finalize) + the context-less min-loc reduction (one per step when N > 1)
+        launches = eng.kernel_launches - launches0 + (args.steps if world > 1 else 0)
+        kern_ms = eng.search_times()               # the K searches' enumeration kernels (CUDA events)
+        assert len(kern_ms) == args.steps
         step_ms = [a.elapsed_time(b) for a, b in ev]
         rank_total_ms = sum(step_ms)
         total_ms = max_over_ranks(rank_total_ms)
         kern_avg = max_over_ranks(sum(kern_ms) / len(kern_ms))
+        results = [(r.time_ns, r.index) for r in map(result_from_bytes, outs)]
         assert all(x == results[0] for x in results), "non-deterministic optimum"
-        # e2e: the public API from host buffers (profile + state copied every step, result to host)
+        assert all(result_from_bytes(o).evaluated == (TOTAL if world > 1 else hi - lo) for o in outs)
+        # e2e: the public API from host buffers (profile + state copied every step, the 40-byte
+        # result read back to the host)
         t_e2e = []
         for k in range(args.steps):
             flush.fill_(k)
@@ -332,11 +335,10 @@ def main():
             t0 = time.perf_counter()
             eng.load_profile(prof.O, prof.G, prof.P)
             eng.set_state(st.f, st.b, st.tau)
-            r = eng.search_optimum(S_STAGES, S_STAGES, 0, lo, hi)
-            best_e2e = minloc(r.time_ns, r.index)
-            torch.cuda.synchronize()
+            r = eng.search_optimum_async(S_STAGES, S_STAGES, 0, lo, hi)
+            best = result_from_bytes(minloc_device(r) if world > 1 else r)
             t_e2e.append(time.perf_counter() - t0)
-        assert best_e2e == results[0]
+            assert (best.time_ns, best.index) == results[0]
         e2e_s = max_over_ranks(sum(t_e2e))
         int_path = eng.int_path
         eng.close()

@@ -144,6 +144,26 @@ int autopipe_eval_partitions(autopipe_ctx *ctx, const autopipe_partition *d_part
 int autopipe_search_optimum(autopipe_ctx *ctx, uint32_t s_min, uint32_t s_max, uint32_t flags,
                             uint64_t begin, uint64_t end, autopipe_result *h_out, void *stream);
 
+/* The same search, asynchronous: the result is written to the DEVICE struct *d_out on `stream` and
+ * the call returns once the kernels are enqueued (it waits for the device only when the context's
+ * previous search has not yet consumed its schedule copy, and for a schedule other than PipeDream
+ * whose state was set from device memory). For a state set with autopipe_set_state_device the host
+ * does not read the state back: the kernels of both integer paths are enqueued and each runs only if
+ * the state kernel chose its path, so an overflowing device state yields evaluated = 0 and
+ * time_ns = index = UINT64_MAX for a non-empty shard (the next synchronous call reports
+ * E_OVERFLOW). An empty shard writes (UINT64_MAX, UINT64_MAX, 0, 0xFF...). The context's scratch is
+ * shared by its calls: issue a context's asynchronous searches on one stream (or order them).
+ * This is the per-rank step of the multi-GPU search (row e): gather the ranks' results and reduce
+ * them with autopipe_reduce_results, with no host round trip. */
+int autopipe_search_optimum_async(autopipe_ctx *ctx, uint32_t s_min, uint32_t s_max, uint32_t flags,
+                                  uint64_t begin, uint64_t end, autopipe_result *d_out, void *stream);
+
+/* Row e (north star: "only a tiny NCCL min-loc allreduce"): d_in[n] results (e.g. all-gathered from
+ * the ranks' asynchronous searches; device memory) -> *d_out = their lexicographic (time_ns, index)
+ * minimum, evaluated = the sum, the record of the winner (on exact ties, the lowest entry's). Async on
+ * `stream`; one warp. n = 0 writes an empty result. Needs no context. */
+int autopipe_reduce_results(const autopipe_result *d_in, uint32_t n, autopipe_result *d_out, void *stream);
+
 /* RL rollout rewards (the arbiter sees the current and the new partition; the
  * reward is one-iteration speed with a switching cost). Device pointers, async on `stream`:
  *   d_parts[count]         proposals; d_time_ns[count] gets T_ns (UINT64_MAX if invalid);
@@ -205,6 +225,9 @@ int autopipe_eval_partitions_w(autopipe_ctx *ctx, const autopipe_partition_w *d_
 int autopipe_rollout_rewards_w(autopipe_ctx *ctx, const autopipe_partition_w *d_parts, uint64_t count,
                                const autopipe_partition_w *h_current, uint64_t *d_time_ns,
                                uint64_t *d_switch_bytes, void *stream);
+int autopipe_search_optimum_async_w(autopipe_ctx *ctx, uint32_t s_min, uint32_t s_max, uint32_t flags,
+                                    uint64_t begin, uint64_t end, autopipe_result_w *d_out, void *stream);
+int autopipe_reduce_results_w(const autopipe_result_w *d_in, uint32_t n, autopipe_result_w *d_out, void *stream);
 int autopipe_search_optimum_w(autopipe_ctx *ctx, uint32_t s_min, uint32_t s_max, uint32_t flags, uint64_t begin,
                               uint64_t end, autopipe_result_w *h_out, void *stream);
 int autopipe_decode_index_w(const autopipe_ctx *ctx, uint32_t s_min, uint32_t s_max, uint32_t flags,
@@ -273,8 +296,14 @@ uint64_t autopipe_kernel_launches(const autopipe_ctx *ctx);
  * reduction and the result copy). */
 int autopipe_set_timing(autopipe_ctx *ctx, int enable);
 
-/* Device milliseconds of the enumeration kernels of the last timed search (-1 if none). */
+/* Device milliseconds of the enumeration kernels of the last timed search (-1 if none); waits for
+ * that search's kernels to finish (an asynchronous search returns before they run). */
 double autopipe_last_search_ms(const autopipe_ctx *ctx);
+
+/* The enumeration-kernel times (ms) of the timed searches issued since the previous call, oldest
+ * first: up to `cap` values into the host array ms[], their number in *count. Waits for those
+ * searches. The context keeps the event pairs of its last 64 timed searches; older ones are lost. */
+int autopipe_search_times(autopipe_ctx *ctx, double *ms, uint32_t cap, uint32_t *count);
 
 #ifdef __cplusplus
 }

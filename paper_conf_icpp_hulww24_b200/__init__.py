@@ -5,6 +5,7 @@ in hand-written sm_100a CUDA kernels behind the C-ABI of include/autopipe.h; thi
 Python binding (``Engine``) plus the multi-GPU driver (``distributed``). There is no CPU fallback.
 """
 from ._lib import AutopipeError, USE_ALL_WORKERS, LIB_PATH  # noqa: F401  (raises if not built)
-from .engine import Engine, SearchResult, U64_MAX, as_u64  # noqa: F401
+from .engine import Engine, SearchResult, U64_MAX, as_u64, reduce_results, result_from_bytes  # noqa: F401
 
-__all__ = ["Engine", "SearchResult", "AutopipeError", "USE_ALL_WORKERS", "U64_MAX", "as_u64", "LIB_PATH"]
+__all__ = ["Engine", "SearchResult", "AutopipeError", "USE_ALL_WORKERS", "U64_MAX", "as_u64", "LIB_PATH",
+           "reduce_results", "result_from_bytes"]

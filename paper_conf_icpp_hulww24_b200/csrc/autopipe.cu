@@ -54,8 +54,15 @@ struct autopipe_ctx {
   cudaEvent_t ev_fork = nullptr, ev_join[NAUX] = {nullptr, nullptr, nullptr, nullptr};
   // optional device timing of the search kernels (autopipe_set_timing)
   bool timing = false;
-  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
-  double last_search_ms = -1.0;
+  // a ring of event pairs: search k (counted while timing is on) records pair k % TRING, so the
+  // times of asynchronous searches can be read after the fact (autopipe_search_times)
+  static const int TRING = 64;
+  cudaEvent_t ev0[TRING] = {}, ev1[TRING] = {};
+  u64 tcount = 0, tread = 0;  // timed searches recorded / already returned by autopipe_search_times
+  // recorded after a search's schedule copies: the pinned schedule slots are rewritten only after it
+  // (an asynchronous search returns before its copies have run)
+  cudaEvent_t ev_hwork = nullptr;
+  bool hwork_pending = false;
 };
 
 static char g_create_err[256] = "";
@@ -185,8 +192,11 @@ extern "C" void autopipe_destroy(autopipe_ctx *c) {
     if (c->h_stage) cudaFreeHost(c->h_stage);
     if (c->h_result) cudaFreeHost(c->h_result);
     if (c->h_status) cudaFreeHost(c->h_status);
-    if (c->ev0) cudaEventDestroy(c->ev0);
-    if (c->ev1) cudaEventDestroy(c->ev1);
+    if (c->ev_hwork) cudaEventDestroy(c->ev_hwork);
+    for (int i = 0; i < autopipe_ctx::TRING; ++i) {
+      if (c->ev0[i]) cudaEventDestroy(c->ev0[i]);
+      if (c->ev1[i]) cudaEventDestroy(c->ev1[i]);
+    }
     for (int i = 0; i < autopipe_ctx::NAUX; ++i) {
       if (c->aux[i]) cudaStreamDestroy(c->aux[i]);
       if (c->ev_join[i]) cudaEventDestroy(c->ev_join[i]);
@@ -507,38 +517,64 @@ extern "C" int autopipe_decode_index_w(const autopipe_ctx *cc, uint32_t s_min, u
 
 // The search of a 16-byte space (wide = false) or a wide one (row f4). Writes time, index, evaluated
 // and the best record (16 or 32 bytes) to the host.
+// d_out != nullptr: the asynchronous form (autopipe_search_optimum_async): the result goes to device
+// memory on `stream`, nothing waits for the device, and a state set from device memory is not read
+// back: the kernels of both integer paths are enqueued and the state kernel's choice gates them.
 static int search_impl(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, u64 begin, u64 end, bool wide,
-                       u64 *h_tie, uint8_t *h_rec, void *stream) {
+                       u64 *h_tie, uint8_t *h_rec, void *stream, void *d_out = nullptr) {
   if (!c) return AUTOPIPE_E_INVAL;
   c->err[0] = 0;
+  const bool async = d_out != nullptr;
   if (!c->has_state) return fail(c, AUTOPIPE_E_STATE, "search before set_state");
-  if (!h_tie || !h_rec) return fail(c, AUTOPIPE_E_INVAL, "NULL result pointer");
+  if (!async && (!h_tie || !h_rec)) return fail(c, AUTOPIPE_E_INVAL, "NULL result pointer");
   int rc = check_space_args(c, s_min, s_max, flags, wide);
   if (rc) return rc;
   SearchSpace sp;
   if (!build_space(c, s_min, s_max, flags, sp)) return fail(c, AUTOPIPE_E_OVERFLOW, "space exceeds 2^64");
   const u64 total = sp.off[s_max + 1];
   if (end > total) end = total;
-  h_tie[0] = U64MAX;
-  h_tie[1] = U64MAX;
-  h_tie[2] = 0;
-  memset(h_rec, 0xFF, wide ? 32 : 16);
-  if (begin >= end) return AUTOPIPE_OK;
+  const int rec_bytes = wide ? 32 : 16;
   DeviceGuard dg(c->device);
   cudaStream_t st = (cudaStream_t)stream;
-  rc = sync_status(c, st);
-  if (rc) return rc;
-  rc = check_model(c, st);
-  if (rc) return rc;
+  if (!async) {
+    h_tie[0] = U64MAX;
+    h_tie[1] = U64MAX;
+    h_tie[2] = 0;
+    memset(h_rec, 0xFF, rec_bytes);
+  }
+  if (begin >= end) {
+    if (async) {  // an empty shard: (UINT64_MAX, UINT64_MAX, 0, record of 0xFF)
+      cudaMemsetAsync(d_out, 0xFF, 24 + rec_bytes, st);
+      cudaMemsetAsync((unsigned char *)d_out + 16, 0, 8, st);
+    }
+    return AUTOPIPE_OK;
+  }
+  // the integer path: known on the host, or (async search of a device state) chosen on the device
+  int path = c->path32;
+  if (async && c->state_on_device && c->model.sched == SCHED_PIPEDREAM) {
+    path = -1;
+  } else {
+    rc = sync_status(c, st);
+    if (rc) return rc;
+    rc = check_model(c, st);
+    if (rc) return rc;
+    path = c->path32;
+  }
+  if (c->hwork_pending) {  // the pinned schedule slots may still feed the previous search's copies
+    cudaEventSynchronize(c->ev_hwork);
+    c->hwork_pending = false;
+  }
   if (!c->ev_fork) {  // internal streams and events, created once
-    cudaError_t e = cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming);
+    cudaError_t e = cudaEventCreateWithFlags(&c->ev_hwork, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming);
     for (int i = 0; i < autopipe_ctx::NAUX && e == cudaSuccess; ++i) {
       e = cudaStreamCreateWithFlags(&c->aux[i], cudaStreamNonBlocking);
       if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_join[i], cudaEventDisableTiming);
     }
     if (e != cudaSuccess) return cuda_fail(c, e, "search streams");
   }
-  if (c->timing) cudaEventRecord(c->ev0, st);
+  const int tslot = (int)(c->tcount % autopipe_ctx::TRING);
+  if (c->timing) cudaEventRecord(c->ev0[tslot], st);
   int used = 0, nlaunch = 0;
   bool forked = false;
   auto next_stream = [&]() -> cudaStream_t {  // fork on first use, then round-robin
@@ -573,17 +609,17 @@ static int search_impl(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, u64 beg
     if (r1 && lo < r1hi) {
       const u64 a = lo, b = hi < r1hi ? hi : r1hi;
       int nb = 0;
-      c->launches += launch_search_r1(c->tab, sp, S, a - blo, b - blo, c->path32, c->sms, c->d_blocks + used,
+      c->launches += launch_search_r1(c->tab, sp, S, a - blo, b - blo, path, c->sms, c->d_blocks + used,
                                       MAX_BLOCKS - used, &nb, c->d_work, c->h_work, c->work_bytes, next_stream());
       used += nb;
       if (b < hi) {
-        c->launches += launch_search_generic(c->tab, sp, b, hi, c->path32, c->model, wide, c->sms, c->d_blocks + used,
+        c->launches += launch_search_generic(c->tab, sp, b, hi, path, c->model, wide, c->sms, c->d_blocks + used,
                                              MAX_BLOCKS - used, &nb, next_stream());
         used += nb;
       }
     } else {
       int nb = 0;
-      c->launches += launch_search_generic(c->tab, sp, lo, hi, c->path32, c->model, wide, c->sms, c->d_blocks + used,
+      c->launches += launch_search_generic(c->tab, sp, lo, hi, path, c->model, wide, c->sms, c->d_blocks + used,
                                            MAX_BLOCKS - used, &nb, next_stream());
       used += nb;
     }
@@ -596,7 +632,12 @@ static int search_impl(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, u64 beg
     }
   }
   join();
-  if (c->timing) cudaEventRecord(c->ev1, st);
+  cudaEventRecord(c->ev_hwork, st);
+  c->hwork_pending = true;
+  if (c->timing) {
+    cudaEventRecord(c->ev1[tslot], st);
+    ++c->tcount;
+  }
   if (getenv("AUTOPIPE_R1_STATS") && used > 0) {  // diagnostics: rare-path decisions per search
     BlockOut *hb = new BlockOut[used];
     cudaMemcpyAsync(hb, c->d_blocks, sizeof(BlockOut) * used, cudaMemcpyDeviceToHost, st);
@@ -606,17 +647,19 @@ static int search_impl(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, u64 beg
     fprintf(stderr, "[autopipe] blocks %d candidates %llu rare %llu\n", used, cnt, rare);
     delete[] hb;
   }
+  if (async) {
+    c->launches += launch_finalize(c->d_blocks, used, sp, (ResultDev *)d_out, wide, st, rec_bytes);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(c, e, "search kernel launch");
+    return AUTOPIPE_OK;
+  }
   c->launches += launch_finalize(c->d_blocks, used, sp, c->d_result, wide, st);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "search kernel launch");
   e = cudaMemcpyAsync(c->h_result, c->d_result, sizeof(ResultDev), cudaMemcpyDeviceToHost, st);
   if (e == cudaSuccess) e = cudaStreamSynchronize(st);
   if (e != cudaSuccess) return cuda_fail(c, e, "search");
-  if (c->timing) {
-    float ms = 0.f;
-    cudaEventElapsedTime(&ms, c->ev0, c->ev1);
-    c->last_search_ms = ms;
-  }
+  c->hwork_pending = false;
   h_tie[0] = c->h_result->time_ns;
   h_tie[1] = c->h_result->index;
   h_tie[2] = c->h_result->evaluated;
@@ -634,6 +677,34 @@ extern "C" int autopipe_search_optimum(autopipe_ctx *c, uint32_t s_min, uint32_t
   h_out->index = tie[1];
   h_out->evaluated = tie[2];
   return rc;
+}
+
+extern "C" int autopipe_search_optimum_async(autopipe_ctx *c, uint32_t s_min, uint32_t s_max, uint32_t flags,
+                                             uint64_t begin, uint64_t end, autopipe_result *d_out, void *stream) {
+  if (!c) return AUTOPIPE_E_INVAL;
+  if (!d_out) return fail(c, AUTOPIPE_E_INVAL, "NULL result pointer");
+  return search_impl(c, s_min, s_max, flags, begin, end, false, nullptr, nullptr, stream, d_out);
+}
+
+extern "C" int autopipe_search_optimum_async_w(autopipe_ctx *c, uint32_t s_min, uint32_t s_max, uint32_t flags,
+                                               uint64_t begin, uint64_t end, autopipe_result_w *d_out, void *stream) {
+  if (!c) return AUTOPIPE_E_INVAL;
+  if (!d_out) return fail(c, AUTOPIPE_E_INVAL, "NULL result pointer");
+  return search_impl(c, s_min, s_max, flags, begin, end, true, nullptr, nullptr, stream, d_out);
+}
+
+extern "C" int autopipe_reduce_results(const autopipe_result *d_in, uint32_t n, autopipe_result *d_out,
+                                       void *stream) {
+  if (!d_out || (n > 0 && !d_in)) return AUTOPIPE_E_INVAL;
+  launch_reduce_results(d_in, n, 16, d_out, (cudaStream_t)stream);
+  return cudaGetLastError() == cudaSuccess ? AUTOPIPE_OK : AUTOPIPE_E_CUDA;
+}
+
+extern "C" int autopipe_reduce_results_w(const autopipe_result_w *d_in, uint32_t n, autopipe_result_w *d_out,
+                                         void *stream) {
+  if (!d_out || (n > 0 && !d_in)) return AUTOPIPE_E_INVAL;
+  launch_reduce_results(d_in, n, 32, d_out, (cudaStream_t)stream);
+  return cudaGetLastError() == cudaSuccess ? AUTOPIPE_OK : AUTOPIPE_E_CUDA;
 }
 
 extern "C" int autopipe_search_optimum_w(autopipe_ctx *c, uint32_t s_min, uint32_t s_max, uint32_t flags,
@@ -736,16 +807,43 @@ extern "C" uint64_t autopipe_kernel_launches(const autopipe_ctx *c) { return c ?
 extern "C" int autopipe_set_timing(autopipe_ctx *c, int enable) {
   if (!c) return AUTOPIPE_E_INVAL;
   DeviceGuard dg(c->device);
-  if (enable && !c->ev0) {
-    cudaError_t e = cudaEventCreate(&c->ev0);
-    if (e == cudaSuccess) e = cudaEventCreate(&c->ev1);
-    if (e != cudaSuccess) return cuda_fail(c, e, "event create");
+  if (enable && !c->ev0[0]) {
+    for (int i = 0; i < autopipe_ctx::TRING; ++i) {
+      cudaError_t e = cudaEventCreate(&c->ev0[i]);
+      if (e == cudaSuccess) e = cudaEventCreate(&c->ev1[i]);
+      if (e != cudaSuccess) return cuda_fail(c, e, "event create");
+    }
   }
   c->timing = enable != 0;
   return AUTOPIPE_OK;
 }
 
-extern "C" double autopipe_last_search_ms(const autopipe_ctx *c) { return c ? c->last_search_ms : -1.0; }
+static double pair_ms(autopipe_ctx *c, u64 k) {
+  const int i = (int)(k % autopipe_ctx::TRING);
+  float ms = 0.f;
+  cudaEventSynchronize(c->ev1[i]);
+  if (cudaEventElapsedTime(&ms, c->ev0[i], c->ev1[i]) != cudaSuccess) return -1.0;
+  return ms;
+}
+
+extern "C" double autopipe_last_search_ms(const autopipe_ctx *cc) {
+  autopipe_ctx *c = const_cast<autopipe_ctx *>(cc);
+  if (!c || c->tcount == 0) return -1.0;
+  DeviceGuard dg(c->device);
+  return pair_ms(c, c->tcount - 1);
+}
+
+extern "C" int autopipe_search_times(autopipe_ctx *c, double *ms, uint32_t cap, uint32_t *count) {
+  if (!c || !count || (cap > 0 && !ms)) return AUTOPIPE_E_INVAL;
+  DeviceGuard dg(c->device);
+  u64 k = c->tread;
+  if (c->tcount - k > (u64)autopipe_ctx::TRING) k = c->tcount - autopipe_ctx::TRING;  // older pairs reused
+  uint32_t n = 0;
+  for (; k < c->tcount && n < cap; ++k) ms[n++] = pair_ms(c, k);
+  c->tread = k;
+  *count = n;
+  return AUTOPIPE_OK;
+}
 
 // --- NEXT row f1: the two-worker neighbourhood (reading F-1) ----------------
 static int neigh_prepare(autopipe_ctx *c, const autopipe_partition *h_current, u64 &nslots, cudaStream_t st) {

@@ -8,9 +8,13 @@ namespace ap {
 // Binomial coefficients C(n, k), n < 256, k <= 16 (saturated at UINT64_MAX: a space whose size
 // fits 64 bits only ever reads entries below its size), uploaded once per context by autopipe_create.
 __constant__ u64 c_binom[BINOM_N][BINOM_K];
+// the same table in global memory, for the kernels that stage rows of it into shared memory: threads
+// read different entries, which __constant__ would serialise; global loads coalesce (L2-resident)
+__device__ u64 g_binom[BINOM_N][BINOM_K];
 
 void upload_binomials(const u64 (*tab)[BINOM_K]) {
   cudaMemcpyToSymbol(c_binom, tab, sizeof(u64) * BINOM_N * BINOM_K);
+  cudaMemcpyToSymbol(g_binom, tab, sizeof(u64) * BINOM_N * BINOM_K);
 }
 
 // Lexicographic rank of a sorted k-subset {c_0 < ... < c_{k-1}} of {0..n-1} (itertools order):

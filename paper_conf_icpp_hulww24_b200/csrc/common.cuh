@@ -129,6 +129,22 @@ __device__ __forceinline__ u64 warp_sum(u64 v) {
 struct BlockOut {
   u64 t, idx, count, pad;
 };
+// Device-side path choice for a search launched before the host knows the state's path (state set
+// from device memory, asynchronous search): the launcher enqueues the kernel of each path with
+// gate = 1 (32-bit) or 0 (64-bit); a block whose path the state kernel did not choose, or any block
+// after an overflowing state, writes an empty result and returns (uniformly, before any barrier).
+__device__ __forceinline__ bool state_gated_out(const DevTables &g, int gate, BlockOut *out) {
+  const u64 s = *(volatile const u64 *)g.status;
+  if (!(s & 1) && (int)((s >> 1) & 1) == gate) return false;
+  if (threadIdx.x == 0) {
+    out[blockIdx.x].t = U64MAX;
+    out[blockIdx.x].idx = U64MAX;
+    out[blockIdx.x].count = 0;
+    out[blockIdx.x].pad = 0;
+  }
+  return true;
+}
+
 template <int NT>
 __device__ __forceinline__ void block_minloc_store(u64 t, u64 idx, u64 cnt, BlockOut *dst) {
   __shared__ u64 st[NT / 32], si[NT / 32], sc[NT / 32];

@@ -37,7 +37,13 @@ int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, 
 int launch_search_r1(const DevTables &g, const SearchSpace &sp, int S, u64 k_begin, u64 k_end,
                      int path32, int sms, BlockOut *out, int max_blocks, int *nblocks, void *work,
                      void *pinned, size_t work_bytes, cudaStream_t st);
-int launch_finalize(const BlockOut *in, int n, const SearchSpace &sp, ResultDev *out, bool wide, cudaStream_t st);
+// rec_bytes: record bytes written into out->part (32 for the context's own ResultDev; 16 or 32 when
+// out is the caller's autopipe_result / autopipe_result_w)
+int launch_finalize(const BlockOut *in, int n, const SearchSpace &sp, ResultDev *out, bool wide, cudaStream_t st,
+                    int rec_bytes = 32);
+// lexicographic (time_ns, index) minimum of n results of stride 24 + rec_bytes bytes (the autopipe_result
+// layout), evaluated counts summed, the winner's record copied (autopipe_reduce_results)
+int launch_reduce_results(const void *in, unsigned n, int rec_bytes, void *out, cudaStream_t st);
 
 void upload_binomials(const u64 (*tab)[BINOM_K]);
 

@@ -88,7 +88,8 @@ __device__ __forceinline__ void unrank_global_smem(const SearchSpace &sp, u64 id
 
 template <int NT, bool P32, int MODE, typename P>
 __global__ void __launch_bounds__(NT) k_search_generic(DevTables g, SearchSpace sp, u64 begin, u64 end,
-                                                       u64 per_thread, BlockOut *out, ModelP m) {
+                                                       u64 per_thread, BlockOut *out, ModelP m, int gate) {
+  if (gate >= 0 && state_gated_out(g, gate, out)) return;  // see state_gated_out
   typedef SpaceT<P> SP;
   typedef typename SP::PK PK;
   constexpr int BK = SP::BK;
@@ -96,7 +97,7 @@ __global__ void __launch_bounds__(NT) k_search_generic(DevTables g, SearchSpace 
   // binomial rows n <= L (n = N <= 16 <= L + 1 for the compositions too) after the state tables
   u64 *Bn = sm + smem_words(g.L, g.N);
   const int nb = ((int)g.L + 1 > MAXNW + 1 ? (int)g.L + 1 : MAXNW + 1) * BK;
-  for (int i = threadIdx.x; i < nb; i += NT) Bn[i] = c_binom[i / BK][i % BK];
+  for (int i = threadIdx.x; i < nb; i += NT) Bn[i] = g_binom[i / BK][i % BK];
   const SmemTab t = stage_tables(g, sm);  // ends with __syncthreads()
   const u64 gtid = (u64)blockIdx.x * NT + threadIdx.x;
   u64 bestT = U64MAX, bestI = U64MAX, cnt = 0;
@@ -135,12 +136,16 @@ template <int NT, typename P>
 static void run_search_generic(unsigned nbk, size_t smem, cudaStream_t st, const DevTables &g, const SearchSpace &sp,
                                u64 begin, u64 end, u64 pt, BlockOut *out, const ModelP &m, int path32) {
   switch (m.sched) {
-    case SCHED_2BW: k_search_generic<NT, false, SCHED_2BW, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m); break;
-    case SCHED_GPIPE: k_search_generic<NT, false, SCHED_GPIPE, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m); break;
-    case SCHED_DAPPLE: k_search_generic<NT, false, SCHED_DAPPLE, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m); break;
+    case SCHED_2BW: k_search_generic<NT, false, SCHED_2BW, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1); break;
+    case SCHED_GPIPE: k_search_generic<NT, false, SCHED_GPIPE, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1); break;
+    case SCHED_DAPPLE: k_search_generic<NT, false, SCHED_DAPPLE, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1); break;
     default:
-      if (path32) k_search_generic<NT, true, SCHED_PIPEDREAM, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m);
-      else k_search_generic<NT, false, SCHED_PIPEDREAM, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m);
+      if (path32 == 1) k_search_generic<NT, true, SCHED_PIPEDREAM, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1);
+      else if (path32 == 0) k_search_generic<NT, false, SCHED_PIPEDREAM, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1);
+      else {  // path chosen on the device (state_gated_out): both, writing disjoint block ranges
+        k_search_generic<NT, true, SCHED_PIPEDREAM, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, 1);
+        k_search_generic<NT, false, SCHED_PIPEDREAM, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out + nbk, m, 0);
+      }
   }
 }
 
@@ -154,7 +159,9 @@ int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, 
   const u64 min_per = (m.sched == SCHED_GPIPE || m.sched == SCHED_DAPPLE || span <= (u64)sms * 8 * NT * 4) ? 1 : 4;
   u64 threads = (span + min_per - 1) / min_per;
   u64 blocks = (threads + NT - 1) / NT;
-  const u64 cap = (u64)sms * 8 < (u64)max_blocks ? (u64)sms * 8 : (u64)max_blocks;
+  const bool both = path32 < 0 && m.sched == SCHED_PIPEDREAM;  // two gated launches share max_blocks
+  const u64 room = both ? (u64)max_blocks / 2 : (u64)max_blocks;
+  const u64 cap = (u64)sms * 8 < room ? (u64)sms * 8 : room;
   if (blocks > cap) blocks = cap;
   if (blocks == 0) blocks = 1;
   const u64 per = (span + blocks * NT - 1) / (blocks * NT);
@@ -165,21 +172,24 @@ int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, 
   const u64 pt = per ? per : 1;
   if (wide) run_search_generic<NT, P16>(nbk, smem, st, g, sp, begin, end, pt, out, m, path32);
   else run_search_generic<NT, P8>(nbk, smem, st, g, sp, begin, end, pt, out, m, path32);
-  *nblocks = (int)blocks;
-  return 1;
+  *nblocks = (int)blocks * (both ? 2 : 1);
+  return both ? 2 : 1;
 }
 
 // ---------------------------------------------------------------------------------------------
 // grid-level finalisation: one block reduces the per-block (T, index, count) entries, then decodes
 // the winning index into its partition record (16 bytes, or 32 for a wide space).
 // ---------------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(256) k_finalize(const BlockOut *in, int n, SearchSpace sp, ResultDev *res, int wide) {
+// res: the ResultDev layout (time_ns, index, evaluated, record) with the record cut to rec_bytes (16 or
+// 32), so it can be the caller's autopipe_result / autopipe_result_w directly (asynchronous search)
+__global__ void __launch_bounds__(256) k_finalize(const BlockOut *in, int n, SearchSpace sp, ResultDev *res, int wide,
+                                                 int rec_bytes) {
   // binomial rows 0..L (all the unranking needs) in shared memory: the winner is decoded with
   // fixed-length binary searches instead of a serial walk over __constant__ (which misses its cache)
   __shared__ u64 Bn[(MAXL + 1) * BINOM_K];
   const int BK = wide ? BINOM_K : BK8;
   const int rows = (sp.L > sp.N ? sp.L : sp.N) + 1;  // cut sets of {0..L-2}, compositions of {1..N}
-  for (int i = threadIdx.x; i < rows * BK; i += 256) Bn[i] = c_binom[i / BK][i % BK];
+  for (int i = threadIdx.x; i < rows * BK; i += 256) Bn[i] = g_binom[i / BK][i % BK];
   u64 t = U64MAX, idx = U64MAX, cnt = 0;
   for (int i = threadIdx.x; i < n; i += 256) {
     const BlockOut b = in[i];
@@ -218,12 +228,53 @@ __global__ void __launch_bounds__(256) k_finalize(const BlockOut *in, int n, Sea
             if ((p.mask(s) >> w) & 1) rec[off + w] = (unsigned char)s;
       }
     }
-    for (int i = 0; i < 32; ++i) res->part[i] = rec[i];
+    for (int i = 0; i < rec_bytes; ++i) res->part[i] = rec[i];
   }
 }
 
-int launch_finalize(const BlockOut *in, int n, const SearchSpace &sp, ResultDev *out, bool wide, cudaStream_t st) {
-  k_finalize<<<1, 256, 0, st>>>(in, n, sp, out, wide ? 1 : 0);
+int launch_finalize(const BlockOut *in, int n, const SearchSpace &sp, ResultDev *out, bool wide, cudaStream_t st,
+                    int rec_bytes) {
+  k_finalize<<<1, 256, 0, st>>>(in, n, sp, out, wide ? 1 : 0, rec_bytes);
+  return 1;
+}
+
+// Row e (multi-GPU): the per-rank search results gathered into one array (an all-gather of
+// autopipe_result bytes) reduced to their lexicographic (time_ns, index) minimum, evaluated counts
+// summed, the winner's record copied. One warp; n is the number of ranks.
+__global__ void k_reduce_results(const unsigned char *in, unsigned n, int rec_bytes, unsigned char *out) {
+  const unsigned stride = 24u + (unsigned)rec_bytes;
+  u64 t = U64MAX, idx = U64MAX, cnt = 0;
+  unsigned who = 0xFFFFFFFFu;
+  for (unsigned i = threadIdx.x; i < n; i += 32) {
+    const u64 *r = (const u64 *)(in + (size_t)i * stride);
+    if (who == 0xFFFFFFFFu || better(r[0], r[1], t, idx)) {  // ascending i: the first of equals stays
+      t = r[0];
+      idx = r[1];
+      who = i;
+    }
+    cnt += r[2];
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const u64 t2 = __shfl_xor_sync(0xffffffffu, t, o), i2 = __shfl_xor_sync(0xffffffffu, idx, o);
+    const unsigned w2 = __shfl_xor_sync(0xffffffffu, who, o);
+    // ties on (t, idx) (empty results: both UINT64_MAX) resolve to the lower rank, so the copied record
+    // is deterministic
+    if (better(t2, i2, t, idx) || (t2 == t && i2 == idx && w2 < who)) { t = t2; idx = i2; who = w2; }
+    cnt += __shfl_xor_sync(0xffffffffu, cnt, o);
+  }
+  if (threadIdx.x == 0) {
+    u64 *o = (u64 *)out;
+    o[0] = t;
+    o[1] = idx;
+    o[2] = cnt;
+    const unsigned char *src = in + (size_t)(who == 0xFFFFFFFFu ? 0 : who) * stride + 24;
+    for (int b = 0; b < rec_bytes; ++b) out[24 + b] = (n == 0) ? (unsigned char)0xFF : src[b];
+  }
+}
+
+int launch_reduce_results(const void *in, unsigned n, int rec_bytes, void *out, cudaStream_t st) {
+  k_reduce_results<<<1, 32, 0, st>>>((const unsigned char *)in, n, rec_bytes, (unsigned char *)out);
   return 1;
 }
 

@@ -300,8 +300,11 @@ struct XUpd<u32> {  // 32-bit path: every table value is < 2^32 - 16, so clamp o
 template <int S, typename T, int NT>
 __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? R1_MINB32 : R1_MINB64) k_search_r1(DevTables g, const R1Header *__restrict__ hdr_g,
                                                      const R1YEntry *__restrict__ yt_g, R1Header *counter_hdr,
-                                                     BlockOut *out) {
+                                                     BlockOut *out, int gate) {
   constexpr int p = S - 2, q = S - 1, P = S - 4;
+  // gate >= 0: the state was set from device memory and the host launched both paths; only the one
+  // the state kernel chose (status bit 1) runs, and neither after an overflow (status bit 0)
+  if (gate >= 0 && state_gated_out(g, gate, out)) return;
   extern __shared__ __align__(16) unsigned char smraw[];
   const int L = (int)g.L, Lp1 = L + 1, n = L - 1;
   __shared__ R1Header hdr;
@@ -318,7 +321,7 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? R1_MINB32 : R1_MINB64) k_
   // per-warp folded tables follow the schedule (16-byte aligned)
   const int FN = (n + 16 + 3) & ~3;  // columns per warp table (rows of whole 16-byte units)
   T *foldall = (T *)(((uintptr_t)(yt + hdr_g->ny) + 15) & ~(uintptr_t)15);
-  for (int i = threadIdx.x; i < Lp1 * BK8; i += NT) Bn[i] = c_binom[i / BK8][i % BK8];
+  for (int i = threadIdx.x; i < Lp1 * BK8; i += NT) Bn[i] = g_binom[i / BK8][i % BK8];
   for (int i = threadIdx.x; i < S * Lp1; i += NT) PC[i] = g.PC[i];
   for (int i = threadIdx.x; i < (S - 1) * L; i += NT) {
     Z[i] = g.Z[i];
@@ -728,119 +731,126 @@ static u64 count_less(int x, int k, const int *t) {
   return cnt;
 }
 
+// prep = false: the schedule for this (S, shard) was just built and copied by the launch of the other
+// path (gate >= 0 launches both); reuse it
 template <int S, typename T>
 static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u64 k_end, int sms,
                        BlockOut *out, int max_blocks, int *nblocks, void *work, void *pinned, size_t work_bytes,
-                       cudaStream_t st) {
+                       cudaStream_t st, int gate, bool prep) {
   constexpr int P = S - 4, NT = sizeof(T) == 4 ? R1_NT32 : R1_NT64;
   const int L = (int)g.L, n = L - 1, k = S - 1;
-  init_hb();
-  int lo[8], hi[8];
-  host_unrank(k_begin, k, n, lo);
-  host_unrank(k_end - 1, k, n, hi);
-  // schedule staged in the context's pinned buffer (one 16 KB slot per S, like the device work area),
-  // so the copy below is a true async DMA and never waits for earlier work on the stream
   unsigned char *hbuf = (unsigned char *)pinned + (size_t)S * 16384;
   R1Header *h = (R1Header *)hbuf;
-  R1YEntry *yt = (R1YEntry *)(hbuf + sizeof(R1Header));
-  memset(h, 0, sizeof(*h));
-  h->theta = env_u64("AUTOPIPE_R1_THETA0", U64MAX);  // experiment knob: a known bound (unset: none)
-  static const u64 share = env_u64("AUTOPIPE_R1_SHARE", 7);
-  h->share = (u32)share;
-  h->off = sp.off[S];
-  for (int i = 0; i < P; ++i) {
-    h->lo_pre |= (u64)lo[i] << (8 * i);
-    h->hi_pre |= (u64)hi[i] << (8 * i);
-  }
-  h->lo_y = lo[P]; h->lo_x = lo[P + 1]; h->lo_e = lo[P + 2];
-  h->hi_y = hi[P]; h->hi_x = hi[P + 1]; h->hi_e = hi[P + 2];
   int ny = 0;
   u64 tasks = 0;
-  // Task size by estimated cost (thread-instructions per lane): a row costs ~150 (prefix terms) +
-  // ~26 per x + ~6 per candidate. The target per lane-task is set so the shard splits into ~40 tasks
-  // per resident warp (2 x 8 warps per SM): the dynamic schedule's tail stays small at any shard size
-  // (a full 96-layer space on one GPU, or 1/8 of it per GPU), and the per-task unrank is amortised.
-  u64 rb_[256], re_[256], cost_[256];
-  u64 total_cost = 0;
-  for (int y = P; y <= L - 4; ++y) {
-    // rows (prefix, y) whose candidates intersect [lo, hi]: a contiguous range of prefix ranks
-    const bool lo_fits = (P == 0) || lo[P - 1] < y;
-    const bool hi_fits = (P == 0) || hi[P - 1] < y;
-    rb_[y] = count_less(y, P, lo) + ((lo_fits && y < lo[P]) ? 1 : 0);
-    re_[y] = count_less(y, P, hi) + ((hi_fits && y <= hi[P]) ? 1 : 0);
-    const u64 m = (u64)(L - 2 - y);
-    cost_[y] = 150 + 26 * (m - 1) + 6 * (m * (m - 1) / 2);
-    if (re_[y] > rb_[y]) total_cost += (re_[y] - rb_[y]) * cost_[y];
-  }
-  static const u64 tpw = env_u64("AUTOPIPE_R1_TPW", 30), min_target = env_u64("AUTOPIPE_R1_MINTARGET", 12000);
-  const u64 lane_tasks = (u64)sms * 16 * 32 * tpw;
-  u64 TARGET = total_cost / (lane_tasks ? lane_tasks : 1);
-  // Floor on the task size: 12,000 amortises the per-task unrank and seed, but a small space (a
-  // 21-26-layer model) would then be a handful of tasks on 2-6 blocks, latency-bound for 100-300 us.
-  // Small spaces get tasks sized to give every resident warp slot about two (floor 300).
-  u64 floor_t = min_target;
-  const u64 fill = total_cost / ((u64)sms * 16 * 32 * 2);
-  if (fill < floor_t) floor_t = fill > 300 ? fill : 300;
-  if (TARGET < floor_t) TARGET = floor_t;
-  // Guided sizes: warps take tasks in schedule order, so the kernel ends about one task length after
-  // the last task starts. Tasks in the final 15 % of the cost shrink linearly to 1/4 of the target
-  // (smaller ones pay more per-task overhead than they save in tail; measured on B200).
-  static const u64 guided = env_u64("AUTOPIPE_R1_GUIDED", 2);
-  u64 cum = 0;
-  for (int y = P; y <= L - 4; ++y) {
-    const u64 rb = rb_[y], re = re_[y];
-    if (re <= rb) continue;
-    const u64 row_cost = cost_[y];
-    u64 tgt = TARGET;
-    if (guided && total_cost) {
-      const double frac = (double)cum / (double)total_cost, left = 1.0 - frac;
-      const double zone = guided == 1 ? 0.25 : 0.15, floor_ = guided == 1 ? 1.0 / 16 : 0.25;
-      if (left < zone) {
-        const double g = left / zone > floor_ ? left / zone : floor_;
-        tgt = (u64)((double)TARGET * g);
-        if (tgt < 1) tgt = 1;
+  if (prep) {
+    init_hb();
+    int lo[8], hi[8];
+    host_unrank(k_begin, k, n, lo);
+    host_unrank(k_end - 1, k, n, hi);
+    R1YEntry *yt = (R1YEntry *)(hbuf + sizeof(R1Header));
+    memset(h, 0, sizeof(*h));
+    h->theta = env_u64("AUTOPIPE_R1_THETA0", U64MAX);  // experiment knob: a known bound (unset: none)
+    static const u64 share = env_u64("AUTOPIPE_R1_SHARE", 7);
+    h->share = (u32)share;
+    h->off = sp.off[S];
+    for (int i = 0; i < P; ++i) {
+      h->lo_pre |= (u64)lo[i] << (8 * i);
+      h->hi_pre |= (u64)hi[i] << (8 * i);
+    }
+    h->lo_y = lo[P]; h->lo_x = lo[P + 1]; h->lo_e = lo[P + 2];
+    h->hi_y = hi[P]; h->hi_x = hi[P + 1]; h->hi_e = hi[P + 2];
+    // Task size by estimated cost (thread-instructions per lane): a row costs ~150 (prefix terms) +
+    // ~26 per x + ~6 per candidate. The target per lane-task is set so the shard splits into ~40 tasks
+    // per resident warp (2 x 8 warps per SM): the dynamic schedule's tail stays small at any shard size
+    // (a full 96-layer space on one GPU, or 1/8 of it per GPU), and the per-task unrank is amortised.
+    u64 rb_[256], re_[256], cost_[256];
+    u64 total_cost = 0;
+    for (int y = P; y <= L - 4; ++y) {
+      // rows (prefix, y) whose candidates intersect [lo, hi]: a contiguous range of prefix ranks
+      const bool lo_fits = (P == 0) || lo[P - 1] < y;
+      const bool hi_fits = (P == 0) || hi[P - 1] < y;
+      rb_[y] = count_less(y, P, lo) + ((lo_fits && y < lo[P]) ? 1 : 0);
+      re_[y] = count_less(y, P, hi) + ((hi_fits && y <= hi[P]) ? 1 : 0);
+      const u64 m = (u64)(L - 2 - y);
+      cost_[y] = 150 + 26 * (m - 1) + 6 * (m * (m - 1) / 2);
+      if (re_[y] > rb_[y]) total_cost += (re_[y] - rb_[y]) * cost_[y];
+    }
+    static const u64 tpw = env_u64("AUTOPIPE_R1_TPW", 30), min_target = env_u64("AUTOPIPE_R1_MINTARGET", 12000);
+    const u64 lane_tasks = (u64)sms * 16 * 32 * tpw;
+    u64 TARGET = total_cost / (lane_tasks ? lane_tasks : 1);
+    // Floor on the task size: 12,000 amortises the per-task unrank and seed, but a small space (a
+    // 21-26-layer model) would then be a handful of tasks on 2-6 blocks, latency-bound for 100-300 us.
+    // Small spaces get tasks sized to give every resident warp slot about two (floor 300).
+    u64 floor_t = min_target;
+    const u64 fill = total_cost / ((u64)sms * 16 * 32 * 2);
+    if (fill < floor_t) floor_t = fill > 300 ? fill : 300;
+    if (TARGET < floor_t) TARGET = floor_t;
+    // Guided sizes: warps take tasks in schedule order, so the kernel ends about one task length after
+    // the last task starts. Tasks in the final 15 % of the cost shrink linearly to 1/4 of the target
+    // (smaller ones pay more per-task overhead than they save in tail; measured on B200).
+    static const u64 guided = env_u64("AUTOPIPE_R1_GUIDED", 2);
+    u64 cum = 0;
+    for (int y = P; y <= L - 4; ++y) {
+      const u64 rb = rb_[y], re = re_[y];
+      if (re <= rb) continue;
+      const u64 row_cost = cost_[y];
+      u64 tgt = TARGET;
+      if (guided && total_cost) {
+        const double frac = (double)cum / (double)total_cost, left = 1.0 - frac;
+        const double zone = guided == 1 ? 0.25 : 0.15, floor_ = guided == 1 ? 1.0 / 16 : 0.25;
+        if (left < zone) {
+          const double g = left / zone > floor_ ? left / zone : floor_;
+          tgt = (u64)((double)TARGET * g);
+          if (tgt < 1) tgt = 1;
+        }
       }
+      cum += (re - rb) * row_cost;
+      const u64 R = row_cost >= tgt ? 1 : (tgt + row_cost - 1) / row_cost;
+      R1YEntry &ye = yt[ny++];
+      memset(&ye, 0, sizeof(ye));
+      // a row longer than the target is split into x chunks of about equal candidate counts, so a
+      // small shard still gives every warp many tasks (a whole row can hold ~4000 candidates)
+      const int x_first = y + 1, x_end = L - 2;  // x in [y+1, L-3]
+      static const u64 max_chunks = env_u64("AUTOPIPE_R1_CHUNKS", 16);
+      u64 nch = row_cost > tgt ? (row_cost + tgt - 1) / tgt : 1;
+      if (nch > max_chunks) nch = max_chunks;
+      if (nch > (u64)R1_MAXCHUNK) nch = R1_MAXCHUNK;
+      if (nch > (u64)(x_end - x_first)) nch = (u64)(x_end - x_first);
+      if (nch < 1) nch = 1;
+      const u64 m = (u64)(L - 2 - y), pairs = m * (m - 1) / 2;
+      int nc = 0;
+      ye.xcut[nc++] = (unsigned char)x_first;
+      u64 acc = 0;
+      for (int x = x_first; x < x_end && nc < (int)nch; ++x) {
+        acc += (u64)(L - 2 - x);  // pairs with this x
+        if (acc * nch >= pairs * (u64)nc && x + 1 < x_end) ye.xcut[nc++] = (unsigned char)(x + 1);
+      }
+      ye.xcut[nc] = (unsigned char)x_end;
+      const u64 nt = (re - rb + 32 * R - 1) / (32 * R);
+      ye.y = y;
+      ye.rows_per_lane = (u32)R;
+      ye.row_begin = rb;
+      ye.row_end = re;
+      ye.task_begin = tasks;
+      ye.nchunks = (u32)nc;
+      tasks += nt * (u64)nc;
     }
-    cum += (re - rb) * row_cost;
-    const u64 R = row_cost >= tgt ? 1 : (tgt + row_cost - 1) / row_cost;
-    R1YEntry &ye = yt[ny++];
-    memset(&ye, 0, sizeof(ye));
-    // a row longer than the target is split into x chunks of about equal candidate counts, so a
-    // small shard still gives every warp many tasks (a whole row can hold ~4000 candidates)
-    const int x_first = y + 1, x_end = L - 2;  // x in [y+1, L-3]
-    static const u64 max_chunks = env_u64("AUTOPIPE_R1_CHUNKS", 16);
-    u64 nch = row_cost > tgt ? (row_cost + tgt - 1) / tgt : 1;
-    if (nch > max_chunks) nch = max_chunks;
-    if (nch > (u64)R1_MAXCHUNK) nch = R1_MAXCHUNK;
-    if (nch > (u64)(x_end - x_first)) nch = (u64)(x_end - x_first);
-    if (nch < 1) nch = 1;
-    const u64 m = (u64)(L - 2 - y), pairs = m * (m - 1) / 2;
-    int nc = 0;
-    ye.xcut[nc++] = (unsigned char)x_first;
-    u64 acc = 0;
-    for (int x = x_first; x < x_end && nc < (int)nch; ++x) {
-      acc += (u64)(L - 2 - x);  // pairs with this x
-      if (acc * nch >= pairs * (u64)nc && x + 1 < x_end) ye.xcut[nc++] = (unsigned char)(x + 1);
-    }
-    ye.xcut[nc] = (unsigned char)x_end;
-    const u64 nt = (re - rb + 32 * R - 1) / (32 * R);
-    ye.y = y;
-    ye.rows_per_lane = (u32)R;
-    ye.row_begin = rb;
-    ye.row_end = re;
-    ye.task_begin = tasks;
-    ye.nchunks = (u32)nc;
-    tasks += nt * (u64)nc;
+    h->ny = ny;
+    h->ntasks = tasks;
+  } else {
+    ny = h->ny;
+    tasks = h->ntasks;
   }
-  h->ny = ny;
-  h->ntasks = tasks;
   *nblocks = 0;
   if (tasks == 0) return 0;
   const size_t hbytes = sizeof(R1Header) + (size_t)ny * sizeof(R1YEntry);
   // one 16 KB slot per S, so the launches of one search never share a schedule buffer
   if ((size_t)(S + 1) * 16384 > work_bytes || hbytes > 16384) return 0;
   work = (unsigned char *)work + (size_t)S * 16384;
-  cudaMemcpyAsync(work, hbuf, hbytes, cudaMemcpyHostToDevice, st);
+  // the schedule is staged in the context's pinned buffer (one 16 KB slot per S, like the device work
+  // area), so the copy is a true async DMA and never waits for earlier work on the stream
+  if (prep) cudaMemcpyAsync(work, hbuf, hbytes, cudaMemcpyHostToDevice, st);
   const size_t smem = (size_t)(n + 16) * sizeof(ColT<T>) + (size_t)n * sizeof(XT) + (size_t)S * (L + 1) * 8 +
                       2 * (size_t)(S - 1) * L * 8 + (size_t)(L + 1) * BK8 * 8 + (size_t)ny * sizeof(R1YEntry) + 16 +
                       (size_t)(NT / 32) * (size_t)((n + 16 + 3) & ~3) * sizeof(T);
@@ -865,19 +875,19 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
   if (blocks > (u64)max_blocks) blocks = (u64)max_blocks;
   const R1Header *hd = (const R1Header *)work;
   const R1YEntry *yd = (const R1YEntry *)((unsigned char *)work + sizeof(R1Header));
-  k_search_r1<S, T, NT><<<(unsigned)blocks, NT, smem, st>>>(g, hd, yd, (R1Header *)work, out);
+  k_search_r1<S, T, NT><<<(unsigned)blocks, NT, smem, st>>>(g, hd, yd, (R1Header *)work, out, gate);
   *nblocks = (int)blocks;
   return 1;
 }
 
 template <typename T>
 static int launch_r1_s(int S, const DevTables &g, const SearchSpace &sp, u64 a, u64 b, int sms, BlockOut *out,
-                       int mb, int *nb, void *w, void *pin, size_t wb, cudaStream_t st) {
+                       int mb, int *nb, void *w, void *pin, size_t wb, cudaStream_t st, int gate, bool prep) {
   switch (S) {
-    case 5: return launch_r1_t<5, T>(g, sp, a, b, sms, out, mb, nb, w, pin, wb, st);
-    case 6: return launch_r1_t<6, T>(g, sp, a, b, sms, out, mb, nb, w, pin, wb, st);
-    case 7: return launch_r1_t<7, T>(g, sp, a, b, sms, out, mb, nb, w, pin, wb, st);
-    case 8: return launch_r1_t<8, T>(g, sp, a, b, sms, out, mb, nb, w, pin, wb, st);
+    case 5: return launch_r1_t<5, T>(g, sp, a, b, sms, out, mb, nb, w, pin, wb, st, gate, prep);
+    case 6: return launch_r1_t<6, T>(g, sp, a, b, sms, out, mb, nb, w, pin, wb, st, gate, prep);
+    case 7: return launch_r1_t<7, T>(g, sp, a, b, sms, out, mb, nb, w, pin, wb, st, gate, prep);
+    case 8: return launch_r1_t<8, T>(g, sp, a, b, sms, out, mb, nb, w, pin, wb, st, gate, prep);
   }
   *nb = 0;
   return 0;
@@ -886,9 +896,21 @@ static int launch_r1_s(int S, const DevTables &g, const SearchSpace &sp, u64 a, 
 int launch_search_r1(const DevTables &g, const SearchSpace &sp, int S, u64 k_begin, u64 k_end, int path32,
                      int sms, BlockOut *out, int max_blocks, int *nblocks, void *work, void *pinned,
                      size_t work_bytes, cudaStream_t st) {
-  if (path32)
-    return launch_r1_s<u32>(S, g, sp, k_begin, k_end, sms, out, max_blocks, nblocks, work, pinned, work_bytes, st);
-  return launch_r1_s<u64>(S, g, sp, k_begin, k_end, sms, out, max_blocks, nblocks, work, pinned, work_bytes, st);
+  if (path32 == 1)
+    return launch_r1_s<u32>(S, g, sp, k_begin, k_end, sms, out, max_blocks, nblocks, work, pinned, work_bytes, st,
+                            -1, true);
+  if (path32 == 0)
+    return launch_r1_s<u64>(S, g, sp, k_begin, k_end, sms, out, max_blocks, nblocks, work, pinned, work_bytes, st,
+                            -1, true);
+  // path unknown on the host (state set from device memory, asynchronous search): both paths, each
+  // gated on the state kernel's choice; one schedule serves both
+  int n32 = 0, n64 = 0;
+  int k = launch_r1_s<u32>(S, g, sp, k_begin, k_end, sms, out, max_blocks, &n32, work, pinned, work_bytes, st, 1, true);
+  if (n32 > 0)
+    k += launch_r1_s<u64>(S, g, sp, k_begin, k_end, sms, out + n32, max_blocks - n32, &n64, work, pinned, work_bytes,
+                          st, 0, false);
+  *nblocks = n32 + n64;
+  return k;
 }
 
 }  // namespace ap

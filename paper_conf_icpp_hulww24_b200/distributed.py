@@ -1,10 +1,13 @@
 """Multi-GPU search: split the global index space of SPEC.md §5 into one contiguous
 shard per rank, search each shard on its own GPU, and combine with a (T, index) min-loc.
 
-The only exchange is the min-loc: two `all_reduce(MIN)` of one int64 each (plus one SUM for the
-evaluated count), over NCCL between GPUs (or gloo in the CPU tests). Every rank holds the full,
-KB-sized profile and state. The shard arithmetic is exact, so the result is the same for every
-world size.
+The only exchange is the min-loc. On GPUs (`minloc_device`) each rank's asynchronous search leaves its
+40-byte result in device memory; one NCCL all-gather (40 B per rank) and one device reduction
+(autopipe_reduce_results) give every rank the global (T, index) minimum, the summed evaluated count and
+the winner's record, with no host round trip until the caller reads the 40 bytes. `minloc` is the
+host-value form (two all_reduce(MIN) and one SUM), used by the CPU (gloo) tests and the e2e path.
+Every rank holds the full, KB-sized profile and state. The shard arithmetic is exact, so the result
+is the same for every world size.
 """
 from __future__ import annotations
 
@@ -13,7 +16,7 @@ from typing import Callable, List, Optional, Tuple
 import torch
 import torch.distributed as dist
 
-from .engine import SearchResult, U64_MAX
+from .engine import SearchResult, U64_MAX, reduce_results, result_from_bytes
 
 I64_MAX = (1 << 63) - 1
 
@@ -58,15 +61,33 @@ def minloc(T: int, idx: int, evaluated: int, group=None, device=None) -> Tuple[i
     return tmin, imin, int(n.item())
 
 
+def minloc_device(res: torch.Tensor, group=None, reduce_fn: Optional[Callable] = None) -> torch.Tensor:
+    """Row e: all-gather the ranks' result bytes (uint8 [40] or [56] each) and reduce them on the
+    device. `reduce_fn` ([world, nbytes] -> [nbytes]) defaults to autopipe_reduce_results; the CPU
+    tests pass a stand-in."""
+    world = dist.get_world_size(group)
+    if dist.get_backend(group) == "nccl":
+        gathered = torch.empty((world, res.numel()), dtype=torch.uint8, device=res.device)
+        dist.all_gather_into_tensor(gathered.view(-1), res.contiguous(), group=group)
+    else:  # gloo (CPU tests, test-only bench mode): exchange host copies
+        g = torch.empty((world, res.numel()), dtype=torch.uint8)
+        dist.all_gather(list(g.unbind(0)), res.contiguous().cpu(), group=group)
+        gathered = g.to(res.device)
+    return (reduce_fn or reduce_results)(gathered)
+
+
 def search_distributed(engine, s_min: int, s_max: int, flags: int = 0, group=None,
                        shard_search: Optional[Callable[[int, int], SearchResult]] = None,
-                       device=None, balanced: bool = True) -> SearchResult:
+                       device=None, balanced: bool = True,
+                       reduce_fn: Optional[Callable] = None) -> SearchResult:
     """Exhaustive search of the whole space across the ranks of `group`.
 
-    `shard_search(begin, end)` defaults to the engine's CUDA search of that shard; tests pass a
-    stand-in to exercise the distributed logic on CPU. `balanced` splits by estimated device cost
-    (balanced_bounds) instead of equal candidate counts; the result is the same either way. The winner's record is decoded from its
-    global index on every rank (no record broadcast needed)."""
+    By default each rank runs the engine's asynchronous search of its shard and the ranks combine with
+    `minloc_device` (the winner's record travels in its 40-byte result). `shard_search(begin, end)`
+    replaces the shard search with a stand-in (the CPU tests), combined by the host-value `minloc`, the
+    record then decoded from the global index on every rank. `balanced` splits by estimated device
+    cost (balanced_bounds) instead of equal candidate counts; the result is the same either way.
+    `reduce_fn` replaces the device reduction of `minloc_device` (the CPU tests)."""
     rank, world = dist.get_rank(group), dist.get_world_size(group)
     if balanced:
         b = balanced_bounds(engine.L, engine.N, s_min, s_max, flags, world)
@@ -75,10 +96,9 @@ def search_distributed(engine, s_min: int, s_max: int, flags: int = 0, group=Non
         total = engine.count_candidates(s_min, s_max, flags)
         lo, hi = shard_bounds(total, rank, world)
     if shard_search is None:
-        def shard_search(b, e):
-            return engine.search_optimum(s_min, s_max, flags, begin=b, end=e)
-        if device is None:
-            device = engine.device
+        # the engine's asynchronous shard search + the device min-loc: one host read of 40 bytes
+        out = minloc_device(engine.search_optimum_async(s_min, s_max, flags, begin=lo, end=hi), group, reduce_fn)
+        return result_from_bytes(out)
     r = shard_search(lo, hi)
     T, idx, n = minloc(r.time_ns, r.index, r.evaluated, group=group, device=device)
     part = engine.decode_index(s_min, s_max, flags, idx) if idx != U64_MAX else bytes([0xFF] * 16)

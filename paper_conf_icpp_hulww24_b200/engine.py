@@ -51,6 +51,33 @@ class SearchResult:
         return self.index == U64_MAX
 
 
+def result_from_bytes(b) -> SearchResult:
+    """A SearchResult from the bytes of an autopipe_result (40) or autopipe_result_w (56)."""
+    raw = bytes(b.cpu().numpy().tobytes()) if isinstance(b, torch.Tensor) else bytes(b)
+    if len(raw) not in (40, 56):
+        raise ValueError("an autopipe_result is 40 or 56 bytes, got %d" % len(raw))
+    t, i, n = (int.from_bytes(raw[k:k + 8], "little") for k in (0, 8, 16))
+    return SearchResult(t, i, n, raw[24:])
+
+
+def reduce_results(gathered: torch.Tensor, stream=None) -> torch.Tensor:
+    """Row e: device uint8 [n, 40] (or [n, 56]) results -> [40] (or [56]): the lexicographic
+    (time_ns, index) minimum, evaluated summed, the winner's record (autopipe_reduce_results)."""
+    if gathered.dim() != 2 or gathered.shape[1] not in (40, 56) or gathered.dtype != torch.uint8 \
+            or not gathered.is_cuda or not gathered.is_contiguous():
+        raise ValueError("gathered must be a contiguous CUDA uint8 tensor [n, 40] or [n, 56]")
+    out = torch.empty(gathered.shape[1], dtype=torch.uint8, device=gathered.device)
+    fn = lib.autopipe_reduce_results_w if gathered.shape[1] == 56 else lib.autopipe_reduce_results
+    if stream is None:
+        stream = torch.cuda.current_stream(gathered.device)
+    with torch.cuda.device(gathered.device):
+        rc = fn(ctypes.c_void_p(gathered.data_ptr()), gathered.shape[0], ctypes.c_void_p(out.data_ptr()),
+                ctypes.c_void_p(stream.cuda_stream))
+    if rc != 0:
+        raise AutopipeError(rc, "autopipe_reduce_results")
+    return out
+
+
 class Engine:
     """One engine per CUDA device (not thread-safe), mirroring ``autopipe_ctx``."""
 
@@ -196,6 +223,25 @@ class Engine:
         self._check(fn(self._h, s_min, s_max, flags, int(begin), e, ctypes.byref(res), self._stream(stream)))
         return SearchResult(int(res.time_ns), int(res.index), int(res.evaluated), record_bytes(res.part))
 
+    def search_optimum_async(self, s_min: int, s_max: int, flags: int = 0, begin: int = 0,
+                             end: Optional[int] = None, out: Optional[torch.Tensor] = None, stream=None,
+                             wide: Optional[bool] = None) -> torch.Tensor:
+        """The same search, enqueued on the stream with no host wait: the result is a device uint8
+        tensor of 40 bytes (56 for a wide space) in the autopipe_result layout (decode a host copy
+        with `result_from_bytes`). A state set from device memory is not read back (both integer
+        paths are enqueued, the state kernel's choice gates them)."""
+        w = self._wide(s_max, wide)
+        nb = 56 if w else 40
+        if out is None:
+            out = torch.empty(nb, dtype=torch.uint8, device=self.device)
+        if out.numel() != nb or out.dtype != torch.uint8 or out.device != self.device or not out.is_contiguous():
+            raise ValueError("out must be a contiguous uint8 tensor of %d bytes on %s" % (nb, self.device))
+        e = U64_MAX if end is None else int(end)
+        fn = lib.autopipe_search_optimum_async_w if w else lib.autopipe_search_optimum_async
+        self._check(fn(self._h, s_min, s_max, flags, int(begin), e, ctypes.c_void_p(out.data_ptr()),
+                       self._stream(stream)))
+        return out
+
     # -- NEXT row f1: the two-worker neighbourhood (PAPER.md:896-906) ------------------------
     def neighbourhood(self, current: bytes, capacity: int = 1 << 15, stream=None) -> torch.Tensor:
         """All partitions differing from `current` in one or two workers' layer sets (uint8 [n, 16])."""
@@ -266,6 +312,14 @@ class Engine:
     def last_search_ms(self) -> float:
         """Device time of the enumeration kernels of the last search (needs set_timing(True))."""
         return float(lib.autopipe_last_search_ms(self._h))
+
+    def search_times(self) -> list:
+        """Enumeration-kernel times (ms) of the timed searches since the previous call, oldest first
+        (the last 64 at most; waits for them)."""
+        buf = (ctypes.c_double * 64)()
+        n = ctypes.c_uint32()
+        self._check(lib.autopipe_search_times(self._h, buf, 64, ctypes.byref(n)))
+        return [float(buf[i]) for i in range(n.value)]
 
     @property
     def kernel_launches(self) -> int:

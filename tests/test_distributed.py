@@ -29,10 +29,33 @@ class _OracleEngine:
         from oracle.enumerate import count
         return count(self.L, self.N, s_min, s_max, flags)
 
+    def search_optimum_async(self, s_min, s_max, flags, begin, end):
+        """The 40-byte autopipe_result of the oracle's brute force over the shard (a CPU tensor)."""
+        import workloads as W
+        from oracle.model import encode_partition
+        from oracle.search import brute_force
+        T, idx, part, n = brute_force(W.toy(), W.toy_state(), s_min, s_max, flags, begin=begin, end=end)
+        if n == 0:
+            T = idx = (1 << 64) - 1
+        rec = encode_partition(part) if n else bytes([0xFF] * 16)
+        raw = T.to_bytes(8, "little") + idx.to_bytes(8, "little") + n.to_bytes(8, "little") + rec
+        return torch.frombuffer(bytearray(raw), dtype=torch.uint8).clone()
+
     def decode_index(self, s_min, s_max, flags, idx):
         from oracle.enumerate import decode
         from oracle.model import encode_partition
         return encode_partition(decode(self.L, self.N, s_min, s_max, flags, idx))
+
+
+def _reduce_py(gathered):
+    """Stand-in for autopipe_reduce_results on CPU: lexicographic (T, index) minimum, evaluated summed,
+    the first minimal entry's record (its own definition, not the kernel's code)."""
+    rows = [bytes(r.numpy().tobytes()) for r in gathered]
+    key = lambda b: (int.from_bytes(b[0:8], "little"), int.from_bytes(b[8:16], "little"))
+    best = min(range(len(rows)), key=lambda i: (key(rows[i]), i))
+    total = sum(int.from_bytes(b[16:24], "little") for b in rows)
+    out = rows[best][:16] + total.to_bytes(8, "little") + rows[best][24:]
+    return torch.frombuffer(bytearray(out), dtype=torch.uint8).clone()
 
 
 def _worker(rank, world, port, q, case):
@@ -59,7 +82,10 @@ def _worker(rank, world, port, q, case):
             if n == 0:
                 return SearchResult((1 << 64) - 1, (1 << 64) - 1, 0, bytes([0xFF] * 16))
             return SearchResult(T, idx, n, b"")
-        r = search_distributed(eng, 1, 4, 0, shard_search=shard)
+        if case == "search_device":  # the default path: per-rank result bytes, gathered and reduced
+            r = search_distributed(eng, 1, 4, 0, reduce_fn=_reduce_py)
+        else:
+            r = search_distributed(eng, 1, 4, 0, shard_search=shard)
         q.put((rank, (r.time_ns, r.index, r.evaluated, r.partition)))
     finally:
         dist.destroy_process_group()
@@ -105,6 +131,20 @@ def test_search_distributed_gloo_world2_matches_single():
     prof, st = W.toy(), W.toy_state()
     T, idx, part, n = brute_force(prof, st, 1, 4)
     out = _run(2, "search")
+    for rank in (0, 1):
+        assert out[rank] == (T, idx, n, encode_partition(part))
+
+
+def test_search_distributed_device_minloc_gloo_world2():
+    """The GPU path's exchange (all-gather of each rank's 40-byte result, then one reduction) with
+    the shard searches and the reduction replaced by CPU stand-ins: same optimum, count and record as
+    one process."""
+    from oracle.model import encode_partition
+    from oracle.search import brute_force
+    import workloads as W
+    prof, st = W.toy(), W.toy_state()
+    T, idx, part, n = brute_force(prof, st, 1, 4)
+    out = _run(2, "search_device")
     for rank in (0, 1):
         assert out[rank] == (T, idx, n, encode_partition(part))
 
