@@ -112,6 +112,9 @@ def _load():
         "autopipe_search_times": (i32, [P, ctypes.POINTER(ctypes.c_double), u32, ctypes.POINTER(u32)]),
     }
     for name, (res, args) in sig.items():
+        fn = getattr(lib, name, None)
+        if fn is None and os.environ.get("AUTOPIPE_LIB"):
+            continue  # an older variant build named by AUTOPIPE_LIB (experiments): calls it lacks fail
         fn = getattr(lib, name)
         fn.restype = res
         fn.argtypes = args

@@ -946,10 +946,11 @@ extern "C" int autopipe_switch_rewards(autopipe_ctx *c, const autopipe_partition
 // --- cost-balanced contiguous shards of a search space ---------------
 // Estimated device cost (thread-instructions per lane) of the r = 1 kernel: a row (prefix, y) costs
 // ROW + X * (m - 1) + CAND * m (m - 1) / 2 with m = L - 2 - y (calibrated on B200: the per-row term
-// is what makes the high-index shards, whose rows are short, slower per candidate); the generic
+// is what makes the high-index shards, whose rows are short, slower per candidate; re-fitted with
+// the seeded sweep: max/min of 8 C(95,7) shards 1.07 (C4a), 1.05 (C4b)); the generic
 // kernel costs GEN * S per candidate.
 namespace {
-const u64 COST_ROW = 400, COST_X = 26, COST_CAND = 6, COST_GEN = 40;
+const u64 COST_ROW = 600, COST_X = 30, COST_CAND = 4, COST_GEN = 40;
 u64 hbin[256][9];
 void hbin_init() {
   static bool done = false;
@@ -982,8 +983,12 @@ u64 count_less_t(int x, int k, const int *t) {
   return cnt;
 }
 inline double row_cost(int L, int y) {
+  // AUTOPIPE_COST_{ROW,X,CAND}: experiment knobs for re-fitting the model (unset: the constants)
+  static const double cr = getenv("AUTOPIPE_COST_ROW") ? atof(getenv("AUTOPIPE_COST_ROW")) : (double)COST_ROW;
+  static const double cx = getenv("AUTOPIPE_COST_X") ? atof(getenv("AUTOPIPE_COST_X")) : (double)COST_X;
+  static const double cc = getenv("AUTOPIPE_COST_CAND") ? atof(getenv("AUTOPIPE_COST_CAND")) : (double)COST_CAND;
   const double m = (double)(L - 2 - y);
-  return (double)COST_ROW + COST_X * (m - 1) + COST_CAND * m * (m - 1) / 2;
+  return cr + cx * (m - 1) + cc * m * (m - 1) / 2;
 }
 // cost of the first `kappa` cut sets (lexicographic) of an r = 1 block with S stages
 double r1_prefix_cost(int L, int S, u64 kappa, u64 ncut) {

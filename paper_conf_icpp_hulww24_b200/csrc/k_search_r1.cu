@@ -60,6 +60,9 @@ constexpr int R1_MAXCHUNK = 16;
 #ifndef R1_NT64
 #define R1_NT64 256
 #endif
+#ifndef R1_GBINOM
+#define R1_GBINOM 1
+#endif
 #ifndef R1_MINB32
 #define R1_MINB32 3
 #endif
@@ -109,8 +112,10 @@ constexpr i64 THETA_ALL = 1ll << 60;
 
 __device__ __forceinline__ i64 smin(i64 a, i64 b) { return a < b ? a : b; }
 
-// exact T of an r = 1 candidate (all divisions), from the u64 tables in shared memory
-template <int S>
+// exact T of an r = 1 candidate (all divisions), from u64 tables (shared memory in the sweep's rare
+// path, global memory in the seed kernel: Seed = true gives the seed its own copy, so the sweep's
+// call keeps its specialised calling convention)
+template <int S, bool Seed = false>
 __device__ __noinline__ u64 exact_T_r1(const u64 *PC, const u64 *Z, const u64 *LM, int L, u64 cuts) {
   const int Lp1 = L + 1;
   u64 c[S], z[S];
@@ -321,7 +326,11 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? R1_MINB32 : R1_MINB64) k_
   // per-warp folded tables follow the schedule (16-byte aligned)
   const int FN = (n + 16 + 3) & ~3;  // columns per warp table (rows of whole 16-byte units)
   T *foldall = (T *)(((uintptr_t)(yt + hdr_g->ny) + 15) & ~(uintptr_t)15);
+#if R1_GBINOM
   for (int i = threadIdx.x; i < Lp1 * BK8; i += NT) Bn[i] = g_binom[i / BK8][i % BK8];
+#else
+  for (int i = threadIdx.x; i < Lp1 * BK8; i += NT) Bn[i] = c_binom[i / BK8][i % BK8];
+#endif
   for (int i = threadIdx.x; i < S * Lp1; i += NT) PC[i] = g.PC[i];
   for (int i = threadIdx.x; i < (S - 1) * L; i += NT) {
     Z[i] = g.Z[i];
@@ -689,6 +698,162 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? R1_MINB32 : R1_MINB64) k_
 }
 
 // ------------------------------------------------------------------------------------------------
+// Seed bound (before the sweep; same stream): a good in-shard candidate found by a cheap heuristic
+// gives the grid's shared theta a tight start, so the sweep's early rows are not flooded with rare-path
+// decisions while the lanes' own bests are still poor. It never changes a result: theta is the T of a
+// real candidate of the shard, the sweep still decides every candidate against the running theta
+// (non-strict against the shared value), and the shard's (T, index) minimum has T <= theta.
+// One warp per variant: the first cut free (v = 0) or fixed next to the shard's first / last cut
+// (v = 1..4). The rest of the cuts: the min-max greedy (each stage as long as its cost c_s and its
+// boundary term lm_s stay <= theta), theta found by a 33-way parallel search over the warp; then up to
+// R1_SEED_ROUNDS rounds of the best single-cut move (+-1, +-2) by exact T, moves kept inside the shard.
+// ------------------------------------------------------------------------------------------------
+#ifndef R1_SEED_ROUNDS
+#define R1_SEED_ROUNDS 4
+#endif
+
+template <int S>
+__device__ __forceinline__ bool cuts_in_shard(const R1Header &h, const int *c) {
+  constexpr int P = S - 4;
+  int lo[S - 1], hi[S - 1];
+#pragma unroll
+  for (int i = 0; i < P; ++i) {
+    lo[i] = (int)((h.lo_pre >> (8 * i)) & 0xFF);
+    hi[i] = (int)((h.hi_pre >> (8 * i)) & 0xFF);
+  }
+  lo[P] = h.lo_y; lo[P + 1] = h.lo_x; lo[P + 2] = h.lo_e;
+  hi[P] = h.hi_y; hi[P + 1] = h.hi_x; hi[P + 2] = h.hi_e;
+  int cl = 0, ch = 0;  // lexicographic comparison against lo and hi (first differing cut decides)
+#pragma unroll
+  for (int i = 0; i < S - 1; ++i) {
+    if (cl == 0 && c[i] != lo[i]) cl = c[i] < lo[i] ? -1 : 1;
+    if (ch == 0 && c[i] != hi[i]) ch = c[i] < hi[i] ? -1 : 1;
+  }
+  return cl >= 0 && ch <= 0;
+}
+
+// greedy cuts for stages j..S-1 (stage s on worker s) over layers [a, L-1] under theta; false if some
+// stage cannot be placed. Cut s is the largest e with c_s <= theta, backed off while lm_s(e) > theta,
+// leaving one layer per later stage.
+template <int S>
+__device__ bool greedy_cuts(const DevTables &g, int L, int j, int a, u64 th, int *c) {
+  const int Lp1 = L + 1;
+  int pos = a;
+  for (int s = j; s < S - 1; ++s) {
+    const u64 *pc = g.PC + (size_t)s * Lp1;
+    const int emax = L - 1 - (S - 1 - s);
+    if (pos > emax) return false;
+    const u64 lim = pc[pos] + th;
+    int lo = pos - 1, hi = emax;  // largest e in [pos, emax] with pc[e + 1] <= lim (binary search)
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (pc[mid + 1] <= lim) lo = mid;
+      else hi = mid - 1;
+    }
+    int e = lo;
+    while (e >= pos && g.LM[(size_t)s * L + e] > th) --e;
+    if (e < pos) return false;
+    c[s] = e;
+    pos = e + 1;
+  }
+  return g.PC[(size_t)(S - 1) * Lp1 + L] - g.PC[(size_t)(S - 1) * Lp1 + pos] <= th;
+}
+
+template <int S>
+__device__ __forceinline__ u64 pack_cuts(const int *c) {
+  u64 p = 0;
+#pragma unroll
+  for (int i = 0; i < S - 1; ++i) p |= (u64)c[i] << (8 * i);
+  return p;
+}
+
+template <int S>
+__global__ void __launch_bounds__(160) k_seed_r1(DevTables gd, R1Header *hdr) {
+  if (gd.status[0] & 1) return;  // overflowing state: the search kernels exit too
+  // the walks below are chains of dependent loads: stage PC (stages 0..S-1), Z and LM in shared memory
+  __shared__ u64 sPC[S * (MAXL + 1)], sZ[(S - 1) * MAXL], sLM[(S - 1) * MAXL];
+  const int L = (int)gd.L, Lp1 = L + 1, lane = threadIdx.x & 31, v = threadIdx.x >> 5;
+  for (int i = threadIdx.x; i < S * Lp1; i += blockDim.x) sPC[i] = gd.PC[i];
+  for (int i = threadIdx.x; i < (S - 1) * L; i += blockDim.x) {
+    sZ[i] = gd.Z[i];
+    sLM[i] = gd.LM[i];
+  }
+  __syncthreads();
+  DevTables g = gd;
+  g.PC = sPC;
+  g.Z = sZ;
+  g.LM = sLM;
+  const R1Header h = *hdr;
+  const int lo0 = (int)(h.lo_pre & 0xFF), hi0 = (int)(h.hi_pre & 0xFF);
+  int j = 0, e0 = 0;
+  if (v > 0) {
+    j = 1;
+    e0 = v == 1 ? lo0 : v == 2 ? lo0 + 1 : v == 3 ? hi0 - 1 : hi0;
+    if (e0 < 0 || e0 > L - S || (v == 2 && e0 > hi0) || (v == 3 && e0 < lo0)) return;
+  }
+  const int a = j ? e0 + 1 : 0;
+  // theta range: [0, an upper bound that is feasible]
+  u64 tlo = 0, thi = 0;
+  for (int s = 0; s < S; ++s) thi = umax(thi, g.PC[(size_t)s * Lp1 + L]);
+  for (int s = 0; s < S - 1; ++s)
+    for (int e = lane; e < L; e += 32) thi = umax(thi, g.LM[(size_t)s * L + e]);
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) thi = umax(thi, __shfl_xor_sync(0xffffffffu, thi, o));
+  int c[S - 1];
+  if (j) c[0] = e0;
+  if (!greedy_cuts<S>(g, L, j, a, thi, c)) return;
+  while (thi - tlo > 1) {  // invariant: tlo infeasible (or 0), thi feasible
+    const u64 step = (thi - tlo) / 33 ? (thi - tlo) / 33 : 1;
+    const u64 t = tlo + step * (u64)(lane + 1);
+    int cc[S - 1];
+    if (j) cc[0] = e0;
+    const bool ok = t < thi && greedy_cuts<S>(g, L, j, a, t, cc);
+    const unsigned m = __ballot_sync(0xffffffffu, ok);
+    const unsigned bad = __ballot_sync(0xffffffffu, !ok && t < thi);
+    if (m) {
+      const int f = __ffs(m) - 1;  // the smallest feasible t
+      thi = __shfl_sync(0xffffffffu, t, f);
+      const unsigned below = bad & ((1u << f) - 1u);
+      if (below) tlo = __shfl_sync(0xffffffffu, t, 31 - __clz(below));
+    } else {
+      const unsigned lastbad = bad ? 31 - __clz(bad) : 0;
+      tlo = bad ? __shfl_sync(0xffffffffu, t, lastbad) : tlo;
+      if (!bad) break;
+    }
+  }
+  if (j) c[0] = e0;
+  greedy_cuts<S>(g, L, j, a, thi, c);
+  u64 bestT = cuts_in_shard<S>(h, c) ? exact_T_r1<S, true>(g.PC, g.Z, g.LM, L, pack_cuts<S>(c)) : U64MAX;
+  // refinement: lane m tries move m (cut i = j + m / 4, delta -2, -1, +1, +2); the best improving
+  // in-shard move of the warp is applied
+  for (int round = 0; round < R1_SEED_ROUNDS; ++round) {
+    int cc[S - 1];
+#pragma unroll
+    for (int i = 0; i < S - 1; ++i) cc[i] = c[i];
+    const int i = j + lane / 4, d = (lane & 3) < 2 ? (lane & 3) - 2 : (lane & 3) - 1;
+    u64 T = U64MAX;
+    if (i < S - 1) {
+      cc[i] += d;
+      const int lo = i == 0 ? 0 : cc[i - 1] + 1, hi = i == S - 2 ? L - 2 : cc[i + 1] - 1;
+      if (cc[i] >= lo && cc[i] <= hi && cuts_in_shard<S>(h, cc)) T = exact_T_r1<S, true>(g.PC, g.Z, g.LM, L, pack_cuts<S>(cc));
+    }
+    u64 bt = T;
+    int bl = lane;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      const u64 t2 = __shfl_xor_sync(0xffffffffu, bt, o);
+      const int l2 = __shfl_xor_sync(0xffffffffu, bl, o);
+      if (t2 < bt || (t2 == bt && l2 < bl)) { bt = t2; bl = l2; }
+    }
+    if (bt >= bestT) break;
+    bestT = bt;
+    const int bi = j + bl / 4, bd = (bl & 3) < 2 ? (bl & 3) - 2 : (bl & 3) - 1;
+    c[bi] += bd;
+  }
+  if (lane == 0 && bestT != U64MAX) atomicMin(&hdr->theta, (unsigned long long)bestT);
+}
+
+// ------------------------------------------------------------------------------------------------
 // host side: the task schedule (rows per y restricted to the shard) and the launch
 // ------------------------------------------------------------------------------------------------
 static u64 env_u64(const char *name, u64 dflt) {  // tuning knobs for experiments (unset: defaults)
@@ -850,7 +1015,17 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
   work = (unsigned char *)work + (size_t)S * 16384;
   // the schedule is staged in the context's pinned buffer (one 16 KB slot per S, like the device work
   // area), so the copy is a true async DMA and never waits for earlier work on the stream
-  if (prep) cudaMemcpyAsync(work, hbuf, hbytes, cudaMemcpyHostToDevice, st);
+  int launched = 1;  // the sweep kernel below, + the seed kernel
+  if (prep) {
+    cudaMemcpyAsync(work, hbuf, hbytes, cudaMemcpyHostToDevice, st);
+    // before the sweep, on its stream. (Beside it, on a stream of its own with a block slot left free,
+    // it came too late for the 32-bit C4a search: 3.08 ms against 2.85.) Experiment knob: 0 = off.
+    static const u64 seed = env_u64("AUTOPIPE_R1_SEED", 1);
+    if (seed) {
+      k_seed_r1<S><<<1, 160, 0, st>>>(g, (R1Header *)work);
+      ++launched;
+    }
+  }
   const size_t smem = (size_t)(n + 16) * sizeof(ColT<T>) + (size_t)n * sizeof(XT) + (size_t)S * (L + 1) * 8 +
                       2 * (size_t)(S - 1) * L * 8 + (size_t)(L + 1) * BK8 * 8 + (size_t)ny * sizeof(R1YEntry) + 16 +
                       (size_t)(NT / 32) * (size_t)((n + 16 + 3) & ~3) * sizeof(T);
@@ -877,7 +1052,7 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
   const R1YEntry *yd = (const R1YEntry *)((unsigned char *)work + sizeof(R1Header));
   k_search_r1<S, T, NT><<<(unsigned)blocks, NT, smem, st>>>(g, hd, yd, (R1Header *)work, out, gate);
   *nblocks = (int)blocks;
-  return 1;
+  return launched;
 }
 
 template <typename T>
