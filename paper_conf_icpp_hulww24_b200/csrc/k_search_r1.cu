@@ -1021,7 +1021,9 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
     // before the sweep, on its stream. (Beside it, on a stream of its own with a block slot left free,
     // it came too late for the 32-bit C4a search: 3.08 ms against 2.85.) Experiment knob: 0 = off.
     static const u64 seed = env_u64("AUTOPIPE_R1_SEED", 1);
-    if (seed) {
+    // a small block (a short model's space, C2/C3) is over before a bad start costs anything, while
+    // the seed's ~20 us would sit on its critical path
+    if (seed && k_end - k_begin >= (1ull << 26)) {
       k_seed_r1<S><<<1, 160, 0, st>>>(g, (R1Header *)work);
       ++launched;
     }
