@@ -38,9 +38,14 @@
 namespace ap {
 
 constexpr int R1_MAXCHUNK = 16;
-// x values per pass of the column sweep
-#ifndef R1_NX
-#define R1_NX 2
+// x values per pass of the column sweep, per path (B200: 2 for the 32-bit tables, whose aligned
+// 8-column scan is cheap and whose 80-register budget is tight; 3 for the 64-bit ones: C4b 4.56 ->
+// 4.27 ms, while 3 on the 32-bit path ran 2.80 -> 3.07 ms)
+#ifndef R1_NX32
+#define R1_NX32 2
+#endif
+#ifndef R1_NX64
+#define R1_NX64 3
 #endif
 // aligned 4-column groups in the sweep body (128-bit shared loads)
 #ifndef R1_V4
@@ -529,7 +534,7 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? R1_MINB32 : R1_MINB64) k_
       // candidates and their compare chains are independent. Hits of the first x are decided at
       // once; a later x only records its first hit and is rescanned (sweep1) after the pass, in x
       // order, so a lane decides its candidates in increasing index order (tie-break, reading C-13).
-      constexpr int NX = R1_NX;
+      constexpr int NX = sizeof(T) == 4 ? R1_NX32 : R1_NX64;
       for (int x = xa; x < xb; x += NX) {
         const int nx = xb - x < NX ? xb - x : NX;
         T H1[NX];
