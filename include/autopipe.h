@@ -273,6 +273,8 @@ int autopipe_get_schedule(const autopipe_ctx *ctx, uint32_t *schedule, uint32_t 
  * in autopipe_search_optimum; L layers, N workers) cost about the same device time: the estimate
  * counts rows and columns of the fast kernel (short rows cost more per candidate), so shards are not
  * equal in candidates. Host-only (no context, no GPU); any split gives the same global optimum.
+ * Wide spaces (row f4: N <= 16, s_max <= min(16, N); the index order of autopipe_search_optimum_w)
+ * are split the same way (their S > 8 blocks cost as generic-kernel candidates).
  * E_INVAL on bad arguments, E_OVERFLOW if the space exceeds 2^64. */
 int autopipe_balanced_shards(uint32_t L, uint32_t N, uint32_t s_min, uint32_t s_max, uint32_t flags, uint32_t G,
                              uint64_t *bounds);

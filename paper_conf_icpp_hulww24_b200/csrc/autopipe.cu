@@ -951,12 +951,15 @@ extern "C" int autopipe_switch_rewards(autopipe_ctx *c, const autopipe_partition
 // kernel costs GEN * S per candidate.
 namespace {
 const u64 COST_ROW = 600, COST_X = 30, COST_CAND = 4, COST_GEN = 40;
-u64 hbin[256][9];
+u64 hbin[256][17];  // C(n, k), k <= 16 (wide spaces), saturated at 2^64 - 1
 void hbin_init() {
   static bool done = false;
   if (done) return;
   for (int n = 0; n < 256; ++n)
-    for (int k = 0; k < 9; ++k) hbin[n][k] = (k == 0) ? 1 : (n == 0 ? 0 : hbin[n - 1][k - 1] + hbin[n - 1][k]);
+    for (int k = 0; k < 17; ++k) {
+      const u64 a = (n == 0) ? 0 : hbin[n - 1][k - (k > 0)], b = (n == 0) ? 0 : hbin[n - 1][k];
+      hbin[n][k] = (k == 0) ? 1 : (a + b < a ? ~0ull : a + b);
+    }
   done = true;
 }
 inline u64 hbn(int n, int k) { return (k < 0 || n < 0 || k > n) ? 0 : hbin[n][k]; }
@@ -1010,9 +1013,10 @@ double r1_prefix_cost(int L, int S, u64 kappa, u64 ncut) {
 
 extern "C" int autopipe_balanced_shards(uint32_t L, uint32_t N, uint32_t s_min, uint32_t s_max, uint32_t flags,
                                         uint32_t G, uint64_t *bounds) {
-  if (!bounds || G < 1 || L < 1 || L > MAXL || N < 1 || N > MAXN) return AUTOPIPE_E_INVAL;
+  if (!bounds || G < 1 || L < 1 || L > MAXL || N < 1 || N > MAXNW) return AUTOPIPE_E_INVAL;
   if (flags & ~AUTOPIPE_USE_ALL_WORKERS) return AUTOPIPE_E_INVAL;
-  const u32 smax_lim = N < (u32)MAXS ? N : (u32)MAXS;
+  // 16-byte spaces (S, N <= 8) and wide ones (row f4: S, N <= 16; their S > 8 blocks are generic)
+  const u32 smax_lim = N < (u32)MAXSW ? N : (u32)MAXSW;
   if (s_min < 1 || s_min > s_max || s_max > smax_lim) return AUTOPIPE_E_INVAL;
   hbin_init();
   const bool all = flags & AUTOPIPE_USE_ALL_WORKERS;
@@ -1027,7 +1031,7 @@ extern "C" int autopipe_balanced_shards(uint32_t L, uint32_t N, uint32_t s_min, 
     const u64 nc = (S - 1 <= (int)L - 1) ? hbn((int)L - 1, S - 1) : 0;
     const u128 sz = (u128)K * nc;
     if ((off + sz) >> 64) return AUTOPIPE_E_OVERFLOW;
-    const bool r1 = S >= 5 && (!all || (int)N == S) && nc > 0;
+    const bool r1 = S >= 5 && S <= MAXS && (!all || (int)N == S) && nc > 0;
     u64 start = (u64)off;
     if (r1) {
       const double c = r1_prefix_cost((int)L, S, nc, nc);

@@ -163,6 +163,13 @@ def test_balanced_bounds_partition_the_space():
             b = balanced_bounds(L, N, smin, smax, flags, G)
             assert len(b) == G + 1 and b[0] == 0 and b[-1] == total
             assert all(x <= y for x, y in zip(b, b[1:]))
+    # wide spaces (row f4): 10 and 16 workers, stages beyond 8
+    for (L, N, smin, smax, flags) in ((12, 10, 1, 10, 0), (20, 16, 9, 12, 1), (30, 12, 5, 12, 0)):
+        total = count(L, N, smin, smax, flags)
+        for G in (1, 3, 8):
+            b = balanced_bounds(L, N, smin, smax, flags, G)
+            assert len(b) == G + 1 and b[0] == 0 and b[-1] == total
+            assert all(x <= y for x, y in zip(b, b[1:]))
     # the 96-layer space: later shards (short rows) get fewer candidates than earlier ones
     b = balanced_bounds(96, 8, 8, 8, 0, 8)
     sizes = [y - x for x, y in zip(b, b[1:])]
@@ -172,6 +179,7 @@ def test_balanced_bounds_partition_the_space():
 def test_balanced_bounds_rejects_bad_arguments():
     from paper_conf_icpp_hulww24_b200.distributed import balanced_bounds
     for args in ((96, 8, 0, 8, 0, 2), (96, 8, 3, 2, 0, 2), (96, 4, 1, 5, 0, 2), (96, 8, 1, 8, 2, 2),
-                 (96, 8, 1, 8, 0, 0), (0, 8, 1, 1, 0, 1), (256, 8, 1, 8, 0, 1)):
+                 (96, 8, 1, 8, 0, 0), (0, 8, 1, 1, 0, 1), (256, 8, 1, 8, 0, 1), (96, 17, 1, 8, 0, 2),
+                 (96, 16, 1, 17, 0, 2)):
         with pytest.raises(ValueError):
             balanced_bounds(*args)

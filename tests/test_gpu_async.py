@@ -157,3 +157,19 @@ def test_async_wide_testbed(eng):
     want = eng.search_optimum(1, 10)
     got = _async(eng, 1, 10)
     assert _tuple(got) == _tuple(want) and len(got.partition) == 32
+
+
+def test_wide_sharded_search_reduced(eng):
+    """Row e on a wide space (row f4): cost-balanced shards of the 10-worker testbed space, each
+    searched asynchronously, reduced on the device = the single search."""
+    from paper_conf_icpp_hulww24_b200 import reduce_results, result_from_bytes
+    from paper_conf_icpp_hulww24_b200.distributed import balanced_bounds
+    prof = W.vgg16()
+    st = W.testbed_state(prof, seed=10)
+    eng.load(prof, st)
+    want = eng.search_optimum(1, 10)
+    for G in (2, 3, 8):
+        b = balanced_bounds(prof.L, 10, 1, 10, 0, G)
+        outs = [eng.search_optimum_async(1, 10, begin=b[i], end=b[i + 1]) for i in range(G)]
+        got = result_from_bytes(reduce_results(torch.stack(outs)))
+        assert _tuple(got) == _tuple(want)
