@@ -74,6 +74,10 @@ constexpr int R1_MAXCHUNK = 16;
 #ifndef R1_MINB64
 #define R1_MINB64 2
 #endif
+// 1: count rare-path decisions per block (BlockOut.pad, read by AUTOPIPE_R1_STATS)
+#ifndef R1_STATS
+#define R1_STATS 1
+#endif
 struct R1YEntry {      // one y value of the schedule (host-built shard arithmetic, SPEC.md §5)
   int y;               // e_{S-4}
   u32 rows_per_lane;   // R
@@ -498,7 +502,9 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? R1_MINB32 : R1_MINB64) k_
         const u64 cuts = pre | ((u64)y << (8 * P)) | ((u64)xk << (8 * (P + 1))) | ((u64)ee << (8 * (P + 2)));
         const u64 Tc = exact_T_r1<S>(PC, Z, LM, L, cuts);
         const u64 idx = hdr.off + lex_rank_smem(cuts, S - 1, n, Bn);
+#if R1_STATS
         ++nrare;
+#endif
         if (better(Tc, idx, bestT, bestI)) {
           bestT = Tc;
           bestI = idx;
