@@ -158,6 +158,30 @@ int autopipe_search_optimum(autopipe_ctx *ctx, uint32_t s_min, uint32_t s_max, u
 int autopipe_search_optimum_async(autopipe_ctx *ctx, uint32_t s_min, uint32_t s_max, uint32_t flags,
                                   uint64_t begin, uint64_t end, autopipe_result *d_out, void *stream);
 
+/* Row e, cross-shard bound (north star: "split the index space ... NCCL min-loc"). A shard's sweep
+ * filters its candidates against the best T known so far; alone it only knows its own shard, and a
+ * shard far from the optimum filters poorly. The bound lets every shard start from the best seed of
+ * ALL shards:
+ *   1. autopipe_search_seed_async: d_theta (DEVICE u64, caller-owned) is set to UINT64_MAX, then for
+ *      every r = 1 block of [begin, end) with >= 2^26 candidates (the blocks whose sweep seeds
+ *      itself) the seed kernel's exact T of one candidate of the shard is min-folded into it.
+ *      No sweep, no result; asynchronous on `stream`. Blocks with fewer candidates, other S and
+ *      other schedules leave it untouched.
+ *   2. the caller min-reduces d_theta over the ranks (NCCL all_reduce MIN, 8 bytes);
+ *   3. autopipe_set_search_bound(ctx, d_theta): the context's later searches start every r = 1
+ *      sweep from theta = *d_theta (read on the device when the sweep starts) instead of running
+ *      their own seed; NULL clears it. The pointer must stay valid while it is set.
+ * A search under a bound returns the shard's exact (time_ns, index) minimum whenever that minimum
+ * is <= *d_theta; otherwise its result is (UINT64_MAX, UINT64_MAX, evaluated, 0xFF...) or a
+ * candidate with time_ns > *d_theta. Because *d_theta is the exact T of a real candidate of some
+ * shard (candidates are still decided one by one, non-strictly against the bound, so ties keep
+ * their lowest index), the reduction over all shards (autopipe_reduce_results) is the exact
+ * optimum of the whole space, identical to the unbounded search. Errors: E_INVAL (NULL pointer),
+ * E_STATE, the argument checks of autopipe_search_optimum. */
+int autopipe_search_seed_async(autopipe_ctx *ctx, uint32_t s_min, uint32_t s_max, uint32_t flags,
+                               uint64_t begin, uint64_t end, uint64_t *d_theta, void *stream);
+int autopipe_set_search_bound(autopipe_ctx *ctx, const uint64_t *d_bound);
+
 /* Row e (north star: "only a tiny NCCL min-loc allreduce"): d_in[n] results (e.g. all-gathered from
  * the ranks' asynchronous searches; device memory) -> *d_out = their lexicographic (time_ns, index)
  * minimum, evaluated = the sum, the record of the winner (on exact ties, the lowest entry's). Async on

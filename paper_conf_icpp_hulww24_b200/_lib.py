@@ -38,7 +38,8 @@ SYMBOLS = ["autopipe_create", "autopipe_destroy", "autopipe_last_error", "autopi
            "autopipe_switch_rewards", "autopipe_balanced_shards", "autopipe_set_schedule",
            "autopipe_get_schedule", "autopipe_eval_partitions_w", "autopipe_rollout_rewards_w",
            "autopipe_search_optimum_w", "autopipe_decode_index_w", "autopipe_search_optimum_async",
-           "autopipe_search_optimum_async_w", "autopipe_reduce_results", "autopipe_reduce_results_w", "autopipe_search_times"]
+           "autopipe_search_optimum_async_w", "autopipe_reduce_results", "autopipe_reduce_results_w", "autopipe_search_times",
+           "autopipe_search_seed_async", "autopipe_set_search_bound"]
 
 
 class Partition(ctypes.Structure):
@@ -107,6 +108,8 @@ def _load():
         "autopipe_get_schedule": (i32, [P] + [ctypes.POINTER(ctypes.c_uint32)] * 4),
         "autopipe_search_optimum_async": (i32, [P, u32, u32, u32, u64, u64, P, P]),
         "autopipe_search_optimum_async_w": (i32, [P, u32, u32, u32, u64, u64, P, P]),
+        "autopipe_search_seed_async": (i32, [P, u32, u32, u32, u64, u64, P, P]),
+        "autopipe_set_search_bound": (i32, [P, P]),
         "autopipe_reduce_results": (i32, [P, u32, P, P]),
         "autopipe_reduce_results_w": (i32, [P, u32, P, P]),
         "autopipe_search_times": (i32, [P, ctypes.POINTER(ctypes.c_double), u32, ctypes.POINTER(u32)]),

@@ -63,6 +63,12 @@ struct autopipe_ctx {
   // (an asynchronous search returns before its copies have run)
   cudaEvent_t ev_hwork = nullptr;
   bool hwork_pending = false;
+  // row e, cross-shard bound: the device word later searches' r = 1 sweeps start from
+  // (autopipe_set_search_bound), and the seed-only call's own schedule slots (upper half of the work
+  // areas) with their own copy event
+  const u64 *d_bound = nullptr;
+  cudaEvent_t ev_hseed = nullptr;
+  bool hseed_pending = false;
 };
 
 static char g_create_err[256] = "";
@@ -193,6 +199,7 @@ extern "C" void autopipe_destroy(autopipe_ctx *c) {
     if (c->h_result) cudaFreeHost(c->h_result);
     if (c->h_status) cudaFreeHost(c->h_status);
     if (c->ev_hwork) cudaEventDestroy(c->ev_hwork);
+    if (c->ev_hseed) cudaEventDestroy(c->ev_hseed);
     for (int i = 0; i < autopipe_ctx::TRING; ++i) {
       if (c->ev0[i]) cudaEventDestroy(c->ev0[i]);
       if (c->ev1[i]) cudaEventDestroy(c->ev1[i]);
@@ -609,8 +616,10 @@ static int search_impl(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, u64 beg
     if (r1 && lo < r1hi) {
       const u64 a = lo, b = hi < r1hi ? hi : r1hi;
       int nb = 0;
+      R1Ext ext;
+      ext.bound = c->d_bound;
       c->launches += launch_search_r1(c->tab, sp, S, a - blo, b - blo, path, c->sms, c->d_blocks + used,
-                                      MAX_BLOCKS - used, &nb, c->d_work, c->h_work, c->work_bytes, next_stream());
+                                      MAX_BLOCKS - used, &nb, c->d_work, c->h_work, c->work_bytes, next_stream(), ext);
       used += nb;
       if (b < hi) {
         c->launches += launch_search_generic(c->tab, sp, b, hi, path, c->model, wide, c->sms, c->d_blocks + used,
@@ -664,6 +673,59 @@ static int search_impl(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, u64 beg
   h_tie[1] = c->h_result->index;
   h_tie[2] = c->h_result->evaluated;
   memcpy(h_rec, c->h_result->part, wide ? 32 : 16);
+  return AUTOPIPE_OK;
+}
+
+// Row e, cross-shard bound: the seed half of a search. For every r = 1 block of [begin, end) with at
+// least 2^26 candidates, the seed kernel finds a good candidate of the shard; its exact T is
+// min-folded into *d_theta (set to UINT64_MAX first). Nothing else runs: no sweep, no result.
+extern "C" int autopipe_search_seed_async(autopipe_ctx *c, uint32_t s_min, uint32_t s_max, uint32_t flags,
+                                          uint64_t begin, uint64_t end, uint64_t *d_theta, void *stream) {
+  if (!c) return AUTOPIPE_E_INVAL;
+  c->err[0] = 0;
+  if (!d_theta) return fail(c, AUTOPIPE_E_INVAL, "NULL theta pointer");
+  if (!c->has_state) return fail(c, AUTOPIPE_E_STATE, "seed before set_state");
+  int rc = check_space_args(c, s_min, s_max, flags, false);
+  if (rc) return rc;
+  SearchSpace sp;
+  if (!build_space(c, s_min, s_max, flags, sp)) return fail(c, AUTOPIPE_E_OVERFLOW, "space exceeds 2^64");
+  const u64 total = sp.off[s_max + 1];
+  if (end > total) end = total;
+  cudaStream_t st = (cudaStream_t)stream;
+  cudaError_t e = cudaMemsetAsync(d_theta, 0xFF, sizeof(u64), st);
+  if (e != cudaSuccess) return cuda_fail(c, e, "seed");
+  if (!c->ev_hseed) {
+    e = cudaEventCreateWithFlags(&c->ev_hseed, cudaEventDisableTiming);
+    if (e != cudaSuccess) return cuda_fail(c, e, "seed event");
+  }
+  if (c->hseed_pending) {  // the pinned slots may still feed the previous seed call's copies
+    cudaEventSynchronize(c->ev_hseed);
+    c->hseed_pending = false;
+  }
+  const size_t half = c->work_bytes / 2;
+  void *dw = (unsigned char *)c->d_work + half, *hw = (unsigned char *)c->h_work + half;
+  for (int S = (int)s_min; S <= (int)s_max && begin < end; ++S) {
+    const u64 blo = sp.off[S], r1hi = blo + sp.ncut[S];
+    const bool r1 = S >= 5 && S <= MAXS && (!(flags & AUTOPIPE_USE_ALL_WORKERS) || (int)c->N == S) &&
+                    c->model.sched == SCHED_PIPEDREAM;
+    const u64 a = begin > blo ? begin : blo, b = end < r1hi ? end : r1hi;
+    if (!r1 || a >= b) continue;
+    R1Ext ext;
+    ext.theta_out = (u64 *)d_theta;
+    int nb = 0;
+    c->launches += launch_search_r1(c->tab, sp, S, a - blo, b - blo, 0, c->sms, c->d_blocks, MAX_BLOCKS, &nb, dw, hw,
+                                    half, st, ext);
+  }
+  cudaEventRecord(c->ev_hseed, st);
+  c->hseed_pending = true;
+  e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(c, e, "seed kernel launch");
+  return AUTOPIPE_OK;
+}
+
+extern "C" int autopipe_set_search_bound(autopipe_ctx *c, const uint64_t *d_bound) {
+  if (!c) return AUTOPIPE_E_INVAL;
+  c->d_bound = (const u64 *)d_bound;
   return AUTOPIPE_OK;
 }
 

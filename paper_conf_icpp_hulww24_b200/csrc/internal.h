@@ -32,11 +32,18 @@ int launch_eval(const DevTables &g, const void *recs, u64 count, bool wide, u64 
 // into out[out_offset ...] and returns the number of blocks used via *nblocks.
 int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, u64 end, int path32, const ModelP &m,
                           bool wide, int sms, BlockOut *out, int max_blocks, int *nblocks, cudaStream_t st);
+// Cross-shard bound of the r = 1 sweep (row e). bound: device word the sweep's shared theta starts at
+// (replaces the shard's own seed); theta_out: seed only, no sweep — the shard's seed T is atomicMin'ed
+// into this device word.
+struct R1Ext {
+  const u64 *bound = nullptr;
+  u64 *theta_out = nullptr;
+};
 // Fast search over the r = 1 block of one S (all stages on one worker; SPEC.md §5, rho = 0),
 // restricted to the cut ranks [k_begin, k_end). path32 selects the 32-bit tables.
 int launch_search_r1(const DevTables &g, const SearchSpace &sp, int S, u64 k_begin, u64 k_end,
                      int path32, int sms, BlockOut *out, int max_blocks, int *nblocks, void *work,
-                     void *pinned, size_t work_bytes, cudaStream_t st);
+                     void *pinned, size_t work_bytes, cudaStream_t st, const R1Ext &ext = R1Ext());
 // rec_bytes: record bytes written into out->part (32 for the context's own ResultDev; 16 or 32 when
 // out is the caller's autopipe_result / autopipe_result_w)
 int launch_finalize(const BlockOut *in, int n, const SearchSpace &sp, ResultDev *out, bool wide, cudaStream_t st,

@@ -907,12 +907,25 @@ static u64 count_less(int x, int k, const int *t) {
   return cnt;
 }
 
+// Cross-shard bound (row e): k_theta_out folds a shard's seed T into a caller's device word (atomicMin;
+// the caller min-reduces it over ranks), k_theta_in lowers a sweep's shared theta to such a word
+// before the sweep starts. theta is always the exact T of a real candidate of some shard.
+__global__ void k_theta_out(const R1Header *hdr, u64 *theta) {
+  if (threadIdx.x == 0) atomicMin((unsigned long long *)theta, (unsigned long long)hdr->theta);
+}
+__global__ void k_theta_in(R1Header *hdr, const u64 *bound) {
+  if (threadIdx.x == 0) {
+    const u64 b = *bound;
+    if (b < hdr->theta) hdr->theta = b;
+  }
+}
+
 // prep = false: the schedule for this (S, shard) was just built and copied by the launch of the other
 // path (gate >= 0 launches both); reuse it
 template <int S, typename T>
 static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u64 k_end, int sms,
                        BlockOut *out, int max_blocks, int *nblocks, void *work, void *pinned, size_t work_bytes,
-                       cudaStream_t st, int gate, bool prep) {
+                       cudaStream_t st, int gate, bool prep, const R1Ext &ext) {
   constexpr int P = S - 4, NT = sizeof(T) == 4 ? R1_NT32 : R1_NT64;
   const int L = (int)g.L, n = L - 1, k = S - 1;
   unsigned char *hbuf = (unsigned char *)pinned + (size_t)S * 16384;
@@ -1027,7 +1040,18 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
   // the schedule is staged in the context's pinned buffer (one 16 KB slot per S, like the device work
   // area), so the copy is a true async DMA and never waits for earlier work on the stream
   int launched = 1;  // the sweep kernel below, + the seed kernel
-  if (prep) {
+  if (ext.theta_out) {  // seed only (autopipe_search_seed_async): the seed's T into the caller's word
+    cudaMemcpyAsync(work, hbuf, hbytes, cudaMemcpyHostToDevice, st);
+    if (k_end - k_begin < (1ull << 26)) return 0;
+    k_seed_r1<S><<<1, 160, 0, st>>>(g, (R1Header *)work);
+    k_theta_out<<<1, 32, 0, st>>>((const R1Header *)work, ext.theta_out);
+    return 2;
+  }
+  if (prep && ext.bound) {  // a bound from every shard's seed replaces this shard's own seed
+    cudaMemcpyAsync(work, hbuf, hbytes, cudaMemcpyHostToDevice, st);
+    k_theta_in<<<1, 32, 0, st>>>((R1Header *)work, ext.bound);
+    ++launched;
+  } else if (prep) {
     cudaMemcpyAsync(work, hbuf, hbytes, cudaMemcpyHostToDevice, st);
     // before the sweep, on its stream. (Beside it, on a stream of its own with a block slot left free,
     // it came too late for the 32-bit C4a search: 3.08 ms against 2.85.) Experiment knob: 0 = off.
@@ -1070,12 +1094,13 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
 
 template <typename T>
 static int launch_r1_s(int S, const DevTables &g, const SearchSpace &sp, u64 a, u64 b, int sms, BlockOut *out,
-                       int mb, int *nb, void *w, void *pin, size_t wb, cudaStream_t st, int gate, bool prep) {
+                       int mb, int *nb, void *w, void *pin, size_t wb, cudaStream_t st, int gate, bool prep,
+                       const R1Ext &x) {
   switch (S) {
-    case 5: return launch_r1_t<5, T>(g, sp, a, b, sms, out, mb, nb, w, pin, wb, st, gate, prep);
-    case 6: return launch_r1_t<6, T>(g, sp, a, b, sms, out, mb, nb, w, pin, wb, st, gate, prep);
-    case 7: return launch_r1_t<7, T>(g, sp, a, b, sms, out, mb, nb, w, pin, wb, st, gate, prep);
-    case 8: return launch_r1_t<8, T>(g, sp, a, b, sms, out, mb, nb, w, pin, wb, st, gate, prep);
+    case 5: return launch_r1_t<5, T>(g, sp, a, b, sms, out, mb, nb, w, pin, wb, st, gate, prep, x);
+    case 6: return launch_r1_t<6, T>(g, sp, a, b, sms, out, mb, nb, w, pin, wb, st, gate, prep, x);
+    case 7: return launch_r1_t<7, T>(g, sp, a, b, sms, out, mb, nb, w, pin, wb, st, gate, prep, x);
+    case 8: return launch_r1_t<8, T>(g, sp, a, b, sms, out, mb, nb, w, pin, wb, st, gate, prep, x);
   }
   *nb = 0;
   return 0;
@@ -1083,20 +1108,26 @@ static int launch_r1_s(int S, const DevTables &g, const SearchSpace &sp, u64 a, 
 
 int launch_search_r1(const DevTables &g, const SearchSpace &sp, int S, u64 k_begin, u64 k_end, int path32,
                      int sms, BlockOut *out, int max_blocks, int *nblocks, void *work, void *pinned,
-                     size_t work_bytes, cudaStream_t st) {
+                     size_t work_bytes, cudaStream_t st, const R1Ext &ext) {
+  if (ext.theta_out) {  // seed only: no sweep, the 64-bit tables serve either path
+    *nblocks = 0;
+    return launch_r1_s<u64>(S, g, sp, k_begin, k_end, sms, out, max_blocks, nblocks, work, pinned, work_bytes, st,
+                            -1, true, ext);
+  }
   if (path32 == 1)
     return launch_r1_s<u32>(S, g, sp, k_begin, k_end, sms, out, max_blocks, nblocks, work, pinned, work_bytes, st,
-                            -1, true);
+                            -1, true, ext);
   if (path32 == 0)
     return launch_r1_s<u64>(S, g, sp, k_begin, k_end, sms, out, max_blocks, nblocks, work, pinned, work_bytes, st,
-                            -1, true);
+                            -1, true, ext);
   // path unknown on the host (state set from device memory, asynchronous search): both paths, each
   // gated on the state kernel's choice; one schedule serves both
   int n32 = 0, n64 = 0;
-  int k = launch_r1_s<u32>(S, g, sp, k_begin, k_end, sms, out, max_blocks, &n32, work, pinned, work_bytes, st, 1, true);
+  int k = launch_r1_s<u32>(S, g, sp, k_begin, k_end, sms, out, max_blocks, &n32, work, pinned, work_bytes, st, 1, true,
+                           ext);
   if (n32 > 0)
     k += launch_r1_s<u64>(S, g, sp, k_begin, k_end, sms, out + n32, max_blocks - n32, &n64, work, pinned, work_bytes,
-                          st, 0, false);
+                          st, 0, false, ext);
   *nblocks = n32 + n64;
   return k;
 }

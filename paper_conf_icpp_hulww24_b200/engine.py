@@ -242,6 +242,29 @@ class Engine:
                        self._stream(stream)))
         return out
 
+    # -- row e: the cross-shard bound (autopipe_search_seed_async / autopipe_set_search_bound) --
+    def search_seed_async(self, s_min: int, s_max: int, flags: int = 0, begin: int = 0,
+                          end: Optional[int] = None, out: Optional[torch.Tensor] = None, stream=None) -> torch.Tensor:
+        """The shard's seed T (exact T of one of its candidates) as a device int64 [1] tensor holding a
+        uint64 (UINT64_MAX when no r = 1 block of the shard is seeded); min-reduce it over the ranks
+        and pass it to `set_search_bound`."""
+        if out is None:
+            out = torch.empty(1, dtype=torch.int64, device=self.device)
+        if out.numel() != 1 or out.element_size() != 8 or out.device != self.device:
+            raise ValueError("out must be one 8-byte element on %s" % self.device)
+        e = U64_MAX if end is None else int(end)
+        self._check(lib.autopipe_search_seed_async(self._h, s_min, s_max, flags, int(begin), e,
+                                                   ctypes.c_void_p(out.data_ptr()), self._stream(stream)))
+        return out
+
+    def set_search_bound(self, bound: Optional[torch.Tensor]) -> None:
+        """Later searches start their r = 1 sweeps from the device word `bound` (None clears it); the
+        tensor is kept alive while it is set."""
+        if bound is not None and (bound.device != self.device or bound.element_size() != 8):
+            raise ValueError("bound must be one 8-byte element on %s" % self.device)
+        self._bound = bound
+        self._check(lib.autopipe_set_search_bound(self._h, ctypes.c_void_p(bound.data_ptr() if bound is not None else 0)))
+
     # -- NEXT row f1: the two-worker neighbourhood (PAPER.md:896-906) ------------------------
     def neighbourhood(self, current: bytes, capacity: int = 1 << 15, stream=None) -> torch.Tensor:
         """All partitions differing from `current` in one or two workers' layer sets (uint8 [n, 16])."""

@@ -173,3 +173,71 @@ def test_wide_sharded_search_reduced(eng):
         outs = [eng.search_optimum_async(1, 10, begin=b[i], end=b[i + 1]) for i in range(G)]
         got = result_from_bytes(reduce_results(torch.stack(outs)))
         assert _tuple(got) == _tuple(want)
+
+
+def _bounded_shards(eng, G, bounds, s_min, s_max):
+    """Row e with the cross-shard bound, G shards on one GPU: seed every shard, min-reduce the seeds
+    (what NCCL all_reduce MIN does across ranks), search every shard under the bound, reduce."""
+    from paper_conf_icpp_hulww24_b200 import reduce_results
+    seeds = torch.stack([eng.search_seed_async(s_min, s_max, begin=bounds[i], end=bounds[i + 1]).clone()
+                         for i in range(G)])
+    u = seeds.cpu().numpy().view(np.uint64).ravel()
+    theta = torch.tensor(np.array([u.min()], dtype=np.uint64).view(np.int64), device=DEV)
+    eng.set_search_bound(theta)
+    try:
+        outs = [eng.search_optimum_async(s_min, s_max, begin=bounds[i], end=bounds[i + 1]) for i in range(G)]
+        red = reduce_results(torch.stack(outs))
+    finally:
+        eng.set_search_bound(None)
+    return int(u.min()), u, outs, red
+
+
+@pytest.mark.parametrize("kind", ["a-nvlink", "b"])
+def test_gpt96_cross_shard_bound(eng, kind):
+    """Row e, cross-shard bound: 8 cost-balanced shards of C(95,7), each seeded, the seeds' minimum
+    as every shard's starting bound. The reduction = the oracle's parametric DP optimum with every
+    candidate counted; each seed is the exact T of a candidate of its shard (>= the optimum); a shard
+    whose result is kept has its own exact minimum (= the unbounded search of that shard)."""
+    from paper_conf_icpp_hulww24_b200 import result_from_bytes
+    from paper_conf_icpp_hulww24_b200.distributed import balanced_bounds
+    prof, st = W.gpt96(), W.gpt_state(kind)
+    eng.load(prof, st)
+    T, idx = optimum(prof, st, 8, 8)[:2]
+    b = balanced_bounds(96, 8, 8, 8, 0, 8)
+    theta, seeds, outs, red = _bounded_shards(eng, 8, b, 8, 8)
+    got = result_from_bytes(red)
+    assert (got.time_ns, got.index, got.evaluated) == (T, idx, comb(95, 7))
+    assert T <= theta < U64_MAX and all(s >= T for s in seeds)
+    for i in range(8):
+        r = result_from_bytes(outs[i])
+        assert r.evaluated == b[i + 1] - b[i]
+        if r.time_ns <= theta:
+            want = eng.search_optimum(8, 8, begin=b[i], end=b[i + 1])
+            assert _tuple(r) == _tuple(want)
+        else:
+            assert r.index == U64_MAX or r.time_ns > theta
+    # the bound cleared: a shard search is unbounded again
+    want = eng.search_optimum(8, 8, begin=b[7], end=b[8])
+    assert _tuple(_async(eng, 8, 8, begin=b[7], end=b[8])) == _tuple(want)
+
+
+def test_cross_shard_bound_small_spaces_and_device_state(eng):
+    """Spaces whose r = 1 blocks are too small to seed leave the bound at UINT64_MAX (no filtering);
+    a device state (gated paths) under a bound gives the same optimum."""
+    from paper_conf_icpp_hulww24_b200 import result_from_bytes
+    from paper_conf_icpp_hulww24_b200.distributed import balanced_bounds
+    prof, st = W.vgg16(), W.vgg_state()
+    eng.load(prof, st)
+    want = eng.search_optimum(1, 8)
+    b = balanced_bounds(prof.L, 8, 1, 8, 0, 3)
+    theta, _, _, red = _bounded_shards(eng, 3, b, 1, 8)
+    assert theta == U64_MAX
+    assert _tuple(result_from_bytes(red)) == _tuple(want)
+    prof, st = W.gpt96(), W.gpt_state("b")
+    eng.load_profile(prof.O, prof.G, prof.P)
+    eng.set_state_device(_dev(st.f), _dev(st.b), _dev(st.tau))
+    T, idx = optimum(prof, st, 8, 8)[:2]
+    b = balanced_bounds(96, 8, 8, 8, 0, 4)
+    _, _, _, red = _bounded_shards(eng, 4, b, 8, 8)
+    got = result_from_bytes(red)
+    assert (got.time_ns, got.index, got.evaluated) == (T, idx, comb(95, 7))
