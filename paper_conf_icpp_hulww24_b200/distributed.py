@@ -76,6 +76,22 @@ def minloc_device(res: torch.Tensor, group=None, reduce_fn: Optional[Callable] =
     return (reduce_fn or reduce_results)(gathered)
 
 
+def bound_allreduce(seed: torch.Tensor, group=None) -> torch.Tensor:
+    """Row e, cross-shard bound: the minimum over the ranks of one uint64 seed word (held in an 8-byte
+    int64 tensor, as autopipe_search_seed_async writes it), in place. UINT64_MAX ("no seed") reads as
+    -1 in int64, so it is mapped to INT64_MAX for the MIN and back; real seeds are < 2^59."""
+    v = seed.view(torch.int64)
+    v.masked_fill_(v == -1, (1 << 63) - 1)
+    if dist.get_backend(group) == "nccl":
+        dist.all_reduce(v, op=dist.ReduceOp.MIN, group=group)
+    else:  # gloo: host copy
+        h = v.cpu()
+        dist.all_reduce(h, op=dist.ReduceOp.MIN, group=group)
+        v.copy_(h)
+    v.masked_fill_(v == (1 << 63) - 1, -1)
+    return seed
+
+
 def search_distributed(engine, s_min: int, s_max: int, flags: int = 0, group=None,
                        shard_search: Optional[Callable[[int, int], SearchResult]] = None,
                        device=None, balanced: bool = True,

@@ -74,6 +74,16 @@ def _worker(rank, world, port, q, case):
             out.append(minloc(*([(1 << 64) - 1, (1 << 64) - 1, 0], (3, 99, 4))[rank]))
             q.put((rank, out))
             return
+        if case == "bound":  # the cross-shard bound's 8-byte exchange (uint64 in int64 storage)
+            from paper_conf_icpp_hulww24_b200.distributed import bound_allreduce
+            res = []
+            for vals in ((416359965, 500000000), ((1 << 64) - 1, 480722219), ((1 << 64) - 1, (1 << 64) - 1)):
+                t = torch.tensor([vals[rank] - (1 << 64) if vals[rank] >= (1 << 63) else vals[rank]],
+                                 dtype=torch.int64)
+                bound_allreduce(t)
+                res.append(int(t.item()) & ((1 << 64) - 1))
+            q.put((rank, res))
+            return
         prof, st = W.toy(), W.toy_state()
         eng = _OracleEngine(prof.L, st.N)
 
@@ -183,3 +193,11 @@ def test_balanced_bounds_rejects_bad_arguments():
                  (96, 16, 1, 17, 0, 2)):
         with pytest.raises(ValueError):
             balanced_bounds(*args)
+
+
+def test_bound_allreduce_gloo_world2():
+    """Row e, cross-shard bound: the ranks' seed words min-reduced as uint64 (UINT64_MAX = no seed
+    never wins over a real seed, and stays UINT64_MAX when no rank has one)."""
+    out = _run(2, "bound")
+    for rank in (0, 1):
+        assert out[rank] == [416359965, 480722219, (1 << 64) - 1]
