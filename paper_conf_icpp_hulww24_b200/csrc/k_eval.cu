@@ -22,6 +22,14 @@ struct CurPart {  // the current partition of a rollout (16-byte or wide)
   int S, valid;
 };
 
+// resident blocks per SM for the wide (P16) GPipe / DAPPLE evals, whose 16-stage max-plus state
+// spills at the 2-block register budget
+#ifndef EVAL_MINB_WF
+#define EVAL_MINB_WF 2
+#endif
+#define EVAL_BLOCKS(MODE, P)                                                                    \
+  ((MODE == SCHED_PIPEDREAM && P::MS == 8) ? EVAL_MINB                                          \
+   : (P::MS == 16 && (MODE == SCHED_GPIPE || MODE == SCHED_DAPPLE)) ? EVAL_MINB_WF : 2)
 #ifndef EVAL_MINB
 #define EVAL_MINB 4
 #endif
@@ -57,7 +65,7 @@ __device__ __forceinline__ void score_one(const SmemTab &t, int L, int N, bool o
 // MODE: the schedule of the model (row f3; SCHED_PIPEDREAM is the 1F1B closed form of rows a4-a7).
 // Rec / P: 16-byte records (P8) or 32-byte wide records (P16, row f4).
 template <bool ROLLOUT, bool P32, int MODE, typename Rec, typename P>
-__global__ void __launch_bounds__(256, (MODE == SCHED_PIPEDREAM && P::MS == 8) ? EVAL_MINB : 2)
+__global__ void __launch_bounds__(256, EVAL_BLOCKS(MODE, P))
     k_eval(DevTables g, const Rec *__restrict__ recs, u64 count, u64 *__restrict__ out_t, u64 *__restrict__ out_sw,
            CurPart cur, ModelP m) {
   extern __shared__ u64 sm[];
@@ -86,7 +94,7 @@ static int grid_for(u64 count, int sms, int per_sm) {
 template <bool ROLLOUT, bool P32, int MODE, typename Rec, typename P>
 static void run_eval(int sms, size_t smem, cudaStream_t st, const DevTables &g, const void *recs, u64 count,
                      u64 *out_t, u64 *out_sw, const CurPart &cur, const ModelP &m) {
-  const int per_sm = (MODE == SCHED_PIPEDREAM && P::MS == 8) ? EVAL_MINB : 2;
+  const int per_sm = EVAL_BLOCKS(MODE, P);
   k_eval<ROLLOUT, P32, MODE, Rec, P><<<grid_for(count, sms, per_sm), 256, smem, st>>>(g, (const Rec *)recs, count,
                                                                                      out_t, out_sw, cur, m);
 }
