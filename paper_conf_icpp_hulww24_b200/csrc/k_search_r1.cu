@@ -97,7 +97,7 @@ struct R1Header {
   int hi_y, hi_x, hi_e;
   int ny;
   u32 counter;               // task counter (reset by the header copy before each launch)
-  u32 share;                 // 1: lanes share the grid's best T (theta below)
+  u32 share;                 // bits: 1 read / 2 publish the grid's best T (theta below); 4 per-task lane seeds always
   u64 theta;                 // smallest T found so far by any lane (UINT64_MAX at launch; atomicMin)
 };
 
@@ -402,7 +402,8 @@ __global__ void __launch_bounds__(NT, sizeof(T) == 4 ? R1_MINB32 : R1_MINB64) k_
     u64 pre = (r0 < r1 && P > 0) ? lex_unrank_smem(r0, P, y, Bn) : 0ull;
     // Seed: the lane's first row with the remaining layers split evenly over the last three stages.
     // Its exact T (and index) tightens theta before the sweep, so far fewer candidates reach the rare
-    // path while a lane's best is still poor (most visible when a GPU scans a small shard).
+    // path while a lane's best is still poor (most visible when a GPU scans a small shard). Only while
+    // the grid has no bound (a block too small for the seed kernel), unless share bit 4 forces it.
     if (r0 < r1 && ((hdr.share & 4) || tg == U64MAX)) {
       const int rem = L - 1 - y;  // layers y+1 .. L-1 for stages p-1, p, q
       int xs = y + rem / 3, es = y + (2 * rem) / 3;
@@ -940,7 +941,9 @@ static int launch_r1_t(const DevTables &g, const SearchSpace &sp, u64 k_begin, u
     R1YEntry *yt = (R1YEntry *)(hbuf + sizeof(R1Header));
     memset(h, 0, sizeof(*h));
     h->theta = env_u64("AUTOPIPE_R1_THETA0", U64MAX);  // experiment knob: a known bound (unset: none)
-    static const u64 share = env_u64("AUTOPIPE_R1_SHARE", 7);
+    // per-task lane seeds (bit 4) only while the grid has no bound yet: once the seed kernel has set
+    // theta they cost more than they tighten (B200: C(95,7) 2.81 -> 2.73 ms, 8-way shard 0.64 -> 0.58)
+    static const u64 share = env_u64("AUTOPIPE_R1_SHARE", 3);
     h->share = (u32)share;
     h->off = sp.off[S];
     for (int i = 0; i < P; ++i) {
