@@ -170,7 +170,11 @@ int autopipe_search_optimum_async(autopipe_ctx *ctx, uint32_t s_min, uint32_t s_
  *   2. the caller min-reduces d_theta over the ranks (NCCL all_reduce MIN, 8 bytes);
  *   3. autopipe_set_search_bound(ctx, d_theta): the context's later searches start every r = 1
  *      sweep from theta = *d_theta (read on the device when the sweep starts) instead of running
- *      their own seed; NULL clears it. The pointer must stay valid while it is set.
+ *      their own seed; NULL clears it. The pointer must stay valid while it is set. The bound is
+ *      keyed to the context's last seed call: it applies only to searches with that call's
+ *      (s_min, s_max, flags) while the profile, state and schedule are unchanged (any
+ *      load_profile / set_state[_device] / set_schedule retires it, and such searches run
+ *      unbounded). E_STATE if the context has no seed call on its current state.
  * A search under a bound returns the shard's exact (time_ns, index) minimum whenever that minimum
  * is <= *d_theta; otherwise its result is (UINT64_MAX, UINT64_MAX, evaluated, 0xFF...) or a
  * candidate with time_ns > *d_theta. Because *d_theta is the exact T of a real candidate of some

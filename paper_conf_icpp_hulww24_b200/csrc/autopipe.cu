@@ -66,12 +66,27 @@ struct autopipe_ctx {
   // row e, cross-shard bound: the device word later searches' r = 1 sweeps start from
   // (autopipe_set_search_bound), and the seed-only call's own schedule slots (upper half of the work
   // areas) with their own copy event
+  // The bound is valid only for the state, schedule and space it was seeded on: `gen` counts profile,
+  // state and schedule changes; a seed call records (gen, s_min, s_max, flags), set_search_bound
+  // copies that key, and a search applies the bound only when its own key matches.
   const u64 *d_bound = nullptr;
+  u64 gen = 0, seed_gen = ~0ull, bound_gen = ~0ull;
+  u32 seed_key[3] = {0, 0, 0}, bound_key[3] = {0, 0, 0};
   cudaEvent_t ev_hseed = nullptr;
   bool hseed_pending = false;
 };
 
 static char g_create_err[256] = "";
+
+const char *ap::experiment_knob(const char *name) {
+  static const bool on = [] {
+    const char *v = getenv("AUTOPIPE_EXPERIMENTS");
+    return v && v[0] == '1';
+  }();
+  if (!on) return nullptr;
+  const char *v = getenv(name);
+  return (v && *v) ? v : nullptr;
+}
 
 static int fail(autopipe_ctx *c, int code, const char *fmt, ...) {
   va_list ap_;
@@ -242,6 +257,7 @@ extern "C" int autopipe_load_profile(autopipe_ctx *c, uint32_t L, const uint64_t
   c->has_profile = true;
   c->has_state = false;
   c->path32 = 0;
+  ++c->gen;
   return AUTOPIPE_OK;
 }
 
@@ -303,6 +319,7 @@ extern "C" int autopipe_set_state(autopipe_ctx *c, uint32_t N, const uint64_t *f
   if (e != cudaSuccess) return cuda_fail(c, e, "state kernel launch");
   c->has_state = true;
   c->state_on_device = false;
+  ++c->gen;
   return AUTOPIPE_OK;
 }
 
@@ -325,6 +342,7 @@ extern "C" int autopipe_set_state_device(autopipe_ctx *c, uint32_t N, const uint
   if (e != cudaSuccess) return cuda_fail(c, e, "state kernel launch");
   c->has_state = true;
   c->state_on_device = true;  // overflow / path status is read from the device when first needed
+  ++c->gen;
   return AUTOPIPE_OK;
 }
 
@@ -374,6 +392,7 @@ extern "C" int autopipe_set_schedule(autopipe_ctx *c, uint32_t schedule, uint32_
   c->model.sync = sync;
   c->model.M = micro_batches;
   c->model.recompute = (flags & AUTOPIPE_RECOMPUTE) ? 1u : 0u;
+  ++c->gen;
   return AUTOPIPE_OK;
 }
 
@@ -617,7 +636,10 @@ static int search_impl(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, u64 beg
       const u64 a = lo, b = hi < r1hi ? hi : r1hi;
       int nb = 0;
       R1Ext ext;
-      ext.bound = c->d_bound;
+      // the bound only for the state, schedule and space it was seeded on
+      if (c->d_bound && c->bound_gen == c->gen && c->bound_key[0] == s_min && c->bound_key[1] == s_max &&
+          c->bound_key[2] == flags)
+        ext.bound = c->d_bound;
       c->launches += launch_search_r1(c->tab, sp, S, a - blo, b - blo, path, c->sms, c->d_blocks + used,
                                       MAX_BLOCKS - used, &nb, c->d_work, c->h_work, c->work_bytes, next_stream(), ext);
       used += nb;
@@ -647,7 +669,7 @@ static int search_impl(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, u64 beg
     cudaEventRecord(c->ev1[tslot], st);
     ++c->tcount;
   }
-  if (getenv("AUTOPIPE_R1_STATS") && used > 0) {  // diagnostics: rare-path decisions per search
+  if (experiment_knob("AUTOPIPE_R1_STATS") && used > 0) {  // diagnostics: rare-path decisions per search
     BlockOut *hb = new BlockOut[used];
     cudaMemcpyAsync(hb, c->d_blocks, sizeof(BlockOut) * used, cudaMemcpyDeviceToHost, st);
     cudaStreamSynchronize(st);
@@ -691,7 +713,10 @@ extern "C" int autopipe_search_seed_async(autopipe_ctx *c, uint32_t s_min, uint3
   if (!build_space(c, s_min, s_max, flags, sp)) return fail(c, AUTOPIPE_E_OVERFLOW, "space exceeds 2^64");
   const u64 total = sp.off[s_max + 1];
   if (end > total) end = total;
+  DeviceGuard dg(c->device);
   cudaStream_t st = (cudaStream_t)stream;
+  c->seed_gen = c->gen;
+  c->seed_key[0] = s_min; c->seed_key[1] = s_max; c->seed_key[2] = flags;
   cudaError_t e = cudaMemsetAsync(d_theta, 0xFF, sizeof(u64), st);
   if (e != cudaSuccess) return cuda_fail(c, e, "seed");
   if (!c->ev_hseed) {
@@ -725,7 +750,17 @@ extern "C" int autopipe_search_seed_async(autopipe_ctx *c, uint32_t s_min, uint3
 
 extern "C" int autopipe_set_search_bound(autopipe_ctx *c, const uint64_t *d_bound) {
   if (!c) return AUTOPIPE_E_INVAL;
+  c->err[0] = 0;
+  if (!d_bound) {
+    c->d_bound = nullptr;
+    c->bound_gen = ~0ull;
+    return AUTOPIPE_OK;
+  }
+  if (c->seed_gen != c->gen)
+    return fail(c, AUTOPIPE_E_STATE, "no seed call on the current profile, state and schedule");
   c->d_bound = (const u64 *)d_bound;
+  c->bound_gen = c->seed_gen;
+  memcpy(c->bound_key, c->seed_key, sizeof(c->bound_key));
   return AUTOPIPE_OK;
 }
 
@@ -1049,9 +1084,11 @@ u64 count_less_t(int x, int k, const int *t) {
 }
 inline double row_cost(int L, int y) {
   // AUTOPIPE_COST_{ROW,X,CAND}: experiment knobs for re-fitting the model (unset: the constants)
-  static const double cr = getenv("AUTOPIPE_COST_ROW") ? atof(getenv("AUTOPIPE_COST_ROW")) : (double)COST_ROW;
-  static const double cx = getenv("AUTOPIPE_COST_X") ? atof(getenv("AUTOPIPE_COST_X")) : (double)COST_X;
-  static const double cc = getenv("AUTOPIPE_COST_CAND") ? atof(getenv("AUTOPIPE_COST_CAND")) : (double)COST_CAND;
+  static const char *kr = experiment_knob("AUTOPIPE_COST_ROW"), *kx = experiment_knob("AUTOPIPE_COST_X"),
+                    *kc = experiment_knob("AUTOPIPE_COST_CAND");
+  static const double cr = kr ? atof(kr) : (double)COST_ROW;
+  static const double cx = kx ? atof(kx) : (double)COST_X;
+  static const double cc = kc ? atof(kc) : (double)COST_CAND;
   const double m = (double)(L - 2 - y);
   return cr + cx * (m - 1) + cc * m * (m - 1) / 2;
 }

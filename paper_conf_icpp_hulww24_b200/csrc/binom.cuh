@@ -1,5 +1,6 @@
 // binom.cuh — the combinatorial number system of SPEC.md §5 on the device (rows a3, a8).
-// Included once, by kernels.cu (the single device translation unit), which owns c_binom.
+// Included by the search translation units (k_search.cu, k_search_r1.cu); each holds its own copy
+// of the tables (internal linkage), filled by upload_binomials (internal.h) at context creation.
 #pragma once
 #include "common.cuh"
 
@@ -7,12 +8,12 @@ namespace ap {
 
 // Binomial coefficients C(n, k), n < 256, k <= 16 (saturated at UINT64_MAX: a space whose size
 // fits 64 bits only ever reads entries below its size), uploaded once per context by autopipe_create.
-__constant__ u64 c_binom[BINOM_N][BINOM_K];
+static __constant__ u64 c_binom[BINOM_N][BINOM_K];
 // the same table in global memory, for the kernels that stage rows of it into shared memory: threads
 // read different entries, which __constant__ would serialise; global loads coalesce (L2-resident)
-__device__ u64 g_binom[BINOM_N][BINOM_K];
+static __device__ u64 g_binom[BINOM_N][BINOM_K];
 
-void upload_binomials(const u64 (*tab)[BINOM_K]) {
+static void upload_binomials_tu(const u64 (*tab)[BINOM_K]) {
   cudaMemcpyToSymbol(c_binom, tab, sizeof(u64) * BINOM_N * BINOM_K);
   cudaMemcpyToSymbol(g_binom, tab, sizeof(u64) * BINOM_N * BINOM_K);
 }

@@ -52,7 +52,17 @@ int launch_finalize(const BlockOut *in, int n, const SearchSpace &sp, ResultDev 
 // layout), evaluated counts summed, the winner's record copied (autopipe_reduce_results)
 int launch_reduce_results(const void *in, unsigned n, int rec_bytes, void *out, cudaStream_t st);
 
-void upload_binomials(const u64 (*tab)[BINOM_K]);
+// the binomial tables of each search translation unit (binom.cuh)
+void upload_binomials_search(const u64 (*tab)[BINOM_K]);
+void upload_binomials_r1(const u64 (*tab)[BINOM_K]);
+inline void upload_binomials(const u64 (*tab)[BINOM_K]) {
+  upload_binomials_search(tab);
+  upload_binomials_r1(tab);
+}
+
+// Tuning knobs for experiments (AUTOPIPE_R1_*, AUTOPIPE_COST_*): read only when the environment sets
+// AUTOPIPE_EXPERIMENTS=1; otherwise nullptr, so the production path always runs the measured defaults.
+const char *experiment_knob(const char *name);
 
 // NEXT row f1: the two-worker neighbourhood (k_neigh.cu). Slots: (N + C(N,2)) * NEIGH_MAXOPT records.
 constexpr int NEIGH_MAXOPT = 544;  // >= (8+2) + (8+1) + 2*(255-1) options per changed-worker set

@@ -278,4 +278,6 @@ int launch_reduce_results(const void *in, unsigned n, int rec_bytes, void *out, 
   return 1;
 }
 
+void upload_binomials_search(const u64 (*tab)[BINOM_K]) { upload_binomials_tu(tab); }
+
 }  // namespace ap

@@ -76,7 +76,7 @@ constexpr int R1_MAXCHUNK = 16;
 #endif
 // 1: count rare-path decisions per block (BlockOut.pad, read by AUTOPIPE_R1_STATS)
 #ifndef R1_STATS
-#define R1_STATS 1
+#define R1_STATS 0
 #endif
 struct R1YEntry {      // one y value of the schedule (host-built shard arithmetic, SPEC.md §5)
   int y;               // e_{S-4}
@@ -868,8 +868,8 @@ __global__ void __launch_bounds__(160) k_seed_r1(DevTables gd, R1Header *hdr) {
 // ------------------------------------------------------------------------------------------------
 // host side: the task schedule (rows per y restricted to the shard) and the launch
 // ------------------------------------------------------------------------------------------------
-static u64 env_u64(const char *name, u64 dflt) {  // tuning knobs for experiments (unset: defaults)
-  const char *v = getenv(name);
+static u64 env_u64(const char *name, u64 dflt) {  // tuning knobs (AUTOPIPE_EXPERIMENTS=1 only)
+  const char *v = experiment_knob(name);
   return (v && *v) ? strtoull(v, nullptr, 10) : dflt;
 }
 
@@ -1134,5 +1134,7 @@ int launch_search_r1(const DevTables &g, const SearchSpace &sp, int S, u64 k_beg
   *nblocks = n32 + n64;
   return k;
 }
+
+void upload_binomials_r1(const u64 (*tab)[BINOM_K]) { upload_binomials_tu(tab); }
 
 }  // namespace ap

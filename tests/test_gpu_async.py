@@ -241,3 +241,36 @@ def test_cross_shard_bound_small_spaces_and_device_state(eng):
     _, _, _, red = _bounded_shards(eng, 4, b, 8, 8)
     got = result_from_bytes(red)
     assert (got.time_ns, got.index, got.evaluated) == (T, idx, comb(95, 7))
+
+
+def test_cross_shard_bound_retired_by_state_change(eng):
+    """A bound is keyed to the state and space it was seeded on: a bound from C4a (optimum below
+    C4b's) left set while the context moves to C4b must not filter C4b's search, nor a search of
+    another stage range; set_search_bound without a seed on the current state is E_STATE."""
+    from paper_conf_icpp_hulww24_b200 import AutopipeError
+    prof = W.gpt96()
+    sa, sb = W.gpt_state("a-nvlink"), W.gpt_state("b")
+    eng.load(prof, sa)
+    theta = eng.search_seed_async(8, 8).clone()
+    eng.set_search_bound(theta)
+    try:
+        Ta = optimum(prof, sa, 8, 8)[0]
+        Tb, ib = optimum(prof, sb, 8, 8)[:2]
+        assert int(theta.cpu().numpy().view(np.uint64)[0]) < Tb
+        eng.set_state(sb.f, sb.b, sb.tau)
+        got = _async(eng, 8, 8)
+        assert (got.time_ns, got.index, got.evaluated) == (Tb, ib, comb(95, 7))
+        # same state, another stage range: unbounded too
+        eng.set_state(sa.f, sa.b, sa.tau)
+        theta2 = eng.search_seed_async(8, 8).clone()
+        eng.set_search_bound(theta2)
+        got = _async(eng, 7, 7)
+        eng.set_search_bound(None)
+        want = _async(eng, 7, 7)
+        assert _tuple(got) == _tuple(want) and want.index != U64_MAX and want.time_ns >= Ta
+        eng.set_search_bound(theta2)
+        eng.set_state(sb.f, sb.b, sb.tau)
+        with pytest.raises(AutopipeError):
+            eng.set_search_bound(theta2)
+    finally:
+        eng.set_search_bound(None)

@@ -288,8 +288,8 @@ def test_near_overflow_values_exact(eng):
 
 
 # ------------------------------------------------------------------------------------------------
-# the hot r = 1 kernel (S >= 5): shards with partial rows and heavy ties, against the eval kernel
-# (itself bit-exact against the oracle) and the parametric DP
+# the hot r = 1 kernel (S >= 5): shards with partial rows and heavy ties, against the oracle's event
+# simulation of every candidate and the parametric DP
 # ------------------------------------------------------------------------------------------------
 
 def _all_records(L, N, smin, smax, flags):
@@ -310,7 +310,7 @@ def test_r1_kernel_shards_and_ties(eng, S, L, uniform):
         st.b = [[x * 1000 for x in row] for row in st.b]
     eng.load(prof, st)
     recs = _all_records(L, S, S, S, USE_ALL_WORKERS)       # exactly the r = 1 block
-    times = np.array(gpu_eval(eng, recs), dtype=object)
+    times = np.array(score_many(prof, st, recs), dtype=object)
     total = len(recs)
     full = eng.search_optimum(S, S, USE_ALL_WORKERS)
     T, idx, _ = optimum(prof, st, S, S, USE_ALL_WORKERS)
@@ -323,6 +323,37 @@ def test_r1_kernel_shards_and_ties(eng, S, L, uniform):
         want = (m, b + list(sub).index(m), e - b)
         r = eng.search_optimum(S, S, USE_ALL_WORKERS, begin=b, end=e)
         assert (r.time_ns, r.index, r.evaluated) == want, (b, e)
+
+
+@pytest.mark.parametrize("kind", ["a-nvlink", "b"])
+def test_gpt96_shard_boundaries_vs_oracle(eng, kind):
+    """Full size, in the launch configuration bench.py times: the 96-layer, 8-stage space split into
+    the 8 cost-balanced shards of the multi-GPU split. Around every inner shard boundary a window of
+    candidates straddling it is searched on the GPU as two pieces (the end of the left shard, the
+    start of the right one: partial rows on both sides) and each piece is compared with the oracle's
+    brute force over the same indices; the shard holding the optimum returns the parametric DP's
+    optimum."""
+    from paper_conf_icpp_hulww24_b200.distributed import balanced_bounds
+    prof, st = W.gpt96(), W.gpt_state(kind)
+    eng.load(prof, st)
+    total = comb(95, 7)
+    b = balanced_bounds(96, 8, 8, 8, 0, 8)
+    half = 1500
+    for i in range(1, 8):
+        lo, mid, hi = b[i] - half, b[i], b[i] + half
+        recs = records_of_indices(96, 8, 8, 8, 0, range(lo, hi))
+        ts = score_many(prof, st, recs)
+        for a, e in ((lo, mid), (mid, hi)):
+            sub = ts[a - lo:e - lo]
+            m = min(sub)
+            want = (m, a + sub.index(m), e - a)
+            r = eng.search_optimum(8, 8, begin=a, end=e)
+            assert (r.time_ns, r.index, r.evaluated) == want, (kind, i, a, e)
+    T, idx = optimum(prof, st, 8, 8)[:2]
+    k = next(i for i in range(8) if b[i] <= idx < b[i + 1])
+    r = eng.search_optimum(8, 8, begin=b[k], end=b[k + 1])
+    assert (r.time_ns, r.index, r.evaluated) == (T, idx, b[k + 1] - b[k])
+    assert sum(eng.search_optimum(8, 8, begin=b[j], end=b[j + 1]).evaluated for j in range(8)) == total
 
 
 def test_set_state_device_matches_host(eng):
@@ -380,15 +411,38 @@ def test_neighbourhood_matches_oracle(eng, seed):
 
 
 def test_neighbourhood_gpt96_and_local_search(eng):
-    """On the 96-layer space: the neighbourhood's best equals the minimum over the eval kernel of the
-    listed neighbours, and the paper's gradual migration from the even split strictly descends and
-    never beats the exhaustive optimum."""
+    """On the 96-layer space: every listed neighbour is a valid partition at distance 1 or 2 from
+    the current one by the oracle's definition (per-worker layer sets, reading F-1), none twice; the
+    listing contains every single-boundary move (each inner cut shifted to every position between
+    its neighbours: distance 2, enumerated independently here); a sample is scored by the oracle;
+    the best equals the minimum over the listed neighbours, and the paper's gradual migration from
+    the even split strictly descends and never beats the exhaustive optimum."""
+    from oracle.neighbourhood import layer_sets
     prof, st = W.gpt96(), W.gpt_state("b")
     eng.load(prof, st)
-    even = W.contiguous_record(96, [11, 23, 35, 47, 59, 71, 83], [1] * 8)
+    cuts = [11, 23, 35, 47, 59, 71, 83]
+    even = W.contiguous_record(96, cuts, [1] * 8)
     nb = eng.neighbourhood(even)
     t = [int(x) for x in as_u64_list(eng.eval_partitions(nb))]
     recs = [bytes(r) for r in nb.cpu().numpy()]
+    assert len(set(recs)) == len(recs)
+    base = layer_sets(parse_record(even, 96, 8), 96, 8)
+    for rec in recs:
+        q = parse_record(rec, 96, 8)
+        assert q is not None
+        d = sum(1 for x, y in zip(layer_sets(q, 96, 8), base) if x != y)
+        assert 1 <= d <= 2
+    have = set(recs)
+    for j in range(7):
+        lo = cuts[j - 1] + 1 if j > 0 else 0
+        hi = cuts[j + 1] - 1 if j < 6 else 94
+        for c in range(lo, hi + 1):
+            if c != cuts[j]:
+                moved = cuts[:j] + [c] + cuts[j + 1:]
+                assert W.contiguous_record(96, moved, [1] * 8) in have, (j, c)
+    rng = np.random.default_rng(41)
+    pick = sorted(int(x) for x in rng.choice(len(recs), size=min(200, len(recs)), replace=False))
+    assert score_many(prof, st, [recs[i] for i in pick]) == [t[i] for i in pick]
     best = min(zip(t, recs))
     r = eng.best_neighbour(even)
     assert (r.time_ns, r.partition, r.evaluated) == (best[0], best[1], len(recs))

@@ -138,15 +138,22 @@ def test_wide_search_equals_16_byte_search(eng, name, smax):
     assert encode_partition(pa, wide=True) == b.partition
 
 
-def test_testbed_search_ten_workers(eng):
-    """The 10-GPU testbed: exhaustive S <= 10 search of VGG-16 on 10 heterogeneous workers, its
-    optimum re-scored by the oracle, and a seeded sample of the space checked against it."""
-    prof = W.vgg16()
+@pytest.mark.parametrize("name", ["vgg16", "resnet50"])
+def test_testbed_search_ten_workers(eng, name):
+    """The 10-GPU testbed (row f4): exhaustive S <= 10, sum r <= 10 search of VGG-16 (14.3M
+    candidates) and ResNet-50 (12.6e9) on 10 heterogeneous workers, pinned to the oracle's parametric
+    DP (value and lexicographically-first index), the optimum re-scored by the oracle's event
+    simulation, and a seeded sample of the space checked against it."""
+    from oracle.param_dp import optimum
+    prof = W.profile(name)
     st = W.testbed_state(prof, seed=10)
     eng.load(prof, st)
     n = eng.count_candidates(1, 10)
     r = eng.search_optimum(1, 10)
-    assert r.evaluated == n and len(r.partition) == 32
+    T, idx = optimum(prof, st, 1, 10)[:2]
+    assert (r.time_ns, r.index, r.evaluated) == (T, idx, n)
+    assert len(r.partition) == 32
+    assert r.partition == encode_partition(decode(prof.L, 10, 1, 10, 0, idx), wide=True)
     assert score_many(prof, st, [r.partition]) == [r.time_ns]
     rng = np.random.default_rng(5)
     idx = sorted(int(x) for x in rng.choice(n, size=300, replace=False))
