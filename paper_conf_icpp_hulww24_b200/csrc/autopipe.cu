@@ -27,6 +27,9 @@ struct autopipe_ctx {
   bool state_on_device = false;  // last state came from device pointers: status not yet read
   u32 L = 0, N = 0;
   int path32 = 0;
+  // narrow eval path (status bit 2): every per-worker stage sum of f or of b < 2^31 - 16, activation
+  // and gradient bytes < 2^31 and tau < 2^32, so stage costs and shard overlaps are 32-bit
+  int narrow = 0;
   u64 launches = 0;
   u64 maxOG = 0, sumP = 0;
   u64 bound = 0;  // the state's bound on modelled sums (SPEC.md §7)
@@ -40,6 +43,11 @@ struct autopipe_ctx {
   void *d_work = nullptr;
   void *d_nslots = nullptr;  // neighbourhood slots (records), times, count
   u64 *d_ntimes = nullptr, *d_ncount = nullptr, *h_ncount = nullptr;
+  // chunk counters of the eval kernel's dynamic schedule: one slot per launch, round-robin, so
+  // launches on different streams never share one
+  static const int NCTR = 256;
+  u32 *d_ctr = nullptr;
+  u32 ctr_next = 0;
   void *h_work = nullptr;  // pinned mirror of d_work (r = 1 schedules)
   size_t work_bytes = 0;
   // pinned host staging
@@ -77,6 +85,8 @@ struct autopipe_ctx {
 };
 
 static char g_create_err[256] = "";
+
+static u32 *next_counter(autopipe_ctx *c) { return c->d_ctr + (c->ctr_next++ % autopipe_ctx::NCTR); }
 
 const char *ap::experiment_knob(const char *name) {
   static const bool on = [] {
@@ -150,7 +160,7 @@ extern "C" int autopipe_create(int cuda_device, autopipe_ctx **out) {
   // device tables, sized for the limits (L = 255, N = 8): a few hundred KB
   const size_t Lp1 = MAXL + 1, NL = (size_t)MAXNW * Lp1, TT = (size_t)TAUW * TAUW;
   const size_t words = 3 * NL + Lp1 + 2 * MAXL + TT + 2 * 7 * MAXL + 2;
-  const size_t words32 = NL + 2 * 7 * MAXL;
+  const size_t words32 = 3 * NL + 2 * 7 * MAXL;
   e = cudaMalloc(&c->d_tables, words * 8 + words32 * 4 + 64);
   if (e == cudaSuccess) e = cudaMalloc(&c->d_raw, (2 * MAXNW * MAXL + MAXL + TT) * 8);
   if (e == cudaSuccess) e = cudaMalloc(&c->d_blocks, sizeof(BlockOut) * MAX_BLOCKS);
@@ -161,6 +171,7 @@ extern "C" int autopipe_create(int cuda_device, autopipe_ctx **out) {
   if (e == cudaSuccess) e = cudaMalloc(&c->d_nslots, (size_t)NEIGH_ITEMS * NEIGH_MAXOPT * 16);
   if (e == cudaSuccess) e = cudaMalloc(&c->d_ntimes, (size_t)NEIGH_ITEMS * NEIGH_MAXOPT * 8);
   if (e == cudaSuccess) e = cudaMalloc(&c->d_ncount, 8);
+  if (e == cudaSuccess) e = cudaMalloc(&c->d_ctr, sizeof(u32) * autopipe_ctx::NCTR);
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_ncount, 8);
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_stage, (2 * MAXNW * MAXL + TT) * 8);
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_result, sizeof(ResultDev));
@@ -183,6 +194,8 @@ extern "C" int autopipe_create(int cuda_device, autopipe_ctx **out) {
   c->tab.status = p; p += 2;
   u32 *q = (u32 *)p;
   c->tab.PC32 = q; q += NL;
+  c->tab.PF32 = q; q += NL;
+  c->tab.PB32 = q; q += NL;
   c->tab.Z32 = q; q += 7 * MAXL;
   c->tab.LM32 = q; q += 7 * MAXL;
   e = cudaMemset(c->d_tables, 0, words * 8 + words32 * 4 + 64);
@@ -209,6 +222,7 @@ extern "C" void autopipe_destroy(autopipe_ctx *c) {
     if (c->d_nslots) cudaFree(c->d_nslots);
     if (c->d_ntimes) cudaFree(c->d_ntimes);
     if (c->d_ncount) cudaFree(c->d_ncount);
+    if (c->d_ctr) cudaFree(c->d_ctr);
     if (c->h_ncount) cudaFreeHost(c->h_ncount);
     if (c->h_stage) cudaFreeHost(c->h_stage);
     if (c->h_result) cudaFreeHost(c->h_result);
@@ -295,6 +309,20 @@ extern "C" int autopipe_set_state(autopipe_ctx *c, uint32_t N, const uint64_t *f
   if (bound >= LIMIT_TIME) return fail(c, AUTOPIPE_E_OVERFLOW, "modelled times reach 2^59 ns");
   const u128 bound32 = sumMax + (wideN ? 32 : 16) + (u128)(wideN ? 30 : 14) * maxXog;
   c->path32 = bound32 < LIMIT_TIME32 ? 1 : 0;
+  {
+    u128 sf = 0, sb = 0;
+    for (u32 l = 0; l < L; ++l) {
+      u64 mf = 0, mb = 0;
+      for (u32 w = 0; w < N; ++w) {
+        mf = umax(mf, (u64)fp[w * L + l]);
+        mb = umax(mb, (u64)bp[w * L + l]);
+      }
+      sf += mf;
+      sb += mb;
+    }
+    const u128 lim = ((u128)1 << 31) - 16;
+    c->narrow = (sf <= lim && sb <= lim && c->maxOG < (1ull << 31) && maxTau < (1ull << 32)) ? 1 : 0;
+  }
   c->bound = (u64)bound;
   DeviceGuard dg(c->device);
   cudaStream_t st = (cudaStream_t)stream;
@@ -355,6 +383,7 @@ static int sync_status(autopipe_ctx *c, cudaStream_t st) {
   if (e != cudaSuccess) return cuda_fail(c, e, "state status");
   c->state_on_device = false;
   c->path32 = (c->h_status[0] & 2) ? 1 : 0;
+  c->narrow = (c->h_status[0] & 4) ? 1 : 0;
   c->bound = c->h_status[1];
   if (c->h_status[0] & 1) {
     c->has_state = false;
@@ -417,9 +446,9 @@ static int eval_impl(autopipe_ctx *c, const void *d_parts, uint64_t count, bool 
   int rc = check_model(c, (cudaStream_t)stream);
   if (rc) return rc;
   // a state given in device memory has not been classified on the host yet: use the 64-bit path
-  const int p32 = c->state_on_device ? 0 : c->path32;
+  const int p32 = c->state_on_device ? 0 : (c->path32 | (c->narrow << 1));
   c->launches += launch_eval(c->tab, d_parts, count, wide, (u64 *)d_time_ns, nullptr, nullptr, nullptr, nullptr, p32,
-                             c->model, c->sms, (cudaStream_t)stream);
+                             c->model, c->sms, next_counter(c), (cudaStream_t)stream);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "eval kernel launch");
   return AUTOPIPE_OK;
@@ -870,9 +899,10 @@ static int rollout_impl(autopipe_ctx *c, const void *d_parts, uint64_t count, co
   DeviceGuard dg(c->device);
   int rc = check_model(c, (cudaStream_t)stream);
   if (rc) return rc;
-  const int p32 = c->state_on_device ? 0 : c->path32;
+  const int p32 = c->state_on_device ? 0 : (c->path32 | (c->narrow << 1));
   c->launches += launch_eval(c->tab, d_parts, count, wide, (u64 *)d_time_ns, (u64 *)d_switch_bytes,
-                             h_current ? &S : nullptr, cuts, masks, p32, c->model, c->sms, (cudaStream_t)stream);
+                             h_current ? &S : nullptr, cuts, masks, p32, c->model, c->sms, next_counter(c),
+                             (cudaStream_t)stream);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "rollout kernel launch");
   return AUTOPIPE_OK;
@@ -991,7 +1021,7 @@ extern "C" int autopipe_neighbourhood_best(autopipe_ctx *c, const autopipe_parti
   rc = neigh_prepare(c, h_current, nslots, st);
   if (rc) return rc;
   c->launches += launch_eval(c->tab, c->d_nslots, nslots, false, c->d_ntimes, nullptr, nullptr, nullptr, nullptr,
-                             c->path32, c->model, c->sms, st);
+                             c->path32, c->model, c->sms, next_counter(c), st);
   c->launches += launch_neigh_best(c->d_nslots, c->d_ntimes, nslots, c->d_result, st);
   cudaError_t e = cudaMemcpyAsync(c->h_result, c->d_result, sizeof(ResultDev), cudaMemcpyDeviceToHost, st);
   if (e == cudaSuccess) e = cudaStreamSynchronize(st);

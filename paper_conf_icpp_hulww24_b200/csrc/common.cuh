@@ -37,9 +37,12 @@ struct DevTables {
   u64 *Z;     // [7][L]    r = 1 boundary s (worker s -> s+1) cut after layer l: cf + cb   (row a2)
   u64 *LM;    // [7][L]    ... max(cf, cb)                                                (row a2)
   u32 *PC32;  // [N][L+1]  32-bit copies for the 32-bit search path (valid iff path32)
+  u32 *PF32;  // [N][L+1]  32-bit copies of PF, PB for the narrow eval path (valid iff status bit 2)
+  u32 *PB32;
   u32 *Z32;   // [7][L]
   u32 *LM32;  // [7][L]
-  u64 *status; // [2] written by the state kernel: [0] bit0 = overflow, bit1 = 32-bit path; [1] = bound
+  u64 *status; // [2] written by the state kernel: [0] bit0 = overflow, bit1 = 32-bit path,
+               // bit2 = narrow (per-worker stage sums < 2^31 - 16, O and G < 2^31, tau < 2^32); [1] = bound
 };
 
 // The model a scoring call evaluates (NEXT row f3, reading F-3; autopipe_set_schedule).
@@ -66,6 +69,13 @@ __device__ __forceinline__ u64 xfer(u64 bytes, u64 fs_per_byte) {
 // m = ceil(2^(63+l) / d), l = ceil(log2 d), q = mulhi(x, m) >> (l - 1); exact for every x < 2^63
 // (d = 1 is the identity). The multiplier is chosen once per divisor, hoisted out of the loops over
 // replicas and shards.
+struct __align__(16) DivEnt {  // DivR's multipliers for one divisor (see DivR and Div32)
+  u64 m;
+  u32 sh, Ms;
+  u32 m32, k32, pad0, pad1;
+};
+constexpr int DIVTAB_WORDS = 4 * (MAXNW + 1);  // u64 words of the table for d = 0..16 (entry 0 unused)
+
 template <int MAXD = 8>
 struct DivR {
   u64 m;
@@ -95,11 +105,41 @@ struct DivR {
       Ms = (d == 9u) ? 7282u : (d == 10u) ? 6554u : (d == 11u) ? 5958u : (d == 12u) ? 5462u
          : (d == 13u) ? 5042u : (d == 14u) ? 4682u : (d == 15u) ? 4370u : 4096u;
   }
+  // the same multipliers from a table of the 16 divisors staged in shared memory (stage_tables):
+  // one 16-byte shared load instead of the select chains above
+  __device__ __forceinline__ DivR(u32 d_, const DivEnt *tab) : d(d_) {
+    const DivEnt e = tab[d_];
+    m = e.m;
+    sh = e.sh;
+    Ms = e.Ms;
+  }
   __device__ __forceinline__ u64 div(u64 x) const { return d == 1u ? x : (__umul64hi(x, m) >> sh); }
   __device__ __forceinline__ u64 ceil(u64 x) const { return div(x + d - 1); }
   __device__ __forceinline__ u32 small(u32 k) const { return (k * Ms) >> 16; }
 };
 typedef DivR<8> Div8;
+
+// floor(x / d) for d in [1, 16] and 32-bit x < 2^31 (the narrow path: a state whose per-worker
+// stage sums stay below 2^31): m = ceil(2^(31 + c) / d) < 2^32 with c = ceil(log2 d),
+// q = mulhi32(x, m) >> (c - 1). Exact for every x < 2^31 (the error m d - 2^(31+c) < d <= 2^c);
+// tools/check_div32.py checks it exhaustively on the top of the range.
+struct Div32 {
+  u32 m, k, d;
+  __host__ __device__ __forceinline__ static void make(u32 d_, u32 &m_, u32 &k_) {
+    if (d_ <= 1u) { m_ = 0u; k_ = 0u; return; }
+    u32 c = 0;
+    while ((1u << c) < d_) ++c;
+    m_ = (u32)((((unsigned long long)1 << (31 + c)) + d_ - 1) / d_);
+    k_ = c - 1;
+  }
+  __device__ __forceinline__ Div32(u32 d_, const DivEnt *tab) : d(d_) {
+    m = tab[d_].m32;
+    k = tab[d_].k32;
+  }
+  __device__ __forceinline__ u32 div(u32 x) const { return d == 1u ? x : (__umulhi(x, m) >> k); }
+  __device__ __forceinline__ u32 ceil(u32 x) const { return div(x + d - 1); }
+};
+
 
 __device__ __forceinline__ int byte_at(u64 v, int i) { return (int)((v >> (8 * i)) & 0xFF); }
 

@@ -35,34 +35,91 @@ struct P16 {  // 32-byte wide records (row f4): cut bytes in c[0..1], 16-bit sta
   }
 };
 
-// Read-only view of the state tables staged in shared memory.
+// Read-only view of the state tables staged in shared memory. The narrow eval path stages 32-bit
+// copies of the per-worker prefixes (PF32, PB32) and of tau instead of PF, PB.
 struct SmemTab {
   const u64 *PF, *PB, *PP, *O, *G, *tau;
+  const u64 *ring;  // [256] slowest ring link of each worker set of N <= 8 (ascending ring order)
+  const u32 *PF32, *PB32, *tau32;
+  const DivEnt *dv;  // replica-count divisors d = 1..16 (DivR / Div32 multipliers)
   int L, Lp1;
 };
 
-// Number of u64 words the staged tables need: PF, PB (N x (L+1)), PP (L+1), O, G (L), tau (16 x 16).
+// Number of u64 words the staged tables need: the divisor table (17 x 32 B), PF, PB (N x (L+1)),
+// PP (L+1), O, G (L), tau (16 x 16); the narrow path stages PF32, PB32 and a 32-bit tau in about
+// the same space.
 __host__ __device__ __forceinline__ u32 smem_words(u32 L, u32 N) {
-  return 2u * N * (L + 1) + (L + 1) + 2u * L + (u32)(TAUW * TAUW);
+  return (u32)DIVTAB_WORDS + 2u * N * (L + 1) + (L + 1) + 2u * L + (u32)(TAUW * TAUW) + (u32)(TAUW * TAUW / 2) +
+         256u;
 }
 
 // Cooperative copy of the global tables into shared memory (every thread of the block calls it).
+template <bool NARROW = false>
 __device__ __forceinline__ SmemTab stage_tables(const DevTables &g, u64 *sm) {
   const u32 L = g.L, N = g.N, Lp1 = g.Lp1;
-  u64 *PF = sm, *PB = PF + N * Lp1, *PP = PB + N * Lp1, *O = PP + Lp1, *G = O + L, *tau = G + L;
-  for (u32 i = threadIdx.x; i < N * Lp1; i += blockDim.x) {
-    PF[i] = g.PF[i];
-    PB[i] = g.PB[i];
+  DivEnt *dt = (DivEnt *)sm;
+  if (threadIdx.x <= (unsigned)MAXNW) {
+    const u32 dd = threadIdx.x == 0 ? 1u : threadIdx.x;
+    const DivR<16> d(dd);
+    u32 m32, k32;
+    Div32::make(dd, m32, k32);
+    dt[threadIdx.x] = DivEnt{d.m, d.sh, d.Ms, m32, k32, 0u, 0u};
   }
+  sm += DIVTAB_WORDS;
+  SmemTab t;
+  u64 *PP, *O, *G, *tau;
+  if (NARROW) {
+    u32 *PF32 = (u32 *)sm, *PB32 = PF32 + N * Lp1;
+    PP = sm + (N * Lp1 + 1) / 2 * 2;  // 8-byte aligned after the two u32 tables
+    for (u32 i = threadIdx.x; i < N * Lp1; i += blockDim.x) {
+      PF32[i] = g.PF32[i];
+      PB32[i] = g.PB32[i];
+    }
+    t.PF32 = PF32; t.PB32 = PB32;
+    t.PF = t.PB = nullptr;
+  } else {
+    u64 *PF = sm, *PB = PF + N * Lp1;
+    PP = PB + N * Lp1;
+    for (u32 i = threadIdx.x; i < N * Lp1; i += blockDim.x) {
+      PF[i] = g.PF[i];
+      PB[i] = g.PB[i];
+    }
+    t.PF = PF; t.PB = PB;
+    t.PF32 = t.PB32 = nullptr;
+  }
+  O = PP + Lp1; G = O + L; tau = G + L;
+  u32 *tau32 = (u32 *)(tau + TAUW * TAUW);
   for (u32 i = threadIdx.x; i < Lp1; i += blockDim.x) PP[i] = g.PP[i];
   for (u32 i = threadIdx.x; i < L; i += blockDim.x) {
     O[i] = g.O[i];
     G[i] = g.G[i];
   }
-  for (u32 i = threadIdx.x; i < (u32)(TAUW * TAUW); i += blockDim.x) tau[i] = g.tau[i];
+  for (u32 i = threadIdx.x; i < (u32)(TAUW * TAUW); i += blockDim.x) {
+    const u64 v = g.tau[i];
+    tau[i] = v;
+    tau32[i] = (u32)v;  // meaningful on the narrow path only (tau < 2^32 there)
+  }
+  u64 *ring = (u64 *)(tau32 + TAUW * TAUW);
+  // ring[mask]: max over the ring W[0] -> W[1] -> ... -> W[0] (ascending) of tau, read from global
+  for (u32 msk = threadIdx.x; msk < 256u; msk += blockDim.x) {
+    u64 tr = 0;
+    if (__popc(msk) >= 2 && msk < (1u << (N < 8 ? N : 8))) {
+      const int first = __ffs(msk) - 1;
+      int prev = first;
+      u32 m = msk & (msk - 1);
+      while (m) {
+        const int w = __ffs(m) - 1;
+        m &= m - 1;
+        tr = umax(tr, g.tau[prev * TAUW + w]);
+        prev = w;
+      }
+      tr = umax(tr, g.tau[prev * TAUW + first]);
+    }
+    ring[msk] = tr;
+  }
   __syncthreads();
-  SmemTab t;
-  t.PF = PF; t.PB = PB; t.PP = PP; t.O = O; t.G = G; t.tau = tau;
+  t.PP = PP; t.O = O; t.G = G; t.tau = tau; t.tau32 = tau32; t.ring = ring;
+  t.dv = dt;
   t.L = (int)L; t.Lp1 = (int)Lp1;
   return t;
 }
@@ -73,14 +130,14 @@ __device__ __forceinline__ SmemTab stage_tables(const DevTables &g, u64 *sm) {
 // overlapping pairs in order; since the duration is monotone in overlap * tau, the walk keeps the
 // largest product and rounds once. MAXD = the largest replica count (8 or 16).
 template <int MAXD = 8>
-__device__ __forceinline__ u64 boundary_max(u64 A, u32 send, u32 recv, const u64 *tau) {
+__device__ __forceinline__ u64 boundary_max(u64 A, u32 send, u32 recv, const u64 *tau, const DivEnt *dvt) {
   const u32 rs = __popc(send), rr = __popc(recv);
   if (rs == 1 && rr == 1) {
     const int u = __ffs(send) - 1, v = __ffs(recv) - 1;
     return xfer(A, tau[u * TAUW + v]);
   }
   // shard boundaries floor(i A / r) = i q + floor(i rem / r) with A = q r + rem (rem < r <= 16, i <= 16)
-  const DivR<MAXD> ds(rs), dr(rr);
+  const DivR<MAXD> ds(rs, dvt), dr(rr, dvt);
   const u64 qs = ds.div(A), qr = dr.div(A);
   const u32 rems = (u32)(A - qs * rs), remr = (u32)(A - qr * rr);
   u64 best = 0;
@@ -109,7 +166,7 @@ __device__ __forceinline__ u64 boundary_max(u64 A, u32 send, u32 recv, const u64
 // Ring all-reduce of a replicated stage (row a6): 2(r-1) steps of a ceil(P_s/r)-byte chunk over the
 // slowest link of the ring W_s[0] -> W_s[1] -> ... -> W_s[0] (ascending worker order).
 template <int MAXD = 8>
-__device__ __forceinline__ u64 allreduce_time(u64 Ps, u32 mask, const u64 *tau) {
+__device__ __forceinline__ u64 allreduce_time(u64 Ps, u32 mask, const u64 *tau, const DivEnt *dvt) {
   const u32 r = __popc(mask);
   const int first = __ffs(mask) - 1;
   int prev = first;
@@ -122,7 +179,7 @@ __device__ __forceinline__ u64 allreduce_time(u64 Ps, u32 mask, const u64 *tau) 
     prev = w;
   }
   tr = umax(tr, tau[prev * TAUW + first]);
-  return 2ull * (u64)(r - 1) * xfer(DivR<MAXD>(r).ceil(Ps), tr);
+  return 2ull * (u64)(r - 1) * xfer(DivR<MAXD>(r, dvt).ceil(Ps), tr);
 }
 
 // Sharded parameter server of a replicated stage (row f3, reading F-3; PS scheme):
@@ -131,9 +188,9 @@ __device__ __forceinline__ u64 allreduce_time(u64 Ps, u32 mask, const u64 *tau) 
 // after another (and sends its pulls one after another); servers work in parallel:
 //   PS = max_v sum_{u != v} xfer(|shard_v|, tau[u][v]) + max_v sum_{u != v} xfer(|shard_v|, tau[v][u]).
 template <int MAXD = 8>
-__device__ __forceinline__ u64 ps_time(u64 Ps, u32 mask, const u64 *tau) {
+__device__ __forceinline__ u64 ps_time(u64 Ps, u32 mask, const u64 *tau, const DivEnt *dvt) {
   const u32 r = __popc(mask);
-  const DivR<MAXD> dv(r);
+  const DivR<MAXD> dv(r, dvt);
   const u64 q = dv.div(Ps);
   const u32 rem = (u32)(Ps - q * r);
   u64 push = 0, pull = 0, lo = 0;
@@ -160,8 +217,8 @@ __device__ __forceinline__ u64 ps_time(u64 Ps, u32 mask, const u64 *tau) {
 
 // Gradient synchronisation of a replicated stage (r >= 2) under the model's scheme.
 template <int MAXD = 8>
-__device__ __forceinline__ u64 sync_time(int sync, u64 Ps, u32 mask, const u64 *tau) {
-  return sync == SYNC_PS ? ps_time<MAXD>(Ps, mask, tau) : allreduce_time<MAXD>(Ps, mask, tau);
+__device__ __forceinline__ u64 sync_time(int sync, u64 Ps, u32 mask, const u64 *tau, const DivEnt *dvt) {
+  return sync == SYNC_PS ? ps_time<MAXD>(Ps, mask, tau, dvt) : allreduce_time<MAXD>(Ps, mask, tau, dvt);
 }
 
 // The full closed form (rows a4-a7) for one partition; S in [1, P::MS], the partition already validated.
@@ -193,7 +250,7 @@ __device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, const P
       const int e = (u == S - 1) ? t.L - 1 : p.cut(u);
       const u32 mask = p.mask(u);
       const u32 r = __popc(mask);
-      const DivR<P::MN> dv(r);
+      const DivR<P::MN> dv(r, t.dv);
       u32 m = mask;
       // first replica unconditionally; the loop only runs for replicated stages
       int w = __ffs(m) - 1;
@@ -213,13 +270,13 @@ __device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, const P
       const V X = (V)xm, Y = (V)(fm + bm);
       const V xs = BW ? (V)(xm * M) : (V)xm;
       T = T > xs ? T : xs;
-      if (r >= 2) TAR = umax(TAR, sync_time<P::MN>(sync, t.PP[e + 1] - t.PP[a], mask, t.tau));
+      if (r >= 2) TAR = umax(TAR, sync_time<P::MN>(sync, t.PP[e + 1] - t.PP[a], mask, t.tau, t.dv));
       if (u > 0) {
         // row a5: boundary u-1 (activation O[e_{u-1}] forward, gradient G[e_{u-1}+1] backward)
         const int eb = p.cut(u - 1);
         const u32 mp = p.mask(u - 1);
-        const u64 cf = boundary_max<P::MN>(t.O[eb], mp, mask, t.tau);
-        const u64 cb = boundary_max<P::MN>(t.G[eb + 1], mask, mp, t.tau);
+        const u64 cf = boundary_max<P::MN>(t.O[eb], mp, mask, t.tau, t.dv);
+        const u64 cb = boundary_max<P::MN>(t.G[eb + 1], mask, mp, t.tau, t.dv);
         const V Z = (V)(cf + cb);
         const V lm = BW ? (V)(umax(cf, cb) * M) : (V)umax(cf, cb);
         T = T > lm ? T : lm;
@@ -238,35 +295,158 @@ __device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, const P
   return umax((u64)T, TAR);
 }
 
+// ------------------------------------------------------------------------------------------------
+// The narrow path of the closed form (status bit 2; explicit-record scoring under PipeDream): every
+// per-worker stage sum of f or of b is < 2^31 - 16, so F' and B' are 32-bit ceil divisions by the
+// replica count (Div32: one 32-bit mulhi); activation and gradient bytes are < 2^31 and tau < 2^32,
+// so a shard overlap is 32-bit and overlap * tau one 32 x 32 -> 64-bit multiply. Same values as
+// eval_closed_form, bit for bit (the tests score every record both ways against the oracle).
+// ------------------------------------------------------------------------------------------------
+
+// Both transfers of one boundary: forward O[e] from the stage's replicas (send) to the next stage's
+// (recv), backward G[e+1] the other way. When the two byte counts are equal the shard overlaps are
+// the same pairs, so one merge walk serves both directions (tau[u][v] forward, tau[v][u] backward).
+template <int MAXD>
+__device__ __forceinline__ void walk_n(u32 A, u32 send, u32 recv, const u32 *tau32, const DivEnt *dvt, bool both,
+                                       u64 &bf, u64 &bb) {
+  const u32 rs = __popc(send), rr = __popc(recv);
+  const Div32 ds(rs, dvt), dr(rr, dvt);
+  const u32 Ms_s = dvt[rs].Ms, Ms_r = dvt[rr].Ms;
+  const u32 qs = ds.div(A), qr = dr.div(A);
+  const u32 rems = A - qs * rs, remr = A - qr * rr;
+  u32 i = 0, j = 0, lo_i = 0, lo_j = 0;
+  u32 hi_i = qs + ((rems * Ms_s) >> 16), hi_j = qr + ((remr * Ms_r) >> 16);
+  while (i < rs && j < rr) {
+    const u32 lo = lo_i > lo_j ? lo_i : lo_j, hi = hi_i < hi_j ? hi_i : hi_j;
+    if (hi > lo) {
+      const int u = __ffs(send) - 1, v = __ffs(recv) - 1;
+      bf = umax(bf, (u64)(hi - lo) * tau32[u * TAUW + v]);
+      if (both) bb = umax(bb, (u64)(hi - lo) * tau32[v * TAUW + u]);
+    }
+    const bool adv_i = hi_i <= hi_j, adv_j = hi_j <= hi_i;
+    if (adv_i) {
+      ++i; send &= send - 1;
+      lo_i = hi_i; hi_i = (i + 1) * qs + (((i + 1) * rems * Ms_s) >> 16);
+    }
+    if (adv_j) {
+      ++j; recv &= recv - 1;
+      lo_j = hi_j; hi_j = (j + 1) * qr + (((j + 1) * remr * Ms_r) >> 16);
+    }
+  }
+}
+
+template <int MAXD>
+__device__ __forceinline__ void boundary_both_n(u64 Af, u64 Ab, u32 ms, u32 mr, const u32 *tau32, const DivEnt *dvt,
+                                                u64 &cf, u64 &cb) {
+  if (__popc(ms) == 1 && __popc(mr) == 1) {
+    const int u = __ffs(ms) - 1, v = __ffs(mr) - 1;
+    cf = xfer_fs((u64)(u32)Af * tau32[u * TAUW + v]);
+    cb = xfer_fs((u64)(u32)Ab * tau32[v * TAUW + u]);
+    return;
+  }
+  u64 bf = 0, bb = 0;
+  if (Af == Ab) {
+    walk_n<MAXD>((u32)Af, ms, mr, tau32, dvt, true, bf, bb);
+  } else {
+    u64 dummy = 0;
+    walk_n<MAXD>((u32)Af, ms, mr, tau32, dvt, false, bf, dummy);
+    walk_n<MAXD>((u32)Ab, mr, ms, tau32, dvt, false, bb, dummy);
+  }
+  cf = xfer_fs(bf);
+  cb = xfer_fs(bb);
+}
+
+template <bool P32, typename P = P8>
+__device__ __forceinline__ u64 eval_closed_form_n(const SmemTab &t, int S, const P &p, int sync = SYNC_RING) {
+  constexpr int MS = P::MS;
+  typedef typename std::conditional<P32, u32, u64>::type V;
+  V acc[MS];
+  V T = 0;
+  u64 TAR = 0;
+#pragma unroll
+  for (int u = 0; u < MS; ++u) {
+    acc[u] = 0;
+    if (u < S) {
+      const int a = (u == 0) ? 0 : p.cut(u - 1) + 1;
+      const int e = (u == S - 1) ? t.L - 1 : p.cut(u);
+      const u32 mask = p.mask(u);
+      const u32 r = __popc(mask);
+      const Div32 dv(r, t.dv);
+      u32 m = mask;
+      int w = __ffs(m) - 1;
+      m &= m - 1;
+      u32 F = dv.ceil(t.PF32[w * t.Lp1 + e + 1] - t.PF32[w * t.Lp1 + a]);
+      u32 B = dv.ceil(t.PB32[w * t.Lp1 + e + 1] - t.PB32[w * t.Lp1 + a]);
+      u32 fm = F, bm = B, xm = F + B;
+      while (m) {  // row a4: split replicas, ceil(sum / r) per op
+        w = __ffs(m) - 1;
+        m &= m - 1;
+        F = dv.ceil(t.PF32[w * t.Lp1 + e + 1] - t.PF32[w * t.Lp1 + a]);
+        B = dv.ceil(t.PB32[w * t.Lp1 + e + 1] - t.PB32[w * t.Lp1 + a]);
+        fm = fm > F ? fm : F;
+        bm = bm > B ? bm : B;
+        xm = xm > F + B ? xm : F + B;
+      }
+      const V X = (V)xm, Y = (V)fm + (V)bm;
+      T = T > X ? T : X;
+      if (r >= 2) {
+        const u64 Ps = t.PP[e + 1] - t.PP[a];
+        if (P::MN == 8 && sync == SYNC_RING)  // row a6 with the per-state ring table
+          TAR = umax(TAR, 2ull * (u64)(r - 1) * xfer(DivR<8>(r, t.dv).ceil(Ps), t.ring[mask]));
+        else
+          TAR = umax(TAR, sync_time<P::MN>(sync, Ps, mask, t.tau, t.dv));
+      }
+      if (u > 0) {
+        const int eb = p.cut(u - 1);
+        u64 cf, cb;
+        boundary_both_n<P::MN>(t.O[eb], t.G[eb + 1], p.mask(u - 1), mask, t.tau32, t.dv, cf, cb);
+        const V Z = (V)(cf + cb);
+        const V lm = (V)umax(cf, cb);
+        T = T > lm ? T : lm;
+#pragma unroll
+        for (int s = 0; s < u; ++s) {
+          const V W = acc[s] + Z + X;
+          const V c = (W + (V)(u - s)) / (V)(u - s + 1);
+          T = T > c ? T : c;
+          acc[s] += Z + Y;
+        }
+      }
+      acc[u] = X;
+    }
+  }
+  return umax((u64)T, TAR);
+}
+
 // Decode + validate a 16-byte record (SPEC.md §2). Returns false for an invalid record.
 // lo = bytes 0..7 (S, cuts), hi = bytes 8..15 (stage of worker w in byte w).
 __device__ __forceinline__ bool decode_record(u64 lo, u64 hi, int L, int N, int &S, P8 &p) {
   S = (int)(lo & 0xFF);
   if (S < 1 || S > MAXS || S > N) return false;
-  p.cuts = lo >> 8;
-  bool ok = true;
-  int prev = -1;
-#pragma unroll
-  for (int i = 0; i < MAXS - 1; ++i) {
-    if (i < S - 1) {
-      const int e = byte_at(p.cuts, i);
-      ok &= (e > prev) & (e < L - 1);
-      prev = e;
-    }
-  }
+  const u64 cuts = lo >> 8;
+  p.cuts = cuts;
+  // cuts strictly increasing (byte i of `gt` is 0xFF iff e_{i+1} > e_i; the first S - 2 pairs
+  // count) and the last one < L - 1, with per-byte SIMD compares
+  const u64 nxt = cuts >> 8;
+  const u64 gt = (u64)__vcmpgtu4((u32)nxt, (u32)cuts) | ((u64)__vcmpgtu4((u32)(nxt >> 32), (u32)(cuts >> 32)) << 32);
+  const u64 need = S > 2 ? (~0ull >> (64 - 8 * (S - 2))) : 0ull;
+  bool ok = (gt & need) == need;
+  if (S > 1) ok &= (int)((cuts >> (8 * (S - 2))) & 0xFF) < L - 1;
+  // every worker byte is idle (0xFF) or a stage < S, and workers >= N are idle
+  const u32 h0 = (u32)hi, h1 = (u32)(hi >> 32), SS = (u32)S * 0x01010101u;
+  const u32 id0 = __vcmpeq4(h0, 0xFFFFFFFFu), id1 = __vcmpeq4(h1, 0xFFFFFFFFu);
+  ok &= ((id0 | __vcmpltu4(h0, SS)) & (id1 | __vcmpltu4(h1, SS))) == 0xFFFFFFFFu;
+  const u64 busy = ~(((u64)id1 << 32) | id0);
+  ok &= N >= 8 || (busy >> (8 * N)) == 0;
   u64 masks = 0;
 #pragma unroll
   for (int w = 0; w < MAXN; ++w) {
-    const int s = byte_at(hi, w);
-    if (s != 0xFF) {
-      ok &= (w < N) & (s < S);
-      if (s < S) masks |= 1ull << (8 * s + w);
-    }
+    const u32 s = (u32)byte_at(hi, w);
+    masks |= (s < (u32)S) ? 1ull << (8 * s + w) : 0ull;
   }
   p.masks = masks;
-#pragma unroll
-  for (int s = 0; s < MAXS; ++s)
-    if (s < S) ok &= byte_at(masks, s) != 0;
+  // every stage s < S has a worker (byte s of masks nonzero)
+  const u64 empty = (u64)__vcmpeq4((u32)masks, 0u) | ((u64)__vcmpeq4((u32)(masks >> 32), 0u) << 32);
+  ok &= (empty & (~0ull >> (64 - 8 * S))) == 0;
   return ok;
 }
 

@@ -25,9 +25,11 @@ int launch_build_state(const DevTables &g, const u64 *fp, const u64 *bp, const u
                        cudaStream_t st);
 // Explicit records, 16-byte (wide = false) or 32-byte (row f4). cur_cuts / cur_masks: the current
 // partition's packed parts (1 and 1 words, or 2 and 4 words for wide), or cur_S = nullptr.
+// counter: a device word the launch resets (cudaMemsetAsync) and the kernel's warps draw chunks from.
+// path32: bit 0 = the state's 32-bit path, bit 1 = its narrow path (status bit 2; PipeDream only).
 int launch_eval(const DevTables &g, const void *recs, u64 count, bool wide, u64 *out_t, u64 *out_sw,
                 const int *cur_S, const u64 *cur_cuts, const u64 *cur_masks, int path32, const ModelP &m, int sms,
-                cudaStream_t st);
+                u32 *counter, cudaStream_t st);
 // Generic exhaustive search over [begin, end) (any S, any composition); writes one BlockOut per block
 // into out[out_offset ...] and returns the number of blocks used via *nblocks.
 int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, u64 end, int path32, const ModelP &m,

@@ -1,11 +1,12 @@
 // k_eval.cu — batched scoring of explicit partition records (autopipe_eval_partitions) and RL
 // rollout rewards (autopipe_rollout_rewards). Rows a4-a8 for explicit records.
 //
-// Launch: a persistent grid (one wave of resident 256-thread blocks) striding over chunks of 1024
-// records. Each block stages the state tables into shared memory once (PF, PB, PP, O, G, tau), loads
-// a chunk with coalesced 128-bit loads (ld.global.nc), sorts it by shape in shared memory (a
-// counting sort over 64 buckets), and every thread scores records of one shape: the closed form of
-// SPEC.md §4 in registers, one 8-byte store per output at the record's position.
+// Launch: a persistent grid (one wave of resident 256-thread blocks). Each block stages the state
+// tables into shared memory once (PF, PB, PP, O, G, tau, the divisor table); then every warp on its
+// own takes chunks of 256 records (128 wide ones) from a global counter, loads them with coalesced
+// 128-bit loads (ld.global.nc), counting-sorts them by shape in its slice of shared memory
+// (sortchunk.cuh) and scores them 32 at a time in shape order: the closed form of SPEC.md §4 in
+// registers, one 8-byte store per output at the record's position.
 // Invalid records (SPEC.md §2) score UINT64_MAX and never fail the batch.
 #include <cstring>
 
@@ -33,10 +34,7 @@ struct CurPart {  // the current partition of a rollout (16-byte or wide)
 #ifndef EVAL_MINB
 #define EVAL_MINB 4
 #endif
-// 1: each block scores its records in chunks sorted by shape (sortchunk.cuh)
-#ifndef EVAL_SORT
-#define EVAL_SORT 1
-#endif
+constexpr int EVAL_NT = 256;
 // Decode + validate + score one record; Rec16 -> P8 (16-byte records), Rec32 -> P16 (wide, row f4).
 __device__ __forceinline__ bool decode_any(const Rec16 &r, int L, int N, int &S, P8 &p) {
   return decode_record((u64)r.a.x | ((u64)r.a.y << 32), (u64)r.a.z | ((u64)r.a.w << 32), L, N, S, p);
@@ -47,7 +45,7 @@ __device__ __forceinline__ bool decode_any(const Rec32 &r, int L, int N, int &S,
 __device__ __forceinline__ const P8 &cur_part(const CurPart &c, const P8 *) { return c.p8; }
 __device__ __forceinline__ const P16 &cur_part(const CurPart &c, const P16 *) { return c.p16; }
 
-template <bool ROLLOUT, bool P32, int MODE, typename P, typename Rec>
+template <bool ROLLOUT, bool P32, int MODE, bool NARROW, typename P, typename Rec>
 __device__ __forceinline__ void score_one(const SmemTab &t, int L, int N, bool overflow, const Rec &r, u64 i,
                                           u64 *__restrict__ out_t, u64 *__restrict__ out_sw, const CurPart &cur,
                                           const ModelP &m) {
@@ -55,7 +53,8 @@ __device__ __forceinline__ void score_one(const SmemTab &t, int L, int N, bool o
   P p;
   u64 T = U64MAX, sw = U64MAX;
   if (!overflow && decode_any(r, L, N, S, p)) {
-    T = model_time<MODE, P32>(t, S, p, m);
+    if constexpr (NARROW) T = eval_closed_form_n<P32, P>(t, S, p, (int)m.sync);
+    else T = model_time<MODE, P32>(t, S, p, m);
     if (ROLLOUT) sw = switch_bytes(t, S, p, cur.S, cur_part(cur, (const P *)nullptr));
   }
   out_t[i] = T;
@@ -64,51 +63,69 @@ __device__ __forceinline__ void score_one(const SmemTab &t, int L, int N, bool o
 
 // MODE: the schedule of the model (row f3; SCHED_PIPEDREAM is the 1F1B closed form of rows a4-a7).
 // Rec / P: 16-byte records (P8) or 32-byte wide records (P16, row f4).
-template <bool ROLLOUT, bool P32, int MODE, typename Rec, typename P>
-__global__ void __launch_bounds__(256, EVAL_BLOCKS(MODE, P))
+// NARROW (PipeDream only): the 32-bit stage and shard arithmetic of eval_closed_form_n (status bit 2)
+template <bool ROLLOUT, bool P32, int MODE, typename Rec, typename P, bool NARROW = false>
+__global__ void __launch_bounds__(EVAL_NT, EVAL_BLOCKS(MODE, P))
     k_eval(DevTables g, const Rec *__restrict__ recs, u64 count, u64 *__restrict__ out_t, u64 *__restrict__ out_sw,
-           CurPart cur, ModelP m) {
+           CurPart cur, ModelP m, u32 *counter) {
   extern __shared__ u64 sm[];
-  const SmemTab t = stage_tables(g, sm);
+  const SmemTab t = stage_tables<NARROW>(g, sm);
   const int L = t.L, N = (int)g.N;
   // a state that failed the device-side overflow check (set_state_device) scores nothing
   const bool overflow = (g.status[0] & 1ull) != 0;
-#if EVAL_SORT
-  for_each_sorted(recs, count, [&](const Rec &r, u64 i) {
-    score_one<ROLLOUT, P32, MODE, P>(t, L, N, overflow, r, i, out_t, out_sw, cur, m);
+  for_each_sorted_warp<EVAL_NT / 32>(recs, count, counter, [&](const Rec &r, u64 i) {
+    score_one<ROLLOUT, P32, MODE, NARROW, P>(t, L, N, overflow, r, i, out_t, out_sw, cur, m);
   });
-#else
-  const u64 stride = (u64)gridDim.x * blockDim.x;
-  for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < count; i += stride)
-    score_one<ROLLOUT, P32, MODE, P>(t, L, N, overflow, load_rec(recs + i), i, out_t, out_sw, cur, m);
-#endif
 }
 
-static int grid_for(u64 count, int sms, int per_sm) {
-  const u64 per = EVAL_SORT ? (u64)EV_CH : 256;  // records per block and step
-  const u64 need = (count + per - 1) / per;
-  const u64 cap = (u64)sms * (EVAL_SORT ? per_sm : 8);  // one wave of resident blocks
-  return (int)(need < cap ? (need ? need : 1) : cap);
-}
-
-template <bool ROLLOUT, bool P32, int MODE, typename Rec, typename P>
+template <bool ROLLOUT, bool P32, int MODE, typename Rec, typename P, bool NARROW = false>
 static void run_eval(int sms, size_t smem, cudaStream_t st, const DevTables &g, const void *recs, u64 count,
-                     u64 *out_t, u64 *out_sw, const CurPart &cur, const ModelP &m) {
-  const int per_sm = EVAL_BLOCKS(MODE, P);
-  k_eval<ROLLOUT, P32, MODE, Rec, P><<<grid_for(count, sms, per_sm), 256, smem, st>>>(g, (const Rec *)recs, count,
-                                                                                     out_t, out_sw, cur, m);
+                     u64 *out_t, u64 *out_sw, const CurPart &cur, const ModelP &m, u32 *counter) {
+  auto kern = k_eval<ROLLOUT, P32, MODE, Rec, P, NARROW>;
+  // one wave of resident blocks, fewer for a small batch. The dynamic shared memory (state tables)
+  // comes on top of the warps' static sort slices, so the opt-in limit is raised once per kernel;
+  // the occupancy is cached per dynamic size (a few sizes per process: one per (L, N)).
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncAttributes fa;
+    cudaFuncGetAttributes(&fa, kern);
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024 - (int)fa.sharedSizeBytes);
+    attr = true;
+  }
+  static size_t c_smem[8] = {0};
+  static int c_occ[8] = {0};
+  int occ = 0;
+  for (int i = 0; i < 8 && c_occ[i]; ++i)
+    if (c_smem[i] == smem) occ = c_occ[i];
+  if (!occ) {
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, EVAL_NT, smem) != cudaSuccess || occ < 1) occ = 1;
+    static int next = 0;
+    c_smem[next] = smem;
+    c_occ[next] = occ;
+    next = (next + 1) % 8;
+  }
+  constexpr u64 CH = (u64)WarpSort<EVAL_NT / 32, Rec>::CH * (EVAL_NT / 32);  // records per block and round
+  const u64 need = (count + CH - 1) / CH;
+  const u64 cap = (u64)sms * occ;
+  const unsigned grid = (unsigned)(need < cap ? (need ? need : 1) : cap);
+  cudaMemsetAsync(counter, 0, sizeof(u32), st);
+  kern<<<grid, EVAL_NT, smem, st>>>(g, (const Rec *)recs, count, out_t, out_sw, cur, m, counter);
 }
 
 template <bool ROLLOUT, typename Rec, typename P>
 static void dispatch_eval(int sms, size_t smem, cudaStream_t st, const DevTables &g, const void *recs, u64 count,
-                          u64 *out_t, u64 *out_sw, const CurPart &cur, const ModelP &m, int path32) {
+                          u64 *out_t, u64 *out_sw, const CurPart &cur, const ModelP &m, int path32, u32 *ctr) {
   switch (m.sched) {
-    case SCHED_2BW: run_eval<ROLLOUT, false, SCHED_2BW, Rec, P>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m); break;
-    case SCHED_GPIPE: run_eval<ROLLOUT, false, SCHED_GPIPE, Rec, P>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m); break;
-    case SCHED_DAPPLE: run_eval<ROLLOUT, false, SCHED_DAPPLE, Rec, P>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m); break;
-    default:
-      if (path32) run_eval<ROLLOUT, true, SCHED_PIPEDREAM, Rec, P>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m);
-      else run_eval<ROLLOUT, false, SCHED_PIPEDREAM, Rec, P>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m);
+    case SCHED_2BW: run_eval<ROLLOUT, false, SCHED_2BW, Rec, P>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m, ctr); break;
+    case SCHED_GPIPE: run_eval<ROLLOUT, false, SCHED_GPIPE, Rec, P>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m, ctr); break;
+    case SCHED_DAPPLE: run_eval<ROLLOUT, false, SCHED_DAPPLE, Rec, P>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m, ctr); break;
+    default:  // path32: bit 0 = 32-bit segment sums, bit 1 = narrow stage and shard arithmetic
+      switch (path32 & 3) {
+        case 3: run_eval<ROLLOUT, true, SCHED_PIPEDREAM, Rec, P, true>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m, ctr); break;
+        case 2: run_eval<ROLLOUT, false, SCHED_PIPEDREAM, Rec, P, true>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m, ctr); break;
+        case 1: run_eval<ROLLOUT, true, SCHED_PIPEDREAM, Rec, P>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m, ctr); break;
+        default: run_eval<ROLLOUT, false, SCHED_PIPEDREAM, Rec, P>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m, ctr);
+      }
   }
 }
 
@@ -116,7 +133,7 @@ static void dispatch_eval(int sms, size_t smem, cudaStream_t st, const DevTables
 // or nullptr. Its S and parts are decoded here.
 int launch_eval(const DevTables &g, const void *recs, u64 count, bool wide, u64 *out_t, u64 *out_sw,
                 const int *cur_S, const u64 *cur_cuts, const u64 *cur_masks, int path32, const ModelP &m, int sms,
-                cudaStream_t st) {
+                u32 *counter, cudaStream_t st) {
   if (count == 0) return 0;
   const size_t smem = (size_t)smem_words(g.L, g.N) * sizeof(u64);
   CurPart cur;
@@ -134,11 +151,11 @@ int launch_eval(const DevTables &g, const void *recs, u64 count, bool wide, u64 
     cur.valid = 1;
   }
   if (wide) {
-    if (out_sw) dispatch_eval<true, Rec32, P16>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m, path32);
-    else dispatch_eval<false, Rec32, P16>(sms, smem, st, g, recs, count, out_t, nullptr, cur, m, path32);
+    if (out_sw) dispatch_eval<true, Rec32, P16>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m, path32, counter);
+    else dispatch_eval<false, Rec32, P16>(sms, smem, st, g, recs, count, out_t, nullptr, cur, m, path32, counter);
   } else {
-    if (out_sw) dispatch_eval<true, Rec16, P8>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m, path32);
-    else dispatch_eval<false, Rec16, P8>(sms, smem, st, g, recs, count, out_t, nullptr, cur, m, path32);
+    if (out_sw) dispatch_eval<true, Rec16, P8>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m, path32, counter);
+    else dispatch_eval<false, Rec16, P8>(sms, smem, st, g, recs, count, out_t, nullptr, cur, m, path32, counter);
   }
   return 1;
 }

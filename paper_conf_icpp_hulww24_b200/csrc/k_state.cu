@@ -48,8 +48,10 @@ __global__ void k_build_state(DevTables g, const u64 *__restrict__ fp, const u64
       dst = g.PP;
     } else if (kind == 0) {
       dst = g.PF + w * Lp1;
+      dst32 = g.PF32 + w * Lp1;
     } else if (kind == 1) {
       dst = g.PB + w * Lp1;
+      dst32 = g.PB32 + w * Lp1;
     } else {
       dst = g.PC + w * Lp1;
       dst32 = g.PC32 + w * Lp1;
@@ -90,17 +92,27 @@ __global__ void k_build_state(DevTables g, const u64 *__restrict__ fp, const u64
     u64 mog = 0;
     for (int l = lane; l < L; l += 32) mog = umax(mog, umax(g.O[l], g.G[l]));
     const u64 maxOG = warp_max(mog);
-    // sum over layers of max over workers of (f + b), with overflow detection
+    // sum over layers of max over workers of (f + b), with overflow detection; the same for f and b
+    // alone (saturated at 2^32) for the narrow path
     bool ovf = false;
-    u64 part = 0;
+    u64 part = 0, pf = 0, pb = 0;
     for (int l = lane; l < L; l += 32) {
-      u64 m = 0;
+      u64 m = 0, mf = 0, mb = 0;
       for (int w = 0; w < N; ++w) {
         const u64 a = fp[w * L + l], b = bp[w * L + l];
         if (a >= (1ull << 59) || b >= (1ull << 59)) ovf = true;  // then the bound fails anyway
         m = umax(m, a + b);
+        mf = umax(mf, a);
+        mb = umax(mb, b);
       }
       part = (part >= (1ull << 59) || m >= (1ull << 60)) ? (1ull << 59) : part + m;  // saturate
+      pf = umin(pf + umin(mf, 1ull << 32), 1ull << 32);
+      pb = umin(pb + umin(mb, 1ull << 32), 1ull << 32);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      pf = umin(pf + __shfl_xor_sync(0xffffffffu, pf, o), 1ull << 32);
+      pb = umin(pb + __shfl_xor_sync(0xffffffffu, pb, o), 1ull << 32);
     }
     u64 sumMax = part;  // every lane's part <= 2^59 + 2^60, so the 32-lane sum cannot wrap
 #pragma unroll
@@ -124,7 +136,9 @@ __global__ void k_build_state(DevTables g, const u64 *__restrict__ fp, const u64
       }
       if (bound >= (1ull << 59)) ovf = true;
       const u64 path32 = (!ovf && bound32 < 0xFFFFFFF0ull) ? 2ull : 0ull;
-      g.status[0] = (ovf ? 1ull : 0ull) | path32;
+      const u64 lim = (1ull << 31) - 16;
+      const u64 narrow = (!ovf && pf <= lim && pb <= lim && maxOG < (1ull << 31) && maxTau < (1ull << 32)) ? 4ull : 0ull;
+      g.status[0] = (ovf ? 1ull : 0ull) | path32 | narrow;
       g.status[1] = bound;
     }
     return;

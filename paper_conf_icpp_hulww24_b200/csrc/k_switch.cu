@@ -52,7 +52,7 @@ __device__ __forceinline__ u64 startup_completion(const SmemTab &t, int S, u64 c
     if (s != 0xFF) {
       const int a = (s == 0) ? 0 : byte_at(cuts, s - 1) + 1;
       const int e = (s == S - 1) ? t.L - 1 : byte_at(cuts, s);
-      const Div8 dv((u32)__popc((u32)byte_at(masks, s)));
+      const Div8 dv((u32)__popc((u32)byte_at(masks, s)), t.dv);
       Fd[w] = dv.ceil(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a]);
       Bd[w] = dv.ceil(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a]);
     }
@@ -68,8 +68,8 @@ __device__ __forceinline__ u64 startup_completion(const SmemTab &t, int S, u64 c
     if (s < S - 1) {
       const int e = byte_at(cuts, s);
       const u32 ms = (u32)byte_at(masks, s), mn = (u32)byte_at(masks, s + 1);
-      nf = boundary_pairs(t.O[e], ms, mn, t.tau, dF, nf);
-      nb = boundary_pairs(t.G[e + 1], mn, ms, t.tau, dB, nb);
+      nf = boundary_pairs(t.O[e], ms, mn, t.tau, t.dv, dF, nf);
+      nb = boundary_pairs(t.G[e + 1], mn, ms, t.tau, t.dv, dB, nb);
     }
   }
   offF[MAXS - 1] = nf;

@@ -24,13 +24,14 @@ constexpr int MAXPAIRS = 2 * MAXN;  // sum over boundaries of (r_s + r_{s+1} - 1
 
 // Durations of every transfer of one boundary, in merge order (see boundary_max in eval.cuh).
 template <int MAXD = 8>
-__device__ __forceinline__ int boundary_pairs(u64 A, u32 send, u32 recv, const u64 *tau, u64 *d, int n) {
+__device__ __forceinline__ int boundary_pairs(u64 A, u32 send, u32 recv, const u64 *tau, const DivEnt *dvt, u64 *d,
+                                              int n) {
   const u32 rs = __popc(send), rr = __popc(recv);
   if (rs == 1 && rr == 1) {
     d[n] = xfer(A, tau[(__ffs(send) - 1) * TAUW + __ffs(recv) - 1]);
     return n + 1;
   }
-  const DivR<MAXD> ds(rs), dr(rr);
+  const DivR<MAXD> ds(rs, dvt), dr(rr, dvt);
   const u64 qs = ds.div(A), qr = dr.div(A);
   const u32 rems = (u32)(A - qs * rs), remr = (u32)(A - qr * rr);
   u32 i = 0, j = 0;
@@ -85,7 +86,7 @@ __device__ __forceinline__ u64 flush_makespan(const SmemTab &t, int S, const P &
     if (s != 0xFF) {
       const int a = (s == 0) ? 0 : p.cut(s - 1) + 1;
       const int e = (s == S - 1) ? t.L - 1 : p.cut(s);
-      const DivR<MN> dv((u32)__popc(p.mask(s)));
+      const DivR<MN> dv((u32)__popc(p.mask(s)), t.dv);
       Fd[w] = dv.ceil(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a]);
       Bd[w] = dv.ceil(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a]);
       if (SCHED == SCHED_GPIPE && m.recompute) Bd[w] += Fd[w];  // the backward op re-runs the forward
@@ -101,8 +102,8 @@ __device__ __forceinline__ u64 flush_makespan(const SmemTab &t, int S, const P &
     if (s < S - 1) {
       const int e = p.cut(s);
       const u32 ms = p.mask(s), mn = p.mask(s + 1);
-      nf = boundary_pairs<MN>(t.O[e], ms, mn, t.tau, dF, nf);
-      nb = boundary_pairs<MN>(t.G[e + 1], mn, ms, t.tau, dB, nb);
+      nf = boundary_pairs<MN>(t.O[e], ms, mn, t.tau, t.dv, dF, nf);
+      nb = boundary_pairs<MN>(t.G[e + 1], mn, ms, t.tau, t.dv, dB, nb);
     }
   }
   offF[MS - 1] = nf;
@@ -180,7 +181,7 @@ __device__ __forceinline__ u64 flush_makespan(const SmemTab &t, int S, const P &
       if (__popc(mask) >= 2) {
         const int a = (s == 0) ? 0 : p.cut(s - 1) + 1;
         const int e = (s == S - 1) ? t.L - 1 : p.cut(s);
-        x += sync_time<MN>((int)m.sync, t.PP[e + 1] - t.PP[a], mask, t.tau);
+        x += sync_time<MN>((int)m.sync, t.PP[e + 1] - t.PP[a], mask, t.tau, t.dv);
       }
       T = umax(T, x);
     }

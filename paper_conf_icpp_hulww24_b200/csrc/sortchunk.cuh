@@ -1,19 +1,20 @@
-// sortchunk.cuh — shape-ordered traversal of a batch of partition records (k_eval, k_switch).
+// sortchunk.cuh — shape-ordered traversal of a batch of partition records (k_eval).
 //
 // Random rollout records mix S = 1..8 and replica counts; scored in input order, a warp runs the
-// union of its lanes' stage, replica and boundary loops (ncu: ~9 of 32 lanes active). A block here
-// takes chunks of EV_CH consecutive records (coalesced 128-bit loads), counts them into shape buckets
-// in shared memory, and hands them to the scoring function in bucket order, so a warp scores records
-// of one shape. Every record is still scored exactly once, and its outputs go to its own position
-// (8-byte stores scattered within the chunk).
+// union of its lanes' stage, replica and boundary loops (ncu: ~9 of 32 lanes active). A warp here
+// takes chunks of consecutive records (coalesced 128-bit loads), counts them into shape buckets in
+// its slice of shared memory, and hands them to the scoring function in bucket order, so the lanes
+// of a step score records of (nearly) one shape. Every record is still scored exactly once, and its
+// outputs go to its own position (8-byte stores scattered within the chunk).
 #pragma once
 #include "common.cuh"
 
 namespace ap {
 
-constexpr int EV_PER = 4;              // records per thread and chunk
-constexpr int EV_CH = 256 * EV_PER;    // records per chunk
 constexpr int EV_NB = 64;              // shape buckets
+#ifndef EVAL_PER16
+#define EVAL_PER16 8                   // 16-byte records per lane and warp chunk (B200 C5: 8 beat 4 by 5 %)
+#endif
 
 struct Rec16 {  // a 16-byte partition record
   uint4 a;
@@ -41,63 +42,84 @@ __device__ __forceinline__ u32 shape_key(const Rec32 &r) {
   return (((S - 1u) & 15u) << 2) | (extra < 3u ? extra : 3u);
 }
 
-// f(record, global index) for every record of recs[0, count), block-strided over chunks; every thread
-// of the block must call it (it synchronises the block).
-template <typename Rec, typename F>
-__device__ __forceinline__ void for_each_sorted(const Rec *__restrict__ recs, u64 count, F &&f) {
-  __shared__ Rec srec[EV_CH];
-  __shared__ u32 sidx[EV_CH];
-  __shared__ u32 hist[EV_NB];
-  const int tid = threadIdx.x;
-  const u64 nch = (count + EV_CH - 1) / EV_CH;
-  for (u64 ch = blockIdx.x; ch < nch; ch += gridDim.x) {
-    const u64 base = ch * EV_CH;
-    if (tid < EV_NB) hist[tid] = 0;
-    __syncthreads();
-    Rec rr[EV_PER];
-    u32 key[EV_PER], rank[EV_PER];
+// f(record, global index) for every record of recs[0, count). Each warp works on its own: it takes
+// a chunk of 32 * PER consecutive records from a global counter (dynamic schedule: no tail of idle
+// warps whatever the batch size), loads it with coalesced 128-bit loads, counting-sorts it by shape
+// in its own slice of shared memory (no block barrier: a warp that drew cheap records moves on to the
+// next chunk at once) and scores it in shape order, 32 records per step. *counter must be 0 at
+// launch; NW = warps per block.
+template <int NW, typename Rec>
+struct WarpSort {
+  static constexpr int PER = sizeof(Rec) == 16 ? EVAL_PER16 : 4;  // records per lane and chunk
+  static constexpr int CH = 32 * PER;
+};
+
+template <int NW, typename Rec, typename F>
+__device__ __forceinline__ void for_each_sorted_warp(const Rec *__restrict__ recs, u64 count, u32 *counter, F &&f) {
+  constexpr int PER = WarpSort<NW, Rec>::PER, CH = WarpSort<NW, Rec>::CH;
+  __shared__ Rec srec[NW][CH];
+  __shared__ unsigned short sidx[NW][CH];
+  __shared__ u32 hist[NW][EV_NB];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const u64 nch = (count + CH - 1) / CH;
+  Rec *sr = srec[w];
+  unsigned short *si = sidx[w];
+  u32 *h = hist[w];
+  for (;;) {
+    u32 c = 0;
+    if (lane == 0) c = atomicAdd(counter, 1u);
+    c = __shfl_sync(0xffffffffu, c, 0);
+    if ((u64)c >= nch) break;
+    const u64 base = (u64)c * CH;
+    h[lane] = 0;
+    h[lane + 32] = 0;
+    __syncwarp();
+    // records go to shared memory in input order right away (no register copy); a lane keeps only
+    // key | rank << 8 per record, and the sort writes the permutation sorted slot -> input slot
+    u32 kr[PER];
 #pragma unroll
-    for (int j = 0; j < EV_PER; ++j) {
-      const u64 i = base + (u64)(j * 256 + tid);
-      key[j] = EV_NB;
-      rank[j] = 0;
+    for (int j = 0; j < PER; ++j) {
+      const u64 i = base + (u64)(j * 32 + lane);
+      kr[j] = EV_NB;
       if (i < count) {
-        rr[j] = load_rec(recs + i);
-        key[j] = shape_key(rr[j]);
-        rank[j] = atomicAdd(&hist[key[j]], 1u);
+        const Rec r = load_rec(recs + i);
+        sr[j * 32 + lane] = r;
+        const u32 key = shape_key(r);
+        kr[j] = key | (atomicAdd(&h[key], 1u) << 8);
       }
     }
-    __syncthreads();
-    if (tid < 32) {  // exclusive scan of the 64 bucket counts, two per lane
-      const u32 a = hist[2 * tid], b = hist[2 * tid + 1];
-      u32 v = a + b;
+    __syncwarp();
+    {  // exclusive scan of the 64 bucket counts, two per lane
+      const u32 a = h[2 * lane], b2 = h[2 * lane + 1];
+      u32 v = a + b2;
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
         const u32 y = __shfl_up_sync(0xffffffffu, v, o);
-        if (tid >= o) v += y;
+        if (lane >= o) v += y;
       }
-      const u32 ex = v - (a + b);
-      hist[2 * tid] = ex;
-      hist[2 * tid + 1] = ex + a;
+      const u32 ex = v - (a + b2);
+      __syncwarp();
+      h[2 * lane] = ex;
+      h[2 * lane + 1] = ex + a;
     }
-    __syncthreads();
+    __syncwarp();
 #pragma unroll
-    for (int j = 0; j < EV_PER; ++j) {
-      if (key[j] < EV_NB) {
-        const u32 slot = hist[key[j]] + rank[j];
-        srec[slot] = rr[j];
-        sidx[slot] = (u32)(j * 256 + tid);
+    for (int j = 0; j < PER; ++j) {
+      const u32 key = kr[j] & 0xFFu;
+      if (key < EV_NB) si[h[key] + (kr[j] >> 8)] = (unsigned short)(j * 32 + lane);
+    }
+    __syncwarp();
+    const u64 left = count - base;
+    const u32 nvalid = left < (u64)CH ? (u32)left : (u32)CH;
+#pragma unroll 1
+    for (int j = 0; j < PER; ++j) {
+      const u32 slot = (u32)(j * 32 + lane);
+      if (slot < nvalid) {
+        const u32 src = si[slot];
+        f(sr[src], base + src);
       }
     }
-    __syncthreads();
-    const u64 left = count - base;
-    const u32 nvalid = left < (u64)EV_CH ? (u32)left : (u32)EV_CH;
-#pragma unroll 1
-    for (int j = 0; j < EV_PER; ++j) {
-      const u32 slot = (u32)(j * 256 + tid);
-      if (slot < nvalid) f(srec[slot], base + sidx[slot]);
-    }
-    __syncthreads();  // the next chunk reuses srec / sidx / hist
+    __syncwarp();  // the next chunk reuses this warp's slice
   }
 }
 

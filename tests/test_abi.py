@@ -67,3 +67,10 @@ def test_product_path_does_not_import_oracle():
             if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
                 src = open(os.path.join(dirpath, f)).read()
                 assert "oracle" not in re.sub(r"#.*|//.*", "", src), f
+
+
+def test_div32_multipliers_exact():
+    """The narrow eval path's 32-bit division (common.cuh Div32): floor(x / d) = mulhi32(x, m) >> k
+    for every replica count d in [2, 16] on the top of its range x < 2^31 (tools/check_div32.py)."""
+    from tools.check_div32 import main
+    main()

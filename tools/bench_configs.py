@@ -19,19 +19,20 @@ if ROOT not in sys.path:
 
 
 def _timed(fn, reps=5, warm=2):
+    """Device time per call: `reps` calls enqueued back to back between one pair of CUDA events
+    (asynchronous calls keep the GPU busy, so the host's enqueue cost is hidden as it is in a
+    pipeline; calls that synchronise internally are timed with their host round trip)."""
     import torch
     for _ in range(warm):
         fn()
     torch.cuda.synchronize()
-    out = []
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record()
     for _ in range(reps):
-        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        a.record()
         r = fn()
-        b.record()
-        torch.cuda.synchronize()
-        out.append(a.elapsed_time(b))
-    return sum(out) / len(out), r
+    b.record()
+    torch.cuda.synchronize()
+    return a.elapsed_time(b) / reps, r
 
 
 def measure(device: int = 0, rollout_records: int = 1 << 20):

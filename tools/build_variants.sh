@@ -1,10 +1,20 @@
-# Build in-tree variants of libautopipe.so with different compile-time options of the hot kernel
-# (for tools/variant_times.sh): each argument is NAME=FLAGS, e.g. "v4nx2=-DR1_V4=1 -DR1_NX=2".
+# Build in-tree variants of libautopipe.so with different compile-time options (for timing
+# experiments; select one with AUTOPIPE_LIB=<path>): each argument is NAME=FLAGS, e.g.
+# "per8=-DEVAL_PER16=8". Every translation unit is compiled with the flags, in parallel.
 set -e
 cd "$(dirname "$0")/../paper_conf_icpp_hulww24_b200/csrc"
+mkdir -p ../build/variants
 for spec in "$@"; do
   name="${spec%%=*}"; flags="${spec#*=}"
-  nvcc -gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -shared $flags \
-    -o ../libautopipe_${name}.so autopipe.cu kernels.cu &
+  (
+    objs=""
+    for f in autopipe k_state k_eval k_search k_search_r1 k_neigh k_switch; do
+      nvcc -gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -std=c++17 -Xcompiler -fPIC $flags \
+        -c -o ../build/variants/${name}_$f.o $f.cu &
+      objs="$objs ../build/variants/${name}_$f.o"
+    done
+    wait
+    nvcc -gencode arch=compute_100a,code=sm_100a -shared -o ../libautopipe_${name}.so $objs
+  ) &
 done
 wait
