@@ -326,6 +326,13 @@ uint64_t autopipe_kernel_launches(const autopipe_ctx *ctx);
  * reduction and the result copy). */
 int autopipe_set_timing(autopipe_ctx *ctx, int enable);
 
+/* Kernel selection of later searches (the result never depends on it; tests use it to exercise each
+ * kernel on small spaces). options: 0 = default (a range of at most 2^21 candidates is searched by
+ * one dense launch, every candidate's exact T; larger ranges are split per S into the r = 1 sweep
+ * and the threshold walk), AUTOPIPE_SEARCH_SPLIT = always the per-S split. E_INVAL on unknown bits. */
+#define AUTOPIPE_SEARCH_SPLIT 1u
+int autopipe_set_search_options(autopipe_ctx *ctx, uint32_t options);
+
 /* Device milliseconds of the enumeration kernels of the last timed search (-1 if none); waits for
  * that search's kernels to finish (an asynchronous search returns before they run). */
 double autopipe_last_search_ms(const autopipe_ctx *ctx);

@@ -33,7 +33,7 @@ ERROR_NAMES = {AUTOPIPE_E_INVAL: "AUTOPIPE_E_INVAL", AUTOPIPE_E_STATE: "AUTOPIPE
 SYMBOLS = ["autopipe_create", "autopipe_destroy", "autopipe_last_error", "autopipe_load_profile",
            "autopipe_set_state", "autopipe_set_state_device", "autopipe_eval_partitions", "autopipe_search_optimum",
            "autopipe_rollout_rewards", "autopipe_count_candidates", "autopipe_decode_index",
-           "autopipe_int_path", "autopipe_kernel_launches", "autopipe_set_timing",
+           "autopipe_int_path", "autopipe_kernel_launches", "autopipe_set_timing", "autopipe_set_search_options",
            "autopipe_last_search_ms", "autopipe_neighbourhood", "autopipe_neighbourhood_best",
            "autopipe_switch_rewards", "autopipe_balanced_shards", "autopipe_set_schedule",
            "autopipe_get_schedule", "autopipe_eval_partitions_w", "autopipe_rollout_rewards_w",
@@ -95,6 +95,7 @@ def _load():
         "autopipe_int_path": (i32, [P]),
         "autopipe_kernel_launches": (u64, [P]),
         "autopipe_set_timing": (i32, [P, i32]),
+        "autopipe_set_search_options": (i32, [P, u32]),
         "autopipe_last_search_ms": (ctypes.c_double, [P]),
         "autopipe_neighbourhood": (i32, [P, ctypes.POINTER(Partition), P, u64, pu64, P]),
         "autopipe_neighbourhood_best": (i32, [P, ctypes.POINTER(Partition), ctypes.POINTER(Result), P]),

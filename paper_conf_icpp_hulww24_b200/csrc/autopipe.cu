@@ -48,6 +48,9 @@ struct autopipe_ctx {
   static const int NCTR = 256;
   u32 *d_ctr = nullptr;
   u32 ctr_next = 0;
+  // the same for the search kernels' schedules (SEARCH_SCHED_BYTES per launch)
+  unsigned char *d_sched = nullptr;
+  u32 sched_next = 0;
   void *h_work = nullptr;  // pinned mirror of d_work (r = 1 schedules)
   size_t work_bytes = 0;
   // pinned host staging
@@ -62,6 +65,7 @@ struct autopipe_ctx {
   cudaEvent_t ev_fork = nullptr, ev_join[NAUX] = {nullptr, nullptr, nullptr, nullptr};
   // optional device timing of the search kernels (autopipe_set_timing)
   bool timing = false;
+  u32 search_options = 0;  // autopipe_set_search_options
   // a ring of event pairs: search k (counted while timing is on) records pair k % TRING, so the
   // times of asynchronous searches can be read after the fact (autopipe_search_times)
   static const int TRING = 64;
@@ -87,6 +91,9 @@ struct autopipe_ctx {
 static char g_create_err[256] = "";
 
 static u32 *next_counter(autopipe_ctx *c) { return c->d_ctr + (c->ctr_next++ % autopipe_ctx::NCTR); }
+static void *next_sched(autopipe_ctx *c) {
+  return c->d_sched + (size_t)SEARCH_SCHED_BYTES * (c->sched_next++ % autopipe_ctx::NCTR);
+}
 
 const char *ap::experiment_knob(const char *name) {
   static const bool on = [] {
@@ -159,7 +166,7 @@ extern "C" int autopipe_create(int cuda_device, autopipe_ctx **out) {
   upload_binomials(c->binom);
   // device tables, sized for the limits (L = 255, N = 8): a few hundred KB
   const size_t Lp1 = MAXL + 1, NL = (size_t)MAXNW * Lp1, TT = (size_t)TAUW * TAUW;
-  const size_t words = 3 * NL + Lp1 + 2 * MAXL + TT + 2 * 7 * MAXL + 2;
+  const size_t words = 3 * NL + Lp1 + 2 * MAXL + TT + 2 * 7 * MAXL + 2 + 256;
   const size_t words32 = 3 * NL + 2 * 7 * MAXL;
   e = cudaMalloc(&c->d_tables, words * 8 + words32 * 4 + 64);
   if (e == cudaSuccess) e = cudaMalloc(&c->d_raw, (2 * MAXNW * MAXL + MAXL + TT) * 8);
@@ -172,6 +179,7 @@ extern "C" int autopipe_create(int cuda_device, autopipe_ctx **out) {
   if (e == cudaSuccess) e = cudaMalloc(&c->d_ntimes, (size_t)NEIGH_ITEMS * NEIGH_MAXOPT * 8);
   if (e == cudaSuccess) e = cudaMalloc(&c->d_ncount, 8);
   if (e == cudaSuccess) e = cudaMalloc(&c->d_ctr, sizeof(u32) * autopipe_ctx::NCTR);
+  if (e == cudaSuccess) e = cudaMalloc(&c->d_sched, (size_t)SEARCH_SCHED_BYTES * autopipe_ctx::NCTR);
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_ncount, 8);
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_stage, (2 * MAXNW * MAXL + TT) * 8);
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_result, sizeof(ResultDev));
@@ -192,6 +200,7 @@ extern "C" int autopipe_create(int cuda_device, autopipe_ctx **out) {
   c->tab.Z = p; p += 7 * MAXL;
   c->tab.LM = p; p += 7 * MAXL;
   c->tab.status = p; p += 2;
+  c->tab.ring = p; p += 256;
   u32 *q = (u32 *)p;
   c->tab.PC32 = q; q += NL;
   c->tab.PF32 = q; q += NL;
@@ -223,6 +232,7 @@ extern "C" void autopipe_destroy(autopipe_ctx *c) {
     if (c->d_ntimes) cudaFree(c->d_ntimes);
     if (c->d_ncount) cudaFree(c->d_ncount);
     if (c->d_ctr) cudaFree(c->d_ctr);
+    if (c->d_sched) cudaFree(c->d_sched);
     if (c->h_ncount) cudaFreeHost(c->h_ncount);
     if (c->h_stage) cudaFreeHost(c->h_stage);
     if (c->h_result) cudaFreeHost(c->h_result);
@@ -648,9 +658,17 @@ static int search_impl(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, u64 beg
     }
     forked = false;
   };
-  // Split [begin, end) into the r = 1 block of each S (rho = 0: fast kernel) and the rest (generic);
-  // the pieces write disjoint block-result ranges and run concurrently.
+  // A small range: one dense launch on the caller's stream. Otherwise split [begin, end) into the
+  // r = 1 block of each S (rho = 0: fast kernel) and the rest (generic); the pieces write disjoint
+  // block-result ranges and run concurrently.
   u64 cur = begin;
+  if (end - begin <= DENSE_SPAN && !(c->search_options & AUTOPIPE_SEARCH_SPLIT)) {
+    int nb = 0;
+    c->launches += launch_search_generic(c->tab, sp, begin, end, path, c->model, wide, c->sms, c->d_blocks,
+                                         MAX_BLOCKS, &nb, next_sched(c), st, true);
+    used = nb;
+    cur = end;
+  }
   for (int S = (int)s_min; S <= (int)s_max && cur < end; ++S) {
     const u64 blo = sp.off[S], bhi = sp.off[S + 1];
     if (bhi <= cur) continue;
@@ -674,13 +692,13 @@ static int search_impl(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, u64 beg
       used += nb;
       if (b < hi) {
         c->launches += launch_search_generic(c->tab, sp, b, hi, path, c->model, wide, c->sms, c->d_blocks + used,
-                                             MAX_BLOCKS - used, &nb, next_stream());
+                                             MAX_BLOCKS - used, &nb, next_sched(c), next_stream());
         used += nb;
       }
     } else {
       int nb = 0;
       c->launches += launch_search_generic(c->tab, sp, lo, hi, path, c->model, wide, c->sms, c->d_blocks + used,
-                                           MAX_BLOCKS - used, &nb, next_stream());
+                                           MAX_BLOCKS - used, &nb, next_sched(c), next_stream());
       used += nb;
     }
     cur = hi;
@@ -930,6 +948,14 @@ extern "C" int autopipe_int_path(const autopipe_ctx *cc) {
 }
 
 extern "C" uint64_t autopipe_kernel_launches(const autopipe_ctx *c) { return c ? c->launches : 0; }
+
+extern "C" int autopipe_set_search_options(autopipe_ctx *c, uint32_t options) {
+  if (!c) return AUTOPIPE_E_INVAL;
+  c->err[0] = 0;
+  if (options & ~AUTOPIPE_SEARCH_SPLIT) return fail(c, AUTOPIPE_E_INVAL, "unknown search options 0x%x", options);
+  c->search_options = options;
+  return AUTOPIPE_OK;
+}
 
 extern "C" int autopipe_set_timing(autopipe_ctx *c, int enable) {
   if (!c) return AUTOPIPE_E_INVAL;

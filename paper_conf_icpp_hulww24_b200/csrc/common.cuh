@@ -37,6 +37,7 @@ struct DevTables {
   u64 *Z;     // [7][L]    r = 1 boundary s (worker s -> s+1) cut after layer l: cf + cb   (row a2)
   u64 *LM;    // [7][L]    ... max(cf, cb)                                                (row a2)
   u32 *PC32;  // [N][L+1]  32-bit copies for the 32-bit search path (valid iff path32)
+  u64 *ring;  // [256]     slowest link of the ring over each worker set (N <= 8; ascending ring order)
   u32 *PF32;  // [N][L+1]  32-bit copies of PF, PB for the narrow eval path (valid iff status bit 2)
   u32 *PB32;
   u32 *Z32;   // [7][L]

@@ -100,23 +100,7 @@ __device__ __forceinline__ SmemTab stage_tables(const DevTables &g, u64 *sm) {
     tau32[i] = (u32)v;  // meaningful on the narrow path only (tau < 2^32 there)
   }
   u64 *ring = (u64 *)(tau32 + TAUW * TAUW);
-  // ring[mask]: max over the ring W[0] -> W[1] -> ... -> W[0] (ascending) of tau, read from global
-  for (u32 msk = threadIdx.x; msk < 256u; msk += blockDim.x) {
-    u64 tr = 0;
-    if (__popc(msk) >= 2 && msk < (1u << (N < 8 ? N : 8))) {
-      const int first = __ffs(msk) - 1;
-      int prev = first;
-      u32 m = msk & (msk - 1);
-      while (m) {
-        const int w = __ffs(m) - 1;
-        m &= m - 1;
-        tr = umax(tr, g.tau[prev * TAUW + w]);
-        prev = w;
-      }
-      tr = umax(tr, g.tau[prev * TAUW + first]);
-    }
-    ring[msk] = tr;
-  }
+  for (u32 i = threadIdx.x; i < 256u; i += blockDim.x) ring[i] = g.ring[i];
   __syncthreads();
   t.PP = PP; t.O = O; t.G = G; t.tau = tau; t.tau32 = tau32; t.ring = ring;
   t.dv = dt;

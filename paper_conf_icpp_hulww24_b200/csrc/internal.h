@@ -32,8 +32,15 @@ int launch_eval(const DevTables &g, const void *recs, u64 count, bool wide, u64 
                 u32 *counter, cudaStream_t st);
 // Generic exhaustive search over [begin, end) (any S, any composition); writes one BlockOut per block
 // into out[out_offset ...] and returns the number of blocks used via *nblocks.
+// sched: 32 bytes of device memory the PipeDream launch resets and schedules its chunks through (two
+// 16-byte slots: one per gated launch); each concurrent launch needs its own
+constexpr int SEARCH_SCHED_BYTES = 32;
 int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, u64 end, int path32, const ModelP &m,
-                          bool wide, int sms, BlockOut *out, int max_blocks, int *nblocks, cudaStream_t st);
+                          bool wide, int sms, BlockOut *out, int max_blocks, int *nblocks, void *sched,
+                          cudaStream_t st, bool dense = false);
+// spaces (or shards) up to this many candidates are searched by one dense launch (one candidate per
+// thread, exact T): latency-bound, they finish before a threshold walk would pay off
+constexpr unsigned long long DENSE_SPAN = 1ull << 21;
 // Cross-shard bound of the r = 1 sweep (row e). bound: device word the sweep's shared theta starts at
 // (replaces the shard's own seed); theta_out: seed only, no sweep — the shard's seed T is atomicMin'ed
 // into this device word.

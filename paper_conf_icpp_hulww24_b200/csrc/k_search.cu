@@ -132,27 +132,341 @@ __global__ void __launch_bounds__(NT) k_search_generic(DevTables g, SearchSpace 
   block_minloc_store<NT>(bestT, bestI, cnt, out + blockIdx.x);
 }
 
+// ---------------------------------------------------------------------------------------------
+// PipeDream search by prefix thresholds (rows a3-a8 for every composition; SPEC.md §4-§5).
+//
+// A thread walks its contiguous index range in lexicographic order, which is a depth-first walk over
+// the cuts (the last cut moves fastest). It decides, per candidate, whether T <= theta, theta = its
+// best T so far minus 1 (strict: its indices increase) or the block's best T (non-strict: ties keep
+// the lower index), whichever is lower; only a candidate that passes gets its exact T (the full
+// closed form), so every candidate is decided exactly and the thread's result is its lexicographic
+// (T, index) minimum.
+// The decision needs no division by segment lengths: T <= theta iff every single term is <= theta
+// and every segment W(s,t) <= theta (t - s + 1). Scanning stages left to right, the segments still
+// open after stage t are summarised by one number (the parametric DP of SPEC.md §A.6):
+//   O_t = max over s <= t of (X_s + sum_{s<v<=t} Y_v + sum_{s<=v<t} Z_v - theta (t - s + 1))
+//       = max(X_t - theta, O_{t-1} + Z_{t-1} + Y_t - theta),
+// and the segments closing at t fit iff O_{t-1} + Z_{t-1} + X_t - theta <= 0. O_t of the prefix
+// stages 0..S-3 is kept per level, so a lexicographic step recomputes only the levels whose cut
+// moved; along a row (the last cut e) only stage S-2 = [a, e], boundary S-2 and stage S-1 change.
+// A prefix that fails decides every candidate below it at once (they all contain the failing
+// term): the walk jumps over that subtree, whose size is 1 + sum_{j > t} C(L - 2 - e_j, S - 1 - j)
+// from the current position. Along a row, stage S-2 only grows with e (its X, Y, sync terms are
+// non-decreasing), so a failure there decides the rest of the row.
+// ---------------------------------------------------------------------------------------------
+__device__ __forceinline__ void pk_set(u64 &v, int i, int x) {
+  v = (v & ~(0xFFull << (8 * i))) | ((u64)x << (8 * i));
+}
+__device__ __forceinline__ void pk_set(Pk2 &v, int i, int x) {
+  if (i < 8) pk_set(v.lo, i, x);
+  else pk_set(v.hi, i - 8, x);
+}
+
+// lexicographic successor of the k-subset `c` of {0..n-1} moving only positions <= lv; false if none
+template <typename PK>
+__device__ __forceinline__ bool cut_next_from(PK &c, int lv, int k, int n, int &changed) {
+  for (int i = lv; i >= 0; --i) {
+    const int x = pk_get(c, i);
+    if (x < n - k + i) {
+      for (int j = i; j < k; ++j) pk_set(c, j, x + 1 + (j - i));
+      changed = i;
+      return true;
+    }
+  }
+  return false;
+}
+
+__device__ __forceinline__ u32 range_mask(int lo, int hi) {  // workers [lo, hi)
+  return ((hi >= 32 ? 0xFFFFFFFFu : ((1u << hi) - 1u))) & ~((1u << lo) - 1u);
+}
+
+template <typename PK>
+__device__ __forceinline__ u32 stage_mask(const SearchSpace &sp, int S, const PK &Rp, int s) {
+  const bool all = sp.flags & 1;
+  const int R = (all && s == S - 1) ? sp.N : pk_get(Rp, s) + 1;
+  const int R0 = (s == 0) ? 0 : pk_get(Rp, s - 1) + 1;
+  return range_mask(R0, R);
+}
+
+// stage [a, e] on the replicas `mask`: X = max(F' + B'), Y = max F' + max B', AR = its sync term
+template <int MN>
+__device__ __forceinline__ void stage_cost(const SmemTab &t, int a, int e, u32 mask, int sync, u64 &X, u64 &Y,
+                                           u64 &AR) {
+  const u32 r = __popc(mask);
+  const DivR<MN> dv(r, t.dv);
+  u32 m = mask;
+  u64 fm = 0, bm = 0, xm = 0;
+  while (m) {
+    const int w = __ffs(m) - 1;
+    m &= m - 1;
+    const u64 F = dv.ceil(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a]);
+    const u64 B = dv.ceil(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a]);
+    fm = umax(fm, F);
+    bm = umax(bm, B);
+    xm = umax(xm, F + B);
+  }
+  X = xm;
+  Y = fm + bm;
+  AR = (r >= 2) ? sync_time<MN>(sync, t.PP[e + 1] - t.PP[a], mask, t.tau, t.dv) : 0ull;
+}
+
+#ifndef DFS_MINB
+#define DFS_MINB 2  // resident blocks per SM of the threshold walk
+#endif
+#ifndef DFS_MINCH
+#define DFS_MINCH 16  // candidates per chunk at least
+#endif
+
+// Dynamic schedule of the walk: chunks of the shard drawn from a global counter (so a thread whose
+// chunk collapses into a few subtree jumps takes the next one), and the grid's best exact T so far
+// (a bound every thread decides against, non-strictly). Reset by the launcher before each launch.
+struct DfsSched {
+  unsigned int next, pad;
+  unsigned long long best;
+};
+
+template <int NT, typename P>
+__global__ void __launch_bounds__(NT, DFS_MINB) k_search_dfs(DevTables g, SearchSpace sp, u64 begin, u64 end,
+                                                             u64 chunk, BlockOut *out, ModelP m, DfsSched *ds,
+                                                             int gate) {
+  if (gate >= 0 && state_gated_out(g, gate, out)) return;  // see state_gated_out
+  typedef SpaceT<P> SP;
+  typedef typename SP::PK PK;
+  constexpr int BK = SP::BK, MN = P::MN, MS = P::MS;
+  extern __shared__ u64 sm[];
+  __shared__ unsigned long long s_best;  // the block's best exact T so far
+  u64 *Bn = sm + smem_words(g.L, g.N);
+  const int nb = ((int)g.L + 1 > MAXNW + 1 ? (int)g.L + 1 : MAXNW + 1) * BK;
+  for (int i = threadIdx.x; i < nb; i += NT) Bn[i] = g_binom[i / BK][i % BK];
+  if (threadIdx.x == 0) s_best = U64MAX;
+  const SmemTab t = stage_tables(g, sm);  // ends with __syncthreads()
+  const int L = t.L, n = L - 1, sync = (int)m.sync;
+  const u64 nchunks = (end - begin + chunk - 1) / chunk;
+  u64 bestT = U64MAX, bestI = U64MAX, cnt = 0;
+  long long O[MS];
+  for (;;) {
+    const u64 c = atomicAdd(&ds->next, 1u);
+    if (c >= nchunks) break;
+    const u64 i0 = begin + c * chunk;
+    const u64 i1 = (end - i0 < chunk) ? end : i0 + chunk;
+    cnt += i1 - i0;
+    u64 gbest = *(volatile unsigned long long *)&ds->best;  // refreshed per chunk
+    int S;
+    PK Rp, cuts;
+    unrank_global_smem<BK>(sp, i0, S, Rp, cuts, Bn);
+    long long th = 0;
+    bool have_th = false;
+    int valid = 0;  // levels [0, valid) of O are computed for the current cuts and th
+    u64 idx = i0;
+    auto exact = [&]() -> u64 {
+      const P p = part_from<P>(sp, S, Rp, cuts);
+      return eval_closed_form<false, false, P>(t, S, p, sync);
+    };
+    auto next_comp = [&]() -> bool {  // the next composition (or S), first cut set
+      cuts = first_subset<PK>(S - 1);
+      valid = 0;
+      if (SP::next(Rp, comp_k(sp, S), comp_n(sp))) return true;
+      ++S;
+      if (S > sp.s_max) return false;
+      Rp = first_subset<PK>(comp_k(sp, S));
+      cuts = first_subset<PK>(S - 1);
+      return true;
+    };
+    auto after_level = [&](int lv) -> bool {  // past the subtree of level lv (-1: of the composition)
+      int ch = 0;
+      if (lv >= 0 && cut_next_from(cuts, lv, S - 1, n, ch)) {
+        if (ch < valid) valid = ch;
+        return true;
+      }
+      return next_comp();
+    };
+    auto improve = [&](u64 T) {
+      if (T < bestT) {
+        bestT = T;
+        bestI = idx;
+        atomicMin(&s_best, (unsigned long long)T);
+        if (T < gbest) {
+          atomicMin(&ds->best, (unsigned long long)T);
+          gbest = T;
+        }
+      }
+    };
+    bool more = true;
+    while (more) {
+      // threshold: own best - 1 (strict: own indices increase), or a shared best (non-strict: ties
+      // keep the lower index) when lower
+      {
+        const u64 sb = umin(*(volatile unsigned long long *)&s_best, gbest);
+        if (bestT == U64MAX && sb == U64MAX) {  // no bound yet: this candidate is scored exactly
+          improve(exact());
+          ++idx;
+          more = idx < i1 && after_level(S - 2);
+          continue;
+        }
+        long long nth = (bestT == U64MAX) ? (long long)(1ull << 62) : (long long)bestT - 1;
+        if (sb < (u64)nth) nth = (long long)sb;
+        if (!have_th || nth != th) {
+          th = nth;
+          have_th = true;
+          valid = 0;
+        }
+      }
+      // prefix levels valid .. S-3
+      int dead = -1;
+      for (int lv = valid; lv <= S - 3; ++lv) {
+        const int a = (lv == 0) ? 0 : pk_get(cuts, lv - 1) + 1;
+        const int e = pk_get(cuts, lv);
+        const u32 mk = stage_mask(sp, S, Rp, lv);
+        u64 X, Y, AR;
+        stage_cost<MN>(t, a, e, mk, sync, X, Y, AR);
+        bool ok = (long long)X <= th && (long long)AR <= th;
+        long long o = (long long)X - th;
+        if (lv > 0) {
+          const u32 mp = stage_mask(sp, S, Rp, lv - 1);
+          const u64 cf = boundary_max<MN>(t.O[a - 1], mp, mk, t.tau, t.dv);
+          const u64 cb = boundary_max<MN>(t.G[a], mk, mp, t.tau, t.dv);
+          const long long Z = (long long)(cf + cb);
+          ok &= (long long)umax(cf, cb) <= th && O[lv - 1] + Z + (long long)X - th <= 0;
+          const long long o2 = O[lv - 1] + Z + (long long)Y - th;
+          o = o > o2 ? o : o2;
+        }
+        if (!ok) {
+          dead = lv;
+          break;
+        }
+        O[lv] = o;
+        valid = lv + 1;
+      }
+      if (dead >= 0) {
+        // every candidate below the failing prefix is decided: jump over the rest of its subtree
+        u64 rem = 1;
+        for (int j = dead + 1; j <= S - 2; ++j) rem += Bn[(L - 2 - pk_get(cuts, j)) * BK + (S - 1 - j)];
+        if (rem >= i1 - idx) break;
+        idx += rem;
+        more = after_level(dead);
+        continue;
+      }
+      if (S == 1) {  // one stage: one candidate per composition
+        u64 X, Y, AR;
+        stage_cost<MN>(t, 0, L - 1, stage_mask(sp, 1, Rp, 0), sync, X, Y, AR);
+        if ((long long)X <= th && (long long)AR <= th) improve(exact());
+        ++idx;
+        more = idx < i1 && after_level(-1);
+        continue;
+      }
+      // the row: the last cut e sweeps; Pz = the excess of the segments open after stage S-3 plus
+      // boundary S-3 into stage S-2
+      const u32 m2 = stage_mask(sp, S, Rp, S - 2), ml = stage_mask(sp, S, Rp, S - 1);
+      const int a2 = (S >= 3) ? pk_get(cuts, S - 3) + 1 : 0;
+      long long Pz = -(1ll << 62);
+      if (S >= 3) {
+        const u32 mp = stage_mask(sp, S, Rp, S - 3);
+        const u64 cf = boundary_max<MN>(t.O[a2 - 1], mp, m2, t.tau, t.dv);
+        const u64 cb = boundary_max<MN>(t.G[a2], m2, mp, t.tau, t.dv);
+        if ((long long)umax(cf, cb) > th) {  // the whole row fails on boundary S-3
+          const u64 rem = (u64)(L - 1 - pk_get(cuts, S - 2));
+          if (rem >= i1 - idx) break;
+          idx += rem;
+          more = after_level(S - 3);
+          continue;
+        }
+        Pz = O[S - 3] + (long long)(cf + cb);
+      }
+      int e = pk_get(cuts, S - 2);
+      bool moved = false;  // a candidate passed: theta drops, the prefix is re-derived
+      for (; e <= L - 2; ++e, ++idx) {
+        if (idx >= i1) break;
+        u64 X2, Y2, AR2;
+        stage_cost<MN>(t, a2, e, m2, sync, X2, Y2, AR2);
+        if ((long long)X2 > th || (long long)AR2 > th || Pz + (long long)X2 - th > 0) {
+          // stage S-2 only grows with e: the rest of the row fails
+          idx += (u64)(L - 1 - e);
+          e = L - 1;
+          break;
+        }
+        const u64 cf = boundary_max<MN>(t.O[e], m2, ml, t.tau, t.dv);
+        const u64 cb = boundary_max<MN>(t.G[e + 1], ml, m2, t.tau, t.dv);
+        if ((long long)umax(cf, cb) > th) continue;
+        u64 Xl, Yl, ARl;
+        stage_cost<MN>(t, e + 1, L - 1, ml, sync, Xl, Yl, ARl);
+        const long long o2a = (long long)X2 - th, o2b = Pz + (long long)Y2 - th;
+        const long long O2 = o2a > o2b ? o2a : o2b;
+        if ((long long)Xl > th || (long long)ARl > th || O2 + (long long)(cf + cb) + (long long)Xl - th > 0) continue;
+        // passed: T <= th < bestT, the thread's new best
+        pk_set(cuts, S - 2, e);
+        improve(exact());
+        ++idx;
+        ++e;
+        moved = true;
+        break;
+      }
+      if (idx >= i1) break;
+      if (moved && e <= L - 2) {  // continue the row from e under the new threshold
+        pk_set(cuts, S - 2, e);
+        continue;
+      }
+      more = after_level(S - 3);  // row done: the next prefix
+    }
+  }
+  block_minloc_store<NT>(bestT, bestI, cnt, out + blockIdx.x);
+}
+
 template <int NT, typename P>
 static void run_search_generic(unsigned nbk, size_t smem, cudaStream_t st, const DevTables &g, const SearchSpace &sp,
-                               u64 begin, u64 end, u64 pt, BlockOut *out, const ModelP &m, int path32) {
+                               u64 begin, u64 end, u64 pt, BlockOut *out, const ModelP &m, int path32, void *sched) {
   switch (m.sched) {
     case SCHED_2BW: k_search_generic<NT, false, SCHED_2BW, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1); break;
     case SCHED_GPIPE: k_search_generic<NT, false, SCHED_GPIPE, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1); break;
     case SCHED_DAPPLE: k_search_generic<NT, false, SCHED_DAPPLE, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1); break;
-    default:
-      if (path32 == 1) k_search_generic<NT, true, SCHED_PIPEDREAM, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1);
-      else if (path32 == 0) k_search_generic<NT, false, SCHED_PIPEDREAM, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1);
-      else {  // path chosen on the device (state_gated_out): both, writing disjoint block ranges
-        k_search_generic<NT, true, SCHED_PIPEDREAM, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, 1);
-        k_search_generic<NT, false, SCHED_PIPEDREAM, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out + nbk, m, 0);
+    default: {  // PipeDream: the threshold walk (64-bit; the state's integer path does not matter)
+      DfsSched *ds = (DfsSched *)sched;
+      if (path32 >= 0) {
+        cudaMemsetAsync(ds, 0, sizeof(DfsSched), st);
+        cudaMemsetAsync(&ds->best, 0xFF, sizeof(u64), st);
+        k_search_dfs<NT, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, ds, -1);
+      } else {  // path chosen on the device (state_gated_out): both, writing disjoint block ranges
+        cudaMemsetAsync(ds, 0, 2 * sizeof(DfsSched), st);
+        cudaMemsetAsync(&ds[0].best, 0xFF, sizeof(u64), st);
+        cudaMemsetAsync(&ds[1].best, 0xFF, sizeof(u64), st);
+        k_search_dfs<NT, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, ds, 1);
+        k_search_dfs<NT, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out + nbk, m, ds + 1, 0);
       }
+    }
   }
 }
 
 int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, u64 end, int path32, const ModelP &m,
-                          bool wide, int sms, BlockOut *out, int max_blocks, int *nblocks, cudaStream_t st) {
+                          bool wide, int sms, BlockOut *out, int max_blocks, int *nblocks, void *sched,
+                          cudaStream_t st, bool dense) {
   constexpr int NT = 256;
   const u64 span = end - begin;
+  if (dense) {
+    // a small space in one launch, latency first: every candidate scored exactly by its own thread
+    // (or two), as many blocks as the result area holds
+    const bool both = path32 < 0 && m.sched == SCHED_PIPEDREAM;
+    const u64 room = both ? (u64)max_blocks / 2 : (u64)max_blocks;
+    u64 per = (span + room * NT - 1) / (room * NT);
+    if (per == 0) per = 1;
+    u64 blocks = (span + per * NT - 1) / (per * NT);
+    if (blocks == 0) blocks = 1;
+    const int BK = wide ? BINOM_K : BK8;
+    const size_t smem = ((size_t)smem_words(g.L, g.N) +
+                         (size_t)(((int)g.L + 1 > MAXNW + 1 ? (int)g.L + 1 : MAXNW + 1) * BK)) * sizeof(u64);
+    ModelP mm = m;
+    const unsigned nbk = (unsigned)blocks;
+#define DENSE_LAUNCH(PT)                                                                                  \
+  if (m.sched != SCHED_PIPEDREAM) run_search_generic<NT, PT>(nbk, smem, st, g, sp, begin, end, per, out, mm, path32, sched); \
+  else if (path32 == 1) k_search_generic<NT, true, SCHED_PIPEDREAM, PT><<<nbk, NT, smem, st>>>(g, sp, begin, end, per, out, mm, -1); \
+  else if (path32 == 0) k_search_generic<NT, false, SCHED_PIPEDREAM, PT><<<nbk, NT, smem, st>>>(g, sp, begin, end, per, out, mm, -1); \
+  else {                                                                                                  \
+    k_search_generic<NT, true, SCHED_PIPEDREAM, PT><<<nbk, NT, smem, st>>>(g, sp, begin, end, per, out, mm, 1); \
+    k_search_generic<NT, false, SCHED_PIPEDREAM, PT><<<nbk, NT, smem, st>>>(g, sp, begin, end, per, out + nbk, mm, 0); \
+  }
+    if (wide) { DENSE_LAUNCH(P16) } else { DENSE_LAUNCH(P8) }
+#undef DENSE_LAUNCH
+    *nblocks = (int)blocks * (both ? 2 : 1);
+    return both ? 2 : 1;
+  }
   // at least 4 candidates per thread (the unrank is a few binary searches); up to 8 blocks per SM.
   // A flushed schedule costs ~M S stage steps per candidate: one candidate per thread is enough.
   // A small span (a launch of a short model's space) is latency-bound: one candidate per thread.
@@ -164,14 +478,27 @@ int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, 
   const u64 cap = (u64)sms * 8 < room ? (u64)sms * 8 : room;
   if (blocks > cap) blocks = cap;
   if (blocks == 0) blocks = 1;
-  const u64 per = (span + blocks * NT - 1) / (blocks * NT);
+  u64 per = (span + blocks * NT - 1) / (blocks * NT);
+  if (m.sched == SCHED_PIPEDREAM) {
+    // the threshold walk: one wave of resident blocks drawing chunks of about span / (8 x threads)
+    // candidates (at least DFS_MINCH) from the launch's counter
+    const u64 wave = (u64)sms * DFS_MINB < room ? (u64)sms * DFS_MINB : room;
+    u64 chunk = span / (wave * NT * 8);
+    if (chunk < (u64)DFS_MINCH) chunk = DFS_MINCH;
+    while ((span + chunk - 1) / chunk >= (1ull << 31)) chunk *= 2;
+    const u64 nch = (span + chunk - 1) / chunk;
+    blocks = (nch + NT - 1) / NT;
+    if (blocks > wave) blocks = wave;
+    if (blocks == 0) blocks = 1;
+    per = chunk;
+  }
   const int BK = wide ? BINOM_K : BK8;
   const size_t smem = ((size_t)smem_words(g.L, g.N) +
                        (size_t)(((int)g.L + 1 > MAXNW + 1 ? (int)g.L + 1 : MAXNW + 1) * BK)) * sizeof(u64);
   const unsigned nbk = (unsigned)blocks;
   const u64 pt = per ? per : 1;
-  if (wide) run_search_generic<NT, P16>(nbk, smem, st, g, sp, begin, end, pt, out, m, path32);
-  else run_search_generic<NT, P8>(nbk, smem, st, g, sp, begin, end, pt, out, m, path32);
+  if (wide) run_search_generic<NT, P16>(nbk, smem, st, g, sp, begin, end, pt, out, m, path32, sched);
+  else run_search_generic<NT, P8>(nbk, smem, st, g, sp, begin, end, pt, out, m, path32, sched);
   *nblocks = (int)blocks * (both ? 2 : 1);
   return both ? 2 : 1;
 }

@@ -85,6 +85,24 @@ __global__ void k_build_state(DevTables g, const u64 *__restrict__ fp, const u64
       const int u = i / TAUW, v = i % TAUW;
       g.tau[i] = (u < N && v < N && u != v) ? tau[u * N + v] : 0ull;
     }
+    // ring[mask]: the slowest link of the ring W[0] -> W[1] -> ... -> W[0] over each worker set of up
+    // to 8 workers (ascending order; row a6), 0 for sets of fewer than 2
+    for (int msk = lane; msk < 256; msk += 32) {
+      u64 tr = 0;
+      if (__popc(msk) >= 2 && msk < (1 << (N < 8 ? N : 8))) {
+        const int first = __ffs(msk) - 1;
+        int prev = first;
+        int mm = msk & (msk - 1);
+        while (mm) {
+          const int w = __ffs(mm) - 1;
+          mm &= mm - 1;
+          tr = umax(tr, tau[prev * N + w]);
+          prev = w;
+        }
+        tr = umax(tr, tau[prev * N + first]);
+      }
+      g.ring[msk] = tr;
+    }
     u64 mt = 0;
     for (int i = lane; i < N * N; i += 32)
       if (i / N != i % N) mt = umax(mt, tau[i]);

@@ -28,6 +28,15 @@ def eng():
     e.close()
 
 
+@pytest.fixture(params=[False, True], ids=["dense", "split"])
+def split(request, eng):
+    """Both kernel selections of the search (autopipe_set_search_options): the dense launch for
+    small ranges (default) and the per-S split (r = 1 sweep + threshold walk) forced."""
+    eng.set_search_options(request.param)
+    yield request.param
+    eng.set_search_options(False)
+
+
 def gpu_eval(eng, recs):
     from paper_conf_icpp_hulww24_b200 import as_u64
     if isinstance(recs, np.ndarray):
@@ -57,7 +66,7 @@ def test_toy_every_candidate(eng):
 
 
 @pytest.mark.parametrize("flags", [0, USE_ALL_WORKERS])
-def test_toy_search(eng, flags):
+def test_toy_search(eng, flags, split):
     prof, st = W.toy(), W.toy_state()
     eng.load(prof, st)
     T, idx, part, n = brute_force(prof, st, 1, 4, flags)
@@ -114,7 +123,7 @@ def test_invalid_records(eng):
 # ------------------------------------------------------------------------------------------------
 
 @pytest.mark.parametrize("seed", range(4))
-def test_random_search_and_shards(eng, seed):
+def test_random_search_and_shards(eng, seed, split):
     rng = np.random.default_rng(200 + seed)
     for it in range(5):
         L = int(rng.integers(2, 12))
@@ -155,7 +164,7 @@ def _sample_parity(eng, prof, st, smin, smax, flags, n, seed):
     assert gpu_eval(eng, recs) == score_many(prof, st, recs)
 
 
-def test_vgg16_sample_and_optimum(eng):
+def test_vgg16_sample_and_optimum(eng, split):
     prof, st = W.vgg16(), W.vgg_state()
     eng.load(prof, st)
     _sample_parity(eng, prof, st, 1, 8, 0, 10_000, 12345)
@@ -174,7 +183,7 @@ def test_vgg16_random_placement_records(eng):
 
 
 @pytest.mark.parametrize("name", ["gnmt16", "bert24"])
-def test_trace_states(eng, name):
+def test_trace_states(eng, name, split):
     """C3: the fluctuation trace re-scored per state switch; each optimum equals the param DP."""
     prof = W.profile(name)
     for st in W.trace_c3(prof):
@@ -298,7 +307,7 @@ def _all_records(L, N, smin, smax, flags):
 
 
 @pytest.mark.parametrize("S,L,uniform", [(5, 22, False), (6, 24, True), (7, 20, False), (8, 19, True)])
-def test_r1_kernel_shards_and_ties(eng, S, L, uniform):
+def test_r1_kernel_shards_and_ties(eng, S, L, uniform, split):
     rng = np.random.default_rng(300 + S)
     if uniform:   # identical layers and workers: huge numbers of exact ties in T
         prof = W.Profile("u", [1000] * L, [1000] * L, [0] * L, [7] * L, [13] * L)
@@ -326,7 +335,7 @@ def test_r1_kernel_shards_and_ties(eng, S, L, uniform):
 
 
 @pytest.mark.parametrize("kind", ["a-nvlink", "b"])
-def test_gpt96_shard_boundaries_vs_oracle(eng, kind):
+def test_gpt96_shard_boundaries_vs_oracle(eng, kind, split):
     """Full size, in the launch configuration bench.py times: the 96-layer, 8-stage space split into
     the 8 cost-balanced shards of the multi-GPU split. Around every inner shard boundary a window of
     candidates straddling it is searched on the GPU as two pieces (the end of the left shard, the

@@ -25,6 +25,15 @@ def eng():
     e.close()
 
 
+@pytest.fixture(params=[False, True], ids=["dense", "split"])
+def split(request, eng):
+    """Both kernel selections of the search: the dense launch (default for small ranges) and the
+    per-S split (threshold walk) forced."""
+    eng.set_search_options(request.param)
+    yield request.param
+    eng.set_search_options(False)
+
+
 def gpu_eval(eng, recs):
     from paper_conf_icpp_hulww24_b200 import as_u64
     if isinstance(recs, list):
@@ -102,7 +111,7 @@ def _brute(prof, st, L, N, smin, smax, flags):
 
 
 @pytest.mark.parametrize("case", ["n10", "s11", "s15", "s16"])
-def test_search_wide_small_spaces(eng, case):
+def test_search_wide_small_spaces(eng, case, split):
     """Wide exhaustive search = the oracle's minimum over the enumeration (first minimum wins), for 10
     workers and for spaces whose stages exceed 8, with both flags and a shard split."""
     rng = np.random.default_rng({"n10": 1, "s11": 2, "s15": 3, "s16": 4}[case])
@@ -125,7 +134,7 @@ def test_search_wide_small_spaces(eng, case):
 
 
 @pytest.mark.parametrize("name,smax", [("vgg16", 8), ("gnmt16", 8)])
-def test_wide_search_equals_16_byte_search(eng, name, smax):
+def test_wide_search_equals_16_byte_search(eng, name, smax, split):
     """For N <= 8 the wide search scans the same index order with the same kernels (the fast r = 1
     kernel for S >= 5): same optimum, same index, the record in its wide form."""
     prof = W.profile(name)
