@@ -271,6 +271,14 @@ int autopipe_decode_index_w(const autopipe_ctx *ctx, uint32_t s_min, uint32_t s_
  *                 AUTOPIPE_SCHED_2BW        the same steady state, one sync per M micro-batches;
  *                 AUTOPIPE_SCHED_GPIPE      one flushed iteration: F(0..M-1) then B(0..M-1) per worker;
  *                 AUTOPIPE_SCHED_DAPPLE     one flushed iteration in 1F1B order (min(S-s, M) warm-up);
+ *                 AUTOPIPE_SCHED_PIPEDREAM_RR  PipeDream's round-robin replicas (row f4, reading F-5,
+ *                                   PAPER.md:371-377): a replicated stage takes whole mini-batches in
+ *                                   turn (replica k mod r_s), each replica 1F1B with ceil(R_s / r_s) of
+ *                                   its own in flight (R_s = workers of stages s..S-1), one transfer per
+ *                                   boundary and mini-batch, one sync per r_s mini-batches; M = 1;
+ *                                   16-byte records only (N <= 8; wide calls E_INVAL), the state's bound
+ *                                   < 2^45 (E_OVERFLOW); a record whose schedule is not periodic within
+ *                                   2^18 rounds scores AUTOPIPE_T_UNRESOLVED;
  *   sync          AUTOPIPE_SYNC_RING (default) or AUTOPIPE_SYNC_PS (a parameter server sharded over
  *                 the stage's replicas, each server taking its pushes and pulls one at a time);
  *   micro_batches M >= 1 micro-batches per iteration (must be 1 for PIPEDREAM; <= 65536);
@@ -286,6 +294,8 @@ int autopipe_decode_index_w(const autopipe_ctx *ctx, uint32_t s_min, uint32_t s_
 #define AUTOPIPE_SCHED_2BW 1u
 #define AUTOPIPE_SCHED_GPIPE 2u
 #define AUTOPIPE_SCHED_DAPPLE 3u
+#define AUTOPIPE_SCHED_PIPEDREAM_RR 4u
+#define AUTOPIPE_T_UNRESOLVED 0xFFFFFFFFFFFFFFFEull
 #define AUTOPIPE_SYNC_RING 0u
 #define AUTOPIPE_SYNC_PS 1u
 #define AUTOPIPE_RECOMPUTE 1u

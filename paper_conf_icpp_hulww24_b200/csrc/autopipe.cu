@@ -405,10 +405,20 @@ static int sync_status(autopipe_ctx *c, cudaStream_t st) {
 // Row f3: a schedule other than PipeDream scales sums by up to 16 (M + 1) (an iteration of M
 // micro-batches, recomputation, every op and transfer on a critical path); refuse states for which
 // that could reach 2^63. Reads the device status first for a state set from device memory.
-static int check_model(autopipe_ctx *c, cudaStream_t st) {
+static int check_model(autopipe_ctx *c, cudaStream_t st, bool wide = false) {
   if (c->model.sched == SCHED_PIPEDREAM) return AUTOPIPE_OK;
+  if (c->model.sched == SCHED_RR && wide)
+    return fail(c, AUTOPIPE_E_INVAL, "round-robin replicas use 16-byte records (no wide calls)");
   int rc = sync_status(c, st);
   if (rc) return rc;
+  if (c->model.sched == SCHED_RR) {
+    // row f4, round-robin replicas: 16-byte records only; the recurrence runs up to 2^18 rounds and
+    // accumulates the shift of a period, so the state's bound must stay below 2^45 ns
+    if (c->N > (u32)MAXN) return fail(c, AUTOPIPE_E_INVAL, "round-robin replicas use 16-byte records: N <= 8");
+    if (c->bound >= (1ull << 45))
+      return fail(c, AUTOPIPE_E_OVERFLOW, "round-robin replicas need the state's bound below 2^45 ns");
+    return AUTOPIPE_OK;
+  }
   if ((u128)c->bound * 16u * ((u128)c->model.M + 1) >= ((u128)1 << 63))
     return fail(c, AUTOPIPE_E_OVERFLOW, "16 (M + 1) x the state's bound reaches 2^63 ns");
   return AUTOPIPE_OK;
@@ -418,12 +428,12 @@ extern "C" int autopipe_set_schedule(autopipe_ctx *c, uint32_t schedule, uint32_
                                      uint32_t flags) {
   if (!c) return AUTOPIPE_E_INVAL;
   c->err[0] = 0;
-  if (schedule > AUTOPIPE_SCHED_DAPPLE) return fail(c, AUTOPIPE_E_INVAL, "unknown schedule %u", schedule);
+  if (schedule > AUTOPIPE_SCHED_PIPEDREAM_RR) return fail(c, AUTOPIPE_E_INVAL, "unknown schedule %u", schedule);
   if (sync > AUTOPIPE_SYNC_PS) return fail(c, AUTOPIPE_E_INVAL, "unknown sync scheme %u", sync);
   if (micro_batches < 1 || micro_batches > AUTOPIPE_MAX_MICRO_BATCHES)
     return fail(c, AUTOPIPE_E_INVAL, "micro_batches = %u outside [1, %u]", micro_batches, AUTOPIPE_MAX_MICRO_BATCHES);
-  if (schedule == AUTOPIPE_SCHED_PIPEDREAM && micro_batches != 1)
-    return fail(c, AUTOPIPE_E_INVAL, "the PipeDream schedule has one mini-batch per iteration (M = 1)");
+  if ((schedule == AUTOPIPE_SCHED_PIPEDREAM || schedule == AUTOPIPE_SCHED_PIPEDREAM_RR) && micro_batches != 1)
+    return fail(c, AUTOPIPE_E_INVAL, "the PipeDream schedules have one mini-batch per iteration (M = 1)");
   if (flags & ~AUTOPIPE_RECOMPUTE) return fail(c, AUTOPIPE_E_INVAL, "unknown flags 0x%x", flags);
   if ((flags & AUTOPIPE_RECOMPUTE) && schedule != AUTOPIPE_SCHED_GPIPE)
     return fail(c, AUTOPIPE_E_INVAL, "AUTOPIPE_RECOMPUTE applies to the GPipe schedule only");
@@ -453,7 +463,7 @@ static int eval_impl(autopipe_ctx *c, const void *d_parts, uint64_t count, bool 
   if (count == 0) return AUTOPIPE_OK;
   if (!d_parts || !d_time_ns) return fail(c, AUTOPIPE_E_INVAL, "NULL device pointer");
   DeviceGuard dg(c->device);
-  int rc = check_model(c, (cudaStream_t)stream);
+  int rc = check_model(c, (cudaStream_t)stream, wide);
   if (rc) return rc;
   // a state given in device memory has not been classified on the host yet: use the 64-bit path
   const int p32 = c->state_on_device ? 0 : (c->path32 | (c->narrow << 1));
@@ -621,7 +631,7 @@ static int search_impl(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, u64 beg
   } else {
     rc = sync_status(c, st);
     if (rc) return rc;
-    rc = check_model(c, st);
+    rc = check_model(c, st, wide);
     if (rc) return rc;
     path = c->path32;
   }
@@ -915,7 +925,7 @@ static int rollout_impl(autopipe_ctx *c, const void *d_parts, uint64_t count, co
   if (count == 0) return AUTOPIPE_OK;
   if (!d_parts || !d_time_ns) return fail(c, AUTOPIPE_E_INVAL, "NULL device pointer");
   DeviceGuard dg(c->device);
-  int rc = check_model(c, (cudaStream_t)stream);
+  int rc = check_model(c, (cudaStream_t)stream, wide);
   if (rc) return rc;
   const int p32 = c->state_on_device ? 0 : (c->path32 | (c->narrow << 1));
   c->launches += launch_eval(c->tab, d_parts, count, wide, (u64 *)d_time_ns, (u64 *)d_switch_bytes,

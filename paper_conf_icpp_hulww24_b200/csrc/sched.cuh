@@ -17,6 +17,7 @@
 // ready-driven execution exactly.
 #pragma once
 #include "eval.cuh"
+#include "rr.cuh"
 
 namespace ap {
 
@@ -189,12 +190,18 @@ __device__ __forceinline__ u64 flush_makespan(const SmemTab &t, int S, const P &
   return T;
 }
 
-// T_ns of a validated partition under the model (row f3): MODE = the schedule, fixed per kernel.
+// T_ns of a validated partition under the model (rows f3, f4): MODE = the schedule, fixed per kernel.
+// Round-robin replicas (SCHED_RR) are defined for 16-byte records (the host refuses wide ones).
 template <int MODE, bool P32, typename P>
 __device__ __forceinline__ u64 model_time(const SmemTab &t, int S, const P &p, const ModelP &m) {
+  if constexpr (MODE == SCHED_RR) {
+    if constexpr (P::MS == 8) return rr_time(t, S, p, (int)m.sync);
+    else return U64MAX;
+  }
   if (MODE == SCHED_PIPEDREAM) return eval_closed_form<P32, false, P>(t, S, p, (int)m.sync);
   if (MODE == SCHED_2BW) return eval_closed_form<false, true, P>(t, S, p, (int)m.sync, m.M);
-  return flush_makespan<MODE == SCHED_PIPEDREAM || MODE == SCHED_2BW ? SCHED_GPIPE : MODE, P>(t, S, p, m);
+  return flush_makespan<(MODE == SCHED_PIPEDREAM || MODE == SCHED_2BW || MODE == SCHED_RR) ? SCHED_GPIPE : MODE, P>(
+      t, S, p, m);
 }
 
 }  // namespace ap

@@ -301,8 +301,9 @@ class Engine:
     def set_schedule(self, schedule: int = _lib.SCHED_PIPEDREAM, sync: int = _lib.SYNC_RING,
                      micro_batches: int = 1, recompute: bool = False) -> None:
         """Select the model every later scoring call evaluates: the schedule (SCHED_PIPEDREAM, _2BW,
-        _GPIPE, _DAPPLE), the data-parallel sync (SYNC_RING, SYNC_PS), M micro-batches per
-        iteration and GPipe's forward recomputation. Times are then per iteration of M micro-batches."""
+        _GPIPE, _DAPPLE, or SCHED_PIPEDREAM_RR: round-robin replicas, row f4), the data-parallel sync
+        (SYNC_RING, SYNC_PS), M micro-batches per iteration and GPipe's forward recomputation. Times
+        are then per iteration of M micro-batches."""
         self._check(lib.autopipe_set_schedule(self._h, int(schedule), int(sync), int(micro_batches),
                                               _lib.RECOMPUTE if recompute else 0))
 

@@ -91,3 +91,20 @@ def sched_many(prof, st, records: Sequence[bytes], schedule: int, sync: int, M: 
         return [_sched_one(a) for a in args]
     with mp.get_context("fork").Pool(procs, initializer=_init, initargs=(prof, st)) as pool:
         return pool.map(_sched_one, args, chunksize=max(1, len(args) // (procs * 8)))
+
+
+def _rr_one(args):
+    from oracle.roundrobin import score_record
+    rec, sync = args
+    return score_record(_CTX["prof"], _CTX["st"], rec, sync)
+
+
+def rr_many(prof, st, records: Sequence[bytes], sync: int = 0, procs: int = 0) -> List[int]:
+    """oracle.roundrobin.score_record (row f4, round-robin replicas) over many records."""
+    args = [(bytes(r), sync) for r in records]
+    procs = procs or cores()
+    if procs <= 1 or len(args) < 64:
+        _init(prof, st)
+        return [_rr_one(a) for a in args]
+    with mp.get_context("fork").Pool(procs, initializer=_init, initargs=(prof, st)) as pool:
+        return pool.map(_rr_one, args, chunksize=max(1, len(args) // (procs * 8)))
