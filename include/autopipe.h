@@ -279,6 +279,14 @@ int autopipe_decode_index_w(const autopipe_ctx *ctx, uint32_t s_min, uint32_t s_
  *                                   16-byte records only (N <= 8; wide calls E_INVAL), the state's bound
  *                                   < 2^45 (E_OVERFLOW); a record whose schedule is not periodic within
  *                                   2^18 rounds scores AUTOPIPE_T_UNRESOLVED;
+ *                 AUTOPIPE_SCHED_CHIMERA    Chimera's bidirectional pipelines (row f3, reading F-6,
+ *                                   PAPER.md:308-314, 1341-1350): one worker per stage; stage s on w_s
+ *                                   (down) and on w_{S-1-s} (up); ceil(M/2) micro-batches down,
+ *                                   floor(M/2) up, each pipeline in DAPPLE order, a worker's two lists
+ *                                   interleaved by readiness (earliest start; ties: lower down stage,
+ *                                   then down), the two copies of a stage synchronised after their last
+ *                                   backwards; one flushed iteration; 16-byte records only; a record
+ *                                   with a replicated stage scores UINT64_MAX;
  *   sync          AUTOPIPE_SYNC_RING (default) or AUTOPIPE_SYNC_PS (a parameter server sharded over
  *                 the stage's replicas, each server taking its pushes and pulls one at a time);
  *   micro_batches M >= 1 micro-batches per iteration (must be 1 for PIPEDREAM; <= 65536);
@@ -295,6 +303,7 @@ int autopipe_decode_index_w(const autopipe_ctx *ctx, uint32_t s_min, uint32_t s_
 #define AUTOPIPE_SCHED_GPIPE 2u
 #define AUTOPIPE_SCHED_DAPPLE 3u
 #define AUTOPIPE_SCHED_PIPEDREAM_RR 4u
+#define AUTOPIPE_SCHED_CHIMERA 5u
 #define AUTOPIPE_T_UNRESOLVED 0xFFFFFFFFFFFFFFFEull
 #define AUTOPIPE_SYNC_RING 0u
 #define AUTOPIPE_SYNC_PS 1u

@@ -407,8 +407,10 @@ static int sync_status(autopipe_ctx *c, cudaStream_t st) {
 // that could reach 2^63. Reads the device status first for a state set from device memory.
 static int check_model(autopipe_ctx *c, cudaStream_t st, bool wide = false) {
   if (c->model.sched == SCHED_PIPEDREAM) return AUTOPIPE_OK;
-  if (c->model.sched == SCHED_RR && wide)
-    return fail(c, AUTOPIPE_E_INVAL, "round-robin replicas use 16-byte records (no wide calls)");
+  if ((c->model.sched == SCHED_RR || c->model.sched == SCHED_CHIMERA) && wide)
+    return fail(c, AUTOPIPE_E_INVAL, "round-robin replicas and Chimera use 16-byte records (no wide calls)");
+  if (c->model.sched == SCHED_CHIMERA && c->N > (u32)MAXN)
+    return fail(c, AUTOPIPE_E_INVAL, "Chimera uses 16-byte records: N <= 8");
   int rc = sync_status(c, st);
   if (rc) return rc;
   if (c->model.sched == SCHED_RR) {
@@ -428,7 +430,7 @@ extern "C" int autopipe_set_schedule(autopipe_ctx *c, uint32_t schedule, uint32_
                                      uint32_t flags) {
   if (!c) return AUTOPIPE_E_INVAL;
   c->err[0] = 0;
-  if (schedule > AUTOPIPE_SCHED_PIPEDREAM_RR) return fail(c, AUTOPIPE_E_INVAL, "unknown schedule %u", schedule);
+  if (schedule > AUTOPIPE_SCHED_CHIMERA) return fail(c, AUTOPIPE_E_INVAL, "unknown schedule %u", schedule);
   if (sync > AUTOPIPE_SYNC_PS) return fail(c, AUTOPIPE_E_INVAL, "unknown sync scheme %u", sync);
   if (micro_batches < 1 || micro_batches > AUTOPIPE_MAX_MICRO_BATCHES)
     return fail(c, AUTOPIPE_E_INVAL, "micro_batches = %u outside [1, %u]", micro_batches, AUTOPIPE_MAX_MICRO_BATCHES);

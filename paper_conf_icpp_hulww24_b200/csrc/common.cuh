@@ -47,7 +47,7 @@ struct DevTables {
 };
 
 // The model a scoring call evaluates (NEXT row f3, reading F-3; autopipe_set_schedule).
-enum { SCHED_PIPEDREAM = 0, SCHED_2BW = 1, SCHED_GPIPE = 2, SCHED_DAPPLE = 3, SCHED_RR = 4 };
+enum { SCHED_PIPEDREAM = 0, SCHED_2BW = 1, SCHED_GPIPE = 2, SCHED_DAPPLE = 3, SCHED_RR = 4, SCHED_CHIMERA = 5 };
 enum { SYNC_RING = 0, SYNC_PS = 1 };
 struct ModelP {
   u32 sched;      // SCHED_*

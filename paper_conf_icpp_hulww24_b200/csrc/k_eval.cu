@@ -120,6 +120,7 @@ static void dispatch_eval(int sms, size_t smem, cudaStream_t st, const DevTables
     case SCHED_GPIPE: run_eval<ROLLOUT, false, SCHED_GPIPE, Rec, P>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m, ctr); break;
     case SCHED_DAPPLE: run_eval<ROLLOUT, false, SCHED_DAPPLE, Rec, P>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m, ctr); break;
     case SCHED_RR: run_eval<ROLLOUT, false, SCHED_RR, Rec, P>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m, ctr); break;
+    case SCHED_CHIMERA: run_eval<ROLLOUT, false, SCHED_CHIMERA, Rec, P>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m, ctr); break;
     default:  // path32: bit 0 = 32-bit segment sums, bit 1 = narrow stage and shard arithmetic
       switch (path32 & 3) {
         case 3: run_eval<ROLLOUT, true, SCHED_PIPEDREAM, Rec, P, true>(sms, smem, st, g, recs, count, out_t, out_sw, cur, m, ctr); break;

@@ -419,6 +419,7 @@ static void run_search_generic(unsigned nbk, size_t smem, cudaStream_t st, const
     case SCHED_GPIPE: k_search_generic<NT, false, SCHED_GPIPE, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1); break;
     case SCHED_DAPPLE: k_search_generic<NT, false, SCHED_DAPPLE, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1); break;
     case SCHED_RR: k_search_generic<NT, false, SCHED_RR, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1); break;
+    case SCHED_CHIMERA: k_search_generic<NT, false, SCHED_CHIMERA, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1); break;
     default: {  // PipeDream: the threshold walk (64-bit; the state's integer path does not matter)
       DfsSched *ds = (DfsSched *)sched;
       if (path32 >= 0) {
@@ -471,7 +472,7 @@ int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, 
   // at least 4 candidates per thread (the unrank is a few binary searches); up to 8 blocks per SM.
   // A flushed schedule costs ~M S stage steps per candidate: one candidate per thread is enough.
   // A small span (a launch of a short model's space) is latency-bound: one candidate per thread.
-  const u64 min_per = (m.sched == SCHED_GPIPE || m.sched == SCHED_DAPPLE || m.sched == SCHED_RR ||
+  const u64 min_per = (m.sched == SCHED_GPIPE || m.sched == SCHED_DAPPLE || m.sched == SCHED_RR || m.sched == SCHED_CHIMERA ||
                        span <= (u64)sms * 8 * NT * 4) ? 1 : 4;
   u64 threads = (span + min_per - 1) / min_per;
   u64 blocks = (threads + NT - 1) / NT;

@@ -17,6 +17,7 @@
 // ready-driven execution exactly.
 #pragma once
 #include "eval.cuh"
+#include "chimera.cuh"
 #include "rr.cuh"
 
 namespace ap {
@@ -198,9 +199,14 @@ __device__ __forceinline__ u64 model_time(const SmemTab &t, int S, const P &p, c
     if constexpr (P::MS == 8) return rr_time(t, S, p, (int)m.sync);
     else return U64MAX;
   }
+  if constexpr (MODE == SCHED_CHIMERA) {  // row f3, reading F-6; 16-byte records (host-checked)
+    if constexpr (P::MS == 8) return chimera_time(t, S, p, m);
+    else return U64MAX;
+  }
   if (MODE == SCHED_PIPEDREAM) return eval_closed_form<P32, false, P>(t, S, p, (int)m.sync);
   if (MODE == SCHED_2BW) return eval_closed_form<false, true, P>(t, S, p, (int)m.sync, m.M);
-  return flush_makespan<(MODE == SCHED_PIPEDREAM || MODE == SCHED_2BW || MODE == SCHED_RR) ? SCHED_GPIPE : MODE, P>(
+  return flush_makespan<(MODE == SCHED_PIPEDREAM || MODE == SCHED_2BW || MODE == SCHED_RR || MODE == SCHED_CHIMERA)
+                            ? SCHED_GPIPE : MODE, P>(
       t, S, p, m);
 }
 

@@ -108,3 +108,20 @@ def rr_many(prof, st, records: Sequence[bytes], sync: int = 0, procs: int = 0) -
         return [_rr_one(a) for a in args]
     with mp.get_context("fork").Pool(procs, initializer=_init, initargs=(prof, st)) as pool:
         return pool.map(_rr_one, args, chunksize=max(1, len(args) // (procs * 8)))
+
+
+def _ch_one(args):
+    from oracle.chimera import score_record
+    rec, M, sync = args
+    return score_record(_CTX["prof"], _CTX["st"], rec, M, sync)
+
+
+def chimera_many(prof, st, records: Sequence[bytes], M: int, sync: int = 0, procs: int = 0) -> List[int]:
+    """oracle.chimera.score_record (row f3, Chimera) over many records."""
+    args = [(bytes(r), M, sync) for r in records]
+    procs = procs or cores()
+    if procs <= 1 or len(args) < 64:
+        _init(prof, st)
+        return [_ch_one(a) for a in args]
+    with mp.get_context("fork").Pool(procs, initializer=_init, initargs=(prof, st)) as pool:
+        return pool.map(_ch_one, args, chunksize=max(1, len(args) // (procs * 8)))
