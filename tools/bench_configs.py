@@ -112,7 +112,9 @@ def measure(device: int = 0, rollout_records: int = 1 << 20):
                          ("pipedream_ps", (L_.SCHED_PIPEDREAM, L_.SYNC_PS, 1, False)),
                          ("2bw_M8", (L_.SCHED_2BW, L_.SYNC_RING, 8, False)),
                          ("gpipe_M8_recompute", (L_.SCHED_GPIPE, L_.SYNC_RING, 8, True)),
-                         ("dapple_M8", (L_.SCHED_DAPPLE, L_.SYNC_RING, 8, False))):
+                         ("dapple_M8", (L_.SCHED_DAPPLE, L_.SYNC_RING, 8, False)),
+                         ("chimera_M8", (L_.SCHED_CHIMERA, L_.SYNC_RING, 8, False)),
+                         ("pipedream_rr", (L_.SCHED_PIPEDREAM_RR, L_.SYNC_RING, 1, False))):
         eng.set_schedule(*model)
         ms, r = _timed(lambda: eng.search_optimum(1, 8), reps=3, warm=1)
         rec = r.partition
@@ -129,6 +131,27 @@ def measure(device: int = 0, rollout_records: int = 1 << 20):
         eng.set_schedule(*model)
         ms, _ = _timed(lambda: eng.eval_partitions(recs, out=out_t))
         f3[label] = {"records": rollout_records, "ms": ms, "records_per_s": rollout_records / (ms / 1e3)}
+    # Chimera (reading F-6): one worker per stage, ResNet-50 one-worker-per-stage records
+    import numpy as _np
+    rng = _np.random.default_rng(77)
+    crecs = []
+    for _ in range(min(rollout_records, 1 << 16)):  # 64k distinct records, tiled to the batch size
+        S_ = int(rng.integers(1, st.N + 1))
+        cuts = sorted(int(x) for x in rng.choice(prof.L - 1, S_ - 1, replace=False)) if S_ > 1 else []
+        sow = [W.IDLE] * 8
+        for s_, w_ in enumerate(int(x) for x in rng.permutation(st.N)[:S_]):
+            sow[w_] = s_
+        crecs.append(W.encode(S_, cuts, sow))
+    crecs = _np.frombuffer(b"".join(crecs), dtype=_np.uint8).reshape(-1, 16)
+    crecs = torch.from_numpy(_np.ascontiguousarray(_np.resize(crecs, (rollout_records, 16)))).cuda()
+    eng.set_schedule(L_.SCHED_CHIMERA, L_.SYNC_RING, 8, False)
+    ms, _ = _timed(lambda: eng.eval_partitions(crecs, out=out_t))
+    f3["rollout_chimera_M8"] = {"records": rollout_records, "ms": ms, "records_per_s": rollout_records / (ms / 1e3),
+                                "records_kind": "one worker per stage (Chimera partitions)"}
+    eng.set_schedule(L_.SCHED_PIPEDREAM_RR, L_.SYNC_RING, 1, False)
+    ms, _ = _timed(lambda: eng.eval_partitions(recs, out=out_t))
+    f3["rollout_pipedream_rr"] = {"records": rollout_records, "ms": ms, "records_per_s": rollout_records / (ms / 1e3),
+                                  "row": "f4 round-robin replicas"}
     eng.set_schedule()
     res["F3_schedules_bert24_M8"] = dict(candidates=n, **f3)
     # f4: the paper's 10-GPU testbed (wide records): exhaustive S <= 10 search of VGG-16 and

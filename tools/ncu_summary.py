@@ -61,5 +61,38 @@ def full(path):
                 print("  %-72s %s %s" % (k, r[i], units[i]))
 
 
+def short(name):
+    name = re.sub(r"\(.*", "", name).replace("void ", "").replace("ap::", "")
+    name = name.replace("unsigned long long", "u64").replace("unsigned int", "u32").replace("(bool)", "")
+    name = name.replace("(int)", "").replace(", 256>", ">").replace(" ", "")
+    return name
+
+
+def traffic(path):
+    """JSON of dram read + write bytes per captured launch (bench.py's roofline `traffic`)."""
+    import json
+    out = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    rows = list(csv.reader(io.StringIO(out)))
+    hdr, units = rows[0], rows[1]
+    res = OrderedDict()
+    for r in rows[2:]:
+        b = 0.0
+        for k in ("dram__bytes_read.sum", "dram__bytes_write.sum"):
+            i = hdr.index(k)
+            scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(units[i], 1)
+            b += float(r[i].replace(",", "")) * scale
+        name = short(r[hdr.index("Kernel Name")])
+        if name.startswith("k_search_r1<8,"):
+            name = name.split(",")[0] + "," + name.split(",")[1] + ">" if name.count(",") >= 2 else name
+        key = name
+        n = 2
+        while key in res:
+            key = "%s#%d" % (name, n)
+            n += 1
+        res[key] = int(b)
+    res["source"] = "ncu --set full, one launch each (tools/profile_kernels.py)"
+    print(json.dumps(res, indent=1))
+
+
 if __name__ == "__main__":
-    {"launches": launches, "full": full}[sys.argv[1]](sys.argv[2])
+    {"launches": launches, "full": full, "traffic": traffic}[sys.argv[1]](sys.argv[2])

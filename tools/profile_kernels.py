@@ -1,7 +1,9 @@
 #!/usr/bin/env python
-"""One launch of each hot kernel, for ncu captures (not a benchmark):
-C4a search (u32 path), C4b search (u64 path), one 1M-record rollout batch (ResNet-50, App. B C5),
-and one 1M-record switch-reward batch (NEXT row f2)."""
+"""One launch of each hot kernel, for ncu captures (not a benchmark), in this order:
+C4a search (k_search_r1 u32 path), C4b search (u64 path), the 1M-record C5 ResNet-50 rollout and eval
+(k_eval, narrow path), switch rewards (k_switch, f2), DAPPLE M = 8 eval (f3), the 10-GPU ResNet-50
+testbed search (k_search_dfs, f4 wide), C2 VGG-16 (dense k_search_generic), round-robin replicas
+(f4) and Chimera (f3) on 64k records."""
 import os
 import sys
 
@@ -16,6 +18,7 @@ import __graft_entry__  # noqa: E402
 __graft_entry__.build()
 import workloads as W  # noqa: E402
 from paper_conf_icpp_hulww24_b200 import Engine  # noqa: E402
+from paper_conf_icpp_hulww24_b200 import _lib as L_  # noqa: E402
 
 eng = Engine(0)
 for kind in ("a-nvlink", "b"):
@@ -33,14 +36,23 @@ torch.cuda.synchronize()
 print("rollout", int((t == t2).all()))
 out = eng.switch_rewards(recs, bytes(recs[0].cpu().numpy()), 100)
 torch.cuda.synchronize()
-print("switch", int(out["reward"].shape[0]))
-# NEXT row f3: the same records under the DAPPLE schedule (flushed iteration, M = 8)
-eng.set_schedule(3, 0, 8)
+eng.set_schedule(L_.SCHED_DAPPLE, 0, 8)
 t3 = eng.eval_partitions(recs)
 torch.cuda.synchronize()
 eng.set_schedule()
-print("dapple", int(t3.shape[0]))
-# C2 VGG-16: the generic search kernel (replicas, heterogeneous links)
+tb = W.testbed_state(prof, seed=10)
+eng.load(prof, tb)
+r = eng.search_optimum(1, 10)
+print("testbed", r.time_ns, r.index)
 eng.load(W.vgg16(), W.vgg_state())
 r = eng.search_optimum(1, 8)
 print("vgg", r.time_ns, r.index)
+eng.load(prof, st)
+small = recs[: 1 << 16].contiguous()
+eng.set_schedule(L_.SCHED_PIPEDREAM_RR)
+eng.eval_partitions(small)
+eng.set_schedule(L_.SCHED_CHIMERA, 0, 8)
+eng.eval_partitions(small)
+torch.cuda.synchronize()
+eng.set_schedule()
+print("done")
