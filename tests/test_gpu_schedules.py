@@ -173,7 +173,7 @@ def test_errors_and_setting(eng):
     from paper_conf_icpp_hulww24_b200._lib import AUTOPIPE_E_INVAL, AUTOPIPE_E_OVERFLOW, AUTOPIPE_E_STATE
     prof, st = W.vgg16(), W.vgg_state()
     eng.load(prof, st)
-    for bad in [(4, 0, 1, False), (0, 2, 1, False), (0, 0, 2, False), (1, 0, 0, False),
+    for bad in [(6, 0, 1, False), (4, 0, 2, False), (0, 2, 1, False), (0, 0, 2, False), (1, 0, 0, False),
                 (1, 0, 65537, False), (SC.DAPPLE, 0, 4, True), (SC.TWO_BW, 0, 4, True)]:
         with pytest.raises(AutopipeError) as ex:
             eng.set_schedule(*bad)
