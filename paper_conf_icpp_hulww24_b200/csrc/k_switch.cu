@@ -57,25 +57,20 @@ __device__ __forceinline__ u64 startup_completion(const SmemTab &t, int S, u64 c
       Bd[w] = dv.ceil(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a]);
     }
   }
-  // transfers: forward boundary s = pairs [offF[s], offF[s+1]), backward boundary s likewise
-  u64 dF[MAXPAIRS], dB[MAXPAIRS], lfF[MAXPAIRS], lfB[MAXPAIRS];
-  int offF[MAXS], offB[MAXS];
-  int nf = 0, nb = 0;
+  // transfers: one FIFO server per boundary and direction with the boundary's longest transfer (the
+  // transfers of a boundary start together at its barrier on links no other boundary uses; see
+  // flush_makespan in sched.cuh)
+  u64 dF[MAXS], dB[MAXS], lfF[MAXS], lfB[MAXS];
 #pragma unroll
-  for (int s = 0; s < MAXS - 1; ++s) {
-    offF[s] = nf;
-    offB[s] = nb;
+  for (int s = 0; s < MAXS; ++s) {
+    dF[s] = dB[s] = lfF[s] = lfB[s] = 0;
     if (s < S - 1) {
       const int e = byte_at(cuts, s);
       const u32 ms = (u32)byte_at(masks, s), mn = (u32)byte_at(masks, s + 1);
-      nf = boundary_pairs(t.O[e], ms, mn, t.tau, t.dv, dF, nf);
-      nb = boundary_pairs(t.G[e + 1], mn, ms, t.tau, t.dv, dB, nb);
+      dF[s] = boundary_max<8>(t.O[e], ms, mn, t.tau, t.dv);
+      dB[s] = boundary_max<8>(t.G[e + 1], mn, ms, t.tau, t.dv);
     }
   }
-  offF[MAXS - 1] = nf;
-  offB[MAXS - 1] = nb;
-  for (int p = 0; p < nf; ++p) lfF[p] = 0;
-  for (int p = 0; p < nb; ++p) lfB[p] = 0;
 
   u64 fdl[MAXS];  // latest completion of forward boundary s
 #pragma unroll
@@ -93,7 +88,10 @@ __device__ __forceinline__ u64 startup_completion(const SmemTab &t, int S, u64 c
             wf[w] = umax(wf[w], ready) + Fd[w];
             bar = umax(bar, wf[w]);
           }
-        if (s < S - 1) fdl[s] = run_boundary(bar, dF, lfF, offF[s], offF[s + 1]);
+        if (s < S - 1) {
+          lfF[s] = umax(bar, lfF[s]) + dF[s];
+          fdl[s] = lfF[s];
+        }
       }
     }
   }
@@ -112,8 +110,13 @@ __device__ __forceinline__ u64 startup_completion(const SmemTab &t, int S, u64 c
             wf[w] = umax(wf[w], readyB) + Bd[w];
             bar = umax(bar, wf[w]);
           }
-        if (s > 0) bd = run_boundary(bar, dB, lfB, offB[s > 0 ? s - 1 : 0], offB[s]);
-        else C = bar;
+        if (s > 0) {
+          const int sb = s > 0 ? s - 1 : 0;
+          lfB[sb] = umax(bar, lfB[sb]) + dB[sb];
+          bd = lfB[sb];
+        } else {
+          C = bar;
+        }
         const u64 readyF = (s == 0) ? 0 : fdl[s > 0 ? s - 1 : 0];
         u64 barF = 0;
 #pragma unroll
@@ -122,7 +125,10 @@ __device__ __forceinline__ u64 startup_completion(const SmemTab &t, int S, u64 c
             wf[w] = umax(wf[w], readyF) + Fd[w];
             barF = umax(barF, wf[w]);
           }
-        if (s < S - 1) fdl[s] = run_boundary(barF, dF, lfF, offF[s], offF[s + 1]);
+        if (s < S - 1) {
+          lfF[s] = umax(barF, lfF[s]) + dF[s];
+          fdl[s] = lfF[s];
+        }
       }
     }
   }

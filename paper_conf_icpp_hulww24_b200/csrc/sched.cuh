@@ -22,56 +22,11 @@
 
 namespace ap {
 
-constexpr int MAXPAIRS = 2 * MAXN;  // sum over boundaries of (r_s + r_{s+1} - 1) <= 2 sum r - (S-1)
-
-// Durations of every transfer of one boundary, in merge order (see boundary_max in eval.cuh).
-template <int MAXD = 8>
-__device__ __forceinline__ int boundary_pairs(u64 A, u32 send, u32 recv, const u64 *tau, const DivEnt *dvt, u64 *d,
-                                              int n) {
-  const u32 rs = __popc(send), rr = __popc(recv);
-  if (rs == 1 && rr == 1) {
-    d[n] = xfer(A, tau[(__ffs(send) - 1) * TAUW + __ffs(recv) - 1]);
-    return n + 1;
-  }
-  const DivR<MAXD> ds(rs, dvt), dr(rr, dvt);
-  const u64 qs = ds.div(A), qr = dr.div(A);
-  const u32 rems = (u32)(A - qs * rs), remr = (u32)(A - qr * rr);
-  u32 i = 0, j = 0;
-  u64 lo_i = 0, lo_j = 0;
-  u64 hi_i = qs + ds.small(rems), hi_j = qr + dr.small(remr);
-  while (i < rs && j < rr) {
-    const u64 lo = umax(lo_i, lo_j), hi = umin(hi_i, hi_j);
-    if (hi > lo) d[n++] = xfer(hi - lo, tau[(__ffs(send) - 1) * TAUW + __ffs(recv) - 1]);
-    const bool adv_i = hi_i <= hi_j, adv_j = hi_j <= hi_i;
-    if (adv_i) {
-      ++i; send &= send - 1;
-      lo_i = hi_i; hi_i = (u64)(i + 1) * qs + ds.small((i + 1) * rems);
-    }
-    if (adv_j) {
-      ++j; recv &= recv - 1;
-      lo_j = hi_j; hi_j = (u64)(j + 1) * qr + dr.small((j + 1) * remr);
-    }
-  }
-  return n;
-}
-
-// Barrier at `bar`, then the FIFO transfers [lo, hi) of one boundary; returns its completion.
-__device__ __forceinline__ u64 run_boundary(u64 bar, const u64 *d, u64 *lf, int lo, int hi) {
-  u64 done = bar;
-  for (int p = lo; p < hi; ++p) {
-    const u64 e = umax(bar, lf[p]) + d[p];
-    lf[p] = e;
-    done = umax(done, e);
-  }
-  return done;
-}
-
-
 // T_ns of one flushed iteration (GPipe or DAPPLE) of a validated partition (P8 or the wide P16).
 template <int SCHED, typename P>
 __device__ __forceinline__ u64 flush_makespan(const SmemTab &t, int S, const P &p, const ModelP &m) {
   static_assert(SCHED == SCHED_GPIPE || SCHED == SCHED_DAPPLE, "flushed schedules only");
-  constexpr int MS = P::MS, MN = P::MN, NP = 2 * P::MN;
+  constexpr int MS = P::MS, MN = P::MN;
   const int M = (int)m.M;
   u64 Fd[MN], Bd[MN], wf[MN];
   int stg[MN];
@@ -94,24 +49,21 @@ __device__ __forceinline__ u64 flush_makespan(const SmemTab &t, int S, const P &
       if (SCHED == SCHED_GPIPE && m.recompute) Bd[w] += Fd[w];  // the backward op re-runs the forward
     }
   }
-  u64 dF[NP], dB[NP], lfF[NP], lfB[NP];
-  int offF[MS], offB[MS];
-  int nf = 0, nb = 0;
+  // One boundary's transfers all start at its barrier and use links no other boundary uses, so its
+  // completion over the micro-batches is that of a single FIFO server with the longest transfer:
+  // max_p lf_p(k) with lf_p(k) = max(bar_k, lf_p(k-1)) + d_p equals max_j (bar_j + (k-j+1) max_p d_p)
+  // (bar_k is non-decreasing in k). Per boundary and direction: its longest transfer and free time.
+  u64 dF[MS], dB[MS], lfF[MS], lfB[MS];
 #pragma unroll
-  for (int s = 0; s < MS - 1; ++s) {
-    offF[s] = nf;
-    offB[s] = nb;
+  for (int s = 0; s < MS; ++s) {
+    dF[s] = dB[s] = lfF[s] = lfB[s] = 0;
     if (s < S - 1) {
       const int e = p.cut(s);
       const u32 ms = p.mask(s), mn = p.mask(s + 1);
-      nf = boundary_pairs<MN>(t.O[e], ms, mn, t.tau, t.dv, dF, nf);
-      nb = boundary_pairs<MN>(t.G[e + 1], mn, ms, t.tau, t.dv, dB, nb);
+      dF[s] = boundary_max<MN>(t.O[e], ms, mn, t.tau, t.dv);
+      dB[s] = boundary_max<MN>(t.G[e + 1], mn, ms, t.tau, t.dv);
     }
   }
-  offF[MS - 1] = nf;
-  offB[MS - 1] = nb;
-  for (int q = 0; q < nf; ++q) lfF[q] = 0;
-  for (int q = 0; q < nb; ++q) lfB[q] = 0;
 
   u64 fdl[MS], last[MS];
 #pragma unroll
@@ -128,7 +80,10 @@ __device__ __forceinline__ u64 flush_makespan(const SmemTab &t, int S, const P &
       wf[w] = umax(wf[w], ready) + Fd[w];                                           \
       bar = umax(bar, wf[w]);                                                       \
     }                                                                               \
-    if ((s_) < S - 1) fdl[s_] = run_boundary(bar, dF, lfF, offF[s_], offF[(s_) + 1]); \
+    if ((s_) < S - 1) {                                                             \
+      lfF[s_] = umax(bar, lfF[s_]) + dF[s_];                                        \
+      fdl[s_] = lfF[s_];                                                            \
+    }                                                                               \
   }
   // B_s(k) on every replica of stage s (input: bd), then backward boundary s-1 (into bd)
 #define AP_BWD(s_, k_)                                                              \
@@ -139,7 +94,11 @@ __device__ __forceinline__ u64 flush_makespan(const SmemTab &t, int S, const P &
       wf[w] = umax(wf[w], ready) + Bd[w];                                           \
       bar = umax(bar, wf[w]);                                                       \
     }                                                                               \
-    if ((s_) > 0) bd = run_boundary(bar, dB, lfB, offB[(s_) > 0 ? (s_) - 1 : 0], offB[s_]); \
+    if ((s_) > 0) {                                                                 \
+      const int sb_ = (s_) > 0 ? (s_) - 1 : 0;                                      \
+      lfB[sb_] = umax(bar, lfB[sb_]) + dB[sb_];                                     \
+      bd = lfB[sb_];                                                                \
+    }                                                                               \
     if ((k_) == M - 1) last[s_] = bar;                                              \
   }
   if (SCHED == SCHED_GPIPE) {
