@@ -1102,7 +1102,7 @@ extern "C" int autopipe_switch_rewards(autopipe_ctx *c, const autopipe_partition
   for (int w = 0; w < MAXN; ++w) sow |= (u64)h_current->stage_of_worker[w] << (8 * w);
   c->launches += launch_switch(c->tab, d_parts, count, S, cuts, masks, sow, horizon, (u64 *)d_time_ns,
                                (u64 *)d_refill_ns, (u64 *)d_migrate_ns, (u64 *)d_reward_ns, c->path32, (int)c->model.sync,
-                               c->sms, st);
+                               c->sms, next_counter(c), st);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "switch kernel launch");
   return AUTOPIPE_OK;

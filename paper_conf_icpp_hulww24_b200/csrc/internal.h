@@ -83,6 +83,6 @@ int launch_neigh_best(const void *slots, const u64 *times, u64 nslots, ResultDev
 // NEXT row f2: switching cost as time (k_switch.cu).
 int launch_switch(const DevTables &g, const void *recs, u64 count, const int cur_S, const u64 cur_cuts,
                   const u64 cur_masks, const u64 cur_sow, u64 horizon, u64 *out_t, u64 *out_refill,
-                  u64 *out_mig, u64 *out_reward, int path32, int sync, int sms, cudaStream_t st);
+                  u64 *out_mig, u64 *out_reward, int path32, int sync, int sms, u32 *counter, cudaStream_t st);
 
 }  // namespace ap

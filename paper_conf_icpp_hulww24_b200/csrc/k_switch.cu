@@ -26,6 +26,7 @@
 #include "eval.cuh"
 #include "internal.h"
 #include "sched.cuh"
+#include "sortchunk.cuh"
 
 namespace ap {
 
@@ -161,11 +162,17 @@ __device__ __forceinline__ u64 migrate_time(const SmemTab &t, int S, u64 cuts, u
   return best;
 }
 
+#ifndef SWITCH_MINB
+#define SWITCH_MINB 2  // B200: 2 blocks per SM (128 registers) beat 1 (171): 1.09 -> 0.82 ms per 1M
+#endif
+#ifndef SWITCH_SORT
+#define SWITCH_SORT 0  // 1: warp-sorted dynamic chunks (sortchunk.cuh), as k_eval
+#endif
 template <bool P32>
-__global__ void __launch_bounds__(256) k_switch(DevTables g, const uint4 *__restrict__ recs, u64 count,
-                                                SwitchCur cur, u64 horizon, u32 sync, u64 *__restrict__ out_t,
-                                                u64 *__restrict__ out_refill, u64 *__restrict__ out_mig,
-                                                u64 *__restrict__ out_reward) {
+__global__ void __launch_bounds__(256, SWITCH_MINB) k_switch(DevTables g, const uint4 *__restrict__ recs, u64 count,
+                                                             SwitchCur cur, u64 horizon, u32 sync, u64 *__restrict__ out_t,
+                                                             u64 *__restrict__ out_refill, u64 *__restrict__ out_mig,
+                                                             u64 *__restrict__ out_reward, u32 *counter) {
   extern __shared__ u64 sm[];
   const SmemTab t = stage_tables(g, sm);
   __shared__ u64 tmin[MAXS * 8];
@@ -180,9 +187,7 @@ __global__ void __launch_bounds__(256) k_switch(DevTables g, const uint4 *__rest
   __syncthreads();
   const int L = t.L, N = (int)g.N;
   const bool overflow = (g.status[0] & 1ull) != 0;
-  const u64 stride = (u64)gridDim.x * blockDim.x;
-  for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < count; i += stride) {
-    const uint4 r = __ldg(recs + i);
+  auto one = [&](const uint4 &r, u64 i) {
     const u64 lo = (u64)r.x | ((u64)r.y << 32), hi = (u64)r.z | ((u64)r.w << 32);
     int S;
     P8 pp;
@@ -220,12 +225,18 @@ __global__ void __launch_bounds__(256) k_switch(DevTables g, const uint4 *__rest
     if (out_refill) out_refill[i] = R;
     if (out_mig) out_mig[i] = M;
     out_reward[i] = RW;
-  }
+  };
+#if SWITCH_SORT
+  for_each_sorted_warp<8>((const Rec16 *)recs, count, counter, [&](const Rec16 &r, u64 i) { one(r.a, i); });
+#else
+  const u64 stride = (u64)gridDim.x * blockDim.x;
+  for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < count; i += stride) one(__ldg(recs + i), i);
+#endif
 }
 
 int launch_switch(const DevTables &g, const void *recs, u64 count, const int cur_S, const u64 cur_cuts,
                   const u64 cur_masks, const u64 cur_sow, u64 horizon, u64 *out_t, u64 *out_refill,
-                  u64 *out_mig, u64 *out_reward, int path32, int sync, int sms, cudaStream_t st) {
+                  u64 *out_mig, u64 *out_reward, int path32, int sync, int sms, u32 *counter, cudaStream_t st) {
   if (count == 0) return 0;
   SwitchCur cur;
   cur.S = cur_S;
@@ -244,14 +255,26 @@ int launch_switch(const DevTables &g, const void *recs, u64 count, const int cur
     cur.wrange[w] = (s == 0xFF) ? 0xFFFFu : cur.range[s];
   }
   const size_t smem = (size_t)smem_words(g.L, g.N) * sizeof(u64);
-  const u64 need = (count + 255) / 256, cap = (u64)sms * 8;
+  const u64 need = (count + 255) / 256, cap = (u64)sms * (SWITCH_SORT ? SWITCH_MINB : 8);
   const int grid = (int)(need < cap ? need : cap);
+  if (SWITCH_SORT) {
+    static bool attr = false;
+    if (!attr) {
+      for (auto kern : {k_switch<true>, k_switch<false>}) {
+        cudaFuncAttributes fa;
+        cudaFuncGetAttributes(&fa, kern);
+        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024 - (int)fa.sharedSizeBytes);
+      }
+      attr = true;
+    }
+    cudaMemsetAsync(counter, 0, sizeof(u32), st);
+  }
   if (path32)
     k_switch<true><<<grid, 256, smem, st>>>(g, (const uint4 *)recs, count, cur, horizon, (u32)sync, out_t, out_refill, out_mig,
-                                            out_reward);
+                                            out_reward, counter);
   else
     k_switch<false><<<grid, 256, smem, st>>>(g, (const uint4 *)recs, count, cur, horizon, (u32)sync, out_t, out_refill, out_mig,
-                                             out_reward);
+                                             out_reward, counter);
   return 1;
 }
 
