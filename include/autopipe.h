@@ -277,8 +277,7 @@ int autopipe_decode_index_w(const autopipe_ctx *ctx, uint32_t s_min, uint32_t s_
  *                                   its own in flight (R_s = workers of stages s..S-1), one transfer per
  *                                   boundary and mini-batch, one sync per r_s mini-batches; M = 1;
  *                                   16-byte records only (N <= 8; wide calls E_INVAL), the state's bound
- *                                   < 2^45 (E_OVERFLOW); a record whose schedule is not periodic within
- *                                   2^18 rounds scores AUTOPIPE_T_UNRESOLVED;
+ *                                   < 2^45 (E_OVERFLOW);
  *                 AUTOPIPE_SCHED_CHIMERA    Chimera's bidirectional pipelines (row f3, reading F-6,
  *                                   PAPER.md:308-314, 1341-1350): one worker per stage; stage s on w_s
  *                                   (down) and on w_{S-1-s} (up); ceil(M/2) micro-batches down,
@@ -304,7 +303,6 @@ int autopipe_decode_index_w(const autopipe_ctx *ctx, uint32_t s_min, uint32_t s_
 #define AUTOPIPE_SCHED_DAPPLE 3u
 #define AUTOPIPE_SCHED_PIPEDREAM_RR 4u
 #define AUTOPIPE_SCHED_CHIMERA 5u
-#define AUTOPIPE_T_UNRESOLVED 0xFFFFFFFFFFFFFFFEull
 #define AUTOPIPE_SYNC_RING 0u
 #define AUTOPIPE_SYNC_PS 1u
 #define AUTOPIPE_RECOMPUTE 1u

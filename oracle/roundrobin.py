@@ -45,7 +45,8 @@ from .model import U64_MAX, Partition, allreduce_duration, ceil_div, parse_recor
 
 RING, PS = 0, 1
 MAX_ROUNDS = 200_000
-T_UNRESOLVED = U64_MAX - 1   # no periodic regime within MAX_ROUNDS rounds (the GPU caps at 2^18)
+TIME_NS_ROUNDS = 20_000   # time_ns waits this long for the periodic regime, then takes ceil(lambda) from
+                          # the event graph (Bellman-Ford on integer theta; reading R-2's fallback)
 
 
 class NoPeriod(RuntimeError):
@@ -260,15 +261,57 @@ def rr_lambda(prof, st, part: Partition, sync: int = RING, max_rounds: int = MAX
     return lam
 
 
+def ceil_lambda_compute(ing: RRIngredients) -> int:
+    """ceil(lambda_compute) without waiting for the periodic regime: the smallest integer theta such
+    that no cycle of the one-period event graph has sum(durations) - theta * Lam * sum(tokens) > 0
+    (Bellman-Ford positive-cycle test, binary search on theta). Two near-equal cycle ratios can make
+    the transient arbitrarily long (one C5 record needs more than 200,000 rounds); this is exact."""
+    if ing.S == 1:
+        lam = compute_lambda(ing)
+        return ceil_div(lam.numerator, lam.denominator)
+    g = event_graph(ing)
+    nodes = list(g.nodes)
+    pos = {v: i for i, v in enumerate(nodes)}
+    dur = [g.nodes[v]["dur"] for v in nodes]
+    edges = [(pos[u], pos[v], g.edges[u, v]["tokens"]) for u, v in g.edges]
+
+    def positive_cycle(theta: int) -> bool:
+        d = [0] * len(nodes)
+        for _ in range(len(nodes) + 1):
+            changed = False
+            for (u, v, tok) in edges:
+                nd = d[u] + dur[v] - theta * ing.Lam * tok
+                if nd > d[v]:
+                    d[v] = nd
+                    changed = True
+            if not changed:
+                return False
+        return True
+
+    lo, hi = -1, max(1, sum(dur))
+    while hi - lo > 1:
+        mid = (lo + hi) // 2
+        if positive_cycle(mid):
+            lo = mid
+        else:
+            hi = mid
+    return hi
+
+
 def time_ns(prof, st, part: Optional[Partition], sync: int = RING) -> int:
     """T_ns = ceil(lambda); UINT64_MAX for an invalid record."""
     if part is None:
         return U64_MAX
+    ing = RRIngredients(prof, st, part, sync)
     try:
-        lam = rr_lambda(prof, st, part, sync)
+        lam = compute_lambda(ing, TIME_NS_ROUNDS)
+        Tc = ceil_div(lam.numerator, lam.denominator)
     except NoPeriod:
-        return T_UNRESOLVED
-    return ceil_div(lam.numerator, lam.denominator)
+        Tc = ceil_lambda_compute(ing)
+    for s in range(part.S):
+        if ing.r[s] >= 2:
+            Tc = max(Tc, ceil_div(ing.sync[s], ing.r[s]))
+    return Tc
 
 
 def score_record(prof, st, rec: bytes, sync: int = RING) -> int:
@@ -320,7 +363,7 @@ def event_graph(ing: RRIngredients):
     return g
 
 
-def max_cycle_ratio(prof, st, part: Partition) -> Fraction:
+def max_cycle_ratio(prof, st, part: Partition) -> Fraction:  # noqa: D401 (tiny instances only)
     """lambda_compute as the maximum over elementary cycles of (sum of durations) / (sum of tokens),
     per mini-batch (one token = one period of Lam mini-batches)."""
     import networkx as nx

@@ -21,7 +21,6 @@ AUTOPIPE_E_NOMEM = -5
 USE_ALL_WORKERS = 1
 # row f3 (schedule variants, reading F-3)
 SCHED_PIPEDREAM, SCHED_2BW, SCHED_GPIPE, SCHED_DAPPLE, SCHED_PIPEDREAM_RR, SCHED_CHIMERA = 0, 1, 2, 3, 4, 5
-T_UNRESOLVED = (1 << 64) - 2  # round-robin schedule without a periodic regime within 2^18 rounds
 SYNC_RING, SYNC_PS = 0, 1
 RECOMPUTE = 1
 MAX_MICRO_BATCHES = 65536

@@ -22,8 +22,8 @@
 
 namespace ap {
 
-constexpr u64 RR_UNRESOLVED = U64MAX - 1;   // no periodic regime within RR_MAX_ROUNDS (both sides)
-constexpr u32 RR_MAX_ROUNDS = 1u << 18;
+constexpr u32 RR_SIM_ROUNDS = 4096;         // then ceil(lambda) from the event graph (rr_ceil_bf)
+constexpr int RR_BF_NODES = 160;            // 4 S Lam <= 144 nodes for sum r <= 8
 constexpr int RR_LINKS = 32;                // sum over boundaries of lcm(r_s, r_{s+1}) for N <= 8
 constexpr int RR_RING = 16;                 // pending forward transfers per boundary (D_0 <= 15)
 
@@ -34,6 +34,79 @@ __device__ __forceinline__ u32 gcd_u(u32 a, u32 b) {
     b = t;
   }
   return a;
+}
+
+// ceil(lambda_compute) from the timed event graph of one period (the oracle's event_graph): the
+// smallest integer theta with no positive cycle of node durations - theta * Lam * edge tokens
+// (Bellman-Ford from a virtual source, binary search on theta, bracketed around the simulation's
+// estimate th0). Nodes (kind, s, phase p): F_s, B_s, forward and backward transfers of boundary s, for
+// the mini-batches k = p (mod Lam). For the rare records whose simulation has not settled (two
+// near-equal cycle ratios can make the transient arbitrarily long); exact like the simulation.
+template <typename DurF>
+__device__ __forceinline__ u64 rr_ceil_bf(int S, u32 Lam, const int *r, const int *m, const int *lc, DurF dur,
+                                          long long th0) {
+  const int V = 4 * S * (int)Lam;
+  long long dist[RR_BF_NODES];
+  const long long K0 = 64ll * Lam;  // a period index far from the start: every predecessor is >= 0
+  auto node = [&](int kind, int s, long long k) { return (kind * S + s) * (int)Lam + (int)(k % Lam); };
+  auto tok = [&](long long kv, long long ku) { return kv / (long long)Lam - ku / (long long)Lam; };
+  auto positive = [&](long long th) -> bool {
+    for (int v = 0; v < V; ++v) dist[v] = 0;
+    for (int pass = 0; pass <= V; ++pass) {
+      bool changed = false;
+      for (int kind = 0; kind < 4; ++kind)
+        for (int s = 0; s < S; ++s) {
+          if (kind >= 2 && s == S - 1) continue;
+          for (u32 p = 0; p < Lam; ++p) {
+            const long long k = K0 + p;
+            const int v = node(kind, s, k);
+            const long long dv = (long long)dur(kind, s, (int)p);
+            long long best = dist[v];
+            auto relax = [&](int ku_kind, int ku_s, long long ku) {
+              const long long c = dist[node(ku_kind, ku_s, ku)] + dv - th * (long long)Lam * tok(k, ku);
+              if (c > best) best = c;
+            };
+            if (kind == 0) {
+              relax(1, s, k - (long long)m[s] * r[s]);         // worker order: after B(k - m r)
+              if (s > 0) relax(2, s - 1, k);                   // forward transfer of boundary s-1
+            } else if (kind == 1) {
+              relax(0, s, k + (long long)(m[s] - 1) * r[s]);   // worker order: after F(k + (m-1) r)
+              if (s < S - 1) relax(3, s, k);                   // backward transfer of boundary s
+            } else if (kind == 2) {
+              relax(0, s, k);                                  // after F_s(k)
+              relax(2, s, k - lc[s]);                          // FIFO on its link
+            } else {
+              relax(1, s + 1, k);                              // after B_{s+1}(k)
+              relax(3, s, k - lc[s]);
+            }
+            if (best > dist[v]) {
+              dist[v] = best;
+              changed = true;
+            }
+          }
+        }
+      if (!changed) return false;
+    }
+    return true;
+  };
+  // bracket [lo, hi]: positive(lo), !positive(hi), around the estimate
+  long long lo, hi, step = 1;
+  if (positive(th0)) {
+    lo = th0;
+    hi = th0 + step;
+    while (positive(hi)) lo = hi, step *= 2, hi = th0 + step;
+  } else {
+    hi = th0;
+    lo = th0 - step;
+    while (lo >= 0 && !positive(lo)) hi = lo, step *= 2, lo = th0 - step;
+    if (lo < 0) lo = -1;
+  }
+  while (hi - lo > 1) {
+    const long long mid = lo + (hi - lo) / 2;
+    if (positive(mid)) lo = mid;
+    else hi = mid;
+  }
+  return (u64)hi;
 }
 
 // T_ns of a validated 16-byte partition under round-robin replicas.
@@ -94,15 +167,22 @@ static __device__ __noinline__ u64 rr_time(const SmemTab &t, int S, const P8 &p,
   for (int w = 0; w < MAXN; ++w) wf[w] = 0;
   for (int q = 0; q < RR_LINKS; ++q) lff[q] = lfb[q] = 0;
   long long j = -(long long)D[0];  // the first round with an op: F_0(0)
+  // phases of the next op of every stage (mini-batch mod r_s, mod lcm of its boundary), advanced by
+  // one per round once the stage's mini-batch index is >= 0 (no 64-bit modulo in the recurrence)
+  int bph[MAXS], bl[MAXS], fph[MAXS], fl[MAXS];
+  for (int s = 0; s < S; ++s) bph[s] = bl[s] = fph[s] = fl[s] = 0;
+  auto step = [](int &ph, int m) { ph = (ph + 1 == m) ? 0 : ph + 1; };
   auto round = [&]() {
     u64 bd = 0;
     if (j >= 0) {
       for (int s = S - 1; s >= 0; --s) {  // B_s(j), backward boundary s-1 of mini-batch j
-        const int w = (wl[s] >> (4 * (int)(j % r[s]))) & 15;
+        const int w = (wl[s] >> (4 * bph[s])) & 15;
+        step(bph[s], r[s]);
         const u64 end = umax(wf[w], s == S - 1 ? 0ull : bd) + Bw[w];
         wf[w] = end;
         if (s > 0) {
-          const int q = lo[s - 1] + (int)(j % lc[s - 1]);
+          const int q = lo[s - 1] + bl[s];
+          step(bl[s], lc[s - 1]);
           const u64 fin = umax(end, lfb[q]) + tb[q];
           lfb[q] = fin;
           bd = fin;
@@ -112,11 +192,13 @@ static __device__ __noinline__ u64 rr_time(const SmemTab &t, int S, const P8 &p,
     for (int s = 0; s < S; ++s) {  // F_s(j + D_s), forward boundary s of that mini-batch
       const long long k = j + D[s];
       if (k < 0) continue;
-      const int w = (wl[s] >> (4 * (int)(k % r[s]))) & 15;
+      const int w = (wl[s] >> (4 * fph[s])) & 15;
+      step(fph[s], r[s]);
       const u64 end = umax(wf[w], s == 0 ? 0ull : fdr[s - 1][k & (RR_RING - 1)]) + Fw[w];
       wf[w] = end;
       if (s < S - 1) {
-        const int q = lo[s] + (int)(k % lc[s]);
+        const int q = lo[s] + fl[s];
+        step(fl[s], lc[s]);
         const u64 fin = umax(end, lff[q]) + tf[q];
         lff[q] = fin;
         fdr[s][k & (RR_RING - 1)] = fin;
@@ -188,6 +270,7 @@ static __device__ __noinline__ u64 rr_time(const SmemTab &t, int S, const P8 &p,
   save();
   block();
   u32 power = 1, lam = 1, rounds = 2 * Lam;
+  bool settled = true;
   while (!same()) {
     if (power == lam) {
       save();
@@ -197,11 +280,30 @@ static __device__ __noinline__ u64 rr_time(const SmemTab &t, int S, const P8 &p,
     block();
     ++lam;
     rounds += Lam;
-    if (rounds > RR_MAX_ROUNDS) return RR_UNRESOLVED;
+    if (rounds > RR_SIM_ROUNDS) {
+      settled = false;
+      break;
+    }
   }
   const u64 den = (u64)lam * Lam;
   u64 T = 0;
   for (u32 c = 0; c < g; ++c) T = umax(T, (off[c] + den - 1) / den);
+  if (!settled) {
+    int mm[MAXS];
+    {
+      int R = 0;
+      for (int s = S - 1; s >= 0; --s) R += r[s], mm[s] = (R + r[s] - 1) / r[s];
+    }
+    auto dur = [&](int kind, int s, int ph) -> u64 {
+      if (kind <= 1) {
+        const int w = (wl[s] >> (4 * (ph % r[s]))) & 15;
+        return kind == 0 ? Fw[w] : Bw[w];
+      }
+      const int q = lo[s] + ph % lc[s];
+      return kind == 2 ? tf[q] : tb[q];
+    };
+    T = rr_ceil_bf(S, Lam, r, mm, lc, dur, (long long)T);
+  }
   return umax(T, Tsync);
 }
 

@@ -140,3 +140,32 @@ def test_bounds_and_monotonicity(seed):
         # slower workers never speed the pipeline up
         st2 = W.State([[x * 2 for x in row] for row in st.f], st.b, st.tau)
         assert RR.rr_lambda(prof, st2, part) >= lam
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_bellman_ford_ceiling_equals_simulation(seed):
+    """The fallback for long transients (ceil_lambda_compute: Bellman-Ford on integer theta over the
+    one-period event graph) equals ceil of the simulated lambda wherever the simulation settles."""
+    rng = np.random.default_rng(980 + seed)
+    for _ in range(10):
+        L = int(rng.integers(2, 8))
+        N = int(rng.integers(2, 7))
+        S = int(rng.integers(1, min(4, N, L) + 1))
+        prof = W.random_profile(L, rng, f_max=500, bytes_max=10**4)
+        st = W.random_state_small(prof, N, rng, tau_max=2000)
+        part = _random_partition(rng, L, N, S)
+        ing = RR.RRIngredients(prof, st, part)
+        lam = RR.compute_lambda(ing)
+        assert RR.ceil_lambda_compute(ing) == ceil_div(lam.numerator, lam.denominator)
+
+
+def test_long_transient_uses_the_event_graph():
+    """A C5 record (ResNet-50, rollout state 0) with no periodic regime within 20,000 rounds: the
+    simulation gives up and ceil(lambda) comes from the event graph."""
+    prof = W.resnet50()
+    st = W.rollout_state(prof, 0)
+    part = Partition(3, [15, 29], [[4], [0, 3], [2]])
+    ing = RR.RRIngredients(prof, st, part)
+    with pytest.raises(RR.NoPeriod):
+        RR.compute_lambda(ing, RR.TIME_NS_ROUNDS)
+    assert RR.time_ns(prof, st, part) == RR.ceil_lambda_compute(ing) == 591221519

@@ -33,6 +33,10 @@ def main(what):
         cur = bytes(recs[0].cpu().numpy())
         if what.endswith("dapple"):
             eng.set_schedule(3, 0, 8)
+        elif what.endswith("_rr"):
+            eng.set_schedule(4)
+        elif what.endswith("chimera"):
+            eng.set_schedule(5, 0, 8)
         elif what.endswith("gpipe"):
             eng.set_schedule(2, 0, 8, True)
         if what == "c5_rollout":
