@@ -242,8 +242,11 @@ static __device__ __noinline__ u64 rr_time(const SmemTab &t, int S, const P8 &p,
   auto save = [&]() {
     for (int w = 0; w < MAXN; ++w) tw[w] = wf[w];
     for (int q = 0; q < RR_LINKS; ++q) tlf[q] = lff[q], tlb[q] = lfb[q];
-    for (int s = 0; s < S - 1; ++s)
-      for (int q = 0; q < RR_RING; ++q) tfd[s][q] = fdr[s][q];
+    for (int s = 0; s < S - 1; ++s)  // pending forward transfers in logical order (from j + D_{s+1})
+      for (int q = 0; q < D[s] - D[s + 1]; ++q) {
+        const long long k = j + D[s + 1] + q;
+        tfd[s][q] = k >= 0 ? fdr[s][k & (RR_RING - 1)] : U64MAX;
+      }
     for (u32 c = 0; c < g; ++c) off[c] = 0;
   };
   auto same = [&]() -> bool {
@@ -256,8 +259,10 @@ static __device__ __noinline__ u64 rr_time(const SmemTab &t, int S, const P8 &p,
       for (int k = 0; k < lc[s]; ++k)
         if (lff[lo[s] + k] != tlf[lo[s] + k] || lfb[lo[s] + k] != tlb[lo[s] + k]) return false;
     for (int s = 0; s < S - 1; ++s)
-      for (long long k = j + D[s + 1]; k < j + D[s]; ++k)
-        if (k >= 0 && fdr[s][k & (RR_RING - 1)] != tfd[s][k & (RR_RING - 1)]) return false;
+      for (int q = 0; q < D[s] - D[s + 1]; ++q) {
+        const long long k = j + D[s + 1] + q;
+        if ((k >= 0 ? fdr[s][k & (RR_RING - 1)] : U64MAX) != tfd[s][q]) return false;
+      }
     return true;
   };
   auto block = [&]() {
