@@ -676,7 +676,9 @@ static int search_impl(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, u64 beg
   u64 cur = begin;
   if (end - begin <= DENSE_SPAN && !(c->search_options & AUTOPIPE_SEARCH_SPLIT)) {
     int nb = 0;
-    c->launches += launch_search_generic(c->tab, sp, begin, end, path, c->model, wide, c->sms, c->d_blocks,
+    // a host-classified state may take the narrow (32-bit stage arithmetic) closed form (bit 1)
+    const int dpath = path >= 0 ? (path | (c->narrow << 1)) : path;
+    c->launches += launch_search_generic(c->tab, sp, begin, end, dpath, c->model, wide, c->sms, c->d_blocks,
                                          MAX_BLOCKS, &nb, next_sched(c), st, true);
     used = nb;
     cur = end;

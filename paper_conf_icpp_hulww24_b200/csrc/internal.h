@@ -32,6 +32,7 @@ int launch_eval(const DevTables &g, const void *recs, u64 count, bool wide, u64 
                 u32 *counter, cudaStream_t st);
 // Generic exhaustive search over [begin, end) (any S, any composition); writes one BlockOut per block
 // into out[out_offset ...] and returns the number of blocks used via *nblocks.
+// path32 of a dense launch: bit 0 = 32-bit segment sums, bit 1 = the narrow closed form (-1: gated)
 // sched: 32 bytes of device memory the PipeDream launch resets and schedules its chunks through (two
 // 16-byte slots: one per gated launch); each concurrent launch needs its own
 constexpr int SEARCH_SCHED_BYTES = 32;

@@ -86,9 +86,13 @@ __device__ __forceinline__ void unrank_global_smem(const SearchSpace &sp, u64 id
   cuts = lex_unrank_smem<BK, PK>(kappa, S - 1, sp.L - 1, Bn);
 }
 
-template <int NT, bool P32, int MODE, typename P>
-__global__ void __launch_bounds__(NT) k_search_generic(DevTables g, SearchSpace sp, u64 begin, u64 end,
-                                                       u64 per_thread, BlockOut *out, ModelP m, int gate) {
+#ifndef GEN_MINB
+#define GEN_MINB 3  // B200: 3 blocks per SM (C2 VGG-16 0.22 -> 0.18 ms) beat 1 and 2
+#endif
+// NARROW (PipeDream, dense launches of a host-classified state): the 32-bit closed form of k_eval
+template <int NT, bool P32, int MODE, typename P, bool NARROW = false>
+__global__ void __launch_bounds__(NT, GEN_MINB) k_search_generic(DevTables g, SearchSpace sp, u64 begin, u64 end,
+                                                                 u64 per_thread, BlockOut *out, ModelP m, int gate) {
   if (gate >= 0 && state_gated_out(g, gate, out)) return;  // see state_gated_out
   typedef SpaceT<P> SP;
   typedef typename SP::PK PK;
@@ -98,7 +102,7 @@ __global__ void __launch_bounds__(NT) k_search_generic(DevTables g, SearchSpace 
   u64 *Bn = sm + smem_words(g.L, g.N);
   const int nb = ((int)g.L + 1 > MAXNW + 1 ? (int)g.L + 1 : MAXNW + 1) * BK;
   for (int i = threadIdx.x; i < nb; i += NT) Bn[i] = g_binom[i / BK][i % BK];
-  const SmemTab t = stage_tables(g, sm);  // ends with __syncthreads()
+  const SmemTab t = stage_tables<NARROW>(g, sm);  // ends with __syncthreads()
   const u64 gtid = (u64)blockIdx.x * NT + threadIdx.x;
   u64 bestT = U64MAX, bestI = U64MAX, cnt = 0;
   const u64 span = end - begin;
@@ -110,7 +114,9 @@ __global__ void __launch_bounds__(NT) k_search_generic(DevTables g, SearchSpace 
     unrank_global_smem<BK>(sp, i0, S, Rp, cuts, Bn);
     P p = part_from<P>(sp, S, Rp, cuts);
     for (u64 i = i0; i < i1; ++i) {
-      const u64 T = model_time<MODE, P32>(t, S, p, m);
+      u64 T;
+      if constexpr (NARROW) T = eval_closed_form_n<P32, P>(t, S, p, (int)m.sync);
+      else T = model_time<MODE, P32>(t, S, p, m);
       if (T < bestT) {  // indices increase along the thread's range: strict < keeps the first
         bestT = T;
         bestI = i;
@@ -458,8 +464,9 @@ int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, 
     const int BK = wide ? BINOM_K : BK8;
     const size_t smem = ((size_t)smem_words(g.L, g.N) +
                          (size_t)(((int)g.L + 1 > MAXNW + 1 ? (int)g.L + 1 : MAXNW + 1) * BK)) * sizeof(u64);
-    if (wide) run_search_generic<NT, P16>((unsigned)blocks, smem, st, g, sp, begin, end, chunk, out, m, path32, sched);
-    else run_search_generic<NT, P8>((unsigned)blocks, smem, st, g, sp, begin, end, chunk, out, m, path32, sched);
+    const int p32 = path32 >= 0 ? (path32 & 1) : path32;
+    if (wide) run_search_generic<NT, P16>((unsigned)blocks, smem, st, g, sp, begin, end, chunk, out, m, p32, sched);
+    else run_search_generic<NT, P8>((unsigned)blocks, smem, st, g, sp, begin, end, chunk, out, m, p32, sched);
     *nblocks = (int)blocks * (both ? 2 : 1);
     return both ? 2 : 1;
   }
@@ -478,7 +485,9 @@ int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, 
     ModelP mm = m;
     const unsigned nbk = (unsigned)blocks;
 #define DENSE_LAUNCH(PT)                                                                                  \
-  if (m.sched != SCHED_PIPEDREAM) run_search_generic<NT, PT>(nbk, smem, st, g, sp, begin, end, per, out, mm, path32, sched); \
+  if (m.sched != SCHED_PIPEDREAM) run_search_generic<NT, PT>(nbk, smem, st, g, sp, begin, end, per, out, mm, path32 & 1, sched); \
+  else if (path32 == 3) k_search_generic<NT, true, SCHED_PIPEDREAM, PT, true><<<nbk, NT, smem, st>>>(g, sp, begin, end, per, out, mm, -1); \
+  else if (path32 == 2) k_search_generic<NT, false, SCHED_PIPEDREAM, PT, true><<<nbk, NT, smem, st>>>(g, sp, begin, end, per, out, mm, -1); \
   else if (path32 == 1) k_search_generic<NT, true, SCHED_PIPEDREAM, PT><<<nbk, NT, smem, st>>>(g, sp, begin, end, per, out, mm, -1); \
   else if (path32 == 0) k_search_generic<NT, false, SCHED_PIPEDREAM, PT><<<nbk, NT, smem, st>>>(g, sp, begin, end, per, out, mm, -1); \
   else {                                                                                                  \
