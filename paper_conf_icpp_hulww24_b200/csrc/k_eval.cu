@@ -6,7 +6,8 @@
 // own takes chunks of 256 records (128 wide ones) from a global counter, loads them with coalesced
 // 128-bit loads (ld.global.nc), counting-sorts them by shape in its slice of shared memory
 // (sortchunk.cuh) and scores them 32 at a time in shape order: the closed form of SPEC.md §4 in
-// registers, one 8-byte store per output at the record's position.
+// registers, the results written back into the records' shared-memory slots and stored in input
+// order (consecutive lanes, consecutive 8-byte outputs: coalesced).
 // Invalid records (SPEC.md §2) score UINT64_MAX and never fail the batch.
 #include <cstring>
 
@@ -45,20 +46,20 @@ __device__ __forceinline__ bool decode_any(const Rec32 &r, int L, int N, int &S,
 __device__ __forceinline__ const P8 &cur_part(const CurPart &c, const P8 *) { return c.p8; }
 __device__ __forceinline__ const P16 &cur_part(const CurPart &c, const P16 *) { return c.p16; }
 
+// Scores the record in `slot` and overwrites the slot with its results (bytes 0..7: T, 8..15: switch
+// bytes); the traversal then stores the chunk's results in input order, coalesced.
 template <bool ROLLOUT, bool P32, int MODE, bool NARROW, typename P, typename Rec>
-__device__ __forceinline__ void score_one(const SmemTab &t, int L, int N, bool overflow, const Rec &r, u64 i,
-                                          u64 *__restrict__ out_t, u64 *__restrict__ out_sw, const CurPart &cur,
-                                          const ModelP &m) {
+__device__ __forceinline__ void score_one(const SmemTab &t, int L, int N, bool overflow, Rec &slot,
+                                          const CurPart &cur, const ModelP &m) {
   int S;
   P p;
   u64 T = U64MAX, sw = U64MAX;
-  if (!overflow && decode_any(r, L, N, S, p)) {
+  if (!overflow && decode_any(slot, L, N, S, p)) {
     if constexpr (NARROW) T = eval_closed_form_n<P32, P>(t, S, p, (int)m.sync);
     else T = model_time<MODE, P32>(t, S, p, m);
     if (ROLLOUT) sw = switch_bytes(t, S, p, cur.S, cur_part(cur, (const P *)nullptr));
   }
-  out_t[i] = T;
-  if (ROLLOUT) out_sw[i] = sw;
+  slot.a = make_uint4((u32)T, (u32)(T >> 32), (u32)sw, (u32)(sw >> 32));
 }
 
 // MODE: the schedule of the model (row f3; SCHED_PIPEDREAM is the 1F1B closed form of rows a4-a7).
@@ -73,9 +74,13 @@ __global__ void __launch_bounds__(EVAL_NT, EVAL_BLOCKS(MODE, P))
   const int L = t.L, N = (int)g.N;
   // a state that failed the device-side overflow check (set_state_device) scores nothing
   const bool overflow = (g.status[0] & 1ull) != 0;
-  for_each_sorted_warp<EVAL_NT / 32>(recs, count, counter, [&](const Rec &r, u64 i) {
-    score_one<ROLLOUT, P32, MODE, NARROW, P>(t, L, N, overflow, r, i, out_t, out_sw, cur, m);
-  });
+  for_each_sorted_warp<EVAL_NT / 32>(
+      recs, count, counter,
+      [&](Rec &slot, u64) { score_one<ROLLOUT, P32, MODE, NARROW, P>(t, L, N, overflow, slot, cur, m); },
+      [&](const Rec &slot, u64 i) {
+        out_t[i] = (u64)slot.a.x | ((u64)slot.a.y << 32);
+        if (ROLLOUT) out_sw[i] = (u64)slot.a.z | ((u64)slot.a.w << 32);
+      });
 }
 
 template <bool ROLLOUT, bool P32, int MODE, typename Rec, typename P, bool NARROW = false>

@@ -7,6 +7,8 @@
 // of a step score records of (nearly) one shape. Every record is still scored exactly once, and its
 // outputs go to its own position (8-byte stores scattered within the chunk).
 #pragma once
+#include <type_traits>
+
 #include "common.cuh"
 
 namespace ap {
@@ -54,8 +56,16 @@ struct WarpSort {
   static constexpr int CH = 32 * PER;
 };
 
-template <int NW, typename Rec, typename F>
-__device__ __forceinline__ void for_each_sorted_warp(const Rec *__restrict__ recs, u64 count, u32 *counter, F &&f) {
+// f(Rec &slot, u64 i) scores the record in `slot` (global index i) and may overwrite the slot with its
+// results; store(const Rec &slot, u64 i), when given, then writes every slot of the chunk in input
+// order — consecutive lanes, consecutive records: coalesced stores (row a8).
+struct NoStore {
+  template <typename Rec>
+  __device__ void operator()(const Rec &, u64) const {}
+};
+template <int NW, typename Rec, typename F, typename G = NoStore>
+__device__ __forceinline__ void for_each_sorted_warp(const Rec *__restrict__ recs, u64 count, u32 *counter, F &&f,
+                                                     G store = G()) {
   constexpr int PER = WarpSort<NW, Rec>::PER, CH = WarpSort<NW, Rec>::CH;
   __shared__ Rec srec[NW][CH];
   __shared__ unsigned short sidx[NW][CH];
@@ -117,6 +127,14 @@ __device__ __forceinline__ void for_each_sorted_warp(const Rec *__restrict__ rec
       if (slot < nvalid) {
         const u32 src = si[slot];
         f(sr[src], base + src);
+      }
+    }
+    if constexpr (!std::is_same<G, NoStore>::value) {
+      __syncwarp();
+#pragma unroll
+      for (int j = 0; j < PER; ++j) {
+        const u32 q = (u32)(j * 32 + lane);
+        if (q < nvalid) store(sr[q], base + q);
       }
     }
     __syncwarp();  // the next chunk reuses this warp's slice
