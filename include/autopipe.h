@@ -348,6 +348,7 @@ int autopipe_set_timing(autopipe_ctx *ctx, int enable);
  * one dense launch, every candidate's exact T; larger ranges are split per S into the r = 1 sweep
  * and the threshold walk), AUTOPIPE_SEARCH_SPLIT = always the per-S split. E_INVAL on unknown bits. */
 #define AUTOPIPE_SEARCH_SPLIT 1u
+#define AUTOPIPE_SEARCH_NO_R1 2u  /* the r = 1 blocks through the threshold walk instead of the r = 1 sweep */
 int autopipe_set_search_options(autopipe_ctx *ctx, uint32_t options);
 
 /* Device milliseconds of the enumeration kernels of the last timed search (-1 if none); waits for

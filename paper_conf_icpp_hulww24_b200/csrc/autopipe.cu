@@ -691,7 +691,7 @@ static int search_impl(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, u64 beg
     // (R = 1..S) has every r_s = 1, which holds for the default flag and for USE_ALL when N = S.
     // The fast kernel decides the PipeDream closed form; other schedules (row f3) go to the generic one.
     const bool r1 = S >= 5 && S <= MAXS && (!(flags & AUTOPIPE_USE_ALL_WORKERS) || (int)c->N == S) &&
-                    c->model.sched == SCHED_PIPEDREAM;
+                    c->model.sched == SCHED_PIPEDREAM && !(c->search_options & AUTOPIPE_SEARCH_NO_R1);
     const u64 r1hi = blo + sp.ncut[S];
     if (r1 && lo < r1hi) {
       const u64 a = lo, b = hi < r1hi ? hi : r1hi;
@@ -966,7 +966,8 @@ extern "C" uint64_t autopipe_kernel_launches(const autopipe_ctx *c) { return c ?
 extern "C" int autopipe_set_search_options(autopipe_ctx *c, uint32_t options) {
   if (!c) return AUTOPIPE_E_INVAL;
   c->err[0] = 0;
-  if (options & ~AUTOPIPE_SEARCH_SPLIT) return fail(c, AUTOPIPE_E_INVAL, "unknown search options 0x%x", options);
+  if (options & ~(AUTOPIPE_SEARCH_SPLIT | AUTOPIPE_SEARCH_NO_R1))
+    return fail(c, AUTOPIPE_E_INVAL, "unknown search options 0x%x", options);
   c->search_options = options;
   return AUTOPIPE_OK;
 }

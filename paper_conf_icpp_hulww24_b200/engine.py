@@ -329,10 +329,11 @@ class Engine:
     def int_path(self) -> int:
         return int(lib.autopipe_int_path(self._h))
 
-    def set_search_options(self, split: bool = False) -> None:
+    def set_search_options(self, split: bool = False, no_r1: bool = False) -> None:
         """Kernel selection of later searches (autopipe_set_search_options): split=True always uses the
-        per-S split (r = 1 sweep + threshold walk), even for ranges the dense launch would take."""
-        self._check(lib.autopipe_set_search_options(self._h, 1 if split else 0))
+        per-S split (r = 1 sweep + threshold walk), even for ranges the dense launch would take;
+        no_r1=True sends the r = 1 blocks through the threshold walk too."""
+        self._check(lib.autopipe_set_search_options(self._h, (1 if split else 0) | (2 if no_r1 else 0)))
 
     def set_timing(self, enable: bool = True) -> None:
         self._check(lib.autopipe_set_timing(self._h, 1 if enable else 0))

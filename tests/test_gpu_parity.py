@@ -466,3 +466,18 @@ def as_u64_list(t):
     from paper_conf_icpp_hulww24_b200 import as_u64
     torch.cuda.synchronize()
     return as_u64(t)
+
+
+@pytest.mark.parametrize("kind", ["a-nvlink", "b"])
+def test_gpt96_threshold_walk_full_space(eng, kind):
+    """The threshold walk (k_search_dfs) over the whole 96-layer, 8-stage space in place of the r = 1
+    sweep (AUTOPIPE_SEARCH_NO_R1): the same optimum as the parametric DP, every candidate counted."""
+    prof, st = W.gpt96(), W.gpt_state(kind)
+    eng.load(prof, st)
+    eng.set_search_options(False, True)
+    try:
+        r = eng.search_optimum(8, 8)
+    finally:
+        eng.set_search_options(False)
+    T, idx, _ = optimum(prof, st, 8, 8)
+    assert (r.time_ns, r.index, r.evaluated) == (T, idx, comb(95, 7))
