@@ -345,8 +345,9 @@ int autopipe_set_timing(autopipe_ctx *ctx, int enable);
 
 /* Kernel selection of later searches (the result never depends on it; tests use it to exercise each
  * kernel on small spaces). options: 0 = default (a range of at most 2^21 candidates is searched by
- * one dense launch, every candidate's exact T; larger ranges are split per S into the r = 1 sweep
- * and the threshold walk), AUTOPIPE_SEARCH_SPLIT = always the per-S split. E_INVAL on unknown bits. */
+ * one dense launch, every candidate's exact T; a PipeDream range of at most 2^28 by one threshold
+ * walk; larger ranges are split per S into the r = 1 sweep and the threshold walk),
+ * AUTOPIPE_SEARCH_SPLIT = always the per-S split. E_INVAL on unknown bits. */
 #define AUTOPIPE_SEARCH_SPLIT 1u
 #define AUTOPIPE_SEARCH_NO_R1 2u  /* the r = 1 blocks through the threshold walk instead of the r = 1 sweep */
 int autopipe_set_search_options(autopipe_ctx *ctx, uint32_t options);

@@ -670,9 +670,10 @@ static int search_impl(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, u64 beg
     }
     forked = false;
   };
-  // A small range: one dense launch on the caller's stream. Otherwise split [begin, end) into the
-  // r = 1 block of each S (rho = 0: fast kernel) and the rest (generic); the pieces write disjoint
-  // block-result ranges and run concurrently.
+  // A small range: one dense launch on the caller's stream; a medium PipeDream one: one threshold
+  // walk. Otherwise split [begin, end) into the r = 1 block of each S (rho = 0: fast kernel) and the
+  // rest (threshold walk or generic); the pieces write disjoint block-result ranges and run
+  // concurrently.
   u64 cur = begin;
   if (end - begin <= DENSE_SPAN && !(c->search_options & AUTOPIPE_SEARCH_SPLIT)) {
     int nb = 0;
@@ -680,6 +681,20 @@ static int search_impl(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, u64 beg
     const int dpath = path >= 0 ? (path | (c->narrow << 1)) : path;
     c->launches += launch_search_generic(c->tab, sp, begin, end, dpath, c->model, wide, c->sms, c->d_blocks,
                                          MAX_BLOCKS, &nb, next_sched(c), st, true);
+    used = nb;
+    cur = end;
+  }
+#ifndef WALK_SPAN
+#define WALK_SPAN (1ull << 28)
+#endif
+  // a medium PipeDream range (<= 2^28): one threshold-walk launch over all its S, no per-S pieces
+  // (B200: BERT-24 state 0.66 -> 0.43 ms, the VGG-16 testbed 1.2 -> 0.36 ms; the 1.3e10-candidate
+  // ResNet-50 testbed keeps the per-S split with r = 1 sweeps: 10 ms against 29 ms as one walk)
+  if (cur < end && end - begin <= WALK_SPAN && c->model.sched == SCHED_PIPEDREAM &&
+      !(c->search_options & AUTOPIPE_SEARCH_SPLIT)) {
+    int nb = 0;
+    c->launches += launch_search_generic(c->tab, sp, begin, end, path, c->model, wide, c->sms, c->d_blocks,
+                                         MAX_BLOCKS, &nb, next_sched(c), st, false);
     used = nb;
     cur = end;
   }
