@@ -284,8 +284,8 @@ int autopipe_decode_index_w(const autopipe_ctx *ctx, uint32_t s_min, uint32_t s_
  *                                   floor(M/2) up, each pipeline in DAPPLE order, a worker's two lists
  *                                   interleaved by readiness (earliest start; ties: lower down stage,
  *                                   then down), the two copies of a stage synchronised after their last
- *                                   backwards; one flushed iteration; 16-byte records only; a record
- *                                   with a replicated stage scores UINT64_MAX;
+ *                                   backwards; one flushed iteration; 16-byte and wide records; a
+ *                                   record with a replicated stage scores UINT64_MAX;
  *   sync          AUTOPIPE_SYNC_RING (default) or AUTOPIPE_SYNC_PS (a parameter server sharded over
  *                 the stage's replicas, each server taking its pushes and pulls one at a time);
  *   micro_batches M >= 1 micro-batches per iteration (must be 1 for PIPEDREAM; <= 65536);

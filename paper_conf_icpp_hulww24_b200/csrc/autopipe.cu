@@ -407,10 +407,8 @@ static int sync_status(autopipe_ctx *c, cudaStream_t st) {
 // that could reach 2^63. Reads the device status first for a state set from device memory.
 static int check_model(autopipe_ctx *c, cudaStream_t st, bool wide = false) {
   if (c->model.sched == SCHED_PIPEDREAM) return AUTOPIPE_OK;
-  if ((c->model.sched == SCHED_RR || c->model.sched == SCHED_CHIMERA) && wide)
-    return fail(c, AUTOPIPE_E_INVAL, "round-robin replicas and Chimera use 16-byte records (no wide calls)");
-  if (c->model.sched == SCHED_CHIMERA && c->N > (u32)MAXN)
-    return fail(c, AUTOPIPE_E_INVAL, "Chimera uses 16-byte records: N <= 8");
+  if (c->model.sched == SCHED_RR && wide)
+    return fail(c, AUTOPIPE_E_INVAL, "round-robin replicas use 16-byte records (no wide calls)");
   int rc = sync_status(c, st);
   if (rc) return rc;
   if (c->model.sched == SCHED_RR) {

@@ -20,7 +20,12 @@
 
 namespace ap {
 
-constexpr int CH_RING = 8;
+// ring of transfer completions per pipeline and boundary: a stage runs ahead of its successor by at
+// most its warm-up (<= S), so 8 slots serve 16-byte records and 16 the wide ones
+template <typename P>
+struct ChRing {
+  static constexpr int N = P::MS;
+};
 
 // op at position i of DAPPLE's list for stage s of an S-stage pipeline with M micro-batches:
 // kind (0 = F, 1 = B) and micro-batch
@@ -41,9 +46,12 @@ __device__ __forceinline__ void dapple_op(int S, int s, u32 M, u32 i, int &kind,
   }
 }
 
-// T_ns of a validated 16-byte partition under Chimera; UINT64_MAX if a stage is replicated.
-static __device__ __noinline__ u64 chimera_time(const SmemTab &t, int S, const P8 &p, const ModelP &m) {
-  int wk[MAXS];
+// T_ns of a validated partition (16-byte P8 or wide P16) under Chimera; UINT64_MAX if a stage is
+// replicated.
+template <typename P>
+static __device__ __noinline__ u64 chimera_time(const SmemTab &t, int S, const P &p, const ModelP &m) {
+  constexpr int MS = P::MS, CH_RING = ChRing<P>::N;
+  int wk[MS];
   for (int s = 0; s < S; ++s) {
     const u32 mask = p.mask(s);
     if (__popc(mask) != 1) return U64MAX;
@@ -51,7 +59,7 @@ static __device__ __noinline__ u64 chimera_time(const SmemTab &t, int S, const P
   }
   const u32 Mp[2] = {(m.M + 1) / 2, m.M / 2};
   // durations: group g (worker wk[g]) runs down stage g and up stage S-1-g
-  u64 dur[MAXS][2][2];  // [g][pipe][kind]
+  u64 dur[MS][2][2];  // [g][pipe][kind]
   for (int g = 0; g < S; ++g) {
     const int w = wk[g];
     for (int pipe = 0; pipe < 2; ++pipe) {
@@ -63,7 +71,7 @@ static __device__ __noinline__ u64 chimera_time(const SmemTab &t, int S, const P
     }
   }
   // neighbour links: right[g] = w_g -> w_{g+1} (down forward g, up backward), left[g] = w_{g+1} -> w_g
-  u64 lright[MAXS], lleft[MAXS], xr_dn[MAXS], xl_dn[MAXS], xl_up[MAXS], xr_up[MAXS];
+  u64 lright[MS], lleft[MS], xr_dn[MS], xl_dn[MS], xl_up[MS], xr_up[MS];
   for (int g = 0; g + 1 < S; ++g) {
     lright[g] = lleft[g] = 0;
     const u64 tr = t.tau[wk[g] * TAUW + wk[g + 1]], tl = t.tau[wk[g + 1] * TAUW + wk[g]];
@@ -75,10 +83,10 @@ static __device__ __noinline__ u64 chimera_time(const SmemTab &t, int S, const P
     xr_up[g] = xfer(t.G[eu + 1], tr);  // up backward u: w_g -> w_{g+1}
   }
   // boundary rings: [pipe][boundary][slot], forward and backward, with produced counts
-  u64 fr[2][MAXS - 1][CH_RING], br[2][MAXS - 1][CH_RING];
-  u32 fcnt[2][MAXS - 1], bcnt[2][MAXS - 1];
-  u64 fre[MAXS], lastb[MAXS][2];
-  u32 pos[MAXS][2];
+  u64 fr[2][MS - 1][CH_RING], br[2][MS - 1][CH_RING];
+  u32 fcnt[2][MS - 1], bcnt[2][MS - 1];
+  u64 fre[MS], lastb[MS][2];
+  u32 pos[MS][2];
   for (int g = 0; g < S; ++g) {
     fre[g] = 0;
     pos[g][0] = pos[g][1] = 0;
@@ -157,7 +165,7 @@ static __device__ __noinline__ u64 chimera_time(const SmemTab &t, int S, const P
     if (wk[s] != wk[S - 1 - s]) {
       const int a = (s == 0) ? 0 : p.cut(s - 1) + 1;
       const int e = (s == S - 1) ? t.L - 1 : p.cut(s);
-      fin += sync_time<8>((int)m.sync, t.PP[e + 1] - t.PP[a], (1u << wk[s]) | (1u << wk[S - 1 - s]), t.tau, t.dv);
+      fin += sync_time<P::MN>((int)m.sync, t.PP[e + 1] - t.PP[a], (1u << wk[s]) | (1u << wk[S - 1 - s]), t.tau, t.dv);
     }
     T = umax(T, fin);
   }

@@ -158,10 +158,7 @@ __device__ __forceinline__ u64 model_time(const SmemTab &t, int S, const P &p, c
     if constexpr (P::MS == 8) return rr_time(t, S, p, (int)m.sync);
     else return U64MAX;
   }
-  if constexpr (MODE == SCHED_CHIMERA) {  // row f3, reading F-6; 16-byte records (host-checked)
-    if constexpr (P::MS == 8) return chimera_time(t, S, p, m);
-    else return U64MAX;
-  }
+  if constexpr (MODE == SCHED_CHIMERA) return chimera_time<P>(t, S, p, m);  // row f3, reading F-6
   if (MODE == SCHED_PIPEDREAM) return eval_closed_form<P32, false, P>(t, S, p, (int)m.sync);
   if (MODE == SCHED_2BW) return eval_closed_form<false, true, P>(t, S, p, (int)m.sync, m.M);
   return flush_makespan<(MODE == SCHED_PIPEDREAM || MODE == SCHED_2BW || MODE == SCHED_RR || MODE == SCHED_CHIMERA)

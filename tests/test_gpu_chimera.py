@@ -102,14 +102,24 @@ def test_small_space_search(eng, seed):
     eng.set_schedule()
 
 
-def test_refused_calls(eng):
-    from paper_conf_icpp_hulww24_b200 import AutopipeError
-    from paper_conf_icpp_hulww24_b200._lib import AUTOPIPE_E_INVAL
-    prof = W.resnet50()
-    eng.load(prof, W.testbed_state(prof, seed=10))
-    eng.set_schedule(SCHED_CHIMERA, 0, 4)
-    recs = W.sample_records(prof.L, 10, 8, 3, s_max=10, wide=True)
-    with pytest.raises(AutopipeError) as ex:
-        eng.eval_partitions(torch.from_numpy(recs))
-    assert ex.value.code == AUTOPIPE_E_INVAL
+@pytest.mark.parametrize("name", ["bert24", "resnet50"])
+def test_wide_testbed(eng, name):
+    """The paper runs its Chimera comparison on the 10-GPU testbed:
+    32-byte records with up to 10 stages on 10 heterogeneous workers, M = 8."""
+    from paper_conf_icpp_hulww24_b200 import as_u64
+    prof = W.profile(name)
+    st = W.testbed_state(prof, seed=10)
+    eng.load(prof, st)
+    rng = np.random.default_rng(1900)
+    recs = []
+    for _ in range(300):
+        S = int(rng.integers(1, 11))
+        cuts = sorted(int(x) for x in rng.choice(prof.L - 1, S - 1, replace=False)) if S > 1 else []
+        ws = [int(x) for x in rng.permutation(10)[:S]]
+        recs.append(encode_partition(Partition(S, cuts, [[w] for w in ws]), wide=True))
+    recs += [bytes(r) for r in W.sample_records(prof.L, 10, 30, 5, s_max=10, wide=True)]
+    arr = np.frombuffer(b"".join(recs), dtype=np.uint8).reshape(len(recs), 32).copy()
+    eng.set_schedule(SCHED_CHIMERA, 1, 8)
+    got = [int(x) for x in as_u64(eng.eval_partitions(torch.from_numpy(arr)))]
     eng.set_schedule()
+    assert got == chimera_many(prof, st, recs, 8, 1)
