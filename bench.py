@@ -484,6 +484,20 @@ def main():
                               "achieved_GBps": gbs, "hbm_peak_GBps": hbm,
                               "hbm_frac": gbs / hbm if hbm else None, "peak_source": peak_src,
                               "decision_only": False}
+        # the same roofline on the records the 230-op unit describes (S = 8, r = 1, GPT-96, u32 path)
+        c4 = configs.get("C4_gpt96_r1_records")
+        if c4:
+            rps = c4["eval_records_per_s"]
+            ops = rps * ROLLOUT_OPS / 1e12
+            gbs = rps * ROLLOUT_BYTES / 1e9
+            hbm = float(peaks.get("hbm_gbs", 0)) or None
+            c4["roofline"] = {"bound": "alu", "kernel": "k_eval<PipeDream,u32>", "achieved": ops, "unit": "Tops/s",
+                              "peak": peak_t, "frac": ops / peak_t if peak_t else None,
+                              "ops_per_record": ROLLOUT_OPS, "bytes_per_record": ROLLOUT_BYTES,
+                              "achieved_GBps": gbs, "hbm_peak_GBps": hbm,
+                              "hbm_frac": gbs / hbm if hbm else None, "peak_source": peak_src,
+                              "decision_only": False,
+                              "note": "every record is an S = 8, r = 1 partition: the unit's own case"}
 
     cpu = None
     if world == 1 and not args.no_cpu_baseline:

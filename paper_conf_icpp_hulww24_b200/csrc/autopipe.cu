@@ -166,7 +166,7 @@ extern "C" int autopipe_create(int cuda_device, autopipe_ctx **out) {
   upload_binomials(c->binom);
   // device tables, sized for the limits (L = 255, N = 8): a few hundred KB
   const size_t Lp1 = MAXL + 1, NL = (size_t)MAXNW * Lp1, TT = (size_t)TAUW * TAUW;
-  const size_t words = 3 * NL + Lp1 + 2 * MAXL + TT + 2 * 7 * MAXL + 2 + 256;
+  const size_t words = 3 * NL + Lp1 + 2 * MAXL + TT + 2 * 7 * MAXL + 2 + 256 + (size_t)MAXL * TT * 2;
   const size_t words32 = 3 * NL + 2 * 7 * MAXL;
   e = cudaMalloc(&c->d_tables, words * 8 + words32 * 4 + 64);
   if (e == cudaSuccess) e = cudaMalloc(&c->d_raw, (2 * MAXNW * MAXL + MAXL + TT) * 8);
@@ -201,6 +201,7 @@ extern "C" int autopipe_create(int cuda_device, autopipe_ctx **out) {
   c->tab.LM = p; p += 7 * MAXL;
   c->tab.status = p; p += 2;
   c->tab.ring = p; p += 256;
+  c->tab.xp = p; p += (size_t)MAXL * TT * 2;
   u32 *q = (u32 *)p;
   c->tab.PC32 = q; q += NL;
   c->tab.PF32 = q; q += NL;

@@ -38,6 +38,8 @@ struct DevTables {
   u64 *LM;    // [7][L]    ... max(cf, cb)                                                (row a2)
   u32 *PC32;  // [N][L+1]  32-bit copies for the 32-bit search path (valid iff path32)
   u64 *ring;  // [256]     slowest link of the ring over each worker set (N <= 8; ascending ring order)
+  u64 *xp;    // [L-1][16][16][2] single-worker boundary at cut l, sender u, receiver v:
+              //   {xfer(O[l], tau[u][v]), xfer(G[l+1], tau[v][u])} (forward, backward)
   u32 *PF32;  // [N][L+1]  32-bit copies of PF, PB for the narrow eval path (valid iff status bit 2)
   u32 *PB32;
   u32 *Z32;   // [7][L]

@@ -42,6 +42,7 @@ struct SmemTab {
   const u64 *ring;  // [256] slowest ring link of each worker set of N <= 8 (ascending ring order)
   const u32 *PF32, *PB32, *tau32;
   const DivEnt *dv;  // replica-count divisors d = 1..16 (DivR / Div32 multipliers)
+  const u64 *xp;     // global: the single-worker boundary table (DevTables::xp)
   int L, Lp1;
 };
 
@@ -103,6 +104,7 @@ __device__ __forceinline__ SmemTab stage_tables(const DevTables &g, u64 *sm) {
   for (u32 i = threadIdx.x; i < 256u; i += blockDim.x) ring[i] = g.ring[i];
   __syncthreads();
   t.PP = PP; t.O = O; t.G = G; t.tau = tau; t.tau32 = tau32; t.ring = ring;
+  t.xp = g.xp;
   t.dv = dt;
   t.L = (int)L; t.Lp1 = (int)Lp1;
   return t;
@@ -145,6 +147,22 @@ __device__ __forceinline__ u64 boundary_max(u64 A, u32 send, u32 recv, const u64
     }
   }
   return xfer_fs(best);
+}
+
+// Both transfers of the boundary after layer eb between the replica sets ms (sending forward) and mr:
+// a single-worker boundary reads the per-state table (one 16-byte load), a replicated one walks its
+// shards (boundary_max).
+template <int MAXD = 8>
+__device__ __forceinline__ void boundary_cf_cb(const SmemTab &t, int eb, u32 ms, u32 mr, u64 &cf, u64 &cb) {
+  if (__popc(ms) == 1 && __popc(mr) == 1) {
+    const int u = __ffs(ms) - 1, v = __ffs(mr) - 1;
+    const ulonglong2 x = __ldg((const ulonglong2 *)t.xp + (eb * TAUW + u) * TAUW + v);
+    cf = x.x;
+    cb = x.y;
+  } else {
+    cf = boundary_max<MAXD>(t.O[eb], ms, mr, t.tau, t.dv);
+    cb = boundary_max<MAXD>(t.G[eb + 1], mr, ms, t.tau, t.dv);
+  }
 }
 
 // Ring all-reduce of a replicated stage (row a6): 2(r-1) steps of a ceil(P_s/r)-byte chunk over the
@@ -234,22 +252,29 @@ __device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, const P
       const int e = (u == S - 1) ? t.L - 1 : p.cut(u);
       const u32 mask = p.mask(u);
       const u32 r = __popc(mask);
-      const DivR<P::MN> dv(r, t.dv);
-      u32 m = mask;
-      // first replica unconditionally; the loop only runs for replicated stages
-      int w = __ffs(m) - 1;
-      m &= m - 1;
-      u64 F = dv.ceil(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a]);
-      u64 B = dv.ceil(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a]);
-      u64 fm = F, bm = B, xm = F + B;
-      while (m) {  // row a4: split replicas, ceil(sum / r) per op
-        w = __ffs(m) - 1;
+      u64 fm, bm, xm;
+      if (r == 1) {  // one worker: no division
+        const int w = __ffs(mask) - 1;
+        fm = t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a];
+        bm = t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a];
+        xm = fm + bm;
+      } else {
+        const DivR<P::MN> dv(r, t.dv);
+        u32 m = mask;
+        int w = __ffs(m) - 1;
         m &= m - 1;
-        F = dv.ceil(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a]);
-        B = dv.ceil(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a]);
-        fm = umax(fm, F);
-        bm = umax(bm, B);
-        xm = umax(xm, F + B);
+        u64 F = dv.ceil(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a]);
+        u64 B = dv.ceil(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a]);
+        fm = F, bm = B, xm = F + B;
+        while (m) {  // row a4: split replicas, ceil(sum / r) per op
+          w = __ffs(m) - 1;
+          m &= m - 1;
+          F = dv.ceil(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a]);
+          B = dv.ceil(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a]);
+          fm = umax(fm, F);
+          bm = umax(bm, B);
+          xm = umax(xm, F + B);
+        }
       }
       const V X = (V)xm, Y = (V)(fm + bm);
       const V xs = BW ? (V)(xm * M) : (V)xm;
@@ -259,8 +284,8 @@ __device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, const P
         // row a5: boundary u-1 (activation O[e_{u-1}] forward, gradient G[e_{u-1}+1] backward)
         const int eb = p.cut(u - 1);
         const u32 mp = p.mask(u - 1);
-        const u64 cf = boundary_max<P::MN>(t.O[eb], mp, mask, t.tau, t.dv);
-        const u64 cb = boundary_max<P::MN>(t.G[eb + 1], mask, mp, t.tau, t.dv);
+        u64 cf, cb;
+        boundary_cf_cb<P::MN>(t, eb, mp, mask, cf, cb);
         const V Z = (V)(cf + cb);
         const V lm = BW ? (V)(umax(cf, cb) * M) : (V)umax(cf, cb);
         T = T > lm ? T : lm;
@@ -320,12 +345,15 @@ __device__ __forceinline__ void walk_n(u32 A, u32 send, u32 recv, const u32 *tau
 }
 
 template <int MAXD>
-__device__ __forceinline__ void boundary_both_n(u64 Af, u64 Ab, u32 ms, u32 mr, const u32 *tau32, const DivEnt *dvt,
-                                                u64 &cf, u64 &cb) {
-  if (__popc(ms) == 1 && __popc(mr) == 1) {
+__device__ __forceinline__ void boundary_both_n(const SmemTab &t, int eb, u32 ms, u32 mr, u64 &cf, u64 &cb) {
+  const u64 Af = t.O[eb], Ab = t.G[eb + 1];
+  const u32 *tau32 = t.tau32;
+  const DivEnt *dvt = t.dv;
+  if (__popc(ms) == 1 && __popc(mr) == 1) {  // single-worker boundary: the per-state table
     const int u = __ffs(ms) - 1, v = __ffs(mr) - 1;
-    cf = xfer_fs((u64)(u32)Af * tau32[u * TAUW + v]);
-    cb = xfer_fs((u64)(u32)Ab * tau32[v * TAUW + u]);
+    const ulonglong2 x = __ldg((const ulonglong2 *)t.xp + (eb * TAUW + u) * TAUW + v);
+    cf = x.x;
+    cb = x.y;
     return;
   }
   u64 bf = 0, bb = 0;
@@ -383,7 +411,7 @@ __device__ __forceinline__ u64 eval_closed_form_n(const SmemTab &t, int S, const
       if (u > 0) {
         const int eb = p.cut(u - 1);
         u64 cf, cb;
-        boundary_both_n<P::MN>(t.O[eb], t.G[eb + 1], p.mask(u - 1), mask, t.tau32, t.dv, cf, cb);
+        boundary_both_n<P::MN>(t, eb, p.mask(u - 1), mask, cf, cb);
         const V Z = (V)(cf + cb);
         const V lm = (V)umax(cf, cb);
         T = T > lm ? T : lm;

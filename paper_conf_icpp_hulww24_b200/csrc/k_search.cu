@@ -199,6 +199,15 @@ template <int MN>
 __device__ __forceinline__ void stage_cost(const SmemTab &t, int a, int e, u32 mask, int sync, u64 &X, u64 &Y,
                                            u64 &AR) {
   const u32 r = __popc(mask);
+  if (r == 1) {  // one worker: no division, no sync
+    const int w = __ffs(mask) - 1;
+    X = t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a];
+    Y = t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a];
+    X += Y;
+    Y = X;
+    AR = 0;
+    return;
+  }
   const DivR<MN> dv(r, t.dv);
   u32 m = mask;
   u64 fm = 0, bm = 0, xm = 0;
@@ -329,8 +338,8 @@ __global__ void __launch_bounds__(NT, DFS_MINB) k_search_dfs(DevTables g, Search
         long long o = (long long)X - th;
         if (lv > 0) {
           const u32 mp = stage_mask(sp, S, Rp, lv - 1);
-          const u64 cf = boundary_max<MN>(t.O[a - 1], mp, mk, t.tau, t.dv);
-          const u64 cb = boundary_max<MN>(t.G[a], mk, mp, t.tau, t.dv);
+          u64 cf, cb;
+          boundary_cf_cb<MN>(t, a - 1, mp, mk, cf, cb);
           const long long Z = (long long)(cf + cb);
           ok &= (long long)umax(cf, cb) <= th && O[lv - 1] + Z + (long long)X - th <= 0;
           const long long o2 = O[lv - 1] + Z + (long long)Y - th;
@@ -367,8 +376,8 @@ __global__ void __launch_bounds__(NT, DFS_MINB) k_search_dfs(DevTables g, Search
       long long Pz = -(1ll << 62);
       if (S >= 3) {
         const u32 mp = stage_mask(sp, S, Rp, S - 3);
-        const u64 cf = boundary_max<MN>(t.O[a2 - 1], mp, m2, t.tau, t.dv);
-        const u64 cb = boundary_max<MN>(t.G[a2], m2, mp, t.tau, t.dv);
+        u64 cf, cb;
+        boundary_cf_cb<MN>(t, a2 - 1, mp, m2, cf, cb);
         if ((long long)umax(cf, cb) > th) {  // the whole row fails on boundary S-3
           const u64 rem = (u64)(L - 1 - pk_get(cuts, S - 2));
           if (rem >= i1 - idx) break;
@@ -390,8 +399,8 @@ __global__ void __launch_bounds__(NT, DFS_MINB) k_search_dfs(DevTables g, Search
           e = L - 1;
           break;
         }
-        const u64 cf = boundary_max<MN>(t.O[e], m2, ml, t.tau, t.dv);
-        const u64 cb = boundary_max<MN>(t.G[e + 1], ml, m2, t.tau, t.dv);
+        u64 cf, cb;
+        boundary_cf_cb<MN>(t, e, m2, ml, cf, cb);
         if ((long long)umax(cf, cb) > th) continue;
         u64 Xl, Yl, ARl;
         stage_cost<MN>(t, e + 1, L - 1, ml, sync, Xl, Yl, ARl);

@@ -161,10 +161,20 @@ __global__ void k_build_state(DevTables g, const u64 *__restrict__ fp, const u64
     }
     return;
   }
-  // link tables: one thread per (s, l), s in [0, N-2], l in [0, L-2]
+  // link tables: one thread per (s, l), s in [0, N-2], l in [0, L-2]; then one per (l, u, v) for the
+  // single-worker boundary table xp (forward and backward transfer of the cut after layer l)
   const int t = (blockIdx.x * blockDim.x + threadIdx.x) - (scan_warps + 1) * 32;
   const int per = (L > 1) ? L - 1 : 0;
-  if (t < 0 || per == 0 || t >= (N - 1) * per) return;
+  if (t < 0 || per == 0) return;
+  if (t >= (N - 1) * per) {
+    const int q = t - (N - 1) * per;
+    if (q >= per * N * N) return;
+    const int l = q / (N * N), u = (q / N) % N, v = q % N;
+    u64 *x = g.xp + 2 * ((l * TAUW + u) * TAUW + v);
+    x[0] = (u == v) ? 0ull : xfer(g.O[l], tau[u * N + v]);
+    x[1] = (u == v) ? 0ull : xfer(g.G[l + 1], tau[v * N + u]);
+    return;
+  }
   const int s = t / per, l = t % per;
   const u64 cf = xfer(g.O[l], tau[s * N + s + 1]);
   const u64 cb = xfer(g.G[l + 1], tau[(s + 1) * N + s]);
@@ -177,7 +187,8 @@ __global__ void k_build_state(DevTables g, const u64 *__restrict__ fp, const u64
 int launch_build_state(const DevTables &g, const u64 *fp, const u64 *bp, const u64 *P, const u64 *tau, u64 sumP,
                        cudaStream_t st) {
   const int scan_warps = 3 * (int)g.N + 1;
-  const int links = ((int)g.N - 1) * ((int)g.L > 1 ? (int)g.L - 1 : 0);
+  const int per = (int)g.L > 1 ? (int)g.L - 1 : 0;
+  const int links = ((int)g.N - 1) * per + per * (int)(g.N * g.N);
   const int threads = (scan_warps + 1) * 32 + (links > 0 ? links : 0);
   const int bs = 256;
   const int blocks = (threads + bs - 1) / bs;

@@ -68,8 +68,7 @@ __device__ __forceinline__ u64 startup_completion(const SmemTab &t, int S, u64 c
     if (s < S - 1) {
       const int e = byte_at(cuts, s);
       const u32 ms = (u32)byte_at(masks, s), mn = (u32)byte_at(masks, s + 1);
-      dF[s] = boundary_max<8>(t.O[e], ms, mn, t.tau, t.dv);
-      dB[s] = boundary_max<8>(t.G[e + 1], mn, ms, t.tau, t.dv);
+      boundary_cf_cb<8>(t, e, ms, mn, dF[s], dB[s]);
     }
   }
 

@@ -60,8 +60,7 @@ __device__ __forceinline__ u64 flush_makespan(const SmemTab &t, int S, const P &
     if (s < S - 1) {
       const int e = p.cut(s);
       const u32 ms = p.mask(s), mn = p.mask(s + 1);
-      dF[s] = boundary_max<MN>(t.O[e], ms, mn, t.tau, t.dv);
-      dB[s] = boundary_max<MN>(t.G[e + 1], mn, ms, t.tau, t.dv);
+      boundary_cf_cb<MN>(t, e, ms, mn, dF[s], dB[s]);
     }
   }
 

@@ -481,3 +481,13 @@ def test_gpt96_threshold_walk_full_space(eng, kind):
         eng.set_search_options(False)
     T, idx, _ = optimum(prof, st, 8, 8)
     assert (r.time_ns, r.index, r.evaluated) == (T, idx, comb(95, 7))
+
+
+def test_gpt96_r1_records(eng):
+    """The records of the bench's full-T roofline (workloads.r1_records: S = 8, one worker per stage,
+    uniform cut sets; state C4a, 32-bit path) against the oracle."""
+    prof, st = W.gpt96(), W.gpt_state("a-nvlink")
+    eng.load(prof, st)
+    recs = W.r1_records(prof.L, 8, 600, 5)
+    assert all(parse_record(bytes(r), 96, 8) is not None for r in recs)
+    assert gpu_eval(eng, recs) == score_many(prof, st, [bytes(r) for r in recs])

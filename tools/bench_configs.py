@@ -83,6 +83,14 @@ def measure(device: int = 0, rollout_records: int = 1 << 20):
                                   "rollout_ms": ms_r, "rollout_records_per_s": rollout_records / (ms_r / 1e3),
                                   "eval_GBps_algorithmic": rollout_records * 24 / (ms_e / 1e3) / 1e9,
                                   "int_path": eng.int_path}
+    # full-T scoring of the records the SURVEY's 230-op unit describes: 1M random S = 8, r = 1
+    # partitions of the 96-layer profile (state C4a, 32-bit path), every T computed in full
+    gp = W.gpt96()
+    eng.load(gp, W.gpt_state("a-nvlink"))
+    r1recs = torch.from_numpy(W.r1_records(gp.L, 8, rollout_records, 96)).cuda()
+    ms_r1, _ = _timed(lambda: eng.eval_partitions(r1recs, out=out_t))
+    res["C4_gpt96_r1_records"] = {"records": rollout_records, "eval_ms": ms_r1,
+                                  "eval_records_per_s": rollout_records / (ms_r1 / 1e3), "int_path": eng.int_path}
     # f1: the paper's two-worker neighbourhood step and its gradual migration on
     # the 96-layer profile, heterogeneous state C4b, starting from the even split
     prof, st = W.gpt96(), W.gpt_state("b")

@@ -45,6 +45,10 @@ def main(what):
             eng.switch_rewards(recs, cur, 100)
         else:
             eng.eval_partitions(recs)
+    elif what == "c4_r1_records":
+        gp = W.gpt96()
+        eng.load(gp, W.gpt_state("a-nvlink"))
+        eng.eval_partitions(torch.from_numpy(W.r1_records(gp.L, 8, 1 << 20, 96)).cuda())
     elif what == "vgg_search":
         eng.load(W.vgg16(), W.vgg_state())
         eng.search_optimum(1, 8)

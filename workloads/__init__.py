@@ -406,6 +406,23 @@ def sample_records(L: int, N: int, count: int, seed: int, random_placement_p: fl
     return out
 
 
+def r1_records(L: int, S: int, count: int, seed: int) -> np.ndarray:
+    """`count` 16-byte records of S stages with one worker each (stage s on worker s) and a uniform
+    random cut set: the S = 8, r = 1 candidates the SURVEY's 230-op full-T unit describes. Chunked so
+    the random keys stay small."""
+    rng = np.random.default_rng(seed)
+    out = np.full((count, 16), IDLE, dtype=np.uint8)
+    out[:, 0] = S
+    out[:, 8:8 + S] = np.arange(S, dtype=np.uint8)
+    step = 1 << 16
+    for a in range(0, count, step):
+        n = min(step, count - a)
+        keys = rng.random((n, L - 1), dtype=np.float32)
+        cuts = np.sort(np.argpartition(keys, S - 1, axis=1)[:, :S - 1], axis=1)
+        out[a:a + n, 1:S] = cuts.astype(np.uint8)
+    return out
+
+
 def corrupt_records(recs: np.ndarray, L: int, N: int, seed: int, frac: float = 0.2) -> np.ndarray:
     """Mutate a fraction of records with random field edits (some stay valid, most become invalid)."""
     rng = np.random.default_rng(seed)
