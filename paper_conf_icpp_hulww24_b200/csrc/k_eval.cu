@@ -3,7 +3,7 @@
 //
 // Launch: a persistent grid (one wave of resident 256-thread blocks). Each block stages the state
 // tables into shared memory once (PF, PB, PP, O, G, tau, the divisor table); then every warp on its
-// own takes chunks of 256 records (128 wide ones) from a global counter, loads them with coalesced
+// own takes an equal share of the records in chunks of 256 (128 wide ones), loads them with coalesced
 // 128-bit loads (ld.global.nc), counting-sorts them by shape in its slice of shared memory
 // (sortchunk.cuh) and scores them 32 at a time in shape order: the closed form of SPEC.md §4 in
 // registers, the results written back into the records' shared-memory slots and stored in input
@@ -113,7 +113,7 @@ static void run_eval(int sms, size_t smem, cudaStream_t st, const DevTables &g, 
   const u64 need = (count + CH - 1) / CH;
   const u64 cap = (u64)sms * occ;
   const unsigned grid = (unsigned)(need < cap ? (need ? need : 1) : cap);
-  cudaMemsetAsync(counter, 0, sizeof(u32), st);
+  if (!EvalStatic<Rec>::value) cudaMemsetAsync(counter, 0, sizeof(u32), st);
   kern<<<grid, EVAL_NT, smem, st>>>(g, (const Rec *)recs, count, out_t, out_sw, cur, m, counter);
 }
 

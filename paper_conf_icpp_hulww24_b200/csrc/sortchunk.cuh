@@ -14,6 +14,13 @@
 namespace ap {
 
 constexpr int EV_NB = 64;              // shape buckets
+// equal record ranges per warp for 16-byte records (B200: S = 8 r = 1 GPT-96 records 90 -> 74 us per
+// 1M, C5 -1 %); chunks from a global counter for the wide ones, whose costs vary more (static was 10 %
+// slower there)
+template <typename Rec>
+struct EvalStatic {
+  static constexpr bool value = sizeof(Rec) == 16;
+};
 #ifndef EVAL_PER16
 #define EVAL_PER16 8                   // 16-byte records per lane and warp chunk (B200 C5: 8 beat 4 by 5 %)
 #endif
@@ -75,12 +82,23 @@ __device__ __forceinline__ void for_each_sorted_warp(const Rec *__restrict__ rec
   Rec *sr = srec[w];
   unsigned short *si = sidx[w];
   u32 *h = hist[w];
-  for (;;) {
-    u32 c = 0;
-    if (lane == 0) c = atomicAdd(counter, 1u);
-    c = __shfl_sync(0xffffffffu, c, 0);
-    if ((u64)c >= nch) break;
-    const u64 base = (u64)c * CH;
+  // static split: warp gw of W takes records [count gw / W, count (gw + 1) / W), in chunks of CH
+  // (the same number of records per warp); dynamic: chunks of CH from the global counter
+  constexpr bool STATIC = EvalStatic<Rec>::value;
+  const u64 W = (u64)gridDim.x * NW, gw = (u64)blockIdx.x * NW + w;
+  const u64 r1 = STATIC ? count * (gw + 1) / W : count;
+  u64 base = STATIC ? count * gw / W : 0;
+  for (;; base += CH) {
+    if (STATIC) {
+      if (base >= r1) break;
+    } else {
+      u32 c = 0;
+      if (lane == 0) c = atomicAdd(counter, 1u);
+      c = __shfl_sync(0xffffffffu, c, 0);
+      if ((u64)c >= nch) break;
+      base = (u64)c * CH;
+    }
+    const u64 cend = (r1 - base < (u64)CH) ? r1 : base + CH;
     h[lane] = 0;
     h[lane + 32] = 0;
     __syncwarp();
@@ -91,7 +109,7 @@ __device__ __forceinline__ void for_each_sorted_warp(const Rec *__restrict__ rec
     for (int j = 0; j < PER; ++j) {
       const u64 i = base + (u64)(j * 32 + lane);
       kr[j] = EV_NB;
-      if (i < count) {
+      if (i < cend) {
         const Rec r = load_rec(recs + i);
         sr[j * 32 + lane] = r;
         const u32 key = shape_key(r);
@@ -119,8 +137,7 @@ __device__ __forceinline__ void for_each_sorted_warp(const Rec *__restrict__ rec
       if (key < EV_NB) si[h[key] + (kr[j] >> 8)] = (unsigned short)(j * 32 + lane);
     }
     __syncwarp();
-    const u64 left = count - base;
-    const u32 nvalid = left < (u64)CH ? (u32)left : (u32)CH;
+    const u32 nvalid = (u32)(cend - base);
 #pragma unroll 1
     for (int j = 0; j < PER; ++j) {
       const u32 slot = (u32)(j * 32 + lane);
