@@ -47,11 +47,11 @@ struct SmemTab {
 };
 
 // Number of u64 words the staged tables need: the divisor table (17 x 32 B), PF, PB (N x (L+1)),
-// PP (L+1), O, G (L), tau (16 x 16); the narrow path stages PF32, PB32 and a 32-bit tau in about
-// the same space.
-__host__ __device__ __forceinline__ u32 smem_words(u32 L, u32 N) {
-  return (u32)DIVTAB_WORDS + 2u * N * (L + 1) + (L + 1) + 2u * L + (u32)(TAUW * TAUW) + (u32)(TAUW * TAUW / 2) +
-         256u;
+// PP (L+1), O, G (L), tau (16 x 16); the narrow path stages PF32, PB32 in half the PF/PB space and
+// adds a 32-bit tau and the ring table.
+__host__ __device__ __forceinline__ u32 smem_words(u32 L, u32 N, bool narrow = false) {
+  return (u32)DIVTAB_WORDS + 2u * N * (L + 1) + (L + 1) + 2u * L + (u32)(TAUW * TAUW) +
+         (narrow ? (u32)(TAUW * TAUW / 2) + 256u : 0u);
 }
 
 // Cooperative copy of the global tables into shared memory (every thread of the block calls it).
@@ -95,15 +95,18 @@ __device__ __forceinline__ SmemTab stage_tables(const DevTables &g, u64 *sm) {
     O[i] = g.O[i];
     G[i] = g.G[i];
   }
+  u64 *ring = (u64 *)(tau32 + TAUW * TAUW);
   for (u32 i = threadIdx.x; i < (u32)(TAUW * TAUW); i += blockDim.x) {
     const u64 v = g.tau[i];
     tau[i] = v;
-    tau32[i] = (u32)v;  // meaningful on the narrow path only (tau < 2^32 there)
+    if (NARROW) tau32[i] = (u32)v;  // tau < 2^32 on the narrow path
   }
-  u64 *ring = (u64 *)(tau32 + TAUW * TAUW);
-  for (u32 i = threadIdx.x; i < 256u; i += blockDim.x) ring[i] = g.ring[i];
+  if (NARROW)
+    for (u32 i = threadIdx.x; i < 256u; i += blockDim.x) ring[i] = g.ring[i];
   __syncthreads();
-  t.PP = PP; t.O = O; t.G = G; t.tau = tau; t.tau32 = tau32; t.ring = ring;
+  t.PP = PP; t.O = O; t.G = G; t.tau = tau;
+  t.tau32 = NARROW ? tau32 : nullptr;
+  t.ring = NARROW ? ring : nullptr;
   t.xp = g.xp;
   t.dv = dt;
   t.L = (int)L; t.Lp1 = (int)Lp1;

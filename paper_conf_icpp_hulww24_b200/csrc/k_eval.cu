@@ -142,7 +142,7 @@ int launch_eval(const DevTables &g, const void *recs, u64 count, bool wide, u64 
                 const int *cur_S, const u64 *cur_cuts, const u64 *cur_masks, int path32, const ModelP &m, int sms,
                 u32 *counter, cudaStream_t st) {
   if (count == 0) return 0;
-  const size_t smem = (size_t)smem_words(g.L, g.N) * sizeof(u64);
+  const size_t smem = (size_t)smem_words(g.L, g.N, (path32 & 2) != 0) * sizeof(u64);
   CurPart cur;
   memset(&cur, 0, sizeof(cur));
   if (cur_S) {

@@ -99,7 +99,7 @@ __global__ void __launch_bounds__(NT, GEN_MINB) k_search_generic(DevTables g, Se
   constexpr int BK = SP::BK;
   extern __shared__ u64 sm[];
   // binomial rows n <= L (n = N <= 16 <= L + 1 for the compositions too) after the state tables
-  u64 *Bn = sm + smem_words(g.L, g.N);
+  u64 *Bn = sm + smem_words(g.L, g.N, NARROW);
   const int nb = ((int)g.L + 1 > MAXNW + 1 ? (int)g.L + 1 : MAXNW + 1) * BK;
   for (int i = threadIdx.x; i < nb; i += NT) Bn[i] = g_binom[i / BK][i % BK];
   const SmemTab t = stage_tables<NARROW>(g, sm);  // ends with __syncthreads()
@@ -489,7 +489,7 @@ int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, 
     u64 blocks = (span + per * NT - 1) / (per * NT);
     if (blocks == 0) blocks = 1;
     const int BK = wide ? BINOM_K : BK8;
-    const size_t smem = ((size_t)smem_words(g.L, g.N) +
+    const size_t smem = ((size_t)smem_words(g.L, g.N, true) +
                          (size_t)(((int)g.L + 1 > MAXNW + 1 ? (int)g.L + 1 : MAXNW + 1) * BK)) * sizeof(u64);
     ModelP mm = m;
     const unsigned nbk = (unsigned)blocks;
