@@ -219,6 +219,14 @@ int autopipe_rollout_rewards(autopipe_ctx *ctx, const autopipe_partition *d_part
  * An invalid *h_current -> E_INVAL; requires a state (E_STATE). */
 int autopipe_neighbourhood(autopipe_ctx *ctx, const autopipe_partition *h_current, autopipe_partition *d_out,
                            uint64_t capacity, uint64_t *h_count, void *stream);
+/* The paper's gradual migration ("gradually migrate ... to the best neighbour"):
+ * from *h_start, repeatedly move to the best two-worker neighbour (autopipe_neighbourhood_best)
+ * while it is strictly faster, at most max_steps moves. h_path[capacity] (HOST) receives the path:
+ * entry 0 = the start (its T_ns, evaluated = 1), then one entry per move (T_ns, evaluated =
+ * neighbourhood size, the record); *h_count = entries written. Synchronous; every score comes from
+ * the kernels. Errors as autopipe_neighbourhood_best; E_INVAL for NULL pointers or capacity 0. */
+int autopipe_local_search(autopipe_ctx *ctx, const autopipe_partition *h_start, uint32_t max_steps,
+                          autopipe_result *h_path, uint32_t capacity, uint32_t *h_count, void *stream);
 int autopipe_neighbourhood_best(autopipe_ctx *ctx, const autopipe_partition *h_current, autopipe_result *h_out,
                                 void *stream);
 

@@ -39,7 +39,7 @@ SYMBOLS = ["autopipe_create", "autopipe_destroy", "autopipe_last_error", "autopi
            "autopipe_get_schedule", "autopipe_eval_partitions_w", "autopipe_rollout_rewards_w",
            "autopipe_search_optimum_w", "autopipe_decode_index_w", "autopipe_search_optimum_async",
            "autopipe_search_optimum_async_w", "autopipe_reduce_results", "autopipe_reduce_results_w", "autopipe_search_times",
-           "autopipe_search_seed_async", "autopipe_set_search_bound"]
+           "autopipe_search_seed_async", "autopipe_set_search_bound", "autopipe_local_search"]
 
 
 class Partition(ctypes.Structure):
@@ -96,6 +96,7 @@ def _load():
         "autopipe_kernel_launches": (u64, [P]),
         "autopipe_set_timing": (i32, [P, i32]),
         "autopipe_set_search_options": (i32, [P, u32]),
+        "autopipe_local_search": (i32, [P, P, u32, P, u32, P, P]),
         "autopipe_last_search_ms": (ctypes.c_double, [P]),
         "autopipe_neighbourhood": (i32, [P, ctypes.POINTER(Partition), P, u64, pu64, P]),
         "autopipe_neighbourhood_best": (i32, [P, ctypes.POINTER(Partition), ctypes.POINTER(Result), P]),

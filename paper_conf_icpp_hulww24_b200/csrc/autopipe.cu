@@ -1088,6 +1088,48 @@ extern "C" int autopipe_neighbourhood_best(autopipe_ctx *c, const autopipe_parti
   return AUTOPIPE_OK;
 }
 
+// The paper's gradual migration: from *h_start, move to the best two-worker
+// neighbour while it is strictly faster. Every score comes from the eval kernel; the loop runs here.
+extern "C" int autopipe_local_search(autopipe_ctx *c, const autopipe_partition *h_start, uint32_t max_steps,
+                                     autopipe_result *h_path, uint32_t capacity, uint32_t *h_count, void *stream) {
+  if (!c) return AUTOPIPE_E_INVAL;
+  c->err[0] = 0;
+  if (!h_start || !h_path || !h_count || capacity == 0) return fail(c, AUTOPIPE_E_INVAL, "NULL pointer or zero capacity");
+  if (!c->has_state) return fail(c, AUTOPIPE_E_STATE, "local search before set_state");
+  if (c->N > (u32)MAXN) return fail(c, AUTOPIPE_E_INVAL, "the neighbourhood uses 16-byte records: N <= 8");
+  int S = 0;
+  u64 cuts = 0, masks = 0;
+  if (!host_decode(h_start, c->L, c->N, S, cuts, masks)) return fail(c, AUTOPIPE_E_INVAL, "invalid start partition");
+  DeviceGuard dg(c->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  int rc = sync_status(c, st);
+  if (rc) return rc;
+  rc = check_model(c, st);
+  if (rc) return rc;
+  // T of the start: one record through the eval kernel (slot 0 of the neighbourhood area)
+  cudaError_t e = cudaMemcpyAsync(c->d_nslots, h_start, 16, cudaMemcpyHostToDevice, st);
+  if (e != cudaSuccess) return cuda_fail(c, e, "local search");
+  c->launches += launch_eval(c->tab, c->d_nslots, 1, false, c->d_ntimes, nullptr, nullptr, nullptr, nullptr, c->path32,
+                             c->model, c->sms, next_counter(c), st);
+  e = cudaMemcpyAsync(&c->h_result->time_ns, c->d_ntimes, 8, cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  if (e != cudaSuccess) return cuda_fail(c, e, "local search");
+  h_path[0].time_ns = c->h_result->time_ns;
+  h_path[0].index = U64MAX;
+  h_path[0].evaluated = 1;
+  memcpy(&h_path[0].part, h_start, 16);
+  uint32_t n = 1;
+  for (uint32_t step = 0; step < max_steps && n < capacity; ++step) {
+    autopipe_result r;
+    rc = autopipe_neighbourhood_best(c, &h_path[n - 1].part, &r, stream);
+    if (rc) return rc;
+    if (r.time_ns >= h_path[n - 1].time_ns) break;  // no strictly faster neighbour: a local optimum
+    h_path[n++] = r;
+  }
+  *h_count = n;
+  return AUTOPIPE_OK;
+}
+
 // --- NEXT row f2: switching cost as time (reading F-2) ----
 static const u64 LIMIT_SWITCH = 1ull << 52;  // startup event times < 2^10 * bound (DESIGN.md §3 F-2)
 

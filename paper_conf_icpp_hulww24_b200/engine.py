@@ -286,16 +286,16 @@ class Engine:
         return SearchResult(int(res.time_ns), int(res.index), int(res.evaluated), record_bytes(res.part))
 
     def local_search(self, start: bytes, max_steps: int = 100):
-        """The paper's gradual migration: move to the best two-worker neighbour while
-        it is strictly faster. Returns the path [(T_ns, record), ...] starting at `start`."""
-        t0 = self.eval_partitions(torch.frombuffer(bytearray(start), dtype=torch.uint8).view(1, 16))
-        path = [(int(t0.cpu().numpy().view(np.uint64)[0]), bytes(start))]
-        for _ in range(max_steps):
-            r = self.best_neighbour(path[-1][1])
-            if r.time_ns >= path[-1][0]:
-                break
-            path.append((r.time_ns, r.partition))
-        return path
+        """The paper's gradual migration (autopipe_local_search): move to the best
+        two-worker neighbour while it is strictly faster. Returns the path [(T_ns, record), ...]
+        starting at `start`."""
+        cap = max_steps + 1
+        path = (Result * cap)()
+        n = ctypes.c_uint32()
+        cur = Partition.from_buffer_copy(bytes(start))
+        self._check(lib.autopipe_local_search(self._h, ctypes.byref(cur), int(max_steps), path, cap,
+                                              ctypes.byref(n), self._stream()))
+        return [(int(path[i].time_ns), record_bytes(path[i].part)) for i in range(n.value)]
 
     # -- NEXT row f3: schedule variants (PAPER.md:279-299, 347-352, 1081-1082; reading F-3) -----
     def set_schedule(self, schedule: int = _lib.SCHED_PIPEDREAM, sync: int = _lib.SYNC_RING,

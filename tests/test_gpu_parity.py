@@ -491,3 +491,25 @@ def test_gpt96_r1_records(eng):
     recs = W.r1_records(prof.L, 8, 600, 5)
     assert all(parse_record(bytes(r), 96, 8) is not None for r in recs)
     assert gpu_eval(eng, recs) == score_many(prof, st, [bytes(r) for r in recs])
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_local_search_matches_oracle(eng, seed):
+    """autopipe_local_search (the paper's gradual migration) equals the same loop
+    over the oracle's best_neighbour, step by step, on tiny spaces."""
+    from oracle.neighbourhood import all_partitions, best_neighbour
+    from oracle.sim import time_ns
+    rng = np.random.default_rng(2100 + seed)
+    L, N = int(rng.integers(3, 7)), int(rng.integers(2, 5))
+    prof = W.random_profile(L, rng, f_max=1000, bytes_max=10**6)
+    st = W.random_state_small(prof, N, rng, tau_max=10**4)
+    eng.load(prof, st)
+    parts = list(all_partitions(L, N))
+    start = encode_partition(parts[int(rng.integers(len(parts)))])
+    want = [(time_ns(prof, st, parse_record(start, L, N)), start)]
+    for _ in range(50):
+        T, rec, _ = best_neighbour(prof, st, want[-1][1])
+        if T >= want[-1][0]:
+            break
+        want.append((T, rec))
+    assert eng.local_search(start, max_steps=50) == want

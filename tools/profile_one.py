@@ -52,6 +52,10 @@ def main(what):
     elif what == "vgg_search":
         eng.load(W.vgg16(), W.vgg_state())
         eng.search_optimum(1, 8)
+    elif what == "testbed_resnet":
+        prof = W.resnet50()
+        eng.load(prof, W.testbed_state(prof, seed=10))
+        eng.search_optimum(1, 10)
     elif what == "testbed_search":
         prof = W.vgg16()
         eng.load(prof, W.testbed_state(prof, seed=10))
