@@ -307,6 +307,50 @@ __device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, const P
   return umax((u64)T, TAR);
 }
 
+// The closed form for a partition with one worker per stage (every r_s = 1; the r = 1 records of a
+// batch, grouped together by the shape sort): X_s = Y_s = F_s + B_s, no division, no sync term,
+// boundaries from the per-state table. Same value as eval_closed_form (tests score both kinds of
+// batches against the oracle). NARROW: the 32-bit prefix tables are staged.
+template <bool P32, bool NARROW, typename P>
+__device__ __forceinline__ u64 eval_r1(const SmemTab &t, int S, const P &p) {
+  constexpr int MS = P::MS;
+  typedef typename std::conditional<P32, u32, u64>::type V;
+  V acc[MS];
+  V T = 0;
+  int prevw = 0;
+#pragma unroll
+  for (int u = 0; u < MS; ++u) {
+    acc[u] = 0;
+    if (u < S) {
+      const int a = (u == 0) ? 0 : p.cut(u - 1) + 1;
+      const int e = (u == S - 1) ? t.L - 1 : p.cut(u);
+      const int w = __ffs(p.mask(u)) - 1;
+      V X;
+      if constexpr (NARROW)
+        X = (V)(t.PF32[w * t.Lp1 + e + 1] - t.PF32[w * t.Lp1 + a]) + (V)(t.PB32[w * t.Lp1 + e + 1] - t.PB32[w * t.Lp1 + a]);
+      else
+        X = (V)((t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a]) + (t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a]));
+      T = T > X ? T : X;
+      if (u > 0) {
+        const ulonglong2 x = __ldg((const ulonglong2 *)t.xp + (p.cut(u - 1) * TAUW + prevw) * TAUW + w);
+        const V Z = (V)(x.x + x.y);
+        const V lm = (V)umax(x.x, x.y);
+        T = T > lm ? T : lm;
+#pragma unroll
+        for (int s = 0; s < u; ++s) {
+          const V W = acc[s] + Z + X;
+          const V c = (W + (V)(u - s)) / (V)(u - s + 1);
+          T = T > c ? T : c;
+          acc[s] += Z + X;
+        }
+      }
+      acc[u] = X;
+      prevw = w;
+    }
+  }
+  return (u64)T;
+}
+
 // ------------------------------------------------------------------------------------------------
 // The narrow path of the closed form (status bit 2; explicit-record scoring under PipeDream): every
 // per-worker stage sum of f or of b is < 2^31 - 16, so F' and B' are 32-bit ceil divisions by the

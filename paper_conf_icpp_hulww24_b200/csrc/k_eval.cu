@@ -43,6 +43,11 @@ __device__ __forceinline__ bool decode_any(const Rec16 &r, int L, int N, int &S,
 __device__ __forceinline__ bool decode_any(const Rec32 &r, int L, int N, int &S, P16 &p) {
   return decode_record_w(r.a, r.b, L, N, S, p);
 }
+// every stage has exactly one worker (sum of the stage masks' bits = S)
+__device__ __forceinline__ bool all_single(const P8 &p, int S) { return __popcll(p.masks) == S; }
+__device__ __forceinline__ bool all_single(const P16 &p, int S) {
+  return __popcll(p.m[0]) + __popcll(p.m[1]) + __popcll(p.m[2]) + __popcll(p.m[3]) == S;
+}
 __device__ __forceinline__ const P8 &cur_part(const CurPart &c, const P8 *) { return c.p8; }
 __device__ __forceinline__ const P16 &cur_part(const CurPart &c, const P16 *) { return c.p16; }
 
@@ -54,8 +59,13 @@ __device__ __forceinline__ void score_one(const SmemTab &t, int L, int N, bool o
   int S;
   P p;
   u64 T = U64MAX, sw = U64MAX;
-  if (!overflow && decode_any(slot, L, N, S, p)) {
-    if constexpr (NARROW) T = eval_closed_form_n<P32, P>(t, S, p, (int)m.sync);
+  const bool ok = !overflow && decode_any(slot, L, N, S, p);
+  // the lean r = 1 closed form when every active lane holds a one-worker-per-stage record (the
+  // shape sort puts them together); a mixed step keeps the general form, so lanes do not diverge
+  const bool lean = MODE == SCHED_PIPEDREAM && __all_sync(__activemask(), ok && all_single(p, S));
+  if (ok) {
+    if (lean) T = eval_r1<P32, NARROW, P>(t, S, p);
+    else if constexpr (NARROW) T = eval_closed_form_n<P32, P>(t, S, p, (int)m.sync);
     else T = model_time<MODE, P32>(t, S, p, m);
     if (ROLLOUT) sw = switch_bytes(t, S, p, cur.S, cur_part(cur, (const P *)nullptr));
   }
