@@ -358,6 +358,13 @@ int autopipe_set_timing(autopipe_ctx *ctx, int enable);
  * AUTOPIPE_SEARCH_SPLIT = always the per-S split. E_INVAL on unknown bits. */
 #define AUTOPIPE_SEARCH_SPLIT 1u
 #define AUTOPIPE_SEARCH_NO_R1 2u  /* the r = 1 blocks through the threshold walk instead of the r = 1 sweep */
+/* Round-robin replicas (AUTOPIPE_SCHED_PIPEDREAM_RR) evaluations: a record whose schedule is not
+ * pinned within a budget of rounds is deferred to a drain kernel (a warp per record, Bellman-Ford in
+ * the bracket its simulation gives). RR_DEFER_ALL: a budget of one round (nearly every record takes
+ * the drain); RR_NO_DEFER: no deferral (every record finished in its own thread). Results are
+ * identical either way. */
+#define AUTOPIPE_RR_DEFER_ALL 4u
+#define AUTOPIPE_RR_NO_DEFER 8u
 int autopipe_set_search_options(autopipe_ctx *ctx, uint32_t options);
 
 /* Device milliseconds of the enumeration kernels of the last timed search (-1 if none); waits for

@@ -47,6 +47,12 @@ struct autopipe_ctx {
   // launches on different streams never share one
   static const int NCTR = 256;
   u32 *d_ctr = nullptr;
+  // row f4, round-robin replicas: the deferral queue of the eval kernels (RRQueue) and the event of
+  // the last drain that used it (the next evaluation's stream waits for it)
+  static const u32 RRQ_CAP = 1u << 14;
+  u64 *d_rrq = nullptr;
+  u32 *d_rrq_n = nullptr;
+  cudaEvent_t ev_rrq = nullptr;
   u32 ctr_next = 0;
   // the same for the search kernels' schedules (SEARCH_SCHED_BYTES per launch)
   unsigned char *d_sched = nullptr;
@@ -89,6 +95,22 @@ struct autopipe_ctx {
 };
 
 static char g_create_err[256] = "";
+
+// The round-robin deferral queue for an evaluation on stream st (row f4): st first waits for the
+// previous drain that used the queue, and the caller records ev_rrq after its own launch.
+static RRQueue rr_queue(autopipe_ctx *c, cudaStream_t st, bool wide) {
+  RRQueue q;
+  if (c->model.sched != SCHED_RR || wide || (c->search_options & AUTOPIPE_RR_NO_DEFER)) return q;
+  cudaStreamWaitEvent(st, c->ev_rrq, 0);
+  q.buf = c->d_rrq;
+  q.n = c->d_rrq_n;
+  q.cap = autopipe_ctx::RRQ_CAP;
+  q.rounds = (c->search_options & AUTOPIPE_RR_DEFER_ALL) ? 1u : RR_DEFER_ROUNDS;
+  return q;
+}
+static void rr_queue_done(autopipe_ctx *c, cudaStream_t st, const RRQueue &q) {
+  if (q.buf) cudaEventRecord(c->ev_rrq, st);
+}
 
 static u32 *next_counter(autopipe_ctx *c) { return c->d_ctr + (c->ctr_next++ % autopipe_ctx::NCTR); }
 static void *next_sched(autopipe_ctx *c) {
@@ -179,6 +201,9 @@ extern "C" int autopipe_create(int cuda_device, autopipe_ctx **out) {
   if (e == cudaSuccess) e = cudaMalloc(&c->d_ntimes, (size_t)NEIGH_ITEMS * NEIGH_MAXOPT * 8);
   if (e == cudaSuccess) e = cudaMalloc(&c->d_ncount, 8);
   if (e == cudaSuccess) e = cudaMalloc(&c->d_ctr, sizeof(u32) * autopipe_ctx::NCTR);
+  if (e == cudaSuccess) e = cudaMalloc(&c->d_rrq, sizeof(u64) * 3 * autopipe_ctx::RRQ_CAP);
+  if (e == cudaSuccess) e = cudaMalloc(&c->d_rrq_n, sizeof(u32));
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_rrq, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaMalloc(&c->d_sched, (size_t)SEARCH_SCHED_BYTES * autopipe_ctx::NCTR);
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_ncount, 8);
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_stage, (2 * MAXNW * MAXL + TT) * 8);
@@ -233,6 +258,9 @@ extern "C" void autopipe_destroy(autopipe_ctx *c) {
     if (c->d_ntimes) cudaFree(c->d_ntimes);
     if (c->d_ncount) cudaFree(c->d_ncount);
     if (c->d_ctr) cudaFree(c->d_ctr);
+    if (c->d_rrq) cudaFree(c->d_rrq);
+    if (c->d_rrq_n) cudaFree(c->d_rrq_n);
+    if (c->ev_rrq) cudaEventDestroy(c->ev_rrq);
     if (c->d_sched) cudaFree(c->d_sched);
     if (c->h_ncount) cudaFreeHost(c->h_ncount);
     if (c->h_stage) cudaFreeHost(c->h_stage);
@@ -468,8 +496,10 @@ static int eval_impl(autopipe_ctx *c, const void *d_parts, uint64_t count, bool 
   if (rc) return rc;
   // a state given in device memory has not been classified on the host yet: use the 64-bit path
   const int p32 = c->state_on_device ? 0 : (c->path32 | (c->narrow << 1));
+  const RRQueue q = rr_queue(c, (cudaStream_t)stream, wide);
   c->launches += launch_eval(c->tab, d_parts, count, wide, (u64 *)d_time_ns, nullptr, nullptr, nullptr, nullptr, p32,
-                             c->model, c->sms, next_counter(c), (cudaStream_t)stream);
+                             c->model, c->sms, next_counter(c), (cudaStream_t)stream, q);
+  rr_queue_done(c, (cudaStream_t)stream, q);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "eval kernel launch");
   return AUTOPIPE_OK;
@@ -674,7 +704,24 @@ static int search_impl(autopipe_ctx *c, u32 s_min, u32 s_max, u32 flags, u64 beg
   // rest (threshold walk or generic); the pieces write disjoint block-result ranges and run
   // concurrently.
   u64 cur = begin;
-  if (end - begin <= DENSE_SPAN && !(c->search_options & AUTOPIPE_SEARCH_SPLIT)) {
+  if (c->model.sched == SCHED_RR && !wide) {
+    // row f4, round-robin replicas: one bound-pruned launch over the whole range plus the drain of
+    // its deferred candidates (the deferral queue is the context's; the stream waits for its last user)
+    RRQueue q = rr_queue(c, st, false);
+    if (!q.buf) {  // AUTOPIPE_RR_NO_DEFER: a queue of capacity 0 (every candidate in its thread)
+      cudaStreamWaitEvent(st, c->ev_rrq, 0);
+      q.n = c->d_rrq_n;
+      q.buf = c->d_rrq;
+      q.cap = 0;
+    }
+    int nb = 0;
+    c->launches += launch_search_rr(c->tab, sp, begin, end, c->model, c->sms, c->d_blocks, MAX_BLOCKS, &nb,
+                                    next_sched(c), q, st);
+    cudaEventRecord(c->ev_rrq, st);
+    used = nb;
+    cur = end;
+  }
+  if (cur < end && end - begin <= DENSE_SPAN && !(c->search_options & AUTOPIPE_SEARCH_SPLIT)) {
     int nb = 0;
     // a host-classified state may take the narrow (32-bit stage arithmetic) closed form (bit 1)
     const int dpath = path >= 0 ? (path | (c->narrow << 1)) : path;
@@ -946,9 +993,11 @@ static int rollout_impl(autopipe_ctx *c, const void *d_parts, uint64_t count, co
   int rc = check_model(c, (cudaStream_t)stream, wide);
   if (rc) return rc;
   const int p32 = c->state_on_device ? 0 : (c->path32 | (c->narrow << 1));
+  const RRQueue q = rr_queue(c, (cudaStream_t)stream, wide);
   c->launches += launch_eval(c->tab, d_parts, count, wide, (u64 *)d_time_ns, (u64 *)d_switch_bytes,
                              h_current ? &S : nullptr, cuts, masks, p32, c->model, c->sms, next_counter(c),
-                             (cudaStream_t)stream);
+                             (cudaStream_t)stream, q);
+  rr_queue_done(c, (cudaStream_t)stream, q);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "rollout kernel launch");
   return AUTOPIPE_OK;
@@ -980,7 +1029,7 @@ extern "C" uint64_t autopipe_kernel_launches(const autopipe_ctx *c) { return c ?
 extern "C" int autopipe_set_search_options(autopipe_ctx *c, uint32_t options) {
   if (!c) return AUTOPIPE_E_INVAL;
   c->err[0] = 0;
-  if (options & ~(AUTOPIPE_SEARCH_SPLIT | AUTOPIPE_SEARCH_NO_R1))
+  if (options & ~(AUTOPIPE_SEARCH_SPLIT | AUTOPIPE_SEARCH_NO_R1 | AUTOPIPE_RR_DEFER_ALL | AUTOPIPE_RR_NO_DEFER))
     return fail(c, AUTOPIPE_E_INVAL, "unknown search options 0x%x", options);
   c->search_options = options;
   return AUTOPIPE_OK;

@@ -27,9 +27,19 @@ int launch_build_state(const DevTables &g, const u64 *fp, const u64 *bp, const u
 // partition's packed parts (1 and 1 words, or 2 and 4 words for wide), or cur_S = nullptr.
 // counter: a device word the launch resets (cudaMemsetAsync) and the kernel's warps draw chunks from.
 // path32: bit 0 = the state's 32-bit path, bit 1 = its narrow path (status bit 2; PipeDream only).
+// rrq (round-robin replicas only, row f4): the context's deferral queue; records whose schedule has
+// not been pinned within RR_DEFER_ROUNDS rounds go there and a drain kernel finishes them, a warp
+// per record (k_eval.cu). Without a queue every record is finished in its own thread.
+struct RRQueue {
+  u64 *buf = nullptr;  // [cap][3]: record index, bracket low, bracket high
+  u32 *n = nullptr;    // entries claimed (may exceed cap: those records were finished in the thread)
+  u32 cap = 0;
+  u32 rounds = 0;      // round budget before a record is deferred
+};
+constexpr u32 RR_DEFER_ROUNDS = 256;
 int launch_eval(const DevTables &g, const void *recs, u64 count, bool wide, u64 *out_t, u64 *out_sw,
                 const int *cur_S, const u64 *cur_cuts, const u64 *cur_masks, int path32, const ModelP &m, int sms,
-                u32 *counter, cudaStream_t st);
+                u32 *counter, cudaStream_t st, const RRQueue &rrq = RRQueue());
 // Generic exhaustive search over [begin, end) (any S, any composition); writes one BlockOut per block
 // into out[out_offset ...] and returns the number of blocks used via *nblocks.
 // path32 of a dense launch: bit 0 = 32-bit segment sums, bit 1 = the narrow closed form (-1: gated)
@@ -49,6 +59,11 @@ struct R1Ext {
   const u64 *bound = nullptr;
   u64 *theta_out = nullptr;
 };
+// Round-robin replicas search (row f4, 16-byte spaces): the bound-pruned kernel over [begin, end)
+// and the drain of its deferred candidates; writes the blocks of both (*nblocks). sched: a 32-byte
+// schedule slot; q: the context's deferral queue (not shared with a concurrent launch).
+int launch_search_rr(const DevTables &g, const SearchSpace &sp, u64 begin, u64 end, const ModelP &m, int sms,
+                     BlockOut *out, int max_blocks, int *nblocks, void *sched, const RRQueue &q, cudaStream_t st);
 // Fast search over the r = 1 block of one S (all stages on one worker; SPEC.md §5, rho = 0),
 // restricted to the cut ranks [k_begin, k_end). path32 selects the 32-bit tables.
 int launch_search_r1(const DevTables &g, const SearchSpace &sp, int S, u64 k_begin, u64 k_end,

@@ -13,6 +13,7 @@
 #include "eval.cuh"
 #include "internal.h"
 #include "sched.cuh"
+#include "rr.cuh"
 
 namespace ap {
 
@@ -450,6 +451,160 @@ static void run_search_generic(unsigned nbk, size_t smem, cudaStream_t st, const
       }
     }
   }
+}
+
+// ---------------------------------------------------------------------------------------------
+// Round-robin replicas search (row f4, 16-byte spaces). Every candidate is decided exactly, but most
+// are decided by bounds: a candidate whose lower bound exceeds theta cannot be the lexicographic
+// minimum (theta = min(the thread's best - 1, the launch's best so far); the launch's best is the T
+// of a real candidate, so a strictly greater bound is safe whatever the indices). The lower bound is
+// first the single-resource one (rr_lower, Tsync), then the recurrence's own growth bound, which
+// stops the simulation as soon as it passes theta. A candidate the recurrence has not pinned within
+// RR_DEFER_ROUNDS rounds goes to the deferral queue with its bracket; the drain kernel finishes the
+// queued candidates that can still win (bracket low <= the launch's best) with warp-parallel
+// Bellman-Ford and contributes one (T, index) per block to the final reduction.
+// Launch: one wave of 256-thread blocks drawing chunks of consecutive indices from a counter (the
+// costs of neighbouring candidates vary together); a thread unranks its chunk's first index once,
+// then steps with the lexicographic successor.
+struct RRSearchSched {
+  u64 best;   // the launch's best T so far (atomicMin)
+  u32 chunk;  // next chunk
+  u32 pad;
+};
+constexpr int RR_NT = 256;
+__global__ void __launch_bounds__(RR_NT, 2) k_search_rr(DevTables g, SearchSpace sp, u64 begin, u64 end, u64 chunk,
+                                                        BlockOut *out, ModelP m, RRSearchSched *rs, RRQueue q) {
+  typedef SpaceT<P8> SP;
+  typedef typename SP::PK PK;
+  constexpr int BK = SP::BK;
+  extern __shared__ u64 sm[];
+  u64 *Bn = sm + smem_words(g.L, g.N);
+  const int nb = ((int)g.L + 1 > MAXNW + 1 ? (int)g.L + 1 : MAXNW + 1) * BK;
+  for (int i = threadIdx.x; i < nb; i += RR_NT) Bn[i] = g_binom[i / BK][i % BK];
+  const SmemTab t = stage_tables<false>(g, sm);  // ends with __syncthreads()
+  const int sync = (int)m.sync;
+  const u64 span = end - begin, nch = (span + chunk - 1) / chunk;
+  volatile u64 *gbest = &rs->best;
+  u64 bestT = U64MAX, bestI = U64MAX, cnt = 0;
+  for (;;) {
+    const u64 c = atomicAdd(&rs->chunk, 1u);
+    if (c >= nch) break;
+    const u64 i0 = begin + c * chunk, i1 = (end - i0 < chunk) ? end : i0 + chunk;
+    int S;
+    PK Rp, cuts;
+    unrank_global_smem<BK>(sp, i0, S, Rp, cuts, Bn);
+    for (u64 i = i0; i < i1; ++i) {
+      const P8 p = part_from<P8>(sp, S, Rp, cuts);
+      const u64 gb = *gbest;
+      const u64 theta = umin(bestT - 1, gb);  // bestT = U64MAX: no own best yet
+      RRSetup R;
+      rr_setup(t, S, p, sync, R);
+      u64 T = U64MAX;
+      if (S == 1) {
+        T = umax(rr_single_stage(R), R.Tsync);
+      } else if (umax(rr_lower(R), R.Tsync) <= theta) {
+        u64 t_lo, t_hi;
+        const int rc = rr_sim(R, q.rounds ? q.rounds : RR_SIM_ROUNDS, theta, t_lo, t_hi, nullptr);
+        if (rc == RR_MET || (rc == RR_BUDGET && R.Tsync >= t_hi)) {
+          T = umax(t_lo, R.Tsync);
+        } else if (rc == RR_BUDGET && umax(t_lo, R.Tsync) <= theta) {
+          const u32 k = atomicAdd(q.n, 1u);
+          if (k < q.cap) {
+            q.buf[3 * (u64)k] = i;
+            q.buf[3 * (u64)k + 1] = t_lo;
+            q.buf[3 * (u64)k + 2] = t_hi;
+          } else {
+            T = umax(rr_ceil_bf(R, t_lo, t_hi), R.Tsync);
+          }
+        }
+      }
+      if (T < bestT) {  // indices increase along the chunk: strict < keeps the first
+        bestT = T;
+        bestI = i;
+        if (T < gb) atomicMin((unsigned long long *)&rs->best, T);
+      }
+      ++cnt;
+      if (i + 1 == i1) break;
+      if (!SP::next(cuts, S - 1, sp.L - 1)) {  // cut set exhausted: next composition
+        cuts = first_subset<PK>(S - 1);
+        if (!SP::next(Rp, comp_k(sp, S), comp_n(sp))) {  // compositions exhausted: next S
+          ++S;
+          if (S > sp.s_max) break;
+          Rp = first_subset<PK>(comp_k(sp, S));
+          cuts = first_subset<PK>(S - 1);
+        }
+      }
+    }
+  }
+  block_minloc_store<RR_NT>(bestT, bestI, cnt, out + blockIdx.x);
+}
+
+// The deferred candidates of k_search_rr that can still win (bracket low <= the launch's best; a tie
+// may win on its index), a warp each; one (T, index) per block into out (count 0: the search kernel
+// counted them).
+__global__ void __launch_bounds__(RR_NT) k_rr_drain_search(DevTables g, SearchSpace sp, BlockOut *out, ModelP m,
+                                                           const RRSearchSched *rs, RRQueue q) {
+  const u32 n = umin(*q.n, q.cap);
+  u64 bestT = U64MAX, bestI = U64MAX;
+  if (n > 0) {
+    typedef SpaceT<P8> SP;
+    typedef typename SP::PK PK;
+    constexpr int BK = SP::BK;
+    extern __shared__ u64 sm[];
+    __shared__ long long dist[RR_NT / 32][RR_BF_NODES];
+    u64 *Bn = sm + smem_words(g.L, g.N);
+    const int nb = ((int)g.L + 1 > MAXNW + 1 ? (int)g.L + 1 : MAXNW + 1) * BK;
+    for (int i = threadIdx.x; i < nb; i += RR_NT) Bn[i] = g_binom[i / BK][i % BK];
+    const SmemTab t = stage_tables<false>(g, sm);
+    const u64 best = rs->best;
+    const int w = threadIdx.x >> 5;
+    for (u32 k = blockIdx.x * (RR_NT / 32) + w; k < n; k += gridDim.x * (RR_NT / 32)) {
+      const u64 i = q.buf[3 * (u64)k], t_lo = q.buf[3 * (u64)k + 1], t_hi = q.buf[3 * (u64)k + 2];
+      if (t_lo > best) continue;  // warp-uniform
+      int S;
+      PK Rp, cuts;
+      unrank_global_smem<BK>(sp, i, S, Rp, cuts, Bn);
+      const P8 p = part_from<P8>(sp, S, Rp, cuts);
+      RRSetup R;
+      rr_setup(t, S, p, (int)m.sync, R);
+      const u64 T = umax(rr_ceil_bf_warp(R, t_lo, t_hi, dist[w]), R.Tsync);
+      if (better(T, i, bestT, bestI)) bestT = T, bestI = i;
+    }
+  }
+  block_minloc_store<RR_NT>(bestT, bestI, 0, out + blockIdx.x);
+}
+
+int launch_search_rr(const DevTables &g, const SearchSpace &sp, u64 begin, u64 end, const ModelP &m, int sms,
+                     BlockOut *out, int max_blocks, int *nblocks, void *sched, const RRQueue &q, cudaStream_t st) {
+  static_assert(sizeof(RRSearchSched) <= SEARCH_SCHED_BYTES, "schedule slot");
+  const u64 span = end - begin;
+  const size_t smem = ((size_t)smem_words(g.L, g.N) +
+                       (size_t)(((int)g.L + 1 > MAXNW + 1 ? (int)g.L + 1 : MAXNW + 1) * BK8)) * sizeof(u64);
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncAttributes fa;
+    cudaFuncGetAttributes(&fa, k_rr_drain_search);
+    cudaFuncSetAttribute(k_rr_drain_search, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         227 * 1024 - (int)fa.sharedSizeBytes);
+    attr = true;
+  }
+  u64 wave = (u64)sms * 2;
+  if (wave > (u64)max_blocks / 2) wave = (u64)max_blocks / 2;
+  u64 chunk = span / (wave * RR_NT * 8);
+  if (chunk < 1) chunk = 1;
+  while ((span + chunk - 1) / chunk >= (1ull << 31)) chunk *= 2;
+  u64 blocks = ((span + chunk - 1) / chunk + RR_NT - 1) / RR_NT;
+  if (blocks > wave) blocks = wave;
+  if (blocks == 0) blocks = 1;
+  u64 dblocks = (u64)sms < (u64)max_blocks - blocks ? (u64)sms : (u64)max_blocks - blocks;
+  RRSearchSched *rs = (RRSearchSched *)sched;
+  cudaMemsetAsync(rs, 0, sizeof(RRSearchSched), st);
+  cudaMemsetAsync(&rs->best, 0xFF, sizeof(u64), st);
+  cudaMemsetAsync(q.n, 0, sizeof(u32), st);
+  k_search_rr<<<(unsigned)blocks, RR_NT, smem, st>>>(g, sp, begin, end, chunk, out, m, rs, q);
+  k_rr_drain_search<<<(unsigned)dblocks, RR_NT, smem, st>>>(g, sp, out + blocks, m, rs, q);
+  *nblocks = (int)(blocks + dblocks);
+  return 2;
 }
 
 int launch_search_generic(const DevTables &g, const SearchSpace &sp, u64 begin, u64 end, int path32, const ModelP &m,

@@ -8,24 +8,37 @@
 // (forward O[e_s]) and back (G[e_s + 1]), FIFO per directed link; a replicated stage synchronises
 // once per r_s mini-batches, overlapped: T = max(ceil(lambda_compute), max_s ceil(d_s / r_s)).
 //
-// lambda_compute has no closed form here; one thread finds it exactly by running the schedule's
-// max-plus recurrence round by round in dependency order (round j: B_s(j) for s descending, then
-// F_s(j + D_s) for s ascending, D_s = min_{u<=s} m_u r_u; every op's inputs are produced earlier)
-// and detecting the periodic regime with Brent's cycle search over the state at the start of
-// every block of Lam = lcm(r) rounds: the free time of every worker and link and the forward
-// transfers not yet consumed, rebased per class of mini-batches (k mod gcd(r): classes share no
-// worker and no link). When the rebased state repeats after c blocks, each class has advanced by
-// its shift D_c: lambda_compute = max_c D_c / (c Lam). The oracle finds the same period by hashing
-// windows of rounds in a generic ready-driven simulation.
+// lambda_compute has no closed form here. One thread runs the schedule's max-plus recurrence round
+// by round in dependency order (round j: B_s(j) for s descending, then F_s(j + D_s) for s ascending,
+// D_s = min_{u<=s} m_u r_u; every op's inputs are produced earlier), one block of Lam = lcm(r)
+// rounds at a time, and compares the state (the free time of every worker and link and the forward
+// transfers not yet consumed) with a saved one (Brent's tortoise): per class of mini-batches
+// (k mod gcd(r): classes share no worker and no link) the growth of every component since the save
+// bounds that class's rate from both sides (max-plus homogeneity), and T is exact as soon as the
+// ceilings of the two bounds agree — in particular when the schedule has repeated (every component
+// of a class moved by the same amount). The oracle finds the period by hashing windows of rounds in
+// a generic ready-driven simulation.
+//
+// Records whose bounds have not met within a round budget (two near-equal cycle ratios can make the
+// transient arbitrarily long) take ceil(lambda) from the timed event graph of one period: the
+// smallest integer theta with no positive cycle (Bellman-Ford, binary search on theta inside the
+// bracket the bounds give). The eval kernel defers them to a drain kernel that runs the
+// Bellman-Ford passes with a whole warp per record (k_eval.cu), so one slow record does not hold up
+// the 31 other lanes of its warp; the search kernels run it in the thread.
 #pragma once
+#include <climits>
+
 #include "eval.cuh"
 
 namespace ap {
 
-constexpr u32 RR_SIM_ROUNDS = 4096;         // then ceil(lambda) from the event graph (rr_ceil_bf)
-constexpr int RR_BF_NODES = 160;            // 4 S Lam <= 144 nodes for sum r <= 8
-constexpr int RR_LINKS = 32;                // sum over boundaries of lcm(r_s, r_{s+1}) for N <= 8
-constexpr int RR_RING = 16;                 // pending forward transfers per boundary (D_0 <= 15)
+#ifndef RR_STATS
+#define RR_STATS 0
+#endif
+constexpr u32 RR_SIM_ROUNDS = 4096;    // in-thread budget (search; eval when the deferral queue is full)
+constexpr int RR_BF_NODES = 160;       // 4 S Lam <= 144 nodes for sum r <= 8
+constexpr int RR_LINKS = 32;           // sum over boundaries of lcm(r_s, r_{s+1}) for N <= 8
+constexpr int RR_RING = 16;            // pending forward transfers per boundary (D_0 <= 15)
 
 __device__ __forceinline__ u32 gcd_u(u32 a, u32 b) {
   while (b) {
@@ -36,280 +49,371 @@ __device__ __forceinline__ u32 gcd_u(u32 a, u32 b) {
   return a;
 }
 
-// ceil(lambda_compute) from the timed event graph of one period (the oracle's event_graph): the
-// smallest integer theta with no positive cycle of node durations - theta * Lam * edge tokens
-// (Bellman-Ford from a virtual source, binary search on theta, bracketed around the simulation's
-// estimate th0). Nodes (kind, s, phase p): F_s, B_s, forward and backward transfers of boundary s, for
-// the mini-batches k = p (mod Lam). For the rare records whose simulation has not settled (two
-// near-equal cycle ratios can make the transient arbitrarily long); exact like the simulation.
-template <typename DurF>
-__device__ __forceinline__ u64 rr_ceil_bf(int S, u32 Lam, const int *r, const int *m, const int *lc, DurF dur,
-                                          long long th0) {
-  const int V = 4 * S * (int)Lam;
-  long long dist[RR_BF_NODES];
-  const long long K0 = 64ll * Lam;  // a period index far from the start: every predecessor is >= 0
-  auto node = [&](int kind, int s, long long k) { return (kind * S + s) * (int)Lam + (int)(k % Lam); };
-  auto tok = [&](long long kv, long long ku) { return kv / (long long)Lam - ku / (long long)Lam; };
-  auto positive = [&](long long th) -> bool {
-    for (int v = 0; v < V; ++v) dist[v] = 0;
-    for (int pass = 0; pass <= V; ++pass) {
-      bool changed = false;
-      for (int kind = 0; kind < 4; ++kind)
-        for (int s = 0; s < S; ++s) {
-          if (kind >= 2 && s == S - 1) continue;
-          for (u32 p = 0; p < Lam; ++p) {
-            const long long k = K0 + p;
-            const int v = node(kind, s, k);
-            const long long dv = (long long)dur(kind, s, (int)p);
-            long long best = dist[v];
-            auto relax = [&](int ku_kind, int ku_s, long long ku) {
-              const long long c = dist[node(ku_kind, ku_s, ku)] + dv - th * (long long)Lam * tok(k, ku);
-              if (c > best) best = c;
-            };
-            if (kind == 0) {
-              relax(1, s, k - (long long)m[s] * r[s]);         // worker order: after B(k - m r)
-              if (s > 0) relax(2, s - 1, k);                   // forward transfer of boundary s-1
-            } else if (kind == 1) {
-              relax(0, s, k + (long long)(m[s] - 1) * r[s]);   // worker order: after F(k + (m-1) r)
-              if (s < S - 1) relax(3, s, k);                   // backward transfer of boundary s
-            } else if (kind == 2) {
-              relax(0, s, k);                                  // after F_s(k)
-              relax(2, s, k - lc[s]);                          // FIFO on its link
-            } else {
-              relax(1, s + 1, k);                              // after B_{s+1}(k)
-              relax(3, s, k - lc[s]);
-            }
-            if (best > dist[v]) {
-              dist[v] = best;
-              changed = true;
-            }
-          }
-        }
-      if (!changed) return false;
-    }
-    return true;
-  };
-  // bracket [lo, hi]: positive(lo), !positive(hi), around the estimate
-  long long lo, hi, step = 1;
-  if (positive(th0)) {
-    lo = th0;
-    hi = th0 + step;
-    while (positive(hi)) lo = hi, step *= 2, hi = th0 + step;
-  } else {
-    hi = th0;
-    lo = th0 - step;
-    while (lo >= 0 && !positive(lo)) hi = lo, step *= 2, lo = th0 - step;
-    if (lo < 0) lo = -1;
-  }
-  while (hi - lo > 1) {
-    const long long mid = lo + (hi - lo) / 2;
-    if (positive(mid)) lo = mid;
-    else hi = mid;
-  }
-  return (u64)hi;
-}
+// Everything the recurrence and the event graph need about one validated 16-byte record.
+struct RRSetup {
+  int S;
+  u32 Lam, g;   // lcm and gcd of the replica counts
+  u64 Tsync;    // max_s ceil(sync_s / r_s) over the replicated stages
+  u64 dsum;     // sum of every op and transfer duration of one period
+  int negtok;   // the most negative token count of an edge, negated (B_s(k) after F_s(k + (m - 1) r))
+  int r[MAXS], wl[MAXS], D[MAXS], mm[MAXS], lc[MAXS], lo[MAXS];
+  u64 Fw[MAXN], Bw[MAXN], tf[RR_LINKS], tb[RR_LINKS];
+};
 
-// T_ns of a validated 16-byte partition under round-robin replicas.
-static __device__ __noinline__ u64 rr_time(const SmemTab &t, int S, const P8 &p, int sync) {
-  int r[MAXS], wl[MAXS], D[MAXS], lc[MAXS], lo[MAXS];
-  u64 Fw[MAXN], Bw[MAXN];
-  u64 Tsync = 0;
-  u32 Lam = 1, g = 0;
+__device__ __forceinline__ void rr_setup(const SmemTab &t, int S, const P8 &p, int sync, RRSetup &R) {
+  R.S = S;
+  R.Tsync = 0;
+  R.Lam = 1;
+  R.g = 0;
   for (int s = 0; s < S; ++s) {
     const u32 mask = p.mask(s);
-    r[s] = __popc(mask);
+    R.r[s] = __popc(mask);
     const int a = (s == 0) ? 0 : p.cut(s - 1) + 1;
     const int e = (s == S - 1) ? t.L - 1 : p.cut(s);
     int packed = 0, i = 0;
     for (u32 mm = mask; mm; mm &= mm - 1, ++i) {
       const int w = __ffs(mm) - 1;
       packed |= w << (4 * i);
-      Fw[w] = t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a];  // whole mini-batch: no split
-      Bw[w] = t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a];
+      R.Fw[w] = t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a];  // whole mini-batch: no split
+      R.Bw[w] = t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a];
     }
-    wl[s] = packed;
-    if (r[s] >= 2) {  // one synchronisation per r_s mini-batches
+    R.wl[s] = packed;
+    if (R.r[s] >= 2) {  // one synchronisation per r_s mini-batches
       const u64 d = sync_time<8>(sync, t.PP[e + 1] - t.PP[a], mask, t.tau, t.dv);
-      Tsync = umax(Tsync, (d + r[s] - 1) / (u64)r[s]);
+      R.Tsync = umax(R.Tsync, (d + R.r[s] - 1) / (u64)R.r[s]);
     }
-    Lam = Lam / gcd_u(Lam, (u32)r[s]) * (u32)r[s];
-    g = gcd_u(g, (u32)r[s]);
-  }
-  if (S == 1) {  // no boundary: each replica on its own, one mini-batch in every r
-    u64 T = 0;
-    for (int i = 0; i < r[0]; ++i) {
-      const int w = (wl[0] >> (4 * i)) & 15;
-      T = umax(T, (Fw[w] + Bw[w] + r[0] - 1) / (u64)r[0]);
-    }
-    return umax(T, Tsync);
+    R.Lam = R.Lam / gcd_u(R.Lam, (u32)R.r[s]) * (u32)R.r[s];
+    R.g = gcd_u(R.g, (u32)R.r[s]);
   }
   // in flight per replica, forward round offsets, link slots (one per phase k mod lcm(r_s, r_{s+1}))
-  u64 tf[RR_LINKS], tb[RR_LINKS];
-  {
-    int R = 0;
-    for (int s = S - 1; s >= 0; --s) R += r[s], D[s] = ((R + r[s] - 1) / r[s]) * r[s];
-    for (int s = 1; s < S; ++s) D[s] = D[s] < D[s - 1] ? D[s] : D[s - 1];
-    int off = 0;
-    for (int s = 0; s < S - 1; ++s) {
-      lc[s] = r[s] / (int)gcd_u((u32)r[s], (u32)r[s + 1]) * r[s + 1];
-      lo[s] = off;
-      const int eb = p.cut(s);
-      for (int k = 0; k < lc[s]; ++k) {
-        const int u = (wl[s] >> (4 * (k % r[s]))) & 15, v = (wl[s + 1] >> (4 * (k % r[s + 1]))) & 15;
-        tf[off + k] = xfer(t.O[eb], t.tau[u * TAUW + v]);
-        tb[off + k] = xfer(t.G[eb + 1], t.tau[v * TAUW + u]);
-      }
-      off += lc[s];
-    }
+  int Rs = 0;
+  for (int s = S - 1; s >= 0; --s) {
+    Rs += R.r[s];
+    R.mm[s] = (Rs + R.r[s] - 1) / R.r[s];
+    R.D[s] = R.mm[s] * R.r[s];
   }
-  // schedule state
+  for (int s = 1; s < S; ++s) R.D[s] = R.D[s] < R.D[s - 1] ? R.D[s] : R.D[s - 1];
+  R.negtok = 0;
+  for (int s = 0; s < S; ++s) {
+    const int nt = ((R.mm[s] - 1) * R.r[s]) / (int)R.Lam + 1;
+    R.negtok = nt > R.negtok ? nt : R.negtok;
+  }
+  u64 dsum = 0;
+  for (int s = 0; s < S; ++s)
+    for (int i = 0; i < R.r[s]; ++i) {
+      const int w = (R.wl[s] >> (4 * i)) & 15;
+      dsum += (R.Fw[w] + R.Bw[w]) * (R.Lam / (u32)R.r[s]);
+    }
+  int off = 0;
+  for (int s = 0; s < S - 1; ++s) {
+    R.lc[s] = R.r[s] / (int)gcd_u((u32)R.r[s], (u32)R.r[s + 1]) * R.r[s + 1];
+    R.lo[s] = off;
+    const int eb = p.cut(s);
+    for (int k = 0; k < R.lc[s]; ++k) {
+      const int u = (R.wl[s] >> (4 * (k % R.r[s]))) & 15, v = (R.wl[s + 1] >> (4 * (k % R.r[s + 1]))) & 15;
+      R.tf[off + k] = xfer(t.O[eb], t.tau[u * TAUW + v]);
+      R.tb[off + k] = xfer(t.G[eb + 1], t.tau[v * TAUW + u]);
+      dsum += (R.tf[off + k] + R.tb[off + k]) * (R.Lam / (u32)R.lc[s]);
+    }
+    off += R.lc[s];
+  }
+  R.dsum = dsum;
+}
+
+// S = 1: no boundary; each replica runs F, B, F, B, ... on its own mini-batches (one in every r)
+__device__ __forceinline__ u64 rr_single_stage(const RRSetup &R) {
+  u64 T = 0;
+  for (int i = 0; i < R.r[0]; ++i) {
+    const int w = (R.wl[0] >> (4 * i)) & 15;
+    T = umax(T, (R.Fw[w] + R.Bw[w] + R.r[0] - 1) / (u64)R.r[0]);
+  }
+  return T;
+}
+
+// A lower bound on ceil(lambda_compute) from single-resource cycles: a replica of stage s runs F + B
+// of one in every r_s mini-batches, a link slot of boundary s carries one in every lcm(r_s, r_{s+1}).
+__device__ __forceinline__ u64 rr_lower(const RRSetup &R) {
+  u64 lb = 0;
+  for (int s = 0; s < R.S; ++s)
+    for (int i = 0; i < R.r[s]; ++i) {
+      const int w = (R.wl[s] >> (4 * i)) & 15;
+      lb = umax(lb, (R.Fw[w] + R.Bw[w] + R.r[s] - 1) / (u64)R.r[s]);
+    }
+  for (int s = 0; s < R.S - 1; ++s)
+    for (int k = 0; k < R.lc[s]; ++k) {
+      const int q = R.lo[s] + k;
+      lb = umax(lb, (umax(R.tf[q], R.tb[q]) + R.lc[s] - 1) / (u64)R.lc[s]);
+    }
+  return lb;
+}
+
+enum { RR_MET = 0, RR_BUDGET = 1, RR_PRUNED = 2 };
+// The recurrence for up to `cap` rounds (S >= 2). RR_MET: t_lo = t_hi = ceil(lambda_compute), the
+// growth bounds met; RR_BUDGET: the bracket t_lo <= ceil(lambda_compute) <= t_hi after the budget;
+// RR_PRUNED: t_lo > prune (a search candidate that cannot win). *rounds_out (optional): rounds run.
+static __device__ __noinline__ int rr_sim(const RRSetup &R, u32 cap, u64 prune, u64 &t_lo, u64 &t_hi,
+                                          u32 *rounds_out) {
+  const int S = R.S;
+  const u32 Lam = R.Lam, g = R.g;
+  // absolute times (no rebasing: < 2^58 within the round cap for a state bound below 2^45, checked by
+  // the host)
   u64 wf[MAXN], lff[RR_LINKS], lfb[RR_LINKS], fdr[MAXS - 1][RR_RING];
   for (int w = 0; w < MAXN; ++w) wf[w] = 0;
   for (int q = 0; q < RR_LINKS; ++q) lff[q] = lfb[q] = 0;
-  long long j = -(long long)D[0];  // the first round with an op: F_0(0)
+  long long j = -(long long)R.D[0];  // the first round with an op: F_0(0)
   // phases of the next op of every stage (mini-batch mod r_s, mod lcm of its boundary), advanced by
   // one per round once the stage's mini-batch index is >= 0 (no 64-bit modulo in the recurrence)
   int bph[MAXS], bl[MAXS], fph[MAXS], fl[MAXS];
   for (int s = 0; s < S; ++s) bph[s] = bl[s] = fph[s] = fl[s] = 0;
-  auto step = [](int &ph, int m) { ph = (ph + 1 == m) ? 0 : ph + 1; };
-  auto round = [&]() {
-    u64 bd = 0;
-    if (j >= 0) {
-      for (int s = S - 1; s >= 0; --s) {  // B_s(j), backward boundary s-1 of mini-batch j
-        const int w = (wl[s] >> (4 * bph[s])) & 15;
-        step(bph[s], r[s]);
-        const u64 end = umax(wf[w], s == S - 1 ? 0ull : bd) + Bw[w];
+  // one block = Lam rounds; round j: B_s(j) for s descending (with the backward transfer of boundary
+  // s - 1), then F_s(j + D_s) for s ascending (with the forward transfer of boundary s)
+  auto block = [&]() {
+    for (u32 q = 0; q < Lam; ++q, ++j) {
+      u64 bd = 0;
+      if (j >= 0) {
+        for (int s = S - 1; s >= 0; --s) {
+          const int w = (R.wl[s] >> (4 * bph[s])) & 15;
+          bph[s] = bph[s] + 1 == R.r[s] ? 0 : bph[s] + 1;
+          const u64 end = umax(wf[w], bd) + R.Bw[w];
+          wf[w] = end;
+          if (s > 0) {
+            const int ql = R.lo[s - 1] + bl[s];
+            bl[s] = bl[s] + 1 == R.lc[s - 1] ? 0 : bl[s] + 1;
+            bd = umax(end, lfb[ql]) + R.tb[ql];
+            lfb[ql] = bd;
+          }
+        }
+      }
+      for (int s = 0; s < S; ++s) {
+        const long long k = j + R.D[s];
+        if (k < 0) continue;
+        const int w = (R.wl[s] >> (4 * fph[s])) & 15;
+        fph[s] = fph[s] + 1 == R.r[s] ? 0 : fph[s] + 1;
+        const u64 in = s == 0 ? 0ull : fdr[s - 1][k & (RR_RING - 1)];
+        const u64 end = umax(wf[w], in) + R.Fw[w];
         wf[w] = end;
-        if (s > 0) {
-          const int q = lo[s - 1] + bl[s];
-          step(bl[s], lc[s - 1]);
-          const u64 fin = umax(end, lfb[q]) + tb[q];
-          lfb[q] = fin;
-          bd = fin;
+        if (s < S - 1) {
+          const int ql = R.lo[s] + fl[s];
+          fl[s] = fl[s] + 1 == R.lc[s] ? 0 : fl[s] + 1;
+          const u64 fd = umax(end, lff[ql]) + R.tf[ql];
+          lff[ql] = fd;
+          fdr[s][k & (RR_RING - 1)] = fd;
         }
       }
     }
-    for (int s = 0; s < S; ++s) {  // F_s(j + D_s), forward boundary s of that mini-batch
-      const long long k = j + D[s];
-      if (k < 0) continue;
-      const int w = (wl[s] >> (4 * fph[s])) & 15;
-      step(fph[s], r[s]);
-      const u64 end = umax(wf[w], s == 0 ? 0ull : fdr[s - 1][k & (RR_RING - 1)]) + Fw[w];
-      wf[w] = end;
-      if (s < S - 1) {
-        const int q = lo[s] + fl[s];
-        step(fl[s], lc[s]);
-        const u64 fin = umax(end, lff[q]) + tf[q];
-        lff[q] = fin;
-        fdr[s][k & (RR_RING - 1)] = fin;
-      }
-    }
-    ++j;
   };
-  // the live state at a block boundary (j = the next round): per class c = k mod g, its minimum is
-  // subtracted (rebase) and added to off[c]
-  u64 off[MAXN], tw[MAXN], tlf[RR_LINKS], tlb[RR_LINKS], tfd[MAXS - 1][RR_RING];
-  auto rebase = [&]() {
-    u64 mn[MAXN];
-    for (u32 c = 0; c < g; ++c) mn[c] = U64MAX;
-    for (int s = 0; s < S; ++s)
-      for (int i = 0; i < r[s]; ++i) {
-        const int w = (wl[s] >> (4 * i)) & 15;
-        mn[i % g] = umin(mn[i % g], wf[w]);
-      }
-    for (int s = 0; s < S - 1; ++s)
-      for (int k = 0; k < lc[s]; ++k) {
-        mn[k % g] = umin(mn[k % g], umin(lff[lo[s] + k], lfb[lo[s] + k]));
-      }
-    for (int s = 0; s < S - 1; ++s)  // pending forward transfers of boundary s: k in (j-1+D_{s+1}, j-1+D_s]
-      for (long long k = j + D[s + 1]; k < j + D[s]; ++k)
-        if (k >= 0) mn[(u32)(k % g)] = umin(mn[(u32)(k % g)], fdr[s][k & (RR_RING - 1)]);
-    for (u32 c = 0; c < g; ++c) off[c] += mn[c];
-    for (int s = 0; s < S; ++s)
-      for (int i = 0; i < r[s]; ++i) {
-        const int w = (wl[s] >> (4 * i)) & 15;
-        wf[w] -= mn[i % g];
-      }
-    for (int s = 0; s < S - 1; ++s)
-      for (int k = 0; k < lc[s]; ++k) {
-        lff[lo[s] + k] -= mn[k % g];
-        lfb[lo[s] + k] -= mn[k % g];
-      }
-    for (int s = 0; s < S - 1; ++s)
-      for (long long k = j + D[s + 1]; k < j + D[s]; ++k)
-        if (k >= 0) fdr[s][k & (RR_RING - 1)] -= mn[(u32)(k % g)];
-  };
+  // The saved state (Brent's tortoise): worker and link free times and the forward transfers not yet
+  // consumed, in logical order (mini-batch j + D_{s+1} + q).
+  u64 tw[MAXN], tlf[RR_LINKS], tlb[RR_LINKS], tfd[MAXS - 1][RR_RING];
   auto save = [&]() {
     for (int w = 0; w < MAXN; ++w) tw[w] = wf[w];
     for (int q = 0; q < RR_LINKS; ++q) tlf[q] = lff[q], tlb[q] = lfb[q];
-    for (int s = 0; s < S - 1; ++s)  // pending forward transfers in logical order (from j + D_{s+1})
-      for (int q = 0; q < D[s] - D[s + 1]; ++q) {
-        const long long k = j + D[s + 1] + q;
-        tfd[s][q] = k >= 0 ? fdr[s][k & (RR_RING - 1)] : U64MAX;
-      }
-    for (u32 c = 0; c < g; ++c) off[c] = 0;
+    for (int s = 0; s < S - 1; ++s)
+      for (int q = 0; q < R.D[s] - R.D[s + 1]; ++q) tfd[s][q] = fdr[s][(j + R.D[s + 1] + q) & (RR_RING - 1)];
   };
-  auto same = [&]() -> bool {
+  // Growth since the save, lam blocks ago (max-plus): the block map is monotone and additively
+  // homogeneous per class, so if every live component of class c moved by delta_i, class c's rate
+  // lies in [min delta_i, max delta_i] per lam blocks; lambda = max_c rate_c.
+  auto bounds = [&](u64 den) {
+    long long mn[MAXN], mx[MAXN];
+    for (u32 c = 0; c < g; ++c) mn[c] = LLONG_MAX, mx[c] = LLONG_MIN;
     for (int s = 0; s < S; ++s)
-      for (int i = 0; i < r[s]; ++i) {
-        const int w = (wl[s] >> (4 * i)) & 15;
-        if (wf[w] != tw[w]) return false;
+      for (int i = 0; i < R.r[s]; ++i) {
+        const int w = (R.wl[s] >> (4 * i)) & 15;
+        const long long d = (long long)(wf[w] - tw[w]);
+        const u32 c = (u32)i % g;
+        mn[c] = d < mn[c] ? d : mn[c];
+        mx[c] = d > mx[c] ? d : mx[c];
       }
     for (int s = 0; s < S - 1; ++s)
-      for (int k = 0; k < lc[s]; ++k)
-        if (lff[lo[s] + k] != tlf[lo[s] + k] || lfb[lo[s] + k] != tlb[lo[s] + k]) return false;
-    for (int s = 0; s < S - 1; ++s)
-      for (int q = 0; q < D[s] - D[s + 1]; ++q) {
-        const long long k = j + D[s + 1] + q;
-        if ((k >= 0 ? fdr[s][k & (RR_RING - 1)] : U64MAX) != tfd[s][q]) return false;
+      for (int k = 0; k < R.lc[s]; ++k) {
+        const int ql = R.lo[s] + k;
+        const long long d1 = (long long)(lff[ql] - tlf[ql]), d2 = (long long)(lfb[ql] - tlb[ql]);
+        const u32 c = (u32)k % g;
+        mn[c] = d1 < mn[c] ? d1 : mn[c];
+        mx[c] = d1 > mx[c] ? d1 : mx[c];
+        mn[c] = d2 < mn[c] ? d2 : mn[c];
+        mx[c] = d2 > mx[c] ? d2 : mx[c];
       }
-    return true;
+    for (int s = 0; s < S - 1; ++s)
+      for (int q = 0; q < R.D[s] - R.D[s + 1]; ++q) {
+        const long long k = j + R.D[s + 1] + q;
+        const long long d = (long long)(fdr[s][k & (RR_RING - 1)] - tfd[s][q]);
+        const u32 c = (u32)(k % g);
+        mn[c] = d < mn[c] ? d : mn[c];
+        mx[c] = d > mx[c] ? d : mx[c];
+      }
+    long long lo = 0, hi = 0;
+    for (u32 c = 0; c < g; ++c) lo = mn[c] > lo ? mn[c] : lo, hi = mx[c] > hi ? mx[c] : hi;
+    t_lo = ((u64)lo + den - 1) / den;
+    t_hi = ((u64)hi + den - 1) / den;
   };
-  auto block = [&]() {
-    for (u32 q = 0; q < Lam; ++q) round();
-    rebase();
-  };
-  for (u32 c = 0; c < MAXN; ++c) off[c] = 0;
-  // Brent: the tortoise jumps to the hare at powers of two; lam = blocks since the tortoise
-  block();
+  // Brent: the tortoise jumps to the hare at powers of two; lam = blocks since the tortoise. The
+  // first save waits for every stage to have started (j >= 0): from there the block map is the same
+  // every block.
+  u32 rounds = 0;
+  do {
+    block();
+    rounds += Lam;
+  } while (j < 0);
   save();
-  block();
-  u32 power = 1, lam = 1, rounds = 2 * Lam;
-  bool settled = true;
-  while (!same()) {
+  u32 power = 1, lam = 0;
+  int rc = RR_BUDGET;
+  for (;;) {
+    block();
+    ++lam;
+    rounds += Lam;
+    bounds((u64)lam * Lam);
+    if (t_lo == t_hi) {
+      rc = RR_MET;
+      break;
+    }
+    if (t_lo > prune) {
+      rc = RR_PRUNED;
+      break;
+    }
+    if (rounds > cap) break;
     if (power == lam) {
       save();
       power *= 2;
       lam = 0;
     }
-    block();
-    ++lam;
-    rounds += Lam;
-    if (rounds > RR_SIM_ROUNDS) {
-      settled = false;
-      break;
-    }
   }
-  const u64 den = (u64)lam * Lam;
-  u64 T = 0;
-  for (u32 c = 0; c < g; ++c) T = umax(T, (off[c] + den - 1) / den);
-  if (!settled) {
-    int mm[MAXS];
-    {
-      int R = 0;
-      for (int s = S - 1; s >= 0; --s) R += r[s], mm[s] = (R + r[s] - 1) / r[s];
-    }
-    auto dur = [&](int kind, int s, int ph) -> u64 {
-      if (kind <= 1) {
-        const int w = (wl[s] >> (4 * (ph % r[s]))) & 15;
-        return kind == 0 ? Fw[w] : Bw[w];
+  if (rounds_out) *rounds_out = rounds;
+  return rc;
+}
+
+// Node (kind, s, phase p) of the one-period event graph: F_s, B_s, forward and backward transfer of
+// boundary s, for the mini-batches k = p (mod Lam); V = 4 S Lam (the transfer nodes of s = S - 1 are
+// unused). Its duration, and the relaxation of its (at most two) predecessors at theta, where an
+// edge's weight is -theta Lam (its token count: periods between the two mini-batches).
+__device__ __forceinline__ u64 rr_dur(const RRSetup &R, int kind, int s, int ph) {
+  if (kind <= 1) {
+    const int w = (R.wl[s] >> (4 * (ph % R.r[s]))) & 15;
+    return kind == 0 ? R.Fw[w] : R.Bw[w];
+  }
+  const int q = R.lo[s] + ph % R.lc[s];
+  return kind == 2 ? R.tf[q] : R.tb[q];
+}
+template <typename Dist>
+__device__ __forceinline__ long long rr_relax(const RRSetup &R, const Dist &dist, int kind, int s, int p,
+                                              long long dv, long long th) {
+  const int S = R.S;
+  const long long Lam = R.Lam, K0 = 64ll * Lam;  // a period index far from the start
+  const long long k = K0 + p;
+  auto at = [&](int kk, int ss, long long ku) {
+    const long long tok = k / Lam - ku / Lam;
+    return dist[(kk * S + ss) * (int)Lam + (int)(ku % Lam)] + dv - th * Lam * tok;
+  };
+  long long best = LLONG_MIN;
+  auto take = [&](long long c) { best = c > best ? c : best; };
+  if (kind == 0) {
+    take(at(1, s, k - (long long)R.mm[s] * R.r[s]));  // worker order: after B(k - m r)
+    if (s > 0) take(at(2, s - 1, k));                   // forward transfer of boundary s - 1
+  } else if (kind == 1) {
+    take(at(0, s, k + (long long)(R.mm[s] - 1) * R.r[s]));  // worker order: after F(k + (m - 1) r)
+    if (s < S - 1) take(at(3, s, k));                        // backward transfer of boundary s
+  } else if (kind == 2) {
+    take(at(0, s, k));            // after F_s(k)
+    take(at(2, s, k - R.lc[s]));  // FIFO on its link
+  } else {
+    take(at(1, s + 1, k));  // after B_{s+1}(k)
+    take(at(3, s, k - R.lc[s]));
+  }
+  return best;
+}
+
+// Positive cycle at theta (single thread, Gauss-Seidel passes in node order).
+// A simple path weighs at most the sum of all node durations plus theta Lam negtok per edge (the
+// worker-order edges B_s(k) <- F_s(k + (m - 1) r) can carry negative tokens); a larger distance
+// proves a positive cycle.
+__device__ __forceinline__ long long rr_path_cap(const RRSetup &R, long long th) {
+  const long long V = 4ll * R.S * R.Lam;
+  return (long long)R.dsum + V * (th > 0 ? th : 0) * (long long)R.Lam * R.negtok;
+}
+__device__ __forceinline__ bool rr_positive(const RRSetup &R, long long th, long long *dist) {
+  const int S = R.S, Lam = (int)R.Lam, V = 4 * S * Lam;
+  const long long cap = rr_path_cap(R, th);
+  for (int v = 0; v < V; ++v) dist[v] = 0;
+  for (int pass = 0; pass <= V; ++pass) {
+    bool changed = false;
+    for (int v = 0; v < V; ++v) {
+      const int kind = v / (S * Lam), s = (v / Lam) % S, p = v % Lam;
+      if (kind >= 2 && s == S - 1) continue;
+      const long long c = rr_relax(R, dist, kind, s, p, (long long)rr_dur(R, kind, s, p), th);
+      if (c > dist[v]) {
+        dist[v] = c;
+        changed = true;
+        if (c > cap) return true;  // heavier than any simple path: a positive cycle
       }
-      const int q = lo[s] + ph % lc[s];
-      return kind == 2 ? tf[q] : tb[q];
-    };
-    T = rr_ceil_bf(S, Lam, r, mm, lc, dur, (long long)T);
+    }
+    if (!changed) return false;
   }
-  return umax(T, Tsync);
+  return true;
+}
+
+// Positive cycle at theta, one warp (every lane calls it; dist: V words of the warp's shared memory).
+// Lane l relaxes nodes l, l + 32, ... in place: a value read mid-pass is the old or the new one, both
+// lower bounds of the pass's result, so V + 1 passes still decide (chaotic Bellman-Ford).
+__device__ __forceinline__ bool rr_positive_warp(const RRSetup &R, long long th, volatile long long *dist) {
+  const int S = R.S, Lam = (int)R.Lam, V = 4 * S * Lam, lane = threadIdx.x & 31;
+  const long long cap = rr_path_cap(R, th);
+  for (int v = lane; v < V; v += 32) dist[v] = 0;
+  __syncwarp();
+  for (int pass = 0; pass <= V; ++pass) {
+    bool changed = false, big = false;
+    for (int v = lane; v < V; v += 32) {
+      const int kind = v / (S * Lam), s = (v / Lam) % S, p = v % Lam;
+      if (kind >= 2 && s == S - 1) continue;
+      const long long c = rr_relax(R, dist, kind, s, p, (long long)rr_dur(R, kind, s, p), th);
+      if (c > dist[v]) {
+        dist[v] = c;
+        changed = true;
+        big |= c > cap;
+      }
+    }
+    __syncwarp();
+    if (__any_sync(0xffffffffu, big)) return true;
+    if (!__any_sync(0xffffffffu, changed)) return false;
+  }
+  return true;
+}
+
+// ceil(lambda_compute) inside the bracket t_lo <= T <= t_hi the simulation's bounds give:
+// positive(t_lo - 1) holds and positive(t_hi) does not, so a binary search on theta decides it.
+__device__ __forceinline__ u64 rr_ceil_bf(const RRSetup &R, u64 t_lo, u64 t_hi) {
+  long long dist[RR_BF_NODES];
+  long long lo = (long long)t_lo - 1, hi = (long long)t_hi;
+  while (hi - lo > 1) {
+    const long long mid = lo + (hi - lo) / 2;
+    if (rr_positive(R, mid, dist)) lo = mid;
+    else hi = mid;
+  }
+  return (u64)hi;
+}
+__device__ __forceinline__ u64 rr_ceil_bf_warp(const RRSetup &R, u64 t_lo, u64 t_hi, volatile long long *dist) {
+  long long lo = (long long)t_lo - 1, hi = (long long)t_hi;
+  while (hi - lo > 1) {
+    const long long mid = lo + (hi - lo) / 2;
+    if (rr_positive_warp(R, mid, dist)) lo = mid;
+    else hi = mid;
+  }
+  return (u64)hi;
+}
+
+// T_ns of a validated 16-byte partition under round-robin replicas, in the thread.
+static __device__ __noinline__ u64 rr_time(const SmemTab &t, int S, const P8 &p, int sync) {
+  RRSetup R;
+  rr_setup(t, S, p, sync, R);
+  if (S == 1) return umax(rr_single_stage(R), R.Tsync);
+  u64 t_lo, t_hi;
+  u32 rounds;
+  const bool met = rr_sim(R, RR_SIM_ROUNDS, U64MAX, t_lo, t_hi, &rounds) == RR_MET;
+#if RR_STATS  // diagnostics (tools/rr_stats.py): rounds simulated, bit 32 = bounds not met in the budget
+  return rounds | (met ? 0ull : 1ull << 32);
+#endif
+  if (met || R.Tsync >= t_hi) return umax(t_lo, R.Tsync);
+  return umax(rr_ceil_bf(R, t_lo, t_hi), R.Tsync);
 }
 
 }  // namespace ap

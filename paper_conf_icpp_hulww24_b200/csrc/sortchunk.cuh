@@ -70,7 +70,9 @@ struct NoStore {
   template <typename Rec>
   __device__ void operator()(const Rec &, u64) const {}
 };
-template <int NW, typename Rec, typename F, typename G = NoStore>
+// DYNAMIC forces the chunk counter for 16-byte records too (scoring costs that vary by orders of
+// magnitude between records: round-robin replicas).
+template <int NW, typename Rec, bool DYNAMIC = false, typename F, typename G = NoStore>
 __device__ __forceinline__ void for_each_sorted_warp(const Rec *__restrict__ recs, u64 count, u32 *counter, F &&f,
                                                      G store = G()) {
   constexpr int PER = WarpSort<NW, Rec>::PER, CH = WarpSort<NW, Rec>::CH;
@@ -84,7 +86,7 @@ __device__ __forceinline__ void for_each_sorted_warp(const Rec *__restrict__ rec
   u32 *h = hist[w];
   // static split: warp gw of W takes records [count gw / W, count (gw + 1) / W), in chunks of CH
   // (the same number of records per warp); dynamic: chunks of CH from the global counter
-  constexpr bool STATIC = EvalStatic<Rec>::value;
+  constexpr bool STATIC = EvalStatic<Rec>::value && !DYNAMIC;
   const u64 W = (u64)gridDim.x * NW, gw = (u64)blockIdx.x * NW + w;
   const u64 r1 = STATIC ? count * (gw + 1) / W : count;
   u64 base = STATIC ? count * gw / W : 0;

@@ -329,11 +329,15 @@ class Engine:
     def int_path(self) -> int:
         return int(lib.autopipe_int_path(self._h))
 
-    def set_search_options(self, split: bool = False, no_r1: bool = False) -> None:
-        """Kernel selection of later searches (autopipe_set_search_options): split=True always uses the
-        per-S split (r = 1 sweep + threshold walk), even for ranges the dense launch would take;
-        no_r1=True sends the r = 1 blocks through the threshold walk too."""
-        self._check(lib.autopipe_set_search_options(self._h, (1 if split else 0) | (2 if no_r1 else 0)))
+    def set_search_options(self, split: bool = False, no_r1: bool = False, rr_defer_all: bool = False,
+                           rr_no_defer: bool = False) -> None:
+        """Kernel selection of later calls (autopipe_set_search_options; never changes a result):
+        split=True always uses the per-S split (r = 1 sweep + threshold walk), even for ranges the dense
+        launch would take; no_r1=True sends the r = 1 blocks through the threshold walk too;
+        rr_defer_all / rr_no_defer: round-robin evaluations defer (nearly) every record to the
+        warp-per-record drain kernel / none."""
+        self._check(lib.autopipe_set_search_options(
+            self._h, (1 if split else 0) | (2 if no_r1 else 0) | (4 if rr_defer_all else 0) | (8 if rr_no_defer else 0)))
 
     def set_timing(self, enable: bool = True) -> None:
         self._check(lib.autopipe_set_timing(self._h, 1 if enable else 0))

@@ -34,10 +34,18 @@ def gpu_eval(eng, recs):
     return [int(x) for x in out]
 
 
+DEFER_MODES = {"default": {}, "defer_all": {"rr_defer_all": True}, "no_defer": {"rr_no_defer": True}}
+
+
+@pytest.mark.parametrize("mode", list(DEFER_MODES))
 @pytest.mark.parametrize("seed", range(6))
 @pytest.mark.parametrize("sync", [0, 1])
-def test_random_records(eng, seed, sync):
+def test_random_records(eng, seed, sync, mode):
+    """Every record three ways: the default (simulation, deferral of the slow ones to the warp-per-
+    record drain kernel), defer_all (a one-round budget: nearly every record is finished by the
+    drain's Bellman-Ford inside the bracket of its first block) and no_defer (in the thread)."""
     rng = np.random.default_rng(1100 + seed)
+    eng.set_search_options(**DEFER_MODES[mode])
     for _ in range(3):
         L = int(rng.integers(2, 14))
         N = int(rng.integers(1, 9))
@@ -49,6 +57,7 @@ def test_random_records(eng, seed, sync):
         recs += [bytes([3, 5, 1] + [0xFF] * 13)]                      # an invalid record (cuts)
         assert gpu_eval(eng, recs) == rr_many(prof, st, recs, sync)
     eng.set_schedule()
+    eng.set_search_options()
 
 
 def test_r1_records_equal_pipedream(eng):
@@ -71,18 +80,22 @@ def test_r1_records_equal_pipedream(eng):
     assert got == gpu_eval(eng, recs) == score_many(prof, st, recs)
 
 
-def test_resnet50_rollout_state(eng):
+@pytest.mark.parametrize("mode", list(DEFER_MODES))
+def test_resnet50_rollout_state(eng, mode):
     prof = W.resnet50()
     st = W.rollout_state(prof, 0)
     eng.load(prof, st)
     eng.set_schedule(SCHED_RR)
+    eng.set_search_options(**DEFER_MODES[mode])
     recs = [bytes(r) for r in W.sample_records(prof.L, st.N, 1500, 31)]
     assert gpu_eval(eng, recs) == rr_many(prof, st, recs)
     eng.set_schedule()
+    eng.set_search_options()
 
 
+@pytest.mark.parametrize("mode", list(DEFER_MODES))
 @pytest.mark.parametrize("seed", range(4))
-def test_small_space_search(eng, seed):
+def test_small_space_search(eng, seed, mode):
     rng = np.random.default_rng(1300 + seed)
     L = int(rng.integers(3, 8))
     N = int(rng.integers(2, 6))
@@ -95,7 +108,7 @@ def test_small_space_search(eng, seed):
     m = min(ts)
     eng.set_schedule(SCHED_RR)
     for split in (False, True):
-        eng.set_search_options(split)
+        eng.set_search_options(split, **DEFER_MODES[mode])
         r = eng.search_optimum(1, smax)
         assert (r.time_ns, r.index, r.evaluated) == (m, ts.index(m), count(L, N, 1, smax))
     eng.set_search_options(False)

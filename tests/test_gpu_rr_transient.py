@@ -14,13 +14,15 @@ pytestmark = pytest.mark.gpu
 REC = W.encode(3, [15, 29], [1, W.IDLE, 2, 1, 0])
 
 
-def test_long_transient_record():
+@pytest.mark.parametrize("mode", [{}, {"rr_defer_all": True}, {"rr_no_defer": True}])
+def test_long_transient_record(mode):
     from paper_conf_icpp_hulww24_b200 import Engine, as_u64
     prof = W.resnet50()
     st = W.rollout_state(prof, 0)
     eng = Engine(0)
     eng.load(prof, st)
     eng.set_schedule(4)
+    eng.set_search_options(**mode)
     got = as_u64(eng.eval_partitions(torch.from_numpy(np.frombuffer(REC, dtype=np.uint8).reshape(1, 16).copy())))
     eng.close()
     assert int(got[0]) == RR.score_record(prof, st, REC) == 591221519
