@@ -93,11 +93,14 @@ __device__ __forceinline__ void unrank_global_smem(const SearchSpace &sp, u64 id
 // NARROW (PipeDream, dense launches of a host-classified state): the 32-bit closed form of k_eval
 template <int NT, bool P32, int MODE, typename P, bool NARROW = false>
 __global__ void __launch_bounds__(NT, GEN_MINB) k_search_generic(DevTables g, SearchSpace sp, u64 begin, u64 end,
-                                                                 u64 per_thread, BlockOut *out, ModelP m, int gate) {
+                                                                 u64 per_thread, BlockOut *out, ModelP m, int gate,
+                                                                 u64 *gbest = nullptr) {
   if (gate >= 0 && state_gated_out(g, gate, out)) return;  // see state_gated_out
   typedef SpaceT<P> SP;
   typedef typename SP::PK PK;
   constexpr int BK = SP::BK;
+  // flushed schedules and Chimera: candidates decided by a lower bound against the best so far
+  constexpr bool PRUNED = MODE == SCHED_GPIPE || MODE == SCHED_DAPPLE || MODE == SCHED_CHIMERA;
   extern __shared__ u64 sm[];
   // binomial rows n <= L (n = N <= 16 <= L + 1 for the compositions too) after the state tables
   u64 *Bn = sm + smem_words(g.L, g.N, NARROW);
@@ -116,11 +119,21 @@ __global__ void __launch_bounds__(NT, GEN_MINB) k_search_generic(DevTables g, Se
     P p = part_from<P>(sp, S, Rp, cuts);
     for (u64 i = i0; i < i1; ++i) {
       u64 T;
-      if constexpr (NARROW) T = eval_closed_form_n<P32, P>(t, S, p, (int)m.sync);
-      else T = model_time<MODE, P32>(t, S, p, m);
+      if constexpr (NARROW) {
+        T = eval_closed_form_n<P32, P>(t, S, p, (int)m.sync);
+      } else if constexpr (PRUNED) {
+        // a candidate whose lower bound exceeds theta cannot be the lexicographic minimum: theta =
+        // the thread's best - 1 (its later indices lose ties) or the launch's best (the T of a real
+        // candidate: a strictly greater bound loses whatever the index)
+        const u64 theta = umin(bestT - 1, *(volatile u64 *)gbest);
+        T = model_lower<MODE, P>(t, S, p, m) > theta ? U64MAX : model_time<MODE, P32>(t, S, p, m);
+      } else {
+        T = model_time<MODE, P32>(t, S, p, m);
+      }
       if (T < bestT) {  // indices increase along the thread's range: strict < keeps the first
         bestT = T;
         bestI = i;
+        if constexpr (PRUNED) atomicMin((unsigned long long *)gbest, T);
       }
       ++cnt;
       if (i + 1 == i1) break;
@@ -430,12 +443,16 @@ __global__ void __launch_bounds__(NT, DFS_MINB) k_search_dfs(DevTables g, Search
 template <int NT, typename P>
 static void run_search_generic(unsigned nbk, size_t smem, cudaStream_t st, const DevTables &g, const SearchSpace &sp,
                                u64 begin, u64 end, u64 pt, BlockOut *out, const ModelP &m, int path32, void *sched) {
+  // the pruned schedules keep the launch's best T in the first word of their schedule slot
+  u64 *gbest = (u64 *)sched;
+  if (m.sched == SCHED_GPIPE || m.sched == SCHED_DAPPLE || m.sched == SCHED_CHIMERA)
+    cudaMemsetAsync(gbest, 0xFF, sizeof(u64), st);
   switch (m.sched) {
     case SCHED_2BW: k_search_generic<NT, false, SCHED_2BW, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1); break;
-    case SCHED_GPIPE: k_search_generic<NT, false, SCHED_GPIPE, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1); break;
-    case SCHED_DAPPLE: k_search_generic<NT, false, SCHED_DAPPLE, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1); break;
+    case SCHED_GPIPE: k_search_generic<NT, false, SCHED_GPIPE, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1, gbest); break;
+    case SCHED_DAPPLE: k_search_generic<NT, false, SCHED_DAPPLE, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1, gbest); break;
     case SCHED_RR: k_search_generic<NT, false, SCHED_RR, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1); break;
-    case SCHED_CHIMERA: k_search_generic<NT, false, SCHED_CHIMERA, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1); break;
+    case SCHED_CHIMERA: k_search_generic<NT, false, SCHED_CHIMERA, P><<<nbk, NT, smem, st>>>(g, sp, begin, end, pt, out, m, -1, gbest); break;
     default: {  // PipeDream: the threshold walk (64-bit; the state's integer path does not matter)
       DfsSched *ds = (DfsSched *)sched;
       if (path32 >= 0) {

@@ -149,6 +149,58 @@ __device__ __forceinline__ u64 flush_makespan(const SmemTab &t, int S, const P &
   return T;
 }
 
+// A lower bound on T_ns under a flushed schedule (GPipe, DAPPLE) or Chimera, for the pruned searches:
+// GPipe / DAPPLE: worker w of stage s runs its M forwards and M backwards one after another, after
+// micro-batch 0 has crossed stages 0..s-1 (each stage's slowest replica, then the boundary) and before
+// micro-batch M-1's gradient crosses back to stage 0:
+//   T >= sum_{u<s} (maxF_u + dF_u) + M (F_w + B_w) + sum_{u<s} (dB_u + maxB_u);
+// Chimera: worker g runs ceil(M/2) micro-batches of its down stage and floor(M/2) of its up stage.
+// UINT64_MAX for a record the model refuses (Chimera: a replicated stage).
+template <int MODE, typename P>
+__device__ __forceinline__ u64 model_lower(const SmemTab &t, int S, const P &p, const ModelP &m) {
+  constexpr int MN = P::MN;
+  const u64 M = m.M;
+  if constexpr (MODE == SCHED_CHIMERA) {
+    const u64 Md = (M + 1) / 2, Mu = M / 2;
+    u64 lb = 0;
+    for (int g = 0; g < S; ++g) {
+      const u32 mask = p.mask(g);
+      if (__popc(mask) != 1) return U64MAX;
+      const int w = __ffs(mask) - 1, su = S - 1 - g;
+      const int a = (g == 0) ? 0 : p.cut(g - 1) + 1, e = (g == S - 1) ? t.L - 1 : p.cut(g);
+      const int au = (su == 0) ? 0 : p.cut(su - 1) + 1, eu = (su == S - 1) ? t.L - 1 : p.cut(su);
+      const u64 *F = t.PF + w * t.Lp1, *B = t.PB + w * t.Lp1;
+      lb = umax(lb, Md * (F[e + 1] - F[a] + B[e + 1] - B[a]) + Mu * (F[eu + 1] - F[au] + B[eu + 1] - B[au]));
+    }
+    return lb;
+  } else {
+    static_assert(MODE == SCHED_GPIPE || MODE == SCHED_DAPPLE, "flushed schedules and Chimera");
+    u64 lb = 0, pre = 0;  // pre: forward crossing to stage s plus backward crossing from it
+    for (int s = 0; s < S; ++s) {
+      const u32 mask = p.mask(s);
+      const int a = (s == 0) ? 0 : p.cut(s - 1) + 1, e = (s == S - 1) ? t.L - 1 : p.cut(s);
+      const DivR<MN> dv((u32)__popc(mask), t.dv);
+      u64 mF = 0, mB = 0, work = 0;
+      for (u32 mm = mask; mm; mm &= mm - 1) {
+        const int w = __ffs(mm) - 1;
+        const u64 Fw = dv.ceil(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a]);
+        u64 Bw = dv.ceil(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a]);
+        if (MODE == SCHED_GPIPE && m.recompute) Bw += Fw;
+        mF = umax(mF, Fw);
+        mB = umax(mB, Bw);
+        work = umax(work, Fw + Bw);
+      }
+      lb = umax(lb, pre + M * work);
+      if (s < S - 1) {
+        u64 cf, cb;
+        boundary_cf_cb<MN>(t, p.cut(s), mask, p.mask(s + 1), cf, cb);
+        pre += mF + cf + cb + mB;
+      }
+    }
+    return lb;
+  }
+}
+
 // T_ns of a validated partition under the model (rows f3, f4): MODE = the schedule, fixed per kernel.
 // Round-robin replicas (SCHED_RR) are defined for 16-byte records (the host refuses wide ones).
 template <int MODE, bool P32, typename P>
