@@ -70,7 +70,9 @@ def main():
     prof = W.bert24()
     eng.load(prof, W.trace_c3(prof)[0])
     for k, model in (("rr", (L_.SCHED_PIPEDREAM_RR, L_.SYNC_RING, 1, False)),
-                     ("chimera", (L_.SCHED_CHIMERA, L_.SYNC_RING, 8, False))):
+                     ("chimera", (L_.SCHED_CHIMERA, L_.SYNC_RING, 8, False)),
+                     ("gpipe", (L_.SCHED_GPIPE, L_.SYNC_RING, 8, True)),
+                     ("dapple", (L_.SCHED_DAPPLE, L_.SYNC_RING, 8, False))):
         if k in which:
             eng.set_schedule(*model)
             ms, r = timed(lambda: eng.search_optimum(1, 8), reps=2)
