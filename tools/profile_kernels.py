@@ -3,7 +3,8 @@
 C4a search (k_search_r1 u32 path), C4b search (u64 path), the 1M-record C5 ResNet-50 rollout and eval
 (k_eval, narrow path), switch rewards (k_switch, f2), DAPPLE M = 8 eval (f3), the 10-GPU ResNet-50
 testbed search (k_search_dfs, f4 wide), C2 VGG-16 (dense k_search_generic), round-robin replicas
-(f4) and Chimera (f3) on 64k records."""
+(f4) on the 1M C5 records, Chimera (f3) on 64k records, and the BERT-24 round-robin search
+(k_search_rr and its drain)."""
 import os
 import sys
 
@@ -48,11 +49,16 @@ eng.load(W.vgg16(), W.vgg_state())
 r = eng.search_optimum(1, 8)
 print("vgg", r.time_ns, r.index)
 eng.load(prof, st)
-small = recs[: 1 << 16].contiguous()
 eng.set_schedule(L_.SCHED_PIPEDREAM_RR)
-eng.eval_partitions(small)
+eng.eval_partitions(recs)  # round-robin replicas: k_eval + the drain of its deferred records
+small = recs[: 1 << 16].contiguous()
 eng.set_schedule(L_.SCHED_CHIMERA, 0, 8)
 eng.eval_partitions(small)
 torch.cuda.synchronize()
+bert = W.bert24()
+eng.load(bert, W.trace_c3(bert)[0])
+eng.set_schedule(L_.SCHED_PIPEDREAM_RR)
+r = eng.search_optimum(1, 8)  # k_search_rr + k_rr_drain_search
+print("rr search", r.time_ns, r.index)
 eng.set_schedule()
 print("done")
