@@ -37,8 +37,8 @@ namespace ap {
 #endif
 constexpr u32 RR_SIM_ROUNDS = 4096;    // in-thread budget (search; eval when the deferral queue is full)
 constexpr int RR_BF_NODES = 160;       // 4 S Lam <= 144 nodes for sum r <= 8
-constexpr int RR_LINKS = 32;           // sum over boundaries of lcm(r_s, r_{s+1}) for N <= 8
-constexpr int RR_RING = 16;            // pending forward transfers per boundary (D_0 <= 15)
+constexpr int RR_LINKS = 16;           // max over sum r <= 8 of sum_s lcm(r_s, r_{s+1}) (r = 1, 4, 3)
+constexpr int RR_PEND = 24;            // pending forward transfers: sum_s (D_s - D_{s+1} + 1) <= 15 + 7
 
 __device__ __forceinline__ u32 gcd_u(u32 a, u32 b) {
   while (b) {
@@ -147,28 +147,35 @@ __device__ __forceinline__ u64 rr_lower(const RRSetup &R) {
   return lb;
 }
 
-enum { RR_MET = 0, RR_BUDGET = 1, RR_PRUNED = 2 };
-// The recurrence for up to `cap` rounds (S >= 2). RR_MET: t_lo = t_hi = ceil(lambda_compute), the
-// growth bounds met; RR_BUDGET: the bracket t_lo <= ceil(lambda_compute) <= t_hi after the budget;
-// RR_PRUNED: t_lo > prune (a search candidate that cannot win). *rounds_out (optional): rounds run.
-static __device__ __noinline__ int rr_sim(const RRSetup &R, u32 cap, u64 prune, u64 &t_lo, u64 &t_hi,
-                                          u32 *rounds_out) {
-  const int S = R.S;
-  const u32 Lam = R.Lam, g = R.g;
+enum { RR_MET = 0, RR_BUDGET = 1, RR_PRUNED = 2, RR_CONT = 3 };
+// The recurrence as a resumable state machine (S >= 2): init() runs the warm-up blocks (until every
+// stage has started, j >= 0) and saves the tortoise; each step() runs one block of Lam rounds and
+// decides: RR_MET: t_lo = t_hi = ceil(lambda_compute), the growth bounds met; RR_PRUNED: t_lo > prune
+// (a search candidate that cannot win); RR_BUDGET: more than `cap` rounds, t_lo <= ceil(lambda_compute)
+// <= t_hi; RR_CONT: not decided yet. A lane of the eval kernel resumes it block by block, so a lane
+// whose record is decided can take the warp's next record (k_eval.cu).
+struct RRSim {
   // absolute times (no rebasing: < 2^58 within the round cap for a state bound below 2^45, checked by
   // the host)
-  u64 wf[MAXN], lff[RR_LINKS], lfb[RR_LINKS], fdr[MAXS - 1][RR_RING];
-  for (int w = 0; w < MAXN; ++w) wf[w] = 0;
-  for (int q = 0; q < RR_LINKS; ++q) lff[q] = lfb[q] = 0;
-  long long j = -(long long)R.D[0];  // the first round with an op: F_0(0)
+  // forward transfers not yet consumed: boundary s keeps a FIFO of D_s - D_{s+1} + 1 slots at
+  // fo[s] in fdr (F_s(k) writes the slot F_{s+1}(k) reads D_s - D_{s+1} rounds later; the extra slot
+  // lets the write of round j precede that round's read), write / read positions fw[s] / fr[s]
+  u64 wf[MAXN], lff[RR_LINKS], lfb[RR_LINKS], fdr[RR_PEND];
+  // the saved state (Brent's tortoise): worker and link free times and the pending forward
+  // transfers in logical order (mini-batch j + D_{s+1} + q, boundary s at fo[s])
+  u64 tw[MAXN], tlf[RR_LINKS], tlb[RR_LINKS], tfd[RR_PEND];
+  int fo[MAXS], fw[MAXS], fr[MAXS];
+  long long j;  // the next round
   // phases of the next op of every stage (mini-batch mod r_s, mod lcm of its boundary), advanced by
   // one per round once the stage's mini-batch index is >= 0 (no 64-bit modulo in the recurrence)
   int bph[MAXS], bl[MAXS], fph[MAXS], fl[MAXS];
-  for (int s = 0; s < S; ++s) bph[s] = bl[s] = fph[s] = fl[s] = 0;
+  u32 rounds, power, lam;
+
   // one block = Lam rounds; round j: B_s(j) for s descending (with the backward transfer of boundary
   // s - 1), then F_s(j + D_s) for s ascending (with the forward transfer of boundary s)
-  auto block = [&]() {
-    for (u32 q = 0; q < Lam; ++q, ++j) {
+  __device__ __forceinline__ void block(const RRSetup &R) {
+    const int S = R.S;
+    for (u32 q = 0; q < R.Lam; ++q, ++j) {
       u64 bd = 0;
       if (j >= 0) {
         for (int s = S - 1; s >= 0; --s) {
@@ -189,7 +196,12 @@ static __device__ __noinline__ int rr_sim(const RRSetup &R, u32 cap, u64 prune, 
         if (k < 0) continue;
         const int w = (R.wl[s] >> (4 * fph[s])) & 15;
         fph[s] = fph[s] + 1 == R.r[s] ? 0 : fph[s] + 1;
-        const u64 in = s == 0 ? 0ull : fdr[s - 1][k & (RR_RING - 1)];
+        u64 in = 0;
+        if (s > 0) {
+          const int len = R.D[s - 1] - R.D[s] + 1;
+          in = fdr[fo[s - 1] + fr[s - 1]];
+          fr[s - 1] = fr[s - 1] + 1 == len ? 0 : fr[s - 1] + 1;
+        }
         const u64 end = umax(wf[w], in) + R.Fw[w];
         wf[w] = end;
         if (s < S - 1) {
@@ -197,24 +209,27 @@ static __device__ __noinline__ int rr_sim(const RRSetup &R, u32 cap, u64 prune, 
           fl[s] = fl[s] + 1 == R.lc[s] ? 0 : fl[s] + 1;
           const u64 fd = umax(end, lff[ql]) + R.tf[ql];
           lff[ql] = fd;
-          fdr[s][k & (RR_RING - 1)] = fd;
+          const int len = R.D[s] - R.D[s + 1] + 1;
+          fdr[fo[s] + fw[s]] = fd;
+          fw[s] = fw[s] + 1 == len ? 0 : fw[s] + 1;
         }
       }
     }
-  };
-  // The saved state (Brent's tortoise): worker and link free times and the forward transfers not yet
-  // consumed, in logical order (mini-batch j + D_{s+1} + q).
-  u64 tw[MAXN], tlf[RR_LINKS], tlb[RR_LINKS], tfd[MAXS - 1][RR_RING];
-  auto save = [&]() {
+  }
+  __device__ __forceinline__ void save(const RRSetup &R) {
     for (int w = 0; w < MAXN; ++w) tw[w] = wf[w];
     for (int q = 0; q < RR_LINKS; ++q) tlf[q] = lff[q], tlb[q] = lfb[q];
-    for (int s = 0; s < S - 1; ++s)
-      for (int q = 0; q < R.D[s] - R.D[s + 1]; ++q) tfd[s][q] = fdr[s][(j + R.D[s + 1] + q) & (RR_RING - 1)];
-  };
+    for (int s = 0; s < R.S - 1; ++s) {
+      const int len = R.D[s] - R.D[s + 1] + 1;
+      for (int q = 0, x = fr[s]; q < len - 1; ++q, x = x + 1 == len ? 0 : x + 1) tfd[fo[s] + q] = fdr[fo[s] + x];
+    }
+  }
   // Growth since the save, lam blocks ago (max-plus): the block map is monotone and additively
   // homogeneous per class, so if every live component of class c moved by delta_i, class c's rate
   // lies in [min delta_i, max delta_i] per lam blocks; lambda = max_c rate_c.
-  auto bounds = [&](u64 den) {
+  __device__ __forceinline__ void bounds(const RRSetup &R, u64 den, u64 &t_lo, u64 &t_hi) const {
+    const int S = R.S;
+    const u32 g = R.g;
     long long mn[MAXN], mx[MAXN];
     for (u32 c = 0; c < g; ++c) mn[c] = LLONG_MAX, mx[c] = LLONG_MIN;
     for (int s = 0; s < S; ++s)
@@ -235,51 +250,69 @@ static __device__ __noinline__ int rr_sim(const RRSetup &R, u32 cap, u64 prune, 
         mn[c] = d2 < mn[c] ? d2 : mn[c];
         mx[c] = d2 > mx[c] ? d2 : mx[c];
       }
-    for (int s = 0; s < S - 1; ++s)
-      for (int q = 0; q < R.D[s] - R.D[s + 1]; ++q) {
+    for (int s = 0; s < S - 1; ++s) {
+      const int len = R.D[s] - R.D[s + 1] + 1;
+      for (int q = 0, x = fr[s]; q < len - 1; ++q, x = x + 1 == len ? 0 : x + 1) {
         const long long k = j + R.D[s + 1] + q;
-        const long long d = (long long)(fdr[s][k & (RR_RING - 1)] - tfd[s][q]);
+        const long long d = (long long)(fdr[fo[s] + x] - tfd[fo[s] + q]);
         const u32 c = (u32)(k % g);
         mn[c] = d < mn[c] ? d : mn[c];
         mx[c] = d > mx[c] ? d : mx[c];
       }
+    }
     long long lo = 0, hi = 0;
     for (u32 c = 0; c < g; ++c) lo = mn[c] > lo ? mn[c] : lo, hi = mx[c] > hi ? mx[c] : hi;
     t_lo = ((u64)lo + den - 1) / den;
     t_hi = ((u64)hi + den - 1) / den;
-  };
+  }
   // Brent: the tortoise jumps to the hare at powers of two; lam = blocks since the tortoise. The
   // first save waits for every stage to have started (j >= 0): from there the block map is the same
   // every block.
-  u32 rounds = 0;
-  do {
-    block();
-    rounds += Lam;
-  } while (j < 0);
-  save();
-  u32 power = 1, lam = 0;
-  int rc = RR_BUDGET;
-  for (;;) {
-    block();
+  __device__ __forceinline__ void init(const RRSetup &R) {
+    for (int w = 0; w < MAXN; ++w) wf[w] = 0;
+    for (int q = 0; q < RR_LINKS; ++q) lff[q] = lfb[q] = 0;
+    for (int s = 0; s < R.S; ++s) bph[s] = bl[s] = fph[s] = fl[s] = fw[s] = fr[s] = 0;
+    for (int s = 0, o = 0; s < R.S - 1; ++s) {
+      fo[s] = o;
+      o += R.D[s] - R.D[s + 1] + 1;
+    }
+    j = -(long long)R.D[0];  // the first round with an op: F_0(0)
+    rounds = 0;
+    do {
+      block(R);
+      rounds += R.Lam;
+    } while (j < 0);
+    save(R);
+    power = 1;
+    lam = 0;
+  }
+  __device__ __forceinline__ int step(const RRSetup &R, u32 cap, u64 prune, u64 &t_lo, u64 &t_hi) {
+    block(R);
     ++lam;
-    rounds += Lam;
-    bounds((u64)lam * Lam);
-    if (t_lo == t_hi) {
-      rc = RR_MET;
-      break;
-    }
-    if (t_lo > prune) {
-      rc = RR_PRUNED;
-      break;
-    }
-    if (rounds > cap) break;
+    rounds += R.Lam;
+    bounds(R, (u64)lam * R.Lam, t_lo, t_hi);
+    if (t_lo == t_hi) return RR_MET;
+    if (t_lo > prune) return RR_PRUNED;
+    if (rounds > cap) return RR_BUDGET;
     if (power == lam) {
-      save();
+      save(R);
       power *= 2;
       lam = 0;
     }
+    return RR_CONT;
   }
-  if (rounds_out) *rounds_out = rounds;
+};
+
+// The whole recurrence in the thread, up to `cap` rounds (S >= 2); see RRSim. *rounds_out
+// (optional): rounds run.
+static __device__ __noinline__ int rr_sim(const RRSetup &R, u32 cap, u64 prune, u64 &t_lo, u64 &t_hi,
+                                          u32 *rounds_out) {
+  RRSim sim;
+  sim.init(R);
+  int rc;
+  do rc = sim.step(R, cap, prune, t_lo, t_hi);
+  while (rc == RR_CONT);
+  if (rounds_out) *rounds_out = sim.rounds;
   return rc;
 }
 
