@@ -41,6 +41,7 @@ struct SmemTab {
   const u64 *PF, *PB, *PP, *O, *G, *tau;
   const u64 *ring;  // [256] slowest ring link of each worker set of N <= 8 (ascending ring order)
   const u32 *PF32, *PB32, *tau32;
+  const u32 *PC32;   // [N][L+1] exclusive prefix of fp + bp (32-bit), staged for the r = 1 closed form or nullptr
   const DivEnt *dv;  // replica-count divisors d = 1..16 (DivR / Div32 multipliers)
   const u64 *xp;     // global: the single-worker boundary table (DevTables::xp)
   int L, Lp1;
@@ -49,13 +50,17 @@ struct SmemTab {
 // Number of u64 words the staged tables need: the divisor table (17 x 32 B), PF, PB (N x (L+1)),
 // PP (L+1), O, G (L), tau (16 x 16); the narrow path stages PF32, PB32 in half the PF/PB space and
 // adds a 32-bit tau and the ring table.
-__host__ __device__ __forceinline__ u32 smem_words(u32 L, u32 N, bool narrow = false) {
+// pc: also the 32-bit r = 1 stage-cost prefix PC32 (eval kernels of 16-byte records under PipeDream
+// on a 32-bit or narrow state).
+__host__ __device__ __forceinline__ u32 smem_words(u32 L, u32 N, bool narrow = false, bool pc = false) {
   return (u32)DIVTAB_WORDS + 2u * N * (L + 1) + (L + 1) + 2u * L + (u32)(TAUW * TAUW) +
-         (narrow ? (u32)(TAUW * TAUW / 2) + 256u : 0u);
+         (narrow ? (u32)(TAUW * TAUW / 2) + 256u : 0u) + (pc ? (N * (L + 1) + 1u) / 2u : 0u);
 }
 
 // Cooperative copy of the global tables into shared memory (every thread of the block calls it).
-template <bool NARROW = false>
+// PC: stage PC32 = PF + PB (32-bit) after the other tables: from the narrow 32-bit tables (each
+// < 2^31, the sum < 2^32) or from DevTables::PC32 (valid on a 32-bit-path state).
+template <bool NARROW = false, bool PC = false>
 __device__ __forceinline__ SmemTab stage_tables(const DevTables &g, u64 *sm) {
   const u32 L = g.L, N = g.N, Lp1 = g.Lp1;
   DivEnt *dt = (DivEnt *)sm;
@@ -103,9 +108,13 @@ __device__ __forceinline__ SmemTab stage_tables(const DevTables &g, u64 *sm) {
   }
   if (NARROW)
     for (u32 i = threadIdx.x; i < 256u; i += blockDim.x) ring[i] = g.ring[i];
+  u32 *PC32 = (u32 *)(NARROW ? ring + 256 : tau + TAUW * TAUW);
+  if (PC)
+    for (u32 i = threadIdx.x; i < N * Lp1; i += blockDim.x) PC32[i] = NARROW ? g.PF32[i] + g.PB32[i] : g.PC32[i];
   __syncthreads();
   t.PP = PP; t.O = O; t.G = G; t.tau = tau;
   t.tau32 = NARROW ? tau32 : nullptr;
+  t.PC32 = PC ? PC32 : nullptr;
   t.ring = NARROW ? ring : nullptr;
   t.xp = g.xp;
   t.dv = dt;
@@ -311,7 +320,7 @@ __device__ __forceinline__ u64 eval_closed_form(const SmemTab &t, int S, const P
 // batch, grouped together by the shape sort): X_s = Y_s = F_s + B_s, no division, no sync term,
 // boundaries from the per-state table. Same value as eval_closed_form (tests score both kinds of
 // batches against the oracle). NARROW: the 32-bit prefix tables are staged.
-template <bool P32, bool NARROW, typename P>
+template <bool P32, bool NARROW, typename P, bool PC = false>
 __device__ __forceinline__ u64 eval_r1(const SmemTab &t, int S, const P &p) {
   constexpr int MS = P::MS;
   typedef typename std::conditional<P32, u32, u64>::type V;
@@ -326,7 +335,9 @@ __device__ __forceinline__ u64 eval_r1(const SmemTab &t, int S, const P &p) {
       const int e = (u == S - 1) ? t.L - 1 : p.cut(u);
       const int w = __ffs(p.mask(u)) - 1;
       V X;
-      if constexpr (NARROW)
+      if constexpr (PC)  // the staged F + B prefix: two loads instead of four
+        X = (V)(t.PC32[w * t.Lp1 + e + 1] - t.PC32[w * t.Lp1 + a]);
+      else if constexpr (NARROW)
         X = (V)(t.PF32[w * t.Lp1 + e + 1] - t.PF32[w * t.Lp1 + a]) + (V)(t.PB32[w * t.Lp1 + e + 1] - t.PB32[w * t.Lp1 + a]);
       else
         X = (V)((t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a]) + (t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a]));
@@ -496,12 +507,17 @@ __device__ __forceinline__ bool decode_record(u64 lo, u64 hi, int L, int N, int 
   ok &= ((id0 | __vcmpltu4(h0, SS)) & (id1 | __vcmpltu4(h1, SS))) == 0xFFFFFFFFu;
   const u64 busy = ~(((u64)id1 << 32) | id0);
   ok &= N >= 8 || (busy >> (8 * N)) == 0;
-  u64 masks = 0;
+  // byte s of masks = the workers of stage s, built in two 32-bit halves (stages 0-3, 4-7): 32-bit
+  // shifts instead of 64-bit ones
+  u32 m0 = 0, m1 = 0;
 #pragma unroll
   for (int w = 0; w < MAXN; ++w) {
     const u32 s = (u32)byte_at(hi, w);
-    masks |= (s < (u32)S) ? 1ull << (8 * s + w) : 0ull;
+    const u32 bit = (s < (u32)S) ? 1u << (8 * (s & 3u) + w) : 0u;
+    if (s & 4u) m1 |= bit;
+    else m0 |= bit;
   }
+  const u64 masks = (u64)m0 | ((u64)m1 << 32);
   p.masks = masks;
   // every stage s < S has a worker (byte s of masks nonzero)
   const u64 empty = (u64)__vcmpeq4((u32)masks, 0u) | ((u64)__vcmpeq4((u32)(masks >> 32), 0u) << 32);

@@ -80,6 +80,13 @@ __device__ __forceinline__ u64 rr_eval(const SmemTab &, int, const P &, int, u64
   return U64MAX;  // wide records: refused by the host
 }
 
+// The 32-bit F + B prefix is staged for the r = 1 closed form of 16-byte records under PipeDream on a
+// 32-bit or narrow state (launch_eval sizes the dynamic shared memory to match).
+template <int MODE, bool P32, bool NARROW, typename P>
+struct PCT {
+  static constexpr bool value = MODE == SCHED_PIPEDREAM && P::MS == 8 && (P32 || NARROW);
+};
+
 // Scores the record in `slot` and overwrites the slot with its results (bytes 0..7: T, 8..15: switch
 // bytes); the traversal then stores the chunk's results in input order, coalesced.
 template <bool ROLLOUT, bool P32, int MODE, bool NARROW, typename P, typename Rec>
@@ -93,7 +100,7 @@ __device__ __forceinline__ void score_one(const SmemTab &t, int L, int N, bool o
   // shape sort puts them together); a mixed step keeps the general form, so lanes do not diverge
   const bool lean = MODE == SCHED_PIPEDREAM && __all_sync(__activemask(), ok && all_single(p, S));
   if (ok) {
-    if (lean) T = eval_r1<P32, NARROW, P>(t, S, p);
+    if (lean) T = eval_r1<P32, NARROW, P, PCT<MODE, P32, NARROW, P>::value>(t, S, p);
     else if constexpr (MODE == SCHED_RR) T = rr_eval(t, S, p, (int)m.sync, i, q);
     else if constexpr (NARROW) T = eval_closed_form_n<P32, P>(t, S, p, (int)m.sync);
     else T = model_time<MODE, P32>(t, S, p, m);
@@ -110,7 +117,7 @@ __global__ void __launch_bounds__(EVAL_NT, EVAL_BLOCKS(MODE, P))
     k_eval(DevTables g, const Rec *__restrict__ recs, u64 count, u64 *__restrict__ out_t, u64 *__restrict__ out_sw,
            CurPart cur, ModelP m, u32 *counter, RRQueue rrq) {
   extern __shared__ u64 sm[];
-  const SmemTab t = stage_tables<NARROW>(g, sm);
+  const SmemTab t = stage_tables<NARROW, PCT<MODE, P32, NARROW, P>::value>(g, sm);
   const int L = t.L, N = (int)g.N;
   // a state that failed the device-side overflow check (set_state_device) scores nothing
   const bool overflow = (g.status[0] & 1ull) != 0;
@@ -224,7 +231,9 @@ int launch_eval(const DevTables &g, const void *recs, u64 count, bool wide, u64 
                 const int *cur_S, const u64 *cur_cuts, const u64 *cur_masks, int path32, const ModelP &m, int sms,
                 u32 *counter, cudaStream_t st, const RRQueue &rrq) {
   if (count == 0) return 0;
-  const size_t smem = (size_t)smem_words(g.L, g.N, (path32 & 2) != 0) * sizeof(u64);
+  // + the 32-bit F + B prefix for the PipeDream r = 1 closed form (PCT), when the kernel stages it
+  const bool pc = !wide && m.sched == SCHED_PIPEDREAM && (path32 & 3) != 0;
+  const size_t smem = (size_t)smem_words(g.L, g.N, (path32 & 2) != 0, pc) * sizeof(u64);
   CurPart cur;
   memset(&cur, 0, sizeof(cur));
   if (cur_S) {

@@ -56,6 +56,8 @@ def main():
     n = 1 << 20
     recs = torch.from_numpy(W.sample_records(prof.L, st.N, n, 1000)).cuda()
     out = torch.empty(n, dtype=torch.int64, device="cuda")
+    if "c5" in which:
+        res["c5_eval_1M_ms"], _ = timed(lambda: eng.eval_partitions(recs, out=out), reps=20, warm=3)
     if "rr" in which or "rr_eval" in which:
         eng.set_schedule(L_.SCHED_PIPEDREAM_RR, L_.SYNC_RING, 1, False)
         res["rr_eval_1M_ms"], _ = timed(lambda: eng.eval_partitions(recs, out=out))
@@ -67,6 +69,11 @@ def main():
         eng.set_schedule(L_.SCHED_CHIMERA, L_.SYNC_RING, 8, False)
         res["chimera_eval_1M_ms"], _ = timed(lambda: eng.eval_partitions(crecs, out=out))
     eng.set_schedule()
+    if "r1" in which:
+        gp = W.gpt96()
+        eng.load(gp, W.gpt_state("a-nvlink"))
+        r1 = torch.from_numpy(W.r1_records(gp.L, 8, n, 5)).cuda()
+        res["gpt96_r1_eval_1M_ms"], _ = timed(lambda: eng.eval_partitions(r1, out=out), reps=20, warm=3)
     prof = W.bert24()
     eng.load(prof, W.trace_c3(prof)[0])
     for k, model in (("rr", (L_.SCHED_PIPEDREAM_RR, L_.SYNC_RING, 1, False)),
