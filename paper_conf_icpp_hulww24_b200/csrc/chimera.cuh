@@ -14,7 +14,8 @@
 // One thread per partition runs that list schedule directly: per worker its free time and two list
 // positions, per pipeline and boundary a ring of the last transfer completions (a boundary never has
 // more than S <= 8 outstanding: a stage runs ahead of its successor by at most its warm-up), per
-// directed neighbour link its free time. Each step scans the 2S list heads for the earliest start.
+// directed neighbour link its free time. Each step picks the earliest start among the 2S list heads,
+// whose start times are cached and recomputed only where the step changed them.
 #pragma once
 #include "eval.cuh"
 
@@ -93,51 +94,60 @@ static __device__ __noinline__ u64 chimera_time(const SmemTab &t, int S, const P
     lastb[g][0] = lastb[g][1] = 0;
   }
   for (int q = 0; q < S - 1; ++q) fcnt[0][q] = fcnt[1][q] = bcnt[0][q] = bcnt[1][q] = 0;
+  // the start time of every list head (UINT64_MAX: exhausted or its input not produced yet), kept
+  // up to date incrementally: an op changes only its worker's two heads and the head that consumes
+  // the transfer it starts, so a step recomputes at most four heads and then picks the earliest
+  // start among the 2S cached ones (scan order = the tie order: lower worker, then down)
+  auto head_start = [&](int g, int pipe) -> u64 {
+    const u32 M = Mp[pipe];
+    if (pos[g][pipe] >= 2 * M) return U64MAX;
+    const int s = pipe == 0 ? g : S - 1 - g;  // stage index within the pipeline
+    int kind;
+    u32 k;
+    dapple_op(S, s, M, pos[g][pipe], kind, k);
+    u64 ready = 0;
+    if (kind == 0 && s > 0) {
+      if (k >= fcnt[pipe][s - 1]) return U64MAX;
+      ready = fr[pipe][s - 1][k & (CH_RING - 1)];
+    } else if (kind == 1 && s < S - 1) {
+      if (k >= bcnt[pipe][s]) return U64MAX;
+      ready = br[pipe][s][k & (CH_RING - 1)];
+    }
+    return umax(fre[g], ready);
+  };
+  u64 hs[MS][2];
+  for (int g = 0; g < S; ++g) hs[g][0] = head_start(g, 0), hs[g][1] = head_start(g, 1);
   const u32 total = 2u * (u32)S * m.M;
   for (u32 step = 0; step < total; ++step) {
     u64 best = U64MAX;
-    int bg = -1, bp = 0, bkind = 0;
-    u32 bk = 0;
-    for (int g = 0; g < S; ++g) {
-      for (int pipe = 0; pipe < 2; ++pipe) {
-        const u32 M = Mp[pipe];
-        if (pos[g][pipe] >= 2 * M) continue;
-        const int s = pipe == 0 ? g : S - 1 - g;  // stage index within the pipeline
-        int kind;
-        u32 k;
-        dapple_op(S, s, M, pos[g][pipe], kind, k);
-        u64 ready = 0;
-        if (kind == 0 && s > 0) {
-          if (k >= fcnt[pipe][s - 1]) continue;
-          ready = fr[pipe][s - 1][k & (CH_RING - 1)];
-        } else if (kind == 1 && s < S - 1) {
-          if (k >= bcnt[pipe][s]) continue;
-          ready = br[pipe][s][k & (CH_RING - 1)];
-        }
-        const u64 st = umax(fre[g], ready);
-        if (st < best) {
-          best = st;
+    int bg = -1, bp = 0;
+    for (int g = 0; g < S; ++g)
+      for (int pipe = 0; pipe < 2; ++pipe)
+        if (hs[g][pipe] < best) {
+          best = hs[g][pipe];
           bg = g;
           bp = pipe;
-          bkind = kind;
-          bk = k;
         }
-      }
-    }
     if (bg < 0) return U64MAX;  // cannot happen: the lists of both pipelines are live
     const int s = bp == 0 ? bg : S - 1 - bg;
+    int bkind;
+    u32 bk;
+    dapple_op(S, s, Mp[bp], pos[bg][bp], bkind, bk);
     const u64 end = best + dur[bg][bp][bkind];
     fre[bg] = end;
     ++pos[bg][bp];
+    int cg = -1;  // the group whose head consumes the transfer this op starts
     if (bkind == 0 && s < S - 1) {
       // forward transfer to the pipeline's next stage: down g -> g+1 on the right link, up on the left
       u64 fin;
       if (bp == 0) {
         fin = umax(end, lright[bg]) + xr_dn[bg];
         lright[bg] = fin;
+        cg = bg + 1;
       } else {
         fin = umax(end, lleft[bg - 1]) + xl_up[bg - 1];
         lleft[bg - 1] = fin;
+        cg = bg - 1;
       }
       fr[bp][s][bk & (CH_RING - 1)] = fin;
       ++fcnt[bp][s];
@@ -149,14 +159,19 @@ static __device__ __noinline__ u64 chimera_time(const SmemTab &t, int S, const P
         if (bp == 0) {
           fin = umax(end, lleft[bg - 1]) + xl_dn[bg - 1];
           lleft[bg - 1] = fin;
+          cg = bg - 1;
         } else {
           fin = umax(end, lright[bg]) + xr_up[bg];
           lright[bg] = fin;
+          cg = bg + 1;
         }
         br[bp][s - 1][bk & (CH_RING - 1)] = fin;
         ++bcnt[bp][s - 1];
       }
     }
+    hs[bg][0] = head_start(bg, 0);
+    hs[bg][1] = head_start(bg, 1);
+    if (cg >= 0) hs[cg][bp] = head_start(cg, bp);
   }
   u64 T = 0;
   for (int s = 0; s < S; ++s) {
