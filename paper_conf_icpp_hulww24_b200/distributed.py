@@ -7,7 +7,9 @@ The only exchange is the min-loc. On GPUs (`minloc_device`) each rank's asynchro
 the winner's record, with no host round trip until the caller reads the 40 bytes. `minloc` is the
 host-value form (two all_reduce(MIN) and one SUM), used by the CPU (gloo) tests and the e2e path.
 Every rank holds the full, KB-sized profile and state. The shard arithmetic is exact, so the result
-is the same for every world size.
+is the same for every world size. Rollout batches (`rollout_distributed`) split into
+one contiguous slice of records per rank; the per-record outputs stay on their rank or are
+all-gathered (8 bytes per record and output) into the full batch on every rank.
 """
 from __future__ import annotations
 
@@ -119,3 +121,43 @@ def search_distributed(engine, s_min: int, s_max: int, flags: int = 0, group=Non
     T, idx, n = minloc(r.time_ns, r.index, r.evaluated, group=group, device=device)
     part = engine.decode_index(s_min, s_max, flags, idx) if idx != U64_MAX else bytes([0xFF] * 16)
     return SearchResult(T, idx, n, part)
+
+
+def rollout_distributed(engine, records: torch.Tensor, current: Optional[bytes] = None, group=None,
+                        gather: bool = True, score: Optional[Callable] = None):
+    """Row e for the RL rollout rewards: rank r of G scores the records
+    [floor(r n / G), floor((r + 1) n / G)) of the batch (every rank holds the same batch, or at least
+    its slice) with the engine's autopipe_rollout_rewards. gather=False returns the rank's slice
+    bounds and its outputs (T_ns, switch bytes or None); gather=True all-gathers the outputs into the
+    whole batch on every rank (NCCL all_gather_into_tensor of equal, padded slices; gloo: host copies)
+    and returns (T_ns, switch bytes or None) for all n records. `score(slice, current)` replaces the
+    engine call (the CPU tests)."""
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    n = int(records.shape[0])
+    lo, hi = shard_bounds(n, rank, world)
+    if score is None:
+        t, sw = engine.rollout_rewards(records[lo:hi], current)
+    else:
+        t, sw = score(records[lo:hi], current)
+    if not gather:
+        return (lo, hi), t, sw
+    per = (n + world - 1) // world  # slices padded to the longest (at most one record longer)
+    outs = []
+    for x in (t, sw):
+        if x is None:
+            outs.append(None)
+            continue
+        pad = torch.zeros(per, dtype=torch.int64, device=x.device)
+        pad[: hi - lo] = x
+        if dist.get_backend(group) == "nccl":
+            full = torch.empty(world * per, dtype=torch.int64, device=x.device)
+            dist.all_gather_into_tensor(full, pad, group=group)
+        else:  # gloo: host copies
+            parts = [torch.empty(per, dtype=torch.int64) for _ in range(world)]
+            dist.all_gather(parts, pad.cpu(), group=group)
+            full = torch.cat(parts).to(x.device)
+        # rank q's slice starts at q * per in `full`; keep its hi_q - lo_q records
+        keep = [full[q * per: q * per + (shard_bounds(n, q, world)[1] - shard_bounds(n, q, world)[0])]
+                for q in range(world)]
+        outs.append(torch.cat(keep))
+    return outs[0], outs[1]

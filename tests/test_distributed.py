@@ -84,6 +84,24 @@ def _worker(rank, world, port, q, case):
                 res.append(int(t.item()) & ((1 << 64) - 1))
             q.put((rank, res))
             return
+        if case == "rollout":  # rollout batches: one slice per rank, outputs all-gathered (row e)
+            from oracle.rollout import rollout_rewards
+            from paper_conf_icpp_hulww24_b200.distributed import rollout_distributed
+            prof, st = W.toy(), W.toy_state()
+            recs = torch.from_numpy(W.sample_records(prof.L, st.N, 101, 7))
+            cur = bytes(recs[3].numpy().tobytes())
+
+            def score(sl, current):  # the oracle over the rank's slice (stand-in for the GPU call)
+                ts, sws = rollout_rewards(prof, st, [bytes(r.numpy().tobytes()) for r in sl], current)
+                to64 = lambda v: v - (1 << 64) if v >= (1 << 63) else v
+                t = torch.tensor([to64(a) for a in ts], dtype=torch.int64)
+                sw = torch.tensor([to64(b) for b in sws], dtype=torch.int64) if current is not None else None
+                return t, sw
+            t, sw = rollout_distributed(None, recs, cur, score=score)
+            (lo, hi), t_own, _ = rollout_distributed(None, recs, None, score=score, gather=False)
+            q.put((rank, ([int(x) & ((1 << 64) - 1) for x in t], [int(x) & ((1 << 64) - 1) for x in sw],
+                          (lo, hi), [int(x) & ((1 << 64) - 1) for x in t_own])))
+            return
         prof, st = W.toy(), W.toy_state()
         eng = _OracleEngine(prof.L, st.N)
 
@@ -201,3 +219,22 @@ def test_bound_allreduce_gloo_world2():
     out = _run(2, "bound")
     for rank in (0, 1):
         assert out[rank] == [416359965, 480722219, (1 << 64) - 1]
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_rollout_distributed_gloo(world):
+    """Row e for rollout batches: 101 records split over 2 or 3 ranks (uneven slices, padded for the
+    all-gather), every rank ends with the whole batch's (T, switch bytes) = the oracle's, in order."""
+    import workloads as W
+    from oracle.rollout import rollout_rewards
+    from paper_conf_icpp_hulww24_b200.distributed import shard_bounds
+    prof, st = W.toy(), W.toy_state()
+    recs = W.sample_records(prof.L, st.N, 101, 7)
+    cur = bytes(recs[3])
+    want = list(zip(*rollout_rewards(prof, st, [bytes(r) for r in recs], cur)))
+    out = _run(world, "rollout")
+    for rank in range(world):
+        t, sw, (lo, hi), t_own = out[rank]
+        assert t == [a for a, _ in want] and sw == [b for _, b in want]
+        assert (lo, hi) == shard_bounds(101, rank, world)
+        assert t_own == [a for a, _ in want[lo:hi]]

@@ -1,7 +1,8 @@
 """Row e's NCCL code path on the one GPU a test box has: a process group of world size 1 over the
 "nccl" backend runs `minloc_device` (all_gather_into_tensor of the 40-byte result, then the device
-reduction autopipe_reduce_results) and `bound_allreduce` (all_reduce MIN of the seed word) exactly as
-an 8-rank job does, minus the other ranks. The 96-layer 8-stage optimum (C4b, 64-bit path) must equal
+reduction autopipe_reduce_results), `bound_allreduce` (all_reduce MIN of the seed word) and
+`rollout_distributed` (all_gather_into_tensor of the padded per-rank output slices) exactly as an
+8-rank job does, minus the other ranks. The 96-layer 8-stage optimum (C4b, 64-bit path) must equal
 the oracle's parametric DP, through both the plain and the bounded search. (Several ranks on one GPU
 cannot share an NCCL communicator; the multi-rank exchange itself is covered by the gloo tests.)"""
 import json
@@ -37,9 +38,17 @@ theta = bound_allreduce(eng.search_seed_async(8, 8, begin=b[0], end=b[1]))
 eng.set_search_bound(theta)
 rb = result_from_bytes(minloc_device(eng.search_optimum_async(8, 8, begin=b[0], end=b[1])))
 eng.set_search_bound(None)
+from paper_conf_icpp_hulww24_b200.distributed import rollout_distributed
+rp = W.resnet50()
+rst = W.rollout_state(rp, 0)
+eng.load(rp, rst)
+recs = torch.from_numpy(W.sample_records(rp.L, rst.N, 5000, 1000)).cuda()
+rt, rsw = rollout_distributed(eng, recs, bytes(recs[0].cpu().numpy()))
 torch.cuda.synchronize()
+m = (1 << 64) - 1
 print(json.dumps({"T": r.time_ns, "idx": r.index, "n": r.evaluated, "Tb": rb.time_ns, "idxb": rb.index,
-                  "nb": rb.evaluated, "part": list(r.partition)}))
+                  "nb": rb.evaluated, "part": list(r.partition),
+                  "rt": [int(x) & m for x in rt.cpu()], "rsw": [int(x) & m for x in rsw.cpu()]}))
 dist.destroy_process_group()
 """
 
@@ -63,3 +72,12 @@ def test_nccl_minloc_and_bound_world1():
     assert (got["T"], got["idx"], got["n"]) == (T, idx, 11_050_084_695)
     assert (got["Tb"], got["idxb"], got["nb"]) == (T, idx, 11_050_084_695)
     assert parse_record(bytes(got["part"]), 96, 8) == part
+    # rollout_distributed (row e for rollout batches) through NCCL: the gathered batch, sampled
+    from tests._oracle_pool import rollout_many
+    rp = W.resnet50()
+    rst = W.rollout_state(rp, 0)
+    recs = W.sample_records(rp.L, rst.N, 5000, 1000)
+    idx = list(range(0, 5000, 7))
+    ot, osw = rollout_many(rp, rst, [bytes(recs[i]) for i in idx], bytes(recs[0]))
+    assert len(got["rt"]) == len(got["rsw"]) == 5000
+    assert [got["rt"][i] for i in idx] == ot and [got["rsw"][i] for i in idx] == osw
