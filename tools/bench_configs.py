@@ -78,7 +78,32 @@ def measure(device: int = 0, rollout_records: int = 1 << 20):
     ms_s, _ = _timed(lambda: eng.switch_rewards(recs, cur, 100, outputs=(), stream=None))
     res["F2_resnet50_switch_rewards"] = {"records": rollout_records, "ms": ms_s,
                                          "records_per_s": rollout_records / (ms_s / 1e3), "horizon": 100}
+    # C5 step latency: every step a new cluster state (rollout_state(step)) and a new
+    # batch (seed 1000 + step, already on the device): set_state from host arrays (host overflow check,
+    # H2D, state kernel) + rollout rewards, one CUDA-event pair per step around both
+    import numpy as _np
+    nst = 4
+    states = [W.rollout_state(prof, k) for k in range(nst)]
+    batches = [torch.from_numpy(W.sample_records(prof.L, states[k].N, rollout_records, 1000 + k)).cuda()
+               for k in range(nst)]
+    curs = [bytes(bt[0].cpu().numpy()) for bt in batches]
+    step_ms = []
+    for rep in range(2):
+        for k in range(nst):
+            torch.cuda.synchronize()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            eng.set_state(states[k].f, states[k].b, states[k].tau)
+            eng.rollout_rewards(batches[k], curs[k], out_t=out_t, out_sw=out_s)
+            b.record()
+            torch.cuda.synchronize()
+            if rep:
+                step_ms.append(a.elapsed_time(b))
+    del batches
+    eng.load(prof, st)
     res["C5_resnet50_rollout"] = {"records": rollout_records, "eval_ms": ms_e,
+                                  "step_ms_set_state_plus_rollout": float(_np.mean(step_ms)),
+                                  "step_states": nst,
                                   "eval_records_per_s": rollout_records / (ms_e / 1e3),
                                   "rollout_ms": ms_r, "rollout_records_per_s": rollout_records / (ms_r / 1e3),
                                   "eval_GBps_algorithmic": rollout_records * 24 / (ms_e / 1e3) / 1e9,
