@@ -36,7 +36,7 @@ struct autopipe_ctx {
   ModelP model{SCHED_PIPEDREAM, SYNC_RING, 1, 0};  // row f3: schedule variant + sync scheme
   DevTables tab{};
   // device buffers
-  u64 *d_raw = nullptr;      // fp [8*255] | bp [8*255] | P [255] | tau [64]
+  u64 *d_raw = nullptr;      // fp [N*L] | bp [N*L] | tau [N*N] (contiguous, one copy) ... | P [255] at RAW_P
   u64 *d_tables = nullptr;   // all DevTables arrays
   BlockOut *d_blocks = nullptr;
   ResultDev *d_result = nullptr;
@@ -60,7 +60,13 @@ struct autopipe_ctx {
   void *h_work = nullptr;  // pinned mirror of d_work (r = 1 schedules)
   size_t work_bytes = 0;
   // pinned host staging
-  u64 *h_stage = nullptr;    // fp | bp | tau(64)
+  u64 *h_stage = nullptr;    // fp | bp | tau (pinned staging of set_state, the layout of d_raw)
+  u64 *h_prof = nullptr;     // O [255] | G [255] | P [255] (pinned staging of load_profile)
+  // load_profile copies on its own stream (no host wait); set_state's stream waits for ev_prof.
+  // ev_stage / ev_prof mark the last copies out of the two staging buffers (a refill waits for them).
+  cudaStream_t pstream = nullptr;
+  cudaEvent_t ev_prof = nullptr, ev_stage = nullptr;
+  bool prof_pending = false, stage_pending = false;
   ResultDev *h_result = nullptr;
   u64 *h_status = nullptr;   // pinned copy of the device status word
   u64 binom[BINOM_N][BINOM_K];
@@ -95,6 +101,8 @@ struct autopipe_ctx {
 };
 
 static char g_create_err[256] = "";
+// word offset of P in d_raw: after the largest fp | bp | tau block (2 * 16 * 255 + 16 * 16 words)
+static const size_t RAW_P = 2 * (size_t)MAXNW * MAXL + (size_t)TAUW * TAUW;
 
 // The round-robin deferral queue for an evaluation on stream st (row f4): st first waits for the
 // previous drain that used the queue, and the caller records ev_rrq after its own launch.
@@ -207,6 +215,10 @@ extern "C" int autopipe_create(int cuda_device, autopipe_ctx **out) {
   if (e == cudaSuccess) e = cudaMalloc(&c->d_sched, (size_t)SEARCH_SCHED_BYTES * autopipe_ctx::NCTR);
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_ncount, 8);
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_stage, (2 * MAXNW * MAXL + TT) * 8);
+  if (e == cudaSuccess) e = cudaMallocHost(&c->h_prof, 3 * MAXL * 8);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&c->pstream, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_prof, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_stage, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_result, sizeof(ResultDev));
   if (e == cudaSuccess) e = cudaMallocHost(&c->h_status, 2 * sizeof(u64));
   if (e != cudaSuccess) {
@@ -264,6 +276,10 @@ extern "C" void autopipe_destroy(autopipe_ctx *c) {
     if (c->d_sched) cudaFree(c->d_sched);
     if (c->h_ncount) cudaFreeHost(c->h_ncount);
     if (c->h_stage) cudaFreeHost(c->h_stage);
+    if (c->h_prof) cudaFreeHost(c->h_prof);
+    if (c->pstream) cudaStreamDestroy(c->pstream);
+    if (c->ev_prof) cudaEventDestroy(c->ev_prof);
+    if (c->ev_stage) cudaEventDestroy(c->ev_stage);
     if (c->h_result) cudaFreeHost(c->h_result);
     if (c->h_status) cudaFreeHost(c->h_status);
     if (c->ev_hwork) cudaEventDestroy(c->ev_hwork);
@@ -299,11 +315,21 @@ extern "C" int autopipe_load_profile(autopipe_ctx *c, uint32_t L, const uint64_t
   }
   if (sumP >= LIMIT_BYTES) return fail(c, AUTOPIPE_E_OVERFLOW, "sum of weight bytes >= 2^56");
   DeviceGuard dg(c->device);
-  // O, G go straight to their tables; P to the raw area (the state kernel builds its prefix)
-  cudaError_t e = cudaMemcpy(c->tab.O, O, L * 8, cudaMemcpyHostToDevice);
-  if (e == cudaSuccess) e = cudaMemcpy(c->tab.G, G, L * 8, cudaMemcpyHostToDevice);
-  if (e == cudaSuccess) e = cudaMemcpy(c->d_raw + 2 * MAXNW * MAXL, P, L * 8, cudaMemcpyHostToDevice);
+  // O, G go straight to their (adjacent) tables, P to the raw area (the state kernel builds its
+  // prefix): staged in pinned memory and copied on the context's profile stream without a host wait;
+  // the next set_state's stream waits for the copies (ev_prof)
+  cudaError_t e = cudaSuccess;
+  if (c->prof_pending) e = cudaEventSynchronize(c->ev_prof);  // the staging buffer may still be read
+  if (e != cudaSuccess) return cuda_fail(c, e, "load_profile sync");
+  u64 *hO = c->h_prof, *hG = hO + MAXL, *hP = hG + MAXL;
+  memcpy(hO, O, L * 8);
+  memcpy(hG, G, L * 8);
+  memcpy(hP, P, L * 8);
+  e = cudaMemcpyAsync(c->tab.O, hO, (MAXL + L) * 8, cudaMemcpyHostToDevice, c->pstream);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(c->d_raw + RAW_P, hP, L * 8, cudaMemcpyHostToDevice, c->pstream);
+  if (e == cudaSuccess) e = cudaEventRecord(c->ev_prof, c->pstream);
   if (e != cudaSuccess) return cuda_fail(c, e, "load_profile copy");
+  c->prof_pending = true;
   c->L = L;
   c->maxOG = maxOG;
   c->sumP = (u64)sumP;
@@ -365,18 +391,22 @@ extern "C" int autopipe_set_state(autopipe_ctx *c, uint32_t N, const uint64_t *f
   c->bound = (u64)bound;
   DeviceGuard dg(c->device);
   cudaStream_t st = (cudaStream_t)stream;
-  // stage into pinned memory so the copies are truly asynchronous
-  cudaError_t e = cudaStreamSynchronize(st);  // the staging buffer may still feed a previous copy
+  // stage into pinned memory (fp | bp | tau contiguous: one truly asynchronous copy); a refill waits
+  // only for the previous copy out of the buffer (ev_stage), not for the stream's other work
+  cudaError_t e = cudaSuccess;
+  if (c->stage_pending) e = cudaEventSynchronize(c->ev_stage);
   if (e != cudaSuccess) return cuda_fail(c, e, "set_state sync");
-  u64 *hf = c->h_stage, *hb = hf + MAXNW * MAXL, *ht = hb + MAXNW * MAXL;
-  memcpy(hf, fp, (size_t)N * L * 8);
-  memcpy(hb, bp, (size_t)N * L * 8);
+  const size_t NL = (size_t)N * L;
+  u64 *hf = c->h_stage, *hb = hf + NL, *ht = hb + NL;
+  memcpy(hf, fp, NL * 8);
+  memcpy(hb, bp, NL * 8);
   memcpy(ht, tau, (size_t)N * N * 8);
-  u64 *rf = c->d_raw, *rb = rf + MAXNW * MAXL, *rP = rb + MAXNW * MAXL, *rt = rP + MAXL;
-  e = cudaMemcpyAsync(rf, hf, (size_t)N * L * 8, cudaMemcpyHostToDevice, st);
-  if (e == cudaSuccess) e = cudaMemcpyAsync(rb, hb, (size_t)N * L * 8, cudaMemcpyHostToDevice, st);
-  if (e == cudaSuccess) e = cudaMemcpyAsync(rt, ht, (size_t)N * N * 8, cudaMemcpyHostToDevice, st);
+  u64 *rf = c->d_raw, *rb = rf + NL, *rt = rb + NL, *rP = c->d_raw + RAW_P;
+  e = cudaStreamWaitEvent(st, c->ev_prof, 0);  // the profile's copies
+  if (e == cudaSuccess) e = cudaMemcpyAsync(rf, hf, (2 * NL + (size_t)N * N) * 8, cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess) e = cudaEventRecord(c->ev_stage, st);
   if (e != cudaSuccess) return cuda_fail(c, e, "set_state copy");
+  c->stage_pending = true;
   c->tab.L = L;
   c->tab.N = N;
   c->tab.Lp1 = L + 1;
@@ -403,7 +433,9 @@ extern "C" int autopipe_set_state_device(autopipe_ctx *c, uint32_t N, const uint
   c->tab.N = N;
   c->tab.Lp1 = c->L + 1;
   c->N = N;
-  const u64 *rP = c->d_raw + 2 * MAXNW * MAXL;
+  const u64 *rP = c->d_raw + RAW_P;
+  cudaError_t ew = cudaStreamWaitEvent(st, c->ev_prof, 0);  // the profile's copies
+  if (ew != cudaSuccess) return cuda_fail(c, ew, "set_state_device wait");
   c->launches += launch_build_state(c->tab, (const u64 *)d_fp, (const u64 *)d_bp, rP, (const u64 *)d_tau, c->sumP, st);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(c, e, "state kernel launch");
