@@ -154,6 +154,8 @@ __device__ __forceinline__ u64 flush_makespan(const SmemTab &t, int S, const P &
 // micro-batch 0 has crossed stages 0..s-1 (each stage's slowest replica, then the boundary) and before
 // micro-batch M-1's gradient crosses back to stage 0:
 //   T >= sum_{u<s} (maxF_u + dF_u) + M (F_w + B_w) + sum_{u<s} (dB_u + maxB_u);
+// plus each schedule's fill term (DAPPLE: micro-batch 0's round trip beyond s before B_s(0); GPipe:
+// the last stage's M forwards before any backward), below;
 // Chimera: worker g runs ceil(M/2) micro-batches of its down stage and floor(M/2) of its up stage.
 // UINT64_MAX for a record the model refuses (Chimera: a replicated stage).
 template <int MODE, typename P>
@@ -175,12 +177,16 @@ __device__ __forceinline__ u64 model_lower(const SmemTab &t, int S, const P &p, 
     return lb;
   } else {
     static_assert(MODE == SCHED_GPIPE || MODE == SCHED_DAPPLE, "flushed schedules and Chimera");
-    u64 lb = 0, pre = 0;  // pre: forward crossing to stage s plus backward crossing from it
+    // per stage u: maxF_u, maxB_u (the slowest replica: a stage op ends at its replicas' barrier),
+    // cf_u, cb_u (boundary u). tot = one micro-batch's whole round trip; pre = the crossing to stage s
+    // and back; fwd = the forward crossing to stage S - 1.
+    u64 lb = 0, pre = 0, tot = 0, fwd = 0, sumB = 0, sumCB = 0, dap = 0, gmaxB = 0, qlast = 0;
     for (int s = 0; s < S; ++s) {
       const u32 mask = p.mask(s);
       const int a = (s == 0) ? 0 : p.cut(s - 1) + 1, e = (s == S - 1) ? t.L - 1 : p.cut(s);
       const DivR<MN> dv((u32)__popc(mask), t.dv);
-      u64 mF = 0, mB = 0, work = 0;
+      const u64 ns = (u64)(S - s) < M ? (u64)(S - s) : M;  // DAPPLE's warm-up forwards
+      u64 mF = 0, mB = 0, work = 0, kd = 0, q = 0;
       for (u32 mm = mask; mm; mm &= mm - 1) {
         const int w = __ffs(mm) - 1;
         const u64 Fw = dv.ceil(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a]);
@@ -189,13 +195,36 @@ __device__ __forceinline__ u64 model_lower(const SmemTab &t, int S, const P &p, 
         mF = umax(mF, Fw);
         mB = umax(mB, Bw);
         work = umax(work, Fw + Bw);
+        kd = umax(kd, M * Bw + (M - ns) * Fw);
+        q = umax(q, M * Fw + Bw);
       }
+      // a worker's M forwards and backwards between the crossings (both schedules)
       lb = umax(lb, pre + M * work);
+      tot += mF + mB;
+      dap = umax(dap, kd - mB);  // kd >= M mB >= mB
       if (s < S - 1) {
         u64 cf, cb;
         boundary_cf_cb<MN>(t, p.cut(s), mask, p.mask(s + 1), cf, cb);
         pre += mF + cf + cb + mB;
+        tot += cf + cb;
+        fwd += mF + cf;
+        sumB += mB;
+        sumCB += cb;
+        gmaxB = umax(gmaxB, mB);
+      } else {
+        qlast = q;
       }
+    }
+    if (MODE == SCHED_DAPPLE) {
+      // a worker of stage s starts B_s(0) after micro-batch 0's round trip beyond s and then still
+      // runs M backwards and M - n_s forwards; micro-batch M - 1's gradient crosses back:
+      //   T >= tot - maxB_s + M B_w + (M - n_s) F_w
+      lb = umax(lb, tot + dap);
+    } else if (S > 1) {
+      // GPipe: B_s(0) (s < S - 1) waits for the last stage's M forwards and the backward chain down
+      // to s; then the worker runs M backwards and the gradient crosses back to stage 0:
+      //   T >= fwd + max_w(M F_w + B_w)[S - 1] + sum_{u < S-1} cb_u + sum_{u < S-1, u != s} maxB_u + M maxB_s
+      lb = umax(lb, fwd + qlast + sumCB + sumB + (M - 1) * gmaxB);
     }
     return lb;
   }

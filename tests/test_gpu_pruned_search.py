@@ -39,6 +39,9 @@ def eng():
 MODELS = {
     "gpipe_M4_recompute": ((SC.GPIPE, SC.RING, 4, True), lambda p, s, r: sched_many(p, s, r, SC.GPIPE, SC.RING, 4, True)),
     "dapple_M8_ps": ((SC.DAPPLE, SC.PS, 8, False), lambda p, s, r: sched_many(p, s, r, SC.DAPPLE, SC.PS, 8, False)),
+    "gpipe_M2": ((SC.GPIPE, SC.PS, 2, False), lambda p, s, r: sched_many(p, s, r, SC.GPIPE, SC.PS, 2, False)),
+    "dapple_M3": ((SC.DAPPLE, SC.RING, 3, False), lambda p, s, r: sched_many(p, s, r, SC.DAPPLE, SC.RING, 3, False)),
+    "dapple_M1": ((SC.DAPPLE, SC.RING, 1, False), lambda p, s, r: sched_many(p, s, r, SC.DAPPLE, SC.RING, 1, False)),
     "chimera_M6": ((SCHED_CHIMERA, 0, 6, False), lambda p, s, r: chimera_many(p, s, r, 6)),
     "roundrobin": ((SCHED_RR, 0, 1, False), lambda p, s, r: rr_many(p, s, r)),
 }
