@@ -61,6 +61,8 @@ __device__ __forceinline__ const P16 &cur_part(const CurPart &c, const P16 *) { 
 // drain kernel), or, when the queue is full, is finished here.
 __device__ __forceinline__ u64 rr_eval(const SmemTab &t, int S, const P8 &p, int sync, u64 i, const RRQueue &q) {
   if (!q.buf) return rr_time(t, S, p, sync);
+  // one worker per stage: the split model's closed form (reading F-5, C-2 the case r = 1)
+  if (__popcll(p.masks) == S) return eval_closed_form<false, false, P8>(t, S, p, sync);
   RRSetup R;
   rr_setup(t, S, p, sync, R);
   if (S == 1) return umax(rr_single_stage(R), R.Tsync);

@@ -514,24 +514,28 @@ __global__ void __launch_bounds__(RR_NT, 2) k_search_rr(DevTables g, SearchSpace
       const P8 p = part_from<P8>(sp, S, Rp, cuts);
       const u64 gb = *gbest;
       const u64 theta = umin(bestT - 1, gb);  // bestT = U64MAX: no own best yet
-      RRSetup R;
-      rr_setup(t, S, p, sync, R);
       u64 T = U64MAX;
-      if (S == 1) {
-        T = umax(rr_single_stage(R), R.Tsync);
-      } else if (umax(rr_lower(R), R.Tsync) <= theta) {
-        u64 t_lo, t_hi;
-        const int rc = rr_sim(R, q.rounds ? q.rounds : RR_SIM_ROUNDS, theta, t_lo, t_hi, nullptr);
-        if (rc == RR_MET || (rc == RR_BUDGET && R.Tsync >= t_hi)) {
-          T = umax(t_lo, R.Tsync);
-        } else if (rc == RR_BUDGET && umax(t_lo, R.Tsync) <= theta) {
-          const u32 k = atomicAdd(q.n, 1u);
-          if (k < q.cap) {
-            q.buf[3 * (u64)k] = i;
-            q.buf[3 * (u64)k + 1] = t_lo;
-            q.buf[3 * (u64)k + 2] = t_hi;
-          } else {
-            T = umax(rr_ceil_bf(R, t_lo, t_hi), R.Tsync);
+      if (__popcll(p.masks) == S) {  // one worker per stage: the split model's closed form (F-5)
+        T = eval_closed_form<false, false, P8>(t, S, p, sync);
+      } else {
+        RRSetup R;
+        rr_setup(t, S, p, sync, R);
+        if (S == 1) {
+          T = umax(rr_single_stage(R), R.Tsync);
+        } else if (umax(rr_lower(R), R.Tsync) <= theta) {
+          u64 t_lo, t_hi;
+          const int rc = rr_sim(R, q.rounds ? q.rounds : RR_SIM_ROUNDS, theta, t_lo, t_hi, nullptr);
+          if (rc == RR_MET || (rc == RR_BUDGET && R.Tsync >= t_hi)) {
+            T = umax(t_lo, R.Tsync);
+          } else if (rc == RR_BUDGET && umax(t_lo, R.Tsync) <= theta) {
+            const u32 k = atomicAdd(q.n, 1u);
+            if (k < q.cap) {
+              q.buf[3 * (u64)k] = i;
+              q.buf[3 * (u64)k + 1] = t_lo;
+              q.buf[3 * (u64)k + 2] = t_hi;
+            } else {
+              T = umax(rr_ceil_bf(R, t_lo, t_hi), R.Tsync);
+            }
           }
         }
       }

@@ -435,6 +435,11 @@ __device__ __forceinline__ u64 rr_ceil_bf_warp(const RRSetup &R, u64 t_lo, u64 t
 
 // T_ns of a validated 16-byte partition under round-robin replicas, in the thread.
 static __device__ __noinline__ u64 rr_time(const SmemTab &t, int S, const P8 &p, int sync) {
+#if !RR_STATS
+  // one worker per stage: round-robin replicas coincide with the split model (reading F-5: C-2 is
+  // the case r = 1), whose closed form replaces the recurrence
+  if (__popcll(p.masks) == S) return eval_closed_form<false, false, P8>(t, S, p, sync);
+#endif
   RRSetup R;
   rr_setup(t, S, p, sync, R);
   if (S == 1) return umax(rr_single_stage(R), R.Tsync);
