@@ -56,6 +56,9 @@ def main():
     n = 1 << 20
     recs = torch.from_numpy(W.sample_records(prof.L, st.N, n, 1000)).cuda()
     out = torch.empty(n, dtype=torch.int64, device="cuda")
+    if "switch" in which:
+        cur = bytes(recs[0].cpu().numpy())
+        res["switch_1M_ms"], _ = timed(lambda: eng.switch_rewards(recs, cur, 100, outputs=()), reps=10, warm=2)
     if "c5" in which:
         res["c5_eval_1M_ms"], _ = timed(lambda: eng.eval_partitions(recs, out=out), reps=20, warm=3)
     if "rr" in which or "rr_eval" in which:
