@@ -35,7 +35,7 @@ namespace ap {
 #ifndef RR_STATS
 #define RR_STATS 0
 #endif
-constexpr u32 RR_SIM_ROUNDS = 4096;    // in-thread budget (search; eval when the deferral queue is full)
+constexpr u32 RR_SIM_ROUNDS = 4096;    // in-thread budget when nothing is deferred (AUTOPIPE_RR_NO_DEFER)
 constexpr int RR_BF_NODES = 160;       // 4 S Lam <= 144 nodes for sum r <= 8
 constexpr int RR_LINKS = 16;           // max over sum r <= 8 of sum_s lcm(r_s, r_{s+1}) (r = 1, 4, 3)
 constexpr int RR_PEND = 24;            // pending forward transfers: sum_s (D_s - D_{s+1} + 1) <= 15 + 7
@@ -152,8 +152,8 @@ enum { RR_MET = 0, RR_BUDGET = 1, RR_PRUNED = 2, RR_CONT = 3 };
 // stage has started, j >= 0) and saves the tortoise; each step() runs one block of Lam rounds and
 // decides: RR_MET: t_lo = t_hi = ceil(lambda_compute), the growth bounds met; RR_PRUNED: t_lo > prune
 // (a search candidate that cannot win); RR_BUDGET: more than `cap` rounds, t_lo <= ceil(lambda_compute)
-// <= t_hi; RR_CONT: not decided yet. A lane of the eval kernel resumes it block by block, so a lane
-// whose record is decided can take the warp's next record (k_eval.cu).
+// <= t_hi; RR_CONT: not decided yet. (Resuming it block by block to refill decided lanes with the
+// warp's next records was measured no faster: DESIGN.md §10.)
 struct RRSim {
   // absolute times (no rebasing: < 2^58 within the round cap for a state bound below 2^45, checked by
   // the host)
