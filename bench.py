@@ -322,10 +322,7 @@ def main():
         if world > 1:
             dist.destroy_process_group()
         return
-    # contiguous shards of about equal device cost (host-only estimate; any split gives the same optimum)
     from paper_conf_icpp_hulww24_b200.distributed import balanced_bounds
-    bounds = balanced_bounds(96, 8, S_STAGES, S_STAGES, 0, world)
-    lo, hi = bounds[rank], bounds[rank + 1]
 
     from paper_conf_icpp_hulww24_b200 import result_from_bytes
     from paper_conf_icpp_hulww24_b200.distributed import minloc_device
@@ -350,6 +347,11 @@ def main():
         prof, st = W.gpt96(), W.gpt_state(kind)
         eng = Engine(local)
         eng.load_profile(prof.O, prof.G, prof.P)
+        # contiguous shards of about equal device cost under the state's integer path (the host
+        # classifies it from the state; host-only estimate, any split gives the same optimum)
+        eng.set_state(st.f, st.b, st.tau)
+        bounds = balanced_bounds(96, 8, S_STAGES, S_STAGES, 0, world, eng.int_path)
+        lo, hi = bounds[rank], bounds[rank + 1]
         d_fp = torch.tensor(np.asarray(st.f, dtype=np.uint64).view(np.int64), device=dev)
         d_bp = torch.tensor(np.asarray(st.b, dtype=np.uint64).view(np.int64), device=dev)
         d_tau = torch.tensor(np.asarray(st.tau, dtype=np.uint64).view(np.int64), device=dev)
@@ -414,7 +416,7 @@ def main():
         int_path = eng.int_path
         eng.close()
         h2d = 3 * 96 * 8 + 2 * 8 * 96 * 8 + 8 * 8 * 8
-        return {"total_ms": total_ms, "ms_per_step": total_ms / args.steps, "kernel_ms": kern_avg,
+        return {"total_ms": total_ms, "ms_per_step": total_ms / args.steps, "kernel_ms": kern_avg, "cands": hi - lo,
                 "value": TOTAL * args.steps / (total_ms / 1000.0), "optimum": results[0],
                 "launches": launches, "clocks": clk.summary(), "int_path": int_path,
                 "e2e": {"value": TOTAL * args.steps / e2e_s, "unit": UNIT, "h2d_bytes_per_step": h2d,
@@ -444,7 +446,7 @@ def main():
         pass
     peak_issue, peak_alu, peak_src = alu_peaks(live, saved)
     ops_per_cand = OPS_PER_CANDIDATE[main_res["int_path"]]
-    cands_per_rank = hi - lo
+    cands_per_rank = main_res["cands"]
     achieved = ops_per_cand * cands_per_rank / (main_res["kernel_ms"] / 1000.0) / 1e12
     kname = "k_search_r1<8,%s>" % ("u32" if main_res["int_path"] == 32 else "u64")
     traffic = None

@@ -331,6 +331,11 @@ int autopipe_get_schedule(const autopipe_ctx *ctx, uint32_t *schedule, uint32_t 
  * E_INVAL on bad arguments, E_OVERFLOW if the space exceeds 2^64. */
 int autopipe_balanced_shards(uint32_t L, uint32_t N, uint32_t s_min, uint32_t s_max, uint32_t flags, uint32_t G,
                              uint64_t *bounds);
+/* The same split with the cost model of the integer path the shards' state runs (int_path = 32 or
+ * 64, as autopipe_int_path reports it: the 32-bit sweep's candidates are cheaper against its per-row
+ * work, so its shards move their bounds toward the short rows). E_INVAL for another int_path. */
+int autopipe_balanced_shards_path(uint32_t L, uint32_t N, uint32_t s_min, uint32_t s_max, uint32_t flags,
+                                  uint32_t G, uint32_t int_path, uint64_t *bounds);
 
 /* Number of candidates of a search space (requires a state for L and N); S up to min(16, N). */
 int autopipe_count_candidates(const autopipe_ctx *ctx, uint32_t s_min, uint32_t s_max, uint32_t flags,

@@ -39,7 +39,8 @@ SYMBOLS = ["autopipe_create", "autopipe_destroy", "autopipe_last_error", "autopi
            "autopipe_get_schedule", "autopipe_eval_partitions_w", "autopipe_rollout_rewards_w",
            "autopipe_search_optimum_w", "autopipe_decode_index_w", "autopipe_search_optimum_async",
            "autopipe_search_optimum_async_w", "autopipe_reduce_results", "autopipe_reduce_results_w", "autopipe_search_times",
-           "autopipe_search_seed_async", "autopipe_set_search_bound", "autopipe_local_search"]
+           "autopipe_search_seed_async", "autopipe_set_search_bound", "autopipe_local_search",
+           "autopipe_balanced_shards_path"]
 
 
 class Partition(ctypes.Structure):
@@ -102,6 +103,7 @@ def _load():
         "autopipe_neighbourhood_best": (i32, [P, ctypes.POINTER(Partition), ctypes.POINTER(Result), P]),
         "autopipe_switch_rewards": (i32, [P, P, u64, ctypes.POINTER(Partition), u64, P, P, P, P, P]),
         "autopipe_balanced_shards": (i32, [u32, u32, u32, u32, u32, u32, pu64]),
+        "autopipe_balanced_shards_path": (i32, [u32, u32, u32, u32, u32, u32, u32, pu64]),
         "autopipe_set_schedule": (i32, [P, u32, u32, u32, u32]),
         "autopipe_eval_partitions_w": (i32, [P, P, u64, P, P]),
         "autopipe_rollout_rewards_w": (i32, [P, P, u64, ctypes.POINTER(PartitionW), P, P, P]),

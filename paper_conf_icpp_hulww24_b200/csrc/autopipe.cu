@@ -1255,7 +1255,10 @@ extern "C" int autopipe_switch_rewards(autopipe_ctx *c, const autopipe_partition
 // the seeded sweep: max/min of 8 C(95,7) shards 1.07 (C4a), 1.05 (C4b)); the generic
 // kernel costs GEN * S per candidate.
 namespace {
-const u64 COST_ROW = 600, COST_X = 30, COST_CAND = 4, COST_GEN = 40;
+// per-row fixed cost of the r = 1 sweep: the 64-bit path (the default), and the 32-bit one, whose
+// candidates are cheaper against the same per-row work (B200, the 96-layer 8-stage space, slowest of
+// 8 shards: C4a 0.499 ms at 600, 0.479 at 1000; C4b 0.652 at 600, 0.669 at 1000)
+const u64 COST_ROW = 600, COST_ROW32 = 1000, COST_X = 30, COST_CAND = 4, COST_GEN = 40;
 u64 hbin[256][17];  // C(n, k), k <= 16 (wide spaces), saturated at 2^64 - 1
 void hbin_init() {
   static bool done = false;
@@ -1290,18 +1293,18 @@ u64 count_less_t(int x, int k, const int *t) {
   }
   return cnt;
 }
-inline double row_cost(int L, int y) {
+inline double row_cost(int L, int y, double row) {
   // AUTOPIPE_COST_{ROW,X,CAND}: experiment knobs for re-fitting the model (unset: the constants)
   static const char *kr = experiment_knob("AUTOPIPE_COST_ROW"), *kx = experiment_knob("AUTOPIPE_COST_X"),
                     *kc = experiment_knob("AUTOPIPE_COST_CAND");
-  static const double cr = kr ? atof(kr) : (double)COST_ROW;
+  const double cr = kr ? atof(kr) : row;
   static const double cx = kx ? atof(kx) : (double)COST_X;
   static const double cc = kc ? atof(kc) : (double)COST_CAND;
   const double m = (double)(L - 2 - y);
   return cr + cx * (m - 1) + cc * m * (m - 1) / 2;
 }
 // cost of the first `kappa` cut sets (lexicographic) of an r = 1 block with S stages
-double r1_prefix_cost(int L, int S, u64 kappa, u64 ncut) {
+double r1_prefix_cost(int L, int S, u64 kappa, u64 ncut, double row) {
   if (kappa == 0) return 0.0;
   const int P = S - 4, n = L - 1, k = S - 1;
   int lo[8];
@@ -1312,14 +1315,14 @@ double r1_prefix_cost(int L, int S, u64 kappa, u64 ncut) {
     const bool fits = (P == 0) || lo[P - 1] < y;
     u64 rows = count_less_t(y, P, lo) + ((fits && y < lo[P]) ? 1 : 0);
     if (end && fits && y == lo[P]) rows += 1;  // the last row itself
-    c += (double)rows * row_cost(L, y);
+    c += (double)rows * row_cost(L, y, row);
   }
   return c;
 }
 }  // namespace
 
-extern "C" int autopipe_balanced_shards(uint32_t L, uint32_t N, uint32_t s_min, uint32_t s_max, uint32_t flags,
-                                        uint32_t G, uint64_t *bounds) {
+static int balanced_shards(uint32_t L, uint32_t N, uint32_t s_min, uint32_t s_max, uint32_t flags, uint32_t G,
+                           double row, uint64_t *bounds) {
   if (!bounds || G < 1 || L < 1 || L > MAXL || N < 1 || N > MAXNW) return AUTOPIPE_E_INVAL;
   if (flags & ~AUTOPIPE_USE_ALL_WORKERS) return AUTOPIPE_E_INVAL;
   // 16-byte spaces (S, N <= 8) and wide ones (row f4: S, N <= 16; their S > 8 blocks are generic)
@@ -1341,7 +1344,7 @@ extern "C" int autopipe_balanced_shards(uint32_t L, uint32_t N, uint32_t s_min, 
     const bool r1 = S >= 5 && S <= MAXS && (!all || (int)N == S) && nc > 0;
     u64 start = (u64)off;
     if (r1) {
-      const double c = r1_prefix_cost((int)L, S, nc, nc);
+      const double c = r1_prefix_cost((int)L, S, nc, nc, row);
       blk[nb++] = {start, start + nc, S, true, acc, acc + c};
       acc += c;
       start += nc;
@@ -1370,7 +1373,7 @@ extern "C" int autopipe_balanced_shards(uint32_t L, uint32_t N, uint32_t s_min, 
         u64 a = 0, z = B.hi - B.lo;
         while (a < z) {
           const u64 mid = a + (z - a) / 2;
-          if (B.c0 + r1_prefix_cost((int)L, B.S, mid, B.hi - B.lo) < target) a = mid + 1;
+          if (B.c0 + r1_prefix_cost((int)L, B.S, mid, B.hi - B.lo, row) < target) a = mid + 1;
           else z = mid;
         }
         b = B.lo + a;
@@ -1382,4 +1385,15 @@ extern "C" int autopipe_balanced_shards(uint32_t L, uint32_t N, uint32_t s_min, 
     bounds[g] = b;
   }
   return AUTOPIPE_OK;
+}
+
+extern "C" int autopipe_balanced_shards(uint32_t L, uint32_t N, uint32_t s_min, uint32_t s_max, uint32_t flags,
+                                        uint32_t G, uint64_t *bounds) {
+  return balanced_shards(L, N, s_min, s_max, flags, G, (double)COST_ROW, bounds);
+}
+
+extern "C" int autopipe_balanced_shards_path(uint32_t L, uint32_t N, uint32_t s_min, uint32_t s_max, uint32_t flags,
+                                             uint32_t G, uint32_t int_path, uint64_t *bounds) {
+  if (int_path != 32 && int_path != 64) return AUTOPIPE_E_INVAL;
+  return balanced_shards(L, N, s_min, s_max, flags, G, (double)(int_path == 32 ? COST_ROW32 : COST_ROW), bounds);
 }

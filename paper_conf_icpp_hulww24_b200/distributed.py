@@ -30,14 +30,20 @@ def shard_bounds(total: int, rank: int, world: int) -> Tuple[int, int]:
     return rank * total // world, (rank + 1) * total // world
 
 
-def balanced_bounds(L: int, N: int, s_min: int, s_max: int, flags: int, world: int) -> List[int]:
+def balanced_bounds(L: int, N: int, s_min: int, s_max: int, flags: int, world: int,
+                    int_path: Optional[int] = None) -> List[int]:
     """world + 1 global indices splitting the space into contiguous shards of about equal device cost
     (autopipe_balanced_shards: host-only, no GPU). Equal-candidate shards leave the last rank, whose
-    rows are short, up to ~1.3x slower than the first on the 96-layer space."""
+    rows are short, up to ~1.3x slower than the first on the 96-layer space. int_path (32 or 64, the
+    state's integer path as Engine.int_path reports it) selects that path's cost model
+    (autopipe_balanced_shards_path)."""
     import ctypes
     from ._lib import lib
     out = (ctypes.c_uint64 * (world + 1))()
-    rc = lib.autopipe_balanced_shards(L, N, s_min, s_max, flags, world, out)
+    if int_path in (32, 64):
+        rc = lib.autopipe_balanced_shards_path(L, N, s_min, s_max, flags, world, int_path, out)
+    else:
+        rc = lib.autopipe_balanced_shards(L, N, s_min, s_max, flags, world, out)
     if rc != 0:
         raise ValueError("autopipe_balanced_shards failed (%d)" % rc)
     return [int(x) for x in out]
@@ -108,7 +114,8 @@ def search_distributed(engine, s_min: int, s_max: int, flags: int = 0, group=Non
     `reduce_fn` replaces the device reduction of `minloc_device` (the CPU tests)."""
     rank, world = dist.get_rank(group), dist.get_world_size(group)
     if balanced:
-        b = balanced_bounds(engine.L, engine.N, s_min, s_max, flags, world)
+        path = getattr(engine, "int_path", None) if hasattr(engine, "_h") else None
+        b = balanced_bounds(engine.L, engine.N, s_min, s_max, flags, world, path)
         lo, hi = b[rank], b[rank + 1]
     else:
         total = engine.count_candidates(s_min, s_max, flags)

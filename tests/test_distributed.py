@@ -202,6 +202,18 @@ def test_balanced_bounds_partition_the_space():
     b = balanced_bounds(96, 8, 8, 8, 0, 8)
     sizes = [y - x for x, y in zip(b, b[1:])]
     assert sizes[-1] < sizes[0] and abs(sum(sizes) - comb(95, 7)) == 0
+    # per integer path (autopipe_balanced_shards_path): the 64-bit model is the default one; the
+    # 32-bit model weighs rows more, so its interior bounds move toward the end of the space
+    assert balanced_bounds(96, 8, 8, 8, 0, 8, 64) == b
+    b32 = balanced_bounds(96, 8, 8, 8, 0, 8, 32)
+    assert b32[0] == 0 and b32[-1] == comb(95, 7) and all(x <= y for x, y in zip(b32, b32[1:]))
+    assert all(x >= y for x, y in zip(b32[1:-1], b[1:-1]))
+    for (L, N, smin, smax, flags) in ((21, 8, 1, 8, 0), (26, 8, 5, 8, 1)):
+        total = count(L, N, smin, smax, flags)
+        for G in (1, 3, 8):
+            b = balanced_bounds(L, N, smin, smax, flags, G, 32)
+            assert len(b) == G + 1 and b[0] == 0 and b[-1] == total
+            assert all(x <= y for x, y in zip(b, b[1:]))
 
 
 def test_balanced_bounds_rejects_bad_arguments():
@@ -211,6 +223,10 @@ def test_balanced_bounds_rejects_bad_arguments():
                  (96, 16, 1, 17, 0, 2)):
         with pytest.raises(ValueError):
             balanced_bounds(*args)
+    import ctypes
+    from paper_conf_icpp_hulww24_b200._lib import lib
+    out = (ctypes.c_uint64 * 3)()
+    assert lib.autopipe_balanced_shards_path(96, 8, 8, 8, 0, 2, 16, out) != 0  # int_path must be 32 or 64
 
 
 def test_bound_allreduce_gloo_world2():

@@ -28,11 +28,13 @@ def main(kind="a-nvlink", steps=10, warm=3):
     d_fp = torch.tensor(np.asarray(st.f, dtype=np.uint64).view(np.int64), device=dev)
     d_bp = torch.tensor(np.asarray(st.b, dtype=np.uint64).view(np.int64), device=dev)
     d_tau = torch.tensor(np.asarray(st.tau, dtype=np.uint64).view(np.int64), device=dev)
+    eng.set_state(st.f, st.b, st.tau)  # the host classifies the integer path (the shard cost model's)
+    path = eng.int_path
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device=dev)
     stream = torch.cuda.current_stream(dev)
-    out = {"state": kind}
+    out = {"state": kind, "int_path": path}
     for G in (1, 2, 4, 8):
-        b = balanced_bounds(96, 8, 8, 8, 0, G)
+        b = balanced_bounds(96, 8, 8, 8, 0, G, path)
         per = []
         for r in range(G):
             for _ in range(warm):
