@@ -286,15 +286,58 @@ struct RRSim {
     power = 1;
     lam = 0;
   }
+  // An exact repeat: every live component of each class moved by its class's first component's
+  // delta since the save (stops at the first mismatch, the common case); then t_lo = t_hi = T.
+  __device__ __forceinline__ bool repeated(const RRSetup &R, u64 den, u64 &t_lo, u64 &t_hi) const {
+    const int S = R.S;
+    const u32 g = R.g;
+    long long ref[MAXN];
+    bool seen[MAXN];
+    for (u32 c = 0; c < g; ++c) seen[c] = false;
+    auto same = [&](u32 c, long long d) {
+      if (!seen[c]) {
+        seen[c] = true;
+        ref[c] = d;
+        return true;
+      }
+      return d == ref[c];
+    };
+    for (int s = 0; s < S; ++s)
+      for (int i = 0; i < R.r[s]; ++i) {
+        const int w = (R.wl[s] >> (4 * i)) & 15;
+        if (!same((u32)i % g, (long long)(wf[w] - tw[w]))) return false;
+      }
+    for (int s = 0; s < S - 1; ++s)
+      for (int k = 0; k < R.lc[s]; ++k) {
+        const int ql = R.lo[s] + k;
+        if (!same((u32)k % g, (long long)(lff[ql] - tlf[ql])) || !same((u32)k % g, (long long)(lfb[ql] - tlb[ql])))
+          return false;
+      }
+    for (int s = 0; s < S - 1; ++s) {
+      const int len = R.D[s] - R.D[s + 1] + 1;
+      for (int q = 0, x = fr[s]; q < len - 1; ++q, x = x + 1 == len ? 0 : x + 1) {
+        const long long k = j + R.D[s + 1] + q;
+        if (!same((u32)(k % g), (long long)(fdr[fo[s] + x] - tfd[fo[s] + q]))) return false;
+      }
+    }
+    long long mx = 0;
+    for (u32 c = 0; c < g; ++c) mx = ref[c] > mx ? ref[c] : mx;
+    t_lo = t_hi = ((u64)mx + den - 1) / den;
+    return true;
+  }
+  // One block, then the decision: the cheap exact-repeat test after every block, the growth bounds
+  // (met, pruned, budget) at Brent's doublings and when the budget runs out.
   __device__ __forceinline__ int step(const RRSetup &R, u32 cap, u64 prune, u64 &t_lo, u64 &t_hi) {
     block(R);
     ++lam;
     rounds += R.Lam;
-    bounds(R, (u64)lam * R.Lam, t_lo, t_hi);
-    if (t_lo == t_hi) return RR_MET;
-    if (t_lo > prune) return RR_PRUNED;
-    if (rounds > cap) return RR_BUDGET;
-    if (power == lam) {
+    const u64 den = (u64)lam * R.Lam;
+    if (repeated(R, den, t_lo, t_hi)) return RR_MET;
+    if (power == lam || rounds > cap) {
+      bounds(R, den, t_lo, t_hi);
+      if (t_lo == t_hi) return RR_MET;
+      if (t_lo > prune) return RR_PRUNED;
+      if (rounds > cap) return RR_BUDGET;
       save(R);
       power *= 2;
       lam = 0;
