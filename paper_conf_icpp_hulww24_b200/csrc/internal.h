@@ -36,7 +36,10 @@ struct RRQueue {
   u32 cap = 0;
   u32 rounds = 0;      // round budget before a record is deferred
 };
-constexpr u32 RR_DEFER_ROUNDS = 256;
+#ifndef RR_DEFER_ROUNDS_DEF
+#define RR_DEFER_ROUNDS_DEF 256  // B200, 1M C5 records: 128 / 256 / 1024 rounds -> 9.8 / 8.4 / 9.5 ms
+#endif
+constexpr u32 RR_DEFER_ROUNDS = RR_DEFER_ROUNDS_DEF;
 int launch_eval(const DevTables &g, const void *recs, u64 count, bool wide, u64 *out_t, u64 *out_sw,
                 const int *cur_S, const u64 *cur_cuts, const u64 *cur_masks, int path32, const ModelP &m, int sms,
                 u32 *counter, cudaStream_t st, const RRQueue &rrq = RRQueue());
