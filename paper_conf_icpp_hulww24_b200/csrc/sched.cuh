@@ -12,9 +12,9 @@
 // In both orders every op's inputs are produced before it (B_s(j) reads backward boundary s of j,
 // produced just before by stage s+1; F_s(k) reads forward boundary s-1 of k, produced earlier by
 // stage s-1), each worker's ops are visited in its own list order, and each boundary's transfers in
-// micro-batch order, so one "latest" value per boundary, one free time per worker (registers) and one
-// free time per directed link (the links of different boundaries are distinct) reproduce the
-// ready-driven execution exactly.
+// micro-batch order, so one "latest" value per boundary, one free time per worker and one free time per
+// boundary direction (its links are used by no other boundary) reproduce the ready-driven execution
+// exactly.
 #pragma once
 #include "eval.cuh"
 #include "chimera.cuh"
@@ -22,129 +22,99 @@
 
 namespace ap {
 
-// T_ns of one flushed iteration (GPipe or DAPPLE) of a validated partition (P8 or the wide P16).
+// T_ns of one flushed iteration (GPipe or DAPPLE) of a validated partition (P8 or the wide P16). Loops
+// run over the actual stages and over each stage's own workers (its mask bits), with the per-worker
+// and per-stage state in small arrays: the unrolled form with every worker slot predicated in every
+// stage step (S x N slot visits per round, registers for 16-byte records, spills for wide ones) was
+// slower at both widths (B200, 1M records, M = 8: GPipe 0.70 -> 0.56 ms, DAPPLE 0.68 -> 0.64; wide
+// GPipe + recompute 6.0 -> 2.2, wide DAPPLE 9.0 -> 2.4; BERT-24 searches GPipe 1.8 -> 1.2, DAPPLE
+// 3.5 -> 2.2).
 template <int SCHED, typename P>
 __device__ __forceinline__ u64 flush_makespan(const SmemTab &t, int S, const P &p, const ModelP &m) {
   static_assert(SCHED == SCHED_GPIPE || SCHED == SCHED_DAPPLE, "flushed schedules only");
   constexpr int MS = P::MS, MN = P::MN;
   const int M = (int)m.M;
   u64 Fd[MN], Bd[MN], wf[MN];
-  int stg[MN];
-#pragma unroll
-  for (int w = 0; w < MN; ++w) {
-    stg[w] = 0xFF;  // idle: never matches a stage
-#pragma unroll
-    for (int s = 0; s < MS; ++s)
-      if (s < S && ((p.mask(s) >> w) & 1u)) stg[w] = s;
-    wf[w] = 0;
-    Fd[w] = 0;
-    Bd[w] = 0;
-    const int s = stg[w];
-    if (s != 0xFF) {
-      const int a = (s == 0) ? 0 : p.cut(s - 1) + 1;
-      const int e = (s == S - 1) ? t.L - 1 : p.cut(s);
-      const DivR<MN> dv((u32)__popc(p.mask(s)), t.dv);
+  u32 msk[MS];
+  u64 dF[MS], dB[MS], lfF[MS], lfB[MS], fdl[MS], last[MS];
+  for (int s = 0; s < S; ++s) {
+    const u32 mask = p.mask(s);
+    msk[s] = mask;
+    const int a = (s == 0) ? 0 : p.cut(s - 1) + 1;
+    const int e = (s == S - 1) ? t.L - 1 : p.cut(s);
+    const DivR<MN> dv((u32)__popc(mask), t.dv);
+    for (u32 mm = mask; mm; mm &= mm - 1) {
+      const int w = __ffs(mm) - 1;
       Fd[w] = dv.ceil(t.PF[w * t.Lp1 + e + 1] - t.PF[w * t.Lp1 + a]);
       Bd[w] = dv.ceil(t.PB[w * t.Lp1 + e + 1] - t.PB[w * t.Lp1 + a]);
       if (SCHED == SCHED_GPIPE && m.recompute) Bd[w] += Fd[w];  // the backward op re-runs the forward
+      wf[w] = 0;
     }
+    // One boundary's transfers all start at its barrier and use links no other boundary uses, so its
+    // completion over the micro-batches is that of a single FIFO server with the longest transfer:
+    // max_p lf_p(k) with lf_p(k) = max(bar_k, lf_p(k-1)) + d_p equals max_j (bar_j + (k-j+1) max_p d_p)
+    // (bar_k is non-decreasing in k). Per boundary and direction: its longest transfer and free time.
+    dF[s] = dB[s] = lfF[s] = lfB[s] = fdl[s] = last[s] = 0;
+    if (s < S - 1) boundary_cf_cb<MN>(t, p.cut(s), mask, p.mask(s + 1), dF[s], dB[s]);
   }
-  // One boundary's transfers all start at its barrier and use links no other boundary uses, so its
-  // completion over the micro-batches is that of a single FIFO server with the longest transfer:
-  // max_p lf_p(k) with lf_p(k) = max(bar_k, lf_p(k-1)) + d_p equals max_j (bar_j + (k-j+1) max_p d_p)
-  // (bar_k is non-decreasing in k). Per boundary and direction: its longest transfer and free time.
-  u64 dF[MS], dB[MS], lfF[MS], lfB[MS];
-#pragma unroll
-  for (int s = 0; s < MS; ++s) {
-    dF[s] = dB[s] = lfF[s] = lfB[s] = 0;
+  // F_s(k) on every replica of stage s, then forward boundary s (as flush_makespan)
+  auto fwd = [&](int s) {
+    const u64 ready = s == 0 ? 0ull : fdl[s - 1];
+    u64 bar = 0;
+    for (u32 mm = msk[s]; mm; mm &= mm - 1) {
+      const int w = __ffs(mm) - 1;
+      wf[w] = umax(wf[w], ready) + Fd[w];
+      bar = umax(bar, wf[w]);
+    }
     if (s < S - 1) {
-      const int e = p.cut(s);
-      const u32 ms = p.mask(s), mn = p.mask(s + 1);
-      boundary_cf_cb<MN>(t, e, ms, mn, dF[s], dB[s]);
+      lfF[s] = umax(bar, lfF[s]) + dF[s];
+      fdl[s] = lfF[s];
     }
-  }
-
-  u64 fdl[MS], last[MS];
-#pragma unroll
-  for (int s = 0; s < MS; ++s) {
-    fdl[s] = 0;
-    last[s] = 0;
-  }
-  // F_s(k) on every replica of stage s, then forward boundary s
-#define AP_FWD(s_)                                                                  \
-  {                                                                                 \
-    const u64 ready = ((s_) == 0) ? 0 : fdl[(s_) > 0 ? (s_) - 1 : 0];               \
-    u64 bar = 0;                                                                    \
-    _Pragma("unroll") for (int w = 0; w < MN; ++w) if (stg[w] == (s_)) {          \
-      wf[w] = umax(wf[w], ready) + Fd[w];                                           \
-      bar = umax(bar, wf[w]);                                                       \
-    }                                                                               \
-    if ((s_) < S - 1) {                                                             \
-      lfF[s_] = umax(bar, lfF[s_]) + dF[s_];                                        \
-      fdl[s_] = lfF[s_];                                                            \
-    }                                                                               \
-  }
+  };
   // B_s(k) on every replica of stage s (input: bd), then backward boundary s-1 (into bd)
-#define AP_BWD(s_, k_)                                                              \
-  {                                                                                 \
-    const u64 ready = ((s_) == S - 1) ? 0 : bd;                                     \
-    u64 bar = 0;                                                                    \
-    _Pragma("unroll") for (int w = 0; w < MN; ++w) if (stg[w] == (s_)) {          \
-      wf[w] = umax(wf[w], ready) + Bd[w];                                           \
-      bar = umax(bar, wf[w]);                                                       \
-    }                                                                               \
-    if ((s_) > 0) {                                                                 \
-      const int sb_ = (s_) > 0 ? (s_) - 1 : 0;                                      \
-      lfB[sb_] = umax(bar, lfB[sb_]) + dB[sb_];                                     \
-      bd = lfB[sb_];                                                                \
-    }                                                                               \
-    if ((k_) == M - 1) last[s_] = bar;                                              \
-  }
-  if (SCHED == SCHED_GPIPE) {
-    for (int k = 0; k < M; ++k) {
-#pragma unroll
-      for (int s = 0; s < MS; ++s)
-        if (s < S) AP_FWD(s)
+  auto bwd = [&](int s, int k, u64 &bd) {
+    const u64 ready = s == S - 1 ? 0ull : bd;
+    u64 bar = 0;
+    for (u32 mm = msk[s]; mm; mm &= mm - 1) {
+      const int w = __ffs(mm) - 1;
+      wf[w] = umax(wf[w], ready) + Bd[w];
+      bar = umax(bar, wf[w]);
     }
+    if (s > 0) {
+      lfB[s - 1] = umax(bar, lfB[s - 1]) + dB[s - 1];
+      bd = lfB[s - 1];
+    }
+    if (k == M - 1) last[s] = bar;
+  };
+  if (SCHED == SCHED_GPIPE) {
+    for (int k = 0; k < M; ++k)
+      for (int s = 0; s < S; ++s) fwd(s);
     for (int k = 0; k < M; ++k) {
       u64 bd = 0;
-#pragma unroll
-      for (int s = MS - 1; s >= 0; --s)
-        if (s < S) AP_BWD(s, k)
+      for (int s = S - 1; s >= 0; --s) bwd(s, k, bd);
     }
   } else {
     const int nw = S < M ? S : M;  // n_0 = min(S, M) warm-up rounds
-    for (int k = 0; k < nw; ++k) {
-#pragma unroll
-      for (int s = 0; s < MS; ++s)
-        if (s < S && k < S - s) AP_FWD(s)  // k < n_s = min(S - s, M) (k < M already)
-    }
+    for (int k = 0; k < nw; ++k)
+      for (int s = 0; s < S; ++s)
+        if (k < S - s) fwd(s);  // k < n_s = min(S - s, M) (k < M already)
     for (int j = 0; j < M; ++j) {
       u64 bd = 0;
-#pragma unroll
-      for (int s = MS - 1; s >= 0; --s) {
-        if (s < S) {
-          AP_BWD(s, j)
-          if (j + (S - s) < M) AP_FWD(s)  // F_s(j + n_s), n_s = S - s when j + n_s < M
-        }
+      for (int s = S - 1; s >= 0; --s) {
+        bwd(s, j, bd);
+        if (j + (S - s) < M) fwd(s);  // F_s(j + n_s), n_s = S - s when j + n_s < M
       }
     }
   }
-#undef AP_FWD
-#undef AP_BWD
   u64 T = 0;
-#pragma unroll
-  for (int s = 0; s < MS; ++s) {
-    if (s < S) {
-      const u32 mask = p.mask(s);
-      u64 x = last[s];
-      if (__popc(mask) >= 2) {
-        const int a = (s == 0) ? 0 : p.cut(s - 1) + 1;
-        const int e = (s == S - 1) ? t.L - 1 : p.cut(s);
-        x += sync_time<MN>((int)m.sync, t.PP[e + 1] - t.PP[a], mask, t.tau, t.dv);
-      }
-      T = umax(T, x);
+  for (int s = 0; s < S; ++s) {
+    u64 x = last[s];
+    if (__popc(msk[s]) >= 2) {
+      const int a = (s == 0) ? 0 : p.cut(s - 1) + 1;
+      const int e = (s == S - 1) ? t.L - 1 : p.cut(s);
+      x += sync_time<MN>((int)m.sync, t.PP[e + 1] - t.PP[a], msk[s], t.tau, t.dv);
     }
+    T = umax(T, x);
   }
   return T;
 }
@@ -241,9 +211,9 @@ __device__ __forceinline__ u64 model_time(const SmemTab &t, int S, const P &p, c
   if constexpr (MODE == SCHED_CHIMERA) return chimera_time<P>(t, S, p, m);  // row f3, reading F-6
   if (MODE == SCHED_PIPEDREAM) return eval_closed_form<P32, false, P>(t, S, p, (int)m.sync);
   if (MODE == SCHED_2BW) return eval_closed_form<false, true, P>(t, S, p, (int)m.sync, m.M);
-  return flush_makespan<(MODE == SCHED_PIPEDREAM || MODE == SCHED_2BW || MODE == SCHED_RR || MODE == SCHED_CHIMERA)
-                            ? SCHED_GPIPE : MODE, P>(
-      t, S, p, m);
+  constexpr int FS = (MODE == SCHED_PIPEDREAM || MODE == SCHED_2BW || MODE == SCHED_RR || MODE == SCHED_CHIMERA)
+                         ? SCHED_GPIPE : MODE;
+  return flush_makespan<FS, P>(t, S, p, m);
 }
 
 }  // namespace ap

@@ -59,6 +59,11 @@ def main():
     if "switch" in which:
         cur = bytes(recs[0].cpu().numpy())
         res["switch_1M_ms"], _ = timed(lambda: eng.switch_rewards(recs, cur, 100, outputs=()), reps=10, warm=2)
+    if "flush" in which:
+        for k, model in (("gpipe", (L_.SCHED_GPIPE, L_.SYNC_RING, 8, False)), ("dapple", (L_.SCHED_DAPPLE, L_.SYNC_PS, 8, False))):
+            eng.set_schedule(*model)
+            res[k + "_eval_1M_ms"], _ = timed(lambda: eng.eval_partitions(recs, out=out), reps=10, warm=2)
+        eng.set_schedule()
     if "c5" in which:
         res["c5_eval_1M_ms"], _ = timed(lambda: eng.eval_partitions(recs, out=out), reps=20, warm=3)
     if "rr" in which or "rr_eval" in which:
