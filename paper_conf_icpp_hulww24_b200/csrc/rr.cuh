@@ -27,6 +27,7 @@
 // the 31 other lanes of its warp; the search kernels run it in the thread.
 #pragma once
 #include <climits>
+#include <cmath>
 
 #include "eval.cuh"
 
@@ -455,12 +456,167 @@ __device__ __forceinline__ bool rr_positive_warp(const RRSetup &R, long long th,
   return true;
 }
 
+// Predecessor `which` (0 or 1) of node v of the one-period event graph, as in rr_relax: its node id
+// and the edge's token count (periods between the two mini-batches); false if v has no such edge.
+__device__ __forceinline__ bool rr_pred(const RRSetup &R, int v, int which, int &u, long long &tok) {
+  const int S = R.S, Lam = (int)R.Lam;
+  const int kind = v / (S * Lam), s = (v / Lam) % S, p = v % Lam;
+  const long long K0 = 64ll * Lam, k = K0 + p;
+  int kk, ss;
+  long long ku;
+  if (kind == 0) {
+    if (which == 0) kk = 1, ss = s, ku = k - (long long)R.mm[s] * R.r[s];
+    else if (s > 0) kk = 2, ss = s - 1, ku = k;
+    else return false;
+  } else if (kind == 1) {
+    if (which == 0) kk = 0, ss = s, ku = k + (long long)(R.mm[s] - 1) * R.r[s];
+    else if (s < S - 1) kk = 3, ss = s, ku = k;
+    else return false;
+  } else if (kind == 2) {
+    if (which == 0) kk = 0, ss = s, ku = k;
+    else kk = 2, ss = s, ku = k - R.lc[s];
+  } else {
+    if (which == 0) kk = 1, ss = s + 1, ku = k;
+    else kk = 3, ss = s, ku = k - R.lc[s];
+  }
+  u = (kk * S + ss) * Lam + (int)(ku % Lam);
+  tok = k / Lam - ku / Lam;
+  return true;
+}
+
+// An estimate of lambda_compute by Howard's policy iteration on the one-period event graph (the
+// maximum cycle ratio sum(durations) / (Lam sum(tokens))), in double precision: each node keeps one
+// in-edge (the policy); the policy graph's cycles give their ratios, every node the ratio of the cycle
+// its policy chain reaches and a bias along the chain; a node switches to an in-edge whose source
+// reaches a larger ratio, or an equal ratio with a larger bias, until none does. Only a guess for the
+// exact search below (which verifies it with two Bellman-Ford tests), so rounding cannot hurt.
+static __device__ __noinline__ double rr_howard(const RRSetup &R) {
+  const int S = R.S, Lam = (int)R.Lam, V = 4 * S * Lam;
+  unsigned char pol[RR_BF_NODES], state[RR_BF_NODES];
+  double eta[RR_BF_NODES], x[RR_BF_NODES];
+  int path[RR_BF_NODES];
+  auto live = [&](int v) { const int kind = v / (S * Lam), s = (v / Lam) % S; return !(kind >= 2 && s == S - 1); };
+  auto edge = [&](int v, int which, int &u, double &w, double &tau) {
+    long long tok;
+    if (!rr_pred(R, v, which, u, tok)) return false;
+    const int kind = v / (S * Lam), s = (v / Lam) % S, p = v % Lam;
+    w = (double)rr_dur(R, kind, s, p);
+    tau = (double)Lam * (double)tok;
+    return true;
+  };
+  for (int v = 0; v < V; ++v) pol[v] = 0;
+  double best = 0.0;
+  for (int it = 0; it < 64; ++it) {
+    // value determination for the current policy
+    for (int v = 0; v < V; ++v) state[v] = live(v) ? 0 : 2;
+    for (int v0 = 0; v0 < V; ++v0) {
+      if (state[v0]) continue;
+      int n = 0, u = v0;
+      while (state[u] == 0) {  // follow the policy backwards (to the predecessors) until a known node
+        state[u] = 1;
+        path[n++] = u;
+        int pu;
+        double w, tau;
+        edge(u, pol[u], pu, w, tau);
+        u = pu;
+      }
+      if (state[u] == 1) {  // a new cycle through u: its ratio, biases around it
+        double W = 0.0, Tk = 0.0;
+        int c = u;
+        do {
+          int pc;
+          double w, tau;
+          edge(c, pol[c], pc, w, tau);
+          W += w;
+          Tk += tau;
+          c = pc;
+        } while (c != u);
+        const double r = Tk > 0.0 ? W / Tk : 1e300;  // a live schedule has no token-free cycle
+        x[u] = 0.0;
+        eta[u] = r;
+        c = u;
+        for (;;) {  // x(pred(c)) = x(c) - (w_c - r tau)
+          int pc;
+          double w, tau;
+          edge(c, pol[c], pc, w, tau);
+          if (pc == u) break;
+          x[pc] = x[c] - (w - r * tau);
+          eta[pc] = r;
+          c = pc;
+        }
+        c = u;
+        do {
+          state[c] = 2;
+          int pc;
+          double w, tau;
+          edge(c, pol[c], pc, w, tau);
+          c = pc;
+        } while (c != u);
+      }
+      for (int i = n - 1; i >= 0; --i) {  // the chain's nodes, nearest the resolved one first
+        const int v = path[i];
+        if (state[v] == 2) continue;
+        int pv;
+        double w, tau;
+        edge(v, pol[v], pv, w, tau);
+        eta[v] = eta[pv];
+        x[v] = x[pv] + w - eta[pv] * tau;
+        state[v] = 2;
+      }
+    }
+    best = 0.0;
+    for (int v = 0; v < V; ++v)
+      if (live(v) && eta[v] > best) best = eta[v];
+    // policy improvement
+    bool changed = false;
+    for (int v = 0; v < V; ++v) {
+      if (!live(v)) continue;
+      int u0, u1;
+      double w0, t0, w1, t1;
+      if (!edge(v, 1, u1, w1, t1)) continue;  // a single in-edge: nothing to choose
+      edge(v, 0, u0, w0, t0);
+      const double e0 = eta[u0], e1 = eta[u1];
+      const double tol = 1e-12 * (e0 > e1 ? e0 : e1) + 1e-9;
+      int pick = pol[v];
+      if (e0 > e1 + tol) pick = 0;
+      else if (e1 > e0 + tol) pick = 1;
+      else {
+        const double b0 = x[u0] + w0 - e0 * t0, b1 = x[u1] + w1 - e1 * t1;
+        const double bt = 1e-9 * (fabs(b0) > fabs(b1) ? fabs(b0) : fabs(b1)) + 1e-6;
+        if (b0 > b1 + bt) pick = 0;
+        else if (b1 > b0 + bt) pick = 1;
+      }
+      if (pick != pol[v]) {
+        pol[v] = (unsigned char)pick;
+        changed = true;
+      }
+    }
+    if (!changed) break;
+  }
+  return best;
+}
+
 // ceil(lambda_compute) inside the bracket t_lo <= T <= t_hi the simulation's bounds give:
 // positive(t_lo - 1) holds and positive(t_hi) does not, so a binary search on theta decides it.
 // (Galloping down from t_hi first was measured no faster on the C5 records: 2.2 -> 2.6 ms drain.)
 template <typename Pos>
-__device__ __forceinline__ u64 rr_ceil_search(u64 t_lo, u64 t_hi, Pos positive) {
+__device__ __forceinline__ u64 rr_ceil_search(u64 t_lo, u64 t_hi, Pos positive, double guess = -1.0) {
   long long lo = (long long)t_lo - 1, hi = (long long)t_hi;
+  // a guess (Howard's estimate) inside the bracket is checked first: positive(g - 1) and not
+  // positive(g) settle T = g with two tests; otherwise each test still halves the bracket's side
+  if (guess > 0.0) {
+    // lambda = p / q with q <= Lam sum(tokens) (a few thousand): a non-integral ratio sits >= 1 / q away
+    // from an integer, while the double sums err by ~1e-16 relative; the nudge only absorbs that
+    const long long g = (long long)ceil(guess - (1e-6 + 1e-13 * guess));
+    if (g - 1 > lo && g - 1 < hi) {
+      if (positive(g - 1)) lo = g - 1;
+      else hi = g - 1;
+    }
+    if (g > lo && g < hi) {
+      if (positive(g)) lo = g;
+      else hi = g;
+    }
+  }
   while (hi - lo > 1) {
     const long long mid = lo + (hi - lo) / 2;
     if (positive(mid)) lo = mid;
@@ -470,10 +626,11 @@ __device__ __forceinline__ u64 rr_ceil_search(u64 t_lo, u64 t_hi, Pos positive) 
 }
 __device__ __forceinline__ u64 rr_ceil_bf(const RRSetup &R, u64 t_lo, u64 t_hi) {
   long long dist[RR_BF_NODES];
-  return rr_ceil_search(t_lo, t_hi, [&](long long th) { return rr_positive(R, th, dist); });
+  return rr_ceil_search(t_lo, t_hi, [&](long long th) { return rr_positive(R, th, dist); }, rr_howard(R));
 }
 __device__ __forceinline__ u64 rr_ceil_bf_warp(const RRSetup &R, u64 t_lo, u64 t_hi, volatile long long *dist) {
-  return rr_ceil_search(t_lo, t_hi, [&](long long th) { return rr_positive_warp(R, th, dist); });
+  // every lane computes the same estimate (no broadcast needed)
+  return rr_ceil_search(t_lo, t_hi, [&](long long th) { return rr_positive_warp(R, th, dist); }, rr_howard(R));
 }
 
 // T_ns of a validated 16-byte partition under round-robin replicas, in the thread.
