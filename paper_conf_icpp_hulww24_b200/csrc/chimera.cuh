@@ -115,13 +115,22 @@ static __device__ __noinline__ u64 chimera_time(const SmemTab &t, int S, const P
     }
     return umax(fre[g], ready);
   };
+  // the cached head starts stay in registers: the scan and the updates index them only with
+  // unrolled (compile-time) indices, updates by selects (the head recomputations read the other
+  // arrays once per step)
   u64 hs[MS][2];
-  for (int g = 0; g < S; ++g) hs[g][0] = head_start(g, 0), hs[g][1] = head_start(g, 1);
+#pragma unroll
+  for (int g = 0; g < MS; ++g) {
+    hs[g][0] = g < S ? head_start(g, 0) : U64MAX;
+    hs[g][1] = g < S ? head_start(g, 1) : U64MAX;
+  }
   const u32 total = 2u * (u32)S * m.M;
   for (u32 step = 0; step < total; ++step) {
     u64 best = U64MAX;
     int bg = -1, bp = 0;
-    for (int g = 0; g < S; ++g)
+#pragma unroll
+    for (int g = 0; g < MS; ++g)
+#pragma unroll
       for (int pipe = 0; pipe < 2; ++pipe)
         if (hs[g][pipe] < best) {
           best = hs[g][pipe];
@@ -169,9 +178,15 @@ static __device__ __noinline__ u64 chimera_time(const SmemTab &t, int S, const P
         ++bcnt[bp][s - 1];
       }
     }
-    hs[bg][0] = head_start(bg, 0);
-    hs[bg][1] = head_start(bg, 1);
-    if (cg >= 0) hs[cg][bp] = head_start(cg, bp);
+    const u64 h0 = head_start(bg, 0), h1 = head_start(bg, 1), hc = cg >= 0 ? head_start(cg, bp) : 0;
+#pragma unroll
+    for (int g = 0; g < MS; ++g) {
+      if (g == bg) hs[g][0] = h0, hs[g][1] = h1;
+      if (g == cg) {
+        if (bp == 0) hs[g][0] = hc;
+        else hs[g][1] = hc;
+      }
+    }
   }
   u64 T = 0;
   for (int s = 0; s < S; ++s) {
