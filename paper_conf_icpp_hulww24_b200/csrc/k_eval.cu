@@ -30,13 +30,16 @@ struct CurPart {  // the current partition of a rollout (16-byte or wide)
 #define EVAL_MINB_WF 2
 #endif
 // resident blocks per SM for the round-robin evals (a latency-bound recurrence in local memory)
+#ifndef EVAL_MINB_CH
+#define EVAL_MINB_CH 2  // B200, 1M Chimera records: 1 / 2 / 3 blocks per SM within 0.5 % (4.44 / 4.44 / 4.42 ms)
+#endif
 #ifndef EVAL_MINB_RR
 #define EVAL_MINB_RR 2
 #endif
 #define EVAL_BLOCKS(MODE, P)                                                                    \
   ((MODE == SCHED_PIPEDREAM && P::MS == 8) ? EVAL_MINB                                          \
    : (P::MS == 16 && (MODE == SCHED_GPIPE || MODE == SCHED_DAPPLE)) ? EVAL_MINB_WF              \
-   : (MODE == SCHED_RR) ? EVAL_MINB_RR : 2)
+   : (MODE == SCHED_RR) ? EVAL_MINB_RR : (MODE == SCHED_CHIMERA) ? EVAL_MINB_CH : 2)
 #ifndef EVAL_MINB
 #define EVAL_MINB 4
 #endif
