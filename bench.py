@@ -35,6 +35,35 @@ TOTAL = comb(95, 7)
 PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
 INT_PEAK_PATH = os.path.join(ROOT, "profiles", "int_peak.json")
 TRAFFIC_PATH = os.path.join(ROOT, "profiles", "round2_traffic.json")
+KERNELS_PATH = os.path.join(ROOT, "profiles", "round2_kernels_full.txt")
+
+
+def ncu_kernel_metrics(prefix: str):
+    """Issue-slot and ALU-pipe use of the first kernel whose name starts with `prefix` in the committed
+    ncu --set full summary (a capture of the same kernel on this tree; not measured by this run)."""
+    want = {"smsp__issue_active.avg.pct_of_peak_sustained_active": "issue_active_pct",
+            "sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_active": "alu_pipe_active_pct",
+            "sm__warps_active.avg.pct_of_peak_sustained_active": "warps_active_pct"}
+    out, inside = {}, False
+    try:
+        with open(KERNELS_PATH) as fh:
+            for line in fh:
+                if line.startswith("kernel:"):
+                    if inside:
+                        break
+                    inside = line[len("kernel: void ap::"):].startswith(prefix) or \
+                        line[len("kernel: void "):].startswith(prefix)
+                    continue
+                if inside:
+                    parts = line.split()
+                    if parts and parts[0] in want:
+                        out[want[parts[0]]] = float(parts[1])
+    except OSError:
+        return None
+    if not out:
+        return None
+    out["source"] = "profiles/round2_kernels_full.txt (ncu --set full, committed capture)"
+    return out
 # Algorithmic integer ops per candidate (SURVEY.md §8(d)): the incremental full-T evaluation of an
 # S = 8, r = 1 candidate under the lexicographic successor is 85 ops on the 32-bit path (x2 on the
 # 64-bit path). The hot kernel only DECIDES "T <= theta" per candidate (exact T on the rare path), so
@@ -457,6 +486,8 @@ def main():
         pass
     peak_t = peak_issue / 1e12 if peak_issue else None
     frac = achieved / peak_t if peak_t else None
+    ncu = ncu_kernel_metrics(("k_search_r1<8, unsigned int" if main_res["int_path"] == 32
+                              else "k_search_r1<8, unsigned long long"))
     roofline = {"bound": "alu", "achieved": achieved, "peak": peak_t, "unit": "Tops/s", "frac": frac,
                 "traffic": traffic, "traffic_unit": "bytes per launch (ncu dram read + write)",
                 "kernel": kname, "ops_per_candidate": ops_per_cand,
@@ -468,7 +499,8 @@ def main():
                         "the rare path), so it does less than the algorithmic unit per candidate and the "
                         "fraction is not bounded by 1; its issue-slot use is in profiles/round2_kernels_full.txt",
                 "peak_source": peak_src, "peak_alu_pipe_only": peak_alu / 1e12 if peak_alu else None,
-                "kernel_ms": main_res["kernel_ms"], "candidates_per_launch": cands_per_rank}
+                "kernel_ms": main_res["kernel_ms"], "candidates_per_launch": cands_per_rank,
+                "ncu": ncu}
 
     configs = None
     if world == 1 and not args.no_configs:
